@@ -1,0 +1,104 @@
+"""ORACLE — test infrastructure only.
+
+Executes an augmented schedule (sim.expand) piece by piece in fp64: every
+micro-op runs the plain op definition (oracle.ops via oracle.net) on its block
+of samples, swap-out moves a piece to a host dict, swap-in moves it back, a
+recompute replay re-runs the producer micro-op, and a freed piece is deleted.
+A read of a piece that is not resident raises.  Pins SURVEY.md §4 T1 / P:L42:
+any split/swap/recompute plan yields the gradients of unsplit execution.
+"""
+
+from __future__ import annotations
+
+import numpy as np
+
+from . import net, sim
+
+F = np.float64
+
+
+def execute(graph, cfg, params, inputs, step=0):
+    items, f_alloc, f_free, fwd_end, an = sim.expand(graph, cfg)
+    ts, ops = graph["tensors"], graph["ops"]
+    n, B = an.n, graph["samples"]
+    pval = {t["id"]: np.asarray(params[t["name"]], F) for t in ts if t["kind"] == "param"}
+    pgrad = {tid: np.zeros_like(v) for tid, v in pval.items()}
+    store, host = {}, {}
+
+    def p_of(t):
+        return cfg[t][1] if (an.sample[t] and ts[t]["kind"] == "act") else 1
+
+    def rows_per_sample(t):
+        return ts[t]["shape"][0] // B
+
+    def piece_shape(t):
+        sh = list(ts[t]["shape"])
+        if an.sample[t]:
+            sh[0] //= p_of(t)
+        return tuple(sh)
+
+    for t in ts:
+        if t["kind"] in ("input", "label"):
+            a = np.asarray(inputs[t["name"]])
+            store[(t["id"], 0)] = a.astype(np.int64) if t["dtype"] == "i32" else a.astype(F)
+
+    def P_op(o):
+        P = 1
+        for t in ops[o]["inputs"] + ops[o]["outputs"]:
+            if an.sample[t]:
+                P = max(P, p_of(t))
+        return P
+
+    def view(t, s0, s1, grad=False):
+        """Rows of samples [s0, s1) of tensor t inside its resident piece."""
+        if not an.sample[t]:
+            return store[(n + t if grad else t, 0)]
+        p = p_of(t)
+        per = B // p
+        j = s0 // per
+        assert s1 <= (j + 1) * per
+        r = rows_per_sample(t)
+        arr = store[(n + t if grad else t, j)]
+        return arr[(s0 - j * per) * r:(s1 - j * per) * r]
+
+    for i, it in enumerate(items):
+        for pc in f_alloc.get(i, []):
+            key, j = pc
+            t = key - n if key >= n else key
+            if it.kind == "SI":
+                store[pc] = host.pop(pc)
+            else:
+                store[pc] = np.zeros(piece_shape(t), F)
+        if it.kind in ("F", "R", "B"):
+            o = ops[it.op]
+            P = P_op(it.op)
+            s0, s1 = it.k * B // P, (it.k + 1) * B // P
+            out = o["outputs"][0]
+            val = dict(pval)
+            reads = an.saved[it.op] if it.kind == "B" else [t for t in o["inputs"] if an.sample[t]]
+            for t in reads:
+                val[t] = view(t, s0, s1)
+            row0 = s0 * rows_per_sample(out) if an.sample[out] else s0
+            elem0 = s0 * (int(np.prod(ts[out]["shape"])) // B) if an.sample[out] else 0
+            if it.kind in ("F", "R"):
+                y = net.forward_op(graph, o, val, row0=row0, elem0=elem0, step=step)
+                if an.is_loss[out]:
+                    store[(out, 0)] += y
+                else:
+                    view(out, s0, s1)[...] = y
+            else:
+                dy = None if an.is_loss[out] else view(out, s0, s1, grad=True)
+                contrib = net.backward_op(graph, o, val, dy, row0=row0, elem0=elem0, step=step)
+                for tid, g in contrib.items():
+                    if ts[tid]["kind"] == "param":
+                        pgrad[tid] += g
+                    elif tid in an.needs_grad:
+                        view(tid, s0, s1, grad=True)[...] += g
+        elif it.kind == "SO":
+            pc = it.reads[0]
+            host[pc] = store[pc].copy()
+        for pc in f_free.get(i, []):
+            del store[pc]
+    loss_id = next(o["outputs"][0] for o in ops if o["kind"] == "xent")
+    loss = float(store[(loss_id, 0)][0])
+    return loss, {ts[tid]["name"]: g for tid, g in pgrad.items()}

@@ -1,0 +1,144 @@
+"""ORACLE — test infrastructure only.
+
+Unsplit fp64 training step of a DFG (§II: feed-forward pass, loss
+L, back-propagation "to obtain the gradients dL/dw of each model parameter").
+This is the plain definition every TSPLIT plan must reproduce (T1).
+Ops run in definition order (the tsinputs builders emit a topological order);
+the backward pass visits ops in reverse and sums gradient contributions.
+"""
+
+from __future__ import annotations
+
+import numpy as np
+
+from . import ops
+
+F = np.float64
+
+
+def _attrs(op):
+    return op["iattrs"], op["fattrs"]
+
+
+def forward_op(graph, op, val, row0=0, elem0=0, step=0):
+    """Evaluate one op on `val` (tensor id -> fp64/int array) for a block of samples
+    starting at global sample-row `row0` / element `elem0` of the output."""
+    k = op["kind"]
+    ia, fa = _attrs(op)
+    x = [val[i] for i in op["inputs"]]
+    if k == "linear":
+        return ops.linear_fwd(x[0], x[1], x[2])
+    if k == "relu":
+        return ops.relu_fwd(x[0])
+    if k == "gelu":
+        return ops.gelu_fwd(x[0])
+    if k == "tanh":
+        return ops.tanh_fwd(x[0])
+    if k == "layernorm":
+        return ops.layernorm_fwd(x[0], x[1], x[2], fa[0])
+    if k == "add":
+        return ops.add_fwd(x[0], x[1])
+    if k == "dropout":
+        return ops.dropout_fwd(x[0], fa[0], ia[0], elem0, step)
+    if k == "softmax":
+        return ops.softmax_fwd(x[0])
+    if k == "attn_qk":
+        return ops.attn_qk_fwd(x[0], x[1], ia[0], ia[1], fa[0])
+    if k == "attn_pv":
+        return ops.attn_pv_fwd(x[0], x[1], ia[0], ia[1])
+    if k == "embed":
+        return ops.embed_fwd(x[0], x[1], x[2], x[3], x[4], ia[0], row0)
+    if k == "cls":
+        return ops.cls_fwd(x[0], ia[0])
+    if k == "xent":
+        return np.array([ops.xent_fwd(x[0], x[1], graph["samples"])])
+    raise ValueError(k)
+
+
+def backward_op(graph, op, val, dy, row0=0, elem0=0, step=0):
+    """Returns {tensor id: gradient contribution} for the op's inputs.
+
+    `dy` is the gradient of the op's output (None for xent, whose output is L)."""
+    k = op["kind"]
+    ia, fa = _attrs(op)
+    ins = op["inputs"]
+    x = [val.get(i) for i in ins]
+    out = {}
+    if k == "linear":
+        dx, dw, db = ops.linear_bwd(dy, x[0], x[1])
+        out = {ins[0]: dx, ins[1]: dw, ins[2]: db}
+    elif k == "relu":
+        out = {ins[0]: ops.relu_bwd(dy, val[op["outputs"][0]])}
+    elif k == "gelu":
+        out = {ins[0]: ops.gelu_bwd(dy, x[0])}
+    elif k == "tanh":
+        out = {ins[0]: ops.tanh_bwd(dy, val[op["outputs"][0]])}
+    elif k == "layernorm":
+        dx, dg, db = ops.layernorm_bwd(dy, x[0], x[1], fa[0])
+        out = {ins[0]: dx, ins[1]: dg, ins[2]: db}
+    elif k == "add":
+        out = {ins[0]: dy, ins[1]: dy}
+    elif k == "dropout":
+        out = {ins[0]: ops.dropout_bwd(dy, fa[0], ia[0], elem0, step)}
+    elif k == "softmax":
+        out = {ins[0]: ops.softmax_bwd(dy, val[op["outputs"][0]])}
+    elif k == "attn_qk":
+        dq, dk = ops.attn_qk_bwd(dy, x[0], x[1], ia[0], ia[1], fa[0])
+        out = {ins[0]: dq, ins[1]: dk}
+    elif k == "attn_pv":
+        dp, dv = ops.attn_pv_bwd(dy, x[0], x[1], ia[0], ia[1])
+        out = {ins[0]: dp, ins[1]: dv}
+    elif k == "embed":
+        shapes = [graph["tensors"][i]["shape"] for i in ins[2:5]]
+        dw, dp, dt = ops.embed_bwd(dy, x[0], x[1], ia[0], row0, shapes)
+        out = {ins[2]: dw, ins[3]: dp, ins[4]: dt}
+    elif k == "cls":
+        rows = dy.shape[0] * ia[0]
+        out = {ins[0]: ops.cls_bwd(dy, ia[0], rows)}
+    elif k == "xent":
+        out = {ins[0]: ops.xent_bwd(x[0], x[1], graph["samples"])}
+    else:
+        raise ValueError(k)
+    return out
+
+
+def needs_grad(graph):
+    """Tensor ids that carry a gradient: params, and activations downstream of one."""
+    ng = {t["id"] for t in graph["tensors"] if t["kind"] == "param"}
+    for op in graph["ops"]:
+        if any(i in ng for i in op["inputs"]):
+            ng.update(op["outputs"])
+    return ng
+
+
+def initial_values(graph, params, inputs):
+    val = {}
+    for t in graph["tensors"]:
+        if t["kind"] == "param":
+            val[t["id"]] = np.asarray(params[t["name"]], F)
+        elif t["kind"] in ("input", "label"):
+            a = np.asarray(inputs[t["name"]])
+            val[t["id"]] = a.astype(np.int64) if t["dtype"] == "i32" else a.astype(F)
+    return val
+
+
+def train_step(graph, params, inputs, step=0):
+    """Unsplit fp64 forward + backward.  Returns (loss, {param name: grad})."""
+    val = initial_values(graph, params, inputs)
+    for op in graph["ops"]:
+        val[op["outputs"][0]] = forward_op(graph, op, val, step=step)
+    loss_id = next(op["outputs"][0] for op in graph["ops"] if op["kind"] == "xent")
+    ng = needs_grad(graph)
+    grad = {}
+    for op in reversed(graph["ops"]):
+        o = op["outputs"][0]
+        if o != loss_id and o not in grad:
+            continue
+        contrib = backward_op(graph, op, val, grad.get(o), step=step)
+        for tid, g in contrib.items():
+            if tid not in ng:
+                continue
+            grad[tid] = grad[tid] + g if tid in grad else g
+    pg = {t["name"]: grad.get(t["id"], np.zeros(t["shape"]))
+          for t in graph["tensors"] if t["kind"] == "param"}
+    return float(val[loss_id][0]), pg, val, grad

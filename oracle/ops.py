@@ -1,0 +1,220 @@
+"""ORACLE — test infrastructure only (see oracle/__init__.py).
+
+Plain fp64 numpy forward and vector-Jacobian products of the operations the
+DFGs in tsinputs.graphs use.  TSPLIT itself does not change any operator
+(§VI-D: "TSPLIT will not result in changes in existing operator
+implementation"; L42: swap/recompute have "no accuracy loss"), so the numeric
+oracle is the plain textbook definition of each op, evaluated unsplit.
+Silent points of the paper are taken as SURVEY.md §8(c) R15/R16 read them:
+erf-GELU, biased LayerNorm variance, attention scale 1/sqrt(d_head) without a
+padding mask, Philox-keyed dropout, mean cross-entropy over the *global* batch
+(R14).  Every function works on a contiguous block of samples; `row0`/`elem0`
+give the global offset of that block so that position embeddings and dropout
+masks are the same whichever split executes them (R15).
+"""
+
+from __future__ import annotations
+
+import numpy as np
+from scipy.special import erf
+
+F = np.float64
+
+# ---------------------------------------------------------------------------
+# Philox4x32-10 counter-based RNG (Salmon et al., SC'11), SURVEY.md §8(c) R15.
+# counter = (idx_lo, idx_hi, step, 0), key = (seed, 0x5453504C).  The mask bit
+# of element idx is keep = (word0 >= floor(p * 2^32)).  Pure integer maths, so
+# both sides of the parity test take the identical keep/drop decision.
+# ---------------------------------------------------------------------------
+_M0, _M1 = np.uint64(0xD2511F53), np.uint64(0xCD9E8D57)
+_W0, _W1 = 0x9E3779B9, 0xBB67AE85
+_MASK32 = np.uint64(0xFFFFFFFF)
+PHILOX_KEY1 = 0x5453504C
+
+
+def philox4x32_10(c, k0, k1):
+    """Philox4x32-10 on a tuple of four uint64 arrays holding 32-bit counters."""
+    c0, c1, c2, c3 = c
+    k0, k1 = k0 & 0xFFFFFFFF, k1 & 0xFFFFFFFF
+    for r in range(10):
+        p0 = _M0 * c0
+        p1 = _M1 * c2
+        hi0, lo0 = p0 >> np.uint64(32), p0 & _MASK32
+        hi1, lo1 = p1 >> np.uint64(32), p1 & _MASK32
+        c0, c1, c2, c3 = (hi1 ^ c1 ^ np.uint64(k0)), lo1, (hi0 ^ c3 ^ np.uint64(k1)), lo0
+        k0 = (k0 + _W0) & 0xFFFFFFFF
+        k1 = (k1 + _W1) & 0xFFFFFFFF
+    return c0, c1, c2, c3
+
+
+def philox_word0(idx: np.ndarray, seed: int, step: int = 0) -> np.ndarray:
+    idx = idx.astype(np.uint64)
+    c0 = idx & _MASK32
+    c1 = idx >> np.uint64(32)
+    c2 = np.full_like(c0, np.uint64(step & 0xFFFFFFFF))
+    c3 = np.zeros_like(c0)
+    return philox4x32_10((c0, c1, c2, c3), seed, PHILOX_KEY1)[0]
+
+
+def dropout_keep(shape, elem0: int, p: float, seed: int, step: int = 0) -> np.ndarray:
+    n = int(np.prod(shape))
+    w = philox_word0(np.arange(elem0, elem0 + n, dtype=np.uint64), seed, step)
+    thr = np.uint64(int(np.floor(p * 4294967296.0)))
+    return (w >= thr).reshape(shape)
+
+
+# ---------------------------------------------------------------------------
+# Forward / backward of each op kind.  Arrays are fp64.
+# ---------------------------------------------------------------------------
+
+def linear_fwd(x, w, b):
+    return x @ w.T + b
+
+
+def linear_bwd(dy, x, w):
+    """dX = dY W, dW = dY^T X, db = sum_rows dY."""
+    return dy @ w, dy.T @ x, dy.sum(axis=0)
+
+
+def relu_fwd(x):
+    return np.maximum(x, 0.0)
+
+
+def relu_bwd(dy, y):
+    return dy * (y > 0)
+
+
+def gelu_fwd(x):
+    return 0.5 * x * (1.0 + erf(x / np.sqrt(2.0)))
+
+
+def gelu_bwd(dy, x):
+    cdf = 0.5 * (1.0 + erf(x / np.sqrt(2.0)))
+    pdf = np.exp(-0.5 * x * x) / np.sqrt(2.0 * np.pi)
+    return dy * (cdf + x * pdf)
+
+
+def tanh_fwd(x):
+    return np.tanh(x)
+
+
+def tanh_bwd(dy, y):
+    return dy * (1.0 - y * y)
+
+
+def layernorm_fwd(x, g, b, eps):
+    mu = x.mean(axis=-1, keepdims=True)
+    var = ((x - mu) ** 2).mean(axis=-1, keepdims=True)
+    xhat = (x - mu) / np.sqrt(var + eps)
+    return xhat * g + b
+
+
+def layernorm_bwd(dy, x, g, eps):
+    """Returns dX, dgamma, dbeta (biased variance, per-row statistics)."""
+    mu = x.mean(axis=-1, keepdims=True)
+    var = ((x - mu) ** 2).mean(axis=-1, keepdims=True)
+    rstd = 1.0 / np.sqrt(var + eps)
+    xhat = (x - mu) * rstd
+    dxhat = dy * g
+    dx = rstd * (dxhat - dxhat.mean(axis=-1, keepdims=True)
+                 - xhat * (dxhat * xhat).mean(axis=-1, keepdims=True))
+    return dx, (dy * xhat).sum(axis=0), dy.sum(axis=0)
+
+
+def add_fwd(a, b):
+    return a + b
+
+
+def dropout_fwd(x, p, seed, elem0, step=0):
+    if p == 0.0:
+        return x.copy()
+    keep = dropout_keep(x.shape, elem0, p, seed, step)
+    return np.where(keep, x / (1.0 - p), 0.0)
+
+
+def dropout_bwd(dy, p, seed, elem0, step=0):
+    return dropout_fwd(dy, p, seed, elem0, step)
+
+
+def softmax_fwd(x):
+    m = x.max(axis=-1, keepdims=True)
+    e = np.exp(x - m)
+    return e / e.sum(axis=-1, keepdims=True)
+
+
+def softmax_bwd(dy, y):
+    return y * (dy - (dy * y).sum(axis=-1, keepdims=True))
+
+
+def _heads(x, heads, seq):
+    """[nb*s, h] -> [nb, a, s, d]."""
+    nb = x.shape[0] // seq
+    return x.reshape(nb, seq, heads, -1).transpose(0, 2, 1, 3)
+
+
+def _merge(xh):
+    """[nb, a, s, d] -> [nb*s, h]."""
+    nb, a, s, d = xh.shape
+    return xh.transpose(0, 2, 1, 3).reshape(nb * s, a * d)
+
+
+def attn_qk_fwd(q, k, heads, seq, alpha):
+    return alpha * (_heads(q, heads, seq) @ _heads(k, heads, seq).transpose(0, 1, 3, 2))
+
+
+def attn_qk_bwd(ds, q, k, heads, seq, alpha):
+    qh, kh = _heads(q, heads, seq), _heads(k, heads, seq)
+    dq = alpha * (ds @ kh)
+    dk = alpha * (ds.transpose(0, 1, 3, 2) @ qh)
+    return _merge(dq), _merge(dk)
+
+
+def attn_pv_fwd(p, v, heads, seq):
+    return _merge(p @ _heads(v, heads, seq))
+
+
+def attn_pv_bwd(dc, p, v, heads, seq):
+    dch = _heads(dc, heads, seq)
+    vh = _heads(v, heads, seq)
+    dp = dch @ vh.transpose(0, 1, 3, 2)
+    dv = p.transpose(0, 1, 3, 2) @ dch
+    return dp, _merge(dv)
+
+
+def embed_fwd(ids, tt, wword, wpos, wtype, seq, row0):
+    pos = (np.arange(row0, row0 + ids.shape[0]) % seq)
+    return wword[ids] + wpos[pos] + wtype[tt]
+
+
+def embed_bwd(dy, ids, tt, seq, row0, shapes):
+    dword = np.zeros(shapes[0], F)
+    dpos = np.zeros(shapes[1], F)
+    dtype_ = np.zeros(shapes[2], F)
+    pos = (np.arange(row0, row0 + ids.shape[0]) % seq)
+    np.add.at(dword, ids, dy)
+    np.add.at(dpos, pos, dy)
+    np.add.at(dtype_, tt, dy)
+    return dword, dpos, dtype_
+
+
+def cls_fwd(x, seq):
+    return x[::seq].copy()
+
+
+def cls_bwd(dy, seq, rows):
+    dx = np.zeros((rows, dy.shape[1]), F)
+    dx[::seq] = dy
+    return dx
+
+
+def xent_fwd(z, labels, b_global):
+    """Sum over this block of (logsumexp(z) - z[label]) / B_global (R14)."""
+    m = z.max(axis=1, keepdims=True)
+    lse = (m + np.log(np.exp(z - m).sum(axis=1, keepdims=True)))[:, 0]
+    return float((lse - z[np.arange(z.shape[0]), labels]).sum() / b_global)
+
+
+def xent_bwd(z, labels, b_global):
+    dz = softmax_fwd(z)
+    dz[np.arange(z.shape[0]), labels] -= 1.0
+    return dz / b_global

@@ -1,0 +1,464 @@
+"""ORACLE — test infrastructure only.
+
+Plan-execution simulator, followed step by step from PAPER.md and the readings
+DESIGN.md §4 fixes:
+
+  schedule()  Alg. 1 (§II) with the garbled line 5 read as
+              `ref_cnt -= 1` and line 6 as `== 0` (R1).
+  expand()    augmented schedule (Fig. 10): op-major micro-ops
+              (R10), swap-out after the last forward use / swap-in at the
+              "previous computation operation", memory-centric
+              recompute replay (Fig. 11), in-place re-split: a
+              micro-op reads a sub-range of a coarser piece.
+  Pool        best-fit over one pre-allocated slab ("best-fit memory
+              allocation", "pre-allocate a large piece of GPU memory"),
+              256 B alignment, lowest offset on ties, coalescing (R11).  The
+              block that reaches the end of the slab is used only when no
+              other block fits, so a finite slab and an unbounded one give the
+              identical trace whenever the plan fits.
+  simulate()  allocation only at the beginning and free only at the end of an
+              operation; M_i = sum of live sizes.
+"""
+
+from __future__ import annotations
+
+from dataclasses import dataclass, field
+
+DTYPE_BYTES = {"f32": 4, "bf16": 2, "i32": 4}
+ALIGN = 256
+WS_ROWS = 256
+INF = 1 << 62
+
+RESIDE, SWAP, RECOMPUTE = 0, 1, 2
+
+# Forward tensors each backward op reads (DESIGN.md §3 table "saved").
+SAVED = {
+    "linear": ("in", 0),
+    "relu": ("out", 0),
+    "gelu": ("in", 0),
+    "tanh": ("out", 0),
+    "layernorm": ("in", 0),
+    "add": None,
+    "dropout": None,
+    "softmax": ("out", 0),
+    "attn_qk": ("in", 0, 1),
+    "attn_pv": ("in", 0, 1),
+    "embed": ("in", 0, 1),
+    "cls": None,
+    "xent": ("in", 0, 1),
+}
+
+
+def align(n):
+    return (n + ALIGN - 1) // ALIGN * ALIGN
+
+
+def numel(shape):
+    n = 1
+    for s in shape:
+        n *= s
+    return n
+
+
+def tbytes(t):
+    return numel(t["shape"]) * DTYPE_BYTES[t["dtype"]]
+
+
+def static_bytes(graph):
+    """Static region: fp32 master + (bf16 copy) + fp32 grad per param, + workspace."""
+    total = 0
+    max1d = 1
+    for t in graph["tensors"]:
+        if t["kind"] != "param":
+            continue
+        n = numel(t["shape"])
+        total += align(4 * n) + align(4 * n)
+        if graph["dtype"] == "bf16":
+            total += align(2 * n)
+        if len(t["shape"]) == 1:
+            max1d = max(max1d, n)
+    return total + align(WS_ROWS * 2 * max1d * 4)
+
+
+def schedule(graph):
+    """Alg. 1: DFS-manner topological order of the forward ops (R1)."""
+    ops = graph["ops"]
+    producer = {}
+    for o in ops:
+        for t in o["outputs"]:
+            producer[t] = o["id"]
+    preds = []
+    succ = [[] for _ in ops]
+    for o in ops:
+        ps = []
+        for t in o["inputs"]:
+            if t in producer and producer[t] not in ps:
+                ps.append(producer[t])
+        preds.append(ps)
+        for p in ps:
+            if o["id"] not in succ[p]:
+                succ[p].append(o["id"])
+    for s in succ:
+        s.sort()
+    ref_cnt = [len(p) for p in preds]
+    order = []
+
+    def execution_scheduler(layer):
+        order.append(layer)
+        for nxt in succ[layer]:
+            ref_cnt[nxt] -= 1
+            if ref_cnt[nxt] == 0:
+                execution_scheduler(nxt)
+
+    for o in ops:
+        if not preds[o["id"]]:
+            execution_scheduler(o["id"])
+    assert len(order) == len(ops), "graph has a cycle"
+    return order
+
+
+@dataclass
+class Analysis:
+    n: int
+    producer: dict
+    sample: list            # tensor id -> is a sample (splittable) tensor
+    is_loss: list
+    needs_grad: set
+    has_bwd: list
+    saved: list             # op id -> tensor ids bwd reads (non-param)
+    bytes_: list
+
+
+def analyze(graph):
+    ts, ops = graph["tensors"], graph["ops"]
+    n = len(ts)
+    producer = {}
+    for o in ops:
+        for t in o["outputs"]:
+            producer[t] = o["id"]
+    is_loss = [False] * n
+    for o in ops:
+        if o["kind"] == "xent":
+            is_loss[o["outputs"][0]] = True
+    sample = [t["kind"] != "param" and not is_loss[t["id"]] for t in ts]
+    ng = {t["id"] for t in ts if t["kind"] == "param"}
+    for o in ops:
+        if any(i in ng for i in o["inputs"]):
+            ng.update(o["outputs"])
+    has_bwd = [o["kind"] == "xent" or any(i in ng for i in o["inputs"]) for o in ops]
+    saved = []
+    for o in ops:
+        spec = SAVED[o["kind"]]
+        lst = []
+        if spec is not None:
+            src = o["inputs"] if spec[0] == "in" else o["outputs"]
+            for idx in spec[1:]:
+                t = src[idx]
+                if ts[t]["kind"] != "param" and t not in lst:
+                    lst.append(t)
+        saved.append(lst)
+    return Analysis(n, producer, sample, is_loss, ng, has_bwd, saved, [tbytes(t) for t in ts])
+
+
+@dataclass
+class Item:
+    kind: str          # 'F' forward, 'B' backward, 'R' recompute replay, 'SO' swap-out, 'SI' swap-in
+    op: int = -1
+    k: int = 0
+    reads: list = field(default_factory=list)    # (key, piece)
+    writes: list = field(default_factory=list)
+    group: int = -1    # backward group id (replays + the B item they serve)
+
+
+class Pool:
+    """Best-fit allocator over [base, capacity) — R11 and the tail rule above."""
+
+    def __init__(self, base, capacity=INF):
+        self.capacity = capacity
+        self.free = [(base, capacity - base)]   # sorted by offset
+        self.extent = base
+
+    def alloc(self, nbytes):
+        need = align(nbytes)
+        best = None
+        for idx, (off, ln) in enumerate(self.free):
+            if off + ln == self.capacity:
+                continue
+            if ln >= need and (best is None or ln < self.free[best][1]):
+                best = idx
+        if best is None:
+            idx = len(self.free) - 1
+            off, ln = self.free[idx]
+            if off + ln != self.capacity or ln < need:
+                raise MemoryError("pool exhausted")
+            best = idx
+        off, ln = self.free[best]
+        if ln == need:
+            self.free.pop(best)
+        else:
+            self.free[best] = (off + need, ln - need)
+        self.extent = max(self.extent, off + need)
+        return off
+
+    def release(self, off, nbytes):
+        need = align(nbytes)
+        i = 0
+        while i < len(self.free) and self.free[i][0] < off:
+            i += 1
+        self.free.insert(i, (off, need))
+        # coalesce with the next, then the previous block
+        if i + 1 < len(self.free) and self.free[i][0] + self.free[i][1] == self.free[i + 1][0]:
+            self.free[i] = (off, need + self.free[i + 1][1])
+            self.free.pop(i + 1)
+        if i > 0 and self.free[i - 1][0] + self.free[i - 1][1] == self.free[i][0]:
+            self.free[i - 1] = (self.free[i - 1][0], self.free[i - 1][1] + self.free[i][1])
+            self.free.pop(i)
+
+
+def default_cfg(graph):
+    return {t["id"]: (RESIDE, 1, 1) for t in graph["tensors"]}
+
+
+def expand(graph, cfg, order=None, an=None):
+    """Augmented schedule: returns (items, alloc_at, free_after, fwd_end) where
+    alloc_at / free_after map item index -> ordered list of (key, piece)."""
+    an = an or analyze(graph)
+    order = order if order is not None else schedule(graph)
+    ts, ops = graph["tensors"], graph["ops"]
+    n = an.n
+
+    def p_of(t):
+        if t >= n:
+            t -= n
+        if not an.sample[t] or ts[t]["kind"] != "act":
+            return 1
+        return cfg[t][1]
+
+    def opt_of(t):
+        return cfg[t][0]
+
+    def P_op(o):
+        P = 1
+        for t in ops[o]["inputs"] + ops[o]["outputs"]:
+            if an.sample[t]:
+                P = max(P, p_of(t))
+        return P
+
+    def piece(t, k, P):
+        if t < n and not an.sample[t]:
+            return 0
+        return k * p_of(t) // P
+
+    def ins_sample(o):
+        return [t for t in ops[o]["inputs"] if an.sample[t]]
+
+    items = []
+    for o in order:
+        P = P_op(o)
+        for k in range(P):
+            it = Item("F", o, k)
+            it.reads = [(t, piece(t, k, P)) for t in ins_sample(o)]
+            it.writes = [(t, piece(t, k, P)) for t in ops[o]["outputs"]]
+            items.append(it)
+    fwd_end = len(items)
+
+    gid = 0
+    for o in reversed(order):
+        if not an.has_bwd[o]:
+            continue
+        P = P_op(o)
+        for k in range(P):
+            group = []
+            live_temp = set()
+
+            def need(t, j):
+                if ts[t]["kind"] != "act" or opt_of(t) != RECOMPUTE or (t, j) in live_temp:
+                    return
+                po = an.producer[t]
+                Q = P_op(po)
+                pt = p_of(t)
+                for kk in range(j * Q // pt, (j + 1) * Q // pt):
+                    for u in ins_sample(po):
+                        need(u, piece(u, kk, Q))
+                    r = Item("R", po, kk, group=gid)
+                    r.reads = [(u, piece(u, kk, Q)) for u in ins_sample(po)]
+                    r.writes = [(t, j)]
+                    group.append(r)
+                live_temp.add((t, j))
+
+            saved_pieces = [(t, piece(t, k, P)) for t in an.saved[o]]
+            for (t, j) in saved_pieces:
+                need(t, j)
+            b = Item("B", o, k, group=gid)
+            b.reads = list(saved_pieces)
+            for t in ops[o]["outputs"]:
+                if not an.is_loss[t]:
+                    b.reads.append((n + t, piece(t, k, P)))
+            for t in ops[o]["inputs"]:
+                if ts[t]["kind"] == "act" and t in an.needs_grad:
+                    w = (n + t, piece(t, k, P))
+                    if w not in b.writes:
+                        b.writes.append(w)
+            group.append(b)
+            items.extend(group)
+            gid += 1
+
+    # ---- lifetimes -------------------------------------------------------------
+    touches = {}
+    for i, it in enumerate(items):
+        for pc in it.writes + it.reads:
+            touches.setdefault(pc, []).append(i)
+
+    def cls(key):
+        if key >= n:
+            return "grad"
+        t = ts[key]
+        if t["kind"] in ("input", "label"):
+            return "input"
+        if an.is_loss[key]:
+            return "loss"
+        return "act"
+
+    alloc_at, free_after = {}, {}
+    swap_out_after = {}       # forward item index -> [pieces]
+    swap_in_before = {}       # pre-insertion item index -> [pieces]
+    temp_spans = []
+    for pc, idxs in touches.items():
+        key, j = pc
+        c = cls(key)
+        if c == "input":
+            free_after.setdefault(max(idxs), []).append(pc)
+            continue
+        if c == "loss":
+            alloc_at.setdefault(min(idxs), []).append(pc)
+            continue
+        if c == "grad":
+            alloc_at.setdefault(min(idxs), []).append(pc)
+            free_after.setdefault(max(idxs), []).append(pc)
+            continue
+        fw = [i for i in idxs if i < fwd_end]
+        bw = [i for i in idxs if i >= fwd_end]
+        opt = opt_of(key)
+        alloc_at.setdefault(min(fw), []).append(pc)
+        if not bw or opt == RESIDE:
+            free_after.setdefault(max(idxs), []).append(pc)
+        elif opt == SWAP:
+            swap_out_after.setdefault(max(fw), []).append(pc)
+            lead = max(1, cfg[key][2])
+            pos = max(min(bw) - lead, fwd_end)
+            swap_in_before.setdefault(pos, []).append(pc)
+            free_after.setdefault(max(bw), []).append(pc)
+        else:  # RECOMPUTE: forward lifetime, then per-group temporaries
+            free_after.setdefault(max(fw), []).append(pc)
+            by_group = {}
+            for i in bw:
+                by_group.setdefault(items[i].group, []).append(i)
+            for g, gi in by_group.items():
+                alloc_at.setdefault(min(gi), []).append(pc)
+                free_after.setdefault(max(gi), []).append(pc)
+                temp_spans.append((pc, min(gi), max(gi)))
+
+    # ---- final item list with SO / SI items -----------------------------------
+    final = []
+    f_alloc, f_free = {}, {}
+    for i, it in enumerate(items):
+        for pc in sorted(swap_in_before.get(i, [])):
+            si = Item("SI")
+            si.writes = [pc]
+            f_alloc[len(final)] = [pc]
+            final.append(si)
+        idx = len(final)
+        final.append(it)
+        # allocation order: the item's write order, then its reads (temps never
+        # appear as reads before a write; inputs are allocated at start)
+        allocs = alloc_at.get(i, [])
+        ordered = [pc for pc in it.writes if pc in allocs] + [pc for pc in it.reads if pc in allocs and pc not in it.writes]
+        assert len(ordered) == len(set(allocs)), (it, allocs)
+        if ordered:
+            f_alloc[idx] = ordered
+        if i in free_after:
+            f_free[idx] = sorted(free_after[i])
+        for pc in sorted(swap_out_after.get(i, [])):
+            so = Item("SO")
+            so.reads = [pc]
+            f_free[len(final)] = [pc]
+            final.append(so)
+    return final, f_alloc, f_free, fwd_end, an
+
+
+@dataclass
+class SimResult:
+    items: list
+    trace: list            # (seq, item, 'A'|'F', key, piece, offset, bytes)
+    static: int
+    peak_live: int
+    peak_extent: int
+    live_after_alloc: list  # per item, dynamic live bytes
+    n_replay: int
+    d2h_bytes: int
+    h2d_bytes: int
+
+
+def simulate(graph, cfg=None, order=None, capacity=INF):
+    cfg = cfg or default_cfg(graph)
+    items, f_alloc, f_free, fwd_end, an = expand(graph, cfg, order)
+    ts = graph["tensors"]
+    n = an.n
+    base = static_bytes(graph)
+    pool = Pool(base, capacity)
+
+    def pbytes(pc):
+        key, j = pc
+        t = key - n if key >= n else key
+        if not an.sample[t] or ts[t]["kind"] != "act":
+            return an.bytes_[t]
+        return an.bytes_[t] // cfg[t][1]
+
+    where = {}
+    trace = []
+    live = 0
+    peak = 0
+    lal = []
+
+    def do_alloc(item_idx, pc):
+        nonlocal live
+        b = pbytes(pc)
+        off = pool.alloc(b)
+        assert pc not in where, ("double alloc", pc)
+        where[pc] = off
+        live += align(b)
+        trace.append((len(trace), item_idx, "A", pc[0], pc[1], off, b))
+
+    def do_free(item_idx, pc):
+        nonlocal live
+        b = pbytes(pc)
+        off = where.pop(pc)
+        pool.release(off, b)
+        live -= align(b)
+        trace.append((len(trace), item_idx, "F", pc[0], pc[1], off, b))
+
+    for t in ts:
+        if t["kind"] in ("input", "label"):
+            do_alloc(-1, (t["id"], 0))
+    peak = live
+    d2h = h2d = nrep = 0
+    for i, it in enumerate(items):
+        for pc in f_alloc.get(i, []):
+            do_alloc(i, pc)
+        for pc in it.reads:
+            assert pc in where, ("read of non-resident piece", i, it, pc)
+        for pc in it.writes:
+            assert pc in where, ("write to unallocated piece", i, it, pc)
+        lal.append(live)
+        peak = max(peak, live)
+        if it.kind == "SO":
+            d2h += pbytes(it.reads[0])
+        elif it.kind == "SI":
+            h2d += pbytes(it.writes[0])
+        elif it.kind == "R":
+            nrep += 1
+        for pc in f_free.get(i, []):
+            do_free(i, pc)
+    for pc in sorted(list(where.keys())):
+        do_free(len(items), pc)
+    return SimResult(items, trace, base, base + peak, pool.extent, lal, nrep, d2h, h2d)

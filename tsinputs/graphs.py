@@ -1,0 +1,191 @@
+"""Workload dataflow graphs (DFGs) — plain data, no arithmetic of the method.
+
+The DFG is the *input* of TSPLIT (§II: "the computation of DNNs is
+typically expressed as a dataflow graph (DFG) ... nodes are operations, and the
+edges are tensors"; Alg. 1 "Data: G: Computation Graph", L62-75).  This module
+only lists tensors (name, dtype, shape, kind) and operations (kind, inputs,
+outputs, attributes) for the networks named in BASELINE.json's configs.  Both
+the fp64 oracle (`oracle/`) and the product binding consume these lists; neither
+side's computation lives here.
+
+Tensor kinds: "param" (model weights, static region), "input" (sample data),
+"label", "act" (activations produced by an op).  Every non-param tensor except
+the scalar loss has a leading *sample* dimension of `samples` (batch) units —
+the dimension TSPLIT splits along ("split along the dim of sample").
+
+Operation kinds and attributes (semantics in DESIGN.md §3):
+  linear     in (X[R,K], W[N,K], b[N])      out Y[R,N] = X W^T + b
+  relu/gelu/tanh  in (X)                    out elementwise
+  layernorm  in (X[R,H], gamma[H], beta[H]) out;  f: eps
+  add        in (A, B)                      out A + B
+  dropout    in (X)                         out; f: p, i: seed (Philox counter)
+  softmax    in (X[..., L])                 out row softmax over the last dim
+  attn_qk    in (Q[T,h], K[T,h])            out S[b,a,s,s] = alpha Q_h K_h^T; i: heads, seq; f: alpha
+  attn_pv    in (P[b,a,s,s], V[T,h])        out C[T,h] (heads re-merged); i: heads, seq
+  embed      in (ids[T], tt[T], Wword[V,h], Wpos[S,h], Wtype[2,h])  out [T,h]; i: seq
+  cls        in (X[T,h])                    out [b,h] = rows b*seq; i: seq
+  xent       in (logits[b,C], labels[b])    out loss[1] = mean_b CE (global batch)
+"""
+
+from __future__ import annotations
+
+import math
+
+DTYPE_BYTES = {"f32": 4, "bf16": 2, "i32": 4}
+
+
+class GraphBuilder:
+    def __init__(self, name: str, dtype: str, samples: int):
+        self.name = name
+        self.dtype = dtype
+        self.samples = samples
+        self.tensors: list[dict] = []
+        self.ops: list[dict] = []
+
+    def tensor(self, name, shape, kind, dtype=None):
+        t = {
+            "id": len(self.tensors),
+            "name": name,
+            "dtype": dtype or self.dtype,
+            "shape": tuple(int(s) for s in shape),
+            "kind": kind,
+        }
+        self.tensors.append(t)
+        return t["id"]
+
+    def param(self, name, shape):
+        return self.tensor(name, shape, "param")
+
+    def op(self, kind, name, inputs, out_shape, out_name=None, iattrs=(), fattrs=(), out_dtype=None):
+        out = self.tensor(out_name or name, out_shape, "act", dtype=out_dtype)
+        self.ops.append({
+            "id": len(self.ops),
+            "kind": kind,
+            "name": name,
+            "inputs": list(inputs),
+            "outputs": [out],
+            "iattrs": [int(v) for v in iattrs],
+            "fattrs": [float(v) for v in fattrs],
+        })
+        return out
+
+    def done(self) -> dict:
+        return {
+            "name": self.name,
+            "dtype": self.dtype,
+            "samples": self.samples,
+            "tensors": self.tensors,
+            "ops": self.ops,
+        }
+
+
+def mlp(batch=8, hidden=256, depth=3, in_dim=256, classes=10, dtype="f32") -> dict:
+    """Config 1 (BASELINE.json configs[0]): 3-layer MLP 256->256->256->10, ReLU.
+
+    5 forward ops + loss.
+    """
+    g = GraphBuilder(f"mlp{depth}_h{hidden}_b{batch}", dtype, batch)
+    x = g.tensor("x", (batch, in_dim), "input")
+    y = g.tensor("labels", (batch,), "label", dtype="i32")
+    h = x
+    dims = [in_dim] + [hidden] * (depth - 1) + [classes]
+    for li in range(depth):
+        w = g.param(f"fc{li}.w", (dims[li + 1], dims[li]))
+        b = g.param(f"fc{li}.b", (dims[li + 1],))
+        h = g.op("linear", f"fc{li}", [h, w, b], (batch, dims[li + 1]))
+        if li < depth - 1:
+            h = g.op("relu", f"relu{li}", [h], (batch, dims[li + 1]))
+    g.op("xent", "loss", [h, y], (1,), out_dtype="f32")
+    return g.done()
+
+
+def bert(layers=24, hidden=1024, heads=16, seq=512, batch=32, vocab=30522, ffn=None,
+         classes=2, dtype="bf16", attn_dropout=0.1, emb_dropout=0.1, seed=1234) -> dict:
+    """Canonical unfused BERT encoder + pooler/classifier head (MRPC-like).
+
+    Per layer it emits exactly the tensors SURVEY.md §4 T2 reconciles with
+    PAPER.md Table II (L85-112): 3 x [b,a,s,s] (scores, softmax, attention
+    dropout), 2 x [T,4h] (FFN1, GELU), 10 x [T,h] (Q, K, V, context, proj, res1,
+    LN1, FFN2, res2, LN2), weights 2 x [h,4h] and 4 x [h,h].
+    """
+    ffn = ffn or 4 * hidden
+    assert hidden % heads == 0
+    dh = hidden // heads
+    T = batch * seq
+    g = GraphBuilder(f"bert_L{layers}_h{hidden}_a{heads}_s{seq}_b{batch}", dtype, batch)
+    ids = g.tensor("input_ids", (T,), "input", dtype="i32")
+    tts = g.tensor("token_type_ids", (T,), "input", dtype="i32")
+    labels = g.tensor("labels", (batch,), "label", dtype="i32")
+    wword = g.param("emb.word", (vocab, hidden))
+    wpos = g.param("emb.pos", (seq, hidden))
+    wtype = g.param("emb.type", (2, hidden))
+    e = g.op("embed", "emb", [ids, tts, wword, wpos, wtype], (T, hidden), iattrs=[seq])
+    lg = g.param("emb.ln.g", (hidden,))
+    lb = g.param("emb.ln.b", (hidden,))
+    e = g.op("layernorm", "emb.ln", [e, lg, lb], (T, hidden), fattrs=[1e-12])
+    x = g.op("dropout", "emb.drop", [e], (T, hidden), fattrs=[emb_dropout], iattrs=[seed])
+    alpha = 1.0 / math.sqrt(dh)
+    for l in range(layers):
+        p = f"l{l}."
+
+        def lin(name, inp, n_out, n_in):
+            w = g.param(p + name + ".w", (n_out, n_in))
+            b = g.param(p + name + ".b", (n_out,))
+            return g.op("linear", p + name, [inp, w, b], (T, n_out))
+
+        q = lin("q", x, hidden, hidden)
+        k = lin("k", x, hidden, hidden)
+        v = lin("v", x, hidden, hidden)
+        s = g.op("attn_qk", p + "scores", [q, k], (batch, heads, seq, seq), iattrs=[heads, seq], fattrs=[alpha])
+        pr = g.op("softmax", p + "probs", [s], (batch, heads, seq, seq))
+        pd = g.op("dropout", p + "attn_drop", [pr], (batch, heads, seq, seq), fattrs=[attn_dropout],
+                  iattrs=[seed + 1 + l])
+        c = g.op("attn_pv", p + "ctx", [pd, v], (T, hidden), iattrs=[heads, seq])
+        o = lin("proj", c, hidden, hidden)
+        r1 = g.op("add", p + "res1", [o, x], (T, hidden))
+        g1 = g.param(p + "ln1.g", (hidden,))
+        b1 = g.param(p + "ln1.b", (hidden,))
+        n1 = g.op("layernorm", p + "ln1", [r1, g1, b1], (T, hidden), fattrs=[1e-12])
+        f1 = lin("ffn1", n1, ffn, hidden)
+        ge = g.op("gelu", p + "gelu", [f1], (T, ffn))
+        f2 = lin("ffn2", ge, hidden, ffn)
+        r2 = g.op("add", p + "res2", [f2, n1], (T, hidden))
+        g2 = g.param(p + "ln2.g", (hidden,))
+        b2 = g.param(p + "ln2.b", (hidden,))
+        x = g.op("layernorm", p + "ln2", [r2, g2, b2], (T, hidden), fattrs=[1e-12])
+    cls = g.op("cls", "pool.cls", [x], (batch, hidden), iattrs=[seq])
+    pw = g.param("pool.w", (hidden, hidden))
+    pb = g.param("pool.b", (hidden,))
+    pl = g.op("linear", "pool.fc", [cls, pw, pb], (batch, hidden))
+    pt = g.op("tanh", "pool.tanh", [pl], (batch, hidden))
+    cw = g.param("cls.w", (classes, hidden))
+    cb = g.param("cls.b", (classes,))
+    lo = g.op("linear", "cls.fc", [pt, cw, cb], (batch, classes))
+    g.op("xent", "loss", [lo, labels], (1,), out_dtype="f32")
+    return g.done()
+
+
+def tensor_bytes(t: dict) -> int:
+    n = 1
+    for s in t["shape"]:
+        n *= s
+    return n * DTYPE_BYTES[t["dtype"]]
+
+
+def config_graph(name: str, **over) -> dict:
+    """Graphs for BASELINE.json configs by short name."""
+    if name == "mlp":
+        return mlp(**over)
+    if name == "bert_large":
+        kw = dict(layers=24, hidden=1024, heads=16, seq=512, batch=32)
+        kw.update(over)
+        return bert(**kw)
+    if name == "bert_tiny":
+        kw = dict(layers=2, hidden=128, heads=2, seq=64, batch=4, vocab=512)
+        kw.update(over)
+        return bert(**kw)
+    if name == "bert_scaled":
+        kw = dict(layers=24, hidden=2560, heads=40, seq=512, batch=64)
+        kw.update(over)
+        return bert(**kw)
+    raise KeyError(name)
