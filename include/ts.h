@@ -1,0 +1,247 @@
+/*
+ * ts.h — C ABI of the B200-native TSPLIT hot path.
+ *
+ * TSPLIT (Nie et al., ICDE'22, /root/reference/PAPER.md, cited "P:L<line>")
+ * takes a dataflow graph and an available GPU memory M and finds, for every
+ * tensor, a configuration {opt, p_num, dim} (§IV-A Eq. 1, §V-A,
+ * Fig. 9 `struct config`) so that the memory requirement M_i of every
+ * operation stays under M while the added time is small; it then executes the
+ * augmented graph (Fig. 10) with a compute stream, a D2H stream and
+ * an H2D stream ordered by CUDA events over a pre-allocated pool.
+ *
+ * Conventions for every entry point:
+ *  - Returns ts_status; on failure the out-parameters are untouched and
+ *    ts_last_error() returns a thread-local message.
+ *  - Arrays passed in are copied at call time (the caller keeps ownership).
+ *  - Handles are owned by the caller until the matching *_destroy.
+ *  - "device pointer" arguments are CUDA device addresses on the session's
+ *    device; "host pointer" arguments are ordinary (pageable or pinned) host
+ *    memory.  No torch types cross this boundary.
+ *  - Sizes are in bytes unless stated; shapes are row-major (last dim
+ *    contiguous).  Tensor ids are indices into the descriptor array.
+ */
+#ifndef TSPLIT_TS_H
+#define TSPLIT_TS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  TS_OK = 0,
+  TS_ERR_ARG = 1,         /* bad argument (null pointer, out-of-range id, bad size) */
+  TS_ERR_GRAPH = 2,       /* graph does not validate (shape mismatch, cycle, ...)   */
+  TS_ERR_INFEASIBLE = 3,  /* Alg. 2 ran out of candidates ("fail because of
+                             no more available tensors"); message names the op     */
+  TS_ERR_BUDGET = 4,      /* runtime pool overflow: the slab is smaller than the plan */
+  TS_ERR_HOST_MEM = 5,    /* pinned host pool allocation failed                     */
+  TS_ERR_CUDA = 6,        /* a CUDA runtime/driver call failed (message has it)     */
+  TS_ERR_NCCL = 7,        /* NCCL failure                                           */
+  TS_ERR_STATE = 8,       /* call made in the wrong order / unsupported here        */
+  TS_ERR_NO_GPU = 9       /* no CUDA device: compute entry points refuse (no CPU fallback) */
+} ts_status;
+
+typedef enum { TS_F32 = 0, TS_BF16 = 1, TS_I32 = 2 } ts_dtype;
+typedef enum { TS_PARAM = 0, TS_INPUT = 1, TS_LABEL = 2, TS_ACT = 3 } ts_kind;
+/* Fig. 9 `opt`: memory option of every micro-tensor of a tensor. */
+typedef enum { TS_RESIDE = 0, TS_SWAP = 1, TS_RECOMPUTE = 2 } ts_opt;
+
+/* Operation kinds; semantics and attribute layout in DESIGN.md §3. */
+typedef enum {
+  TS_OP_LINEAR = 0,    /* in X[R,K], W[N,K], b[N]      out Y = X W^T + b              */
+  TS_OP_RELU = 1,
+  TS_OP_GELU = 2,      /* erf GELU                                                     */
+  TS_OP_TANH = 3,
+  TS_OP_LAYERNORM = 4, /* in X[R,H], gamma, beta; fattr[0] = eps                       */
+  TS_OP_ADD = 5,
+  TS_OP_DROPOUT = 6,   /* fattr[0] = p; iattr[0] = seed (Philox4x32-10 key)             */
+  TS_OP_SOFTMAX = 7,   /* over the last dim                                            */
+  TS_OP_ATTN_QK = 8,   /* in Q[T,h], K[T,h] out S[b,a,s,s]; iattr {heads, seq}; fattr[0] = alpha */
+  TS_OP_ATTN_PV = 9,   /* in P[b,a,s,s], V[T,h] out C[T,h]; iattr {heads, seq}         */
+  TS_OP_EMBED = 10,    /* in ids, type_ids (i32 [T]), Wword, Wpos, Wtype; iattr[0] = seq */
+  TS_OP_CLS = 11,      /* in X[T,h] out [b,h] (row b*seq); iattr[0] = seq              */
+  TS_OP_XENT = 12      /* in logits[b,C], labels i32[b] out loss f32[1], mean over the
+                          global batch                                     */
+} ts_op_kind;
+
+typedef struct {
+  int32_t dtype;       /* ts_dtype */
+  int32_t kind;        /* ts_kind  */
+  int32_t ndim;        /* 1..6     */
+  int64_t shape[6];    /* leading dim of every non-param tensor except the loss is a
+                          multiple of `samples` (the split "sample" dim)      */
+} ts_tensor_desc;
+
+typedef struct {
+  int32_t kind;        /* ts_op_kind */
+  int32_t n_in, n_out;
+  const int32_t* in;   /* tensor ids */
+  const int32_t* out;
+  int32_t n_iattr;
+  const int64_t* iattr;
+  int32_t n_fattr;
+  const double* fattr;
+} ts_op_desc;
+
+/* Per-tensor configuration: Fig. 9 `struct config` {opt, p_num, dim} plus the
+ * prefetch lead of a swapped tensor (swap-in starts `prefetch_lead` compute
+ * items before its first backward use; 1 = "the previous computation
+ * operation").  dim 0 = the sample dim (the only one in this build). */
+typedef struct {
+  int32_t tensor_id;
+  int32_t opt;           /* ts_opt */
+  int32_t p_num;         /* 1, 2, 4, 8, 16; must divide `samples` */
+  int32_t dim;
+  int32_t prefetch_lead; /* >= 1 */
+} ts_tensor_cfg;
+
+typedef struct {
+  uint64_t static_bytes;   /* params (fp32 master [+bf16 copy] + fp32 grad) + workspace */
+  uint64_t peak_live;      /* static + max_i sum of live micro-tensor bytes (M_i) */
+  uint64_t peak_extent;    /* highest pool offset used (includes fragmentation)          */
+  uint64_t d2h_bytes;      /* swap-out bytes per step                                    */
+  uint64_t h2d_bytes;      /* swap-in bytes per step                                     */
+  int64_t n_items;         /* augmented schedule length                                  */
+  int64_t n_compute;       /* forward + backward micro-ops                               */
+  int64_t n_replay;        /* recompute replays (memory-centric)                 */
+  double predicted_s;      /* planner's predicted step time                              */
+  double compute_flop;     /* algorithmic FLOP per step incl. replays                    */
+  int64_t n_split_tensors; /* tensors with p_num > 1                                     */
+  int64_t n_swap_tensors;
+  int64_t n_recompute_tensors;
+} ts_plan_stats_t;
+
+typedef struct {
+  int64_t seq;
+  int32_t item;          /* augmented-schedule index, -1 = step start           */
+  int32_t kind;          /* 0 = ALLOC, 1 = FREE                                 */
+  int32_t key;           /* tensor id, or n_tensors + id for its gradient       */
+  int32_t piece;         /* micro-tensor index                                   */
+  uint64_t offset;       /* byte offset in the pool slab                        */
+  uint64_t bytes;        /* unaligned size                                      */
+} ts_alloc_event;
+
+/* Hardware model used by the planner (bytes/s and FLOP/s). */
+typedef struct {
+  double tensor_flops;   /* dense bf16 tensor FLOP/s (MEASURED_PEAKS bf16_tflops_sustained) */
+  double simt_flops;     /* fp32 FFMA FLOP/s                                          */
+  double hbm_bw;         /* HBM bytes/s (MEASURED_PEAKS hbm_gbs)                       */
+  double d2h_bw, h2d_bw; /* PCIe bytes/s, measured per pod                             */
+  double launch_s;       /* per-kernel overhead inside a CUDA graph                     */
+} ts_hw;
+
+typedef struct ts_graph_s ts_graph_t;
+typedef struct ts_profile_s ts_profile_t;
+typedef struct ts_plan_s ts_plan_t;
+typedef struct ts_session_s ts_session_t;
+
+const char* ts_last_error(void);
+const char* ts_version(void);
+
+/* ---- graph (host only) ------------------------------------------------------ */
+/* Validates the DFG and builds the Alg. 1 forward schedule (read as
+ * ref_cnt -= 1 / == 0); backward = reverse order (R2). */
+ts_status ts_graph_define(const ts_tensor_desc* tensors, int32_t n_tensors,
+                          const ts_op_desc* ops, int32_t n_ops,
+                          int32_t samples, int32_t compute_dtype, ts_graph_t** out);
+void ts_graph_destroy(ts_graph_t* g);
+/* Writes the forward schedule O (op ids) into order[cap]; *n = number of ops. */
+ts_status ts_graph_schedule(const ts_graph_t* g, int32_t* order, int32_t cap, int32_t* n);
+ts_status ts_graph_static_bytes(const ts_graph_t* g, uint64_t* out);
+
+/* ---- profile --------------------------------- */
+/* Analytic profile from a hardware model: per-op T(p) = launch + max(flop/peak,
+ * bytes/bw) for every p in {1,2,4,8,16}. */
+ts_status ts_profile_analytic(const ts_graph_t* g, const ts_hw* hw, ts_profile_t** out);
+/* Overwrite one measured entry: op id, p_num, forward and backward seconds of the
+ * WHOLE op (sum over its p_num micro-ops), e.g. from cudaEvent timing. */
+ts_status ts_profile_set(ts_profile_t* pr, int32_t op, int32_t p_num, double fwd_s, double bwd_s);
+ts_status ts_profile_set_pcie(ts_profile_t* pr, double d2h_bw, double h2d_bw);
+void ts_profile_destroy(ts_profile_t* pr);
+
+/* ---- plan ------------------------------------------------------------------- */
+/* All tensors reside, p_num = 1 (the "Base" of P:L304). */
+ts_status ts_plan_default(const ts_graph_t* g, ts_plan_t** out);
+/* Profiling-based greedy planning (Alg. 2, reconstructed from P:L178/L270, SURVEY
+ * R8) under `budget_bytes` for the whole pool (static + dynamic, R4).  `profile`
+ * may be NULL (analytic model with B200 defaults).  Returns TS_ERR_INFEASIBLE
+ * when no candidate remains. */
+ts_status ts_plan(const ts_graph_t* g, uint64_t budget_bytes, const ts_profile_t* profile, ts_plan_t** out);
+ts_status ts_plan_get(const ts_plan_t* p, int32_t tensor_id, ts_tensor_cfg* out);
+/* Forced configuration (Fig. 9 set_config); the plan is re-expanded and
+ * re-simulated.  Only TS_ACT tensors accept opt != RESIDE or p_num > 1. */
+ts_status ts_plan_set(ts_plan_t* p, const ts_tensor_cfg* cfg);
+ts_status ts_plan_stats(const ts_plan_t* p, ts_plan_stats_t* out);
+/* Simulated allocation trace (R3, R11); *n = total events (buf may be NULL). */
+ts_status ts_plan_trace(const ts_plan_t* p, ts_alloc_event* buf, uint64_t cap, uint64_t* n);
+/* Augmented schedule as int32 quadruples (kind, op, k, aux) — kind 0 F, 1 B, 2 R,
+ * 3 SO, 4 SI; aux = piece key for SO/SI (key*65536+piece), else group id. */
+ts_status ts_plan_items(const ts_plan_t* p, int32_t* buf, uint64_t cap, uint64_t* n);
+ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n);
+ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, ts_plan_t** out);
+void ts_plan_destroy(ts_plan_t* p);
+
+/* ---- session (device) ---------------------------------------------------------- */
+typedef struct {
+  int32_t device;            /* CUDA ordinal                                          */
+  void* slab;                /* device pointer lent by the caller (torch), >= bytes   */
+  uint64_t slab_bytes;       /* the pool: static region + dynamic pool (= budget)     */
+  void* stream_compute;      /* cudaStream_t or NULL (session creates its own)        */
+  void* stream_d2h;
+  void* stream_h2d;
+  void* nccl_comm;           /* ncclComm_t for data-parallel allreduce, or NULL       */
+  int32_t world_size;        /* gradient scale 1/world after the allreduce            */
+  int32_t use_cuda_graph;    /* capture the whole step once and replay it             */
+  float lr;                  /* SGD learning rate (0 = no update)                     */
+  uint32_t step0;            /* dropout counter base                                  */
+} ts_session_cfg;
+
+/* Lays out the static region, allocates the pinned host swap pool, uploads
+ * nothing (parameters start at zero until ts_set_param). */
+ts_status ts_session_create(const ts_graph_t* g, const ts_plan_t* p, const ts_session_cfg* cfg,
+                            ts_session_t** out);
+void ts_session_destroy(ts_session_t* s);
+/* Upload a parameter from host fp32 (count = numel); also refreshes its bf16 copy. */
+ts_status ts_set_param(ts_session_t* s, int32_t tensor_id, const float* host_f32);
+/* Download the fp32 master / fp32 gradient of a parameter to host. */
+ts_status ts_get_param(ts_session_t* s, int32_t tensor_id, float* host_f32);
+ts_status ts_get_grad(ts_session_t* s, int32_t tensor_id, float* host_f32);
+ts_status ts_param_ptr(ts_session_t* s, int32_t tensor_id, void** dev_f32);
+ts_status ts_grad_ptr(ts_session_t* s, int32_t tensor_id, void** dev_f32);
+/* One training step: forward, backward, allreduce (if a comm is set), SGD.
+ * inputs[i] = pointer to the i-th INPUT/LABEL tensor in tensor-id order
+ * (int32 or the graph dtype), on the host if inputs_on_host != 0 (copied H2D
+ * inside the step) else on the device (copied D2D).  Synchronous on return;
+ * *loss_out = the global-batch mean loss of this rank's samples. */
+ts_status ts_step(ts_session_t* s, const void* const* inputs, int32_t inputs_on_host, float* loss_out);
+/* Same as ts_step but does not synchronise or read the loss back (bench loop). */
+ts_status ts_step_async(ts_session_t* s, const void* const* inputs, int32_t inputs_on_host);
+/* Allocation trace the runtime recorded on its last step (must equal ts_plan_trace). */
+ts_status ts_session_trace(const ts_session_t* s, ts_alloc_event* buf, uint64_t cap, uint64_t* n);
+/* Kernel launches per step issued by the session (for gpu_launches accounting). */
+ts_status ts_session_launches(const ts_session_t* s, int64_t* n);
+/* Device time of the last step's compute-stream items, by op kind and phase
+ * (seconds, cudaEvent; only when profiling was enabled). */
+ts_status ts_session_profile_items(ts_session_t* s, int32_t enable);
+ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, uint64_t* n);
+
+/* ---- kernels exposed for unit tests (device pointers, compute stream) -------- */
+/* C[b] = alpha * op(A[b]) op(B[b]) (+ beta*C + bias): bf16 in, fp32 accumulate on
+ * tcgen05 (TMEM), out bf16 or f32.  ta/tb = 1 when the operand's contiguous dim is
+ * M (resp. N) rather than K.  Strides are in elements. */
+ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch,
+                       const void* A, int64_t lda, int64_t strideA, int32_t ta,
+                       const void* B, int64_t ldb, int64_t strideB, int32_t tb,
+                       void* C, int64_t ldc, int64_t strideC, int32_t c_dtype,
+                       float alpha, float beta, const void* bias_bf16, void* stream);
+ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K,
+                      const float* A, int64_t lda, int32_t ta,
+                      const float* B, int64_t ldb, int32_t tb,
+                      float* C, int64_t ldc, float alpha, float beta, const float* bias, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,244 @@
+// C ABI: graph, profile and plan entry points (host only; no CUDA calls).
+#include <cstring>
+#include <memory>
+#include <new>
+
+#include "capi_internal.h"
+
+namespace ts {
+thread_local std::string g_last_error;
+void set_error(const std::string& msg) { g_last_error = msg; }
+}  // namespace ts
+
+using namespace ts;
+
+extern "C" {
+
+const char* ts_last_error(void) { return g_last_error.c_str(); }
+const char* ts_version(void) { return "tsplit-b200 0.1 (sm_100a)"; }
+
+ts_status ts_graph_define(const ts_tensor_desc* tensors, int32_t n_tensors, const ts_op_desc* ops,
+                          int32_t n_ops, int32_t samples, int32_t compute_dtype, ts_graph_t** out) {
+  if (!out) return set_error("out is null"), TS_ERR_ARG;
+  auto g = std::make_unique<ts_graph_t>();
+  ts_status st = build_graph(tensors, n_tensors, ops, n_ops, samples, compute_dtype, g->g);
+  if (st != TS_OK) return st;
+  *out = g.release();
+  return TS_OK;
+}
+
+void ts_graph_destroy(ts_graph_t* g) { delete g; }
+
+ts_status ts_graph_schedule(const ts_graph_t* g, int32_t* order, int32_t cap, int32_t* n) {
+  if (!g || !n) return set_error("null argument"), TS_ERR_ARG;
+  *n = (int32_t)g->g.order.size();
+  if (order)
+    for (int i = 0; i < (int)g->g.order.size() && i < cap; ++i) order[i] = g->g.order[i];
+  return TS_OK;
+}
+
+ts_status ts_graph_static_bytes(const ts_graph_t* g, uint64_t* out) {
+  if (!g || !out) return set_error("null argument"), TS_ERR_ARG;
+  *out = g->g.static_bytes;
+  return TS_OK;
+}
+
+ts_status ts_profile_analytic(const ts_graph_t* g, const ts_hw* hw, ts_profile_t** out) {
+  if (!g || !out) return set_error("null argument"), TS_ERR_ARG;
+  auto p = std::make_unique<ts_profile_t>();
+  profile_analytic(g->g, hw ? *hw : default_hw(), p->pr);
+  *out = p.release();
+  return TS_OK;
+}
+
+ts_status ts_profile_set(ts_profile_t* pr, int32_t op, int32_t p_num, double fwd_s, double bwd_s) {
+  if (!pr || op < 0 || op >= (int)pr->pr.tf.size()) return set_error("bad op"), TS_ERR_ARG;
+  int l = 0;
+  while ((1 << l) < p_num && l < 4) ++l;
+  if ((1 << l) != p_num) return set_error("p_num must be 1,2,4,8,16"), TS_ERR_ARG;
+  pr->pr.tf[op][l] = fwd_s;
+  pr->pr.tb[op][l] = bwd_s;
+  return TS_OK;
+}
+
+ts_status ts_profile_set_pcie(ts_profile_t* pr, double d2h_bw, double h2d_bw) {
+  if (!pr || d2h_bw <= 0 || h2d_bw <= 0) return set_error("bad bandwidth"), TS_ERR_ARG;
+  pr->pr.hw.d2h_bw = d2h_bw;
+  pr->pr.hw.h2d_bw = h2d_bw;
+  return TS_OK;
+}
+
+void ts_profile_destroy(ts_profile_t* pr) { delete pr; }
+
+static ts_plan_t* new_plan(const ts_graph_t* g) {
+  auto* p = new (std::nothrow) ts_plan_t();
+  if (!p) return nullptr;
+  p->graph = &g->g;
+  p->st.cfg.assign(g->g.n(), Cfg());
+  return p;
+}
+
+ts_status ts_plan_default(const ts_graph_t* g, ts_plan_t** out) {
+  if (!g || !out) return set_error("null argument"), TS_ERR_ARG;
+  ts_plan_t* p = new_plan(g);
+  Profile pr;
+  profile_analytic(g->g, default_hw(), pr);
+  plan_refresh(g->g, p->st, &pr);
+  p->budget = p->st.sim.peak_extent;
+  *out = p;
+  return TS_OK;
+}
+
+ts_status ts_plan(const ts_graph_t* g, uint64_t budget_bytes, const ts_profile_t* profile, ts_plan_t** out) {
+  if (!g || !out) return set_error("null argument"), TS_ERR_ARG;
+  std::unique_ptr<ts_plan_t> p(new_plan(g));
+  Profile local;
+  const Profile* pr = profile ? &profile->pr : nullptr;
+  if (!pr) {
+    profile_analytic(g->g, default_hw(), local);
+    pr = &local;
+  }
+  ts_status st = plan_greedy(g->g, budget_bytes, *pr, p->st);
+  if (st != TS_OK) return st;
+  p->budget = budget_bytes;
+  *out = p.release();
+  return TS_OK;
+}
+
+ts_status ts_plan_get(const ts_plan_t* p, int32_t tid, ts_tensor_cfg* out) {
+  if (!p || !out || tid < 0 || tid >= p->graph->n()) return set_error("bad argument"), TS_ERR_ARG;
+  const Cfg& c = p->st.cfg[tid];
+  out->tensor_id = tid;
+  out->opt = c.opt;
+  out->p_num = c.p;
+  out->dim = c.dim;
+  out->prefetch_lead = c.lead;
+  return TS_OK;
+}
+
+ts_status ts_plan_set(ts_plan_t* p, const ts_tensor_cfg* cfg) {
+  if (!p || !cfg) return set_error("null argument"), TS_ERR_ARG;
+  const Graph& g = *p->graph;
+  int t = cfg->tensor_id;
+  if (t < 0 || t >= g.n()) return set_error("bad tensor id"), TS_ERR_ARG;
+  bool pow2 = cfg->p_num >= 1 && cfg->p_num <= 16 && (cfg->p_num & (cfg->p_num - 1)) == 0;
+  if (!pow2 || g.samples % cfg->p_num) return set_error("p_num must be a power of 2 <= 16 dividing samples"), TS_ERR_ARG;
+  if (cfg->opt < 0 || cfg->opt > 2 || cfg->dim != 0 || cfg->prefetch_lead < 1)
+    return set_error("bad opt/dim/prefetch_lead (only the sample dim 0 is splittable)"), TS_ERR_ARG;
+  const Tensor& x = g.t[t];
+  if ((x.kind != TS_ACT || x.is_loss) && (cfg->opt != TS_RESIDE || cfg->p_num != 1))
+    return set_error("only activations can be split, swapped or recomputed"), TS_ERR_ARG;
+  Cfg& c = p->st.cfg[t];
+  c.opt = cfg->opt;
+  c.p = cfg->p_num;
+  c.dim = cfg->dim;
+  c.lead = cfg->prefetch_lead;
+  Profile pr;
+  profile_analytic(g, default_hw(), pr);
+  plan_refresh(g, p->st, &pr);
+  return TS_OK;
+}
+
+ts_status ts_plan_stats(const ts_plan_t* p, ts_plan_stats_t* out) {
+  if (!p || !out) return set_error("null argument"), TS_ERR_ARG;
+  const auto& s = p->st;
+  std::memset(out, 0, sizeof(*out));
+  out->static_bytes = p->graph->static_bytes;
+  out->peak_live = s.sim.peak_live;
+  out->peak_extent = s.sim.peak_extent;
+  out->d2h_bytes = s.sim.d2h;
+  out->h2d_bytes = s.sim.h2d;
+  out->n_items = (int64_t)s.ex.items.size();
+  out->n_compute = s.sim.n_compute;
+  out->n_replay = s.sim.n_replay;
+  out->predicted_s = s.predicted_s;
+  out->compute_flop = s.flop;
+  for (int t = 0; t < p->graph->n(); ++t) {
+    const Cfg& c = s.cfg[t];
+    out->n_split_tensors += c.p > 1;
+    out->n_swap_tensors += c.opt == TS_SWAP;
+    out->n_recompute_tensors += c.opt == TS_RECOMPUTE;
+  }
+  return TS_OK;
+}
+
+static void copy_events(const std::vector<Event>& tr, ts_alloc_event* buf, uint64_t cap, uint64_t* n) {
+  *n = tr.size();
+  if (!buf) return;
+  for (uint64_t i = 0; i < tr.size() && i < cap; ++i) {
+    const Event& e = tr[i];
+    buf[i] = ts_alloc_event{e.seq, e.item, e.kind, e.key, e.piece, e.offset, e.bytes};
+  }
+}
+
+ts_status ts_plan_trace(const ts_plan_t* p, ts_alloc_event* buf, uint64_t cap, uint64_t* n) {
+  if (!p || !n) return set_error("null argument"), TS_ERR_ARG;
+  copy_events(p->st.sim.trace, buf, cap, n);
+  return TS_OK;
+}
+
+ts_status ts_plan_items(const ts_plan_t* p, int32_t* buf, uint64_t cap, uint64_t* n) {
+  if (!p || !n) return set_error("null argument"), TS_ERR_ARG;
+  const auto& items = p->st.ex.items;
+  *n = items.size();
+  if (!buf) return TS_OK;
+  for (uint64_t i = 0; i < items.size() && (i + 1) * 4 <= cap; ++i) {
+    const Item& it = items[i];
+    int32_t aux = it.group;
+    if (it.kind == IT_SO) aux = pk_key(it.reads[0]) * 65536 + pk_j(it.reads[0]);
+    if (it.kind == IT_SI) aux = pk_key(it.writes[0]) * 65536 + pk_j(it.writes[0]);
+    buf[4 * i + 0] = it.kind;
+    buf[4 * i + 1] = it.op;
+    buf[4 * i + 2] = it.k;
+    buf[4 * i + 3] = aux;
+  }
+  return TS_OK;
+}
+
+// Serialized form: magic, n_tensors, budget, then (opt, p, dim, lead) per tensor.
+ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n) {
+  if (!p || !n) return set_error("null argument"), TS_ERR_ARG;
+  const int nt = p->graph->n();
+  uint64_t need = 16 + 16ull * nt;
+  *n = need;
+  if (!buf) return TS_OK;
+  if (cap < need) return set_error("buffer too small"), TS_ERR_ARG;
+  auto* w = static_cast<int32_t*>(buf);
+  w[0] = 0x54535031;  // 'TSP1'
+  w[1] = nt;
+  std::memcpy(w + 2, &p->budget, 8);
+  for (int t = 0; t < nt; ++t) {
+    const Cfg& c = p->st.cfg[t];
+    w[4 + 4 * t + 0] = c.opt;
+    w[4 + 4 * t + 1] = c.p;
+    w[4 + 4 * t + 2] = c.dim;
+    w[4 + 4 * t + 3] = c.lead;
+  }
+  return TS_OK;
+}
+
+ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, ts_plan_t** out) {
+  if (!g || !buf || !out) return set_error("null argument"), TS_ERR_ARG;
+  auto* r = static_cast<const int32_t*>(buf);
+  const int nt = g->g.n();
+  if (n < 16 || r[0] != 0x54535031 || r[1] != nt || n < 16 + 16ull * nt)
+    return set_error("not a plan for this graph"), TS_ERR_ARG;
+  std::unique_ptr<ts_plan_t> p(new_plan(g));
+  std::memcpy(&p->budget, r + 2, 8);
+  for (int t = 0; t < nt; ++t) {
+    Cfg& c = p->st.cfg[t];
+    c.opt = r[4 + 4 * t];
+    c.p = r[4 + 4 * t + 1];
+    c.dim = r[4 + 4 * t + 2];
+    c.lead = r[4 + 4 * t + 3];
+  }
+  Profile pr;
+  profile_analytic(g->g, default_hw(), pr);
+  plan_refresh(g->g, p->st, &pr);
+  *out = p.release();
+  return TS_OK;
+}
+
+void ts_plan_destroy(ts_plan_t* p) { delete p; }
+
+}  // extern "C"

@@ -1,0 +1,151 @@
+// Host-side core of the TSPLIT runtime: graph, Alg. 1 schedule, augmented
+// schedule expansion, best-fit pool simulation and the Alg. 2 planner.
+// Semantics: DESIGN.md §4 (readings R1-R3, R10-R12 of SURVEY.md §8(c)).
+#pragma once
+#include <array>
+#include <cstdint>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "../../../include/ts.h"
+
+namespace ts {
+
+constexpr uint64_t kAlign = 256;
+constexpr uint64_t kWsRows = 256;
+constexpr uint64_t kInf = uint64_t(1) << 62;
+
+inline uint64_t align_up(uint64_t n) { return (n + kAlign - 1) / kAlign * kAlign; }
+inline int dtype_bytes(int d) { return d == TS_BF16 ? 2 : 4; }
+
+void set_error(const std::string& msg);
+
+struct Tensor {
+  int id = 0, dtype = TS_F32, kind = TS_ACT, ndim = 0;
+  int64_t shape[6] = {0, 0, 0, 0, 0, 0};
+  int64_t numel = 0;
+  uint64_t bytes = 0;
+  bool sample = false;    // carries the split (sample) leading dim
+  bool is_loss = false;
+  bool needs_grad = false;
+  int producer = -1;
+  std::vector<int> consumers;  // op ids, ascending
+  int64_t rows_per_sample = 0; // shape[0] / samples
+  int64_t elems_per_sample = 0;
+};
+
+struct Op {
+  int id = 0, kind = 0;
+  std::vector<int> in, out;
+  std::vector<int64_t> ia;
+  std::vector<double> fa;
+  bool has_bwd = false;
+  std::vector<int> saved;  // non-param forward tensors the backward reads
+};
+
+struct Graph {
+  int samples = 1, dtype = TS_F32;
+  std::vector<Tensor> t;
+  std::vector<Op> ops;
+  std::vector<int> order;  // Alg. 1 forward schedule
+  int loss = -1;
+  // static region layout: masters | bf16 copies | grads | workspace
+  std::vector<uint64_t> master_off, copy_off, grad_off;
+  uint64_t ws_off = 0, ws_bytes = 0, static_bytes = 0;
+  int n() const { return (int)t.size(); }
+};
+
+// Build + validate; returns TS_OK or an error with set_error().
+ts_status build_graph(const ts_tensor_desc* td, int nt, const ts_op_desc* od, int no, int samples,
+                      int dtype, Graph& g);
+
+struct Cfg {
+  int opt = TS_RESIDE, p = 1, dim = 0, lead = 1;
+};
+
+// Piece = (key, j) with key = tensor id or n + id for the gradient of id.
+using PieceKey = int64_t;
+inline PieceKey pk(int key, int j) { return (int64_t(key) << 20) | int64_t(j); }
+inline int pk_key(PieceKey p) { return int(p >> 20); }
+inline int pk_j(PieceKey p) { return int(p & 0xFFFFF); }
+
+enum ItemKind : int { IT_F = 0, IT_B = 1, IT_R = 2, IT_SO = 3, IT_SI = 4 };
+
+struct Item {
+  int kind = IT_F, op = -1, k = 0, group = -1;
+  std::vector<PieceKey> reads, writes;
+};
+
+struct Expansion {
+  std::vector<Item> items;
+  std::vector<std::vector<PieceKey>> alloc_at;  // per item, ordered
+  std::vector<std::vector<PieceKey>> free_after;
+  int fwd_end = 0;
+  std::vector<int> P;  // micro-op count per op
+};
+
+struct Event {
+  int64_t seq;
+  int item, kind, key, piece;
+  uint64_t offset, bytes;
+};
+
+struct SimResult {
+  std::vector<Event> trace;
+  std::vector<uint64_t> top;   // per item: end of the highest live block after allocs
+  std::vector<uint64_t> live;  // per item: dynamic live bytes after allocs
+  uint64_t peak_live = 0, peak_extent = 0;
+  uint64_t d2h = 0, h2d = 0;
+  int64_t n_replay = 0, n_compute = 0;
+  std::unordered_map<PieceKey, uint64_t> offset;  // placement of each piece (last)
+};
+
+int piece_count(const Graph& g, const std::vector<Cfg>& cfg, int key);
+uint64_t piece_bytes(const Graph& g, const std::vector<Cfg>& cfg, int key);
+void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex);
+// capacity = kInf for planning; the runtime uses the slab size (identical trace if it fits).
+bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, uint64_t capacity,
+              SimResult& r, std::vector<std::vector<std::pair<PieceKey, uint64_t>>>* placements = nullptr);
+
+// Best-fit pool with the tail rule.
+class Pool {
+ public:
+  void reset(uint64_t base, uint64_t capacity);
+  bool alloc(uint64_t bytes, uint64_t* off);
+  void release(uint64_t off, uint64_t bytes);
+  uint64_t top() const;  // start of the tail block
+  uint64_t extent() const { return extent_; }
+
+ private:
+  std::vector<std::pair<uint64_t, uint64_t>> free_;  // (offset, len) sorted
+  uint64_t cap_ = 0, extent_ = 0;
+};
+
+// ---- profile + planner ------------------------------------------------------
+struct OpCost {
+  double flop_f = 0, flop_b = 0;    // whole op
+  double bytes_f = 0, bytes_b = 0;  // algorithmic HBM bytes, whole op
+  int kern_f = 1, kern_b = 1;       // kernels per micro-op
+};
+OpCost op_cost(const Graph& g, int op);
+
+struct Profile {
+  ts_hw hw;
+  // time[op][log2 p] for fwd and bwd (whole op, all micro-ops)
+  std::vector<std::array<double, 5>> tf, tb;
+};
+void profile_analytic(const Graph& g, const ts_hw& hw, Profile& pr);
+ts_hw default_hw();
+
+struct PlanState {
+  std::vector<Cfg> cfg;
+  Expansion ex;
+  SimResult sim;
+  double predicted_s = 0, flop = 0;
+};
+void plan_refresh(const Graph& g, PlanState& ps, const Profile* pr);
+ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps);
+
+}  // namespace ts
+

@@ -1,0 +1,329 @@
+// Augmented-schedule expansion and pool simulation.
+//   P:L262-264 Fig. 10 — split ops into p_num micro-ops, insert memory-option ops
+//   P:L287             — in-place re-split (a micro-op reads a sub-range of a piece),
+//                        best-fit allocation over one pre-allocated pool
+//   P:L281             — swap-out begins at generation, swap-in at the previous op
+//   P:L291             — compute / D2H / H2D streams, pre-allocated pool
+//   P:L293-294 Fig. 11 — memory-centric recompute (regenerate for every backward use)
+//   P:L56, P:L134      — allocate at the beginning, free at the end of an operation
+#include <algorithm>
+#include <functional>
+#include <map>
+#include <set>
+
+#include "core.h"
+
+namespace ts {
+
+int piece_count(const Graph& g, const std::vector<Cfg>& cfg, int key) {
+  int t = key >= g.n() ? key - g.n() : key;
+  const Tensor& x = g.t[t];
+  if (!x.sample || x.kind != TS_ACT) return 1;
+  return cfg[t].p;
+}
+
+uint64_t piece_bytes(const Graph& g, const std::vector<Cfg>& cfg, int key) {
+  int t = key >= g.n() ? key - g.n() : key;
+  return g.t[t].bytes / uint64_t(piece_count(g, cfg, key));
+}
+
+void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
+  const int n = g.n();
+  ex = Expansion();
+  ex.P.assign(g.ops.size(), 1);
+  for (auto& o : g.ops) {
+    int P = 1;
+    for (int x : o.in)
+      if (g.t[x].sample) P = std::max(P, piece_count(g, cfg, x));
+    for (int x : o.out)
+      if (g.t[x].sample) P = std::max(P, piece_count(g, cfg, x));
+    ex.P[o.id] = P;
+  }
+  auto piece = [&](int t, int k, int P) -> int {
+    if (!g.t[t].sample) return 0;
+    return k * piece_count(g, cfg, t) / P;
+  };
+  std::vector<Item>& items = ex.items;
+  // ---- forward phase: op-major micro-ops (R10) ------------------------------
+  for (int o : g.order) {
+    const Op& op = g.ops[o];
+    int P = ex.P[o];
+    for (int k = 0; k < P; ++k) {
+      Item it;
+      it.kind = IT_F;
+      it.op = o;
+      it.k = k;
+      for (int x : op.in)
+        if (g.t[x].sample) it.reads.push_back(pk(x, piece(x, k, P)));
+      for (int x : op.out) it.writes.push_back(pk(x, piece(x, k, P)));
+      items.push_back(std::move(it));
+    }
+  }
+  ex.fwd_end = (int)items.size();
+  // ---- backward phase: reverse order, replays inline --------------------------
+  int gid = 0;
+  for (auto rit = g.order.rbegin(); rit != g.order.rend(); ++rit) {
+    const Op& op = g.ops[*rit];
+    if (!op.has_bwd) continue;
+    int P = ex.P[op.id];
+    for (int k = 0; k < P; ++k) {
+      std::vector<Item> group;
+      std::set<PieceKey> regenerated;
+      std::function<void(int, int)> regen = [&](int t, int j) {
+        const Tensor& x = g.t[t];
+        if (x.kind != TS_ACT || cfg[t].opt != TS_RECOMPUTE) return;
+        if (regenerated.count(pk(t, j))) return;
+        const Op& po = g.ops[x.producer];
+        int Q = ex.P[po.id];
+        int pt = piece_count(g, cfg, t);
+        for (int kk = j * Q / pt; kk < (j + 1) * Q / pt; ++kk) {
+          for (int u : po.in)
+            if (g.t[u].sample) regen(u, piece(u, kk, Q));
+          Item r;
+          r.kind = IT_R;
+          r.op = po.id;
+          r.k = kk;
+          r.group = gid;
+          for (int u : po.in)
+            if (g.t[u].sample) r.reads.push_back(pk(u, piece(u, kk, Q)));
+          r.writes.push_back(pk(t, j));
+          group.push_back(std::move(r));
+        }
+        regenerated.insert(pk(t, j));
+      };
+      std::vector<PieceKey> saved;
+      for (int t : op.saved) saved.push_back(pk(t, piece(t, k, P)));
+      for (PieceKey s : saved) regen(pk_key(s), pk_j(s));
+      Item b;
+      b.kind = IT_B;
+      b.op = op.id;
+      b.k = k;
+      b.group = gid;
+      b.reads = saved;
+      for (int x : op.out)
+        if (!g.t[x].is_loss) b.reads.push_back(pk(n + x, piece(x, k, P)));
+      for (int x : op.in)
+        if (g.t[x].kind == TS_ACT && g.t[x].needs_grad) {
+          PieceKey w = pk(n + x, piece(x, k, P));
+          if (std::find(b.writes.begin(), b.writes.end(), w) == b.writes.end()) b.writes.push_back(w);
+        }
+      group.push_back(std::move(b));
+      for (auto& it : group) items.push_back(std::move(it));
+      ++gid;
+    }
+  }
+  const int nitems = (int)items.size();
+  // ---- lifetimes (R3, R12) --------------------------------------------------
+  std::map<PieceKey, std::vector<int>> touches;
+  for (int i = 0; i < nitems; ++i) {
+    for (PieceKey p : items[i].writes) touches[p].push_back(i);
+    for (PieceKey p : items[i].reads) touches[p].push_back(i);
+  }
+  std::vector<std::vector<PieceKey>> alloc_at(nitems), free_after(nitems), so_after(nitems), si_before(nitems);
+  for (auto& [pc, idx] : touches) {
+    std::sort(idx.begin(), idx.end());
+    idx.erase(std::unique(idx.begin(), idx.end()), idx.end());
+    int key = pk_key(pc);
+    int first = idx.front(), lastt = idx.back();
+    if (key >= n) {  // gradient piece
+      alloc_at[first].push_back(pc);
+      free_after[lastt].push_back(pc);
+      continue;
+    }
+    const Tensor& x = g.t[key];
+    if (x.kind == TS_INPUT || x.kind == TS_LABEL) {
+      free_after[lastt].push_back(pc);
+      continue;
+    }
+    if (x.is_loss) {
+      alloc_at[first].push_back(pc);
+      continue;
+    }
+    int last_fw = -1, first_bw = -1;
+    for (int i : idx) {
+      if (i < ex.fwd_end) last_fw = i;
+      else if (first_bw < 0) first_bw = i;
+    }
+    alloc_at[first].push_back(pc);  // first touch is its producing forward micro-op
+    int opt = cfg[key].opt;
+    if (first_bw < 0 || opt == TS_RESIDE) {
+      free_after[lastt].push_back(pc);
+    } else if (opt == TS_SWAP) {
+      so_after[last_fw].push_back(pc);
+      int pos = std::max(first_bw - std::max(1, cfg[key].lead), ex.fwd_end);
+      si_before[pos].push_back(pc);
+      free_after[lastt].push_back(pc);
+    } else {  // recompute: forward lifetime, then one temporary per backward group
+      free_after[last_fw].push_back(pc);
+      std::map<int, std::pair<int, int>> span;
+      for (int i : idx)
+        if (i >= ex.fwd_end) {
+          auto it = span.find(items[i].group);
+          if (it == span.end()) span[items[i].group] = {i, i};
+          else it->second.second = i;
+        }
+      for (auto& [gg, se] : span) {
+        alloc_at[se.first].push_back(pc);
+        free_after[se.second].push_back(pc);
+      }
+    }
+  }
+  // ---- final list with swap-out / swap-in items ------------------------------
+  std::vector<Item> fin;
+  fin.reserve(nitems * 2);
+  for (int i = 0; i < nitems; ++i) {
+    std::sort(si_before[i].begin(), si_before[i].end());
+    for (PieceKey pc : si_before[i]) {
+      Item si;
+      si.kind = IT_SI;
+      si.writes.push_back(pc);
+      ex.alloc_at.push_back({pc});
+      ex.free_after.push_back({});
+      fin.push_back(std::move(si));
+    }
+    const Item& it = items[i];
+    std::vector<PieceKey> order;
+    auto& al = alloc_at[i];
+    for (PieceKey p : it.writes)
+      if (std::find(al.begin(), al.end(), p) != al.end() && std::find(order.begin(), order.end(), p) == order.end())
+        order.push_back(p);
+    for (PieceKey p : it.reads)
+      if (std::find(al.begin(), al.end(), p) != al.end() && std::find(order.begin(), order.end(), p) == order.end())
+        order.push_back(p);
+    std::vector<PieceKey> fr = free_after[i];
+    std::sort(fr.begin(), fr.end());
+    ex.alloc_at.push_back(order);
+    ex.free_after.push_back(fr);
+    fin.push_back(it);
+    std::sort(so_after[i].begin(), so_after[i].end());
+    for (PieceKey pc : so_after[i]) {
+      Item so;
+      so.kind = IT_SO;
+      so.reads.push_back(pc);
+      ex.alloc_at.push_back({});
+      ex.free_after.push_back({pc});
+      fin.push_back(std::move(so));
+    }
+  }
+  // fwd_end in the final numbering = index of the first backward-phase item
+  int fe = 0;
+  for (size_t i = 0; i < fin.size(); ++i)
+    if (fin[i].kind == IT_F || fin[i].kind == IT_SO) fe = (int)i + 1;
+  ex.items = std::move(fin);
+  ex.fwd_end = fe;
+}
+
+// ---- pool --------------------------------------------------------------------
+void Pool::reset(uint64_t base, uint64_t capacity) {
+  cap_ = capacity;
+  extent_ = base;
+  free_.clear();
+  if (capacity > base) free_.push_back({base, capacity - base});
+}
+
+bool Pool::alloc(uint64_t bytes, uint64_t* off) {
+  uint64_t need = align_up(bytes);
+  int best = -1;
+  for (int i = 0; i < (int)free_.size(); ++i) {
+    if (free_[i].first + free_[i].second == cap_) continue;  // tail: last resort
+    if (free_[i].second >= need && (best < 0 || free_[i].second < free_[best].second)) best = i;
+  }
+  if (best < 0) {
+    if (free_.empty()) return false;
+    int t = (int)free_.size() - 1;
+    if (free_[t].first + free_[t].second != cap_ || free_[t].second < need) return false;
+    best = t;
+  }
+  *off = free_[best].first;
+  if (free_[best].second == need) free_.erase(free_.begin() + best);
+  else {
+    free_[best].first += need;
+    free_[best].second -= need;
+  }
+  extent_ = std::max(extent_, *off + need);
+  return true;
+}
+
+void Pool::release(uint64_t off, uint64_t bytes) {
+  uint64_t need = align_up(bytes);
+  size_t i = 0;
+  while (i < free_.size() && free_[i].first < off) ++i;
+  free_.insert(free_.begin() + i, {off, need});
+  if (i + 1 < free_.size() && free_[i].first + free_[i].second == free_[i + 1].first) {
+    free_[i].second += free_[i + 1].second;
+    free_.erase(free_.begin() + i + 1);
+  }
+  if (i > 0 && free_[i - 1].first + free_[i - 1].second == free_[i].first) {
+    free_[i - 1].second += free_[i].second;
+    free_.erase(free_.begin() + i);
+  }
+}
+
+uint64_t Pool::top() const {
+  if (!free_.empty() && free_.back().first + free_.back().second == cap_) return free_.back().first;
+  return cap_;
+}
+
+bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, uint64_t capacity,
+              SimResult& r, std::vector<std::vector<std::pair<PieceKey, uint64_t>>>* placements) {
+  r = SimResult();
+  Pool pool;
+  pool.reset(g.static_bytes, capacity);
+  std::unordered_map<PieceKey, uint64_t> where;
+  uint64_t live = 0, peak = 0, top = g.static_bytes;
+  int64_t seq = 0;
+  bool ok = true;
+  auto do_alloc = [&](int item, PieceKey pc) {
+    uint64_t b = piece_bytes(g, cfg, pk_key(pc)), off = 0;
+    if (!pool.alloc(b, &off)) {
+      ok = false;
+      return;
+    }
+    where[pc] = off;
+    r.offset[pc] = off;
+    live += align_up(b);
+    r.trace.push_back({seq++, item, 0, pk_key(pc), pk_j(pc), off, b});
+    if (placements && item >= 0) (*placements)[item].push_back({pc, off});
+  };
+  auto do_free = [&](int item, PieceKey pc) {
+    uint64_t b = piece_bytes(g, cfg, pk_key(pc));
+    auto it = where.find(pc);
+    uint64_t off = it->second;
+    where.erase(it);
+    pool.release(off, b);
+    live -= align_up(b);
+    r.trace.push_back({seq++, item, 1, pk_key(pc), pk_j(pc), off, b});
+  };
+  if (placements) placements->assign(ex.items.size(), {});
+  for (auto& t : g.t)
+    if (t.kind == TS_INPUT || t.kind == TS_LABEL) do_alloc(-1, pk(t.id, 0));
+  if (!ok) return false;
+  peak = live;
+  r.top.resize(ex.items.size());
+  r.live.resize(ex.items.size());
+  for (size_t i = 0; i < ex.items.size(); ++i) {
+    const Item& it = ex.items[i];
+    for (PieceKey pc : ex.alloc_at[i]) {
+      do_alloc((int)i, pc);
+      if (!ok) return false;
+    }
+    top = pool.top();
+    r.top[i] = top;
+    r.live[i] = live;
+    peak = std::max(peak, live);
+    if (it.kind == IT_SO) r.d2h += piece_bytes(g, cfg, pk_key(it.reads[0]));
+    else if (it.kind == IT_SI) r.h2d += piece_bytes(g, cfg, pk_key(it.writes[0]));
+    else if (it.kind == IT_R) ++r.n_replay;
+    else ++r.n_compute;
+    for (PieceKey pc : ex.free_after[i]) do_free((int)i, pc);
+  }
+  std::vector<PieceKey> rest;
+  for (auto& kv : where) rest.push_back(kv.first);
+  std::sort(rest.begin(), rest.end());
+  for (PieceKey pc : rest) do_free((int)ex.items.size(), pc);
+  r.peak_live = g.static_bytes + peak;
+  r.peak_extent = pool.extent();
+  return true;
+}
+
+}  // namespace ts

@@ -1,0 +1,280 @@
+"""Thin ctypes binding of libtsplit.so (include/ts.h).  Argument marshalling only:
+every step of the hot path runs inside the library.  Fails loudly when the
+library is missing — there is no CPU fallback."""
+
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libtsplit.so")
+
+OPS = {"linear": 0, "relu": 1, "gelu": 2, "tanh": 3, "layernorm": 4, "add": 5, "dropout": 6,
+       "softmax": 7, "attn_qk": 8, "attn_pv": 9, "embed": 10, "cls": 11, "xent": 12}
+DTYPES = {"f32": 0, "bf16": 1, "i32": 2}
+KINDS = {"param": 0, "input": 1, "label": 2, "act": 3}
+RESIDE, SWAP, RECOMPUTE = 0, 1, 2
+STATUS = ["OK", "ERR_ARG", "ERR_GRAPH", "ERR_INFEASIBLE", "ERR_BUDGET", "ERR_HOST_MEM",
+          "ERR_CUDA", "ERR_NCCL", "ERR_STATE", "ERR_NO_GPU"]
+
+
+class TensorDesc(C.Structure):
+    _fields_ = [("dtype", C.c_int32), ("kind", C.c_int32), ("ndim", C.c_int32), ("shape", C.c_int64 * 6)]
+
+
+class OpDesc(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("n_in", C.c_int32), ("n_out", C.c_int32),
+                ("inp", C.POINTER(C.c_int32)), ("out", C.POINTER(C.c_int32)),
+                ("n_iattr", C.c_int32), ("iattr", C.POINTER(C.c_int64)),
+                ("n_fattr", C.c_int32), ("fattr", C.POINTER(C.c_double))]
+
+
+class TensorCfg(C.Structure):
+    _fields_ = [("tensor_id", C.c_int32), ("opt", C.c_int32), ("p_num", C.c_int32), ("dim", C.c_int32),
+                ("prefetch_lead", C.c_int32)]
+
+
+class PlanStats(C.Structure):
+    _fields_ = [("static_bytes", C.c_uint64), ("peak_live", C.c_uint64), ("peak_extent", C.c_uint64),
+                ("d2h_bytes", C.c_uint64), ("h2d_bytes", C.c_uint64), ("n_items", C.c_int64),
+                ("n_compute", C.c_int64), ("n_replay", C.c_int64), ("predicted_s", C.c_double),
+                ("compute_flop", C.c_double), ("n_split_tensors", C.c_int64), ("n_swap_tensors", C.c_int64),
+                ("n_recompute_tensors", C.c_int64)]
+
+
+class AllocEvent(C.Structure):
+    _fields_ = [("seq", C.c_int64), ("item", C.c_int32), ("kind", C.c_int32), ("key", C.c_int32),
+                ("piece", C.c_int32), ("offset", C.c_uint64), ("bytes", C.c_uint64)]
+
+
+class Hw(C.Structure):
+    _fields_ = [("tensor_flops", C.c_double), ("simt_flops", C.c_double), ("hbm_bw", C.c_double),
+                ("d2h_bw", C.c_double), ("h2d_bw", C.c_double), ("launch_s", C.c_double)]
+
+
+class SessionCfg(C.Structure):
+    _fields_ = [("device", C.c_int32), ("slab", C.c_void_p), ("slab_bytes", C.c_uint64),
+                ("stream_compute", C.c_void_p), ("stream_d2h", C.c_void_p), ("stream_h2d", C.c_void_p),
+                ("nccl_comm", C.c_void_p), ("world_size", C.c_int32), ("use_cuda_graph", C.c_int32),
+                ("lr", C.c_float), ("step0", C.c_uint32)]
+
+
+class TsError(RuntimeError):
+    def __init__(self, status, msg):
+        self.status = STATUS[status] if 0 <= status < len(STATUS) else str(status)
+        super().__init__(f"{self.status}: {msg}")
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} missing: run `python -m paper_conf_icde_niemyc22_b200.build` "
+                              "(no CPU fallback exists)")
+        L = C.CDLL(LIB_PATH)
+        vp, u64, i32, i64 = C.c_void_p, C.c_uint64, C.c_int32, C.c_int64
+        P = C.POINTER
+        sig = {
+            "ts_last_error": (C.c_char_p, []),
+            "ts_version": (C.c_char_p, []),
+            "ts_graph_define": (i32, [P(TensorDesc), i32, P(OpDesc), i32, i32, i32, P(vp)]),
+            "ts_graph_destroy": (None, [vp]),
+            "ts_graph_schedule": (i32, [vp, P(i32), i32, P(i32)]),
+            "ts_graph_static_bytes": (i32, [vp, P(u64)]),
+            "ts_profile_analytic": (i32, [vp, P(Hw), P(vp)]),
+            "ts_profile_set": (i32, [vp, i32, i32, C.c_double, C.c_double]),
+            "ts_profile_set_pcie": (i32, [vp, C.c_double, C.c_double]),
+            "ts_profile_destroy": (None, [vp]),
+            "ts_plan_default": (i32, [vp, P(vp)]),
+            "ts_plan": (i32, [vp, u64, vp, P(vp)]),
+            "ts_plan_get": (i32, [vp, i32, P(TensorCfg)]),
+            "ts_plan_set": (i32, [vp, P(TensorCfg)]),
+            "ts_plan_stats": (i32, [vp, P(PlanStats)]),
+            "ts_plan_trace": (i32, [vp, P(AllocEvent), u64, P(u64)]),
+            "ts_plan_items": (i32, [vp, P(i32), u64, P(u64)]),
+            "ts_plan_serialize": (i32, [vp, vp, u64, P(u64)]),
+            "ts_plan_deserialize": (i32, [vp, vp, u64, P(vp)]),
+            "ts_plan_destroy": (None, [vp]),
+        }
+        optional = {
+            "ts_session_create": (i32, [vp, vp, P(SessionCfg), P(vp)]),
+            "ts_session_destroy": (None, [vp]),
+            "ts_set_param": (i32, [vp, i32, vp]),
+            "ts_get_param": (i32, [vp, i32, vp]),
+            "ts_get_grad": (i32, [vp, i32, vp]),
+            "ts_param_ptr": (i32, [vp, i32, P(vp)]),
+            "ts_grad_ptr": (i32, [vp, i32, P(vp)]),
+            "ts_step": (i32, [vp, P(vp), i32, P(C.c_float)]),
+            "ts_step_async": (i32, [vp, P(vp), i32]),
+            "ts_session_trace": (i32, [vp, P(AllocEvent), u64, P(u64)]),
+            "ts_session_launches": (i32, [vp, P(i64)]),
+            "ts_session_profile_items": (i32, [vp, i32]),
+            "ts_session_item_times": (i32, [vp, P(C.c_float), u64, P(u64)]),
+            "ts_gemm_bf16": (i32, [i32, i32, i32, i32, vp, i64, i64, i32, vp, i64, i64, i32,
+                                   vp, i64, i64, i32, C.c_float, C.c_float, vp, vp]),
+            "ts_gemm_f32": (i32, [i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, C.c_float,
+                                  vp, vp]),
+        }
+        for name, (res, args) in list(sig.items()) + list(optional.items()):
+            if not hasattr(L, name):
+                if name in sig:
+                    raise ImportError(f"libtsplit.so lacks {name}")
+                continue
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def check(status):
+    if status != 0:
+        raise TsError(status, lib().ts_last_error().decode())
+
+
+def exported_symbols():
+    """Names of the ts_* functions include/ts.h declares."""
+    import re
+    hdr = open(os.path.join(os.path.dirname(_PKG), "include", "ts.h")).read()
+    return sorted(set(re.findall(r"^\s*(?:ts_status|void|const char\*)\s+(ts_\w+)\s*\(", hdr, re.M)))
+
+
+# --------------------------------------------------------------------------- graph
+class Graph:
+    def __init__(self, spec: dict):
+        self.spec = spec
+        ts, ops = spec["tensors"], spec["ops"]
+        self.n = len(ts)
+        td = (TensorDesc * len(ts))()
+        for i, t in enumerate(ts):
+            td[i].dtype = DTYPES[t["dtype"]]
+            td[i].kind = KINDS[t["kind"]]
+            td[i].ndim = len(t["shape"])
+            for d, s in enumerate(t["shape"]):
+                td[i].shape[d] = s
+        od = (OpDesc * len(ops))()
+        self._keep = []
+        for i, o in enumerate(ops):
+            ins = (C.c_int32 * len(o["inputs"]))(*o["inputs"])
+            outs = (C.c_int32 * len(o["outputs"]))(*o["outputs"])
+            ia = (C.c_int64 * max(1, len(o["iattrs"])))(*o["iattrs"])
+            fa = (C.c_double * max(1, len(o["fattrs"])))(*o["fattrs"])
+            self._keep += [ins, outs, ia, fa]
+            od[i].kind = OPS[o["kind"]]
+            od[i].n_in, od[i].n_out = len(o["inputs"]), len(o["outputs"])
+            od[i].inp, od[i].out = ins, outs
+            od[i].n_iattr, od[i].iattr = len(o["iattrs"]), ia
+            od[i].n_fattr, od[i].fattr = len(o["fattrs"]), fa
+        h = C.c_void_p()
+        check(lib().ts_graph_define(td, len(ts), od, len(ops), spec["samples"], DTYPES[spec["dtype"]], C.byref(h)))
+        self.h = h
+        self.names = {t["name"]: t["id"] for t in ts}
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib().ts_graph_destroy(self.h)
+
+    def schedule(self):
+        n = C.c_int32()
+        buf = (C.c_int32 * len(self.spec["ops"]))()
+        check(lib().ts_graph_schedule(self.h, buf, len(buf), C.byref(n)))
+        return list(buf[:n.value])
+
+    def static_bytes(self):
+        v = C.c_uint64()
+        check(lib().ts_graph_static_bytes(self.h, C.byref(v)))
+        return v.value
+
+
+class Profile:
+    def __init__(self, graph: Graph, hw: dict | None = None):
+        self.graph = graph
+        h = C.c_void_p()
+        hwp = None
+        if hw:
+            hwp = C.byref(Hw(**hw))
+        check(lib().ts_profile_analytic(graph.h, hwp, C.byref(h)))
+        self.h = h
+
+    def set(self, op, p_num, fwd_s, bwd_s):
+        check(lib().ts_profile_set(self.h, op, p_num, fwd_s, bwd_s))
+
+    def set_pcie(self, d2h, h2d):
+        check(lib().ts_profile_set_pcie(self.h, d2h, h2d))
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib().ts_profile_destroy(self.h)
+
+
+class Plan:
+    def __init__(self, graph: Graph, h):
+        self.graph, self.h = graph, h
+
+    @classmethod
+    def default(cls, graph):
+        h = C.c_void_p()
+        check(lib().ts_plan_default(graph.h, C.byref(h)))
+        return cls(graph, h)
+
+    @classmethod
+    def plan(cls, graph, budget_bytes, profile: Profile | None = None):
+        h = C.c_void_p()
+        check(lib().ts_plan(graph.h, int(budget_bytes), profile.h if profile else None, C.byref(h)))
+        return cls(graph, h)
+
+    @classmethod
+    def deserialize(cls, graph, blob: bytes):
+        h = C.c_void_p()
+        buf = C.create_string_buffer(blob, len(blob))
+        check(lib().ts_plan_deserialize(graph.h, buf, len(blob), C.byref(h)))
+        return cls(graph, h)
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib().ts_plan_destroy(self.h)
+
+    def get(self, tid):
+        c = TensorCfg()
+        check(lib().ts_plan_get(self.h, tid, C.byref(c)))
+        return (c.opt, c.p_num, c.prefetch_lead)
+
+    def set(self, tid, opt=RESIDE, p_num=1, prefetch_lead=1, dim=0):
+        c = TensorCfg(tid, opt, p_num, dim, prefetch_lead)
+        check(lib().ts_plan_set(self.h, C.byref(c)))
+
+    def stats(self):
+        s = PlanStats()
+        check(lib().ts_plan_stats(self.h, C.byref(s)))
+        return {f: getattr(s, f) for f, _ in PlanStats._fields_}
+
+    def trace(self):
+        n = C.c_uint64()
+        check(lib().ts_plan_trace(self.h, None, 0, C.byref(n)))
+        buf = (AllocEvent * n.value)()
+        check(lib().ts_plan_trace(self.h, buf, n.value, C.byref(n)))
+        return [(e.seq, e.item, "A" if e.kind == 0 else "F", e.key, e.piece, e.offset, e.bytes) for e in buf]
+
+    def items(self):
+        n = C.c_uint64()
+        check(lib().ts_plan_items(self.h, None, 0, C.byref(n)))
+        buf = (C.c_int32 * (4 * n.value))()
+        check(lib().ts_plan_items(self.h, buf, len(buf), C.byref(n)))
+        kinds = ["F", "B", "R", "SO", "SI"]
+        return [(kinds[buf[4 * i]], buf[4 * i + 1], buf[4 * i + 2], buf[4 * i + 3]) for i in range(n.value)]
+
+    def serialize(self) -> bytes:
+        n = C.c_uint64()
+        check(lib().ts_plan_serialize(self.h, None, 0, C.byref(n)))
+        buf = C.create_string_buffer(n.value)
+        check(lib().ts_plan_serialize(self.h, buf, n.value, C.byref(n)))
+        return buf.raw
+
+    def cfg_dict(self):
+        return {t: self.get(t) for t in range(self.graph.n)}

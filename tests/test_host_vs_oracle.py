@@ -1,0 +1,139 @@
+"""Host C++ core (libtsplit.so, no GPU calls) against the oracle simulator:
+Alg. 1 order, static region, allocation trace bit for bit, peaks, and the
+planner's feasibility (T8)."""
+
+import random
+
+import pytest
+
+from oracle import brute, sim
+from paper_conf_icde_niemyc22_b200 import tsplit
+from tsinputs import graphs
+
+
+def _apply(plan, cfg, acts):
+    for t in acts:
+        o, p, lead = cfg[t]
+        plan.set(t, o, p, lead)
+
+
+def _compare(g, cfg):
+    G = tsplit.Graph(g)
+    plan = tsplit.Plan.default(G)
+    _apply(plan, cfg, brute.act_tensors(g))
+    ref = sim.simulate(g, cfg)
+    got = plan.trace()
+    assert len(got) == len(ref.trace)
+    for a, b in zip(got, ref.trace):
+        assert a == tuple(b), (a, b)
+    st = plan.stats()
+    assert st["peak_live"] == ref.peak_live
+    assert st["peak_extent"] == ref.peak_extent
+    assert st["n_replay"] == ref.n_replay
+    assert st["d2h_bytes"] == ref.d2h_bytes and st["h2d_bytes"] == ref.h2d_bytes
+    kinds = [it[0] for it in plan.items()]
+    assert kinds == [it.kind for it in ref.items]
+
+
+def test_library_exports_every_declared_symbol():
+    L = tsplit.lib()
+    names = tsplit.exported_symbols()
+    assert len(names) > 30
+    missing = [n for n in names if not hasattr(L, n)]
+    assert not missing, missing
+
+
+@pytest.mark.parametrize("gname", ["mlp", "bert_tiny", "bert_large"])
+def test_schedule_and_static_match_oracle(gname):
+    g = graphs.config_graph(gname)
+    G = tsplit.Graph(g)
+    assert G.schedule() == sim.schedule(g)
+    assert G.static_bytes() == sim.static_bytes(g)
+
+
+def test_trace_bit_exact_all_plans_tiny_mlp():
+    g = graphs.mlp(batch=4, hidden=8, depth=2, in_dim=8, classes=3)
+    for cfg in brute.enumerate_plans(g, ps=(1, 2, 4)):
+        _compare(g, cfg)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_trace_bit_exact_random_plans_bert_tiny(seed):
+    g = graphs.config_graph("bert_tiny")
+    r = random.Random(seed)
+    cfg = sim.default_cfg(g)
+    for t in brute.act_tensors(g):
+        cfg[t] = (r.choice([0, 1, 2]), r.choice([1, 2, 4]), r.choice([1, 2, 3]))
+    _compare(g, cfg)
+
+
+def test_default_trace_bert_large():
+    g = graphs.config_graph("bert_large")
+    _compare(g, sim.default_cfg(g))
+
+
+def test_config1_forced_plan():
+    """Config 1: 2-way batch split on every op plus one swapped activation."""
+    g = graphs.mlp()
+    cfg = sim.default_cfg(g)
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    for t in brute.act_tensors(g):
+        cfg[t] = (sim.RESIDE, 2, 1)
+    cfg[names["relu0"]] = (sim.SWAP, 2, 1)
+    _compare(g, cfg)
+    ref = sim.simulate(g, cfg)
+    assert ref.d2h_bytes == ref.h2d_bytes == 8 * 256 * 4
+
+
+def test_plan_serialize_roundtrip():
+    g = graphs.config_graph("bert_tiny")
+    G = tsplit.Graph(g)
+    P = tsplit.Plan.default(G)
+    t = G.names["l0.probs"]
+    P.set(t, tsplit.RECOMPUTE, 2, 1)
+    blob = P.serialize()
+    Q = tsplit.Plan.deserialize(G, blob)
+    assert Q.trace() == P.trace()
+    assert Q.get(t) == (tsplit.RECOMPUTE, 2, 1)
+
+
+def test_planner_feasible_plans_fit_and_simulate_exactly():
+    g = graphs.config_graph("bert_tiny")
+    G = tsplit.Graph(g)
+    base = tsplit.Plan.default(G).stats()
+    static = base["static_bytes"]
+    for frac in (1.0, 0.6, 0.35):
+        budget = static + int(frac * (base["peak_extent"] - static))
+        P = tsplit.Plan.plan(G, budget)
+        st = P.stats()
+        assert st["peak_extent"] <= budget
+        cfg = {t: P.get(t) for t in range(G.n)}
+        ref = sim.simulate(g, cfg)
+        assert ref.peak_extent == st["peak_extent"]
+        assert [tuple(e) for e in ref.trace] == P.trace()
+
+
+def test_planner_infeasible_only_when_brute_force_agrees():
+    g = graphs.mlp(batch=4, hidden=8, depth=2, in_dim=8, classes=3)
+    G = tsplit.Graph(g)
+    best, _ = brute.min_peak(g, ps=(1, 2, 4))
+    # below the brute-force optimum the planner must fail
+    with pytest.raises(tsplit.TsError) as e:
+        tsplit.Plan.plan(G, best - 256)
+    assert e.value.status == "ERR_INFEASIBLE"
+    # at the unsplit peak it must succeed
+    P = tsplit.Plan.plan(G, tsplit.Plan.default(G).stats()["peak_extent"])
+    assert P.stats()["peak_extent"] <= tsplit.Plan.default(G).stats()["peak_extent"]
+
+
+def test_planner_bert_large_quarter_budget():
+    """North-star config: BERT-Large b32 under 25% of the unsplit dynamic peak (R4)."""
+    g = graphs.config_graph("bert_large")
+    G = tsplit.Graph(g)
+    base = tsplit.Plan.default(G).stats()
+    static = base["static_bytes"]
+    budget = static + (base["peak_extent"] - static) // 4
+    P = tsplit.Plan.plan(G, budget)
+    st = P.stats()
+    assert st["peak_extent"] <= budget
+    assert st["n_recompute_tensors"] + st["n_swap_tensors"] > 0
