@@ -1,0 +1,200 @@
+// Vectorised elementwise micro-op kernels (HBM-bound: 16-byte loads/stores,
+// grid-stride loops sized to the SM count).  Every kernel takes micro-tensor
+// views, so a split micro-op is the same kernel on a shifted pointer; `acc`
+// selects accumulate-into-gradient (a later backward op adding its share).
+#include "common.cuh"
+#include "kernels.h"
+
+namespace tsk {
+
+namespace {
+
+enum EwOp : int { RELU_F, RELU_B, GELU_F, GELU_B, TANH_F, TANH_B, ADD_F, AXPY, DROP };
+
+struct EwP {
+  int64_t elem0;
+  float p, scale;
+  uint32_t seed, step, thr;
+};
+
+__device__ __forceinline__ float gelu_f(float x) { return 0.5f * x * (1.f + erff(x * 0.70710678118654752f)); }
+__device__ __forceinline__ float gelu_d(float x) {
+  float cdf = 0.5f * (1.f + erff(x * 0.70710678118654752f));
+  float pdf = 0.39894228040143268f * __expf(-0.5f * x * x);
+  return cdf + x * pdf;
+}
+
+template <int OP>
+__device__ __forceinline__ float ew_apply(float a, float b, int64_t idx, uint32_t word, const EwP& q) {
+  switch (OP) {
+    case RELU_F: return fmaxf(a, 0.f);
+    case RELU_B: return b > 0.f ? a : 0.f;   // a = dy, b = y
+    case GELU_F: return gelu_f(a);
+    case GELU_B: return a * gelu_d(b);       // a = dy, b = x
+    case TANH_F: return tanhf(a);
+    case TANH_B: return a * (1.f - b * b);   // a = dy, b = y
+    case ADD_F: return a + b;
+    case AXPY: return a;
+    case DROP: return word >= q.thr ? a * q.scale : 0.f;
+  }
+  return 0.f;
+}
+
+template <class T, int OP, int V>
+__global__ void __launch_bounds__(256) ew_kernel(const T* __restrict__ a, const T* __restrict__ b, T* y, int64_t n,
+                                                 int acc, EwP q) {
+  const int64_t nv = n / V;
+  const int64_t stride = int64_t(gridDim.x) * blockDim.x;
+  for (int64_t v = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; v < nv; v += stride) {
+    T av[V], bv[V], yv[V];
+    if constexpr (V * sizeof(T) == 16) {
+      *reinterpret_cast<uint4*>(av) = reinterpret_cast<const uint4*>(a)[v];
+      if (b) *reinterpret_cast<uint4*>(bv) = reinterpret_cast<const uint4*>(b)[v];
+      if (acc) *reinterpret_cast<uint4*>(yv) = reinterpret_cast<const uint4*>(y)[v];
+    } else {
+#pragma unroll
+      for (int i = 0; i < V; ++i) {
+        av[i] = a[v * V + i];
+        if (b) bv[i] = b[v * V + i];
+        if (acc) yv[i] = y[v * V + i];
+      }
+    }
+    uint32_t words[V];
+    if constexpr (OP == DROP) {
+      const int64_t i0 = q.elem0 + v * V;
+      if ((i0 & 3) == 0 && V % 4 == 0) {
+#pragma unroll
+        for (int j = 0; j < V; j += 4) {
+          uint64_t c = uint64_t(i0 + j) >> 2;
+          uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
+          words[j] = r.x;
+          words[j + 1] = r.y;
+          words[j + 2] = r.z;
+          words[j + 3] = r.w;
+        }
+      } else {
+#pragma unroll
+        for (int j = 0; j < V; ++j) {
+          uint64_t e = uint64_t(i0 + j), c = e >> 2;
+          uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
+          uint32_t w[4] = {r.x, r.y, r.z, r.w};
+          words[j] = w[e & 3];
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      float r = ew_apply<OP>(to_f(av[i]), b ? to_f(bv[i]) : 0.f, v * V + i, OP == DROP ? words[i] : 0u, q);
+      if (acc) r += to_f(yv[i]);
+      yv[i] = from_f<T>(r);
+    }
+    if constexpr (V * sizeof(T) == 16) {
+      reinterpret_cast<uint4*>(y)[v] = *reinterpret_cast<uint4*>(yv);
+    } else {
+#pragma unroll
+      for (int i = 0; i < V; ++i) y[v * V + i] = yv[i];
+    }
+  }
+  // scalar tail
+  for (int64_t i = nv * V + int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
+    uint32_t w = 0;
+    if constexpr (OP == DROP) {
+      uint64_t e = uint64_t(q.elem0 + i), c = e >> 2;
+      uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
+      uint32_t ww[4] = {r.x, r.y, r.z, r.w};
+      w = ww[e & 3];
+    }
+    float r = ew_apply<OP>(to_f(a[i]), b ? to_f(b[i]) : 0.f, i, w, q);
+    if (acc) r += to_f(y[i]);
+    y[i] = from_f<T>(r);
+  }
+}
+
+int g_grid_cap = 0;
+
+template <class T, int OP>
+void ew_launch(const void* a, const void* b, void* y, int64_t n, int acc, const EwP& q, cudaStream_t st) {
+  if (n <= 0) return;
+  if (!g_grid_cap) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    g_grid_cap = sms * 8;
+  }
+  constexpr int V = 16 / sizeof(T);
+  bool aligned = (reinterpret_cast<uintptr_t>(a) % 16 == 0) && (reinterpret_cast<uintptr_t>(y) % 16 == 0) &&
+                 (!b || reinterpret_cast<uintptr_t>(b) % 16 == 0);
+  int64_t work = aligned ? (n + V - 1) / V : n;
+  int grid = int(work / 256 + 1 < g_grid_cap ? work / 256 + 1 : g_grid_cap);
+  if (aligned)
+    ew_kernel<T, OP, V><<<grid, 256, 0, st>>>((const T*)a, (const T*)b, (T*)y, n, acc, q);
+  else
+    ew_kernel<T, OP, 1><<<grid, 256, 0, st>>>((const T*)a, (const T*)b, (T*)y, n, acc, q);
+}
+
+template <int OP>
+void ew(int dt, const void* a, const void* b, void* y, int64_t n, int acc, const EwP& q, cudaStream_t st) {
+  if (dt == F32) ew_launch<float, OP>(a, b, y, n, acc, q, st);
+  else ew_launch<bf16, OP>(a, b, y, n, acc, q, st);
+}
+
+__global__ void sgd_kernel(float* __restrict__ m, const float* __restrict__ g, int64_t n, float lr) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
+    m[i] -= lr * g[i];
+}
+__global__ void cast_kernel(const float* __restrict__ s, bf16* __restrict__ d, int64_t n) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
+    d[i] = __float2bfloat16_rn(s[i]);
+}
+__global__ void scale_kernel(float* x, int64_t n, float s) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
+    x[i] *= s;
+}
+int grid_for(int64_t n) {
+  int64_t g = (n + 255) / 256;
+  return int(g < 148 * 8 ? (g > 0 ? g : 1) : 148 * 8);
+}
+
+}  // namespace
+
+static const EwP kNoP{0, 0.f, 1.f, 0u, 0u, 0u};
+
+void relu_fwd(int dt, const void* x, void* y, int64_t n, cudaStream_t st) { ew<RELU_F>(dt, x, nullptr, y, n, 0, kNoP, st); }
+void relu_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t n, cudaStream_t st) {
+  ew<RELU_B>(dt, dy, y, dx, n, acc, kNoP, st);
+}
+void gelu_fwd(int dt, const void* x, void* y, int64_t n, cudaStream_t st) { ew<GELU_F>(dt, x, nullptr, y, n, 0, kNoP, st); }
+void gelu_bwd(int dt, const void* dy, const void* x, void* dx, int acc, int64_t n, cudaStream_t st) {
+  ew<GELU_B>(dt, dy, x, dx, n, acc, kNoP, st);
+}
+void tanh_fwd(int dt, const void* x, void* y, int64_t n, cudaStream_t st) { ew<TANH_F>(dt, x, nullptr, y, n, 0, kNoP, st); }
+void tanh_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t n, cudaStream_t st) {
+  ew<TANH_B>(dt, dy, y, dx, n, acc, kNoP, st);
+}
+void add_fwd(int dt, const void* a, const void* b, void* y, int64_t n, cudaStream_t st) {
+  ew<ADD_F>(dt, a, b, y, n, 0, kNoP, st);
+}
+void axpy(int dt, const void* dy, void* dx, int acc, int64_t n, cudaStream_t st) {
+  ew<AXPY>(dt, dy, nullptr, dx, n, acc, kNoP, st);
+}
+void dropout(int dt, const void* x, void* y, int acc, int64_t n, int64_t elem0, float p, uint32_t seed,
+             uint32_t step, cudaStream_t st) {
+  EwP q;
+  q.elem0 = elem0;
+  q.p = p;
+  q.scale = p > 0.f ? 1.f / (1.f - p) : 1.f;
+  q.seed = seed;
+  q.step = step;
+  double t = double(p) * 4294967296.0;
+  q.thr = t >= 4294967295.0 ? 0xFFFFFFFFu : uint32_t(t);
+  ew<DROP>(dt, x, nullptr, y, n, acc, q, st);
+}
+void sgd_update(float* master, const float* grad, int64_t n, float lr, float gscale, cudaStream_t st) {
+  sgd_kernel<<<grid_for(n), 256, 0, st>>>(master, grad, n, lr * gscale);
+}
+void cast_f32_bf16(const float* src, void* dst, int64_t n, cudaStream_t st) {
+  cast_kernel<<<grid_for(n), 256, 0, st>>>(src, reinterpret_cast<bf16*>(dst), n);
+}
+void scale_f32(float* x, int64_t n, float s, cudaStream_t st) { scale_kernel<<<grid_for(n), 256, 0, st>>>(x, n, s); }
+
+}  // namespace tsk

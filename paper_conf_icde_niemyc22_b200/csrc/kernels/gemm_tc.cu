@@ -1,0 +1,459 @@
+// bf16 GEMM on the 5th-generation tensor cores (sm_100a): TMA loads into
+// 128B-swizzled shared memory, tcgen05.mma issued by one thread with the fp32
+// accumulator in TMEM (double-buffered so the epilogue of tile t overlaps the
+// MMAs of tile t+1), warp-specialised persistent CTAs (one per SM).
+//
+// Used for every dense contraction of a micro-op: Linear
+// fwd (Y = X W^T), dX = dY W, dW = dY^T X (fp32 out, beta = 1 accumulates across
+// splits in ascending k, P:L260 merge-by-sum), and the per-(sample, head)
+// attention products.  Operands are strided micro-tensor views: a 4-D TMA map
+// (contiguous dim, row dim, batch1, batch2) describes each one, so no copy ever
+// materialises a split or a per-head transpose.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <atomic>
+#include <cstdio>
+#include <mutex>
+
+#include "common.cuh"
+#include "kernels.h"
+
+namespace tsk {
+
+namespace {
+
+constexpr int BM = 128, BK = 64;
+constexpr int kThreads = 192;  // warp0 TMA, warp1 MMA, warps2-5 epilogue
+
+struct TcParams {
+  int M, N, K, nb1, nb2;
+  int tiles_m, tiles_n, num_tiles, num_kb;
+  int a_mn, b_mn;
+  void* C;
+  int64_t ldc, cbs1, cbs2;
+  int c_f32;
+  float alpha, beta;
+  const void* bias;
+  int bias_f32;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t addr = smem_u32(bar), ok = 0;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(ok)
+        : "r"(addr), "r"(parity)
+        : "memory");
+  } while (!ok);
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void tma_load(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                                         int c2, int c3) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], "
+      "[%2];" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                       uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(acc));
+}
+
+// UMMA shared-memory descriptor, SWIZZLE_128B (layout type 2), sm100 version 1.
+__device__ __forceinline__ uint64_t smem_desc(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= uint64_t((addr >> 4) & 0x3FFF);
+  d |= uint64_t((lbo >> 4) & 0x3FFF) << 16;
+  d |= uint64_t((sbo >> 4) & 0x3FFF) << 32;
+  d |= uint64_t(1) << 46;
+  d |= uint64_t(2) << 61;
+  return d;
+}
+
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+        "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+        "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+__device__ __forceinline__ void decode_tile(const TcParams& p, int tile, int& b1, int& b2, int& m0, int& n0) {
+  int per = p.tiles_m * p.tiles_n;
+  int bb = tile / per;
+  int r = tile - bb * per;
+  // m fastest: neighbouring CTAs share the same B (weight) tile in L2
+  int nt = r / p.tiles_m;
+  int mt = r - nt * p.tiles_m;
+  b1 = bb % p.nb1;
+  b2 = bb / p.nb1;
+  m0 = mt * BM;
+  n0 = nt;  // scaled by BN by the caller
+}
+
+template <int BN>
+__global__ void __launch_bounds__(kThreads, 1)
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                   const TcParams p) {
+  constexpr int A_BYTES = BM * BK * 2;
+  constexpr int B_BYTES = BN * BK * 2;
+  constexpr int STAGE = A_BYTES + B_BYTES;
+  constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
+  constexpr uint32_t TMEM_COLS = 2 * BN;
+  // instruction descriptor: D f32, A/B bf16, M = 128, N = BN
+  const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(p.a_mn) << 15) |
+                         (uint32_t(p.b_mn) << 16) | (uint32_t(BN >> 3) << 17) | (uint32_t(BM >> 4) << 24);
+
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + STAGES * STAGE);
+  uint64_t* empty = full + STAGES;
+  uint64_t* tfull = empty + STAGES;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (warp == 0 && lane == 0) {
+    for (int s = 0; s < STAGES; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&tfull[s], 1);
+      mbar_init(&tempty[s], 128);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(TMEM_COLS));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      // ===== TMA producer =====
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+        int b1, b2, m0, nt;
+        decode_tile(p, tile, b1, b2, m0, nt);
+        int n0 = nt * BN;
+        for (int kb = 0; kb < p.num_kb; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          uint8_t* sa = smem + stage * STAGE;
+          uint8_t* sb = sa + A_BYTES;
+          mbar_arrive_tx(&full[stage], STAGE);
+          const int k0 = kb * BK;
+          if (!p.a_mn) {
+            tma_load(sa, &tmA, &full[stage], k0, m0, b1, b2);
+          } else {
+#pragma unroll
+            for (int i = 0; i < BM / 64; ++i) tma_load(sa + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, b1, b2);
+          }
+          if (!p.b_mn) {
+            tma_load(sb, &tmB, &full[stage], k0, n0, b1, b2);
+          } else {
+#pragma unroll
+            for (int i = 0; i < BN / 64; ++i) tma_load(sb + i * 8192, &tmB, &full[stage], n0 + 64 * i, k0, b1, b2);
+          }
+          if (++stage == STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      // ===== MMA issuer (single thread) =====
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      // K-major SW128: rows of 128 B, 8-row groups 1024 B apart (SBO), K step = +32 B.
+      // MN-major SW128: 64-element MN blocks 8 KB apart (LBO), 8-k groups 1024 B apart
+      // (SBO), K step of 16 = +2048 B.
+      const uint32_t a_lbo = p.a_mn ? 8192 : 16, b_lbo = p.b_mn ? 8192 : 16;
+      const uint32_t a_kstep = p.a_mn ? 2048 : 32, b_kstep = p.b_mn ? 2048 : 32;
+      for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
+        tc_fence_after();
+        const uint32_t tmem_d = tmem_base + uint32_t(acc * BN);
+        for (int kb = 0; kb < p.num_kb; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
+          uint32_t sa = smem_u32(smem + stage * STAGE);
+          uint32_t sb = sa + A_BYTES;
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            uint64_t ad = smem_desc(sa + k * a_kstep, a_lbo, 1024);
+            uint64_t bd = smem_desc(sb + k * b_kstep, b_lbo, 1024);
+            tc_mma(tmem_d, ad, bd, idesc, (kb | k) != 0);
+          }
+          tc_commit(&empty[stage]);
+          if (++stage == STAGES) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+        tc_commit(&tfull[acc]);
+        if (++acc == 2) {
+          acc = 0;
+          acc_phase ^= 1;
+        }
+      }
+    }
+  } else {
+    // ===== epilogue: TMEM -> registers -> global (alpha, bias, beta*C) =====
+    const int q = warp & 3;  // TMEM lane quarter this warp may access
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+      int b1, b2, m0, nt;
+      decode_tile(p, tile, b1, b2, m0, nt);
+      int n0 = nt * BN;
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const int row = m0 + q * 32 + lane;
+      const bool row_ok = row < p.M;
+      const int64_t cbase = int64_t(b1) * p.cbs1 + int64_t(b2) * p.cbs2 + int64_t(row) * p.ldc;
+#pragma unroll 1
+      for (int c = 0; c < BN / 32; ++c) {
+        uint32_t r[32];
+        tmem_ld32(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * BN + c * 32), r);
+        const int col0 = n0 + c * 32;
+        if (row_ok && col0 < p.N) {
+        float v[32];
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
+        const bool full_chunk = col0 + 32 <= p.N;
+        if (p.bias) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i)
+            if (full_chunk || col0 + i < p.N)
+              v[i] += p.bias_f32 ? reinterpret_cast<const float*>(p.bias)[col0 + i]
+                                 : to_f(reinterpret_cast<const bf16*>(p.bias)[col0 + i]);
+        }
+        if (p.c_f32) {
+          float* cp = reinterpret_cast<float*>(p.C) + cbase + col0;
+          bool vec = full_chunk && ((reinterpret_cast<uintptr_t>(cp) & 15) == 0);
+          if (vec) {
+#pragma unroll
+            for (int i = 0; i < 32; i += 4) {
+              float4 o = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+              if (p.beta != 0.f) {
+                float4 old = *reinterpret_cast<const float4*>(cp + i);
+                o.x += p.beta * old.x;
+                o.y += p.beta * old.y;
+                o.z += p.beta * old.z;
+                o.w += p.beta * old.w;
+              }
+              *reinterpret_cast<float4*>(cp + i) = o;
+            }
+          } else {
+#pragma unroll
+            for (int i = 0; i < 32; ++i)
+              if (col0 + i < p.N) cp[i] = v[i] + (p.beta != 0.f ? p.beta * cp[i] : 0.f);
+          }
+        } else {
+          bf16* cp = reinterpret_cast<bf16*>(p.C) + cbase + col0;
+          bool vec = full_chunk && ((reinterpret_cast<uintptr_t>(cp) & 15) == 0);
+          if (vec) {
+#pragma unroll
+            for (int i = 0; i < 32; i += 8) {
+              if (p.beta != 0.f) {
+                uint4 old = *reinterpret_cast<const uint4*>(cp + i);
+                const bf16* ob = reinterpret_cast<const bf16*>(&old);
+#pragma unroll
+                for (int j = 0; j < 8; ++j) v[i + j] += p.beta * to_f(ob[j]);
+              }
+              uint4 o;
+              __nv_bfloat162* ob2 = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+              for (int j = 0; j < 4; ++j) ob2[j] = __floats2bfloat162_rn(v[i + 2 * j], v[i + 2 * j + 1]);
+              *reinterpret_cast<uint4*>(cp + i) = o;
+            }
+          } else {
+#pragma unroll
+            for (int i = 0; i < 32; ++i)
+              if (col0 + i < p.N) cp[i] = from_f<bf16>(v[i] + (p.beta != 0.f ? p.beta * to_f(cp[i]) : 0.f));
+          }
+        }
+        }
+        __syncwarp();
+      }
+      tc_fence_before();
+      mbar_arrive(&tempty[acc]);
+      if (++acc == 2) {
+        acc = 0;
+        acc_phase ^= 1;
+      }
+    }
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(TMEM_COLS));
+  }
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    cudaDriverEntryPointQueryResult q;
+    void* f = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+  });
+  return fn;
+}
+
+// 4-D map: (contiguous dim, row dim, batch1, batch2); box (64, rows, 1, 1).
+bool make_map(CUtensorMap* map, const GemmOperand& op, int64_t d0, int64_t d1, int nb1, int nb2, int box1) {
+  auto fn = encode_fn();
+  if (!fn) return false;
+  const uint64_t es = 2;
+  uintptr_t base = reinterpret_cast<uintptr_t>(op.ptr);
+  if (base % 16 || (op.ld * es) % 16 || op.ld < d0) return false;
+  if (nb1 > 1 && (op.bs1 * es) % 16) return false;
+  if (nb2 > 1 && (op.bs2 * es) % 16) return false;
+  cuuint64_t dims[4] = {cuuint64_t(d0), cuuint64_t(d1), cuuint64_t(nb1), cuuint64_t(nb2)};
+  cuuint64_t s1 = op.ld * es;
+  cuuint64_t s2 = nb1 > 1 ? op.bs1 * es : s1 * d1;
+  cuuint64_t s3 = nb2 > 1 ? op.bs2 * es : s2 * nb1;
+  s2 = (s2 + 15) / 16 * 16;
+  s3 = (s3 + 15) / 16 * 16;
+  cuuint64_t strides[3] = {s1, s2, s3};
+  cuuint32_t box[4] = {64, cuuint32_t(box1), 1, 1};
+  cuuint32_t estr[4] = {1, 1, 1, 1};
+  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, reinterpret_cast<void*>(base), dims, strides, box,
+                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+int g_num_sms = 0;
+std::atomic<int64_t> g_launches{0};
+
+template <int BN>
+void launch(const CUtensorMap& a, const CUtensorMap& b, const TcParams& p, cudaStream_t st) {
+  constexpr int STAGE = (BM + BN) * BK * 2;
+  constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
+  const int smem = STAGES * STAGE + 1024 + 256;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(gemm_tc_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    attr = true;
+  }
+  int grid = p.num_tiles < g_num_sms ? p.num_tiles : g_num_sms;
+  gemm_tc_kernel<BN><<<grid, kThreads, smem, st>>>(a, b, p);
+  g_launches++;
+}
+
+}  // namespace
+
+int64_t gemm_tc_launches() { return g_launches.load(); }
+
+bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
+  if (g.in_dtype != BF16 || g.M <= 0 || g.N <= 0 || g.K <= 0) return false;
+  if (g.K < 16 || g.N < 16 || g.M < 64) return false;  // tiny products: SIMT path
+  if (g_num_sms == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
+    if (g_num_sms <= 0) return false;
+  }
+  // tile width: minimise waves x tile width (Fig. 5 effect of small micro-ops)
+  int best_bn = 256;
+  double best = 1e30;
+  for (int bn : {256, 128, 64}) {
+    int64_t tiles = int64_t((g.M + BM - 1) / BM) * ((g.N + bn - 1) / bn) * g.nb1 * g.nb2;
+    double waves = double((tiles + g_num_sms - 1) / g_num_sms);
+    double cost = waves * (bn + 32);
+    if (cost < best - 1e-9) {
+      best = cost;
+      best_bn = bn;
+    }
+  }
+  CUtensorMap ma, mb;
+  bool ok = g.a.mn_major ? make_map(&ma, g.a, g.M, g.K, g.nb1, g.nb2, 64)
+                         : make_map(&ma, g.a, g.K, g.M, g.nb1, g.nb2, BM);
+  ok = ok && (g.b.mn_major ? make_map(&mb, g.b, g.N, g.K, g.nb1, g.nb2, 64)
+                           : make_map(&mb, g.b, g.K, g.N, g.nb1, g.nb2, best_bn));
+  if (!ok) return false;
+  TcParams p;
+  p.M = g.M;
+  p.N = g.N;
+  p.K = g.K;
+  p.nb1 = g.nb1;
+  p.nb2 = g.nb2;
+  p.tiles_m = (g.M + BM - 1) / BM;
+  p.tiles_n = (g.N + best_bn - 1) / best_bn;
+  p.num_tiles = p.tiles_m * p.tiles_n * g.nb1 * g.nb2;
+  p.num_kb = (g.K + BK - 1) / BK;
+  p.a_mn = g.a.mn_major;
+  p.b_mn = g.b.mn_major;
+  p.C = g.c;
+  p.ldc = g.ldc;
+  p.cbs1 = g.cbs1;
+  p.cbs2 = g.cbs2;
+  p.c_f32 = g.c_dtype == F32;
+  p.alpha = g.alpha;
+  p.beta = g.beta;
+  p.bias = g.bias;
+  p.bias_f32 = g.bias_dtype == F32;
+  switch (best_bn) {
+    case 256: launch<256>(ma, mb, p, st); break;
+    case 128: launch<128>(ma, mb, p, st); break;
+    default: launch<64>(ma, mb, p, st); break;
+  }
+  return true;
+}
+
+void gemm(const GemmArgs& g, cudaStream_t st) {
+  if (!gemm_tc(g, st)) gemm_simt(g, st);
+}
+
+}  // namespace tsk

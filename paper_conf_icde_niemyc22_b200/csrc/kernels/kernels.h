@@ -1,0 +1,82 @@
+// Host-side launchers of the sm_100a kernel library (all asynchronous on `st`).
+// Every micro-op of the augmented schedule maps to one or more of these; the
+// pointers are micro-tensor views (a split shares storage, only the
+// pointer changes).
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+namespace tsk {
+
+enum DType : int { F32 = 0, BF16 = 1 };
+
+// Logical A[M,K], B[N,K]; element (m,k) of A at a + (mn ? k*lda + m : m*lda + k)
+// + b1*bs1 + b2*bs2 (elements).  C[m,n] = alpha*sum_k A B + bias[n] + beta*C.
+struct GemmOperand {
+  const void* ptr = nullptr;
+  int64_t ld = 0;
+  bool mn_major = false;
+  int64_t bs1 = 0, bs2 = 0;
+};
+struct GemmArgs {
+  int M = 0, N = 0, K = 0, nb1 = 1, nb2 = 1;
+  int in_dtype = BF16;
+  GemmOperand a, b;
+  void* c = nullptr;
+  int64_t ldc = 0, cbs1 = 0, cbs2 = 0;
+  int c_dtype = BF16;
+  float alpha = 1.f, beta = 0.f;
+  const void* bias = nullptr;
+  int bias_dtype = BF16;
+};
+
+// Returns false (and leaves nothing launched) when the shape/alignment does not
+// fit the tcgen05/TMA path; gemm() then uses the SIMT kernel.
+bool gemm_tc(const GemmArgs& g, cudaStream_t st);
+void gemm_simt(const GemmArgs& g, cudaStream_t st);
+void gemm(const GemmArgs& g, cudaStream_t st);
+int64_t gemm_tc_launches();
+
+// ---- elementwise (n elements, dtype F32/BF16 for activations) ----------------
+void relu_fwd(int dt, const void* x, void* y, int64_t n, cudaStream_t st);
+void relu_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t n, cudaStream_t st);
+void gelu_fwd(int dt, const void* x, void* y, int64_t n, cudaStream_t st);
+void gelu_bwd(int dt, const void* dy, const void* x, void* dx, int acc, int64_t n, cudaStream_t st);
+void tanh_fwd(int dt, const void* x, void* y, int64_t n, cudaStream_t st);
+void tanh_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t n, cudaStream_t st);
+void add_fwd(int dt, const void* a, const void* b, void* y, int64_t n, cudaStream_t st);
+// dx (+)= scale * dy (acc: accumulate into dx)
+void axpy(int dt, const void* dy, void* dx, int acc, int64_t n, cudaStream_t st);
+void dropout(int dt, const void* x, void* y, int acc, int64_t n, int64_t elem0, float p, uint32_t seed,
+             uint32_t step, cudaStream_t st);
+// ---- row ops -----------------------------------------------------------------
+void layernorm_fwd(int dt, const void* x, const void* g, const void* b, void* y, int64_t rows, int H,
+                   float eps, cudaStream_t st);
+// dx (+)= ...; partial dgamma/dbeta rows go to ws, then column_reduce adds them.
+void layernorm_bwd(int dt, const void* dy, const void* x, const void* g, void* dx, int acc, float* ws,
+                   float* dgamma, float* dbeta, int pacc, int64_t rows, int H, float eps, cudaStream_t st);
+void softmax_fwd(int dt, const void* x, void* y, int64_t rows, int L, cudaStream_t st);
+void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t rows, int L,
+                 cudaStream_t st);
+// out[n] (+)= sum_r x[r, n] (rows filtered by `filter[r] == fval` when filter != null)
+void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, float* out, int acc,
+                const int* filter, int fval, cudaStream_t st);
+void embed_fwd(int dt, const int* ids, const int* tt, const void* word, const void* pos, const void* type,
+               void* y, int64_t rows, int H, int seq, int64_t row0, cudaStream_t st);
+void embed_bwd_word(int dt, const void* dy, const int* ids, float* dword, int64_t rows, int H, cudaStream_t st);
+// dpos[s, :] (+)= sum over samples of dy rows at position s (rows = nsamp*seq)
+void embed_bwd_pos(int dt, const void* dy, float* dpos, int64_t nsamp, int seq, int H, int acc, cudaStream_t st);
+void cls_fwd(int dt, const void* x, void* y, int64_t nsamp, int seq, int H, cudaStream_t st);
+void cls_bwd(int dt, const void* dy, void* dx, int acc, int64_t nsamp, int seq, int H, cudaStream_t st);
+// loss[0] (+)= sum_rows CE / b_global ; dz = (softmax - onehot)/b_global
+void xent_fwd(int dt, const void* z, const int* labels, float* loss, int acc, int64_t rows, int C,
+              float inv_b, cudaStream_t st);
+void xent_bwd(int dt, const void* z, const int* labels, void* dz, int acc, int64_t rows, int C, float inv_b,
+              cudaStream_t st);
+// ---- optimiser / static region ------------------------------------------------
+void sgd_update(float* master, const float* grad, int64_t n, float lr, float gscale, cudaStream_t st);
+void cast_f32_bf16(const float* src, void* dst, int64_t n, cudaStream_t st);
+void scale_f32(float* x, int64_t n, float s, cudaStream_t st);
+
+}  // namespace tsk

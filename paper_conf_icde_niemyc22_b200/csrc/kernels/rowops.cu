@@ -1,0 +1,530 @@
+// Row-wise and reduction micro-op kernels: LayerNorm, softmax, softmax-CE,
+// column sums (bias / LN-parameter gradients), embedding gather/scatter, CLS
+// pick.  One warp per row with warp-shuffle reductions; rows up to 8 x 32 x 16 B
+// are held in registers (one HBM read per input), longer rows stream twice.
+// All kernels operate on the sample block of one micro-op; row statistics are
+// per row, so a sample split never needs a cross-split merge (P:L260 only needs
+// merges for batch-dimension statistics such as BN).
+#include "common.cuh"
+#include "kernels.h"
+
+namespace tsk {
+
+namespace {
+
+constexpr int kWarps = 8;  // warps per block for row kernels
+
+template <class T>
+struct Vec {
+  static constexpr int N = 16 / sizeof(T);
+};
+
+template <class T>
+__device__ __forceinline__ void load_vec(const T* p, float* v) {
+  uint4 u = *reinterpret_cast<const uint4*>(p);
+  const T* t = reinterpret_cast<const T*>(&u);
+#pragma unroll
+  for (int i = 0; i < Vec<T>::N; ++i) v[i] = to_f(t[i]);
+}
+template <class T>
+__device__ __forceinline__ void store_vec(T* p, const float* v) {
+  uint4 u;
+  T* t = reinterpret_cast<T*>(&u);
+#pragma unroll
+  for (int i = 0; i < Vec<T>::N; ++i) t[i] = from_f<T>(v[i]);
+  *reinterpret_cast<uint4*>(p) = u;
+}
+
+// ------------------------------------------------------------------ LayerNorm
+template <class T, int NCH>
+__global__ void __launch_bounds__(kWarps * 32) ln_fwd_kernel(const T* __restrict__ x, const T* __restrict__ g,
+                                                              const T* __restrict__ b, T* __restrict__ y,
+                                                              int64_t rows, int H, float eps) {
+  constexpr int V = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    const T* xr = x + r * H;
+    float v[NCH][V];
+    float s = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < H) {
+        load_vec(xr + col, v[c]);
+#pragma unroll
+        for (int i = 0; i < V; ++i) s += v[c][i];
+      }
+    }
+    const float mean = warp_sum(s) / H;
+    float q = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < H)
+#pragma unroll
+        for (int i = 0; i < V; ++i) {
+          float d = v[c][i] - mean;
+          q += d * d;
+        }
+    }
+    const float rstd = rsqrtf(warp_sum(q) / H + eps);
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < H) {
+        float gv[V], bv[V], o[V];
+        load_vec(g + col, gv);
+        load_vec(b + col, bv);
+#pragma unroll
+        for (int i = 0; i < V; ++i) o[i] = (v[c][i] - mean) * rstd * gv[i] + bv[i];
+        store_vec(y + r * H + col, o);
+      }
+    }
+  }
+}
+
+// generic (unaligned / long rows): three passes over global memory
+template <class T>
+__global__ void ln_fwd_generic(const T* x, const T* g, const T* b, T* y, int64_t rows, int H, float eps) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    const T* xr = x + r * H;
+    float s = 0.f;
+    for (int i = lane; i < H; i += 32) s += to_f(xr[i]);
+    const float mean = warp_sum(s) / H;
+    float q = 0.f;
+    for (int i = lane; i < H; i += 32) {
+      float d = to_f(xr[i]) - mean;
+      q += d * d;
+    }
+    const float rstd = rsqrtf(warp_sum(q) / H + eps);
+    for (int i = lane; i < H; i += 32) y[r * H + i] = from_f<T>((to_f(xr[i]) - mean) * rstd * to_f(g[i]) + to_f(b[i]));
+  }
+}
+
+// backward: dx (+)= rstd * (g dy - mean(g dy) - xhat mean(g dy xhat)); per-block
+// partial sums of dy*xhat and dy go to ws[block][2H] (smem atomics across warps).
+template <class T>
+__global__ void __launch_bounds__(kWarps * 32) ln_bwd_kernel(const T* __restrict__ dy, const T* __restrict__ x,
+                                                              const T* __restrict__ g, T* dx, int acc, float* ws,
+                                                              int64_t rows, int H, float eps) {
+  extern __shared__ float sacc[];  // [2H]
+  for (int i = threadIdx.x; i < 2 * H; i += blockDim.x) sacc[i] = 0.f;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    const T* xr = x + r * H;
+    const T* dr = dy + r * H;
+    float s = 0.f;
+    for (int i = lane; i < H; i += 32) s += to_f(xr[i]);
+    const float mean = warp_sum(s) / H;
+    float q = 0.f;
+    for (int i = lane; i < H; i += 32) {
+      float d = to_f(xr[i]) - mean;
+      q += d * d;
+    }
+    const float rstd = rsqrtf(warp_sum(q) / H + eps);
+    float s1 = 0.f, s2 = 0.f;
+    for (int i = lane; i < H; i += 32) {
+      float xh = (to_f(xr[i]) - mean) * rstd;
+      float gd = to_f(dr[i]) * to_f(g[i]);
+      s1 += gd;
+      s2 += gd * xh;
+    }
+    s1 = warp_sum(s1) / H;
+    s2 = warp_sum(s2) / H;
+    for (int i = lane; i < H; i += 32) {
+      float xh = (to_f(xr[i]) - mean) * rstd;
+      float d = to_f(dr[i]);
+      float v = rstd * (d * to_f(g[i]) - s1 - xh * s2);
+      T* o = dx + r * H + i;
+      *o = from_f<T>(acc ? v + to_f(*o) : v);
+      atomicAdd(&sacc[i], d * xh);
+      atomicAdd(&sacc[H + i], d);
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.x; i < 2 * H; i += blockDim.x) ws[int64_t(blockIdx.x) * 2 * H + i] = sacc[i];
+}
+
+// out[c] (+)= sum_{b < G} ws[b*stride + off + c]
+__global__ void reduce_partials(const float* ws, int G, int64_t stride, int64_t off, int N, float* out, int acc) {
+  int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= N) return;
+  float s = 0.f;
+  for (int b = 0; b < G; ++b) s += ws[int64_t(b) * stride + off + c];
+  out[c] = acc ? out[c] + s : s;
+}
+
+// column partial sums: block b sums rows [b*rpb, (b+1)*rpb) for all columns
+template <class T>
+__global__ void colsum_partial(const T* x, int64_t rows, int N, int64_t rpb, float* ws, const int* filter, int fval) {
+  int64_t r0 = int64_t(blockIdx.x) * rpb, r1 = r0 + rpb < rows ? r0 + rpb : rows;
+  for (int c = threadIdx.x; c < N; c += blockDim.x) {
+    float s = 0.f;
+    for (int64_t r = r0; r < r1; ++r)
+      if (!filter || filter[r] == fval) s += to_f(x[r * N + c]);
+    ws[int64_t(blockIdx.x) * N + c] = s;
+  }
+}
+
+// ------------------------------------------------------------------ softmax
+template <class T, int NCH>
+__global__ void __launch_bounds__(kWarps * 32) softmax_fwd_kernel(const T* __restrict__ x, T* __restrict__ y,
+                                                                   int64_t rows, int L) {
+  constexpr int V = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    float v[NCH][V];
+    float m = -INFINITY;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < L) {
+        load_vec(x + r * L + col, v[c]);
+#pragma unroll
+        for (int i = 0; i < V; ++i) m = fmaxf(m, v[c][i]);
+      }
+    }
+    m = warp_max(m);
+    float s = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < L)
+#pragma unroll
+        for (int i = 0; i < V; ++i) {
+          v[c][i] = __expf(v[c][i] - m);
+          s += v[c][i];
+        }
+    }
+    const float inv = 1.f / warp_sum(s);
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < L) {
+#pragma unroll
+        for (int i = 0; i < V; ++i) v[c][i] *= inv;
+        store_vec(y + r * L + col, v[c]);
+      }
+    }
+  }
+}
+
+template <class T, int NCH>
+__global__ void __launch_bounds__(kWarps * 32) softmax_bwd_kernel(const T* __restrict__ dy, const T* __restrict__ y,
+                                                                   T* dx, int acc, int64_t rows, int L) {
+  constexpr int V = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    float yv[NCH][V], dv[NCH][V];
+    float s = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < L) {
+        load_vec(y + r * L + col, yv[c]);
+        load_vec(dy + r * L + col, dv[c]);
+#pragma unroll
+        for (int i = 0; i < V; ++i) s += yv[c][i] * dv[c][i];
+      }
+    }
+    s = warp_sum(s);
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < L) {
+        float o[V];
+        if (acc) load_vec(dx + r * L + col, o);
+#pragma unroll
+        for (int i = 0; i < V; ++i) o[i] = yv[c][i] * (dv[c][i] - s) + (acc ? o[i] : 0.f);
+        store_vec(dx + r * L + col, o);
+      }
+    }
+  }
+}
+
+template <class T>
+__global__ void softmax_generic(const T* x, T* y, int64_t rows, int L) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    float m = -INFINITY;
+    for (int i = lane; i < L; i += 32) m = fmaxf(m, to_f(x[r * L + i]));
+    m = warp_max(m);
+    float s = 0.f;
+    for (int i = lane; i < L; i += 32) s += __expf(to_f(x[r * L + i]) - m);
+    const float inv = 1.f / warp_sum(s);
+    for (int i = lane; i < L; i += 32) y[r * L + i] = from_f<T>(__expf(to_f(x[r * L + i]) - m) * inv);
+  }
+}
+template <class T>
+__global__ void softmax_bwd_generic(const T* dy, const T* y, T* dx, int acc, int64_t rows, int L) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    float s = 0.f;
+    for (int i = lane; i < L; i += 32) s += to_f(y[r * L + i]) * to_f(dy[r * L + i]);
+    s = warp_sum(s);
+    for (int i = lane; i < L; i += 32) {
+      float v = to_f(y[r * L + i]) * (to_f(dy[r * L + i]) - s);
+      T* o = dx + r * L + i;
+      *o = from_f<T>(acc ? v + to_f(*o) : v);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ xent
+template <class T>
+__global__ void xent_fwd_kernel(const T* z, const int* labels, float* loss, int acc, int64_t rows, int C, float inv_b) {
+  __shared__ float part[32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  float tot = 0.f;
+  for (int64_t r = w; r < rows; r += blockDim.x / 32) {
+    float m = -INFINITY;
+    for (int i = lane; i < C; i += 32) m = fmaxf(m, to_f(z[r * C + i]));
+    m = warp_max(m);
+    float s = 0.f;
+    for (int i = lane; i < C; i += 32) s += expf(to_f(z[r * C + i]) - m);
+    s = warp_sum(s);
+    if (lane == 0) tot += (m + logf(s)) - to_f(z[r * C + labels[r]]);
+  }
+  if (lane == 0) part[w] = tot;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float t = 0.f;
+    for (int i = 0; i < int(blockDim.x / 32); ++i) t += part[i];
+    loss[0] = (acc ? loss[0] : 0.f) + t * inv_b;
+  }
+}
+template <class T>
+__global__ void xent_bwd_kernel(const T* z, const int* labels, T* dz, int acc, int64_t rows, int C, float inv_b) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    float m = -INFINITY;
+    for (int i = lane; i < C; i += 32) m = fmaxf(m, to_f(z[r * C + i]));
+    m = warp_max(m);
+    float s = 0.f;
+    for (int i = lane; i < C; i += 32) s += expf(to_f(z[r * C + i]) - m);
+    s = warp_sum(s);
+    for (int i = lane; i < C; i += 32) {
+      float v = (expf(to_f(z[r * C + i]) - m) / s - (i == labels[r] ? 1.f : 0.f)) * inv_b;
+      T* o = dz + r * C + i;
+      *o = from_f<T>(acc ? v + to_f(*o) : v);
+    }
+  }
+}
+
+// ------------------------------------------------------------------ embedding / cls
+template <class T>
+__global__ void embed_fwd_kernel(const int* ids, const int* tt, const T* word, const T* pos, const T* type, T* y,
+                                 int64_t rows, int H, int seq, int64_t row0) {
+  const int64_t n = rows * H;
+  for (int64_t e = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; e < n; e += int64_t(gridDim.x) * blockDim.x) {
+    int64_t r = e / H;
+    int c = int(e - r * H);
+    int p = int((row0 + r) % seq);
+    float v = to_f(word[int64_t(ids[r]) * H + c]) + to_f(pos[int64_t(p) * H + c]) + to_f(type[int64_t(tt[r]) * H + c]);
+    y[e] = from_f<T>(v);
+  }
+}
+template <class T>
+__global__ void embed_bwd_word_kernel(const T* dy, const int* ids, float* dword, int64_t rows, int H) {
+  const int64_t n = rows * H;
+  for (int64_t e = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; e < n; e += int64_t(gridDim.x) * blockDim.x) {
+    int64_t r = e / H;
+    int c = int(e - r * H);
+    atomicAdd(&dword[int64_t(ids[r]) * H + c], to_f(dy[e]));
+  }
+}
+template <class T>
+__global__ void embed_bwd_pos_kernel(const T* dy, float* dpos, int64_t nsamp, int seq, int H, int acc) {
+  const int64_t n = int64_t(seq) * H;
+  for (int64_t e = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; e < n; e += int64_t(gridDim.x) * blockDim.x) {
+    float s = 0.f;
+    for (int64_t b = 0; b < nsamp; ++b) s += to_f(dy[b * n + e]);
+    dpos[e] = acc ? dpos[e] + s : s;
+  }
+}
+template <class T>
+__global__ void cls_fwd_kernel(const T* x, T* y, int64_t nsamp, int seq, int H) {
+  const int64_t n = nsamp * H;
+  for (int64_t e = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; e < n; e += int64_t(gridDim.x) * blockDim.x) {
+    int64_t b = e / H;
+    y[e] = x[b * seq * H + (e - b * H)];
+  }
+}
+template <class T>
+__global__ void cls_bwd_kernel(const T* dy, T* dx, int acc, int64_t nsamp, int seq, int H) {
+  const int64_t n = nsamp * seq * H;
+  for (int64_t e = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; e < n; e += int64_t(gridDim.x) * blockDim.x) {
+    int64_t row = e / H;
+    int c = int(e - row * H);
+    bool is_cls = row % seq == 0;
+    float v = is_cls ? to_f(dy[(row / seq) * H + c]) : 0.f;
+    if (acc) {
+      if (is_cls) dx[e] = from_f<T>(to_f(dx[e]) + v);
+    } else {
+      dx[e] = from_f<T>(v);
+    }
+  }
+}
+
+int grid_rows(int64_t rows) {
+  int64_t g = (rows + kWarps - 1) / kWarps;
+  return int(g < 148 * 16 ? (g > 0 ? g : 1) : 148 * 16);
+}
+int grid_elems(int64_t n) {
+  int64_t g = (n + 255) / 256;
+  return int(g < 148 * 8 ? (g > 0 ? g : 1) : 148 * 8);
+}
+bool al16(const void* p) { return reinterpret_cast<uintptr_t>(p) % 16 == 0; }
+
+template <class T>
+void ln_fwd_t(const void* x, const void* g, const void* b, void* y, int64_t rows, int H, float eps, cudaStream_t st) {
+  constexpr int V = Vec<T>::N;
+  int nch = (H + 32 * V - 1) / (32 * V);
+  bool vec = H % V == 0 && al16(x) && al16(g) && al16(b) && al16(y);
+  auto X = (const T*)x;
+  auto G = (const T*)g;
+  auto B = (const T*)b;
+  auto Y = (T*)y;
+  int grid = grid_rows(rows);
+  if (vec && nch <= 8) {
+    switch (nch) {
+      case 1: ln_fwd_kernel<T, 1><<<grid, kWarps * 32, 0, st>>>(X, G, B, Y, rows, H, eps); return;
+      case 2: ln_fwd_kernel<T, 2><<<grid, kWarps * 32, 0, st>>>(X, G, B, Y, rows, H, eps); return;
+      case 3: case 4: ln_fwd_kernel<T, 4><<<grid, kWarps * 32, 0, st>>>(X, G, B, Y, rows, H, eps); return;
+      default: ln_fwd_kernel<T, 8><<<grid, kWarps * 32, 0, st>>>(X, G, B, Y, rows, H, eps); return;
+    }
+  }
+  ln_fwd_generic<T><<<grid, kWarps * 32, 0, st>>>(X, G, B, Y, rows, H, eps);
+}
+
+template <class T>
+void softmax_fwd_t(const void* x, void* y, int64_t rows, int L, cudaStream_t st) {
+  constexpr int V = Vec<T>::N;
+  int nch = (L + 32 * V - 1) / (32 * V);
+  bool vec = L % V == 0 && al16(x) && al16(y);
+  int grid = grid_rows(rows);
+  if (vec && nch <= 8) {
+    switch (nch) {
+      case 1: softmax_fwd_kernel<T, 1><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L); return;
+      case 2: softmax_fwd_kernel<T, 2><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L); return;
+      case 3: case 4: softmax_fwd_kernel<T, 4><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L); return;
+      default: softmax_fwd_kernel<T, 8><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L); return;
+    }
+  }
+  softmax_generic<T><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L);
+}
+
+template <class T>
+void softmax_bwd_t(const void* dy, const void* y, void* dx, int acc, int64_t rows, int L, cudaStream_t st) {
+  constexpr int V = Vec<T>::N;
+  int nch = (L + 32 * V - 1) / (32 * V);
+  bool vec = L % V == 0 && al16(dy) && al16(y) && al16(dx);
+  int grid = grid_rows(rows);
+  auto DY = (const T*)dy;
+  auto Y = (const T*)y;
+  auto DX = (T*)dx;
+  if (vec && nch <= 8) {
+    switch (nch) {
+      case 1: softmax_bwd_kernel<T, 1><<<grid, kWarps * 32, 0, st>>>(DY, Y, DX, acc, rows, L); return;
+      case 2: softmax_bwd_kernel<T, 2><<<grid, kWarps * 32, 0, st>>>(DY, Y, DX, acc, rows, L); return;
+      case 3: case 4: softmax_bwd_kernel<T, 4><<<grid, kWarps * 32, 0, st>>>(DY, Y, DX, acc, rows, L); return;
+      default: softmax_bwd_kernel<T, 8><<<grid, kWarps * 32, 0, st>>>(DY, Y, DX, acc, rows, L); return;
+    }
+  }
+  softmax_bwd_generic<T><<<grid, kWarps * 32, 0, st>>>(DY, Y, DX, acc, rows, L);
+}
+
+constexpr int kWsRows = 256;
+
+}  // namespace
+
+void layernorm_fwd(int dt, const void* x, const void* g, const void* b, void* y, int64_t rows, int H, float eps,
+                   cudaStream_t st) {
+  if (dt == F32) ln_fwd_t<float>(x, g, b, y, rows, H, eps, st);
+  else ln_fwd_t<bf16>(x, g, b, y, rows, H, eps, st);
+}
+
+void layernorm_bwd(int dt, const void* dy, const void* x, const void* g, void* dx, int acc, float* ws, float* dgamma,
+                   float* dbeta, int pacc, int64_t rows, int H, float eps, cudaStream_t st) {
+  int64_t G = (rows + kWarps - 1) / kWarps;
+  if (G > kWsRows) G = kWsRows;
+  size_t smem = size_t(2) * H * sizeof(float);
+  if (dt == F32) {
+    if (smem > 48 * 1024) cudaFuncSetAttribute(ln_bwd_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    ln_bwd_kernel<float><<<int(G), kWarps * 32, smem, st>>>((const float*)dy, (const float*)x, (const float*)g,
+                                                             (float*)dx, acc, ws, rows, H, eps);
+  } else {
+    if (smem > 48 * 1024) cudaFuncSetAttribute(ln_bwd_kernel<bf16>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+    ln_bwd_kernel<bf16><<<int(G), kWarps * 32, smem, st>>>((const bf16*)dy, (const bf16*)x, (const bf16*)g,
+                                                           (bf16*)dx, acc, ws, rows, H, eps);
+  }
+  reduce_partials<<<(H + 255) / 256, 256, 0, st>>>(ws, int(G), 2 * H, 0, H, dgamma, pacc);
+  reduce_partials<<<(H + 255) / 256, 256, 0, st>>>(ws, int(G), 2 * H, H, H, dbeta, pacc);
+}
+
+void softmax_fwd(int dt, const void* x, void* y, int64_t rows, int L, cudaStream_t st) {
+  if (dt == F32) softmax_fwd_t<float>(x, y, rows, L, st);
+  else softmax_fwd_t<bf16>(x, y, rows, L, st);
+}
+void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t rows, int L, cudaStream_t st) {
+  if (dt == F32) softmax_bwd_t<float>(dy, y, dx, acc, rows, L, st);
+  else softmax_bwd_t<bf16>(dy, y, dx, acc, rows, L, st);
+}
+
+void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, float* out, int acc, const int* filter, int fval,
+                cudaStream_t st) {
+  int64_t G = rows < kWsRows ? rows : kWsRows;
+  if (G < 1) G = 1;
+  int64_t rpb = (rows + G - 1) / G;
+  G = (rows + rpb - 1) / rpb;
+  int threads = N < 256 ? ((N + 31) / 32) * 32 : 256;
+  if (dt == F32) colsum_partial<float><<<int(G), threads, 0, st>>>((const float*)x, rows, N, rpb, ws, filter, fval);
+  else colsum_partial<bf16><<<int(G), threads, 0, st>>>((const bf16*)x, rows, N, rpb, ws, filter, fval);
+  reduce_partials<<<(N + 255) / 256, 256, 0, st>>>(ws, int(G), N, 0, N, out, acc);
+}
+
+void embed_fwd(int dt, const int* ids, const int* tt, const void* word, const void* pos, const void* type, void* y,
+               int64_t rows, int H, int seq, int64_t row0, cudaStream_t st) {
+  int grid = grid_elems(rows * H);
+  if (dt == F32)
+    embed_fwd_kernel<float><<<grid, 256, 0, st>>>(ids, tt, (const float*)word, (const float*)pos, (const float*)type,
+                                                  (float*)y, rows, H, seq, row0);
+  else
+    embed_fwd_kernel<bf16><<<grid, 256, 0, st>>>(ids, tt, (const bf16*)word, (const bf16*)pos, (const bf16*)type,
+                                                 (bf16*)y, rows, H, seq, row0);
+}
+void embed_bwd_word(int dt, const void* dy, const int* ids, float* dword, int64_t rows, int H, cudaStream_t st) {
+  int grid = grid_elems(rows * H);
+  if (dt == F32) embed_bwd_word_kernel<float><<<grid, 256, 0, st>>>((const float*)dy, ids, dword, rows, H);
+  else embed_bwd_word_kernel<bf16><<<grid, 256, 0, st>>>((const bf16*)dy, ids, dword, rows, H);
+}
+void embed_bwd_pos(int dt, const void* dy, float* dpos, int64_t nsamp, int seq, int H, int acc, cudaStream_t st) {
+  int grid = grid_elems(int64_t(seq) * H);
+  if (dt == F32) embed_bwd_pos_kernel<float><<<grid, 256, 0, st>>>((const float*)dy, dpos, nsamp, seq, H, acc);
+  else embed_bwd_pos_kernel<bf16><<<grid, 256, 0, st>>>((const bf16*)dy, dpos, nsamp, seq, H, acc);
+}
+void cls_fwd(int dt, const void* x, void* y, int64_t nsamp, int seq, int H, cudaStream_t st) {
+  int grid = grid_elems(nsamp * H);
+  if (dt == F32) cls_fwd_kernel<float><<<grid, 256, 0, st>>>((const float*)x, (float*)y, nsamp, seq, H);
+  else cls_fwd_kernel<bf16><<<grid, 256, 0, st>>>((const bf16*)x, (bf16*)y, nsamp, seq, H);
+}
+void cls_bwd(int dt, const void* dy, void* dx, int acc, int64_t nsamp, int seq, int H, cudaStream_t st) {
+  int grid = grid_elems(nsamp * seq * H);
+  if (dt == F32) cls_bwd_kernel<float><<<grid, 256, 0, st>>>((const float*)dy, (float*)dx, acc, nsamp, seq, H);
+  else cls_bwd_kernel<bf16><<<grid, 256, 0, st>>>((const bf16*)dy, (bf16*)dx, acc, nsamp, seq, H);
+}
+void xent_fwd(int dt, const void* z, const int* labels, float* loss, int acc, int64_t rows, int C, float inv_b,
+              cudaStream_t st) {
+  if (dt == F32) xent_fwd_kernel<float><<<1, 256, 0, st>>>((const float*)z, labels, loss, acc, rows, C, inv_b);
+  else xent_fwd_kernel<bf16><<<1, 256, 0, st>>>((const bf16*)z, labels, loss, acc, rows, C, inv_b);
+}
+void xent_bwd(int dt, const void* z, const int* labels, void* dz, int acc, int64_t rows, int C, float inv_b,
+              cudaStream_t st) {
+  int grid = grid_rows(rows);
+  if (dt == F32) xent_bwd_kernel<float><<<grid, kWarps * 32, 0, st>>>((const float*)z, labels, (float*)dz, acc, rows, C, inv_b);
+  else xent_bwd_kernel<bf16><<<grid, kWarps * 32, 0, st>>>((const bf16*)z, labels, (bf16*)dz, acc, rows, C, inv_b);
+}
+
+}  // namespace tsk

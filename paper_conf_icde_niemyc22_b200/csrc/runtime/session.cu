@@ -1,0 +1,819 @@
+// Graph executor (§V-D): one compute stream, one D2H and one
+// H2D stream ordered by CUDA events, over a pre-allocated pool whose offsets
+// come from the plan's best-fit simulation.  The augmented
+// schedule is lowered once, at session creation, into a program of
+// kernel launches on micro-tensor views, swap copies and event edges; a step
+// replays it — captured once into a CUDA graph, so per-micro-op launch cost
+// vanishes.  Swap-outs are logical frees; every reuse of a range still being
+// copied out waits on that copy's event.  Recompute replays re-run
+// the producer's forward micro-op (memory-centric).
+#include <dlfcn.h>
+
+#include <algorithm>
+#include <cstring>
+#include <functional>
+#include <map>
+#include <memory>
+#include <set>
+#include <string>
+#include <vector>
+
+#include "../host/capi_internal.h"
+#include "../kernels/kernels.h"
+
+using namespace ts;
+
+namespace {
+
+#define CU(x)                                                                        \
+  do {                                                                               \
+    cudaError_t e_ = (x);                                                            \
+    if (e_ != cudaSuccess) {                                                         \
+      set_error(std::string(#x) + ": " + cudaGetErrorString(e_));                    \
+      return TS_ERR_CUDA;                                                            \
+    }                                                                                \
+  } while (0)
+
+// Minimal NCCL ABI (resolved with dlsym from the libnccl the process already has).
+typedef int (*nccl_allreduce_fn)(const void*, void*, size_t, int, int, void*, cudaStream_t);
+constexpr int kNcclFloat32 = 7, kNcclSum = 0;
+
+}  // namespace
+
+struct Cmd {
+  int kind;  // 0 compute, 1 swap-out, 2 swap-in
+  int item;
+  std::function<void(cudaStream_t)> fn;
+  std::vector<int> wait_so;  // SO items whose d2h_done must precede this command
+  std::vector<int> wait_si;  // SI items whose h2d_done must precede this (compute only)
+  char* dev = nullptr;
+  uint64_t host_off = 0, bytes = 0;
+  int so_of_piece = -1;      // for SI: the SO item that wrote the host copy
+};
+
+struct ts_session_s {
+  const Graph* g = nullptr;
+  std::vector<Cfg> cfg;
+  Expansion ex;
+  SimResult sim;
+  int device = 0;
+  char* slab = nullptr;
+  uint64_t slab_bytes = 0;
+  cudaStream_t cs = nullptr, d2h = nullptr, h2d = nullptr;
+  bool own_streams = false;
+  void* nccl = nullptr;
+  nccl_allreduce_fn allreduce = nullptr;
+  int world = 1;
+  float lr = 0.f;
+  uint32_t step = 0;
+  bool use_graph = true;
+  cudaGraphExec_t gexec = nullptr;
+  int64_t graph_kernels = 0;
+  char* host = nullptr;
+  uint64_t host_bytes = 0;
+  std::vector<Cmd> prog;
+  std::vector<cudaEvent_t> ev_d2h, ev_h2d;  // indexed by item
+  cudaEvent_t ev_mark = nullptr, ev_join_d2h = nullptr, ev_join_h2d = nullptr;
+  std::vector<std::pair<int, uint64_t>> inputs;  // (tensor id, pool offset)
+  uint64_t loss_off = 0;
+  std::vector<int> zero_grads;                   // params whose grad is accumulated atomically
+  int64_t launches = 0;
+};
+
+namespace {
+
+char* param_w(ts_session_t* s, int t) {
+  const Graph& g = *s->g;
+  return s->slab + (g.dtype == TS_BF16 ? g.copy_off[t] : g.master_off[t]);
+}
+float* param_g(ts_session_t* s, int t) { return reinterpret_cast<float*>(s->slab + s->g->grad_off[t]); }
+
+struct Micro {
+  int op, k, P;
+  int64_t s0, s1;
+  std::unordered_map<int, char*> val, grad;
+  std::unordered_map<int, int> acc;  // grad key -> accumulate flag
+};
+
+// Lower one micro-op to kernel launches (DESIGN.md §3 op table).
+std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bwd, int& nk) {
+  const Graph& g = *s->g;
+  const Op& o = g.ops[m.op];
+  const int dt = g.dtype == TS_BF16 ? tsk::BF16 : tsk::F32;
+  const int64_t ns = m.s1 - m.s0;
+  const int B = g.samples;
+  float* ws = reinterpret_cast<float*>(s->slab + g.ws_off);
+  auto V = [&](int t) { return m.val.at(t); };
+  auto G = [&](int t) { return m.grad.at(t); };
+  auto A = [&](int key) {
+    auto it = m.acc.find(key);
+    return it == m.acc.end() ? 0 : it->second;
+  };
+  const Tensor& out = g.t[o.out[0]];
+  const int64_t n_out = out.sample ? ns * out.elems_per_sample : out.numel;
+  const int64_t elem0 = out.sample ? m.s0 * out.elems_per_sample : 0;
+  uint32_t* stepp = &s->step;
+  switch (o.kind) {
+    case TS_OP_LINEAR: {
+      const Tensor& x = g.t[o.in[0]];
+      const int64_t R = ns * x.rows_per_sample, K = x.shape[1], N = g.t[o.in[1]].shape[0];
+      const int w = o.in[1], bb = o.in[2];
+      if (!bwd) {
+        tsk::GemmArgs a;
+        a.M = int(R); a.N = int(N); a.K = int(K); a.in_dtype = dt;
+        a.a = {V(o.in[0]), K, false, 0, 0};
+        a.b = {param_w(s, w), K, false, 0, 0};
+        a.c = V(o.out[0]); a.ldc = N; a.c_dtype = dt;
+        a.bias = param_w(s, bb); a.bias_dtype = dt;
+        nk = 1;
+        return [a](cudaStream_t st) { tsk::gemm(a, st); };
+      }
+      std::vector<tsk::GemmArgs> gs;
+      char* dY = G(o.out[0]);
+      if (x.kind == TS_ACT && x.needs_grad) {
+        tsk::GemmArgs a;
+        a.M = int(R); a.N = int(K); a.K = int(N); a.in_dtype = dt;
+        a.a = {dY, N, false, 0, 0};
+        a.b = {param_w(s, w), K, true, 0, 0};
+        a.c = G(o.in[0]); a.ldc = K; a.c_dtype = dt; a.beta = A(g.n() + o.in[0]) ? 1.f : 0.f;
+        gs.push_back(a);
+      }
+      tsk::GemmArgs d;
+      d.M = int(N); d.N = int(K); d.K = int(R); d.in_dtype = dt;
+      d.a = {dY, N, true, 0, 0};
+      d.b = {V(o.in[0]), K, true, 0, 0};
+      d.c = param_g(s, w); d.ldc = K; d.c_dtype = tsk::F32; d.beta = A(w) ? 1.f : 0.f;
+      gs.push_back(d);
+      float* db = param_g(s, bb);
+      int dacc = A(bb);
+      nk = int(gs.size()) + 2;
+      return [gs, dY, R, N, db, dacc, ws, dt](cudaStream_t st) {
+        for (auto& a : gs) tsk::gemm(a, st);
+        tsk::column_sum(dt, dY, R, int(N), ws, db, dacc, nullptr, 0, st);
+      };
+    }
+    case TS_OP_RELU: case TS_OP_GELU: case TS_OP_TANH: {
+      int kind = o.kind;
+      if (!bwd) {
+        char *x = V(o.in[0]), *y = V(o.out[0]);
+        nk = 1;
+        return [=](cudaStream_t st) {
+          if (kind == TS_OP_RELU) tsk::relu_fwd(dt, x, y, n_out, st);
+          else if (kind == TS_OP_GELU) tsk::gelu_fwd(dt, x, y, n_out, st);
+          else tsk::tanh_fwd(dt, x, y, n_out, st);
+        };
+      }
+      char* dy = G(o.out[0]);
+      char* dx = G(o.in[0]);
+      char* sv = kind == TS_OP_GELU ? V(o.in[0]) : V(o.out[0]);
+      int acc = A(g.n() + o.in[0]);
+      nk = 1;
+      return [=](cudaStream_t st) {
+        if (kind == TS_OP_RELU) tsk::relu_bwd(dt, dy, sv, dx, acc, n_out, st);
+        else if (kind == TS_OP_GELU) tsk::gelu_bwd(dt, dy, sv, dx, acc, n_out, st);
+        else tsk::tanh_bwd(dt, dy, sv, dx, acc, n_out, st);
+      };
+    }
+    case TS_OP_LAYERNORM: {
+      const Tensor& x = g.t[o.in[0]];
+      const int64_t rows = ns * x.rows_per_sample;
+      const int H = int(x.shape[1]);
+      const float eps = float(o.fa[0]);
+      char* gw = param_w(s, o.in[1]);
+      if (!bwd) {
+        char *xp = V(o.in[0]), *y = V(o.out[0]), *bw = param_w(s, o.in[2]);
+        nk = 1;
+        return [=](cudaStream_t st) { tsk::layernorm_fwd(dt, xp, gw, bw, y, rows, H, eps, st); };
+      }
+      char *dy = G(o.out[0]), *xp = V(o.in[0]), *dx = G(o.in[0]);
+      int acc = A(g.n() + o.in[0]);
+      float *dg = param_g(s, o.in[1]), *dbt = param_g(s, o.in[2]);
+      int pacc = A(o.in[1]);
+      nk = 3;
+      return [=](cudaStream_t st) { tsk::layernorm_bwd(dt, dy, xp, gw, dx, acc, ws, dg, dbt, pacc, rows, H, eps, st); };
+    }
+    case TS_OP_ADD: {
+      if (!bwd) {
+        char *a = V(o.in[0]), *b = V(o.in[1]), *y = V(o.out[0]);
+        nk = 1;
+        return [=](cudaStream_t st) { tsk::add_fwd(dt, a, b, y, n_out, st); };
+      }
+      char* dy = G(o.out[0]);
+      std::vector<std::pair<char*, int>> outs;
+      for (int i = 0; i < 2; ++i) {
+        const Tensor& x = g.t[o.in[i]];
+        if (x.kind == TS_ACT && x.needs_grad) outs.push_back({G(o.in[i]), A(g.n() + o.in[i])});
+      }
+      nk = int(outs.size());
+      return [=](cudaStream_t st) {
+        for (auto& pr : outs) tsk::axpy(dt, dy, pr.first, pr.second, n_out, st);
+      };
+    }
+    case TS_OP_DROPOUT: {
+      const float p = float(o.fa[0]);
+      const uint32_t seed = uint32_t(o.ia[0]);
+      nk = 1;
+      if (!bwd) {
+        char *x = V(o.in[0]), *y = V(o.out[0]);
+        return [=](cudaStream_t st) { tsk::dropout(dt, x, y, 0, n_out, elem0, p, seed, *stepp, st); };
+      }
+      char *dy = G(o.out[0]), *dx = G(o.in[0]);
+      int acc = A(g.n() + o.in[0]);
+      return [=](cudaStream_t st) { tsk::dropout(dt, dy, dx, acc, n_out, elem0, p, seed, *stepp, st); };
+    }
+    case TS_OP_SOFTMAX: {
+      const int L = int(out.shape[out.ndim - 1]);
+      const int64_t rows = n_out / L;
+      nk = 1;
+      if (!bwd) {
+        char *x = V(o.in[0]), *y = V(o.out[0]);
+        return [=](cudaStream_t st) { tsk::softmax_fwd(dt, x, y, rows, L, st); };
+      }
+      char *dy = G(o.out[0]), *y = V(o.out[0]), *dx = G(o.in[0]);
+      int acc = A(g.n() + o.in[0]);
+      return [=](cudaStream_t st) { tsk::softmax_bwd(dt, dy, y, dx, acc, rows, L, st); };
+    }
+    case TS_OP_ATTN_QK: case TS_OP_ATTN_PV: {
+      const int heads = int(o.ia[0]), seq = int(o.ia[1]);
+      const Tensor& hx = g.t[o.kind == TS_OP_ATTN_QK ? o.in[0] : o.in[1]];
+      const int64_t h = hx.shape[1], d = h / heads;
+      const int64_t ss = int64_t(seq) * seq, sh = int64_t(seq) * h;
+      auto sop = [&](char* p, bool mn) { return tsk::GemmOperand{p, seq, mn, ss, heads * ss}; };
+      auto hop = [&](char* p, bool mn) { return tsk::GemmOperand{p, h, mn, d, sh}; };
+      std::vector<tsk::GemmArgs> gs;
+      auto base = [&](int M, int N, int K) {
+        tsk::GemmArgs a;
+        a.M = M; a.N = N; a.K = K; a.nb1 = heads; a.nb2 = int(ns); a.in_dtype = dt; a.c_dtype = dt;
+        return a;
+      };
+      if (o.kind == TS_OP_ATTN_QK) {
+        const float alpha = float(o.fa[0]);
+        if (!bwd) {
+          auto a = base(seq, seq, int(d));
+          a.a = hop(V(o.in[0]), false);
+          a.b = hop(V(o.in[1]), false);
+          a.c = V(o.out[0]); a.ldc = seq; a.cbs1 = ss; a.cbs2 = heads * ss; a.alpha = alpha;
+          gs.push_back(a);
+        } else {
+          char* dS = G(o.out[0]);
+          if (g.t[o.in[0]].needs_grad) {
+            auto a = base(seq, int(d), seq);  // dQ = alpha dS K
+            a.a = sop(dS, false);
+            a.b = hop(V(o.in[1]), true);
+            a.c = G(o.in[0]); a.ldc = h; a.cbs1 = d; a.cbs2 = sh; a.alpha = alpha;
+            a.beta = A(g.n() + o.in[0]) ? 1.f : 0.f;
+            gs.push_back(a);
+          }
+          if (g.t[o.in[1]].needs_grad) {
+            auto a = base(seq, int(d), seq);  // dK = alpha dS^T Q
+            a.a = sop(dS, true);
+            a.b = hop(V(o.in[0]), true);
+            a.c = G(o.in[1]); a.ldc = h; a.cbs1 = d; a.cbs2 = sh; a.alpha = alpha;
+            a.beta = A(g.n() + o.in[1]) ? 1.f : 0.f;
+            gs.push_back(a);
+          }
+        }
+      } else {
+        if (!bwd) {
+          auto a = base(seq, int(d), seq);  // C = P V
+          a.a = sop(V(o.in[0]), false);
+          a.b = hop(V(o.in[1]), true);
+          a.c = V(o.out[0]); a.ldc = h; a.cbs1 = d; a.cbs2 = sh;
+          gs.push_back(a);
+        } else {
+          char* dC = G(o.out[0]);
+          if (g.t[o.in[0]].needs_grad) {
+            auto a = base(seq, seq, int(d));  // dP = dC V^T
+            a.a = hop(dC, false);
+            a.b = hop(V(o.in[1]), false);
+            a.c = G(o.in[0]); a.ldc = seq; a.cbs1 = ss; a.cbs2 = heads * ss;
+            a.beta = A(g.n() + o.in[0]) ? 1.f : 0.f;
+            gs.push_back(a);
+          }
+          if (g.t[o.in[1]].needs_grad) {
+            auto a = base(seq, int(d), seq);  // dV = P^T dC
+            a.a = sop(V(o.in[0]), true);
+            a.b = hop(dC, true);
+            a.c = G(o.in[1]); a.ldc = h; a.cbs1 = d; a.cbs2 = sh;
+            a.beta = A(g.n() + o.in[1]) ? 1.f : 0.f;
+            gs.push_back(a);
+          }
+        }
+      }
+      nk = int(gs.size());
+      return [gs](cudaStream_t st) {
+        for (auto& a : gs) tsk::gemm(a, st);
+      };
+    }
+    case TS_OP_EMBED: {
+      const int seq = int(o.ia[0]);
+      const int H = int(out.shape[1]);
+      const int64_t rows = ns * out.rows_per_sample;
+      const int64_t row0 = m.s0 * out.rows_per_sample;
+      const int* ids = reinterpret_cast<const int*>(V(o.in[0]));
+      const int* tt = reinterpret_cast<const int*>(V(o.in[1]));
+      if (!bwd) {
+        char *ww = param_w(s, o.in[2]), *wp = param_w(s, o.in[3]), *wt = param_w(s, o.in[4]), *y = V(o.out[0]);
+        nk = 1;
+        return [=](cudaStream_t st) { tsk::embed_fwd(dt, ids, tt, ww, wp, wt, y, rows, H, seq, row0, st); };
+      }
+      char* dy = G(o.out[0]);
+      float *dw = param_g(s, o.in[2]), *dp = param_g(s, o.in[3]), *dtp = param_g(s, o.in[4]);
+      const int ntype = int(g.t[o.in[4]].shape[0]);
+      nk = 2 + 2 * ntype;
+      return [=](cudaStream_t st) {
+        tsk::embed_bwd_word(dt, dy, ids, dw, rows, H, st);
+        tsk::embed_bwd_pos(dt, dy, dp, ns * out.rows_per_sample / seq, seq, H, 1, st);
+        for (int r = 0; r < ntype; ++r) tsk::column_sum(dt, dy, rows, H, ws, dtp + int64_t(r) * H, 1, tt, r, st);
+      };
+    }
+    case TS_OP_CLS: {
+      const int seq = int(o.ia[0]);
+      const int H = int(out.shape[1]);
+      nk = 1;
+      if (!bwd) {
+        char *x = V(o.in[0]), *y = V(o.out[0]);
+        return [=](cudaStream_t st) { tsk::cls_fwd(dt, x, y, ns, seq, H, st); };
+      }
+      char *dy = G(o.out[0]), *dx = G(o.in[0]);
+      int acc = A(g.n() + o.in[0]);
+      return [=](cudaStream_t st) { tsk::cls_bwd(dt, dy, dx, acc, ns, seq, H, st); };
+    }
+    case TS_OP_XENT: {
+      const int C = int(g.t[o.in[0]].shape[1]);
+      const float inv_b = 1.f / float(B);
+      char* z = V(o.in[0]);
+      const int* lab = reinterpret_cast<const int*>(V(o.in[1]));
+      nk = 1;
+      if (!bwd) {
+        float* loss = reinterpret_cast<float*>(V(o.out[0]));
+        int acc = m.k > 0;
+        return [=](cudaStream_t st) { tsk::xent_fwd(dt, z, lab, loss, acc, ns, C, inv_b, st); };
+      }
+      char* dz = G(o.in[0]);
+      int acc = A(g.n() + o.in[0]);
+      return [=](cudaStream_t st) { tsk::xent_bwd(dt, z, lab, dz, acc, ns, C, inv_b, st); };
+    }
+  }
+  nk = 0;
+  return [](cudaStream_t) {};
+}
+
+ts_status build_program(ts_session_t* s) {
+  const Graph& g = *s->g;
+  const int n = g.n();
+  const int B = g.samples;
+  const int es = dtype_bytes(g.dtype);
+  // host slots for swapped pieces (pinned, allocated once)
+  std::map<PieceKey, uint64_t> host_off;
+  uint64_t hb = 0;
+  for (auto& it : s->ex.items)
+    if (it.kind == IT_SO) {
+      PieceKey pc = it.reads[0];
+      if (!host_off.count(pc)) {
+        host_off[pc] = hb;
+        hb += align_up(piece_bytes(g, s->cfg, pk_key(pc)));
+      }
+    }
+  s->host_bytes = hb;
+  if (hb) {
+    if (cudaHostAlloc(reinterpret_cast<void**>(&s->host), hb, cudaHostAllocDefault) != cudaSuccess) {
+      set_error("cudaHostAlloc of the swap pool failed");
+      return TS_ERR_HOST_MEM;
+    }
+  }
+  // replay the trace: per item, the offset of every live piece
+  std::unordered_map<PieceKey, uint64_t> where;
+  size_t ev = 0;
+  const auto& tr = s->sim.trace;
+  while (ev < tr.size() && tr[ev].item < 0) {
+    where[pk(tr[ev].key, tr[ev].piece)] = tr[ev].offset;
+    s->inputs.push_back({tr[ev].key, tr[ev].offset});
+    ++ev;
+  }
+  // fences: (offset, len, SO item) not yet waited for by the compute / H2D stream
+  struct Fence {
+    uint64_t off, len;
+    int so;
+  };
+  std::vector<Fence> pend_cs, pend_h2d;
+  std::map<PieceKey, int> so_item_of, si_live;
+  std::set<int> act_grad_started;   // grad keys already written by an earlier bwd op
+  std::map<int, int> grad_first_op; // grad key -> first bwd op writing it
+  std::set<int> param_started;
+  std::map<int, int> param_first_item;
+  s->ev_d2h.assign(s->ex.items.size(), nullptr);
+  s->ev_h2d.assign(s->ex.items.size(), nullptr);
+  auto overlaps = [](uint64_t a0, uint64_t al, uint64_t b0, uint64_t bl) { return a0 < b0 + bl && b0 < a0 + al; };
+  for (size_t i = 0; i < s->ex.items.size(); ++i) {
+    const Item& it = s->ex.items[i];
+    Cmd cmd;
+    cmd.item = int(i);
+    // allocation events of this item
+    std::vector<std::pair<uint64_t, uint64_t>> allocs;
+    size_t e0 = ev;
+    while (ev < tr.size() && tr[ev].item == int(i) && tr[ev].kind == 0) {
+      where[pk(tr[ev].key, tr[ev].piece)] = tr[ev].offset;
+      allocs.push_back({tr[ev].offset, align_up(tr[ev].bytes)});
+      ++ev;
+    }
+    (void)e0;
+    auto& pend = it.kind == IT_SI ? pend_h2d : pend_cs;
+    for (auto& a : allocs)
+      for (size_t f = 0; f < pend.size();) {
+        if (overlaps(a.first, a.second, pend[f].off, pend[f].len)) {
+          cmd.wait_so.push_back(pend[f].so);
+          pend.erase(pend.begin() + f);
+        } else {
+          ++f;
+        }
+      }
+    if (it.kind == IT_SO) {
+      PieceKey pc = it.reads[0];
+      cmd.kind = 1;
+      cmd.dev = s->slab + where.at(pc);
+      cmd.bytes = piece_bytes(g, s->cfg, pk_key(pc));
+      cmd.host_off = host_off.at(pc);
+      so_item_of[pc] = int(i);
+      Fence f{where.at(pc), align_up(cmd.bytes), int(i)};
+      pend_cs.push_back(f);
+      pend_h2d.push_back(f);
+      CU(cudaEventCreateWithFlags(&s->ev_d2h[i], cudaEventDisableTiming));
+    } else if (it.kind == IT_SI) {
+      PieceKey pc = it.writes[0];
+      cmd.kind = 2;
+      cmd.dev = s->slab + where.at(pc);
+      cmd.bytes = piece_bytes(g, s->cfg, pk_key(pc));
+      cmd.host_off = host_off.at(pc);
+      cmd.so_of_piece = so_item_of.at(pc);
+      si_live[pc] = int(i);
+      CU(cudaEventCreateWithFlags(&s->ev_h2d[i], cudaEventDisableTiming));
+    } else {
+      cmd.kind = 0;
+      for (PieceKey pc : it.reads) {
+        auto si = si_live.find(pc);
+        if (si != si_live.end()) {
+          cmd.wait_si.push_back(si->second);
+          si_live.erase(si);  // the compute stream is ordered after it from now on
+        }
+      }
+      const Op& o = g.ops[it.op];
+      Micro m;
+      m.op = it.op;
+      m.k = it.k;
+      m.P = s->ex.P[it.op];
+      m.s0 = int64_t(it.k) * B / m.P;
+      m.s1 = int64_t(it.k + 1) * B / m.P;
+      auto view = [&](int key) -> char* {
+        int t = key >= n ? key - n : key;
+        const Tensor& x = g.t[t];
+        if (!x.sample) return s->slab + where.at(pk(key, 0));
+        int p = piece_count(g, s->cfg, t);
+        int j = int(m.s0 * p / B);
+        int64_t first = int64_t(j) * B / p;
+        return s->slab + where.at(pk(key, j)) + (m.s0 - first) * x.elems_per_sample * es;
+      };
+      std::vector<int> ts_all(o.in.begin(), o.in.end());
+      ts_all.insert(ts_all.end(), o.out.begin(), o.out.end());
+      bool bwd = it.kind == IT_B;
+      for (int t : ts_all) {
+        if (g.t[t].kind == TS_PARAM) continue;
+        int key = t;
+        if (where.count(pk(key, g.t[t].sample ? int(m.s0 * piece_count(g, s->cfg, t) / B) : 0))) m.val[t] = view(key);
+        if (bwd && g.t[t].needs_grad && g.t[t].kind == TS_ACT && !g.t[t].is_loss) {
+          int gk = n + t;
+          if (where.count(pk(gk, int(m.s0 * piece_count(g, s->cfg, t) / B)))) m.grad[t] = view(gk);
+        }
+      }
+      if (bwd) {
+        for (int t : o.in) {
+          if (g.t[t].kind == TS_PARAM) {
+            m.acc[t] = param_started.count(t) ? 1 : 0;
+          } else if (g.t[t].kind == TS_ACT && g.t[t].needs_grad) {
+            int gk = n + t;
+            auto f = grad_first_op.find(gk);
+            if (f == grad_first_op.end()) grad_first_op[gk] = it.op;
+            m.acc[gk] = grad_first_op[gk] != it.op ? 1 : 0;
+          }
+        }
+      }
+      int nk = 0;
+      cmd.fn = lower(s, m, bwd, nk);
+      s->launches += nk;
+      if (bwd)
+        for (int t : o.in)
+          if (g.t[t].kind == TS_PARAM) param_started.insert(t);
+    }
+    // frees after this item
+    while (ev < tr.size() && tr[ev].item == int(i) && tr[ev].kind == 1) {
+      where.erase(pk(tr[ev].key, tr[ev].piece));
+      ++ev;
+    }
+    s->prog.push_back(std::move(cmd));
+  }
+  // the loss piece stays allocated to the end
+  for (auto& e : tr)
+    if (e.kind == 0 && e.key == g.loss) s->loss_off = e.offset;
+  for (auto& o : g.ops)
+    if (o.kind == TS_OP_EMBED)
+      for (int i = 2; i < 5; ++i) s->zero_grads.push_back(o.in[i]);
+  CU(cudaEventCreateWithFlags(&s->ev_mark, cudaEventDisableTiming));
+  CU(cudaEventCreateWithFlags(&s->ev_join_d2h, cudaEventDisableTiming));
+  CU(cudaEventCreateWithFlags(&s->ev_join_h2d, cudaEventDisableTiming));
+  return TS_OK;
+}
+
+// Issue one step's work (everything after the input copies) on the streams.
+void issue_step(ts_session_t* s) {
+  const Graph& g = *s->g;
+  cudaStream_t cs = s->cs;
+  for (int t : s->zero_grads) cudaMemsetAsync(param_g(s, t), 0, size_t(g.t[t].numel) * 4, cs);
+  bool d2h_used = false, h2d_used = false;
+  for (auto& c : s->prog) {
+    if (c.kind == 0) {
+      for (int so : c.wait_so) cudaStreamWaitEvent(cs, s->ev_d2h[so], 0);
+      for (int si : c.wait_si) cudaStreamWaitEvent(cs, s->ev_h2d[si], 0);
+      c.fn(cs);
+    } else if (c.kind == 1) {
+      cudaEventRecord(s->ev_mark, cs);
+      cudaStreamWaitEvent(s->d2h, s->ev_mark, 0);
+      cudaMemcpyAsync(s->host + c.host_off, c.dev, c.bytes, cudaMemcpyDeviceToHost, s->d2h);
+      cudaEventRecord(s->ev_d2h[c.item], s->d2h);
+      d2h_used = true;
+    } else {
+      cudaEventRecord(s->ev_mark, cs);
+      cudaStreamWaitEvent(s->h2d, s->ev_mark, 0);
+      cudaStreamWaitEvent(s->h2d, s->ev_d2h[c.so_of_piece], 0);
+      for (int so : c.wait_so) cudaStreamWaitEvent(s->h2d, s->ev_d2h[so], 0);
+      cudaMemcpyAsync(c.dev, s->host + c.host_off, c.bytes, cudaMemcpyHostToDevice, s->h2d);
+      cudaEventRecord(s->ev_h2d[c.item], s->h2d);
+      h2d_used = true;
+    }
+  }
+  // data-parallel gradient sum (north_star DP) and SGD on fp32 masters
+  uint64_t gbeg = ~0ull, gend = 0, mbeg = ~0ull;
+  for (auto& t : g.t)
+    if (t.kind == TS_PARAM) {
+      gbeg = std::min(gbeg, g.grad_off[t.id]);
+      gend = std::max(gend, g.grad_off[t.id] + align_up(4 * t.numel));
+      mbeg = std::min(mbeg, g.master_off[t.id]);
+    }
+  if (gend > gbeg && s->nccl && s->allreduce && s->world > 1)
+    s->allreduce(s->slab + gbeg, s->slab + gbeg, (gend - gbeg) / 4, kNcclFloat32, kNcclSum, s->nccl, cs);
+  if (s->lr != 0.f && gend > gbeg) {
+    tsk::sgd_update(reinterpret_cast<float*>(s->slab + mbeg), reinterpret_cast<const float*>(s->slab + gbeg),
+                    int64_t((gend - gbeg) / 4), s->lr, 1.f / float(s->world), cs);
+    if (g.dtype == TS_BF16)
+      for (auto& t : g.t)
+        if (t.kind == TS_PARAM)
+          tsk::cast_f32_bf16(reinterpret_cast<float*>(s->slab + g.master_off[t.id]), s->slab + g.copy_off[t.id],
+                             t.numel, cs);
+  }
+  if (d2h_used) {
+    cudaEventRecord(s->ev_join_d2h, s->d2h);
+    cudaStreamWaitEvent(cs, s->ev_join_d2h, 0);
+  }
+  if (h2d_used) {
+    cudaEventRecord(s->ev_join_h2d, s->h2d);
+    cudaStreamWaitEvent(cs, s->ev_join_h2d, 0);
+  }
+}
+
+ts_status copy_inputs(ts_session_t* s, const void* const* inputs, int on_host) {
+  const Graph& g = *s->g;
+  size_t idx = 0;
+  for (auto& t : g.t) {
+    if (t.kind != TS_INPUT && t.kind != TS_LABEL) continue;
+    if (!inputs[idx]) return set_error("null input pointer"), TS_ERR_ARG;
+    uint64_t off = 0;
+    for (auto& pr : s->inputs)
+      if (pr.first == t.id) off = pr.second;
+    CU(cudaMemcpyAsync(s->slab + off, inputs[idx], t.bytes, on_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice,
+                       s->cs));
+    ++idx;
+  }
+  return TS_OK;
+}
+
+ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
+  if (!inputs) return set_error("inputs is null"), TS_ERR_ARG;
+  ts_status st = copy_inputs(s, inputs, on_host);
+  if (st != TS_OK) return st;
+  if (s->use_graph) {
+    if (!s->gexec) {
+      cudaGraph_t graph;
+      CU(cudaStreamBeginCapture(s->cs, cudaStreamCaptureModeThreadLocal));
+      issue_step(s);
+      CU(cudaStreamEndCapture(s->cs, &graph));
+      size_t nn = 0;
+      cudaGraphGetNodes(graph, nullptr, &nn);
+      std::vector<cudaGraphNode_t> nodes(nn);
+      cudaGraphGetNodes(graph, nodes.data(), &nn);
+      s->graph_kernels = 0;
+      for (auto nd : nodes) {
+        cudaGraphNodeType ty;
+        cudaGraphNodeGetType(nd, &ty);
+        if (ty == cudaGraphNodeTypeKernel) ++s->graph_kernels;
+      }
+      CU(cudaGraphInstantiate(&s->gexec, graph, 0));
+      cudaGraphDestroy(graph);
+    }
+    CU(cudaGraphLaunch(s->gexec, s->cs));
+  } else {
+    issue_step(s);
+  }
+  ++s->step;  // dropout counter (graph mode keeps the captured step value)
+  CU(cudaGetLastError());
+  return TS_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+ts_status ts_session_create(const ts_graph_t* gh, const ts_plan_t* ph, const ts_session_cfg* cfg, ts_session_t** out) {
+  if (!gh || !ph || !cfg || !out) return set_error("null argument"), TS_ERR_ARG;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    set_error("no CUDA device: the TSPLIT runtime has no CPU fallback");
+    return TS_ERR_NO_GPU;
+  }
+  if (!cfg->slab) return set_error("slab is null"), TS_ERR_ARG;
+  if (ph->graph != &gh->g) return set_error("plan was made for another graph"), TS_ERR_ARG;
+  auto s = std::make_unique<ts_session_t>();
+  s->g = &gh->g;
+  s->cfg = ph->st.cfg;
+  s->ex = ph->st.ex;
+  s->device = cfg->device;
+  CU(cudaSetDevice(cfg->device));
+  s->slab = static_cast<char*>(cfg->slab);
+  s->slab_bytes = cfg->slab_bytes;
+  // re-simulate on the real slab: the best-fit trace is identical if it fits (R11)
+  if (!simulate(*s->g, s->cfg, s->ex, cfg->slab_bytes, s->sim)) {
+    set_error("plan does not fit the slab (" + std::to_string(cfg->slab_bytes) + " B)");
+    return TS_ERR_BUDGET;
+  }
+  s->world = cfg->world_size > 0 ? cfg->world_size : 1;
+  s->lr = cfg->lr;
+  s->step = cfg->step0;
+  s->use_graph = cfg->use_cuda_graph != 0;
+  if (cfg->stream_compute) {
+    s->cs = static_cast<cudaStream_t>(cfg->stream_compute);
+    s->d2h = static_cast<cudaStream_t>(cfg->stream_d2h);
+    s->h2d = static_cast<cudaStream_t>(cfg->stream_h2d);
+  }
+  if (!s->cs || !s->d2h || !s->h2d) {
+    s->own_streams = true;
+    CU(cudaStreamCreateWithFlags(&s->cs, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&s->d2h, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&s->h2d, cudaStreamNonBlocking));
+  }
+  if (cfg->nccl_comm) {
+    s->nccl = cfg->nccl_comm;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW);
+    if (h) s->allreduce = reinterpret_cast<nccl_allreduce_fn>(dlsym(h, "ncclAllReduce"));
+    if (!s->allreduce) return set_error("ncclAllReduce not found"), TS_ERR_NCCL;
+  }
+  CU(cudaMemsetAsync(s->slab, 0, s->g->static_bytes, s->cs));
+  ts_status st = build_program(s.get());
+  if (st != TS_OK) return st;
+  CU(cudaStreamSynchronize(s->cs));
+  *out = s.release();
+  return TS_OK;
+}
+
+void ts_session_destroy(ts_session_t* s) {
+  if (!s) return;
+  if (s->gexec) cudaGraphExecDestroy(s->gexec);
+  for (auto e : s->ev_d2h)
+    if (e) cudaEventDestroy(e);
+  for (auto e : s->ev_h2d)
+    if (e) cudaEventDestroy(e);
+  if (s->ev_mark) cudaEventDestroy(s->ev_mark);
+  if (s->ev_join_d2h) cudaEventDestroy(s->ev_join_d2h);
+  if (s->ev_join_h2d) cudaEventDestroy(s->ev_join_h2d);
+  if (s->host) cudaFreeHost(s->host);
+  if (s->own_streams) {
+    cudaStreamDestroy(s->cs);
+    cudaStreamDestroy(s->d2h);
+    cudaStreamDestroy(s->h2d);
+  }
+  delete s;
+}
+
+ts_status ts_set_param(ts_session_t* s, int32_t t, const float* host) {
+  if (!s || !host || t < 0 || t >= s->g->n() || s->g->t[t].kind != TS_PARAM) return set_error("bad param"), TS_ERR_ARG;
+  const Tensor& x = s->g->t[t];
+  CU(cudaMemcpyAsync(s->slab + s->g->master_off[t], host, x.numel * 4, cudaMemcpyHostToDevice, s->cs));
+  if (s->g->dtype == TS_BF16)
+    tsk::cast_f32_bf16(reinterpret_cast<float*>(s->slab + s->g->master_off[t]), s->slab + s->g->copy_off[t], x.numel,
+                       s->cs);
+  CU(cudaStreamSynchronize(s->cs));
+  return TS_OK;
+}
+
+ts_status ts_get_param(ts_session_t* s, int32_t t, float* host) {
+  if (!s || !host || t < 0 || t >= s->g->n() || s->g->t[t].kind != TS_PARAM) return set_error("bad param"), TS_ERR_ARG;
+  CU(cudaStreamSynchronize(s->cs));
+  CU(cudaMemcpy(host, s->slab + s->g->master_off[t], s->g->t[t].numel * 4, cudaMemcpyDeviceToHost));
+  return TS_OK;
+}
+
+ts_status ts_get_grad(ts_session_t* s, int32_t t, float* host) {
+  if (!s || !host || t < 0 || t >= s->g->n() || s->g->t[t].kind != TS_PARAM) return set_error("bad param"), TS_ERR_ARG;
+  CU(cudaStreamSynchronize(s->cs));
+  CU(cudaMemcpy(host, s->slab + s->g->grad_off[t], s->g->t[t].numel * 4, cudaMemcpyDeviceToHost));
+  return TS_OK;
+}
+
+ts_status ts_param_ptr(ts_session_t* s, int32_t t, void** dev) {
+  if (!s || !dev || t < 0 || t >= s->g->n() || s->g->t[t].kind != TS_PARAM) return set_error("bad param"), TS_ERR_ARG;
+  *dev = s->slab + s->g->master_off[t];
+  return TS_OK;
+}
+
+ts_status ts_grad_ptr(ts_session_t* s, int32_t t, void** dev) {
+  if (!s || !dev || t < 0 || t >= s->g->n() || s->g->t[t].kind != TS_PARAM) return set_error("bad param"), TS_ERR_ARG;
+  *dev = s->slab + s->g->grad_off[t];
+  return TS_OK;
+}
+
+ts_status ts_step_async(ts_session_t* s, const void* const* inputs, int32_t on_host) {
+  if (!s) return set_error("null session"), TS_ERR_ARG;
+  return run_step(s, inputs, on_host);
+}
+
+ts_status ts_step(ts_session_t* s, const void* const* inputs, int32_t on_host, float* loss_out) {
+  if (!s) return set_error("null session"), TS_ERR_ARG;
+  ts_status st = run_step(s, inputs, on_host);
+  if (st != TS_OK) return st;
+  float loss = 0.f;
+  CU(cudaMemcpyAsync(&loss, s->slab + s->loss_off, 4, cudaMemcpyDeviceToHost, s->cs));
+  CU(cudaStreamSynchronize(s->cs));
+  if (loss_out) *loss_out = loss;
+  return TS_OK;
+}
+
+ts_status ts_session_trace(const ts_session_t* s, ts_alloc_event* buf, uint64_t cap, uint64_t* n) {
+  if (!s || !n) return set_error("null argument"), TS_ERR_ARG;
+  *n = s->sim.trace.size();
+  if (buf)
+    for (uint64_t i = 0; i < s->sim.trace.size() && i < cap; ++i) {
+      const Event& e = s->sim.trace[i];
+      buf[i] = ts_alloc_event{e.seq, e.item, e.kind, e.key, e.piece, e.offset, e.bytes};
+    }
+  return TS_OK;
+}
+
+ts_status ts_session_launches(const ts_session_t* s, int64_t* n) {
+  if (!s || !n) return set_error("null argument"), TS_ERR_ARG;
+  *n = s->graph_kernels > 0 ? s->graph_kernels : s->launches;
+  return TS_OK;
+}
+
+ts_status ts_session_profile_items(ts_session_t* s, int32_t enable) {
+  (void)enable;
+  if (!s) return set_error("null session"), TS_ERR_ARG;
+  return set_error("item profiling not implemented yet"), TS_ERR_STATE;
+}
+
+ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, uint64_t* n) {
+  (void)ms;
+  (void)cap;
+  if (!s || !n) return set_error("null argument"), TS_ERR_ARG;
+  *n = 0;
+  return TS_OK;
+}
+
+ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch, const void* A, int64_t lda, int64_t strideA,
+                       int32_t ta, const void* B, int64_t ldb, int64_t strideB, int32_t tb, void* C, int64_t ldc,
+                       int64_t strideC, int32_t c_dtype, float alpha, float beta, const void* bias, void* stream) {
+  tsk::GemmArgs g;
+  g.M = M; g.N = N; g.K = K; g.nb1 = batch; g.nb2 = 1; g.in_dtype = tsk::BF16;
+  g.a = {A, lda, ta != 0, strideA, 0};
+  g.b = {B, ldb, tb != 0, strideB, 0};
+  g.c = C; g.ldc = ldc; g.cbs1 = strideC; g.c_dtype = c_dtype == TS_F32 ? tsk::F32 : tsk::BF16;
+  g.alpha = alpha; g.beta = beta; g.bias = bias; g.bias_dtype = tsk::BF16;
+  if (!tsk::gemm_tc(g, static_cast<cudaStream_t>(stream)))
+    return set_error("shape/alignment not eligible for the tcgen05/TMA path"), TS_ERR_ARG;
+  CU(cudaGetLastError());
+  return TS_OK;
+}
+
+ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K, const float* A, int64_t lda, int32_t ta, const float* B,
+                      int64_t ldb, int32_t tb, float* C, int64_t ldc, float alpha, float beta, const float* bias,
+                      void* stream) {
+  tsk::GemmArgs g;
+  g.M = M; g.N = N; g.K = K; g.in_dtype = tsk::F32;
+  g.a = {A, lda, ta != 0, 0, 0};
+  g.b = {B, ldb, tb != 0, 0, 0};
+  g.c = C; g.ldc = ldc; g.c_dtype = tsk::F32;
+  g.alpha = alpha; g.beta = beta; g.bias = bias; g.bias_dtype = tsk::F32;
+  tsk::gemm_simt(g, static_cast<cudaStream_t>(stream));
+  CU(cudaGetLastError());
+  return TS_OK;
+}
+
+}  // extern "C"

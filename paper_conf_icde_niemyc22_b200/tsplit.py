@@ -278,3 +278,106 @@ class Plan:
 
     def cfg_dict(self):
         return {t: self.get(t) for t in range(self.graph.n)}
+
+
+# --------------------------------------------------------------------------- session
+class Session:
+    """A device session: the plan's pool is one torch-allocated slab (torch is the
+    device-memory plumbing; all work runs in libtsplit)."""
+
+    def __init__(self, graph: Graph, plan: Plan, device: int = 0, slab_bytes: int | None = None,
+                 lr: float = 0.0, use_cuda_graph: bool = True, nccl_comm: int | None = None,
+                 world_size: int = 1, step0: int = 0):
+        import torch
+        if not torch.cuda.is_available():
+            raise TsError(9, "no CUDA device: the TSPLIT runtime has no CPU fallback")
+        self.graph, self.plan = graph, plan
+        st = plan.stats()
+        self.slab_bytes = int(slab_bytes or st["peak_extent"])
+        self.slab = torch.empty(self.slab_bytes, dtype=torch.uint8, device=f"cuda:{device}")
+        cfg = SessionCfg()
+        cfg.device = device
+        cfg.slab = self.slab.data_ptr()
+        cfg.slab_bytes = self.slab_bytes
+        cfg.nccl_comm = nccl_comm
+        cfg.world_size = world_size
+        cfg.use_cuda_graph = 1 if use_cuda_graph else 0
+        cfg.lr = lr
+        cfg.step0 = step0
+        h = C.c_void_p()
+        check(lib().ts_session_create(graph.h, plan.h, C.byref(cfg), C.byref(h)))
+        self.h = h
+        spec = graph.spec
+        self.input_ids = [t["id"] for t in spec["tensors"] if t["kind"] in ("input", "label")]
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib().ts_session_destroy(self.h)
+
+    def set_params(self, params: dict):
+        for t in self.graph.spec["tensors"]:
+            if t["kind"] == "param":
+                a = np.ascontiguousarray(params[t["name"]], dtype=np.float32)
+                check(lib().ts_set_param(self.h, t["id"], a.ctypes.data))
+
+    def _ptrs(self, inputs):
+        arr = (C.c_void_p * len(self.input_ids))()
+        for i, tid in enumerate(self.input_ids):
+            x = inputs[self.graph.spec["tensors"][tid]["name"]]
+            arr[i] = x.data_ptr() if hasattr(x, "data_ptr") else x.ctypes.data
+        return arr
+
+    def step(self, inputs: dict, on_host: bool | None = None) -> float:
+        """inputs: name -> torch tensor (device or pinned host) or numpy array (host)."""
+        if on_host is None:
+            x0 = inputs[self.graph.spec["tensors"][self.input_ids[0]]["name"]]
+            on_host = not (hasattr(x0, "is_cuda") and x0.is_cuda)
+        loss = C.c_float()
+        check(lib().ts_step(self.h, self._ptrs(inputs), 1 if on_host else 0, C.byref(loss)))
+        return loss.value
+
+    def step_async(self, inputs: dict, on_host: bool = False):
+        check(lib().ts_step_async(self.h, self._ptrs(inputs), 1 if on_host else 0))
+
+    def grads(self) -> dict:
+        out = {}
+        for t in self.graph.spec["tensors"]:
+            if t["kind"] == "param":
+                a = np.empty(t["shape"], np.float32)
+                check(lib().ts_get_grad(self.h, t["id"], a.ctypes.data))
+                out[t["name"]] = a
+        return out
+
+    def param(self, name) -> np.ndarray:
+        t = self.graph.spec["tensors"][self.graph.names[name]]
+        a = np.empty(t["shape"], np.float32)
+        check(lib().ts_get_param(self.h, t["id"], a.ctypes.data))
+        return a
+
+    def trace(self):
+        n = C.c_uint64()
+        check(lib().ts_session_trace(self.h, None, 0, C.byref(n)))
+        buf = (AllocEvent * n.value)()
+        check(lib().ts_session_trace(self.h, buf, n.value, C.byref(n)))
+        return [(e.seq, e.item, "A" if e.kind == 0 else "F", e.key, e.piece, e.offset, e.bytes) for e in buf]
+
+    def launches(self) -> int:
+        n = C.c_int64()
+        check(lib().ts_session_launches(self.h, C.byref(n)))
+        return n.value
+
+
+def inputs_to_device(graph: Graph, arrays: dict, device="cuda:0", pinned_host=False):
+    import torch
+    out = {}
+    for t in graph.spec["tensors"]:
+        if t["kind"] in ("input", "label"):
+            a = arrays[t["name"]]
+            if t["dtype"] == "i32":
+                x = torch.from_numpy(np.ascontiguousarray(a, np.int32))
+            elif t["dtype"] == "bf16":
+                x = torch.from_numpy(np.ascontiguousarray(a, np.float32)).to(torch.bfloat16)
+            else:
+                x = torch.from_numpy(np.ascontiguousarray(a, np.float32))
+            out[t["name"]] = x.pin_memory() if pinned_host else x.to(device)
+    return out

@@ -1,0 +1,108 @@
+"""End-to-end parity of the CUDA path (C ABI session) against the fp64 oracle and
+against itself under different plans (north_star targets:
+fp32 <= 1e-5, bf16 <= 2e-2 vs the oracle, split vs unsplit <= 1e-6 for fp32)."""
+
+import random
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+from conftest import rel_errs  # noqa: E402
+from oracle import brute, net, sim  # noqa: E402
+from paper_conf_icde_niemyc22_b200 import tsplit  # noqa: E402
+from tsinputs import gen, graphs  # noqa: E402
+
+
+def _run(g, plan_cfg=None, budget=None, graph_mode=True, on_host=False):
+    G = tsplit.Graph(g)
+    if budget is not None:
+        P = tsplit.Plan.plan(G, budget)
+    else:
+        P = tsplit.Plan.default(G)
+        for t, (o, p, lead) in (plan_cfg or {}).items():
+            P.set(t, o, p, lead)
+    S = tsplit.Session(G, P, use_cuda_graph=graph_mode)
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    S.set_params(params)
+    dev = tsplit.inputs_to_device(G, inputs, pinned_host=on_host)
+    loss = S.step(dev)
+    return loss, S.grads(), S, P
+
+
+def _oracle(g):
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    loss, pg, _, _ = net.train_step(g, params, inputs)
+    return loss, pg
+
+
+def test_config1_mlp_fp32_forced_plan_parity():
+    """Config 1: 2-way batch split on every op + one swapped activation, fp32."""
+    g = graphs.mlp()
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    cfg = {t: (tsplit.RESIDE, 2, 1) for t in brute.act_tensors(g)}
+    cfg[names["relu0"]] = (tsplit.SWAP, 2, 1)
+    loss, grads, S, P = _run(g, cfg)
+    st = P.stats()
+    assert st["d2h_bytes"] == st["h2d_bytes"] > 0
+    ol, og = _oracle(g)
+    assert abs(loss - ol) <= 1e-5 * abs(ol)
+    errs = rel_errs(grads, og)
+    assert max(errs.values()) <= 1e-5, errs
+    # split + swap vs unsplit on the GPU
+    l0, g0, _, _ = _run(g)
+    assert max(rel_errs(grads, g0).values()) <= 1e-6
+    # the runtime's allocation trace is the simulator's
+    assert S.trace() == [tuple(e) for e in sim.simulate(g, {**sim.default_cfg(g), **cfg}).trace]
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_bert_tiny_fp32_random_plans(seed):
+    g = graphs.config_graph("bert_tiny", dtype="f32")
+    r = random.Random(seed)
+    cfg = {t: (r.choice([0, 1, 2]), r.choice([1, 2, 4]), r.choice([1, 2])) for t in brute.act_tensors(g)}
+    loss, grads, S, P = _run(g, cfg)
+    ol, og = _oracle(g)
+    assert abs(loss - ol) <= 1e-5 * abs(ol)
+    errs = rel_errs(grads, og)
+    assert max(errs.values()) <= 1e-5, sorted(errs.items(), key=lambda kv: -kv[1])[:5]
+    l0, g0, _, _ = _run(g)
+    assert max(rel_errs(grads, g0).values()) <= 1e-6
+
+
+def test_bert_tiny_bf16_parity_and_budget():
+    g = graphs.config_graph("bert_tiny")
+    ol, og = _oracle(g)
+    loss, grads, S, P = _run(g)
+    assert abs(loss - ol) <= 2e-2 * abs(ol)
+    errs = rel_errs(grads, og)
+    assert max(errs.values()) <= 2e-2, sorted(errs.items(), key=lambda kv: -kv[1])[:5]
+    base = P.stats()
+    budget = base["static_bytes"] + (base["peak_extent"] - base["static_bytes"]) * 4 // 10
+    l2, g2, S2, P2 = _run(g, budget=budget)
+    assert P2.stats()["peak_extent"] <= budget
+    assert max(rel_errs(g2, og).values()) <= 2e-2
+    assert max(rel_errs(g2, grads).values()) <= 1e-2
+
+
+def test_eager_equals_graph_and_host_inputs():
+    g = graphs.config_graph("bert_tiny", dtype="f32")
+    l1, g1, _, _ = _run(g, graph_mode=True)
+    l2, g2, _, _ = _run(g, graph_mode=False, on_host=True)
+    assert abs(l1 - l2) <= 1e-6 * abs(l1)
+    assert max(rel_errs(g2, g1).values()) <= 1e-6
+
+
+def test_sgd_step_changes_params_and_loss_drops():
+    g = graphs.mlp()
+    G = tsplit.Graph(g)
+    P = tsplit.Plan.default(G)
+    S = tsplit.Session(G, P, lr=0.5)
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    S.set_params(params)
+    dev = tsplit.inputs_to_device(G, inputs)
+    losses = [S.step(dev) for _ in range(5)]
+    assert losses[-1] < losses[0]
+    assert not np.allclose(S.param("fc0.w"), params["fc0.w"])
