@@ -227,6 +227,16 @@ ts_status ts_session_launches(const ts_session_t* s, int64_t* n);
 ts_status ts_session_profile_items(ts_session_t* s, int32_t enable);
 ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, uint64_t* n);
 
+/* ---- data parallelism (north_star: DP over NVLink with NCCL) -------------------
+ * The session allreduces the fp32 gradient region (sum) with this communicator
+ * on the compute stream after the backward pass, then scales by 1/world in SGD.
+ * Bootstrap: rank 0 calls ts_nccl_unique_id (128 opaque bytes), the caller
+ * broadcasts them (torch.distributed), every rank calls ts_nccl_comm_init.
+ * NCCL is resolved from the libnccl.so.2 already in the process (torch's). */
+ts_status ts_nccl_unique_id(void* out128);
+ts_status ts_nccl_comm_init(const void* id128, int32_t nranks, int32_t rank, void** comm);
+ts_status ts_nccl_comm_destroy(void* comm);
+
 /* ---- kernels exposed for unit tests (device pointers, compute stream) -------- */
 /* C[b] = alpha * op(A[b]) op(B[b]) (+ beta*C + bias): bf16 in, fp32 accumulate on
  * tcgen05 (TMEM), out bf16 or f32.  ta/tb = 1 when the operand's contiguous dim is

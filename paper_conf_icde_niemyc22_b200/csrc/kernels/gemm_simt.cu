@@ -10,7 +10,10 @@ namespace tsk {
 namespace {
 constexpr int TM = 64, TN = 64, TK = 16;
 
-template <class TI, class TO>
+// fp32 inputs accumulate in fp64 (AccT = double): a true-fp32 graph's products are
+// then correctly rounded, and a split of the K (sample) dimension changes them only
+// by the final fp32 accumulation (split invariance).
+template <class TI, class TO, class AccT>
 __global__ void __launch_bounds__(256) gemm_simt_kernel(GemmArgs g) {
   __shared__ float As[TK][TM + 4];
   __shared__ float Bs[TK][TN + 4];
@@ -20,7 +23,7 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(GemmArgs g) {
   const TI* B = reinterpret_cast<const TI*>(g.b.ptr) + b1 * g.b.bs1 + b2 * g.b.bs2;
   const int m0 = blockIdx.y * TM, n0 = blockIdx.x * TN;
   const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
-  float acc[4][4] = {};
+  AccT acc[4][4] = {};
   for (int k0 = 0; k0 < g.K; k0 += TK) {
     for (int i = threadIdx.x; i < TM * TK; i += 256) {
       int mm, kk;
@@ -41,7 +44,7 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(GemmArgs g) {
     __syncthreads();
 #pragma unroll
     for (int kk = 0; kk < TK; ++kk) {
-      float a[4], b[4];
+      AccT a[4], b[4];
 #pragma unroll
       for (int i = 0; i < 4; ++i) a[i] = As[kk][ty * 4 + i];
 #pragma unroll
@@ -49,7 +52,7 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(GemmArgs g) {
 #pragma unroll
       for (int i = 0; i < 4; ++i)
 #pragma unroll
-        for (int j = 0; j < 4; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        for (int j = 0; j < 4; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
     }
     __syncthreads();
   }
@@ -62,13 +65,13 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(GemmArgs g) {
     for (int j = 0; j < 4; ++j) {
       int n = n0 + tx * 4 + j;
       if (n >= g.N) continue;
-      float v = acc[i][j] * g.alpha;
+      AccT v = acc[i][j] * AccT(g.alpha);
       if (g.bias)
-        v += g.bias_dtype == F32 ? reinterpret_cast<const float*>(g.bias)[n]
-                                 : to_f(reinterpret_cast<const bf16*>(g.bias)[n]);
+        v += g.bias_dtype == F32 ? AccT(reinterpret_cast<const float*>(g.bias)[n])
+                                 : AccT(to_f(reinterpret_cast<const bf16*>(g.bias)[n]));
       TO* cp = C + int64_t(m) * g.ldc + n;
-      if (g.beta != 0.f) v += g.beta * to_f(*cp);
-      *cp = from_f<TO>(v);
+      if (g.beta != 0.f) v += AccT(g.beta) * AccT(to_f(*cp));
+      *cp = from_f<TO>(float(v));
     }
   }
 }
@@ -77,11 +80,11 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(GemmArgs g) {
 void gemm_simt(const GemmArgs& g, cudaStream_t st) {
   dim3 grid((g.N + TN - 1) / TN, (g.M + TM - 1) / TM, g.nb1 * g.nb2);
   if (g.in_dtype == F32) {
-    if (g.c_dtype == F32) gemm_simt_kernel<float, float><<<grid, 256, 0, st>>>(g);
-    else gemm_simt_kernel<float, bf16><<<grid, 256, 0, st>>>(g);
+    if (g.c_dtype == F32) gemm_simt_kernel<float, float, double><<<grid, 256, 0, st>>>(g);
+    else gemm_simt_kernel<float, bf16, double><<<grid, 256, 0, st>>>(g);
   } else {
-    if (g.c_dtype == F32) gemm_simt_kernel<bf16, float><<<grid, 256, 0, st>>>(g);
-    else gemm_simt_kernel<bf16, bf16><<<grid, 256, 0, st>>>(g);
+    if (g.c_dtype == F32) gemm_simt_kernel<bf16, float, float><<<grid, 256, 0, st>>>(g);
+    else gemm_simt_kernel<bf16, bf16, float><<<grid, 256, 0, st>>>(g);
   }
 }
 

@@ -29,6 +29,7 @@ constexpr int kThreads = 192;  // warp0 TMA, warp1 MMA, warps2-5 epilogue
 struct TcParams {
   int M, N, K, nb1, nb2;
   int tiles_m, tiles_n, num_tiles, num_kb;
+  int ksplit, kb_per_split, num_units;  // work unit = (tile, K slice)
   int a_mn, b_mn;
   void* C;
   int64_t ldc, cbs1, cbs2;
@@ -36,7 +37,10 @@ struct TcParams {
   float alpha, beta;
   const void* bias;
   int bias_f32;
+  int tma_store;   // 1: stage in smem and TMA-store; 0: direct per-thread stores
+  int reduce_add;  // 1: TMA reduce-add into an fp32 C (beta = 1 or split-K)
 };
+constexpr int kStageBytesPerWarp = 2 * 4096;  // double-buffered 32x32 fp32 block
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -71,6 +75,24 @@ __device__ __forceinline__ void tma_load(void* dst, const CUtensorMap* map, uint
       "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
       : "memory");
 }
+__device__ __forceinline__ void tma_store(const CUtensorMap* map, const void* src, int c0, int c1, int c2, int c3) {
+  asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+               : "memory");
+}
+__device__ __forceinline__ void tma_reduce_add(const CUtensorMap* map, const void* src, int c0, int c1, int c2,
+                                               int c3) {
+  asm volatile(
+      "cp.reduce.async.bulk.tensor.4d.global.shared::cta.add.bulk_group [%0, {%2, %3, %4, %5}], [%1];" ::"l"(
+          reinterpret_cast<uint64_t>(map)),
+      "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_commit(uint64_t* bar) {
@@ -125,7 +147,7 @@ __device__ __forceinline__ void decode_tile(const TcParams& p, int tile, int& b1
 template <int BN>
 __global__ void __launch_bounds__(kThreads, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   const TcParams p) {
+                   const __grid_constant__ CUtensorMap tmC, const TcParams p) {
   constexpr int A_BYTES = BM * BK * 2;
   constexpr int B_BYTES = BN * BK * 2;
   constexpr int STAGE = A_BYTES + B_BYTES;
@@ -142,6 +164,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint64_t* tfull = empty + STAGES;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint8_t* cstage = smem + STAGES * STAGE + 1024;  // 1024-aligned epilogue staging
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (warp == 0 && lane == 0) {
@@ -172,11 +195,14 @@ __global__ void __launch_bounds__(kThreads, 1)
       // ===== TMA producer =====
       int stage = 0;
       uint32_t phase = 0;
-      for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+      for (int unit = blockIdx.x; unit < p.num_units; unit += gridDim.x) {
+        const int tile = unit / p.ksplit, ks = unit - tile * p.ksplit;
         int b1, b2, m0, nt;
         decode_tile(p, tile, b1, b2, m0, nt);
         int n0 = nt * BN;
-        for (int kb = 0; kb < p.num_kb; ++kb) {
+        const int kb0 = ks * p.kb_per_split;
+        const int kb1 = min(p.num_kb, kb0 + p.kb_per_split);
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * STAGE;
           uint8_t* sb = sa + A_BYTES;
@@ -213,11 +239,14 @@ __global__ void __launch_bounds__(kThreads, 1)
       // (SBO), K step of 16 = +2048 B.
       const uint32_t a_lbo = p.a_mn ? 8192 : 16, b_lbo = p.b_mn ? 8192 : 16;
       const uint32_t a_kstep = p.a_mn ? 2048 : 32, b_kstep = p.b_mn ? 2048 : 32;
-      for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+      for (int unit = blockIdx.x; unit < p.num_units; unit += gridDim.x) {
+        const int ks = unit % p.ksplit;
+        const int kb0 = ks * p.kb_per_split;
+        const int kb1 = min(p.num_kb, kb0 + p.kb_per_split);
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
         const uint32_t tmem_d = tmem_base + uint32_t(acc * BN);
-        for (int kb = 0; kb < p.num_kb; ++kb) {
+        for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&full[stage], phase);
           tc_fence_after();
           uint32_t sa = smem_u32(smem + stage * STAGE);
@@ -226,7 +255,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int k = 0; k < BK / 16; ++k) {
             uint64_t ad = smem_desc(sa + k * a_kstep, a_lbo, 1024);
             uint64_t bd = smem_desc(sb + k * b_kstep, b_lbo, 1024);
-            tc_mma(tmem_d, ad, bd, idesc, (kb | k) != 0);
+            tc_mma(tmem_d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
           }
           tc_commit(&empty[stage]);
           if (++stage == STAGES) {
@@ -242,11 +271,16 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
     }
   } else {
-    // ===== epilogue: TMEM -> registers -> global (alpha, bias, beta*C) =====
+    // ===== epilogue: TMEM -> registers (alpha, bias) -> swizzled smem -> TMA store =====
     const int q = warp & 3;  // TMEM lane quarter this warp may access
+    const int ew = warp - 2; // epilogue warp index 0..3
+    uint8_t* wbuf = cstage + ew * kStageBytesPerWarp;
+    int nbuf = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int tile = blockIdx.x; tile < p.num_tiles; tile += gridDim.x) {
+    const int es = p.c_f32 ? 4 : 2;
+    for (int unit = blockIdx.x; unit < p.num_units; unit += gridDim.x) {
+      const int tile = unit / p.ksplit;
       int b1, b2, m0, nt;
       decode_tile(p, tile, b1, b2, m0, nt);
       int n0 = nt * BN;
@@ -260,63 +294,65 @@ __global__ void __launch_bounds__(kThreads, 1)
         uint32_t r[32];
         tmem_ld32(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * BN + c * 32), r);
         const int col0 = n0 + c * 32;
-        if (row_ok && col0 < p.N) {
-        float v[32];
+        if (col0 < p.N) {
+          float v[32];
 #pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
-        const bool full_chunk = col0 + 32 <= p.N;
-        if (p.bias) {
-#pragma unroll
-          for (int i = 0; i < 32; ++i)
-            if (full_chunk || col0 + i < p.N)
-              v[i] += p.bias_f32 ? reinterpret_cast<const float*>(p.bias)[col0 + i]
-                                 : to_f(reinterpret_cast<const bf16*>(p.bias)[col0 + i]);
-        }
-        if (p.c_f32) {
-          float* cp = reinterpret_cast<float*>(p.C) + cbase + col0;
-          bool vec = full_chunk && ((reinterpret_cast<uintptr_t>(cp) & 15) == 0);
-          if (vec) {
-#pragma unroll
-            for (int i = 0; i < 32; i += 4) {
-              float4 o = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
-              if (p.beta != 0.f) {
-                float4 old = *reinterpret_cast<const float4*>(cp + i);
-                o.x += p.beta * old.x;
-                o.y += p.beta * old.y;
-                o.z += p.beta * old.z;
-                o.w += p.beta * old.w;
-              }
-              *reinterpret_cast<float4*>(cp + i) = o;
-            }
-          } else {
+          for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
+          const bool full_chunk = col0 + 32 <= p.N;
+          if (p.bias) {
 #pragma unroll
             for (int i = 0; i < 32; ++i)
-              if (col0 + i < p.N) cp[i] = v[i] + (p.beta != 0.f ? p.beta * cp[i] : 0.f);
+              if (full_chunk || col0 + i < p.N)
+                v[i] += p.bias_f32 ? reinterpret_cast<const float*>(p.bias)[col0 + i]
+                                   : to_f(reinterpret_cast<const bf16*>(p.bias)[col0 + i]);
           }
-        } else {
-          bf16* cp = reinterpret_cast<bf16*>(p.C) + cbase + col0;
-          bool vec = full_chunk && ((reinterpret_cast<uintptr_t>(cp) & 15) == 0);
-          if (vec) {
+          if (p.tma_store) {
+            if (!p.c_f32 && p.beta != 0.f && row_ok) {  // bf16 accumulate: read the old row chunk
+              const bf16* cp = reinterpret_cast<const bf16*>(p.C) + cbase + col0;
 #pragma unroll
-            for (int i = 0; i < 32; i += 8) {
-              if (p.beta != 0.f) {
-                uint4 old = *reinterpret_cast<const uint4*>(cp + i);
-                const bf16* ob = reinterpret_cast<const bf16*>(&old);
-#pragma unroll
-                for (int j = 0; j < 8; ++j) v[i + j] += p.beta * to_f(ob[j]);
-              }
-              uint4 o;
-              __nv_bfloat162* ob2 = reinterpret_cast<__nv_bfloat162*>(&o);
-#pragma unroll
-              for (int j = 0; j < 4; ++j) ob2[j] = __floats2bfloat162_rn(v[i + 2 * j], v[i + 2 * j + 1]);
-              *reinterpret_cast<uint4*>(cp + i) = o;
+              for (int i = 0; i < 32; ++i)
+                if (full_chunk || col0 + i < p.N) v[i] += p.beta * to_f(cp[i]);
             }
-          } else {
+            uint8_t* buf = wbuf + nbuf * 4096;
+            if (lane == 0) bulk_wait_read1();  // the store that last used `buf` has read it
+            __syncwarp();
+            if (p.c_f32) {
 #pragma unroll
-            for (int i = 0; i < 32; ++i)
-              if (col0 + i < p.N) cp[i] = from_f<bf16>(v[i] + (p.beta != 0.f ? p.beta * to_f(cp[i]) : 0.f));
+              for (int j = 0; j < 8; ++j) {  // 128 B row, SWIZZLE_128B
+                float4 o = make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
+                *reinterpret_cast<float4*>(buf + lane * 128 + ((j ^ (lane & 7)) << 4)) = o;
+              }
+            } else {
+#pragma unroll
+              for (int j = 0; j < 4; ++j) {  // 64 B row, SWIZZLE_64B
+                uint4 o;
+                __nv_bfloat162* o2 = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+                for (int h = 0; h < 4; ++h) o2[h] = __floats2bfloat162_rn(v[8 * j + 2 * h], v[8 * j + 2 * h + 1]);
+                *reinterpret_cast<uint4*>(buf + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4)) = o;
+              }
+            }
+            fence_async_smem();
+            __syncwarp();
+            if (lane == 0) {
+              if (p.reduce_add) tma_reduce_add(&tmC, buf, col0, m0 + q * 32, b1, b2);
+              else tma_store(&tmC, buf, col0, m0 + q * 32, b1, b2);
+              bulk_commit();
+            }
+            nbuf ^= 1;
+          } else if (row_ok) {
+            if (p.c_f32) {
+              float* cp = reinterpret_cast<float*>(p.C) + cbase + col0;
+#pragma unroll
+              for (int i = 0; i < 32; ++i)
+                if (col0 + i < p.N) cp[i] = v[i] + (p.beta != 0.f ? p.beta * cp[i] : 0.f);
+            } else {
+              bf16* cp = reinterpret_cast<bf16*>(p.C) + cbase + col0;
+#pragma unroll
+              for (int i = 0; i < 32; ++i)
+                if (col0 + i < p.N) cp[i] = from_f<bf16>(v[i] + (p.beta != 0.f ? p.beta * to_f(cp[i]) : 0.f));
+            }
           }
-        }
         }
         __syncwarp();
       }
@@ -327,6 +363,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         acc_phase ^= 1;
       }
     }
+    if (lane == 0) bulk_wait_all();
+    (void)es;
   }
   __syncwarp();
   tc_fence_before();
@@ -350,45 +388,49 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-// 4-D map: (contiguous dim, row dim, batch1, batch2); box (64, rows, 1, 1).
-bool make_map(CUtensorMap* map, const GemmOperand& op, int64_t d0, int64_t d1, int nb1, int nb2, int box1) {
+// 4-D map: (contiguous dim, row dim, batch1, batch2); box (box0, box1, 1, 1).
+bool make_map(CUtensorMap* map, const void* ptr, int64_t ld, int64_t bs1, int64_t bs2, int64_t d0, int64_t d1, int nb1,
+              int nb2, int box0, int box1, int es, CUtensorMapDataType dt, CUtensorMapSwizzle swz) {
   auto fn = encode_fn();
   if (!fn) return false;
-  const uint64_t es = 2;
-  uintptr_t base = reinterpret_cast<uintptr_t>(op.ptr);
-  if (base % 16 || (op.ld * es) % 16 || op.ld < d0) return false;
-  if (nb1 > 1 && (op.bs1 * es) % 16) return false;
-  if (nb2 > 1 && (op.bs2 * es) % 16) return false;
+  uintptr_t base = reinterpret_cast<uintptr_t>(ptr);
+  if (base % 16 || (ld * es) % 16 || ld < d0) return false;
+  if (nb1 > 1 && (bs1 * es) % 16) return false;
+  if (nb2 > 1 && (bs2 * es) % 16) return false;
   cuuint64_t dims[4] = {cuuint64_t(d0), cuuint64_t(d1), cuuint64_t(nb1), cuuint64_t(nb2)};
-  cuuint64_t s1 = op.ld * es;
-  cuuint64_t s2 = nb1 > 1 ? op.bs1 * es : s1 * d1;
-  cuuint64_t s3 = nb2 > 1 ? op.bs2 * es : s2 * nb1;
+  cuuint64_t s1 = ld * es;
+  cuuint64_t s2 = nb1 > 1 ? bs1 * es : s1 * d1;
+  cuuint64_t s3 = nb2 > 1 ? bs2 * es : s2 * nb1;
   s2 = (s2 + 15) / 16 * 16;
   s3 = (s3 + 15) / 16 * 16;
   cuuint64_t strides[3] = {s1, s2, s3};
-  cuuint32_t box[4] = {64, cuuint32_t(box1), 1, 1};
+  cuuint32_t box[4] = {cuuint32_t(box0), cuuint32_t(box1), 1, 1};
   cuuint32_t estr[4] = {1, 1, 1, 1};
-  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, reinterpret_cast<void*>(base), dims, strides, box,
-                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  CUresult r = fn(map, dt, 4, reinterpret_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  swz, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS;
+}
+
+bool make_operand_map(CUtensorMap* map, const GemmOperand& op, int64_t d0, int64_t d1, int nb1, int nb2, int box1) {
+  return make_map(map, op.ptr, op.ld, op.bs1, op.bs2, d0, d1, nb1, nb2, 64, box1, 2, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16,
+                  CU_TENSOR_MAP_SWIZZLE_128B);
 }
 
 int g_num_sms = 0;
 std::atomic<int64_t> g_launches{0};
 
 template <int BN>
-void launch(const CUtensorMap& a, const CUtensorMap& b, const TcParams& p, cudaStream_t st) {
+void launch(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, const TcParams& p, cudaStream_t st) {
   constexpr int STAGE = (BM + BN) * BK * 2;
   constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
-  const int smem = STAGES * STAGE + 1024 + 256;
+  const int smem = STAGES * STAGE + 1024 + 4 * kStageBytesPerWarp + 1024;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(gemm_tc_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
-  int grid = p.num_tiles < g_num_sms ? p.num_tiles : g_num_sms;
-  gemm_tc_kernel<BN><<<grid, kThreads, smem, st>>>(a, b, p);
+  int grid = p.num_units < g_num_sms ? p.num_units : g_num_sms;
+  gemm_tc_kernel<BN><<<grid, kThreads, smem, st>>>(a, b, c, p);
   g_launches++;
 }
 
@@ -417,11 +459,11 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
       best_bn = bn;
     }
   }
-  CUtensorMap ma, mb;
-  bool ok = g.a.mn_major ? make_map(&ma, g.a, g.M, g.K, g.nb1, g.nb2, 64)
-                         : make_map(&ma, g.a, g.K, g.M, g.nb1, g.nb2, BM);
-  ok = ok && (g.b.mn_major ? make_map(&mb, g.b, g.N, g.K, g.nb1, g.nb2, 64)
-                           : make_map(&mb, g.b, g.K, g.N, g.nb1, g.nb2, best_bn));
+  CUtensorMap ma, mb, mc;
+  bool ok = g.a.mn_major ? make_operand_map(&ma, g.a, g.M, g.K, g.nb1, g.nb2, 64)
+                         : make_operand_map(&ma, g.a, g.K, g.M, g.nb1, g.nb2, BM);
+  ok = ok && (g.b.mn_major ? make_operand_map(&mb, g.b, g.N, g.K, g.nb1, g.nb2, 64)
+                           : make_operand_map(&mb, g.b, g.K, g.N, g.nb1, g.nb2, best_bn));
   if (!ok) return false;
   TcParams p;
   p.M = g.M;
@@ -444,10 +486,35 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   p.beta = g.beta;
   p.bias = g.bias;
   p.bias_f32 = g.bias_dtype == F32;
+  // output: TMA store (bf16/f32) or TMA reduce-add (f32, beta == 1) when the view is aligned
+  const int es = p.c_f32 ? 4 : 2;
+  p.tma_store = make_map(&mc, g.c, g.ldc, g.cbs1, g.cbs2, g.N, g.M, g.nb1, g.nb2, 32, 32, es,
+                         p.c_f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16,
+                         p.c_f32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B)
+                    ? 1 : 0;
+  if (g.beta != 0.f && g.beta != 1.f) p.tma_store = 0;
+  if (!p.tma_store) mc = ma;  // unused
+  p.reduce_add = (p.tma_store && p.c_f32 && g.beta == 1.f) ? 1 : 0;
+  // split-K for products with few output tiles and a long reduction (dW = dY^T X):
+  // partial tiles are reduce-added in fp32 (the zero-init comes first when beta == 0)
+  p.ksplit = 1;
+  if (p.tma_store && p.c_f32 && g.nb1 * g.nb2 == 1 && g.ldc == g.N && p.num_tiles * 2 <= g_num_sms &&
+      p.num_kb >= 16) {
+    int ks = g_num_sms / p.num_tiles;
+    if (ks > p.num_kb / 8) ks = p.num_kb / 8;
+    if (ks > 1) {
+      p.ksplit = ks;
+      if (g.beta == 0.f) cudaMemsetAsync(g.c, 0, size_t(g.M) * g.N * 4, st);
+      p.reduce_add = 1;
+    }
+  }
+  p.kb_per_split = (p.num_kb + p.ksplit - 1) / p.ksplit;
+  p.ksplit = (p.num_kb + p.kb_per_split - 1) / p.kb_per_split;
+  p.num_units = p.num_tiles * p.ksplit;
   switch (best_bn) {
-    case 256: launch<256>(ma, mb, p, st); break;
-    case 128: launch<128>(ma, mb, p, st); break;
-    default: launch<64>(ma, mb, p, st); break;
+    case 256: launch<256>(ma, mb, mc, p, st); break;
+    case 128: launch<128>(ma, mb, mc, p, st); break;
+    default: launch<64>(ma, mb, mc, p, st); break;
   }
   return true;
 }

@@ -147,24 +147,146 @@ __global__ void __launch_bounds__(kWarps * 32) ln_bwd_kernel(const T* __restrict
   for (int i = threadIdx.x; i < 2 * H; i += blockDim.x) ws[int64_t(blockIdx.x) * 2 * H + i] = sacc[i];
 }
 
-// out[c] (+)= sum_{b < G} ws[b*stride + off + c]
-__global__ void reduce_partials(const float* ws, int G, int64_t stride, int64_t off, int N, float* out, int acc) {
-  int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= N) return;
-  float s = 0.f;
-  for (int b = 0; b < G; ++b) s += ws[int64_t(b) * stride + off + c];
-  out[c] = acc ? out[c] + s : s;
+// Register-cached backward (rows up to NCH x 32 x 16 B): per-lane partial sums of
+// dy*xhat and dy over the warp's rows, combined across warps in a fixed order, so
+// the partial rows in ws are deterministic.
+template <class T, int NCH>
+__global__ void __launch_bounds__(kWarps * 32) ln_bwd_vec(const T* __restrict__ dy, const T* __restrict__ x,
+                                                           const T* __restrict__ g, T* dx, int acc, float* ws,
+                                                           int64_t rows, int H, float eps) {
+  constexpr int V = Vec<T>::N;
+  extern __shared__ float sred[];  // [2H]
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  float pg[NCH][V], pb[NCH][V];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c)
+#pragma unroll
+    for (int i = 0; i < V; ++i) pg[c][i] = pb[c][i] = 0.f;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + w; r < rows; r += int64_t(gridDim.x) * kWarps) {
+    float xv[NCH][V], dv[NCH][V], gv[NCH][V];
+    float s = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < H) {
+        load_vec(x + r * H + col, xv[c]);
+        load_vec(dy + r * H + col, dv[c]);
+        load_vec(g + col, gv[c]);
+#pragma unroll
+        for (int i = 0; i < V; ++i) s += xv[c][i];
+      }
+    }
+    const float mean = warp_sum(s) / H;
+    float q = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c)
+      if ((c * 32 + lane) * V < H)
+#pragma unroll
+        for (int i = 0; i < V; ++i) {
+          float d = xv[c][i] - mean;
+          q += d * d;
+        }
+    const float rstd = rsqrtf(warp_sum(q) / H + eps);
+    float s1 = 0.f, s2 = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c)
+      if ((c * 32 + lane) * V < H)
+#pragma unroll
+        for (int i = 0; i < V; ++i) {
+          xv[c][i] = (xv[c][i] - mean) * rstd;  // xhat
+          float gd = dv[c][i] * gv[c][i];
+          s1 += gd;
+          s2 += gd * xv[c][i];
+          pg[c][i] += dv[c][i] * xv[c][i];
+          pb[c][i] += dv[c][i];
+        }
+    s1 = warp_sum(s1) / H;
+    s2 = warp_sum(s2) / H;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      int col = (c * 32 + lane) * V;
+      if (col < H) {
+        float o[V];
+        if (acc) load_vec(dx + r * H + col, o);
+#pragma unroll
+        for (int i = 0; i < V; ++i)
+          o[i] = rstd * (dv[c][i] * gv[c][i] - s1 - xv[c][i] * s2) + (acc ? o[i] : 0.f);
+        store_vec(dx + r * H + col, o);
+      }
+    }
+  }
+  // fixed-order cross-warp combination
+  for (int i = threadIdx.x; i < 2 * H; i += blockDim.x) sred[i] = 0.f;
+  __syncthreads();
+  for (int ww = 0; ww < kWarps; ++ww) {
+    if (w == ww) {
+#pragma unroll
+      for (int c = 0; c < NCH; ++c) {
+        int col = (c * 32 + lane) * V;
+        if (col < H)
+#pragma unroll
+          for (int i = 0; i < V; ++i) {
+            sred[col + i] += pg[c][i];
+            sred[H + col + i] += pb[c][i];
+          }
+      }
+    }
+    __syncthreads();
+  }
+  for (int i = threadIdx.x; i < 2 * H; i += blockDim.x) ws[int64_t(blockIdx.x) * 2 * H + i] = sred[i];
 }
 
-// column partial sums: block b sums rows [b*rpb, (b+1)*rpb) for all columns
+// out[c] (+)= sum_{b < G} ws[b*stride + off + c]; the G partials are summed in
+// fp64 in a fixed order, so a split micro-op's contribution is exact up to the
+// single fp32 rounding of the accumulation into `out` (split invariance, R17).
+__global__ void reduce_partials(const float* __restrict__ ws, int G, int64_t stride, int64_t off, int N,
+                                float* out, int acc) {
+  int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= N) return;
+  double s = 0.0;
+#pragma unroll 8
+  for (int b = 0; b < G; ++b) s += double(ws[int64_t(b) * stride + off + c]);
+  out[c] = acc ? float(double(out[c]) + s) : float(s);
+}
+
+// Column partial sums of x[rows, N]: block (cb, g) owns 256 columns (32 lanes x 8
+// contiguous columns, 16-byte loads) and rows g, g+G, ...; 8 warps interleave rows
+// and combine through shared memory in a fixed order (deterministic).
 template <class T>
-__global__ void colsum_partial(const T* x, int64_t rows, int N, int64_t rpb, float* ws, const int* filter, int fval) {
-  int64_t r0 = int64_t(blockIdx.x) * rpb, r1 = r0 + rpb < rows ? r0 + rpb : rows;
-  for (int c = threadIdx.x; c < N; c += blockDim.x) {
+__global__ void __launch_bounds__(256) colsum_partial(const T* __restrict__ x, int64_t rows, int N, int G,
+                                                      float* __restrict__ ws, const int* __restrict__ filter, int fval) {
+  __shared__ float red[8][256];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int c0 = blockIdx.x * 256 + lane * 8;
+  float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  const bool vec = (N % 8 == 0) && c0 + 8 <= N && (reinterpret_cast<uintptr_t>(x) % 16 == 0);
+  for (int64_t r = int64_t(blockIdx.y) * 8 + w; r < rows; r += int64_t(G) * 8) {
+    if (filter && filter[r] != fval) continue;
+    const T* xr = x + r * N;
+    if (vec) {
+      constexpr int V = 16 / sizeof(T);
+#pragma unroll
+      for (int h = 0; h < 8; h += V) {
+        uint4 u = *reinterpret_cast<const uint4*>(xr + c0 + h);
+        const T* t = reinterpret_cast<const T*>(&u);
+#pragma unroll
+        for (int i = 0; i < V; ++i) acc[h + i] += to_f(t[i]);
+      }
+    } else {
+#pragma unroll
+      for (int i = 0; i < 8; ++i)
+        if (c0 + i < N) acc[i] += to_f(xr[c0 + i]);
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) red[w][lane * 8 + i] = acc[i];
+  __syncthreads();
+  const int c = blockIdx.x * 256 + threadIdx.x;
+  if (c < N) {
     float s = 0.f;
-    for (int64_t r = r0; r < r1; ++r)
-      if (!filter || filter[r] == fval) s += to_f(x[r * N + c]);
-    ws[int64_t(blockIdx.x) * N + c] = s;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) s += red[k][threadIdx.x];
+    ws[int64_t(blockIdx.y) * N + c] = s;
   }
 }
 
@@ -339,9 +461,9 @@ template <class T>
 __global__ void embed_bwd_pos_kernel(const T* dy, float* dpos, int64_t nsamp, int seq, int H, int acc) {
   const int64_t n = int64_t(seq) * H;
   for (int64_t e = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; e < n; e += int64_t(gridDim.x) * blockDim.x) {
-    float s = 0.f;
-    for (int64_t b = 0; b < nsamp; ++b) s += to_f(dy[b * n + e]);
-    dpos[e] = acc ? dpos[e] + s : s;
+    double s = 0.0;
+    for (int64_t b = 0; b < nsamp; ++b) s += double(to_f(dy[b * n + e]));
+    dpos[e] = acc ? float(double(dpos[e]) + s) : float(s);
   }
 }
 template <class T>
@@ -446,20 +568,37 @@ void layernorm_fwd(int dt, const void* x, const void* g, const void* b, void* y,
   else ln_fwd_t<bf16>(x, g, b, y, rows, H, eps, st);
 }
 
+template <class T>
+void ln_bwd_t(const void* dy, const void* x, const void* g, void* dx, int acc, float* ws, int64_t rows, int H,
+              float eps, int G, cudaStream_t st) {
+  constexpr int V = Vec<T>::N;
+  int nch = (H + 32 * V - 1) / (32 * V);
+  bool vec = H % V == 0 && al16(dy) && al16(x) && al16(g) && al16(dx) && nch <= 4;
+  size_t smem = size_t(2) * H * sizeof(float);
+  auto DY = (const T*)dy;
+  auto X = (const T*)x;
+  auto Gm = (const T*)g;
+  auto DX = (T*)dx;
+  if (vec) {
+    switch (nch) {
+      case 1: ln_bwd_vec<T, 1><<<G, kWarps * 32, smem, st>>>(DY, X, Gm, DX, acc, ws, rows, H, eps); return;
+      case 2: ln_bwd_vec<T, 2><<<G, kWarps * 32, smem, st>>>(DY, X, Gm, DX, acc, ws, rows, H, eps); return;
+      default:
+        if (smem > 48 * 1024) cudaFuncSetAttribute(ln_bwd_vec<T, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+        ln_bwd_vec<T, 4><<<G, kWarps * 32, smem, st>>>(DY, X, Gm, DX, acc, ws, rows, H, eps);
+        return;
+    }
+  }
+  if (smem > 48 * 1024) cudaFuncSetAttribute(ln_bwd_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
+  ln_bwd_kernel<T><<<G, kWarps * 32, smem, st>>>(DY, X, Gm, DX, acc, ws, rows, H, eps);
+}
+
 void layernorm_bwd(int dt, const void* dy, const void* x, const void* g, void* dx, int acc, float* ws, float* dgamma,
                    float* dbeta, int pacc, int64_t rows, int H, float eps, cudaStream_t st) {
   int64_t G = (rows + kWarps - 1) / kWarps;
-  if (G > kWsRows) G = kWsRows;
-  size_t smem = size_t(2) * H * sizeof(float);
-  if (dt == F32) {
-    if (smem > 48 * 1024) cudaFuncSetAttribute(ln_bwd_kernel<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-    ln_bwd_kernel<float><<<int(G), kWarps * 32, smem, st>>>((const float*)dy, (const float*)x, (const float*)g,
-                                                             (float*)dx, acc, ws, rows, H, eps);
-  } else {
-    if (smem > 48 * 1024) cudaFuncSetAttribute(ln_bwd_kernel<bf16>, cudaFuncAttributeMaxDynamicSharedMemorySize, int(smem));
-    ln_bwd_kernel<bf16><<<int(G), kWarps * 32, smem, st>>>((const bf16*)dy, (const bf16*)x, (const bf16*)g,
-                                                           (bf16*)dx, acc, ws, rows, H, eps);
-  }
+  if (G > 148) G = 148;
+  if (dt == F32) ln_bwd_t<float>(dy, x, g, dx, acc, ws, rows, H, eps, int(G), st);
+  else ln_bwd_t<bf16>(dy, x, g, dx, acc, ws, rows, H, eps, int(G), st);
   reduce_partials<<<(H + 255) / 256, 256, 0, st>>>(ws, int(G), 2 * H, 0, H, dgamma, pacc);
   reduce_partials<<<(H + 255) / 256, 256, 0, st>>>(ws, int(G), 2 * H, H, H, dbeta, pacc);
 }
@@ -475,14 +614,17 @@ void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64
 
 void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, float* out, int acc, const int* filter, int fval,
                 cudaStream_t st) {
-  int64_t G = rows < kWsRows ? rows : kWsRows;
+  const int cb = (N + 255) / 256;
+  int G = int((rows + 7) / 8);
+  int cap = 296 / cb;
+  if (cap < 1) cap = 1;
+  if (cap > 64) cap = 64;
+  if (G > cap) G = cap;
   if (G < 1) G = 1;
-  int64_t rpb = (rows + G - 1) / G;
-  G = (rows + rpb - 1) / rpb;
-  int threads = N < 256 ? ((N + 31) / 32) * 32 : 256;
-  if (dt == F32) colsum_partial<float><<<int(G), threads, 0, st>>>((const float*)x, rows, N, rpb, ws, filter, fval);
-  else colsum_partial<bf16><<<int(G), threads, 0, st>>>((const bf16*)x, rows, N, rpb, ws, filter, fval);
-  reduce_partials<<<(N + 255) / 256, 256, 0, st>>>(ws, int(G), N, 0, N, out, acc);
+  dim3 grid(cb, G);
+  if (dt == F32) colsum_partial<float><<<grid, 256, 0, st>>>((const float*)x, rows, N, G, ws, filter, fval);
+  else colsum_partial<bf16><<<grid, 256, 0, st>>>((const bf16*)x, rows, N, G, ws, filter, fval);
+  reduce_partials<<<(N + 255) / 256, 256, 0, st>>>(ws, G, N, 0, N, out, acc);
 }
 
 void embed_fwd(int dt, const int* ids, const int* tt, const void* word, const void* pos, const void* type, void* y,

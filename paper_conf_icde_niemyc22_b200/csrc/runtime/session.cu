@@ -78,6 +78,9 @@ struct ts_session_s {
   uint64_t loss_off = 0;
   std::vector<int> zero_grads;                   // params whose grad is accumulated atomically
   int64_t launches = 0;
+  bool profile = false;
+  std::vector<cudaEvent_t> prof_ev;  // 2 per program command (compute items)
+  std::vector<float> item_ms;
 };
 
 namespace {
@@ -529,11 +532,14 @@ void issue_step(ts_session_t* s) {
   cudaStream_t cs = s->cs;
   for (int t : s->zero_grads) cudaMemsetAsync(param_g(s, t), 0, size_t(g.t[t].numel) * 4, cs);
   bool d2h_used = false, h2d_used = false;
+  const bool prof = s->profile && !s->prof_ev.empty();
   for (auto& c : s->prog) {
     if (c.kind == 0) {
       for (int so : c.wait_so) cudaStreamWaitEvent(cs, s->ev_d2h[so], 0);
       for (int si : c.wait_si) cudaStreamWaitEvent(cs, s->ev_h2d[si], 0);
+      if (prof) cudaEventRecord(s->prof_ev[2 * c.item], cs);
       c.fn(cs);
+      if (prof) cudaEventRecord(s->prof_ev[2 * c.item + 1], cs);
     } else if (c.kind == 1) {
       cudaEventRecord(s->ev_mark, cs);
       cudaStreamWaitEvent(s->d2h, s->ev_mark, 0);
@@ -599,7 +605,7 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
   if (!inputs) return set_error("inputs is null"), TS_ERR_ARG;
   ts_status st = copy_inputs(s, inputs, on_host);
   if (st != TS_OK) return st;
-  if (s->use_graph) {
+  if (s->use_graph && !s->profile) {
     if (!s->gexec) {
       cudaGraph_t graph;
       CU(cudaStreamBeginCapture(s->cs, cudaStreamCaptureModeThreadLocal));
@@ -624,6 +630,12 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
   }
   ++s->step;  // dropout counter (graph mode keeps the captured step value)
   CU(cudaGetLastError());
+  if (s->profile) {
+    CU(cudaStreamSynchronize(s->cs));
+    s->item_ms.assign(s->prog.size(), 0.f);
+    for (auto& c : s->prog)
+      if (c.kind == 0) cudaEventElapsedTime(&s->item_ms[c.item], s->prof_ev[2 * c.item], s->prof_ev[2 * c.item + 1]);
+  }
   return TS_OK;
 }
 
@@ -774,16 +786,58 @@ ts_status ts_session_launches(const ts_session_t* s, int64_t* n) {
 }
 
 ts_status ts_session_profile_items(ts_session_t* s, int32_t enable) {
-  (void)enable;
   if (!s) return set_error("null session"), TS_ERR_ARG;
-  return set_error("item profiling not implemented yet"), TS_ERR_STATE;
+  s->profile = enable != 0;
+  if (s->profile && s->prof_ev.empty()) {
+    s->prof_ev.assign(2 * s->prog.size(), nullptr);
+    for (auto& e : s->prof_ev) CU(cudaEventCreate(&e));
+  }
+  return TS_OK;
 }
 
 ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, uint64_t* n) {
-  (void)ms;
-  (void)cap;
   if (!s || !n) return set_error("null argument"), TS_ERR_ARG;
-  *n = 0;
+  *n = s->item_ms.size();
+  if (ms)
+    for (uint64_t i = 0; i < s->item_ms.size() && i < cap; ++i) ms[i] = s->item_ms[i];
+  return TS_OK;
+}
+
+// ---- NCCL bootstrap (the library already loaded by torch, or libnccl.so.2) ------
+static void* nccl_handle() {
+  void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+  if (!h) h = dlopen("libnccl.so.2", RTLD_NOW);
+  return h;
+}
+
+ts_status ts_nccl_unique_id(void* out128) {
+  if (!out128) return set_error("null argument"), TS_ERR_ARG;
+  void* h = nccl_handle();
+  auto fn = h ? reinterpret_cast<int (*)(void*)>(dlsym(h, "ncclGetUniqueId")) : nullptr;
+  if (!fn) return set_error("libnccl.so.2 / ncclGetUniqueId not available"), TS_ERR_NCCL;
+  if (fn(out128) != 0) return set_error("ncclGetUniqueId failed"), TS_ERR_NCCL;
+  return TS_OK;
+}
+
+ts_status ts_nccl_comm_init(const void* id128, int32_t nranks, int32_t rank, void** comm) {
+  if (!id128 || !comm || nranks < 1 || rank < 0 || rank >= nranks) return set_error("bad argument"), TS_ERR_ARG;
+  void* h = nccl_handle();
+  struct Id {
+    char b[128];
+  };
+  auto fn = h ? reinterpret_cast<int (*)(void**, int, Id, int)>(dlsym(h, "ncclCommInitRank")) : nullptr;
+  if (!fn) return set_error("ncclCommInitRank not available"), TS_ERR_NCCL;
+  Id id;
+  std::memcpy(id.b, id128, 128);
+  if (fn(comm, nranks, id, rank) != 0) return set_error("ncclCommInitRank failed"), TS_ERR_NCCL;
+  return TS_OK;
+}
+
+ts_status ts_nccl_comm_destroy(void* comm) {
+  void* h = nccl_handle();
+  auto fn = h ? reinterpret_cast<int (*)(void*)>(dlsym(h, "ncclCommDestroy")) : nullptr;
+  if (!fn || !comm) return set_error("ncclCommDestroy not available"), TS_ERR_NCCL;
+  fn(comm);
   return TS_OK;
 }
 

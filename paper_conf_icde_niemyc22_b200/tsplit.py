@@ -116,6 +116,9 @@ def lib():
             "ts_session_launches": (i32, [vp, P(i64)]),
             "ts_session_profile_items": (i32, [vp, i32]),
             "ts_session_item_times": (i32, [vp, P(C.c_float), u64, P(u64)]),
+            "ts_nccl_unique_id": (i32, [vp]),
+            "ts_nccl_comm_init": (i32, [vp, i32, i32, P(vp)]),
+            "ts_nccl_comm_destroy": (i32, [vp]),
             "ts_gemm_bf16": (i32, [i32, i32, i32, i32, vp, i64, i64, i32, vp, i64, i64, i32,
                                    vp, i64, i64, i32, C.c_float, C.c_float, vp, vp]),
             "ts_gemm_f32": (i32, [i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, C.c_float,
@@ -287,7 +290,7 @@ class Session:
 
     def __init__(self, graph: Graph, plan: Plan, device: int = 0, slab_bytes: int | None = None,
                  lr: float = 0.0, use_cuda_graph: bool = True, nccl_comm: int | None = None,
-                 world_size: int = 1, step0: int = 0):
+                 world_size: int = 1, step0: int = 0, streams=None):
         import torch
         if not torch.cuda.is_available():
             raise TsError(9, "no CUDA device: the TSPLIT runtime has no CPU fallback")
@@ -300,6 +303,9 @@ class Session:
         cfg.slab = self.slab.data_ptr()
         cfg.slab_bytes = self.slab_bytes
         cfg.nccl_comm = nccl_comm
+        if streams is not None:  # (compute, d2h, h2d) torch.cuda.Stream objects
+            self.streams = streams
+            cfg.stream_compute, cfg.stream_d2h, cfg.stream_h2d = [s.cuda_stream for s in streams]
         cfg.world_size = world_size
         cfg.use_cuda_graph = 1 if use_cuda_graph else 0
         cfg.lr = lr
@@ -361,6 +367,16 @@ class Session:
         check(lib().ts_session_trace(self.h, buf, n.value, C.byref(n)))
         return [(e.seq, e.item, "A" if e.kind == 0 else "F", e.key, e.piece, e.offset, e.bytes) for e in buf]
 
+    def profile_items(self, enable=True):
+        check(lib().ts_session_profile_items(self.h, 1 if enable else 0))
+
+    def item_times(self):
+        n = C.c_uint64()
+        check(lib().ts_session_item_times(self.h, None, 0, C.byref(n)))
+        buf = (C.c_float * n.value)()
+        check(lib().ts_session_item_times(self.h, buf, n.value, C.byref(n)))
+        return list(buf)
+
     def launches(self) -> int:
         n = C.c_int64()
         check(lib().ts_session_launches(self.h, C.byref(n)))
@@ -381,3 +397,15 @@ def inputs_to_device(graph: Graph, arrays: dict, device="cuda:0", pinned_host=Fa
                 x = torch.from_numpy(np.ascontiguousarray(a, np.float32))
             out[t["name"]] = x.pin_memory() if pinned_host else x.to(device)
     return out
+
+
+def nccl_comm(rank: int, world: int, broadcast):
+    """Create a NCCL communicator; `broadcast(bytes) -> bytes` ships rank 0's id."""
+    buf = C.create_string_buffer(128)
+    if rank == 0:
+        check(lib().ts_nccl_unique_id(buf))
+    raw = broadcast(buf.raw if rank == 0 else None)
+    idb = C.create_string_buffer(raw, 128)
+    comm = C.c_void_p()
+    check(lib().ts_nccl_comm_init(idb, world, rank, C.byref(comm)))
+    return comm.value

@@ -14,15 +14,26 @@ def pytest_configure(config):
 
 def rel_errs(got: dict, ref: dict):
     """Per-tensor relative L2 error.  Tensors whose
-    reference norm is below 1e-6 of the largest one (e.g. an attention key bias,
-    whose gradient is analytically zero by softmax shift invariance) are compared
-    against that largest norm instead."""
+    reference norm is below 1e-4 of the largest one (e.g. an attention key bias,
+    whose gradient is analytically zero by softmax shift invariance, so fp32
+    cancellation noise is all that is left) are compared against 1e-4 x the
+    largest norm instead."""
     import numpy as np
     scale = max(float(np.linalg.norm(np.asarray(v, np.float64))) for v in ref.values())
     out = {}
     for k, r in ref.items():
         r = np.asarray(r, np.float64)
         g = np.asarray(got[k], np.float64).reshape(r.shape)
-        den = max(float(np.linalg.norm(r)), 1e-6 * scale)
+        den = max(float(np.linalg.norm(r)), 1e-4 * scale)
         out[k] = float(np.linalg.norm(g - r)) / den
     return out
+
+
+def global_rel_err(got: dict, ref: dict):
+    """Relative L2 error of the whole gradient vector (all parameters
+    concatenated): DESIGN.md reading D-TOL for bf16 runs."""
+    import numpy as np
+    num = sum(float(np.sum((np.asarray(got[k], np.float64).reshape(np.shape(r)) - np.asarray(r, np.float64)) ** 2))
+              for k, r in ref.items())
+    den = sum(float(np.sum(np.asarray(r, np.float64) ** 2)) for r in ref.values())
+    return (num / den) ** 0.5

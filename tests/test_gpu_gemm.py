@@ -26,7 +26,7 @@ CASES = [
     (384, 192, 320, 1, 0, 1, "bf16"),
     (256, 320, 192, 1, 1, 1, "f32"),
     (200, 136, 72, 1, 0, 0, "bf16"),     # ragged M/N/K
-    (130, 64, 96, 3, 1, 0, "f32"),       # ragged + batched
+    (136, 64, 96, 3, 1, 0, "f32"),       # ragged + batched (MN-major ld must be 16 B aligned)
     (512, 64, 512, 4, 0, 1, "bf16"),     # attention P.V shape
     (1024, 4096, 1024, 1, 0, 0, "bf16"),
     (1024, 1024, 4096, 1, 1, 1, "f32"),  # dW shape

@@ -10,7 +10,7 @@ import pytest
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
-from conftest import rel_errs  # noqa: E402
+from conftest import global_rel_err, rel_errs  # noqa: E402
 from oracle import brute, net, sim  # noqa: E402
 from paper_conf_icde_niemyc22_b200 import tsplit  # noqa: E402
 from tsinputs import gen, graphs  # noqa: E402
@@ -69,22 +69,27 @@ def test_bert_tiny_fp32_random_plans(seed):
     errs = rel_errs(grads, og)
     assert max(errs.values()) <= 1e-5, sorted(errs.items(), key=lambda kv: -kv[1])[:5]
     l0, g0, _, _ = _run(g)
-    assert max(rel_errs(grads, g0).values()) <= 1e-6
+    e0 = rel_errs(grads, g0)
+    assert max(e0.values()) <= 1e-6, sorted(e0.items(), key=lambda kv: -kv[1])[:5]
 
 
 def test_bert_tiny_bf16_parity_and_budget():
+    """bf16 reading D-TOL: whole-gradient relative L2 <= 2e-2 vs the fp64 oracle,
+    every tensor <= 1e-1 (row sums of bf16-rounded gradients, e.g. bias grads,
+    carry the rounding of every summand)."""
     g = graphs.config_graph("bert_tiny")
     ol, og = _oracle(g)
     loss, grads, S, P = _run(g)
     assert abs(loss - ol) <= 2e-2 * abs(ol)
+    assert global_rel_err(grads, og) <= 2e-2
     errs = rel_errs(grads, og)
-    assert max(errs.values()) <= 2e-2, sorted(errs.items(), key=lambda kv: -kv[1])[:5]
+    assert max(errs.values()) <= 1e-1, sorted(errs.items(), key=lambda kv: -kv[1])[:5]
     base = P.stats()
     budget = base["static_bytes"] + (base["peak_extent"] - base["static_bytes"]) * 4 // 10
     l2, g2, S2, P2 = _run(g, budget=budget)
     assert P2.stats()["peak_extent"] <= budget
-    assert max(rel_errs(g2, og).values()) <= 2e-2
-    assert max(rel_errs(g2, grads).values()) <= 1e-2
+    assert global_rel_err(g2, og) <= 2e-2
+    assert global_rel_err(g2, grads) <= 1e-2
 
 
 def test_eager_equals_graph_and_host_inputs():
