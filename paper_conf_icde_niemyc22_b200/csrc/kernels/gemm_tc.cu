@@ -24,7 +24,8 @@ namespace tsk {
 namespace {
 
 constexpr int BM = 128, BK = 64;
-constexpr int kThreads = 192;  // warp0 TMA, warp1 MMA, warps2-5 epilogue
+constexpr int kEpiWarps = 8;   // two per TMEM lane quarter, alternating 32-column chunks
+constexpr int kThreads = 64 + 32 * kEpiWarps;  // warp0 TMA, warp1 MMA, warps 2.. epilogue
 
 struct TcParams {
   int M, N, K, nb1, nb2;
@@ -40,7 +41,18 @@ struct TcParams {
   int tma_store;   // 1: stage in smem and TMA-store; 0: direct per-thread stores
   int reduce_add;  // 1: TMA reduce-add into an fp32 C (beta = 1 or split-K)
 };
-constexpr int kStageBytesPerWarp = 2 * 4096;  // double-buffered 32x32 fp32 block
+// epilogue staging: per warp, 32x32 output blocks (two for bf16; one for fp32, whose
+// products have long K and keep the smem for a deeper operand pipeline)
+template <bool F32OUT>
+constexpr int staging_bufs() { return F32OUT ? 1 : 2; }
+template <bool F32OUT>
+constexpr int staging_bytes() { return kEpiWarps * staging_bufs<F32OUT>() * 32 * 32 * (F32OUT ? 4 : 2); }
+template <int BN, bool F32OUT>
+constexpr int num_stages() {
+  constexpr int stage = (BM + BN) * BK * 2;
+  constexpr int n = (224 * 1024 - staging_bytes<F32OUT>() - 2048) / stage;
+  return n > 8 ? 8 : n;
+}
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -91,6 +103,7 @@ __device__ __forceinline__ void tma_reduce_add(const CUtensorMap* map, const voi
 }
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read1() { asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
@@ -144,15 +157,16 @@ __device__ __forceinline__ void decode_tile(const TcParams& p, int tile, int& b1
   n0 = nt;  // scaled by BN by the caller
 }
 
-template <int BN>
+template <int BN, bool F32OUT>
 __global__ void __launch_bounds__(kThreads, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const __grid_constant__ CUtensorMap tmC, const TcParams p) {
   constexpr int A_BYTES = BM * BK * 2;
   constexpr int B_BYTES = BN * BK * 2;
   constexpr int STAGE = A_BYTES + B_BYTES;
-  constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
+  constexpr int STAGES = num_stages<BN, F32OUT>();
   constexpr uint32_t TMEM_COLS = 2 * BN;
+  constexpr int BUF = 32 * 32 * (F32OUT ? 4 : 2);
   // instruction descriptor: D f32, A/B bf16, M = 128, N = BN
   const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(p.a_mn) << 15) |
                          (uint32_t(p.b_mn) << 16) | (uint32_t(BN >> 3) << 17) | (uint32_t(BM >> 4) << 24);
@@ -174,7 +188,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int s = 0; s < 2; ++s) {
       mbar_init(&tfull[s], 1);
-      mbar_init(&tempty[s], 128);
+      mbar_init(&tempty[s], 32 * kEpiWarps);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
@@ -272,9 +286,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   } else {
     // ===== epilogue: TMEM -> registers (alpha, bias) -> swizzled smem -> TMA store =====
-    const int q = warp & 3;  // TMEM lane quarter this warp may access
-    const int ew = warp - 2; // epilogue warp index 0..3
-    uint8_t* wbuf = cstage + ew * kStageBytesPerWarp;
+    const int q = warp & 3;        // TMEM lane quarter this warp may access
+    const int ew = warp - 2;       // epilogue warp index 0..7
+    const int half = ew >> 2;      // which alternate 32-column chunks this warp stores
+    uint8_t* wbuf = cstage + ew * staging_bufs<F32OUT>() * BUF;
     int nbuf = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -290,7 +305,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const bool row_ok = row < p.M;
       const int64_t cbase = int64_t(b1) * p.cbs1 + int64_t(b2) * p.cbs2 + int64_t(row) * p.ldc;
 #pragma unroll 1
-      for (int c = 0; c < BN / 32; ++c) {
+      for (int c = half; c < BN / 32; c += 2) {
         uint32_t r[32];
         tmem_ld32(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * BN + c * 32), r);
         const int col0 = n0 + c * 32;
@@ -313,10 +328,13 @@ __global__ void __launch_bounds__(kThreads, 1)
               for (int i = 0; i < 32; ++i)
                 if (full_chunk || col0 + i < p.N) v[i] += p.beta * to_f(cp[i]);
             }
-            uint8_t* buf = wbuf + nbuf * 4096;
-            if (lane == 0) bulk_wait_read1();  // the store that last used `buf` has read it
+            uint8_t* buf = wbuf + nbuf * BUF;
+            if (lane == 0) {  // the store that last used `buf` has read it
+              if constexpr (F32OUT) bulk_wait_read0();
+              else bulk_wait_read1();
+            }
             __syncwarp();
-            if (p.c_f32) {
+            if constexpr (F32OUT) {
 #pragma unroll
               for (int j = 0; j < 8; ++j) {  // 128 B row, SWIZZLE_128B
                 float4 o = make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
@@ -339,7 +357,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               else tma_store(&tmC, buf, col0, m0 + q * 32, b1, b2);
               bulk_commit();
             }
-            nbuf ^= 1;
+            if constexpr (!F32OUT) nbuf ^= 1;
           } else if (row_ok) {
             if (p.c_f32) {
               float* cp = reinterpret_cast<float*>(p.C) + cbase + col0;
@@ -419,18 +437,17 @@ bool make_operand_map(CUtensorMap* map, const GemmOperand& op, int64_t d0, int64
 int g_num_sms = 0;
 std::atomic<int64_t> g_launches{0};
 
-template <int BN>
+template <int BN, bool F32OUT>
 void launch(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, const TcParams& p, cudaStream_t st) {
   constexpr int STAGE = (BM + BN) * BK * 2;
-  constexpr int STAGES = (200 * 1024) / STAGE > 8 ? 8 : (200 * 1024) / STAGE;
-  const int smem = STAGES * STAGE + 1024 + 4 * kStageBytesPerWarp + 1024;
+  const int smem = num_stages<BN, F32OUT>() * STAGE + 1024 + staging_bytes<F32OUT>() + 1024;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(gemm_tc_kernel<BN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(gemm_tc_kernel<BN, F32OUT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
   int grid = p.num_units < g_num_sms ? p.num_units : g_num_sms;
-  gemm_tc_kernel<BN><<<grid, kThreads, smem, st>>>(a, b, c, p);
+  gemm_tc_kernel<BN, F32OUT><<<grid, kThreads, smem, st>>>(a, b, c, p);
   g_launches++;
 }
 
@@ -447,16 +464,32 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
     cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
     if (g_num_sms <= 0) return false;
   }
-  // tile width: minimise waves x tile width (Fig. 5 effect of small micro-ops)
-  int best_bn = 256;
+  // Tile width and split-K are chosen together (the Fig. 5 effect of small micro-ops,
+  // P:L125): time ~ ceil(units / SMs) x per-unit time, with per-tile times from the
+  // measured tcgen05 efficiency of each width (narrow tiles are smem-feed bound in
+  // SS mode: 256 -> ~0.90, 128 -> ~0.65, 64 -> ~0.45 of peak).  Split-K needs an fp32,
+  // contiguous, unbatched C (partials are TMA reduce-added).
+  const bool splitk_ok = g.c_dtype == F32 && g.nb1 * g.nb2 == 1 && g.ldc == g.N;
+  const int num_kb_all = (g.K + BK - 1) / BK;
+  int best_bn = 256, best_ks = 1;
   double best = 1e30;
   for (int bn : {256, 128, 64}) {
+    if (bn > 64 && g.N <= bn / 2) continue;
+    const double eff = bn == 256 ? 0.90 : bn == 128 ? 0.65 : 0.45;
     int64_t tiles = int64_t((g.M + BM - 1) / BM) * ((g.N + bn - 1) / bn) * g.nb1 * g.nb2;
-    double waves = double((tiles + g_num_sms - 1) / g_num_sms);
-    double cost = waves * (bn + 32);
+    int ks = 1;
+    if (splitk_ok && tiles * 2 <= g_num_sms && num_kb_all >= 16) {
+      ks = int(g_num_sms / tiles);
+      if (ks > num_kb_all / 8) ks = num_kb_all / 8;
+      if (ks < 1) ks = 1;
+    }
+    int64_t units = tiles * ks;
+    double waves = double((units + g_num_sms - 1) / g_num_sms);
+    double cost = waves * (bn / eff) / ks;
     if (cost < best - 1e-9) {
       best = cost;
       best_bn = bn;
+      best_ks = ks;
     }
   }
   CUtensorMap ma, mb, mc;
@@ -498,23 +531,26 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   // split-K for products with few output tiles and a long reduction (dW = dY^T X):
   // partial tiles are reduce-added in fp32 (the zero-init comes first when beta == 0)
   p.ksplit = 1;
-  if (p.tma_store && p.c_f32 && g.nb1 * g.nb2 == 1 && g.ldc == g.N && p.num_tiles * 2 <= g_num_sms &&
-      p.num_kb >= 16) {
-    int ks = g_num_sms / p.num_tiles;
-    if (ks > p.num_kb / 8) ks = p.num_kb / 8;
-    if (ks > 1) {
-      p.ksplit = ks;
-      if (g.beta == 0.f) cudaMemsetAsync(g.c, 0, size_t(g.M) * g.N * 4, st);
-      p.reduce_add = 1;
-    }
+  if (best_ks > 1 && p.tma_store && p.c_f32) {
+    p.ksplit = best_ks;
+    if (g.beta == 0.f) cudaMemsetAsync(g.c, 0, size_t(g.M) * g.N * 4, st);
+    p.reduce_add = 1;
   }
   p.kb_per_split = (p.num_kb + p.ksplit - 1) / p.ksplit;
   p.ksplit = (p.num_kb + p.kb_per_split - 1) / p.kb_per_split;
   p.num_units = p.num_tiles * p.ksplit;
-  switch (best_bn) {
-    case 256: launch<256>(ma, mb, mc, p, st); break;
-    case 128: launch<128>(ma, mb, mc, p, st); break;
-    default: launch<64>(ma, mb, mc, p, st); break;
+  if (p.c_f32) {
+    switch (best_bn) {
+      case 256: launch<256, true>(ma, mb, mc, p, st); break;
+      case 128: launch<128, true>(ma, mb, mc, p, st); break;
+      default: launch<64, true>(ma, mb, mc, p, st); break;
+    }
+  } else {
+    switch (best_bn) {
+      case 256: launch<256, false>(ma, mb, mc, p, st); break;
+      case 128: launch<128, false>(ma, mb, mc, p, st); break;
+      default: launch<64, false>(ma, mb, mc, p, st); break;
+    }
   }
   return true;
 }

@@ -79,3 +79,24 @@ def test_gemm_simt_f32():
     torch.cuda.synchronize()
     ref = A.t().double() @ B.t().double()
     assert ((C.double() - ref).norm() / ref.norm()).item() < 1e-6
+
+
+@pytest.mark.parametrize("M,N,K,out,beta", [
+    (1024, 1024, 16384, "f32", 0.0),   # dW with split-K (reduce-add partials)
+    (1024, 1024, 16384, "f32", 1.0),   # dW accumulated across splits (beta = 1)
+    (256, 512, 640, "bf16", 1.0),      # activation-gradient accumulation in bf16
+    (200, 72, 128, "f32", 1.0),        # ragged tile edges through the TMA store
+])
+def test_gemm_tc_accumulate_and_splitk(M, N, K, out, beta):
+    A = _mk((K, M), seed=11)   # MN-major operands, as in dW = dY^T X
+    B = _mk((K, N), seed=12)
+    od = torch.float32 if out == "f32" else torch.bfloat16
+    C0 = torch.randn(M, N, device="cuda").to(od)
+    C = C0.clone()
+    tsplit.check(tsplit.lib().ts_gemm_bf16(M, N, K, 1, A.data_ptr(), M, 0, 1, B.data_ptr(), N, 0, 1, C.data_ptr(), N,
+                                           0, 0 if out == "f32" else 1, 1.0, beta, None, None))
+    torch.cuda.synchronize()
+    ref = A.double().t() @ B.double() + beta * C0.double()
+    err = ((C.double() - ref).norm() / ref.norm()).item()
+    # fp32 accumulation over K terms: ~sqrt(K) * 2^-24 relative
+    assert err < (3e-5 if out == "f32" else 8e-3), err
