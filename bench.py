@@ -216,6 +216,7 @@ def main():
     ap.add_argument("--layers", type=int, default=LAYERS)
     ap.add_argument("--no-unbudgeted", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--analytic-profile", action="store_true", help="plan with the analytic model, not measured times")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -258,8 +259,15 @@ def main():
     static = bst["static_bytes"]
     unsplit_peak = bst["peak_extent"]
     budget = static + int(args.budget_frac * (unsplit_peak - static))
+    arrays = gen.make_inputs(spec, seed=rank)
+    dev_inputs = tsplit.inputs_to_device(G, arrays, device=f"cuda:{local}")
     t0 = time.time()
-    blob = tsplit.Plan.plan(G, budget).serialize() if rank == 0 else None
+    blob, pcie = None, None
+    if rank == 0:
+        # profile every op (and split widths) on the GPU before planning
+        prof = tsplit.Profile.measure(G, dev_inputs, max_p=4, device=local) if not args.analytic_profile else None
+        pcie = prof.pcie() if prof else None
+        blob = tsplit.Plan.plan(G, budget, prof).serialize()
     plan_s = time.time() - t0
     plan = tsplit.Plan.deserialize(G, bcast_bytes(blob))
     pst = plan.stats()
@@ -270,8 +278,6 @@ def main():
 
     streams = tuple(torch.cuda.Stream() for _ in range(3))
     params = gen.init_params(spec, seed=1)
-    arrays = gen.make_inputs(spec, seed=rank)
-    dev_inputs = tsplit.inputs_to_device(G, arrays, device=f"cuda:{local}")
     host_inputs = tsplit.inputs_to_device(G, arrays, pinned_host=True)
     h2d_bytes = sum(int(np.prod(t["shape"])) * 4 for t in spec["tensors"] if t["kind"] in ("input", "label"))
 
@@ -353,7 +359,8 @@ def main():
                      "recompute_tensors": pst["n_recompute_tensors"], "replays": pst["n_replay"],
                      "d2h_bytes": pst["d2h_bytes"], "h2d_bytes": pst["h2d_bytes"],
                      "step_flop": pst["compute_flop"], "predicted_ms": pst["predicted_s"] * 1e3,
-                     "planning_s": round(plan_s, 2)},
+                     "profile_and_planning_s": round(plan_s, 2),
+                     "measured_pcie_gbs": [round(x / 1e9, 1) for x in pcie] if pcie else None},
             "l2": "no flush needed: every step streams >10 GB of activations through a 126 MB L2",
         },
         "unbudgeted_samples_per_s": unb,

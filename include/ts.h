@@ -160,6 +160,16 @@ ts_status ts_profile_analytic(const ts_graph_t* g, const ts_hw* hw, ts_profile_t
 ts_status ts_profile_set(ts_profile_t* pr, int32_t op, int32_t p_num, double fwd_s, double bwd_s);
 ts_status ts_profile_set_pcie(ts_profile_t* pr, double d2h_bw, double h2d_bw);
 void ts_profile_destroy(ts_profile_t* pr);
+/* Measured profile (needs the GPU): for p = 1, 2, 4, ... <= max_p, runs one warm-up and
+ * one cudaEvent-timed eager step of the all-reside plan with every activation split p
+ * ways, on the caller's scratch `slab` (device, >= the unsplit peak; parameters are
+ * zero — op times do not depend on the data), and records each op's forward
+ * and backward time; wider splits reuse the widest measured one.  Also measures pinned
+ * D2H/H2D bandwidth (256 MiB copies).  `inputs` as in ts_step. */
+ts_status ts_profile_measure(const ts_graph_t* g, void* slab, uint64_t slab_bytes, const void* const* inputs,
+                             int32_t inputs_on_host, int32_t max_p, ts_profile_t** out);
+ts_status ts_profile_get(const ts_profile_t* pr, int32_t op, int32_t p_num, double* fwd_s, double* bwd_s);
+ts_status ts_profile_pcie(const ts_profile_t* pr, double* d2h_bw, double* h2d_bw);
 
 /* ---- plan ------------------------------------------------------------------- */
 /* All tensors reside, p_num = 1 (the "Base" of P:L304). */

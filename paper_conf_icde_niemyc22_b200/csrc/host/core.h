@@ -99,6 +99,10 @@ struct SimResult {
   uint64_t d2h = 0, h2d = 0;
   int64_t n_replay = 0, n_compute = 0;
   std::unordered_map<PieceKey, uint64_t> offset;  // placement of each piece (last)
+  // R12 fences: for each item, the swap-out items whose logically freed range this
+  // item's allocations overlap and that its stream (compute, or H2D for swap-ins) has
+  // not yet waited for; the runtime waits on exactly these copy events.
+  std::vector<std::vector<int>> wait_so;
 };
 
 int piece_count(const Graph& g, const std::vector<Cfg>& cfg, int key);
@@ -146,6 +150,7 @@ struct PlanState {
 };
 void plan_refresh(const Graph& g, PlanState& ps, const Profile* pr);
 ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps);
+void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps);
 
 }  // namespace ts
 

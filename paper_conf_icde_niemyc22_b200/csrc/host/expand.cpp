@@ -271,6 +271,13 @@ bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, 
   pool.reset(g.static_bytes, capacity);
   std::unordered_map<PieceKey, uint64_t> where;
   uint64_t live = 0, peak = 0, top = g.static_bytes;
+  struct Fence {
+    uint64_t off, len;
+    int so;
+  };
+  std::vector<Fence> pend_cs, pend_h2d;
+  r.wait_so.assign(ex.items.size(), {});
+  int cur_item = -1;
   int64_t seq = 0;
   bool ok = true;
   auto do_alloc = [&](int item, PieceKey pc) {
@@ -282,6 +289,18 @@ bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, 
     where[pc] = off;
     r.offset[pc] = off;
     live += align_up(b);
+    if (item >= 0) {
+      auto& pend = ex.items[item].kind == IT_SI ? pend_h2d : pend_cs;
+      const uint64_t len = align_up(b);
+      for (size_t f = 0; f < pend.size();) {
+        if (off < pend[f].off + pend[f].len && pend[f].off < off + len) {
+          r.wait_so[item].push_back(pend[f].so);
+          pend.erase(pend.begin() + f);
+        } else {
+          ++f;
+        }
+      }
+    }
     r.trace.push_back({seq++, item, 0, pk_key(pc), pk_j(pc), off, b});
     if (placements && item >= 0) (*placements)[item].push_back({pc, off});
   };
@@ -315,8 +334,15 @@ bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, 
     else if (it.kind == IT_SI) r.h2d += piece_bytes(g, cfg, pk_key(it.writes[0]));
     else if (it.kind == IT_R) ++r.n_replay;
     else ++r.n_compute;
+    if (it.kind == IT_SO) {
+      const PieceKey pc = it.reads[0];
+      Fence f{where.at(pc), align_up(piece_bytes(g, cfg, pk_key(pc))), (int)i};
+      pend_cs.push_back(f);
+      pend_h2d.push_back(f);
+    }
     for (PieceKey pc : ex.free_after[i]) do_free((int)i, pc);
   }
+  (void)cur_item;
   std::vector<PieceKey> rest;
   for (auto& kv : where) rest.push_back(kv.first);
   std::sort(rest.begin(), rest.end());

@@ -15,6 +15,8 @@
 #include <algorithm>
 #include <cmath>
 #include <limits>
+#include <cstdio>
+#include <cstdlib>
 #include <set>
 
 #include "core.h"
@@ -143,19 +145,26 @@ void timeline(const Graph& g, const PlanState& ps, const Profile& pr, Timeline& 
   tl.oc_h2d.assign(ni, 0);
   std::vector<double> start(ni, 0);
   std::vector<std::pair<double, double>> busy_d2h, busy_h2d;
-  std::unordered_map<PieceKey, double> ready;
+  std::unordered_map<PieceKey, double> ready, so_end;
+  std::unordered_map<size_t, double> so_end_item;  // SO item -> copy completion time
   double clock = 0, d2h_free = 0, h2d_free = 0;
   for (size_t i = 0; i < ni; ++i) {
     const Item& it = items[i];
     if (it.kind == IT_SO) {
       double s = std::max(clock, d2h_free);
+      so_end_item[i] = 0;
       double e = s + double(piece_bytes(g, ps.cfg, pk_key(it.reads[0]))) / pr.hw.d2h_bw;
       busy_d2h.push_back({s, e});
       d2h_free = e;
+      so_end[it.reads[0]] = e;
+      so_end_item[i] = e;
       continue;
     }
     if (it.kind == IT_SI) {
       double s = std::max(clock, h2d_free);
+      auto so = so_end.find(it.writes[0]);
+      if (so != so_end.end()) s = std::max(s, so->second);
+      for (int f : ps.sim.wait_so[i]) s = std::max(s, so_end_item[size_t(f)]);
       double e = s + double(piece_bytes(g, ps.cfg, pk_key(it.writes[0]))) / pr.hw.h2d_bw;
       busy_h2d.push_back({s, e});
       h2d_free = e;
@@ -166,6 +175,8 @@ void timeline(const Graph& g, const PlanState& ps, const Profile& pr, Timeline& 
       auto r = ready.find(p);
       if (r != ready.end()) clock = std::max(clock, r->second);
     }
+    // reuse of a range still being copied out waits for that copy (R12)
+    for (int f : ps.sim.wait_so[i]) clock = std::max(clock, so_end_item[size_t(f)]);
     int l = lg2(ps.ex.P[it.op]);
     double t = (it.kind == IT_B ? pr.tb[it.op][l] : pr.tf[it.op][l]) / double(ps.ex.P[it.op]);
     start[i] = clock;
@@ -230,6 +241,68 @@ bool better(const Cand& a, const Cand& b) {  // a strictly better than b
 
 }  // namespace
 
+namespace {
+uint64_t max_top(const PlanState& s) {
+  uint64_t m = 0;
+  for (uint64_t t : s.sim.top) m = std::max(m, t);
+  return m;
+}
+}  // namespace
+
+// Post-pass on the greedy plan (reading D-R8c).  Alg. 2 resolves bottlenecks
+// in schedule order, so an eviction chosen at an early bottleneck can become redundant
+// once later ones are fixed, and several prefetches can collide on the H2D link.
+// (1) revert non-reside decisions, most expensive first, whenever the plan still fits;
+// (2) turn remaining recomputes into swaps with longer prefetch leads when that lowers
+// the predicted step time and still fits.  Every change is re-simulated.
+void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps) {
+  plan_refresh(g, ps, &pr);
+  const int n = g.n();
+  auto try_cfg = [&](const std::vector<Cfg>& cfg, PlanState& out) {
+    out.cfg = cfg;
+    plan_refresh(g, out, &pr);
+    return max_top(out) <= budget;
+  };
+  // cost of each decision: predicted time saved by reverting it (ignoring feasibility)
+  std::vector<std::pair<double, int>> order;
+  for (int t = 0; t < n; ++t) {
+    const Cfg& c = ps.cfg[t];
+    if (c.opt == TS_RESIDE && c.p == 1) continue;
+    PlanState tmp;
+    std::vector<Cfg> cfg = ps.cfg;
+    cfg[t] = Cfg();
+    tmp.cfg = cfg;
+    plan_refresh(g, tmp, &pr);
+    order.push_back({ps.predicted_s - tmp.predicted_s, t});
+  }
+  std::sort(order.begin(), order.end(), [](auto& a, auto& b) { return a.first > b.first; });
+  for (auto& [gain, t] : order) {
+    if (gain <= 0) continue;
+    std::vector<Cfg> cfg = ps.cfg;
+    cfg[t] = Cfg();
+    PlanState cand;
+    if (try_cfg(cfg, cand) && cand.predicted_s < ps.predicted_s) ps = std::move(cand);
+  }
+  // recompute -> swap with a prefetch lead that hides the copy behind compute
+  std::vector<std::pair<double, int>> rc;
+  for (int t = 0; t < n; ++t)
+    if (ps.cfg[t].opt == TS_RECOMPUTE) rc.push_back({double(g.t[t].bytes), t});
+  std::sort(rc.begin(), rc.end(), [](auto& a, auto& b) { return a.first > b.first; });
+  for (auto& [bytes, t] : rc) {
+    (void)bytes;
+    for (int lead : {4, 16, 64}) {
+      std::vector<Cfg> cfg = ps.cfg;
+      cfg[t].opt = TS_SWAP;
+      cfg[t].lead = lead;
+      PlanState cand;
+      if (try_cfg(cfg, cand) && cand.predicted_s < ps.predicted_s - 1e-6) {
+        ps = std::move(cand);
+        break;
+      }
+    }
+  }
+}
+
 ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps) {
   const int n = g.n();
   ps.cfg.assign(n, Cfg());
@@ -242,7 +315,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
     for (int x : g.ops[g.order[i]].out) birth[x] = (int)i;
   const int kMaxIter = 20000;
   for (int iter = 0; iter < kMaxIter; ++iter) {
-    plan_refresh(g, ps, nullptr);
+    plan_refresh(g, ps, &pr);
     const auto& items = ps.ex.items;
     int bi = -1;
     for (size_t i = 0; i < items.size(); ++i)
@@ -251,7 +324,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
         break;
       }
     if (bi < 0) {
-      plan_refresh(g, ps, &pr);
+      plan_refine(g, budget, pr, ps);
       return TS_OK;
     }
     // bottleneck op and phase
@@ -337,91 +410,169 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       for (int u = p; u < q; ++u) bw += (1.0 - tl.oc_h2d[u]) * tl.T[u];
       return std::max(0.0, size / pr.hw.d2h_bw - fw) + std::max(0.0, size / pr.hw.h2d_bw - bw);
     };
-    Cand best;
-    // ---- step 1: non-split options on live tensors that are neither inputs nor
-    // outputs of the bottleneck op (Eq. 2, Eq. 3, R6) --------------------------
+    // ---- candidates ---------------------------------------------------------------
+    struct Change {
+      int t, opt, p, lead;
+    };
+    struct Cand2 {
+      std::vector<Change> ch;
+      double analytic = 0;
+      int birth = 0, tensor = 0;
+    };
+    // recompute of t also recomputes producer inputs that would otherwise be held only
+    // for the replay (e.g. attention scores behind a recomputed softmax output)
+    auto with_feeders = [&](Cand2 c, int t) {
+      const Op& po = g.ops[g.t[t].producer];
+      for (int u : po.in) {
+        const Tensor& x = g.t[u];
+        if (x.kind == TS_ACT && !x.is_loss && u != t && ps.cfg[u].opt == TS_RESIDE && first_bw[u] < 0)
+          c.ch.push_back({u, TS_RECOMPUTE, ps.cfg[u].p, 1});
+      }
+      return c;
+    };
+    std::vector<Cand2> step1, step2;
+    // step 1: non-split options on live tensors that are neither inputs nor outputs of
+    // the bottleneck op (Eq. 2 dM, Eq. 3 / R6 dT for the shortlist)
     for (int t : live) {
       const Tensor& x = g.t[t];
       if (x.kind != TS_ACT || x.is_loss || ps.cfg[t].opt != TS_RESIDE || own.count(t)) continue;
-      if (first_bw[t] < 0) continue;  // not held for backward: nothing to gain
+      if (first_bw[t] < 0) continue;                 // not held for backward: nothing to gain
       if (!bwd_phase && last_fw[t] >= bi) continue;  // still read later in the forward pass
-      if (bwd_phase && first_bw[t] - std::max(1, ps.cfg[t].lead) <= bi) {
-        // a swap would already be back by i; a recompute would be live in this group
-        continue;
-      }
+      if (bwd_phase && first_bw[t] - std::max(1, ps.cfg[t].lead) <= bi) continue;
       double dm = double(x.bytes);
-      Cand c1;
-      c1.valid = true;
-      c1.tensor = t;
-      c1.birth = birth[t];
-      c1.p = ps.cfg[t].p;
-      c1.opt = TS_SWAP;
-      c1.ratio = swap_cost(t, dm) / dm;
-      if (better(c1, best)) best = c1;
-      c1.opt = TS_RECOMPUTE;
-      c1.ratio = double(bw_ops[t].size()) * rc_time(rc_time, t, 0) / dm;
-      if (better(c1, best)) best = c1;
-    }
-    // ---- step 2: split options on the bottleneck op's own tensors (Eq. 6) -----
-    auto top_of_op = [&](const PlanState& s) {
-      uint64_t m = 0;
-      for (size_t i = 0; i < s.ex.items.size(); ++i) {
-        const Item& it = s.ex.items[i];
-        if (it.kind == IT_SO || it.kind == IT_SI) continue;
-        bool same_phase = ((int)i >= s.ex.fwd_end) == bwd_phase;
-        if (same_phase && it.op == bop) m = std::max(m, s.sim.top[i]);
+      Cand2 c;
+      c.birth = birth[t];
+      c.tensor = t;
+      c.ch = {{t, TS_SWAP, ps.cfg[t].p, 1}};
+      c.analytic = swap_cost(t, dm) / dm;
+      step1.push_back(c);
+      // the same swap with the prefetch issued early enough to hide the H2D copy
+      // (B200 computes ~30x more per PCIe byte than the paper's GPUs)
+      {
+        double need = 1.25 * dm / pr.hw.h2d_bw, acc_t = 0;
+        int lead = 0;
+        for (int u = first_bw[t] - 1; u >= ps.ex.fwd_end && acc_t < need; --u) {
+          if (items[u].kind == IT_SO || items[u].kind == IT_SI) continue;
+          acc_t += tl.T[u];
+          ++lead;
+        }
+        if (lead > 1) {
+          Cand2 c2 = c;
+          c2.ch = {{t, TS_SWAP, ps.cfg[t].p, lead}};
+          double fw = 0;
+          for (int u = last_fw[t] + 1; u < bi && u < (int)items.size(); ++u) fw += (1.0 - tl.oc_d2h[u]) * tl.T[u];
+          c2.analytic = std::max(0.0, dm / pr.hw.d2h_bw - fw) / dm;
+          step1.push_back(c2);
+        }
       }
-      return m;
-    };
-    uint64_t cur_top = top_of_op(ps);
+      c.ch = {{t, TS_RECOMPUTE, ps.cfg[t].p, 1}};
+      c.analytic = double(bw_ops[t].size()) * rc_time(rc_time, t, 0) / dm;
+      step1.push_back(with_feeders(c, t));
+    }
+    // shortlist by the analytic ratio, keeping the best swaps and the best recomputes
+    {
+      auto by = [](const Cand2& a, const Cand2& b) {
+        if (a.analytic != b.analytic) return a.analytic < b.analytic;
+        return a.birth < b.birth;
+      };
+      std::vector<Cand2> sw, rc;
+      for (auto& c : step1) (c.ch[0].opt == TS_SWAP ? sw : rc).push_back(c);
+      std::stable_sort(sw.begin(), sw.end(), by);
+      std::stable_sort(rc.begin(), rc.end(), by);
+      if (sw.size() > 6) sw.resize(6);
+      if (rc.size() > 8) rc.resize(8);
+      step1 = sw;
+      step1.insert(step1.end(), rc.begin(), rc.end());
+    }
+    // step 2: split options on the bottleneck op's own activations (Eq. 6)
     std::vector<int> split_cands;
     for (int x : g.ops[bop].in)
       if (g.t[x].kind == TS_ACT && !g.t[x].is_loss) split_cands.push_back(x);
     for (int x : g.ops[bop].out)
       if (g.t[x].kind == TS_ACT && !g.t[x].is_loss) split_cands.push_back(x);
-    for (int t : split_cands) {
+    for (int t : split_cands)
       for (int p = 2; p <= 16; p *= 2) {
         if (p <= ps.cfg[t].p || g.samples % p) continue;
         for (int opt : {TS_RESIDE, TS_SWAP, TS_RECOMPUTE}) {
           if (opt != TS_RESIDE && first_bw[t] < 0) continue;
-          PlanState cand;
-          cand.cfg = ps.cfg;
-          cand.cfg[t].opt = opt;
-          cand.cfg[t].p = p;
-          plan_refresh(g, cand, nullptr);
-          uint64_t nt = top_of_op(cand);
-          if (nt >= cur_top) continue;
-          double dm = double(cur_top - nt);
-          double micro = 0;
-          if (opt == TS_SWAP) micro = swap_cost(t, double(g.t[t].bytes) / p);
-          if (opt == TS_RECOMPUTE) micro = double(bw_ops[t].size()) * rc_time(rc_time, t, 0) / p;
-          double dsplit = 0;
-          std::set<int> ops_t(g.t[t].consumers.begin(), g.t[t].consumers.end());
-          ops_t.insert(g.t[t].producer);
-          for (int o : ops_t) {
-            int l0 = lg2(ps.ex.P[o]), l1 = lg2(cand.ex.P[o]);
-            dsplit += pr.tf[o][l1] - pr.tf[o][l0];
-            if (g.ops[o].has_bwd) dsplit += pr.tb[o][l1] - pr.tb[o][l0];
-          }
-          Cand c2;
-          c2.valid = true;
-          c2.tensor = t;
-          c2.birth = birth[t];
-          c2.opt = opt;
-          c2.p = p;
-          c2.ratio = (double(p - 1) * micro + std::max(0.0, dsplit)) / dm;
-          if (better(c2, best)) best = c2;
+          Cand2 c;
+          c.birth = birth[t];
+          c.tensor = t;
+          c.ch = {{t, opt, p, ps.cfg[t].lead}};
+          step2.push_back(opt == TS_RECOMPUTE ? with_feeders(c, t) : c);
         }
       }
+    // step 3: score every proposal by re-simulation — dM = drop of the pool top over
+    // the bottleneck op's items, dT = change of the predicted step time (timeline with
+    // the profile, PCIe occupancy and swap-in stalls) — and take the best.
+    auto top_of_op = [&](const PlanState& st) {
+      uint64_t m = 0;
+      for (size_t i = 0; i < st.ex.items.size(); ++i) {
+        const Item& it = st.ex.items[i];
+        if (it.kind == IT_SO || it.kind == IT_SI) continue;
+        bool same_phase = ((int)i >= st.ex.fwd_end) == bwd_phase;
+        if (same_phase && it.op == bop) m = std::max(m, st.sim.top[i]);
+      }
+      return m;
+    };
+    const uint64_t cur_top = top_of_op(ps);
+    const Cand2* best = nullptr;
+    double best_ratio = 0, best_dm = 0;
+    auto consider = [&](const Cand2& c) {
+      PlanState cs;
+      cs.cfg = ps.cfg;
+      for (auto& chg : c.ch) {
+        cs.cfg[chg.t].opt = chg.opt;
+        cs.cfg[chg.t].p = chg.p;
+        cs.cfg[chg.t].lead = chg.lead;
+      }
+      plan_refresh(g, cs, &pr);
+      uint64_t nt = top_of_op(cs);
+      if (nt >= cur_top) return;
+      double dm = double(cur_top - nt);
+      double ratio = std::max(0.0, cs.predicted_s - ps.predicted_s) / dm;
+      bool take = !best || ratio < best_ratio - 1e-18 ||
+                  (std::fabs(ratio - best_ratio) <= 1e-18 &&
+                   (dm > best_dm || (dm == best_dm && (c.birth < best->birth ||
+                                                      (c.birth == best->birth && c.tensor < best->tensor)))));
+      if (take) {
+        best = &c;
+        best_ratio = ratio;
+        best_dm = dm;
+      }
+    };
+    static const bool log = std::getenv("TS_PLAN_LOG") != nullptr;
+    for (auto& c : step1) {
+      consider(c);
+      if (log) {
+        PlanState cs;
+        cs.cfg = ps.cfg;
+        for (auto& chg : c.ch) {
+          cs.cfg[chg.t].opt = chg.opt;
+          cs.cfg[chg.t].p = chg.p;
+          cs.cfg[chg.t].lead = chg.lead;
+        }
+        plan_refresh(g, cs, &pr);
+        std::fprintf(stderr, "  cand t=%d opt=%d lead=%d analytic=%.3g dT=%.3gms top %llu->%llu\n", c.tensor,
+                     c.ch[0].opt, c.ch[0].lead, c.analytic, 1e3 * (cs.predicted_s - ps.predicted_s),
+                     (unsigned long long)cur_top, (unsigned long long)top_of_op(cs));
+      }
     }
-    if (!best.valid) {
-      set_error("infeasible: no candidate left at op " + std::to_string(bop) + " (item " +
-                std::to_string(bi) + ", needs " + std::to_string(ps.sim.top[bi]) + " B > budget " +
-                std::to_string(budget) + ")");
+    for (auto& c : step2) consider(c);
+    if (log && best)
+      std::fprintf(stderr, "iter %d bottleneck item %d op %d (%s) top %.3f GB: pick t=%d opt=%d p=%d lead=%d ratio %.3g pred %.2f ms\n",
+                   iter, bi, bop, bwd_phase ? "bwd" : "fwd", cur_top / 1e9, best->tensor, best->ch[0].opt,
+                   best->ch[0].p, best->ch[0].lead, best_ratio, 1e3 * ps.predicted_s);
+    if (!best) {
+      set_error("infeasible: no candidate left at op " + std::to_string(bop) + " (item " + std::to_string(bi) +
+                ", needs " + std::to_string(ps.sim.top[bi]) + " B > budget " + std::to_string(budget) + ")");
       return TS_ERR_INFEASIBLE;
     }
-    ps.cfg[best.tensor].opt = best.opt;
-    ps.cfg[best.tensor].p = best.p;
+    for (auto& chg : best->ch) {
+      ps.cfg[chg.t].opt = chg.opt;
+      ps.cfg[chg.t].p = chg.p;
+      ps.cfg[chg.t].lead = chg.lead;
+    }
   }
   set_error("planner did not converge");
   return TS_ERR_INFEASIBLE;

@@ -421,16 +421,7 @@ ts_status build_program(ts_session_t* s) {
       ++ev;
     }
     (void)e0;
-    auto& pend = it.kind == IT_SI ? pend_h2d : pend_cs;
-    for (auto& a : allocs)
-      for (size_t f = 0; f < pend.size();) {
-        if (overlaps(a.first, a.second, pend[f].off, pend[f].len)) {
-          cmd.wait_so.push_back(pend[f].so);
-          pend.erase(pend.begin() + f);
-        } else {
-          ++f;
-        }
-      }
+    cmd.wait_so = s->sim.wait_so[i];  // R12 fences computed by the simulator
     if (it.kind == IT_SO) {
       PieceKey pc = it.reads[0];
       cmd.kind = 1;
@@ -438,9 +429,6 @@ ts_status build_program(ts_session_t* s) {
       cmd.bytes = piece_bytes(g, s->cfg, pk_key(pc));
       cmd.host_off = host_off.at(pc);
       so_item_of[pc] = int(i);
-      Fence f{where.at(pc), align_up(cmd.bytes), int(i)};
-      pend_cs.push_back(f);
-      pend_h2d.push_back(f);
       CU(cudaEventCreateWithFlags(&s->ev_d2h[i], cudaEventDisableTiming));
     } else if (it.kind == IT_SI) {
       PieceKey pc = it.writes[0];
@@ -800,6 +788,118 @@ ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, 
   *n = s->item_ms.size();
   if (ms)
     for (uint64_t i = 0; i < s->item_ms.size() && i < cap; ++i) ms[i] = s->item_ms[i];
+  return TS_OK;
+}
+
+// ---- profiling ("profiles the training process ... before actual execution",
+// P:L268 "profiles every single operation", P:L281 cudaEvent timing and transfer time =
+// size / bandwidth with the hardware monopolised) -------------------------------------
+ts_status ts_profile_measure(const ts_graph_t* gh, void* slab, uint64_t slab_bytes, const void* const* inputs,
+                             int32_t inputs_on_host, int32_t max_p, ts_profile_t** out) {
+  if (!gh || !slab || !inputs || !out) return set_error("null argument"), TS_ERR_ARG;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return set_error("no CUDA device: profiling needs the GPU"), TS_ERR_NO_GPU;
+  }
+  const Graph& g = gh->g;
+  auto prof = std::make_unique<ts_profile_t>();
+  profile_analytic(g, default_hw(), prof->pr);
+  int dev = 0;
+  cudaGetDevice(&dev);
+  for (int p = 1; p <= 16 && p <= max_p; p *= 2) {
+    if (g.samples % p) break;
+    ts_plan_t plan;
+    plan.graph = &g;
+    plan.st.cfg.assign(g.n(), Cfg());
+    for (auto& t : g.t)
+      if (t.kind == TS_ACT && !t.is_loss) plan.st.cfg[t.id].p = p;
+    plan_refresh(g, plan.st, nullptr);
+    if (plan.st.sim.peak_extent > slab_bytes) continue;  // does not fit the scratch slab
+    ts_session_cfg sc;
+    std::memset(&sc, 0, sizeof(sc));
+    sc.device = dev;
+    sc.slab = slab;
+    sc.slab_bytes = slab_bytes;
+    sc.world_size = 1;
+    sc.use_cuda_graph = 0;
+    ts_session_t* s = nullptr;
+    ts_status st = ts_session_create(gh, &plan, &sc, &s);
+    if (st != TS_OK) return st;
+    st = ts_session_profile_items(s, 1);
+    if (st == TS_OK) st = run_step(s, inputs, inputs_on_host);  // warm-up
+    if (st == TS_OK) st = run_step(s, inputs, inputs_on_host);  // timed
+    if (st != TS_OK) {
+      ts_session_destroy(s);
+      return st;
+    }
+    std::vector<double> tf(g.ops.size(), 0.0), tb(g.ops.size(), 0.0);
+    for (size_t i = 0; i < s->ex.items.size(); ++i) {
+      const Item& it = s->ex.items[i];
+      if (it.kind == IT_F) tf[it.op] += 1e-3 * s->item_ms[i];
+      else if (it.kind == IT_B) tb[it.op] += 1e-3 * s->item_ms[i];
+    }
+    int l = 0;
+    while ((1 << l) < p) ++l;
+    for (size_t o = 0; o < g.ops.size(); ++o) {
+      prof->pr.tf[o][l] = tf[o];
+      prof->pr.tb[o][l] = tb[o];
+      // untested wider splits extrapolate from the widest measured one (per-micro-op overhead kept)
+      for (int l2 = l + 1; l2 < 5; ++l2) {
+        prof->pr.tf[o][l2] = tf[o] * (1.0 + 0.05 * (l2 - l));
+        prof->pr.tb[o][l2] = tb[o] * (1.0 + 0.05 * (l2 - l));
+      }
+    }
+    ts_session_destroy(s);
+  }
+  // PCIe bandwidth with pinned host memory (swap time = size / B)
+  const size_t nb = size_t(256) << 20;
+  if (slab_bytes >= nb) {
+    void* host = nullptr;
+    if (cudaHostAlloc(&host, nb, cudaHostAllocDefault) == cudaSuccess) {
+      cudaStream_t st;
+      cudaEvent_t e0, e1;
+      CU(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+      CU(cudaEventCreate(&e0));
+      CU(cudaEventCreate(&e1));
+      float ms_d2h = 0, ms_h2d = 0;
+      for (int rep = 0; rep < 2; ++rep) {
+        cudaEventRecord(e0, st);
+        cudaMemcpyAsync(host, slab, nb, cudaMemcpyDeviceToHost, st);
+        cudaEventRecord(e1, st);
+        cudaEventSynchronize(e1);
+        cudaEventElapsedTime(&ms_d2h, e0, e1);
+        cudaEventRecord(e0, st);
+        cudaMemcpyAsync(slab, host, nb, cudaMemcpyHostToDevice, st);
+        cudaEventRecord(e1, st);
+        cudaEventSynchronize(e1);
+        cudaEventElapsedTime(&ms_h2d, e0, e1);
+      }
+      if (ms_d2h > 0) prof->pr.hw.d2h_bw = double(nb) / (1e-3 * ms_d2h);
+      if (ms_h2d > 0) prof->pr.hw.h2d_bw = double(nb) / (1e-3 * ms_h2d);
+      cudaEventDestroy(e0);
+      cudaEventDestroy(e1);
+      cudaStreamDestroy(st);
+      cudaFreeHost(host);
+    }
+  }
+  *out = prof.release();
+  return TS_OK;
+}
+
+ts_status ts_profile_get(const ts_profile_t* pr, int32_t op, int32_t p_num, double* fwd_s, double* bwd_s) {
+  if (!pr || !fwd_s || !bwd_s || op < 0 || op >= (int)pr->pr.tf.size()) return set_error("bad argument"), TS_ERR_ARG;
+  int l = 0;
+  while ((1 << l) < p_num && l < 4) ++l;
+  *fwd_s = pr->pr.tf[op][l];
+  *bwd_s = pr->pr.tb[op][l];
+  return TS_OK;
+}
+
+ts_status ts_profile_pcie(const ts_profile_t* pr, double* d2h_bw, double* h2d_bw) {
+  if (!pr || !d2h_bw || !h2d_bw) return set_error("bad argument"), TS_ERR_ARG;
+  *d2h_bw = pr->pr.hw.d2h_bw;
+  *h2d_bw = pr->pr.hw.h2d_bw;
   return TS_OK;
 }
 

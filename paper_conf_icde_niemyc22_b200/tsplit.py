@@ -116,6 +116,9 @@ def lib():
             "ts_session_launches": (i32, [vp, P(i64)]),
             "ts_session_profile_items": (i32, [vp, i32]),
             "ts_session_item_times": (i32, [vp, P(C.c_float), u64, P(u64)]),
+            "ts_profile_measure": (i32, [vp, vp, u64, P(vp), i32, i32, P(vp)]),
+            "ts_profile_get": (i32, [vp, i32, i32, P(C.c_double), P(C.c_double)]),
+            "ts_profile_pcie": (i32, [vp, P(C.c_double), P(C.c_double)]),
             "ts_nccl_unique_id": (i32, [vp]),
             "ts_nccl_comm_init": (i32, [vp, i32, i32, P(vp)]),
             "ts_nccl_comm_destroy": (i32, [vp]),
@@ -196,14 +199,43 @@ class Graph:
 
 
 class Profile:
-    def __init__(self, graph: Graph, hw: dict | None = None):
+    def __init__(self, graph: Graph, hw: dict | None = None, _handle=None):
         self.graph = graph
+        if _handle is not None:
+            self.h = _handle
+            return
         h = C.c_void_p()
         hwp = None
         if hw:
             hwp = C.byref(Hw(**hw))
         check(lib().ts_profile_analytic(graph.h, hwp, C.byref(h)))
         self.h = h
+
+    @classmethod
+    def measure(cls, graph: Graph, inputs: dict, max_p: int = 4, device: int = 0):
+        """Measured profile (ts_profile_measure) on a scratch slab of the unsplit peak."""
+        import torch
+        peak = Plan.default(graph).stats()["peak_extent"]
+        slab = torch.empty(peak, dtype=torch.uint8, device=f"cuda:{device}")
+        ids = [t["id"] for t in graph.spec["tensors"] if t["kind"] in ("input", "label")]
+        arr = (C.c_void_p * len(ids))()
+        for i, tid in enumerate(ids):
+            arr[i] = inputs[graph.spec["tensors"][tid]["name"]].data_ptr()
+        h = C.c_void_p()
+        check(lib().ts_profile_measure(graph.h, slab.data_ptr(), peak, arr, 0, max_p, C.byref(h)))
+        del slab
+        torch.cuda.empty_cache()
+        return cls(graph, _handle=h)
+
+    def get(self, op, p_num):
+        f, b = C.c_double(), C.c_double()
+        check(lib().ts_profile_get(self.h, op, p_num, C.byref(f), C.byref(b)))
+        return f.value, b.value
+
+    def pcie(self):
+        d, h = C.c_double(), C.c_double()
+        check(lib().ts_profile_pcie(self.h, C.byref(d), C.byref(h)))
+        return d.value, h.value
 
     def set(self, op, p_num, fwd_s, bwd_s):
         check(lib().ts_profile_set(self.h, op, p_num, fwd_s, bwd_s))
