@@ -17,11 +17,27 @@ struct EwP {
   uint32_t seed, step, thr;
 };
 
-__device__ __forceinline__ float gelu_f(float x) { return 0.5f * x * (1.f + erff(x * 0.70710678118654752f)); }
+// erf(z) by Abramowitz & Stegun 7.1.26 (|error| <= 1.5e-7), given e = exp(-z^2): the
+// GELU derivative needs the same exponential for the normal pdf, so one __expf serves both.
+__device__ __forceinline__ float erf_as(float z, float e) {
+  const float a = fabsf(z);
+  const float t = __frcp_rn(fmaf(0.3275911f, a, 1.f));
+  float p = fmaf(1.061405429f, t, -1.453152027f);
+  p = fmaf(p, t, 1.421413741f);
+  p = fmaf(p, t, -0.284496736f);
+  p = fmaf(p, t, 0.254829592f);
+  const float r = 1.f - p * t * e;
+  return copysignf(r, z);
+}
+__device__ __forceinline__ float gelu_f(float x) {
+  const float z = x * 0.70710678118654752f;
+  return 0.5f * x * (1.f + erf_as(z, __expf(-z * z)));
+}
 __device__ __forceinline__ float gelu_d(float x) {
-  float cdf = 0.5f * (1.f + erff(x * 0.70710678118654752f));
-  float pdf = 0.39894228040143268f * __expf(-0.5f * x * x);
-  return cdf + x * pdf;
+  const float z = x * 0.70710678118654752f;
+  const float e = __expf(-z * z);  // = exp(-x^2/2)
+  const float cdf = 0.5f * (1.f + erf_as(z, e));
+  return cdf + x * 0.39894228040143268f * e;
 }
 
 template <int OP>
@@ -41,58 +57,77 @@ __device__ __forceinline__ float ew_apply(float a, float b, int64_t idx, uint32_
 }
 
 template <class T, int OP, int V>
+__device__ __forceinline__ void ew_vec(const T* __restrict__ a, const T* __restrict__ b, T* y, int64_t v, int acc,
+                                       const EwP& q, const T* av, const T* bv, T* yv) {
+  uint32_t words[V];
+  if constexpr (OP == DROP) {
+    const int64_t i0 = q.elem0 + v * V;
+    if ((i0 & 3) == 0 && V % 4 == 0) {
+#pragma unroll
+      for (int j = 0; j < V; j += 4) {
+        uint64_t c = uint64_t(i0 + j) >> 2;
+        uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
+        words[j] = r.x;
+        words[j + 1] = r.y;
+        words[j + 2] = r.z;
+        words[j + 3] = r.w;
+      }
+    } else {
+#pragma unroll
+      for (int j = 0; j < V; ++j) {
+        uint64_t e = uint64_t(i0 + j), c = e >> 2;
+        uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
+        uint32_t w[4] = {r.x, r.y, r.z, r.w};
+        words[j] = w[e & 3];
+      }
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < V; ++i) {
+    float r = ew_apply<OP>(to_f(av[i]), b ? to_f(bv[i]) : 0.f, v * V + i, OP == DROP ? words[i] : 0u, q);
+    if (acc) r += to_f(yv[i]);
+    yv[i] = from_f<T>(r);
+  }
+}
+
+// U vectors of V elements per thread per iteration, all loads issued before any math,
+// so each SM keeps U x 16 B x threads in flight (HBM latency hiding, guide G7).
+template <class T, int OP, int V>
 __global__ void __launch_bounds__(256) ew_kernel(const T* __restrict__ a, const T* __restrict__ b, T* y, int64_t n,
                                                  int acc, EwP q) {
+  constexpr int U = 1;
   const int64_t nv = n / V;
   const int64_t stride = int64_t(gridDim.x) * blockDim.x;
-  for (int64_t v = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; v < nv; v += stride) {
-    T av[V], bv[V], yv[V];
-    if constexpr (V * sizeof(T) == 16) {
-      *reinterpret_cast<uint4*>(av) = reinterpret_cast<const uint4*>(a)[v];
-      if (b) *reinterpret_cast<uint4*>(bv) = reinterpret_cast<const uint4*>(b)[v];
-      if (acc) *reinterpret_cast<uint4*>(yv) = reinterpret_cast<const uint4*>(y)[v];
-    } else {
+  for (int64_t v0 = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; v0 < nv; v0 += stride * U) {
+    T av[U][V], bv[U][V], yv[U][V];
 #pragma unroll
-      for (int i = 0; i < V; ++i) {
-        av[i] = a[v * V + i];
-        if (b) bv[i] = b[v * V + i];
-        if (acc) yv[i] = y[v * V + i];
-      }
-    }
-    uint32_t words[V];
-    if constexpr (OP == DROP) {
-      const int64_t i0 = q.elem0 + v * V;
-      if ((i0 & 3) == 0 && V % 4 == 0) {
-#pragma unroll
-        for (int j = 0; j < V; j += 4) {
-          uint64_t c = uint64_t(i0 + j) >> 2;
-          uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
-          words[j] = r.x;
-          words[j + 1] = r.y;
-          words[j + 2] = r.z;
-          words[j + 3] = r.w;
-        }
+    for (int u = 0; u < U; ++u) {
+      const int64_t v = v0 + u * stride;
+      if (v >= nv) break;
+      if constexpr (V * sizeof(T) == 16) {
+        *reinterpret_cast<uint4*>(av[u]) = reinterpret_cast<const uint4*>(a)[v];
+        if (b) *reinterpret_cast<uint4*>(bv[u]) = reinterpret_cast<const uint4*>(b)[v];
+        if (acc) *reinterpret_cast<uint4*>(yv[u]) = reinterpret_cast<const uint4*>(y)[v];
       } else {
 #pragma unroll
-        for (int j = 0; j < V; ++j) {
-          uint64_t e = uint64_t(i0 + j), c = e >> 2;
-          uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
-          uint32_t w[4] = {r.x, r.y, r.z, r.w};
-          words[j] = w[e & 3];
+        for (int i = 0; i < V; ++i) {
+          av[u][i] = a[v * V + i];
+          if (b) bv[u][i] = b[v * V + i];
+          if (acc) yv[u][i] = y[v * V + i];
         }
       }
     }
 #pragma unroll
-    for (int i = 0; i < V; ++i) {
-      float r = ew_apply<OP>(to_f(av[i]), b ? to_f(bv[i]) : 0.f, v * V + i, OP == DROP ? words[i] : 0u, q);
-      if (acc) r += to_f(yv[i]);
-      yv[i] = from_f<T>(r);
-    }
-    if constexpr (V * sizeof(T) == 16) {
-      reinterpret_cast<uint4*>(y)[v] = *reinterpret_cast<uint4*>(yv);
-    } else {
+    for (int u = 0; u < U; ++u) {
+      const int64_t v = v0 + u * stride;
+      if (v >= nv) break;
+      ew_vec<T, OP, V>(a, b, y, v, acc, q, av[u], bv[u], yv[u]);
+      if constexpr (V * sizeof(T) == 16) {
+        reinterpret_cast<uint4*>(y)[v] = *reinterpret_cast<uint4*>(yv[u]);
+      } else {
 #pragma unroll
-      for (int i = 0; i < V; ++i) y[v * V + i] = yv[i];
+        for (int i = 0; i < V; ++i) y[v * V + i] = yv[u][i];
+      }
     }
   }
   // scalar tail

@@ -55,12 +55,14 @@ void layernorm_fwd(int dt, const void* x, const void* g, const void* b, void* y,
                    float eps, cudaStream_t st);
 // dx (+)= ...; partial dgamma/dbeta rows go to ws, then column_reduce adds them.
 void layernorm_bwd(int dt, const void* dy, const void* x, const void* g, void* dx, int acc, float* ws,
-                   float* dgamma, float* dbeta, int pacc, int64_t rows, int H, float eps, cudaStream_t st);
+                   uint64_t ws_bytes, float* dgamma, float* dbeta, int pacc, int64_t rows, int H, float eps,
+                   cudaStream_t st);
 void softmax_fwd(int dt, const void* x, void* y, int64_t rows, int L, cudaStream_t st);
 void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t rows, int L,
                  cudaStream_t st);
 // out[n] (+)= sum_r x[r, n] (rows filtered by `filter[r] == fval` when filter != null)
-void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, float* out, int acc,
+// (deterministic; the last 4 KB of the workspace hold the per-launch completion tickets)
+void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, uint64_t ws_bytes, float* out, int acc,
                 const int* filter, int fval, cudaStream_t st);
 void embed_fwd(int dt, const int* ids, const int* tt, const void* word, const void* pos, const void* type,
                void* y, int64_t rows, int H, int seq, int64_t row0, cudaStream_t st);

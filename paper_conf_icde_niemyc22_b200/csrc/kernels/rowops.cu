@@ -13,6 +13,7 @@ namespace tsk {
 namespace {
 
 constexpr int kWarps = 8;  // warps per block for row kernels
+constexpr uint64_t kTicketBytes = 4096;  // tail of the workspace reserved for colsum tickets
 
 template <class T>
 struct Vec {
@@ -151,7 +152,7 @@ __global__ void __launch_bounds__(kWarps * 32) ln_bwd_kernel(const T* __restrict
 // dy*xhat and dy over the warp's rows, combined across warps in a fixed order, so
 // the partial rows in ws are deterministic.
 template <class T, int NCH>
-__global__ void __launch_bounds__(kWarps * 32) ln_bwd_vec(const T* __restrict__ dy, const T* __restrict__ x,
+__global__ void __launch_bounds__(kWarps * 32, 2) ln_bwd_vec(const T* __restrict__ dy, const T* __restrict__ x,
                                                            const T* __restrict__ g, T* dx, int acc, float* ws,
                                                            int64_t rows, int H, float eps) {
   constexpr int V = Vec<T>::N;
@@ -236,29 +237,161 @@ __global__ void __launch_bounds__(kWarps * 32) ln_bwd_vec(const T* __restrict__ 
   for (int i = threadIdx.x; i < 2 * H; i += blockDim.x) ws[int64_t(blockIdx.x) * 2 * H + i] = sred[i];
 }
 
+// Two-kernel LayerNorm backward (rows of up to NCH x 32 x 16 B):
+//  ln_bwd_dx  — one warp per row: dx (+)= rstd*(g*dy - mean(g*dy) - xhat*mean(g*dy*xhat)),
+//               and the row's (mean, rstd) into ws_stats[2*row];
+//  ln_bwd_dgb — coalesced column partials of dy*xhat and dy (256 columns per block, rows
+//               interleaved over G blocks), reduced in fp64 by reduce_partials.
+template <class T, int NCH>
+__global__ void __launch_bounds__(kWarps * 32) ln_bwd_dx(const T* __restrict__ dy, const T* __restrict__ x,
+                                                          const T* __restrict__ g, T* dx, int acc,
+                                                          float* __restrict__ stats, int64_t rows, int H, float eps) {
+  constexpr int V = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  const int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5);
+  if (r >= rows) return;
+  float xv[NCH][V], dv[NCH][V];
+  float s = 0.f;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    int col = (c * 32 + lane) * V;
+    if (col < H) {
+      load_vec(x + r * H + col, xv[c]);
+      load_vec(dy + r * H + col, dv[c]);
+#pragma unroll
+      for (int i = 0; i < V; ++i) s += xv[c][i];
+    }
+  }
+  const float mean = warp_sum(s) / H;
+  float q = 0.f;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c)
+    if ((c * 32 + lane) * V < H)
+#pragma unroll
+      for (int i = 0; i < V; ++i) {
+        float d = xv[c][i] - mean;
+        q += d * d;
+      }
+  const float rstd = rsqrtf(warp_sum(q) / H + eps);
+  float s1 = 0.f, s2 = 0.f;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    int col = (c * 32 + lane) * V;
+    if (col < H) {
+      float gv[V];
+      load_vec(g + col, gv);
+#pragma unroll
+      for (int i = 0; i < V; ++i) {
+        xv[c][i] = (xv[c][i] - mean) * rstd;
+        float gd = dv[c][i] * gv[i];
+        s1 += gd;
+        s2 += gd * xv[c][i];
+      }
+    }
+  }
+  s1 = warp_sum(s1) / H;
+  s2 = warp_sum(s2) / H;
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    int col = (c * 32 + lane) * V;
+    if (col < H) {
+      float gv[V], o[V];
+      load_vec(g + col, gv);
+      if (acc) load_vec(dx + r * H + col, o);
+#pragma unroll
+      for (int i = 0; i < V; ++i) o[i] = rstd * (dv[c][i] * gv[i] - s1 - xv[c][i] * s2) + (acc ? o[i] : 0.f);
+      store_vec(dx + r * H + col, o);
+    }
+  }
+  if (lane == 0) {
+    stats[2 * r] = mean;
+    stats[2 * r + 1] = rstd;
+  }
+}
+
+template <class T>
+__global__ void __launch_bounds__(256) ln_bwd_dgb(const T* __restrict__ dy, const T* __restrict__ x,
+                                                   const float* __restrict__ stats, int64_t rows, int H, int G,
+                                                   float* __restrict__ ws) {
+  __shared__ float red[2][8][256];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int c0 = blockIdx.x * 256 + lane * 8;
+  float pg[8] = {0, 0, 0, 0, 0, 0, 0, 0}, pb[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  if (c0 < H) {
+    for (int64_t r = int64_t(blockIdx.y) * 8 + w; r < rows; r += int64_t(G) * 8) {
+      const float mean = stats[2 * r], rstd = stats[2 * r + 1];
+      constexpr int VV = 16 / sizeof(T);
+#pragma unroll
+      for (int h = 0; h < 8; h += VV) {
+        float xv[VV], dv[VV];
+        load_vec(x + r * H + c0 + h, xv);
+        load_vec(dy + r * H + c0 + h, dv);
+#pragma unroll
+        for (int i = 0; i < VV; ++i) {
+          pg[h + i] += dv[i] * (xv[i] - mean) * rstd;
+          pb[h + i] += dv[i];
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    red[0][w][lane * 8 + i] = pg[i];
+    red[1][w][lane * 8 + i] = pb[i];
+  }
+  __syncthreads();
+  const int c = blockIdx.x * 256 + threadIdx.x;
+  if (c < H) {
+    float a = 0.f, b = 0.f;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      a += red[0][k][threadIdx.x];
+      b += red[1][k][threadIdx.x];
+    }
+    ws[int64_t(blockIdx.y) * 2 * H + c] = a;
+    ws[int64_t(blockIdx.y) * 2 * H + H + c] = b;
+  }
+}
+
 // out[c] (+)= sum_{b < G} ws[b*stride + off + c]; the G partials are summed in
 // fp64 in a fixed order, so a split micro-op's contribution is exact up to the
 // single fp32 rounding of the accumulation into `out` (split invariance, R17).
-__global__ void reduce_partials(const float* __restrict__ ws, int G, int64_t stride, int64_t off, int N,
-                                float* out, int acc) {
-  int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= N) return;
+// Block = 32 columns x 8 warps: warp w sums partial rows w, w+8, ...; the 8 warp
+// sums are combined in warp order (deterministic), so G=256 costs 32 loads/thread.
+__global__ void __launch_bounds__(256) reduce_partials(const float* __restrict__ ws, int G, int64_t stride,
+                                                       int64_t off, int N, float* out, int acc) {
+  __shared__ double red[8][33];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + lane;
   double s = 0.0;
-#pragma unroll 8
-  for (int b = 0; b < G; ++b) s += double(ws[int64_t(b) * stride + off + c]);
-  out[c] = acc ? float(double(out[c]) + s) : float(s);
+  if (c < N) {
+#pragma unroll 4
+    for (int b = w; b < G; b += 8) s += double(ws[int64_t(b) * stride + off + c]);
+  }
+  red[w][lane] = s;
+  __syncthreads();
+  if (w == 0 && c < N) {
+    double t = 0.0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) t += red[k][lane];
+    out[c] = acc ? float(double(out[c]) + t) : float(t);
+  }
 }
 
-// Column partial sums of x[rows, N]: block (cb, g) owns 256 columns (32 lanes x 8
-// contiguous columns, 16-byte loads) and rows g, g+G, ...; 8 warps interleave rows
-// and combine through shared memory in a fixed order (deterministic).
+// Column sums of x[rows, N] into out[N] (+)=: block (cb, g) owns 256 columns (32 lanes x
+// 8 contiguous columns, 16-byte loads) and rows g*8+w, g*8+w+8G, ...; the 8 warps combine
+// in a fixed order into ws[g][N].  The last block to finish (atomic ticket per column
+// block) sums the G partial rows in fp64 in order g = 0..G-1, so the result is
+// deterministic and one launch replaces partial + reduce.
 template <class T>
-__global__ void __launch_bounds__(256) colsum_partial(const T* __restrict__ x, int64_t rows, int N, int G,
-                                                      float* __restrict__ ws, const int* __restrict__ filter, int fval) {
+__global__ void __launch_bounds__(256) colsum_kernel(const T* __restrict__ x, int64_t rows, int N, int G,
+                                                     float* __restrict__ ws, unsigned* __restrict__ tickets,
+                                                     float* out, int acc, const int* __restrict__ filter, int fval) {
   __shared__ float red[8][256];
+  __shared__ bool last;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int c0 = blockIdx.x * 256 + lane * 8;
-  float acc[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  float accv[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   const bool vec = (N % 8 == 0) && c0 + 8 <= N && (reinterpret_cast<uintptr_t>(x) % 16 == 0);
   for (int64_t r = int64_t(blockIdx.y) * 8 + w; r < rows; r += int64_t(G) * 8) {
     if (filter && filter[r] != fval) continue;
@@ -270,16 +403,16 @@ __global__ void __launch_bounds__(256) colsum_partial(const T* __restrict__ x, i
         uint4 u = *reinterpret_cast<const uint4*>(xr + c0 + h);
         const T* t = reinterpret_cast<const T*>(&u);
 #pragma unroll
-        for (int i = 0; i < V; ++i) acc[h + i] += to_f(t[i]);
+        for (int i = 0; i < V; ++i) accv[h + i] += to_f(t[i]);
       }
     } else {
 #pragma unroll
       for (int i = 0; i < 8; ++i)
-        if (c0 + i < N) acc[i] += to_f(xr[c0 + i]);
+        if (c0 + i < N) accv[i] += to_f(xr[c0 + i]);
     }
   }
 #pragma unroll
-  for (int i = 0; i < 8; ++i) red[w][lane * 8 + i] = acc[i];
+  for (int i = 0; i < 8; ++i) red[w][lane * 8 + i] = accv[i];
   __syncthreads();
   const int c = blockIdx.x * 256 + threadIdx.x;
   if (c < N) {
@@ -288,6 +421,18 @@ __global__ void __launch_bounds__(256) colsum_partial(const T* __restrict__ x, i
     for (int k = 0; k < 8; ++k) s += red[k][threadIdx.x];
     ws[int64_t(blockIdx.y) * N + c] = s;
   }
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) last = atomicAdd(&tickets[blockIdx.x], 1u) == unsigned(G - 1);
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  if (c < N) {
+    double t = 0.0;
+    for (int b = 0; b < G; ++b) t += double(__ldcg(&ws[int64_t(b) * N + c]));
+    out[c] = acc ? float(double(out[c]) + t) : float(t);
+  }
+  if (threadIdx.x == 0) tickets[blockIdx.x] = 0u;  // re-arm for the next launch / graph replay
 }
 
 // ------------------------------------------------------------------ softmax
@@ -593,14 +738,50 @@ void ln_bwd_t(const void* dy, const void* x, const void* g, void* dx, int acc, f
   ln_bwd_kernel<T><<<G, kWarps * 32, smem, st>>>(DY, X, Gm, DX, acc, ws, rows, H, eps);
 }
 
-void layernorm_bwd(int dt, const void* dy, const void* x, const void* g, void* dx, int acc, float* ws, float* dgamma,
-                   float* dbeta, int pacc, int64_t rows, int H, float eps, cudaStream_t st) {
+template <class T>
+bool ln_bwd_split_t(const void* dy, const void* x, const void* g, void* dx, int acc, float* ws, uint64_t ws_bytes,
+                    float* dgamma, float* dbeta, int pacc, int64_t rows, int H, float eps, cudaStream_t st) {
+  constexpr int V = Vec<T>::N;
+  const int nch = (H + 32 * V - 1) / (32 * V);
+  if (H % 8 || nch > 4 || !al16(dy) || !al16(x) || !al16(g) || !al16(dx)) return false;
+  const int cb = (H + 255) / 256;
+  int G = int((rows + 7) / 8);
+  int cap = (2 * 148) / cb;
+  if (cap > 64) cap = 64;
+  if (cap < 1) cap = 1;
+  if (G > cap) G = cap;
+  const uint64_t stats_bytes = uint64_t(rows) * 8, part_bytes = uint64_t(G) * 2 * H * 4;
+  if (stats_bytes + part_bytes + kTicketBytes > ws_bytes) return false;
+  float* part = ws;
+  float* stats = ws + (part_bytes / 4);
+  auto DY = (const T*)dy;
+  auto X = (const T*)x;
+  auto Gm = (const T*)g;
+  auto DX = (T*)dx;
+  const int grid = int((rows + kWarps - 1) / kWarps);
+  switch (nch) {
+    case 1: ln_bwd_dx<T, 1><<<grid, kWarps * 32, 0, st>>>(DY, X, Gm, DX, acc, stats, rows, H, eps); break;
+    case 2: ln_bwd_dx<T, 2><<<grid, kWarps * 32, 0, st>>>(DY, X, Gm, DX, acc, stats, rows, H, eps); break;
+    default: ln_bwd_dx<T, 4><<<grid, kWarps * 32, 0, st>>>(DY, X, Gm, DX, acc, stats, rows, H, eps); break;
+  }
+  ln_bwd_dgb<T><<<dim3(cb, G), 256, 0, st>>>(DY, X, stats, rows, H, G, part);
+  reduce_partials<<<(H + 31) / 32, 256, 0, st>>>(part, G, 2 * H, 0, H, dgamma, pacc);
+  reduce_partials<<<(H + 31) / 32, 256, 0, st>>>(part, G, 2 * H, H, H, dbeta, pacc);
+  return true;
+}
+
+void layernorm_bwd(int dt, const void* dy, const void* x, const void* g, void* dx, int acc, float* ws, uint64_t ws_bytes,
+                   float* dgamma, float* dbeta, int pacc, int64_t rows, int H, float eps, cudaStream_t st) {
+  if (dt == F32 ? ln_bwd_split_t<float>(dy, x, g, dx, acc, ws, ws_bytes, dgamma, dbeta, pacc, rows, H, eps, st)
+                : ln_bwd_split_t<bf16>(dy, x, g, dx, acc, ws, ws_bytes, dgamma, dbeta, pacc, rows, H, eps, st))
+    return;
+  // enough warps in flight to cover HBM latency (each row needs x and dy before any math)
   int64_t G = (rows + kWarps - 1) / kWarps;
-  if (G > 148) G = 148;
+  if (G > kWsRows) G = kWsRows;
   if (dt == F32) ln_bwd_t<float>(dy, x, g, dx, acc, ws, rows, H, eps, int(G), st);
   else ln_bwd_t<bf16>(dy, x, g, dx, acc, ws, rows, H, eps, int(G), st);
-  reduce_partials<<<(H + 255) / 256, 256, 0, st>>>(ws, int(G), 2 * H, 0, H, dgamma, pacc);
-  reduce_partials<<<(H + 255) / 256, 256, 0, st>>>(ws, int(G), 2 * H, H, H, dbeta, pacc);
+  reduce_partials<<<(H + 31) / 32, 256, 0, st>>>(ws, int(G), 2 * H, 0, H, dgamma, pacc);
+  reduce_partials<<<(H + 31) / 32, 256, 0, st>>>(ws, int(G), 2 * H, H, H, dbeta, pacc);
 }
 
 void softmax_fwd(int dt, const void* x, void* y, int64_t rows, int L, cudaStream_t st) {
@@ -612,8 +793,8 @@ void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64
   else softmax_bwd_t<bf16>(dy, y, dx, acc, rows, L, st);
 }
 
-void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, float* out, int acc, const int* filter, int fval,
-                cudaStream_t st) {
+void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, uint64_t ws_bytes, float* out, int acc,
+                const int* filter, int fval, cudaStream_t st) {
   const int cb = (N + 255) / 256;
   int G = int((rows + 7) / 8);
   int cap = 296 / cb;
@@ -621,10 +802,13 @@ void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, float* ou
   if (cap > 64) cap = 64;
   if (G > cap) G = cap;
   if (G < 1) G = 1;
+  // completion tickets live in the last 4 KB of the workspace, which no other kernel uses
+  unsigned* tickets = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(ws) + ws_bytes - kTicketBytes);
   dim3 grid(cb, G);
-  if (dt == F32) colsum_partial<float><<<grid, 256, 0, st>>>((const float*)x, rows, N, G, ws, filter, fval);
-  else colsum_partial<bf16><<<grid, 256, 0, st>>>((const bf16*)x, rows, N, G, ws, filter, fval);
-  reduce_partials<<<(N + 255) / 256, 256, 0, st>>>(ws, G, N, 0, N, out, acc);
+  if (dt == F32)
+    colsum_kernel<float><<<grid, 256, 0, st>>>((const float*)x, rows, N, G, ws, tickets, out, acc, filter, fval);
+  else
+    colsum_kernel<bf16><<<grid, 256, 0, st>>>((const bf16*)x, rows, N, G, ws, tickets, out, acc, filter, fval);
 }
 
 void embed_fwd(int dt, const int* ids, const int* tt, const void* word, const void* pos, const void* type, void* y,

@@ -149,10 +149,11 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       gs.push_back(d);
       float* db = param_g(s, bb);
       int dacc = A(bb);
-      nk = int(gs.size()) + 2;
-      return [gs, dY, R, N, db, dacc, ws, dt](cudaStream_t st) {
+      const uint64_t wsb = g.ws_bytes;
+      nk = int(gs.size()) + 1;
+      return [gs, dY, R, N, db, dacc, ws, wsb, dt](cudaStream_t st) {
         for (auto& a : gs) tsk::gemm(a, st);
-        tsk::column_sum(dt, dY, R, int(N), ws, db, dacc, nullptr, 0, st);
+        tsk::column_sum(dt, dY, R, int(N), ws, wsb, db, dacc, nullptr, 0, st);
       };
     }
     case TS_OP_RELU: case TS_OP_GELU: case TS_OP_TANH: {
@@ -193,7 +194,10 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       float *dg = param_g(s, o.in[1]), *dbt = param_g(s, o.in[2]);
       int pacc = A(o.in[1]);
       nk = 3;
-      return [=](cudaStream_t st) { tsk::layernorm_bwd(dt, dy, xp, gw, dx, acc, ws, dg, dbt, pacc, rows, H, eps, st); };
+      const uint64_t wsb = g.ws_bytes;
+      return [=](cudaStream_t st) {
+        tsk::layernorm_bwd(dt, dy, xp, gw, dx, acc, ws, wsb, dg, dbt, pacc, rows, H, eps, st);
+      };
     }
     case TS_OP_ADD: {
       if (!bwd) {
@@ -323,11 +327,13 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       char* dy = G(o.out[0]);
       float *dw = param_g(s, o.in[2]), *dp = param_g(s, o.in[3]), *dtp = param_g(s, o.in[4]);
       const int ntype = int(g.t[o.in[4]].shape[0]);
-      nk = 2 + 2 * ntype;
+      const uint64_t wsb = g.ws_bytes;
+      nk = 2 + ntype;
       return [=](cudaStream_t st) {
         tsk::embed_bwd_word(dt, dy, ids, dw, rows, H, st);
         tsk::embed_bwd_pos(dt, dy, dp, ns * out.rows_per_sample / seq, seq, H, 1, st);
-        for (int r = 0; r < ntype; ++r) tsk::column_sum(dt, dy, rows, H, ws, dtp + int64_t(r) * H, 1, tt, r, st);
+        for (int r = 0; r < ntype; ++r)
+          tsk::column_sum(dt, dy, rows, H, ws, wsb, dtp + int64_t(r) * H, 1, tt, r, st);
       };
     }
     case TS_OP_CLS: {
