@@ -30,6 +30,7 @@ constexpr int kThreads = 64 + 32 * kEpiWarps;  // warp0 TMA, warp1 MMA, warps 2.
 struct TcParams {
   int M, N, K, nb1, nb2;
   int tiles_m, tiles_n, num_tiles, num_kb;
+  int n_fastest;  // 1: consecutive tiles walk N (A, the larger operand, is streamed once)
   int ksplit, kb_per_split, num_units;  // work unit = (tile, K slice)
   int a_mn, b_mn;
   void* C;
@@ -45,12 +46,13 @@ struct TcParams {
 // products have long K and keep the smem for a deeper operand pipeline)
 template <bool F32OUT>
 constexpr int staging_bufs() { return F32OUT ? 1 : 2; }
+constexpr int kSmemLimit = 232448;  // 227 KB opt-in dynamic shared memory per CTA
 template <bool F32OUT>
 constexpr int staging_bytes() { return kEpiWarps * staging_bufs<F32OUT>() * 32 * 32 * (F32OUT ? 4 : 2); }
 template <int BN, bool F32OUT>
 constexpr int num_stages() {
   constexpr int stage = (BM + BN) * BK * 2;
-  constexpr int n = (224 * 1024 - staging_bytes<F32OUT>() - 2048) / stage;
+  constexpr int n = (kSmemLimit - staging_bytes<F32OUT>() - 2048) / stage;
   return n > 8 ? 8 : n;
 }
 
@@ -148,9 +150,16 @@ __device__ __forceinline__ void decode_tile(const TcParams& p, int tile, int& b1
   int per = p.tiles_m * p.tiles_n;
   int bb = tile / per;
   int r = tile - bb * per;
-  // m fastest: neighbouring CTAs share the same B (weight) tile in L2
-  int nt = r / p.tiles_m;
-  int mt = r - nt * p.tiles_m;
+  // walk the smaller operand's tiles fastest so the larger one streams from DRAM once
+  // while the smaller stays in L2
+  int nt, mt;
+  if (p.n_fastest) {
+    mt = r / p.tiles_n;
+    nt = r - mt * p.tiles_n;
+  } else {
+    nt = r / p.tiles_m;
+    mt = r - nt * p.tiles_m;
+  }
   b1 = bb % p.nb1;
   b2 = bb / p.nb1;
   m0 = mt * BM;
@@ -508,6 +517,7 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   p.tiles_n = (g.N + best_bn - 1) / best_bn;
   p.num_tiles = p.tiles_m * p.tiles_n * g.nb1 * g.nb2;
   p.num_kb = (g.K + BK - 1) / BK;
+  p.n_fastest = (int64_t(g.M) >= int64_t(g.N)) ? 1 : 0;
   p.a_mn = g.a.mn_major;
   p.b_mn = g.b.mn_major;
   p.C = g.c;
