@@ -303,15 +303,17 @@ def main():
     if world > 1:
         dist.barrier()
     dt_e2e = max_over_ranks(time_steps(torch, sess, host_inputs, streams[0], args.steps, async_step=False))
-    # roofline of the dominant kernel class (tcgen05 GEMM): one profiled eager step
+    # roofline of the dominant kernel (tcgen05 GEMM): one profiled eager step with a
+    # cudaEvent pair around every GEMM launch on the compute stream
     sess.profile_items(True)
     sess.step(dev_inputs)
     item_ms = sess.item_times()
+    recs = sess.gemm_times()
     sess.profile_items(False)
-    items = plan.items()
-    flops = gemm_flops_per_item(spec, items, micro_counts(spec, plan))
-    g_ms = sum(ms for ms, f in zip(item_ms, flops) if f > 0)
-    g_flop = sum(flops)
+    lin = [(f, ms) for f, ms, bt in recs if f > 0 and bt == 1]
+    att = [(f, ms) for f, ms, bt in recs if f > 0 and bt > 1]
+    g_flop, g_ms = sum(f for f, _ in lin), sum(ms for _, ms in lin)
+    a_flop, a_ms = sum(f for f, _ in att), sum(ms for _, ms in att)
     step_ms_prof = sum(item_ms)
     del sess
     torch.cuda.empty_cache()
@@ -335,6 +337,10 @@ def main():
     value = BATCH * world * args.steps / dt
     achieved = g_flop / (g_ms / 1e3) / 1e12 if g_ms > 0 else 0.0
     peak = pk.get("bf16_tflops_sustained", pk.get("bf16_tflops"))
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "r1_gemm_ncu.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get("traffic_per_launch_bytes")
     line = {
         "metric": "samples/sec under HBM budget (BERT-Large)",
         "value": value,
@@ -369,13 +375,18 @@ def main():
         "clocks": clk.summary(),
         "e2e": {"value": BATCH * world * args.steps / dt_e2e, "unit": "samples/s",
                 "h2d_bytes_per_step": h2d_bytes, "d2h_bytes_per_step": 4},
-        "roofline": {"bound": "tensor", "kernel": "tcgen05 GEMM (all linear/attention micro-ops)",
+        "roofline": {"bound": "tensor", "kernel": "gemm_tc (tcgen05/TMA) on linear micro-ops",
                      "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                     "frac": achieved / peak if peak else None, "traffic": None,
+                     "frac": achieved / peak if peak else None, "traffic": traffic,
                      "peak_source": f"{pk_src} bf16_tflops_sustained",
-                     "gemm_share_of_step": g_ms / step_ms_prof if step_ms_prof else None,
-                     "how": "one eager step with cudaEvents around every micro-op on the compute stream; "
-                            "algorithmic FLOP of the GEMM micro-ops / their summed duration"},
+                     "launches": len(lin), "share_of_step": g_ms / step_ms_prof if step_ms_prof else None,
+                     "how": "one eager step, cudaEvent pair around every GEMM launch on the compute stream; "
+                            "algorithmic FLOP (2MNK) / summed launch durations; traffic = dram read+write of "
+                            "one FFN1-forward launch from the committed ncu --set full capture"},
+        "roofline_attention_gemm": {"bound": "hbm", "kernel": "gemm_tc on per-(sample, head) attention products",
+                                    "achieved_tflops": a_flop / (a_ms / 1e3) / 1e12 if a_ms > 0 else None,
+                                    "launches": len(att),
+                                    "share_of_step": a_ms / step_ms_prof if step_ms_prof else None},
     }
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline_measure()

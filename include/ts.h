@@ -236,6 +236,10 @@ ts_status ts_session_launches(const ts_session_t* s, int64_t* n);
  * (seconds, cudaEvent; only when profiling was enabled). */
 ts_status ts_session_profile_items(ts_session_t* s, int32_t enable);
 ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, uint64_t* n);
+/* Per-GEMM-launch records of the last profiled step: algorithmic FLOP (0 for the SIMT
+ * fallback), cudaEvent duration on the compute stream (ms), batch count (1 = linear). */
+ts_status ts_session_gemm_times(const ts_session_t* s, double* flop, float* ms, int32_t* batch, uint64_t cap,
+                                uint64_t* n);
 
 /* ---- data parallelism (north_star: DP over NVLink with NCCL) -------------------
  * The session allreduces the fp32 gradient region (sum) with this communicator

@@ -565,8 +565,27 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   return true;
 }
 
+static std::vector<GemmRecord>* g_sink = nullptr;
+void gemm_records_enable(std::vector<GemmRecord>* sink) { g_sink = sink; }
+
 void gemm(const GemmArgs& g, cudaStream_t st) {
-  if (!gemm_tc(g, st)) gemm_simt(g, st);
+  GemmRecord rec{};
+  if (g_sink) {
+    cudaEventCreate(&rec.start);
+    cudaEventCreate(&rec.stop);
+    cudaEventRecord(rec.start, st);
+  }
+  rec.tc = gemm_tc(g, st) ? 1 : 0;
+  if (!rec.tc) gemm_simt(g, st);
+  if (g_sink) {
+    cudaEventRecord(rec.stop, st);
+    rec.flop = 2.0 * g.M * double(g.N) * g.K * g.nb1 * g.nb2;
+    rec.M = g.M;
+    rec.N = g.N;
+    rec.K = g.K;
+    rec.batch = g.nb1 * g.nb2;
+    g_sink->push_back(rec);
+  }
 }
 
 }  // namespace tsk

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <vector>
 
 namespace tsk {
 
@@ -37,6 +38,14 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st);
 void gemm_simt(const GemmArgs& g, cudaStream_t st);
 void gemm(const GemmArgs& g, cudaStream_t st);
 int64_t gemm_tc_launches();
+// Per-launch timing of GEMMs (eager profiling only): while enabled, gemm() brackets
+// every launch with CUDA events on its stream and records the algorithmic FLOP.
+struct GemmRecord {
+  cudaEvent_t start, stop;
+  double flop;
+  int M, N, K, batch, tc;
+};
+void gemm_records_enable(std::vector<GemmRecord>* sink);
 
 // ---- elementwise (n elements, dtype F32/BF16 for activations) ----------------
 void relu_fwd(int dt, const void* x, void* y, int64_t n, cudaStream_t st);

@@ -81,6 +81,9 @@ struct ts_session_s {
   bool profile = false;
   std::vector<cudaEvent_t> prof_ev;  // 2 per program command (compute items)
   std::vector<float> item_ms;
+  std::vector<tsk::GemmRecord> gemm_recs;
+  std::vector<double> gemm_flop, gemm_ms;
+  std::vector<int> gemm_batch;
 };
 
 namespace {
@@ -599,6 +602,14 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
   if (!inputs) return set_error("inputs is null"), TS_ERR_ARG;
   ts_status st = copy_inputs(s, inputs, on_host);
   if (st != TS_OK) return st;
+  if (s->profile) {
+    for (auto& r : s->gemm_recs) {
+      cudaEventDestroy(r.start);
+      cudaEventDestroy(r.stop);
+    }
+    s->gemm_recs.clear();
+    tsk::gemm_records_enable(&s->gemm_recs);
+  }
   if (s->use_graph && !s->profile) {
     if (!s->gexec) {
       cudaGraph_t graph;
@@ -625,7 +636,18 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
   ++s->step;  // dropout counter (graph mode keeps the captured step value)
   CU(cudaGetLastError());
   if (s->profile) {
+    tsk::gemm_records_enable(nullptr);
     CU(cudaStreamSynchronize(s->cs));
+    s->gemm_flop.clear();
+    s->gemm_ms.clear();
+    s->gemm_batch.clear();
+    for (auto& r : s->gemm_recs) {
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, r.start, r.stop);
+      s->gemm_flop.push_back(r.tc ? r.flop : 0.0);
+      s->gemm_ms.push_back(ms);
+      s->gemm_batch.push_back(r.batch);
+    }
     s->item_ms.assign(s->prog.size(), 0.f);
     for (auto& c : s->prog)
       if (c.kind == 0) cudaEventElapsedTime(&s->item_ms[c.item], s->prof_ev[2 * c.item], s->prof_ev[2 * c.item + 1]);
@@ -794,6 +816,18 @@ ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, 
   *n = s->item_ms.size();
   if (ms)
     for (uint64_t i = 0; i < s->item_ms.size() && i < cap; ++i) ms[i] = s->item_ms[i];
+  return TS_OK;
+}
+
+ts_status ts_session_gemm_times(const ts_session_t* s, double* flop, float* ms, int32_t* batch, uint64_t cap,
+                                uint64_t* n) {
+  if (!s || !n) return set_error("null argument"), TS_ERR_ARG;
+  *n = s->gemm_ms.size();
+  for (uint64_t i = 0; i < s->gemm_ms.size() && i < cap; ++i) {
+    if (flop) flop[i] = s->gemm_flop[i];
+    if (ms) ms[i] = float(s->gemm_ms[i]);
+    if (batch) batch[i] = s->gemm_batch[i];
+  }
   return TS_OK;
 }
 

@@ -116,6 +116,7 @@ def lib():
             "ts_session_launches": (i32, [vp, P(i64)]),
             "ts_session_profile_items": (i32, [vp, i32]),
             "ts_session_item_times": (i32, [vp, P(C.c_float), u64, P(u64)]),
+            "ts_session_gemm_times": (i32, [vp, P(C.c_double), P(C.c_float), P(i32), u64, P(u64)]),
             "ts_profile_measure": (i32, [vp, vp, u64, P(vp), i32, i32, P(vp)]),
             "ts_profile_get": (i32, [vp, i32, i32, P(C.c_double), P(C.c_double)]),
             "ts_profile_pcie": (i32, [vp, P(C.c_double), P(C.c_double)]),
@@ -408,6 +409,16 @@ class Session:
         buf = (C.c_float * n.value)()
         check(lib().ts_session_item_times(self.h, buf, n.value, C.byref(n)))
         return list(buf)
+
+    def gemm_times(self):
+        """[(flop, ms, batch)] of every GEMM launch of the last profiled step."""
+        n = C.c_uint64()
+        check(lib().ts_session_gemm_times(self.h, None, None, None, 0, C.byref(n)))
+        f = (C.c_double * n.value)()
+        m = (C.c_float * n.value)()
+        b = (C.c_int32 * n.value)()
+        check(lib().ts_session_gemm_times(self.h, f, m, b, n.value, C.byref(n)))
+        return list(zip(f, m, b))
 
     def launches(self) -> int:
         n = C.c_int64()
