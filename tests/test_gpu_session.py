@@ -111,3 +111,36 @@ def test_sgd_step_changes_params_and_loss_drops():
     losses = [S.step(dev) for _ in range(5)]
     assert losses[-1] < losses[0]
     assert not np.allclose(S.param("fc0.w"), params["fc0.w"])
+
+
+def test_bert_large_full_size_properties():
+    """BERT-Large b32 s512 at the bench's 25% budget (properties that hold at any size):
+    the budgeted plan trains the same function as the all-reside plan (T1 on the GPU),
+    the runtime trace is the simulator's, the pool never exceeds the budget, and the
+    initial loss is the 2-class chance level ln 2."""
+    import math
+    g = graphs.config_graph("bert_large")
+    G = tsplit.Graph(g)
+    base = tsplit.Plan.default(G)
+    st = base.stats()
+    budget = st["static_bytes"] + (st["peak_extent"] - st["static_bytes"]) // 4
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    dev = tsplit.inputs_to_device(G, inputs)
+    P = tsplit.Plan.plan(G, budget)
+    assert P.stats()["peak_extent"] <= budget
+    S = tsplit.Session(G, P, slab_bytes=budget)
+    S.set_params(params)
+    l_b = S.step(dev)
+    g_b = S.grads()
+    assert S.trace() == P.trace()
+    del S
+    torch.cuda.empty_cache()
+    S0 = tsplit.Session(G, base)
+    S0.set_params(params)
+    l_0 = S0.step(dev)
+    g_0 = S0.grads()
+    del S0
+    torch.cuda.empty_cache()
+    assert abs(l_b - math.log(2.0)) < 0.05 and abs(l_0 - l_b) <= 1e-3 * abs(l_0)
+    assert all(np.isfinite(v).all() for v in g_b.values())
+    assert global_rel_err(g_b, g_0) <= 1e-2
