@@ -13,6 +13,7 @@ from __future__ import annotations
 import numpy as np
 
 from . import net, sim
+from . import ops as O
 
 F = np.float64
 
@@ -61,6 +62,12 @@ def execute(graph, cfg, params, inputs, step=0):
         arr = store[(n + t if grad else t, j)]
         return arr[(s0 - j * per) * r:(s1 - j * per) * r]
 
+    bn_stats, bn_sums = {}, {}
+
+    def whole(t, grad=False):
+        """All pieces of tensor t concatenated (the full batch)."""
+        return np.concatenate([store[(n + t if grad else t, j)] for j in range(p_of(t))], axis=0)
+
     for i, it in enumerate(items):
         for pc in f_alloc.get(i, []):
             key, j = pc
@@ -80,7 +87,26 @@ def execute(graph, cfg, params, inputs, step=0):
                 val[t] = view(t, s0, s1)
             row0 = s0 * rows_per_sample(out) if an.sample[out] else s0
             elem0 = s0 * (int(np.prod(ts[out]["shape"])) // B) if an.sample[out] else 0
-            if it.kind in ("F", "R"):
+            if o["kind"] == "batchnorm":
+                xin, gid, bid = o["inputs"]
+                eps = o["fattrs"][0]
+                if it.kind == "F" and it.k == 0:
+                    bn_stats[it.op] = O.batchnorm_stats(whole(xin))
+                mu, var = bn_stats[it.op]
+                if it.kind in ("F", "R"):
+                    view(out, s0, s1)[...] = O.batchnorm_fwd_with(val[xin], pval[gid], pval[bid], mu, var, eps)
+                else:
+                    if it.k == 0:
+                        sums = O.batchnorm_bwd_sums(whole(out, grad=True), whole(xin), pval[gid], mu, var, eps)
+                        bn_sums[it.op] = sums
+                        pgrad[gid] += sums[2]
+                        pgrad[bid] += sums[3]
+                    s1_, s2_ = bn_sums[it.op][:2]
+                    m = int(np.prod(ts[xin]["shape"][:-1]))
+                    if xin in an.needs_grad and ts[xin]["kind"] == "act":
+                        view(xin, s0, s1, grad=True)[...] += O.batchnorm_bwd_with(
+                            view(out, s0, s1, grad=True), val[xin], pval[gid], mu, var, s1_, s2_, m, eps)
+            elif it.kind in ("F", "R"):
                 y = net.forward_op(graph, o, val, row0=row0, elem0=elem0, step=step)
                 if an.is_loss[out]:
                     store[(out, 0)] += y

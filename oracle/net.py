@@ -52,6 +52,16 @@ def forward_op(graph, op, val, row0=0, elem0=0, step=0):
         return ops.cls_fwd(x[0], ia[0])
     if k == "xent":
         return np.array([ops.xent_fwd(x[0], x[1], graph["samples"])])
+    if k == "conv2d":
+        return ops.conv2d_fwd(x[0], x[1], x[2] if len(x) > 2 else None, ia[0], ia[1])
+    if k == "batchnorm":
+        return ops.batchnorm_fwd(x[0], x[1], x[2], fa[0])
+    if k == "maxpool":
+        return ops.maxpool_fwd(x[0], ia[0], ia[1], ia[2])
+    if k == "avgpool":
+        return ops.avgpool_fwd(x[0])
+    if k == "flatten":
+        return x[0].reshape(x[0].shape[0], -1).copy()
     raise ValueError(k)
 
 
@@ -97,6 +107,22 @@ def backward_op(graph, op, val, dy, row0=0, elem0=0, step=0):
         out = {ins[0]: ops.cls_bwd(dy, ia[0], rows)}
     elif k == "xent":
         out = {ins[0]: ops.xent_bwd(x[0], x[1], graph["samples"])}
+    elif k == "conv2d":
+        dx, dw, db = ops.conv2d_bwd(dy, x[0], x[1], ia[0], ia[1])
+        out = {ins[0]: dx, ins[1]: dw}
+        if len(ins) > 2:
+            out[ins[2]] = db
+    elif k == "batchnorm":
+        dx, dg, db = ops.batchnorm_bwd(dy, x[0], x[1], fa[0])
+        out = {ins[0]: dx, ins[1]: dg, ins[2]: db}
+    elif k == "maxpool":
+        out = {ins[0]: ops.maxpool_bwd(dy, x[0], ia[0], ia[1], ia[2])}
+    elif k == "avgpool":
+        shape = (dy.shape[0],) + tuple(graph["tensors"][ins[0]]["shape"][1:])
+        out = {ins[0]: ops.avgpool_bwd(dy, shape)}
+    elif k == "flatten":
+        shape = (dy.shape[0],) + tuple(graph["tensors"][ins[0]]["shape"][1:])
+        out = {ins[0]: dy.reshape(shape).copy()}
     else:
         raise ValueError(k)
     return out

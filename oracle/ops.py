@@ -222,3 +222,131 @@ def xent_bwd(z, labels, b_global):
     dz = softmax_fwd(z)
     dz[np.arange(z.shape[0]), labels] -= 1.0
     return dz / b_global
+
+
+# ---------------------------------------------------------------------------
+# CNN ops (configs 2-3).  NHWC activations, KRSC weights; conv via im2col.
+# ---------------------------------------------------------------------------
+
+def _im2col(x, R, S, stride, pad):
+    """x [N,H,W,C] -> cols [N,P,Q,R,S,C] (zero padding)."""
+    N, H, W, C = x.shape
+    P = (H + 2 * pad - R) // stride + 1
+    Q = (W + 2 * pad - S) // stride + 1
+    xp = np.pad(x, ((0, 0), (pad, pad), (pad, pad), (0, 0)))
+    cols = np.empty((N, P, Q, R, S, C), x.dtype)
+    for r in range(R):
+        for s in range(S):
+            cols[:, :, :, r, s, :] = xp[:, r:r + stride * P:stride, s:s + stride * Q:stride, :]
+    return cols
+
+
+def conv2d_fwd(x, w, b, stride, pad):
+    """Y[n,p,q,k] = sum_{r,s,c} X[n, p*st+r-pad, q*st+s-pad, c] W[k,r,s,c] (+ b[k])."""
+    K, R, S, C = w.shape
+    cols = _im2col(x, R, S, stride, pad)
+    N, P, Q = cols.shape[:3]
+    y = cols.reshape(N * P * Q, R * S * C) @ w.reshape(K, R * S * C).T
+    if b is not None:
+        y = y + b
+    return y.reshape(N, P, Q, K)
+
+
+def conv2d_bwd(dy, x, w, stride, pad):
+    """dX (col2im of dY W), dW = dY^T cols, db = sum dY."""
+    K, R, S, C = w.shape
+    N, H, W_, _ = x.shape
+    cols = _im2col(x, R, S, stride, pad)
+    _, P, Q = cols.shape[:3]
+    dy2 = dy.reshape(N * P * Q, K)
+    dw = (dy2.T @ cols.reshape(N * P * Q, R * S * C)).reshape(K, R, S, C)
+    dcols = (dy2 @ w.reshape(K, R * S * C)).reshape(N, P, Q, R, S, C)
+    dxp = np.zeros((N, H + 2 * pad, W_ + 2 * pad, C), F)
+    for r in range(R):
+        for s in range(S):
+            dxp[:, r:r + stride * P:stride, s:s + stride * Q:stride, :] += dcols[:, :, :, r, s, :]
+    dx = dxp[:, pad:pad + H, pad:pad + W_, :]
+    return dx, dw, dy2.sum(axis=0)
+
+
+def batchnorm_fwd(x, g, b, eps):
+    """Train-mode BN over (N,H,W) per channel, biased variance."""
+    mu = x.mean(axis=(0, 1, 2))
+    var = ((x - mu) ** 2).mean(axis=(0, 1, 2))
+    return (x - mu) / np.sqrt(var + eps) * g + b
+
+
+def batchnorm_bwd(dy, x, g, eps):
+    mu = x.mean(axis=(0, 1, 2))
+    var = ((x - mu) ** 2).mean(axis=(0, 1, 2))
+    rstd = 1.0 / np.sqrt(var + eps)
+    xhat = (x - mu) * rstd
+    dxhat = dy * g
+    m = x.shape[0] * x.shape[1] * x.shape[2]
+    dx = rstd * (dxhat - dxhat.sum(axis=(0, 1, 2)) / m - xhat * (dxhat * xhat).sum(axis=(0, 1, 2)) / m)
+    return dx, (dy * xhat).sum(axis=(0, 1, 2)), dy.sum(axis=(0, 1, 2))
+
+
+def maxpool_fwd(x, k, stride, pad):
+    """Max over k x k windows; padding never wins (-inf)."""
+    N, H, W, C = x.shape
+    P = (H + 2 * pad - k) // stride + 1
+    Q = (W + 2 * pad - k) // stride + 1
+    xp = np.pad(x, ((0, 0), (pad, pad), (pad, pad), (0, 0)), constant_values=-np.inf)
+    y = np.full((N, P, Q, C), -np.inf)
+    for r in range(k):
+        for s in range(k):
+            y = np.maximum(y, xp[:, r:r + stride * P:stride, s:s + stride * Q:stride, :])
+    return y
+
+
+def maxpool_bwd(dy, x, k, stride, pad):
+    """Gradient to the first maximum in row-major window order."""
+    N, H, W, C = x.shape
+    P, Q = dy.shape[1], dy.shape[2]
+    xp = np.pad(x, ((0, 0), (pad, pad), (pad, pad), (0, 0)), constant_values=-np.inf)
+    y = maxpool_fwd(x, k, stride, pad)
+    taken = np.zeros(dy.shape, bool)
+    dxp = np.zeros(xp.shape, F)
+    for r in range(k):
+        for s in range(k):
+            win = xp[:, r:r + stride * P:stride, s:s + stride * Q:stride, :]
+            hit = (win == y) & ~taken
+            dxp[:, r:r + stride * P:stride, s:s + stride * Q:stride, :] += np.where(hit, dy, 0.0)
+            taken |= hit
+    return dxp[:, pad:pad + H, pad:pad + W, :]
+
+
+def avgpool_fwd(x):
+    """Global average pool [N,H,W,C] -> [N,C]."""
+    return x.mean(axis=(1, 2))
+
+
+def avgpool_bwd(dy, shape):
+    N, H, W, C = shape
+    return np.broadcast_to(dy[:, None, None, :] / (H * W), shape).copy()
+
+
+def batchnorm_stats(x):
+    """Full-batch mean and biased variance per channel of x [...,C]."""
+    ax = tuple(range(x.ndim - 1))
+    mu = x.mean(axis=ax)
+    return mu, ((x - mu) ** 2).mean(axis=ax)
+
+
+def batchnorm_fwd_with(x, g, b, mu, var, eps):
+    """Normalise a block of samples with the full-batch statistics (R13)."""
+    return (x - mu) / np.sqrt(var + eps) * g + b
+
+
+def batchnorm_bwd_sums(dy, x, g, mu, var, eps):
+    """Full-batch sums for the BN backward: sum(dy*g), sum(dy*g*xhat), dgamma, dbeta."""
+    ax = tuple(range(x.ndim - 1))
+    xhat = (x - mu) / np.sqrt(var + eps)
+    return (dy * g).sum(axis=ax), (dy * g * xhat).sum(axis=ax), (dy * xhat).sum(axis=ax), dy.sum(axis=ax)
+
+
+def batchnorm_bwd_with(dy, x, g, mu, var, s1, s2, m, eps):
+    rstd = 1.0 / np.sqrt(var + eps)
+    xhat = (x - mu) * rstd
+    return rstd * (dy * g - s1 / m - xhat * s2 / m)

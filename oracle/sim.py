@@ -46,7 +46,20 @@ SAVED = {
     "embed": ("in", 0, 1),
     "cls": None,
     "xent": ("in", 0, 1),
+    "conv2d": ("in", 0),
+    "batchnorm": ("in", 0),
+    "maxpool": ("in", 0),
+    "avgpool": None,
+    "flatten": None,
 }
+
+# Ops whose statistics span the whole batch ("the merge of
+# micro-tensors can be required by the operation (e.g., batch normalization)"):
+# their first forward micro-op reads every piece of the input (full-batch mean and
+# variance), their first backward micro-op every piece of the input and of the
+# output gradient (full-batch sums of dy and dy*xhat); the statistics live in a
+# static per-op buffer, so replays and later micro-ops read only their own piece.
+BATCH_REDUCE = {"batchnorm"}
 
 
 def align(n):
@@ -77,7 +90,12 @@ def static_bytes(graph):
             total += align(2 * n)
         if len(t["shape"]) == 1:
             max1d = max(max1d, n)
-    return total + align(WS_ROWS * 2 * max1d * 4)
+    bn = 0
+    for o in graph["ops"]:
+        if o["kind"] in BATCH_REDUCE:
+            C = graph["tensors"][o["inputs"][0]]["shape"][-1]
+            bn += align(16 * C)  # [mean, rstd] (forward) + [sum dy, sum dy*xhat] (backward), fp32
+    return total + align(WS_ROWS * 2 * max1d * 4) + bn
 
 
 def schedule(graph):
@@ -258,6 +276,11 @@ def expand(graph, cfg, order=None, an=None):
         for k in range(P):
             it = Item("F", o, k)
             it.reads = [(t, piece(t, k, P)) for t in ins_sample(o)]
+            if ops[o]["kind"] in BATCH_REDUCE and k == 0:
+                for t in ins_sample(o):
+                    for j in range(p_of(t)):
+                        if (t, j) not in it.reads:
+                            it.reads.append((t, j))
             it.writes = [(t, piece(t, k, P)) for t in ops[o]["outputs"]]
             items.append(it)
     fwd_end = len(items)
@@ -287,6 +310,11 @@ def expand(graph, cfg, order=None, an=None):
                 live_temp.add((t, j))
 
             saved_pieces = [(t, piece(t, k, P)) for t in an.saved[o]]
+            if ops[o]["kind"] in BATCH_REDUCE and k == 0:
+                for t in an.saved[o]:
+                    for j in range(p_of(t)):
+                        if (t, j) not in saved_pieces:
+                            saved_pieces.append((t, j))
             for (t, j) in saved_pieces:
                 need(t, j)
             b = Item("B", o, k, group=gid)
@@ -294,6 +322,10 @@ def expand(graph, cfg, order=None, an=None):
             for t in ops[o]["outputs"]:
                 if not an.is_loss[t]:
                     b.reads.append((n + t, piece(t, k, P)))
+                    if ops[o]["kind"] in BATCH_REDUCE and k == 0:
+                        for j in range(p_of(t)):
+                            if (n + t, j) not in b.reads:
+                                b.reads.append((n + t, j))
             for t in ops[o]["inputs"]:
                 if ts[t]["kind"] == "act" and t in an.needs_grad:
                     w = (n + t, piece(t, k, P))

@@ -35,12 +35,22 @@ def init_params(graph: dict, seed: int = 1) -> dict[str, np.ndarray]:
     """fp32 parameter values keyed by tensor name."""
     out = {}
     is_bert = graph["name"].startswith("bert")
+    is_cnn = graph["name"].startswith(("vgg", "resnet"))
     for t in graph["tensors"]:
         if t["kind"] != "param":
             continue
         name, shape = t["name"], t["shape"]
         r = _rng(seed, name)
-        if is_bert:
+        if is_cnn:
+            if len(shape) == 4:  # conv KRSC: Kaiming-normal, fan_in = R*S*C
+                v = np.sqrt(2.0 / (shape[1] * shape[2] * shape[3])) * r.standard_normal(shape)
+            elif len(shape) == 2:
+                v = np.sqrt(2.0 / shape[1]) * r.standard_normal(shape)
+            elif name.endswith(".bn.g"):
+                v = 1.0 + 0.1 * r.standard_normal(shape)
+            else:
+                v = 0.05 * r.standard_normal(shape)
+        elif is_bert:
             if name.endswith(".g"):
                 v = 1.0 + 0.05 * r.standard_normal(shape)
             else:
@@ -81,7 +91,7 @@ def make_inputs(graph: dict, seed: int = 0) -> dict[str, np.ndarray]:
                 out[name] = np.zeros(shape, np.int32)
             else:
                 out[name] = np.random.default_rng(2000 + seed).integers(0, classes, size=shape).astype(np.int32)
-        else:
+        else:  # MLP features / CNN images: N(0,1); labels uniform in [0, classes)
             if t["kind"] == "input":
                 v = np.random.default_rng(seed).standard_normal(shape).astype(np.float32)
                 if graph["dtype"] == "bf16":

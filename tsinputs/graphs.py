@@ -184,8 +184,107 @@ def config_graph(name: str, **over) -> dict:
         kw = dict(layers=2, hidden=128, heads=2, seq=64, batch=4, vocab=512)
         kw.update(over)
         return bert(**kw)
+    if name == "vgg16":
+        return vgg16(**over)
+    if name == "vgg_tiny":
+        kw = dict(batch=4, img=32, width=0.125, fc=64, classes=10,
+                  cfg=[64, "M", 128, "M", 256, 256, "M"])
+        kw.update(over)
+        return vgg16(**kw)
+    if name == "resnet50":
+        return resnet50(**over)
+    if name == "resnet_tiny":
+        kw = dict(batch=4, img=32, width=0.125, blocks=(1, 1), classes=10)
+        kw.update(over)
+        return resnet50(**kw)
     if name == "bert_scaled":
         kw = dict(layers=24, hidden=2560, heads=40, seq=512, batch=64)
         kw.update(over)
         return bert(**kw)
     raise KeyError(name)
+
+
+def _conv_out(h, k, stride, pad):
+    return (h + 2 * pad - k) // stride + 1
+
+
+def vgg16(batch=64, img=224, classes=1000, width=1.0, fc=4096, dtype="bf16", cfg=None) -> dict:
+    """Config 2 (BASELINE configs[1]): VGG-16 (13 conv3x3 + ReLU, 5 maxpool 2x2/2,
+    3 FC), NHWC activations, KRSC weights; `width` scales the channels (Table V's
+    parameter scale)."""
+    cfg = cfg or [64, 64, "M", 128, 128, "M", 256, 256, 256, "M", 512, 512, 512, "M", 512, 512, 512, "M"]
+    g = GraphBuilder(f"vgg16_b{batch}_i{img}_w{width}", dtype, batch)
+    x = g.tensor("image", (batch, img, img, 3), "input")
+    y = g.tensor("labels", (batch,), "label", dtype="i32")
+    h, c, li = img, 3, 0
+    for v in cfg:
+        if v == "M":
+            h = _conv_out(h, 2, 2, 0)
+            x = g.op("maxpool", f"pool{li}", [x], (batch, h, h, c), iattrs=[2, 2, 0])
+            continue
+        k = max(8, int(v * width))
+        w = g.param(f"conv{li}.w", (k, 3, 3, c))
+        b = g.param(f"conv{li}.b", (k,))
+        x = g.op("conv2d", f"conv{li}", [x, w, b], (batch, h, h, k), iattrs=[1, 1])
+        x = g.op("relu", f"relu{li}", [x], (batch, h, h, k))
+        c = k
+        li += 1
+    x = g.op("flatten", "flatten", [x], (batch, h * h * c))
+    dims = [h * h * c, fc, fc, classes]
+    for i in range(3):
+        w = g.param(f"fc{i}.w", (dims[i + 1], dims[i]))
+        b = g.param(f"fc{i}.b", (dims[i + 1],))
+        x = g.op("linear", f"fc{i}", [x, w, b], (batch, dims[i + 1]))
+        if i < 2:
+            x = g.op("relu", f"fcrelu{i}", [x], (batch, dims[i + 1]))
+    g.op("xent", "loss", [x, y], (1,), out_dtype="f32")
+    return g.done()
+
+
+def resnet50(batch=256, img=224, classes=1000, width=1.0, blocks=(3, 4, 6, 3), dtype="bf16") -> dict:
+    """Config 3 (BASELINE configs[2]): ResNet-50 v1.5 (stride on the 3x3 conv of each
+    stage's first bottleneck), conv without bias + train-mode BN, NHWC."""
+    g = GraphBuilder(f"resnet50_b{batch}_i{img}_w{width}", dtype, batch)
+    x = g.tensor("image", (batch, img, img, 3), "input")
+    y = g.tensor("labels", (batch,), "label", dtype="i32")
+    cnt = [0]
+
+    def conv_bn(name, x, cin, cout, k, stride, h, relu=True):
+        pad = k // 2
+        ho = _conv_out(h, k, stride, pad)
+        w = g.param(name + ".w", (cout, k, k, cin))
+        x = g.op("conv2d", name, [x, w], (batch, ho, ho, cout), iattrs=[stride, pad])
+        gm = g.param(name + ".bn.g", (cout,))
+        bt = g.param(name + ".bn.b", (cout,))
+        x = g.op("batchnorm", name + ".bn", [x, gm, bt], (batch, ho, ho, cout), fattrs=[1e-5])
+        if relu:
+            x = g.op("relu", name + ".relu", [x], (batch, ho, ho, cout))
+        return x, ho
+
+    c0 = max(8, int(64 * width))
+    x, h = conv_bn("stem", x, 3, c0, 7, 2, img)
+    h2 = _conv_out(h, 3, 2, 1)
+    x = g.op("maxpool", "stem.pool", [x], (batch, h2, h2, c0), iattrs=[3, 2, 1])
+    h, cin = h2, c0
+    for si, nb in enumerate(blocks):
+        mid = max(8, int(64 * width * 2 ** si))
+        cout = 4 * mid
+        for bi in range(nb):
+            stride = 2 if (bi == 0 and si > 0) else 1
+            p = f"s{si}b{bi}"
+            a, ha = conv_bn(p + ".c1", x, cin, mid, 1, 1, h)
+            a, hb = conv_bn(p + ".c2", a, mid, mid, 3, stride, ha)
+            a, hc = conv_bn(p + ".c3", a, mid, cout, 1, 1, hb, relu=False)
+            if bi == 0:
+                sc, _ = conv_bn(p + ".down", x, cin, cout, 1, stride, h, relu=False)
+            else:
+                sc = x
+            s = g.op("add", p + ".add", [a, sc], (batch, hc, hc, cout))
+            x = g.op("relu", p + ".relu", [s], (batch, hc, hc, cout))
+            h, cin = hc, cout
+    x = g.op("avgpool", "avgpool", [x], (batch, cin))
+    w = g.param("fc.w", (classes, cin))
+    b = g.param("fc.b", (classes,))
+    x = g.op("linear", "fc", [x, w, b], (batch, classes))
+    g.op("xent", "loss", [x, y], (1,), out_dtype="f32")
+    return g.done()
