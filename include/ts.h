@@ -62,8 +62,15 @@ typedef enum {
   TS_OP_ATTN_PV = 9,   /* in P[b,a,s,s], V[T,h] out C[T,h]; iattr {heads, seq}         */
   TS_OP_EMBED = 10,    /* in ids, type_ids (i32 [T]), Wword, Wpos, Wtype; iattr[0] = seq */
   TS_OP_CLS = 11,      /* in X[T,h] out [b,h] (row b*seq); iattr[0] = seq              */
-  TS_OP_XENT = 12      /* in logits[b,C], labels i32[b] out loss f32[1], mean over the
+  TS_OP_XENT = 12,     /* in logits[b,C], labels i32[b] out loss f32[1], mean over the
                           global batch                                     */
+  TS_OP_CONV2D = 13,   /* in X[N,H,W,C] (NHWC), W[K,R,S,C] (KRSC), [b[K]] out Y[N,P,Q,K];
+                          iattr {stride, pad}                                           */
+  TS_OP_BATCHNORM = 14,/* in X[...,C], gamma[C], beta[C]; fattr[0] = eps; train-mode
+                          batch statistics over all samples even when split (R13)      */
+  TS_OP_MAXPOOL = 15,  /* in X[N,H,W,C] out [N,P,Q,C]; iattr {k, stride, pad}           */
+  TS_OP_AVGPOOL = 16,  /* global average: in X[N,H,W,C] out [N,C]                       */
+  TS_OP_FLATTEN = 17   /* in X[N,...] out [N, prod(...)] (copy)                          */
 } ts_op_kind;
 
 typedef struct {

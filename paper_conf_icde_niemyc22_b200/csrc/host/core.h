@@ -17,6 +17,8 @@ constexpr uint64_t kWsRows = 256;
 constexpr uint64_t kInf = uint64_t(1) << 62;
 
 inline uint64_t align_up(uint64_t n) { return (n + kAlign - 1) / kAlign * kAlign; }
+// Ops whose statistics span the whole batch (R13): first micro-op reads every piece.
+inline bool batch_reduce(int kind) { return kind == TS_OP_BATCHNORM; }
 inline int dtype_bytes(int d) { return d == TS_BF16 ? 2 : 4; }
 
 void set_error(const std::string& msg);
@@ -53,6 +55,7 @@ struct Graph {
   // static region layout: masters | bf16 copies | grads | workspace
   std::vector<uint64_t> master_off, copy_off, grad_off;
   uint64_t ws_off = 0, ws_bytes = 0, static_bytes = 0;
+  std::vector<uint64_t> bn_off;  // per op: [mean, rstd | sum dy*g, sum dy*g*xhat] fp32 (batch-stat ops)
   int n() const { return (int)t.size(); }
 };
 

@@ -55,6 +55,11 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
       it.k = k;
       for (int x : op.in)
         if (g.t[x].sample) it.reads.push_back(pk(x, piece(x, k, P)));
+      if (batch_reduce(op.kind) && k == 0)  // full-batch statistics (R13)
+        for (int x : op.in)
+          if (g.t[x].sample)
+            for (int j = 0; j < piece_count(g, cfg, x); ++j)
+              if (std::find(it.reads.begin(), it.reads.end(), pk(x, j)) == it.reads.end()) it.reads.push_back(pk(x, j));
       for (int x : op.out) it.writes.push_back(pk(x, piece(x, k, P)));
       items.push_back(std::move(it));
     }
@@ -93,6 +98,10 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
       };
       std::vector<PieceKey> saved;
       for (int t : op.saved) saved.push_back(pk(t, piece(t, k, P)));
+      if (batch_reduce(op.kind) && k == 0)
+        for (int t : op.saved)
+          for (int j = 0; j < piece_count(g, cfg, t); ++j)
+            if (std::find(saved.begin(), saved.end(), pk(t, j)) == saved.end()) saved.push_back(pk(t, j));
       for (PieceKey s : saved) regen(pk_key(s), pk_j(s));
       Item b;
       b.kind = IT_B;
@@ -101,7 +110,13 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
       b.group = gid;
       b.reads = saved;
       for (int x : op.out)
-        if (!g.t[x].is_loss) b.reads.push_back(pk(n + x, piece(x, k, P)));
+        if (!g.t[x].is_loss) {
+          b.reads.push_back(pk(n + x, piece(x, k, P)));
+          if (batch_reduce(op.kind) && k == 0)
+            for (int j = 0; j < piece_count(g, cfg, x); ++j)
+              if (std::find(b.reads.begin(), b.reads.end(), pk(n + x, j)) == b.reads.end())
+                b.reads.push_back(pk(n + x, j));
+        }
       for (int x : op.in)
         if (g.t[x].kind == TS_ACT && g.t[x].needs_grad) {
           PieceKey w = pk(n + x, piece(x, k, P));

@@ -107,6 +107,50 @@ bool validate_op(const Graph& g, const Op& o, std::string& why) {
         return (why = "cls shapes"), false;
       return true;
     }
+    case TS_OP_CONV2D: {
+      if ((o.in.size() != 2 && o.in.size() != 3) || o.out.size() != 1) return (why = "conv2d in/out"), false;
+      const Tensor &x = T(o.in[0]), &w = T(o.in[1]), &y = T(o.out[0]);
+      if (o.ia.size() < 2 || o.ia[0] < 1 || o.ia[1] < 0) return (why = "conv2d attrs {stride, pad}"), false;
+      if (x.ndim != 4 || w.ndim != 4 || y.ndim != 4 || w.kind != TS_PARAM) return (why = "conv2d ranks"), false;
+      const int64_t st = o.ia[0], pd = o.ia[1];
+      const int64_t P = (x.shape[1] + 2 * pd - w.shape[1]) / st + 1, Q = (x.shape[2] + 2 * pd - w.shape[2]) / st + 1;
+      if (w.shape[3] != x.shape[3] || y.shape[0] != x.shape[0] || y.shape[1] != P || y.shape[2] != Q ||
+          y.shape[3] != w.shape[0])
+        return (why = "conv2d shapes"), false;
+      if (o.in.size() == 3 && (T(o.in[2]).numel != w.shape[0] || T(o.in[2]).kind != TS_PARAM))
+        return (why = "conv2d bias"), false;
+      return true;
+    }
+    case TS_OP_BATCHNORM: {
+      if (!need(3, 1)) return false;
+      const Tensor& x = T(o.in[0]);
+      if (!same_shape(x, T(o.out[0])) || T(o.in[1]).numel != last(x) || T(o.in[2]).numel != last(x) || o.fa.empty())
+        return (why = "batchnorm shapes/eps"), false;
+      return true;
+    }
+    case TS_OP_MAXPOOL: {
+      if (!need(1, 1)) return false;
+      const Tensor &x = T(o.in[0]), &y = T(o.out[0]);
+      if (o.ia.size() < 3 || x.ndim != 4 || y.ndim != 4) return (why = "maxpool attrs/ranks"), false;
+      const int64_t k = o.ia[0], st = o.ia[1], pd = o.ia[2];
+      if (y.shape[1] != (x.shape[1] + 2 * pd - k) / st + 1 || y.shape[2] != (x.shape[2] + 2 * pd - k) / st + 1 ||
+          y.shape[3] != x.shape[3] || y.shape[0] != x.shape[0])
+        return (why = "maxpool shapes"), false;
+      return true;
+    }
+    case TS_OP_AVGPOOL: {
+      if (!need(1, 1)) return false;
+      const Tensor &x = T(o.in[0]), &y = T(o.out[0]);
+      if (x.ndim != 4 || y.ndim != 2 || y.shape[0] != x.shape[0] || y.shape[1] != x.shape[3])
+        return (why = "avgpool shapes"), false;
+      return true;
+    }
+    case TS_OP_FLATTEN: {
+      if (!need(1, 1)) return false;
+      const Tensor &x = T(o.in[0]), &y = T(o.out[0]);
+      if (y.ndim != 2 || y.shape[0] != x.shape[0] || y.numel != x.numel) return (why = "flatten shapes"), false;
+      return true;
+    }
     case TS_OP_XENT: {
       if (!need(2, 1)) return false;
       const Tensor &z = T(o.in[0]), &l = T(o.in[1]), &y = T(o.out[0]);
@@ -124,7 +168,10 @@ bool validate_op(const Graph& g, const Op& o, std::string& why) {
 std::vector<int> saved_of(const Graph& g, const Op& o) {
   std::vector<int> src;
   switch (o.kind) {
-    case TS_OP_LINEAR: case TS_OP_GELU: case TS_OP_LAYERNORM: src = {o.in[0]}; break;
+    case TS_OP_LINEAR: case TS_OP_GELU: case TS_OP_LAYERNORM: case TS_OP_CONV2D: case TS_OP_BATCHNORM:
+    case TS_OP_MAXPOOL:
+      src = {o.in[0]};
+      break;
     case TS_OP_RELU: case TS_OP_TANH: case TS_OP_SOFTMAX: src = {o.out[0]}; break;
     case TS_OP_ATTN_QK: case TS_OP_ATTN_PV: case TS_OP_EMBED: case TS_OP_XENT: src = {o.in[0], o.in[1]}; break;
     default: break;
@@ -291,7 +338,14 @@ ts_status build_graph(const ts_tensor_desc* td, int nt, const ts_op_desc* od, in
     }
   g.ws_off = off;
   g.ws_bytes = align_up(kWsRows * 2 * uint64_t(max1d) * 4);
-  g.static_bytes = off + g.ws_bytes;
+  off += g.ws_bytes;
+  g.bn_off.assign(no, 0);
+  for (auto& o : g.ops)
+    if (batch_reduce(o.kind)) {
+      g.bn_off[o.id] = off;
+      off += align_up(16 * uint64_t(g.t[o.in[0]].shape[g.t[o.in[0]].ndim - 1]));
+    }
+  g.static_bytes = off;
   return TS_OK;
 }
 

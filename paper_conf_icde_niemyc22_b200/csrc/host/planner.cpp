@@ -79,6 +79,22 @@ OpCost op_cost(const Graph& g, int oi) {
       c.bytes_f = 2 * nb(o.in[0]);
       c.bytes_b = 2 * nb(o.in[0]);
       break;
+    case TS_OP_CONV2D: {
+      const Tensor &w = g.t[o.in[1]], &y = g.t[o.out[0]];
+      const double rsc = double(w.shape[1]) * w.shape[2] * w.shape[3];
+      c.flop_f = 2.0 * double(y.numel) * rsc;
+      c.flop_b = 2 * c.flop_f;
+      c.bytes_f = nb(o.in[0]) + nb(o.out[0]) + double(w.numel) * es;
+      c.bytes_b = 2 * nb(o.in[0]) + 2 * nb(o.out[0]) + 8.0 * w.numel;
+      c.kern_b = 2;
+      break;
+    }
+    case TS_OP_BATCHNORM:
+      c.bytes_f = 3 * nb(o.in[0]);
+      c.bytes_b = 5 * nb(o.in[0]);
+      c.kern_f = 2;
+      c.kern_b = 2;
+      break;
     default:  // elementwise / row ops
       c.bytes_f = nb(o.in[0]) + nb(o.out[0]);
       c.bytes_b = 3 * nb(o.out[0]);

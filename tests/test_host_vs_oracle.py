@@ -137,3 +137,23 @@ def test_planner_bert_large_quarter_budget():
     st = P.stats()
     assert st["peak_extent"] <= budget
     assert st["n_recompute_tensors"] + st["n_swap_tensors"] > 0
+
+
+@pytest.mark.parametrize("gname", ["vgg_tiny", "resnet_tiny", "vgg16", "resnet50"])
+def test_cnn_schedule_static_and_default_trace(gname):
+    g = graphs.config_graph(gname)
+    G = tsplit.Graph(g)
+    assert G.schedule() == sim.schedule(g)
+    assert G.static_bytes() == sim.static_bytes(g)
+    if gname.endswith("tiny"):
+        _compare(g, sim.default_cfg(g))
+
+
+@pytest.mark.parametrize("gname,seed", [("vgg_tiny", 0), ("vgg_tiny", 1), ("resnet_tiny", 0), ("resnet_tiny", 1)])
+def test_cnn_trace_bit_exact_random_plans(gname, seed):
+    g = graphs.config_graph(gname)
+    r = random.Random(seed)
+    cfg = sim.default_cfg(g)
+    for t in brute.act_tensors(g):
+        cfg[t] = (r.choice([0, 1, 2]), r.choice([1, 2, 4]), r.choice([1, 2]))
+    _compare(g, cfg)
