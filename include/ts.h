@@ -272,6 +272,21 @@ ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K,
                       const float* B, int64_t ldb, int32_t tb,
                       float* C, int64_t ldc, float alpha, float beta, const float* bias, void* stream);
 
+/* Convolution micro-op kernels (unit tests; the session uses the same ones).
+ * Cites: SURVEY.md §8(a) a6/a8 (C2/C3 conv as implicit GEMM), P:L260 (a micro-op
+ * is a block of samples; dW merges by summation).  Layout: x [n,H,W,C] (NHWC),
+ * w [K,R,S,C] (KRSC), y / dy [n,P,Q,K] with P = (H + 2 pad - R)/stride + 1 (same
+ * for Q).  geom = {n, H, W, C, K, R, S, stride, pad}; all device pointers.
+ *   mode 1 fprop: out = y (graph dtype) = conv(x, w) (+ bias[K], may be NULL)
+ *   mode 2 dgrad: out = dx (graph dtype) (+)= conv_transpose(dy, w)   (acc != 0 adds)
+ *   mode 3 wgrad: out = dw (fp32 [K,R,S,C]) (+)= sum over pixels of dy (x) im2col(x)
+ * dtype TS_BF16: tcgen05/TMEM implicit GEMM with cp.async gathers (fp32 accumulate)
+ * when eligible (K % 8 == 0; dgrad also C % 8 == 0), else CUDA cores; TS_F32: CUDA
+ * cores with fp64 accumulation.  *used_tc (may be NULL) reports the path taken.
+ * Errors: TS_ERR_ARG for bad geometry, TS_ERR_CUDA for launch failures. */
+ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void* x, const void* w, const void* dy,
+                    void* out, const void* bias, int32_t acc, void* stream, int32_t* used_tc);
+
 #ifdef __cplusplus
 }
 #endif

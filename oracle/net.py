@@ -148,13 +148,23 @@ def initial_values(graph, params, inputs):
     return val
 
 
-def train_step(graph, params, inputs, step=0):
-    """Unsplit fp64 forward + backward.  Returns (loss, {param name: grad})."""
+def train_step(graph, params, inputs, step=0, storage=None):
+    """Unsplit fp64 forward + backward.  Returns (loss, {param name: grad}).
+
+    storage="bf16": every stored activation and activation gradient is rounded to
+    bf16 (ops.round_bf16) where it is written — after each forward op and after
+    each gradient contribution is added — while the arithmetic inside an op stays
+    fp64.  That is the precision a bf16-storage / fp32-compute implementation
+    keeps, so its gradients are compared against this reading
+    (DESIGN.md D-TOL); parameter gradients are never rounded (fp32 masters)."""
+    rnd = ops.round_bf16 if storage == "bf16" else (lambda a: a)
     val = initial_values(graph, params, inputs)
-    for op in graph["ops"]:
-        val[op["outputs"][0]] = forward_op(graph, op, val, step=step)
     loss_id = next(op["outputs"][0] for op in graph["ops"] if op["kind"] == "xent")
+    for op in graph["ops"]:
+        y = forward_op(graph, op, val, step=step)
+        val[op["outputs"][0]] = y if op["outputs"][0] == loss_id else rnd(y)
     ng = needs_grad(graph)
+    is_act = {t["id"] for t in graph["tensors"] if t["kind"] == "act"}
     grad = {}
     for op in reversed(graph["ops"]):
         o = op["outputs"][0]
@@ -165,6 +175,8 @@ def train_step(graph, params, inputs, step=0):
             if tid not in ng:
                 continue
             grad[tid] = grad[tid] + g if tid in grad else g
+            if tid in is_act:
+                grad[tid] = rnd(grad[tid])
     pg = {t["name"]: grad.get(t["id"], np.zeros(t["shape"]))
           for t in graph["tensors"] if t["kind"] == "param"}
     return float(val[loss_id][0]), pg, val, grad

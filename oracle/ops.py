@@ -20,6 +20,17 @@ from scipy.special import erf
 
 F = np.float64
 
+
+def round_bf16(x):
+    """Storage precision of bf16 graphs (DESIGN.md D-TOL):
+    the value a kernel that computes in fp32 stores as bf16 — fp64 -> nearest fp32
+    -> nearest bf16 (round to nearest, ties to even on the 16 dropped bits).
+    Returned widened to fp64."""
+    b = np.ascontiguousarray(np.asarray(x, np.float64).astype(np.float32)).view(np.uint32).astype(np.uint64)
+    b = (b + np.uint64(0x7FFF) + ((b >> np.uint64(16)) & np.uint64(1))) & np.uint64(0xFFFF0000)
+    return b.astype(np.uint32).view(np.float32).astype(F)
+
+
 # ---------------------------------------------------------------------------
 # Philox4x32-10 counter-based RNG (Salmon et al., SC'11), SURVEY.md §8(c) R15.
 # Element idx draws word (idx & 3) of Philox(counter = (c_lo, c_hi, step, 0),

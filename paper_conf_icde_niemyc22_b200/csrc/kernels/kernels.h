@@ -44,8 +44,61 @@ struct GemmRecord {
   cudaEvent_t start, stop;
   double flop;
   int M, N, K, batch, tc;
+  int kind;  // 0 GEMM, 1 conv fprop, 2 conv dgrad, 3 conv wgrad
 };
 void gemm_records_enable(std::vector<GemmRecord>* sink);
+std::vector<GemmRecord>* gemm_records_sink();
+
+// ---- convolution (NHWC activations, KRSC weights; one micro-op = n samples) ------
+// Implicit GEMM (conv_tc.cu): fprop M = n*P*Q, N = K, Kg = R*S*C; dgrad M = n*H*W,
+// N = C, Kg = R*S*K; wgrad M = R*S*C, N = K, Kg = n*P*Q (split-K, fp32 out).
+struct ConvArgs {
+  int dtype = BF16;
+  int n = 0, H = 0, W = 0, C = 0, K = 0, R = 0, S = 0, P = 0, Q = 0, stride = 1, pad = 0;
+  const void* x = nullptr;   // [n,H,W,C]
+  const void* w = nullptr;   // [K,R,S,C]
+  const void* dy = nullptr;  // [n,P,Q,K]
+};
+// y[n,P,Q,K] = conv(x, w) (+ bias[K]) — bias in the graph dtype
+void conv_fprop(const ConvArgs& a, void* y, const void* bias, cudaStream_t st);
+// dx[n,H,W,C] (+)= conv_transpose(dy, w)
+void conv_dgrad(const ConvArgs& a, void* dx, int acc, cudaStream_t st);
+// dw[K,R,S,C] (fp32) (+)= sum over the micro-op's pixels of dy (x) im2col(x)
+void conv_wgrad(const ConvArgs& a, float* dw, int acc, cudaStream_t st);
+// tcgen05 path; false when the shape/alignment is not eligible (then SIMT)
+bool conv_tc(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
+void conv_simt(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
+
+// ---- batch normalisation over all pieces of a split tensor ----------
+// A piece list: `np` pointers, each holding `rows[i]` rows of C channels.
+struct PieceList {
+  static constexpr int kMax = 16;
+  const void* ptr[kMax];
+  int64_t rows[kMax];
+  int np = 0;
+};
+bool bn_supported(int dt, int C);  // whole 16-byte channel vectors, <= 256 vectors per row
+// stats[0:C] = mean, stats[C:2C] = rstd over every row of every piece (fp64 final reduce)
+void bn_stats(int dt, const PieceList& x, int C, float eps, float* ws, uint64_t ws_bytes, float* stats,
+              cudaStream_t st);
+// y = (x - mean) * rstd * gamma + beta on one micro-op's rows
+void bn_apply(int dt, const void* x, const float* stats, const void* gamma, const void* beta, void* y, int64_t rows,
+              int C, cudaStream_t st);
+// full-batch sums: stats[2C:3C] = sum dy*gamma, stats[3C:4C] = sum dy*gamma*xhat;
+// dgamma (+)= sum dy*xhat, dbeta (+)= sum dy
+void bn_bwd_sums(int dt, const PieceList& dy, const PieceList& x, const void* gamma, int C, float* ws,
+                 uint64_t ws_bytes, float* stats, float* dgamma, float* dbeta, int pacc, cudaStream_t st);
+// dx (+)= rstd * (dy*gamma - s1/m - xhat*s2/m), m = rows of the whole batch
+void bn_bwd_apply(int dt, const void* dy, const void* x, const float* stats, const void* gamma, void* dx, int acc,
+                  int64_t rows, int C, int64_t m_total, cudaStream_t st);
+// ---- pooling (NHWC) ----------------------------------------------------------------
+void maxpool_fwd(int dt, const void* x, void* y, int n, int H, int W, int C, int P, int Q, int k, int stride,
+                 int pad, cudaStream_t st);
+// gradient to the first maximum of each window in row-major order
+void maxpool_bwd(int dt, const void* dy, const void* x, void* dx, int acc, int n, int H, int W, int C, int P, int Q,
+                 int k, int stride, int pad, cudaStream_t st);
+void avgpool_fwd(int dt, const void* x, void* y, int n, int HW, int C, cudaStream_t st);
+void avgpool_bwd(int dt, const void* dy, void* dx, int acc, int n, int HW, int C, cudaStream_t st);
 
 // ---- elementwise (n elements, dtype F32/BF16 for activations) ----------------
 void relu_fwd(int dt, const void* x, void* y, int64_t n, cudaStream_t st);

@@ -96,7 +96,9 @@ float* param_g(ts_session_t* s, int t) { return reinterpret_cast<float*>(s->slab
 
 struct Micro {
   int op, k, P;
+  bool replay = false;
   int64_t s0, s1;
+  tsk::PieceList all_x, all_dy;  // batch-statistics ops at k = 0: every piece (R13)
   std::unordered_map<int, char*> val, grad;
   std::unordered_map<int, int> acc;  // grad key -> accumulate flag
 };
@@ -351,6 +353,112 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       int acc = A(g.n() + o.in[0]);
       return [=](cudaStream_t st) { tsk::cls_bwd(dt, dy, dx, acc, ns, seq, H, st); };
     }
+    case TS_OP_CONV2D: {
+      const Tensor& x = g.t[o.in[0]];
+      const Tensor& w = g.t[o.in[1]];
+      tsk::ConvArgs a;
+      a.dtype = dt;
+      a.n = int(ns);
+      a.H = int(x.shape[1]); a.W = int(x.shape[2]); a.C = int(x.shape[3]);
+      a.K = int(w.shape[0]); a.R = int(w.shape[1]); a.S = int(w.shape[2]);
+      a.P = int(out.shape[1]); a.Q = int(out.shape[2]);
+      a.stride = int(o.ia[0]); a.pad = int(o.ia[1]);
+      a.w = param_w(s, o.in[1]);
+      const bool has_bias = o.in.size() > 2;
+      if (!bwd) {
+        a.x = V(o.in[0]);
+        char* y = V(o.out[0]);
+        const void* bias = has_bias ? param_w(s, o.in[2]) : nullptr;
+        nk = 1;
+        return [a, y, bias](cudaStream_t st) { tsk::conv_fprop(a, y, bias, st); };
+      }
+      a.x = V(o.in[0]);
+      a.dy = G(o.out[0]);
+      char* dx = (x.kind == TS_ACT && x.needs_grad) ? G(o.in[0]) : nullptr;
+      const int dxacc = dx ? A(g.n() + o.in[0]) : 0;
+      float* dw = param_g(s, o.in[1]);
+      const int dwacc = A(o.in[1]);
+      float* db = has_bias ? param_g(s, o.in[2]) : nullptr;
+      const int dbacc = has_bias ? A(o.in[2]) : 0;
+      const int64_t pix = ns * int64_t(a.P) * a.Q;
+      const uint64_t wsb = g.ws_bytes;
+      nk = (dx ? 1 : 0) + 1 + (db ? 2 : 0);
+      return [=](cudaStream_t st) {
+        if (dx) tsk::conv_dgrad(a, dx, dxacc, st);
+        tsk::conv_wgrad(a, dw, dwacc, st);
+        if (db) tsk::column_sum(dt, a.dy, pix, a.K, ws, wsb, db, dbacc, nullptr, 0, st);
+      };
+    }
+    case TS_OP_BATCHNORM: {
+      const Tensor& x = g.t[o.in[0]];
+      const int C = int(x.shape[x.ndim - 1]);
+      const int64_t rows = n_out / C;
+      const int64_t m_total = out.numel / C;
+      float* bs = reinterpret_cast<float*>(s->slab + g.bn_off[o.id]);
+      char *gw = param_w(s, o.in[1]), *bw = param_w(s, o.in[2]);
+      const uint64_t wsb = g.ws_bytes;
+      if (!bwd) {
+        const float eps = float(o.fa[0]);
+        const bool stats = m.k == 0 && !m.replay;
+        const tsk::PieceList px = m.all_x;
+        char *xp = V(o.in[0]), *y = V(o.out[0]);
+        nk = stats ? 3 : 1;
+        return [=](cudaStream_t st) {
+          if (stats) tsk::bn_stats(dt, px, C, eps, ws, wsb, bs, st);
+          tsk::bn_apply(dt, xp, bs, gw, bw, y, rows, C, st);
+        };
+      }
+      const bool sums = m.k == 0;
+      const tsk::PieceList px = m.all_x, pdy = m.all_dy;
+      float *dg = param_g(s, o.in[1]), *dbt = param_g(s, o.in[2]);
+      const int pacc = A(o.in[1]);
+      char* dx = (x.kind == TS_ACT && x.needs_grad) ? G(o.in[0]) : nullptr;
+      const int acc = dx ? A(g.n() + o.in[0]) : 0;
+      char *dy = G(o.out[0]), *xp = V(o.in[0]);
+      nk = (sums ? 3 : 0) + (dx ? 1 : 0);
+      return [=](cudaStream_t st) {
+        if (sums) tsk::bn_bwd_sums(dt, pdy, px, gw, C, ws, wsb, bs, dg, dbt, pacc, st);
+        if (dx) tsk::bn_bwd_apply(dt, dy, xp, bs, gw, dx, acc, rows, C, m_total, st);
+      };
+    }
+    case TS_OP_MAXPOOL: {
+      const Tensor& x = g.t[o.in[0]];
+      const int H = int(x.shape[1]), W = int(x.shape[2]), C = int(x.shape[3]);
+      const int P = int(out.shape[1]), Q = int(out.shape[2]);
+      const int kk = int(o.ia[0]), st_ = int(o.ia[1]), pad = int(o.ia[2]);
+      const int nn = int(ns);
+      nk = 1;
+      if (!bwd) {
+        char *xp = V(o.in[0]), *y = V(o.out[0]);
+        return [=](cudaStream_t st) { tsk::maxpool_fwd(dt, xp, y, nn, H, W, C, P, Q, kk, st_, pad, st); };
+      }
+      char *dy = G(o.out[0]), *xp = V(o.in[0]), *dx = G(o.in[0]);
+      const int acc = A(g.n() + o.in[0]);
+      return [=](cudaStream_t st) { tsk::maxpool_bwd(dt, dy, xp, dx, acc, nn, H, W, C, P, Q, kk, st_, pad, st); };
+    }
+    case TS_OP_AVGPOOL: {
+      const Tensor& x = g.t[o.in[0]];
+      const int HW = int(x.shape[1] * x.shape[2]), C = int(x.shape[3]);
+      const int nn = int(ns);
+      nk = 1;
+      if (!bwd) {
+        char *xp = V(o.in[0]), *y = V(o.out[0]);
+        return [=](cudaStream_t st) { tsk::avgpool_fwd(dt, xp, y, nn, HW, C, st); };
+      }
+      char *dy = G(o.out[0]), *dx = G(o.in[0]);
+      const int acc = A(g.n() + o.in[0]);
+      return [=](cudaStream_t st) { tsk::avgpool_bwd(dt, dy, dx, acc, nn, HW, C, st); };
+    }
+    case TS_OP_FLATTEN: {
+      nk = 1;
+      if (!bwd) {
+        char *xp = V(o.in[0]), *y = V(o.out[0]);
+        return [=](cudaStream_t st) { tsk::axpy(dt, xp, y, 0, n_out, st); };
+      }
+      char *dy = G(o.out[0]), *dx = G(o.in[0]);
+      const int acc = A(g.n() + o.in[0]);
+      return [=](cudaStream_t st) { tsk::axpy(dt, dy, dx, acc, n_out, st); };
+    }
     case TS_OP_XENT: {
       const int C = int(g.t[o.in[0]].shape[1]);
       const float inv_b = 1.f / float(B);
@@ -496,6 +604,25 @@ ts_status build_program(ts_session_t* s) {
             m.acc[gk] = grad_first_op[gk] != it.op ? 1 : 0;
           }
         }
+      }
+      m.replay = it.kind == IT_R;
+      if (batch_reduce(o.kind) && it.k == 0 && it.kind != IT_R) {  // replays reuse the step's statistics
+        const int C = int(g.t[o.in[0]].shape[g.t[o.in[0]].ndim - 1]);
+        if (!tsk::bn_supported(g.dtype == TS_BF16 ? tsk::BF16 : tsk::F32, C))
+          return set_error("batchnorm: channel count " + std::to_string(C) + " not supported"), TS_ERR_GRAPH;
+        auto list = [&](int key, tsk::PieceList& L) -> bool {
+          int t = key >= n ? key - n : key;
+          int p = piece_count(g, s->cfg, t);
+          if (p > tsk::PieceList::kMax) return false;
+          L.np = p;
+          for (int j = 0; j < p; ++j) {
+            L.ptr[j] = s->slab + where.at(pk(key, j));
+            L.rows[j] = int64_t(B / p) * (g.t[t].elems_per_sample / C);
+          }
+          return true;
+        };
+        if (!list(o.in[0], m.all_x)) return set_error("batchnorm: too many pieces"), TS_ERR_GRAPH;
+        if (bwd && !list(n + o.out[0], m.all_dy)) return set_error("batchnorm: too many pieces"), TS_ERR_GRAPH;
       }
       int nk = 0;
       cmd.fn = lower(s, m, bwd, nk);
@@ -1007,6 +1134,30 @@ ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K, const float* A, int64_t l
   g.alpha = alpha; g.beta = beta; g.bias = bias; g.bias_dtype = tsk::F32;
   tsk::gemm_simt(g, static_cast<cudaStream_t>(stream));
   CU(cudaGetLastError());
+  return TS_OK;
+}
+
+ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void* x, const void* w, const void* dy,
+                    void* out, const void* bias, int32_t acc, void* stream, int32_t* used_tc) {
+  if (!geom || mode < 1 || mode > 3 || (dtype != TS_BF16 && dtype != TS_F32) || !w || !out)
+    return set_error("ts_conv2d: bad argument"), TS_ERR_ARG;
+  tsk::ConvArgs a;
+  a.dtype = dtype == TS_BF16 ? tsk::BF16 : tsk::F32;
+  a.n = geom[0]; a.H = geom[1]; a.W = geom[2]; a.C = geom[3]; a.K = geom[4]; a.R = geom[5]; a.S = geom[6];
+  a.stride = geom[7]; a.pad = geom[8];
+  if (a.n < 1 || a.H < 1 || a.W < 1 || a.C < 1 || a.K < 1 || a.R < 1 || a.S < 1 || a.stride < 1 || a.pad < 0)
+    return set_error("ts_conv2d: bad geometry"), TS_ERR_ARG;
+  a.P = (a.H + 2 * a.pad - a.R) / a.stride + 1;
+  a.Q = (a.W + 2 * a.pad - a.S) / a.stride + 1;
+  if (a.P < 1 || a.Q < 1) return set_error("ts_conv2d: empty output"), TS_ERR_ARG;
+  if ((mode != 2 && !x) || (mode != 1 && !dy)) return set_error("ts_conv2d: missing operand"), TS_ERR_ARG;
+  a.x = x; a.w = w; a.dy = dy;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  int tc = 0;
+  if (a.dtype == tsk::BF16) tc = tsk::conv_tc(mode, a, out, bias, acc, st) ? 1 : 0;
+  if (!tc) tsk::conv_simt(mode, a, out, bias, acc, st);
+  CU(cudaGetLastError());
+  if (used_tc) *used_tc = tc;
   return TS_OK;
 }
 

@@ -128,6 +128,7 @@ def lib():
                                    vp, i64, i64, i32, C.c_float, C.c_float, vp, vp]),
             "ts_gemm_f32": (i32, [i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, C.c_float,
                                   vp, vp]),
+            "ts_conv2d": (i32, [i32, i32, P(i32), vp, vp, vp, vp, vp, i32, vp, P(i32)]),
         }
         for name, (res, args) in list(sig.items()) + list(optional.items()):
             if not hasattr(L, name):
@@ -453,3 +454,18 @@ def nccl_comm(rank: int, world: int, broadcast):
     comm = C.c_void_p()
     check(lib().ts_nccl_comm_init(idb, world, rank, C.byref(comm)))
     return comm.value
+
+
+def conv2d(mode: int, geom, x, w, dy, out, bias=None, acc: int = 0, stream=None) -> bool:
+    """Run one conv micro-op kernel through the C ABI (`ts_conv2d`, include/ts.h) on
+    torch device tensors (argument marshalling only).  mode 1 fprop -> out = y,
+    2 dgrad -> out = dx, 3 wgrad -> out = dw (fp32).  Returns True when the tcgen05
+    implicit-GEMM path ran."""
+    import torch
+    dt = DTYPES["bf16"] if w.dtype == torch.bfloat16 else DTYPES["f32"]
+    g = (C.c_int32 * 9)(*[int(v) for v in geom])
+    ptr = (lambda t: C.c_void_p(t.data_ptr()) if t is not None else None)
+    used = C.c_int32(0)
+    st = C.c_void_p(stream if stream is not None else torch.cuda.current_stream().cuda_stream)
+    check(lib().ts_conv2d(mode, dt, g, ptr(x), ptr(w), ptr(dy), ptr(out), ptr(bias), acc, st, C.byref(used)))
+    return bool(used.value)

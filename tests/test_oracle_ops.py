@@ -4,7 +4,8 @@ central finite differences, closed forms, invariants and published test vectors.
 import numpy as np
 import pytest
 
-from oracle import ops
+from oracle import net, ops
+from tsinputs import gen, graphs
 
 rng = np.random.default_rng(7)
 H = 1e-6
@@ -156,3 +157,42 @@ def test_dropout_rate_and_split_invariance():
     y = ops.dropout_fwd(x, 0.25, 3, 0)
     k = ops.dropout_keep((50,), 0, 0.25, 3)
     assert np.allclose(y[k], x[k] / 0.75) and (y[~k] == 0).all()
+
+
+def test_round_bf16_pins():
+    """ops.round_bf16 (the bf16 storage reading, SURVEY R20 / DESIGN D-TOL): exact
+    ties-to-even cases worked by hand, and agreement with torch's own fp32 -> bf16
+    conversion (a library routine) on random and edge values."""
+    from oracle import ops as O
+    # spacing of bf16 at 1.0 is 2^-7: 1 + 2^-8 ties -> 1 (even), 1 + 3*2^-8 ties -> 1 + 2^-6 (even)
+    assert O.round_bf16(np.array([1 + 2.0 ** -8]))[0] == 1.0
+    assert O.round_bf16(np.array([1 + 3 * 2.0 ** -8]))[0] == 1 + 2.0 ** -6
+    assert O.round_bf16(np.array([1 + 2.0 ** -8 + 2.0 ** -20]))[0] == 1 + 2.0 ** -7
+    assert O.round_bf16(np.array([-3.0]))[0] == -3.0
+    torch = pytest.importorskip("torch")
+    r = np.random.default_rng(0)
+    x = np.concatenate([r.standard_normal(100000) * 10.0 ** r.integers(-30, 30, 100000),
+                        [0.0, -0.0, 1e-40, -1e-39, 3.3895e38]])
+    ref = torch.from_numpy(x.astype(np.float32)).to(torch.bfloat16).to(torch.float64).numpy()
+    assert np.array_equal(O.round_bf16(x), ref)
+
+
+def test_bf16_storage_reading():
+    """train_step(storage="bf16") rounds exactly the stored values: every activation it
+    keeps is bf16-representable, parameter gradients stay unrounded, and the result is
+    close to (but not equal to) the fp64 definition."""
+    from oracle import ops as O
+    g = graphs.config_graph("bert_tiny", layers=1)
+    P, I = gen.init_params(g), gen.make_inputs(g)
+    l0, g0, _, _ = net.train_step(g, P, I)
+    l1, g1, val, grad = net.train_step(g, P, I, storage="bf16")
+    acts = [t["id"] for t in g["tensors"] if t["kind"] == "act" and t["dtype"] == "bf16"]
+    for tid in acts:
+        assert np.array_equal(O.round_bf16(val[tid]), val[tid])
+        if tid in grad:
+            assert np.array_equal(O.round_bf16(grad[tid]), grad[tid])
+    assert any(not np.array_equal(O.round_bf16(v), v) for v in g1.values())
+    assert abs(l1 - l0) <= 1e-2 * abs(l0)
+    num = sum(float(np.sum((g1[k] - g0[k]) ** 2)) for k in g0)
+    den = sum(float(np.sum(g0[k] ** 2)) for k in g0)
+    assert 0 < (num / den) ** 0.5 <= 5e-2
