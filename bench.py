@@ -2,8 +2,10 @@
 """Benchmark: samples/s of a BERT-Large (24L, h1024, s512, b32, bf16) training
 step under an HBM budget of 25% of its unsplit dynamic peak (BASELINE.json
 configs[3], north_star), on N GPUs as data parallelism (weak scaling: b32 per GPU).
+`--workload vgg16|resnet50` runs configs[1] (VGG-16 b64, 30% budget) or configs[2]
+(ResNet-50 b256, 25% budget) instead; the default line is BERT-Large.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl tsplit|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl tsplit|reference] [--workload W]
     torchrun --nproc-per-node N --master-addr 127.0.0.1 bench.py --gpus N ...
 
 Prints ONE JSON line on rank 0 (contract in the task statement / DESIGN.md §7).
@@ -28,6 +30,27 @@ sys.path.insert(0, ROOT)
 import numpy as np  # noqa: E402
 
 SEQ, HID, HEADS, LAYERS, BATCH = 512, 1024, 16, 24, 32
+
+# BASELINE.json configs by workload (batch per GPU, budget = static + frac x dynamic peak, R4)
+WORKLOADS = {
+    "bert_large": dict(batch=32, frac=0.25, name="bert_large_b32_s512_budget25",
+                       metric="samples/sec under HBM budget (BERT-Large)",
+                       model=f"bert-large ({LAYERS}L h{HID} a{HEADS} s{SEQ})", seq_len=SEQ,
+                       data="synthetic (uniform token ids, random-init weights N(0,0.02))"),
+    "vgg16": dict(batch=64, frac=0.30, name="vgg16_b64_i224_budget30",
+                  metric="samples/sec under HBM budget (VGG-16)", model="vgg-16 (13 conv3x3 + 3 fc, 224x224)",
+                  seq_len=None, data="synthetic (N(0,1) images, uniform labels, Kaiming-normal weights)"),
+    "resnet50": dict(batch=256, frac=0.25, name="resnet50_b256_i224_budget25",
+                     metric="samples/sec under HBM budget (ResNet-50)", model="resnet-50 v1.5 (224x224)",
+                     seq_len=None, data="synthetic (N(0,1) images, uniform labels, Kaiming-normal weights)"),
+}
+
+
+def workload_graph(wl, layers=LAYERS):
+    from tsinputs import graphs
+    if wl == "bert_large":
+        return graphs.bert(layers=layers, batch=BATCH)
+    return graphs.config_graph(wl)
 
 
 def peaks():
@@ -126,8 +149,51 @@ def cpu_baseline_measure():
                       f"({t2:.2f}s) timed, linear extrapolation to 24 layers = {t24:.1f}s/sample"}
 
 
+def cnn_oracle_time(wl, reps=1):
+    """fp64 oracle train step on ONE sample (the per-sample work is identical at any
+    batch; BN statistics then span that sample's pixels)."""
+    from oracle import net
+    from tsinputs import gen, graphs
+    g = graphs.config_graph(wl, batch=1)
+    P, I = gen.init_params(g), gen.make_inputs(g)
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        net.train_step(g, P, I)
+        ts.append(time.perf_counter() - t0)
+    return ts
+
+
+def cnn_cpu_baseline(wl):
+    t = min(cnn_oracle_time(wl))
+    return {"value": 1.0 / t, "unit": "samples/s", "cores": cpu_threads(), "kind": "oracle",
+            "sample": f"1 image (224x224) through the full {wl} fp64 fwd+bwd: {t:.2f}s/sample"}
+
+
 def run_reference(args, rank, world):
     if rank != 0:
+        return
+    if args.workload != "bert_large":
+        W = WORKLOADS[args.workload]
+        cnn_oracle_time(args.workload)  # untimed warm-up
+        times = []
+        for i in range(args.warmup + args.steps):
+            t = cnn_oracle_time(args.workload)[0]
+            if i >= args.warmup:
+                times.append(t)
+        t1 = statistics.mean(times)
+        value = 1.0 / t1
+        line = {
+            "metric": W["metric"], "value": value, "unit": "samples/s", "impl": "reference", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t1 * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": W["name"], "model": W["model"], "global_batch": W["batch"] * world,
+                       "parallelism": f"dp{world}"},
+            "cpu_baseline": {"value": value, "unit": "samples/s", "cores": cpu_threads(), "kind": "oracle",
+                             "sample": f"each step: 1 image through the full {args.workload} in fp64 numpy"},
+            "e2e": {"value": value, "unit": "samples/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+        }
+        print(json.dumps(line), flush=True)
         return
     # calibration (untimed): fixed + per-layer cost from depths 1 and 2
     t1 = min(oracle_time(1))
@@ -212,13 +278,18 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="tsplit", choices=["tsplit", "reference"])
-    ap.add_argument("--budget-frac", type=float, default=0.25)
+    ap.add_argument("--workload", default="bert_large", choices=sorted(WORKLOADS))
+    ap.add_argument("--budget-frac", type=float, default=None)
     ap.add_argument("--layers", type=int, default=LAYERS)
     ap.add_argument("--no-unbudgeted", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--analytic-profile", action="store_true", help="plan with the analytic model, not measured times")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
+    W = WORKLOADS[args.workload]
+    if args.budget_frac is None:
+        args.budget_frac = W["frac"]
+    batch = W["batch"]
 
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -252,7 +323,7 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    spec = graphs.bert(layers=args.layers, batch=BATCH)
+    spec = workload_graph(args.workload, args.layers)
     G = tsplit.Graph(spec)
     base = tsplit.Plan.default(G)
     bst = base.stats()
@@ -279,7 +350,8 @@ def main():
     streams = tuple(torch.cuda.Stream() for _ in range(3))
     params = gen.init_params(spec, seed=1)
     host_inputs = tsplit.inputs_to_device(G, arrays, pinned_host=True)
-    h2d_bytes = sum(int(np.prod(t["shape"])) * 4 for t in spec["tensors"] if t["kind"] in ("input", "label"))
+    h2d_bytes = sum(int(np.prod(t["shape"])) * (2 if t["dtype"] == "bf16" else 4)
+                    for t in spec["tensors"] if t["kind"] in ("input", "label"))
 
     def make_session(p):
         s = tsplit.Session(G, p, device=local, lr=1e-4, streams=streams, nccl_comm=comm, world_size=world)
@@ -309,9 +381,13 @@ def main():
     sess.step(dev_inputs)
     item_ms = sess.item_times()
     recs = sess.gemm_times()
+    kinds = sess.gemm_kinds()
     sess.profile_items(False)
-    lin = [(f, ms) for f, ms, bt in recs if f > 0 and bt == 1]
-    att = [(f, ms) for f, ms, bt in recs if f > 0 and bt > 1]
+    conv = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and kd > 0 and tc]
+    lin = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and bt == 1 and kd == 0 and tc]
+    att = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and bt > 1 and tc]
+    c_flop, c_ms = sum(f for f, _ in conv), sum(ms for _, ms in conv)
+    cnn = args.workload != "bert_large"
     g_flop, g_ms = sum(f for f, _ in lin), sum(ms for _, ms in lin)
     a_flop, a_ms = sum(f for f, _ in att), sum(ms for _, ms in att)
     step_ms_prof = sum(item_ms)
@@ -326,7 +402,7 @@ def main():
         if world > 1:
             dist.barrier()
         t_unb = max_over_ranks(time_steps(torch, s2, dev_inputs, streams[0], args.steps))
-        unb = BATCH * world * args.steps / t_unb
+        unb = batch * world * args.steps / t_unb
         del s2
         torch.cuda.empty_cache()
 
@@ -334,15 +410,49 @@ def main():
         dist.destroy_process_group() if world > 1 else None
         return
     pk, pk_src = peaks()
-    value = BATCH * world * args.steps / dt
-    achieved = g_flop / (g_ms / 1e3) / 1e12 if g_ms > 0 else 0.0
+    value = batch * world * args.steps / dt
     peak = pk.get("bf16_tflops_sustained", pk.get("bf16_tflops"))
     traffic = None
-    tp = os.path.join(ROOT, "profiles", "r1_gemm_ncu.json")
+    tp = os.path.join(ROOT, "profiles", "r1_conv_ncu.json" if cnn else "r1_gemm_ncu.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get("traffic_per_launch_bytes")
+    if cnn:
+        achieved = c_flop / (c_ms / 1e3) / 1e12 if c_ms > 0 else 0.0
+        roof = {"bound": "tensor", "kernel": "conv_tc (tcgen05 implicit GEMM, cp.async gathers): fprop+dgrad+wgrad",
+                "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak if peak else None,
+                "traffic": traffic, "peak_source": f"{pk_src} bf16_tflops_sustained", "launches": len(conv),
+                "share_of_step": c_ms / step_ms_prof if step_ms_prof else None,
+                "how": "one eager step, cudaEvent pair around every conv launch on the compute stream; "
+                       "algorithmic FLOP (2 x N*P*Q x K x R*S*C per product) / summed launch durations"}
+    else:
+        achieved = g_flop / (g_ms / 1e3) / 1e12 if g_ms > 0 else 0.0
+        roof = {"bound": "tensor", "kernel": "gemm_tc (tcgen05/TMA) on linear micro-ops",
+                "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                "frac": achieved / peak if peak else None, "traffic": traffic,
+                "peak_source": f"{pk_src} bf16_tflops_sustained",
+                "launches": len(lin), "share_of_step": g_ms / step_ms_prof if step_ms_prof else None,
+                "how": "one eager step, cudaEvent pair around every GEMM launch on the compute stream; "
+                       "algorithmic FLOP (2MNK) / summed launch durations; traffic = dram read+write of "
+                       "one FFN1-forward launch from the committed ncu --set full capture"}
+    config = {
+        "workload": W["name"], "model": W["model"] if cnn else f"bert-large ({args.layers}L h{HID} a{HEADS} s{SEQ})",
+        "global_batch": batch * world, "seq_len": W["seq_len"], "parallelism": f"dp{world}",
+        "budget_frac_of_unsplit_dynamic_peak": args.budget_frac,
+        "budget_bytes": budget, "unsplit_peak_bytes": unsplit_peak, "static_bytes": static,
+        "plan_peak_extent_bytes": pst["peak_extent"],
+        "plan": {"split_tensors": pst["n_split_tensors"], "swap_tensors": pst["n_swap_tensors"],
+                 "recompute_tensors": pst["n_recompute_tensors"], "replays": pst["n_replay"],
+                 "d2h_bytes": pst["d2h_bytes"], "h2d_bytes": pst["h2d_bytes"],
+                 "step_flop": pst["compute_flop"], "predicted_ms": pst["predicted_s"] * 1e3,
+                 "profile_and_planning_s": round(plan_s, 2),
+                 "measured_pcie_gbs": [round(x / 1e9, 1) for x in pcie] if pcie else None},
+        "l2": "no flush needed: every step streams >10 GB of activations through a 126 MB L2"
+              if not cnn else "no flush needed: every step streams several GB of activations through a 126 MB L2",
+    }
+    if cnn:
+        config.pop("seq_len")
     line = {
-        "metric": "samples/sec under HBM budget (BERT-Large)",
+        "metric": W["metric"],
         "value": value,
         "unit": "samples/s",
         "n_gpus": world,
@@ -353,43 +463,28 @@ def main():
         "scaling": "weak",
         "vs_baseline": None,
         "dtype": "bf16",
-        "data": "synthetic (uniform token ids, random-init weights N(0,0.02))",
-        "config": {
-            "workload": "bert_large_b32_s512_budget25",
-            "model": f"bert-large ({args.layers}L h{HID} a{HEADS} s{SEQ})",
-            "global_batch": BATCH * world, "seq_len": SEQ, "parallelism": f"dp{world}",
-            "budget_frac_of_unsplit_dynamic_peak": args.budget_frac,
-            "budget_bytes": budget, "unsplit_peak_bytes": unsplit_peak, "static_bytes": static,
-            "plan_peak_extent_bytes": pst["peak_extent"],
-            "plan": {"split_tensors": pst["n_split_tensors"], "swap_tensors": pst["n_swap_tensors"],
-                     "recompute_tensors": pst["n_recompute_tensors"], "replays": pst["n_replay"],
-                     "d2h_bytes": pst["d2h_bytes"], "h2d_bytes": pst["h2d_bytes"],
-                     "step_flop": pst["compute_flop"], "predicted_ms": pst["predicted_s"] * 1e3,
-                     "profile_and_planning_s": round(plan_s, 2),
-                     "measured_pcie_gbs": [round(x / 1e9, 1) for x in pcie] if pcie else None},
-            "l2": "no flush needed: every step streams >10 GB of activations through a 126 MB L2",
-        },
+        "data": W["data"],
+        "config": config,
         "unbudgeted_samples_per_s": unb,
         "budget_throughput_ratio": (value / unb) if unb else None,
         "gpu_launches": int(launches * args.steps),
         "clocks": clk.summary(),
-        "e2e": {"value": BATCH * world * args.steps / dt_e2e, "unit": "samples/s",
+        "e2e": {"value": batch * world * args.steps / dt_e2e, "unit": "samples/s",
                 "h2d_bytes_per_step": h2d_bytes, "d2h_bytes_per_step": 4},
-        "roofline": {"bound": "tensor", "kernel": "gemm_tc (tcgen05/TMA) on linear micro-ops",
-                     "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                     "frac": achieved / peak if peak else None, "traffic": traffic,
-                     "peak_source": f"{pk_src} bf16_tflops_sustained",
-                     "launches": len(lin), "share_of_step": g_ms / step_ms_prof if step_ms_prof else None,
-                     "how": "one eager step, cudaEvent pair around every GEMM launch on the compute stream; "
-                            "algorithmic FLOP (2MNK) / summed launch durations; traffic = dram read+write of "
-                            "one FFN1-forward launch from the committed ncu --set full capture"},
-        "roofline_attention_gemm": {"bound": "hbm", "kernel": "gemm_tc on per-(sample, head) attention products",
-                                    "achieved_tflops": a_flop / (a_ms / 1e3) / 1e12 if a_ms > 0 else None,
-                                    "launches": len(att),
-                                    "share_of_step": a_ms / step_ms_prof if step_ms_prof else None},
+        "roofline": roof,
     }
+    if not cnn:
+        line["roofline_attention_gemm"] = {
+            "bound": "hbm", "kernel": "gemm_tc on per-(sample, head) attention products",
+            "achieved_tflops": a_flop / (a_ms / 1e3) / 1e12 if a_ms > 0 else None, "launches": len(att),
+            "share_of_step": a_ms / step_ms_prof if step_ms_prof else None}
+    else:
+        line["roofline_linear_gemm"] = {
+            "kernel": "gemm_tc on the fc layers", "launches": len(lin),
+            "achieved_tflops": g_flop / (g_ms / 1e3) / 1e12 if g_ms > 0 else None,
+            "share_of_step": g_ms / step_ms_prof if step_ms_prof else None}
     if world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline_measure()
+        line["cpu_baseline"] = cnn_cpu_baseline(args.workload) if cnn else cpu_baseline_measure()
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()

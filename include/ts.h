@@ -247,6 +247,9 @@ ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, 
  * fallback), cudaEvent duration on the compute stream (ms), batch count (1 = linear). */
 ts_status ts_session_gemm_times(const ts_session_t* s, double* flop, float* ms, int32_t* batch, uint64_t cap,
                                 uint64_t* n);
+/* Kind of each record of ts_session_gemm_times: 0 GEMM (linear / attention), 1 conv
+ * fprop, 2 conv dgrad, 3 conv wgrad (implicit GEMM); tc[i] = 1 when the tcgen05 path ran. */
+ts_status ts_session_gemm_kinds(const ts_session_t* s, int32_t* kind, int32_t* tc, uint64_t cap, uint64_t* n);
 
 /* ---- data parallelism (north_star: DP over NVLink with NCCL) -------------------
  * The session allreduces the fp32 gradient region (sum) with this communicator

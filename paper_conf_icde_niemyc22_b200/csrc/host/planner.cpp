@@ -518,16 +518,57 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
           step2.push_back(opt == TS_RECOMPUTE ? with_feeders(c, t) : c);
         }
       }
+    // D-R8e: a recomputed tensor regenerated for the bottleneck (a replay chain member,
+    // P:L294) is allocated piece by piece at its own split; splitting it finer shrinks
+    // the replay's working set, so live recompute-opt tensors get split-only proposals.
+    for (int t : live) {
+      const Tensor& x = g.t[t];
+      if (x.kind != TS_ACT || x.is_loss || own.count(t) || ps.cfg[t].opt != TS_RECOMPUTE) continue;
+      for (int p = ps.cfg[t].p * 2; p <= 16; p *= 2) {
+        if (g.samples % p) break;
+        Cand2 c;
+        c.birth = birth[t];
+        c.tensor = t;
+        c.ch = {{t, TS_RECOMPUTE, p, ps.cfg[t].lead}};
+        step2.push_back(c);
+      }
+    }
+    // D-R8d: the whole micro-op split — every activation of the bottleneck op to the same
+    // p at once.  Under op-major execution (R10) an input piece is released while the
+    // output is produced only when both sides are split, so single-tensor splits can
+    // show no gain (dM = 0) where the joint one does (e.g. VGG conv1 -> relu1).
+    for (int p = 2; p <= 16; p *= 2) {
+      if (g.samples % p) continue;
+      Cand2 c;
+      for (int t : split_cands)
+        if (ps.cfg[t].p < p) c.ch.push_back({t, ps.cfg[t].opt, p, ps.cfg[t].lead});
+      if (c.ch.size() < 2) continue;
+      c.birth = birth[c.ch[0].t];
+      c.tensor = c.ch[0].t;
+      step2.push_back(c);
+    }
     // step 3: score every proposal by re-simulation — dM = drop of the pool top over
     // the bottleneck op's items, dT = change of the predicted step time (timeline with
     // the profile, PCIe occupancy and swap-in stalls) — and take the best.
+    // the bottleneck op's items: its micro-ops of this phase and, in the backward, the
+    // recompute replays of its groups (they allocate for it)
     auto top_of_op = [&](const PlanState& st) {
+      std::unordered_map<int, int> group_op;
+      if (bwd_phase)
+        for (const Item& it : st.ex.items)
+          if (it.kind == IT_B) group_op[it.group] = it.op;
       uint64_t m = 0;
       for (size_t i = 0; i < st.ex.items.size(); ++i) {
         const Item& it = st.ex.items[i];
         if (it.kind == IT_SO || it.kind == IT_SI) continue;
         bool same_phase = ((int)i >= st.ex.fwd_end) == bwd_phase;
-        if (same_phase && it.op == bop) m = std::max(m, st.sim.top[i]);
+        if (!same_phase) continue;
+        int op = it.op;
+        if (it.kind == IT_R) {
+          auto f = group_op.find(it.group);
+          op = f == group_op.end() ? -1 : f->second;
+        }
+        if (op == bop) m = std::max(m, st.sim.top[i]);
       }
       return m;
     };
@@ -574,11 +615,35 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
                      (unsigned long long)cur_top, (unsigned long long)top_of_op(cs));
       }
     }
-    for (auto& c : step2) consider(c);
+    for (auto& c : step2) {
+      consider(c);
+      if (log && !best) {
+        PlanState cs;
+        cs.cfg = ps.cfg;
+        for (auto& chg : c.ch) {
+          cs.cfg[chg.t].opt = chg.opt;
+          cs.cfg[chg.t].p = chg.p;
+          cs.cfg[chg.t].lead = chg.lead;
+        }
+        plan_refresh(g, cs, &pr);
+        std::fprintf(stderr, "  cand2 t=%d n=%zu opt=%d p=%d top %llu->%llu\n", c.tensor, c.ch.size(), c.ch[0].opt,
+                     c.ch[0].p, (unsigned long long)cur_top, (unsigned long long)top_of_op(cs));
+      }
+    }
     if (log && best)
       std::fprintf(stderr, "iter %d bottleneck item %d op %d (%s) top %.3f GB: pick t=%d opt=%d p=%d lead=%d ratio %.3g pred %.2f ms\n",
                    iter, bi, bop, bwd_phase ? "bwd" : "fwd", cur_top / 1e9, best->tensor, best->ch[0].opt,
                    best->ch[0].p, best->ch[0].lead, best_ratio, 1e3 * ps.predicted_s);
+    if (!best && log) {
+      std::fprintf(stderr, "stuck at item %d op %d (%s): live tensors\n", bi, bop, bwd_phase ? "bwd" : "fwd");
+      for (int t : live)
+        std::fprintf(stderr, "  t=%d opt=%d p=%d bytes=%llu own=%d first_bw=%d last_fw=%d\n", t, ps.cfg[t].opt,
+                     ps.cfg[t].p, (unsigned long long)g.t[t].bytes, (int)own.count(t), first_bw[t], last_fw[t]);
+      for (auto& e : ps.sim.trace)
+        if (e.item == bi && e.kind == 0)
+          std::fprintf(stderr, "  alloc@bi key=%d piece=%d bytes=%llu off=%llu\n", e.key, e.piece,
+                       (unsigned long long)e.bytes, (unsigned long long)e.offset);
+    }
     if (!best) {
       set_error("infeasible: no candidate left at op " + std::to_string(bop) + " (item " + std::to_string(bi) +
                 ", needs " + std::to_string(ps.sim.top[bi]) + " B > budget " + std::to_string(budget) + ")");

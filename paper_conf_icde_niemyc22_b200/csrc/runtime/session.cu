@@ -83,7 +83,7 @@ struct ts_session_s {
   std::vector<float> item_ms;
   std::vector<tsk::GemmRecord> gemm_recs;
   std::vector<double> gemm_flop, gemm_ms;
-  std::vector<int> gemm_batch;
+  std::vector<int> gemm_batch, gemm_kind, gemm_tc;
 };
 
 namespace {
@@ -768,12 +768,16 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
     s->gemm_flop.clear();
     s->gemm_ms.clear();
     s->gemm_batch.clear();
+    s->gemm_kind.clear();
+    s->gemm_tc.clear();
     for (auto& r : s->gemm_recs) {
       float ms = 0.f;
       cudaEventElapsedTime(&ms, r.start, r.stop);
       s->gemm_flop.push_back(r.tc ? r.flop : 0.0);
       s->gemm_ms.push_back(ms);
       s->gemm_batch.push_back(r.batch);
+      s->gemm_kind.push_back(r.kind);
+      s->gemm_tc.push_back(r.tc);
     }
     s->item_ms.assign(s->prog.size(), 0.f);
     for (auto& c : s->prog)
@@ -954,6 +958,16 @@ ts_status ts_session_gemm_times(const ts_session_t* s, double* flop, float* ms, 
     if (flop) flop[i] = s->gemm_flop[i];
     if (ms) ms[i] = float(s->gemm_ms[i]);
     if (batch) batch[i] = s->gemm_batch[i];
+  }
+  return TS_OK;
+}
+
+ts_status ts_session_gemm_kinds(const ts_session_t* s, int32_t* kind, int32_t* tc, uint64_t cap, uint64_t* n) {
+  if (!s || !n) return set_error("null argument"), TS_ERR_ARG;
+  *n = s->gemm_kind.size();
+  for (uint64_t i = 0; i < s->gemm_kind.size() && i < cap; ++i) {
+    if (kind) kind[i] = s->gemm_kind[i];
+    if (tc) tc[i] = s->gemm_tc[i];
   }
   return TS_OK;
 }

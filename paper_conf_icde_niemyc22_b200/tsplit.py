@@ -118,6 +118,7 @@ def lib():
             "ts_session_profile_items": (i32, [vp, i32]),
             "ts_session_item_times": (i32, [vp, P(C.c_float), u64, P(u64)]),
             "ts_session_gemm_times": (i32, [vp, P(C.c_double), P(C.c_float), P(i32), u64, P(u64)]),
+            "ts_session_gemm_kinds": (i32, [vp, P(i32), P(i32), u64, P(u64)]),
             "ts_profile_measure": (i32, [vp, vp, u64, P(vp), i32, i32, P(vp)]),
             "ts_profile_get": (i32, [vp, i32, i32, P(C.c_double), P(C.c_double)]),
             "ts_profile_pcie": (i32, [vp, P(C.c_double), P(C.c_double)]),
@@ -421,6 +422,15 @@ class Session:
         b = (C.c_int32 * n.value)()
         check(lib().ts_session_gemm_times(self.h, f, m, b, n.value, C.byref(n)))
         return list(zip(f, m, b))
+
+    def gemm_kinds(self):
+        """[(kind, tc)] per record of gemm_times: kind 0 GEMM, 1/2/3 conv fprop/dgrad/wgrad."""
+        n = C.c_uint64()
+        check(lib().ts_session_gemm_kinds(self.h, None, None, 0, C.byref(n)))
+        k = (C.c_int32 * n.value)()
+        t = (C.c_int32 * n.value)()
+        check(lib().ts_session_gemm_kinds(self.h, k, t, n.value, C.byref(n)))
+        return list(zip(k, t))
 
     def launches(self) -> int:
         n = C.c_int64()
