@@ -286,6 +286,8 @@ ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K,
  * dtype TS_BF16: tcgen05/TMEM implicit GEMM with cp.async gathers (fp32 accumulate)
  * when eligible (K % 8 == 0; dgrad also C % 8 == 0), else CUDA cores; TS_F32: CUDA
  * cores with fp64 accumulation.  *used_tc (may be NULL) reports the path taken.
+ * Layers with C % 64 == 0, K % 64 == 0 and stride <= 2 take the TMA-fed kernel
+ * (spatial-box M tiles); mode | 0x10 forces the cp.async gather kernel (tests).
  * Errors: TS_ERR_ARG for bad geometry, TS_ERR_CUDA for launch failures. */
 ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void* x, const void* w, const void* dy,
                     void* out, const void* bias, int32_t acc, void* stream, int32_t* used_tc);

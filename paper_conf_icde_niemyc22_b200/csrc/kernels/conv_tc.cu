@@ -35,7 +35,6 @@ constexpr int kMmaWarp = kEpiWarps;      // warp 4
 constexpr int kProd0 = kEpiWarps + 1;    // warps 5..8
 constexpr int kThreads = 32 * (kEpiWarps + 1 + kProdWarps);
 constexpr int kProdThreads = 32 * kProdWarps;
-constexpr int kLag = 2;                  // cp.async groups in flight per producer thread
 constexpr int kSmemLimit = 232448;
 
 enum Mode : int { FPROP = 1, DGRAD = 2, WGRAD = 3 };
@@ -319,6 +318,10 @@ __global__ void __launch_bounds__(kThreads, 1) conv_tc_kernel(const CtP p) {
   constexpr int B_BYTES = BN * BK * 2;
   constexpr int STAGE = A_BYTES + B_BYTES;
   constexpr int STAGES = conv_stages<BN>();
+  // cp.async groups a producer thread keeps in flight before releasing the oldest
+  // stage: all but two stages, so each SM has ~150 KB of gathers outstanding (the
+  // L2 latency x bandwidth product; fewer leaves the tensor pipe starved)
+  constexpr int kLag = STAGES - 2;
   constexpr uint32_t TMEM_COLS = 2 * BN;
   constexpr int A_MN = MODE == WGRAD ? 1 : 0;
   constexpr int B_MN = MODE == FPROP ? 0 : 1;
@@ -542,6 +545,11 @@ void launch_bn(int bn, const CtP& p, cudaStream_t st) {
 }  // namespace
 
 bool conv_tc(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st) {
+  // 64-channel layers: TMA-fed kernel (conv_tma.cu); the gather kernel covers the rest
+  return conv_tma(mode, a, out, bias, acc, st) || conv_gather(mode, a, out, bias, acc, st);
+}
+
+bool conv_gather(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st) {
   if (a.dtype != BF16 || a.n <= 0) return false;
   if (a.K % 8) return false;                             // dY rows / output rows in 16-byte vectors
   const bool vec = a.C % 8 == 0;

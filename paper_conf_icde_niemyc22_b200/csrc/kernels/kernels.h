@@ -67,6 +67,10 @@ void conv_dgrad(const ConvArgs& a, void* dx, int acc, cudaStream_t st);
 void conv_wgrad(const ConvArgs& a, float* dw, int acc, cudaStream_t st);
 // tcgen05 path; false when the shape/alignment is not eligible (then SIMT)
 bool conv_tc(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
+// TMA-fed variant for C % 64 == 0, K % 64 == 0, stride <= 2 (tried first by conv_tc)
+bool conv_tma(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
+// the cp.async gather kernel alone (tests; conv_tc tries conv_tma first)
+bool conv_gather(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
 void conv_simt(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
 
 // ---- batch normalisation over all pieces of a split tensor ----------

@@ -1153,6 +1153,8 @@ ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K, const float* A, int64_t l
 
 ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void* x, const void* w, const void* dy,
                     void* out, const void* bias, int32_t acc, void* stream, int32_t* used_tc) {
+  const bool gather_only = (mode & 0x10) != 0;
+  mode &= 0xF;
   if (!geom || mode < 1 || mode > 3 || (dtype != TS_BF16 && dtype != TS_F32) || !w || !out)
     return set_error("ts_conv2d: bad argument"), TS_ERR_ARG;
   tsk::ConvArgs a;
@@ -1168,7 +1170,8 @@ ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void
   a.x = x; a.w = w; a.dy = dy;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   int tc = 0;
-  if (a.dtype == tsk::BF16) tc = tsk::conv_tc(mode, a, out, bias, acc, st) ? 1 : 0;
+  if (a.dtype == tsk::BF16)
+    tc = (gather_only ? tsk::conv_gather(mode, a, out, bias, acc, st) : tsk::conv_tc(mode, a, out, bias, acc, st)) ? 1 : 0;
   if (!tc) tsk::conv_simt(mode, a, out, bias, acc, st);
   CU(cudaGetLastError());
   if (used_tc) *used_tc = tc;
