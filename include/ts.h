@@ -196,6 +196,13 @@ ts_status ts_plan_trace(const ts_plan_t* p, ts_alloc_event* buf, uint64_t cap, u
 /* Augmented schedule as int32 quadruples (kind, op, k, aux) — kind 0 F, 1 B, 2 R,
  * 3 SO, 4 SI; aux = piece key for SO/SI (key*65536+piece), else group id. */
 ts_status ts_plan_items(const ts_plan_t* p, int32_t* buf, uint64_t cap, uint64_t* n);
+/* Data-parallel gradient buckets of this plan: parameters grouped, in
+ * the order their gradients become final in the augmented schedule, into buckets of at
+ * least bucket_bytes (the session uses 32 MiB).  buf receives int64 triples
+ * (after_item, grad-region byte offset, bytes) — one per contiguous span, in bucket
+ * order; *n = number of triples (buf may be NULL).  Every rank derives the identical
+ * list from the broadcast plan, so NCCL calls match across ranks. */
+ts_status ts_plan_grad_buckets(const ts_plan_t* p, uint64_t bucket_bytes, int64_t* buf, uint64_t cap, uint64_t* n);
 ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n);
 ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, ts_plan_t** out);
 void ts_plan_destroy(ts_plan_t* p);

@@ -195,6 +195,23 @@ ts_status ts_plan_items(const ts_plan_t* p, int32_t* buf, uint64_t cap, uint64_t
   return TS_OK;
 }
 
+ts_status ts_plan_grad_buckets(const ts_plan_t* p, uint64_t bucket_bytes, int64_t* buf, uint64_t cap, uint64_t* n) {
+  if (!p || !n) return set_error("null argument"), TS_ERR_ARG;
+  auto bk = grad_buckets(*p->graph, p->st.ex, bucket_bytes);
+  uint64_t cnt = 0;
+  for (auto& b : bk)
+    for (auto& sp : b.spans) {
+      if (buf && (cnt + 1) * 3 <= cap) {
+        buf[3 * cnt + 0] = b.after_item;
+        buf[3 * cnt + 1] = int64_t(sp.first);
+        buf[3 * cnt + 2] = int64_t(sp.second);
+      }
+      ++cnt;
+    }
+  *n = cnt;
+  return TS_OK;
+}
+
 // Serialized form: magic, n_tensors, budget, then (opt, p, dim, lead) per tensor.
 ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n) {
   if (!p || !n) return set_error("null argument"), TS_ERR_ARG;

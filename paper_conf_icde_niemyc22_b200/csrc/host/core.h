@@ -129,6 +129,13 @@ class Pool {
   uint64_t cap_ = 0, extent_ = 0;
 };
 
+// ---- data-parallel gradient buckets (dp.cpp) ----------------------------------
+struct GradBucket {
+  int after_item = -1;                                // allreduce once this item has run
+  std::vector<std::pair<uint64_t, uint64_t>> spans;   // (grad-region offset, bytes), contiguous runs
+};
+std::vector<GradBucket> grad_buckets(const Graph& g, const Expansion& ex, uint64_t bucket_bytes);
+
 // ---- profile + planner ------------------------------------------------------
 struct OpCost {
   double flop_f = 0, flop_b = 0;    // whole op

@@ -36,6 +36,7 @@ namespace {
 
 // Minimal NCCL ABI (resolved with dlsym from the libnccl the process already has).
 typedef int (*nccl_allreduce_fn)(const void*, void*, size_t, int, int, void*, cudaStream_t);
+typedef int (*nccl_group_fn)();
 constexpr int kNcclFloat32 = 7, kNcclSum = 0;
 
 }  // namespace
@@ -63,6 +64,12 @@ struct ts_session_s {
   bool own_streams = false;
   void* nccl = nullptr;
   nccl_allreduce_fn allreduce = nullptr;
+  nccl_group_fn group_start = nullptr, group_end = nullptr;
+  cudaStream_t comm = nullptr;                  // allreduce stream (data parallelism)
+  std::vector<GradBucket> buckets;              // DP gradient buckets (dp.cpp)
+  std::vector<std::vector<int>> buckets_after;  // per program command: buckets to launch after it
+  std::vector<cudaEvent_t> ev_bucket;
+  cudaEvent_t ev_comm_done = nullptr;
   int world = 1;
   float lr = 0.f;
   uint32_t step = 0;
@@ -644,6 +651,17 @@ ts_status build_program(ts_session_t* s) {
   for (auto& o : g.ops)
     if (o.kind == TS_OP_EMBED)
       for (int i = 2; i < 5; ++i) s->zero_grads.push_back(o.in[i]);
+  // data parallelism: per-bucket allreduce after the bucket's last gradient writer
+  s->buckets_after.assign(s->prog.size(), {});
+  if (s->nccl) {  // (a 1-rank communicator exercises the same path on one GPU)
+    s->buckets = grad_buckets(g, s->ex, uint64_t(32) << 20);
+    s->ev_bucket.assign(s->buckets.size(), nullptr);
+    for (size_t b = 0; b < s->buckets.size(); ++b) {
+      s->buckets_after[std::max(0, s->buckets[b].after_item)].push_back(int(b));
+      CU(cudaEventCreateWithFlags(&s->ev_bucket[b], cudaEventDisableTiming));
+    }
+    CU(cudaEventCreateWithFlags(&s->ev_comm_done, cudaEventDisableTiming));
+  }
   CU(cudaEventCreateWithFlags(&s->ev_mark, cudaEventDisableTiming));
   CU(cudaEventCreateWithFlags(&s->ev_join_d2h, cudaEventDisableTiming));
   CU(cudaEventCreateWithFlags(&s->ev_join_h2d, cudaEventDisableTiming));
@@ -679,6 +697,17 @@ void issue_step(ts_session_t* s) {
       cudaEventRecord(s->ev_h2d[c.item], s->h2d);
       h2d_used = true;
     }
+    // gradients that became final at this item: allreduce them on the comm stream while
+    // the rest of the backward runs
+    for (int b : s->buckets_after[c.item]) {
+      cudaEventRecord(s->ev_bucket[b], cs);
+      cudaStreamWaitEvent(s->comm, s->ev_bucket[b], 0);
+      if (s->group_start) s->group_start();
+      for (auto& sp : s->buckets[b].spans)
+        s->allreduce(s->slab + sp.first, s->slab + sp.first, sp.second / 4, kNcclFloat32, kNcclSum, s->nccl,
+                     s->comm);
+      if (s->group_end) s->group_end();
+    }
   }
   // data-parallel gradient sum (north_star DP) and SGD on fp32 masters
   uint64_t gbeg = ~0ull, gend = 0, mbeg = ~0ull;
@@ -688,8 +717,10 @@ void issue_step(ts_session_t* s) {
       gend = std::max(gend, g.grad_off[t.id] + align_up(4 * t.numel));
       mbeg = std::min(mbeg, g.master_off[t.id]);
     }
-  if (gend > gbeg && s->nccl && s->allreduce && s->world > 1)
-    s->allreduce(s->slab + gbeg, s->slab + gbeg, (gend - gbeg) / 4, kNcclFloat32, kNcclSum, s->nccl, cs);
+  if (!s->buckets.empty()) {  // SGD waits for the last bucket
+    cudaEventRecord(s->ev_comm_done, s->comm);
+    cudaStreamWaitEvent(cs, s->ev_comm_done, 0);
+  }
   if (s->lr != 0.f && gend > gbeg) {
     tsk::sgd_update(reinterpret_cast<float*>(s->slab + mbeg), reinterpret_cast<const float*>(s->slab + gbeg),
                     int64_t((gend - gbeg) / 4), s->lr, 1.f / float(s->world), cs);
@@ -832,8 +863,13 @@ ts_status ts_session_create(const ts_graph_t* gh, const ts_plan_t* ph, const ts_
     s->nccl = cfg->nccl_comm;
     void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
     if (!h) h = dlopen("libnccl.so.2", RTLD_NOW);
-    if (h) s->allreduce = reinterpret_cast<nccl_allreduce_fn>(dlsym(h, "ncclAllReduce"));
+    if (h) {
+      s->allreduce = reinterpret_cast<nccl_allreduce_fn>(dlsym(h, "ncclAllReduce"));
+      s->group_start = reinterpret_cast<nccl_group_fn>(dlsym(h, "ncclGroupStart"));
+      s->group_end = reinterpret_cast<nccl_group_fn>(dlsym(h, "ncclGroupEnd"));
+    }
     if (!s->allreduce) return set_error("ncclAllReduce not found"), TS_ERR_NCCL;
+    CU(cudaStreamCreateWithFlags(&s->comm, cudaStreamNonBlocking));
   }
   CU(cudaMemsetAsync(s->slab, 0, s->g->static_bytes, s->cs));
   ts_status st = build_program(s.get());
@@ -850,6 +886,10 @@ void ts_session_destroy(ts_session_t* s) {
     if (e) cudaEventDestroy(e);
   for (auto e : s->ev_h2d)
     if (e) cudaEventDestroy(e);
+  for (auto e : s->ev_bucket)
+    if (e) cudaEventDestroy(e);
+  if (s->ev_comm_done) cudaEventDestroy(s->ev_comm_done);
+  if (s->comm) cudaStreamDestroy(s->comm);
   if (s->ev_mark) cudaEventDestroy(s->ev_mark);
   if (s->ev_join_d2h) cudaEventDestroy(s->ev_join_d2h);
   if (s->ev_join_h2d) cudaEventDestroy(s->ev_join_h2d);

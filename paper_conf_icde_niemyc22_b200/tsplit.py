@@ -99,6 +99,7 @@ def lib():
             "ts_plan_stats": (i32, [vp, P(PlanStats)]),
             "ts_plan_trace": (i32, [vp, P(AllocEvent), u64, P(u64)]),
             "ts_plan_items": (i32, [vp, P(i32), u64, P(u64)]),
+            "ts_plan_grad_buckets": (i32, [vp, u64, P(i64), u64, P(u64)]),
             "ts_plan_serialize": (i32, [vp, vp, u64, P(u64)]),
             "ts_plan_deserialize": (i32, [vp, vp, u64, P(vp)]),
             "ts_plan_destroy": (None, [vp]),
@@ -307,6 +308,14 @@ class Plan:
         check(lib().ts_plan_items(self.h, buf, len(buf), C.byref(n)))
         kinds = ["F", "B", "R", "SO", "SI"]
         return [(kinds[buf[4 * i]], buf[4 * i + 1], buf[4 * i + 2], buf[4 * i + 3]) for i in range(n.value)]
+
+    def grad_buckets(self, bucket_bytes: int = 32 << 20):
+        """[(after_item, grad offset, bytes)] spans of the data-parallel allreduce buckets."""
+        n = C.c_uint64()
+        check(lib().ts_plan_grad_buckets(self.h, bucket_bytes, None, 0, C.byref(n)))
+        buf = (C.c_int64 * (3 * n.value))()
+        check(lib().ts_plan_grad_buckets(self.h, bucket_bytes, buf, len(buf), C.byref(n)))
+        return [(buf[3 * i], buf[3 * i + 1], buf[3 * i + 2]) for i in range(n.value)]
 
     def serialize(self) -> bytes:
         n = C.c_uint64()

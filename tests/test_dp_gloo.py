@@ -30,7 +30,8 @@ def _worker(rank, world, port, q):
         items = plan.items()
         # every rank holds the same schedule: compare a digest across ranks
         import hashlib
-        h = hashlib.sha1(repr((trace, items)).encode()).hexdigest()
+        buckets = plan.grad_buckets(1 << 14)  # NCCL call order must match across ranks
+        h = hashlib.sha1(repr((trace, items, buckets)).encode()).hexdigest()
         digest = torch.tensor([int(h[:15], 16)], dtype=torch.int64)
         gathered = [torch.zeros_like(digest) for _ in range(world)]
         dist.all_gather(gathered, digest)

@@ -144,3 +144,26 @@ def test_bert_large_full_size_properties():
     assert abs(l_b - math.log(2.0)) < 0.05 and abs(l_0 - l_b) <= 1e-3 * abs(l_0)
     assert all(np.isfinite(v).all() for v in g_b.values())
     assert global_rel_err(g_b, g_0) <= 1e-2
+
+
+def test_nccl_bucketed_allreduce_single_rank():
+    """The data-parallel path (per-bucket ncclAllReduce on the comm stream, captured in
+    the CUDA graph, SGD after the last bucket) with a 1-rank communicator: gradients
+    and the updated parameters equal the communicator-free session's."""
+    g = graphs.config_graph("bert_tiny", dtype="f32")
+    G = tsplit.Graph(g)
+    P = tsplit.Plan.default(G)
+    comm = tsplit.nccl_comm(0, 1, lambda b: b)
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    dev = tsplit.inputs_to_device(G, inputs)
+    out = []
+    for c in (None, comm):
+        S = tsplit.Session(G, P, lr=0.1, nccl_comm=c, world_size=1)
+        S.set_params(params)
+        S.step(dev)
+        S.step(dev)
+        out.append((S.grads(), S.param("l0.ffn1.w")))
+    assert len(P.grad_buckets()) >= 1
+    # equal up to the run-to-run order of fp32 atomics (embedding rows, split-K partials)
+    assert max(rel_errs(out[1][0], out[0][0]).values()) <= 1e-6
+    assert np.allclose(out[1][1], out[0][1], rtol=1e-6, atol=1e-9)
