@@ -70,7 +70,12 @@ typedef enum {
                           batch statistics over all samples even when split (R13)      */
   TS_OP_MAXPOOL = 15,  /* in X[N,H,W,C] out [N,P,Q,C]; iattr {k, stride, pad}           */
   TS_OP_AVGPOOL = 16,  /* global average: in X[N,H,W,C] out [N,C]                       */
-  TS_OP_FLATTEN = 17   /* in X[N,...] out [N, prod(...)] (copy)                          */
+  TS_OP_FLATTEN = 17,  /* in X[N,...] out [N, prod(...)] (copy)                          */
+  TS_OP_ATTENTION = 18 /* fused attention: in Q[T,h], K[T,h], V[T,h];
+                          out C[T,h] = dropout(softmax(alpha Q_h K_h^T)) V_h (heads merged)
+                          and lse[b,a,s] (f32, auxiliary: read only by its own backward,
+                          never differentiated); iattr {heads, seq, dropout seed},
+                          fattr {alpha, p}; dropout mask = Philox on the [b,a,s,s] index  */
 } ts_op_kind;
 
 typedef struct {

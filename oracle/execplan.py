@@ -108,10 +108,13 @@ def execute(graph, cfg, params, inputs, step=0):
                             view(out, s0, s1, grad=True), val[xin], pval[gid], mu, var, s1_, s2_, m, eps)
             elif it.kind in ("F", "R"):
                 y = net.forward_op(graph, o, val, row0=row0, elem0=elem0, step=step)
-                if an.is_loss[out]:
-                    store[(out, 0)] += y
-                else:
-                    view(out, s0, s1)[...] = y
+                ys = y if isinstance(y, tuple) else (y,)
+                for t, yt in zip(o["outputs"], ys):
+                    if an.is_loss[t]:
+                        store[(t, 0)] += yt
+                    elif it.kind == "F" or t == it.writes[0][0]:
+                        # a replay regenerates only its target piece (other outputs may be away)
+                        view(t, s0, s1)[...] = yt
             else:
                 dy = None if an.is_loss[out] else view(out, s0, s1, grad=True)
                 contrib = net.backward_op(graph, o, val, dy, row0=row0, elem0=elem0, step=step)

@@ -46,6 +46,10 @@ def forward_op(graph, op, val, row0=0, elem0=0, step=0):
         return ops.attn_qk_fwd(x[0], x[1], ia[0], ia[1], fa[0])
     if k == "attn_pv":
         return ops.attn_pv_fwd(x[0], x[1], ia[0], ia[1])
+    if k == "attention":  # two outputs: (C, lse); dropout offset from the first sample
+        b0 = row0 // ia[1]
+        return ops.attention_fwd(x[0], x[1], x[2], ia[0], ia[1], fa[0], fa[1], ia[2],
+                                 b0 * ia[0] * ia[1] * ia[1], step)
     if k == "embed":
         return ops.embed_fwd(x[0], x[1], x[2], x[3], x[4], ia[0], row0)
     if k == "cls":
@@ -98,6 +102,11 @@ def backward_op(graph, op, val, dy, row0=0, elem0=0, step=0):
     elif k == "attn_pv":
         dp, dv = ops.attn_pv_bwd(dy, x[0], x[1], ia[0], ia[1])
         out = {ins[0]: dp, ins[1]: dv}
+    elif k == "attention":
+        b0 = row0 // ia[1]
+        dq, dk, dv = ops.attention_bwd(dy, x[0], x[1], x[2], ia[0], ia[1], fa[0], fa[1], ia[2],
+                                       b0 * ia[0] * ia[1] * ia[1], step)
+        out = {ins[0]: dq, ins[1]: dk, ins[2]: dv}
     elif k == "embed":
         shapes = [graph["tensors"][i]["shape"] for i in ins[2:5]]
         dw, dp, dt = ops.embed_bwd(dy, x[0], x[1], ia[0], row0, shapes)
@@ -128,12 +137,23 @@ def backward_op(graph, op, val, dy, row0=0, elem0=0, step=0):
     return out
 
 
+# Auxiliary outputs: statistics an op saves for its own backward, never read by another
+# op and never differentiated (the fused attention's row log-sum-exp).
+AUX_OUTPUTS = {"attention": (1,)}
+
+
+def grad_outputs(op):
+    """The outputs of `op` that carry a gradient."""
+    aux = AUX_OUTPUTS.get(op["kind"], ())
+    return [t for i, t in enumerate(op["outputs"]) if i not in aux]
+
+
 def needs_grad(graph):
     """Tensor ids that carry a gradient: params, and activations downstream of one."""
     ng = {t["id"] for t in graph["tensors"] if t["kind"] == "param"}
     for op in graph["ops"]:
         if any(i in ng for i in op["inputs"]):
-            ng.update(op["outputs"])
+            ng.update(grad_outputs(op))
     return ng
 
 
@@ -160,9 +180,12 @@ def train_step(graph, params, inputs, step=0, storage=None):
     rnd = ops.round_bf16 if storage == "bf16" else (lambda a: a)
     val = initial_values(graph, params, inputs)
     loss_id = next(op["outputs"][0] for op in graph["ops"] if op["kind"] == "xent")
+    ts = graph["tensors"]
     for op in graph["ops"]:
         y = forward_op(graph, op, val, step=step)
-        val[op["outputs"][0]] = y if op["outputs"][0] == loss_id else rnd(y)
+        ys = y if isinstance(y, tuple) else (y,)
+        for t, yt in zip(op["outputs"], ys):
+            val[t] = rnd(yt) if ts[t]["dtype"] == "bf16" else yt
     ng = needs_grad(graph)
     is_act = {t["id"] for t in graph["tensors"] if t["kind"] == "act"}
     grad = {}

@@ -196,6 +196,31 @@ def attn_pv_bwd(dc, p, v, heads, seq):
     return dp, _merge(dv)
 
 
+def attention_fwd(q, k, v, heads, seq, alpha, p, seed, elem0, step=0):
+    """Fused attention micro-op (the composition of attn_qk,
+    softmax, dropout and attn_pv, P:L119's attention block): C = dropout(softmax(
+    alpha Q_h K_h^T)) V_h with heads merged, plus the row log-sum-exp
+    lse[b,a,i] = log sum_j exp(S_ij) that its backward reads.  The dropout mask is the
+    unfused op's: Philox on the element index of the [b,a,s,s] probabilities
+    (elem0 = first sample's offset there), so fused and unfused graphs compute the
+    same function."""
+    s = attn_qk_fwd(q, k, heads, seq, alpha)
+    m = s.max(axis=-1, keepdims=True)
+    lse = (m + np.log(np.exp(s - m).sum(axis=-1, keepdims=True)))[..., 0]
+    pd = dropout_fwd(softmax_fwd(s), p, seed, elem0, step)
+    return attn_pv_fwd(pd, v, heads, seq), lse
+
+
+def attention_bwd(dc, q, k, v, heads, seq, alpha, p, seed, elem0, step=0):
+    """VJP of attention_fwd w.r.t. Q, K, V: the chain rule through the same four ops."""
+    pr = softmax_fwd(attn_qk_fwd(q, k, heads, seq, alpha))
+    pd = dropout_fwd(pr, p, seed, elem0, step)
+    dpd, dv = attn_pv_bwd(dc, pd, v, heads, seq)
+    ds = softmax_bwd(dropout_bwd(dpd, p, seed, elem0, step), pr)
+    dq, dk = attn_qk_bwd(ds, q, k, heads, seq, alpha)
+    return dq, dk, dv
+
+
 def embed_fwd(ids, tt, wword, wpos, wtype, seq, row0):
     pos = (np.arange(row0, row0 + ids.shape[0]) % seq)
     return wword[ids] + wpos[pos] + wtype[tt]

@@ -51,7 +51,9 @@ SAVED = {
     "maxpool": ("in", 0),
     "avgpool": None,
     "flatten": None,
+    "attention": (("in", 0, 1, 2), ("out", 0, 1)),  # Q, K, V, C, lse (D-SAVED)
 }
+AUX_OUTPUTS = {"attention": (1,)}  # never differentiated (same rule as net.AUX_OUTPUTS)
 
 # Ops whose statistics span the whole batch ("the merge of
 # micro-tensors can be required by the operation (e.g., batch normalization)"):
@@ -162,18 +164,20 @@ def analyze(graph):
     ng = {t["id"] for t in ts if t["kind"] == "param"}
     for o in ops:
         if any(i in ng for i in o["inputs"]):
-            ng.update(o["outputs"])
+            aux = AUX_OUTPUTS.get(o["kind"], ())
+            ng.update(t for i, t in enumerate(o["outputs"]) if i not in aux)
     has_bwd = [o["kind"] == "xent" or any(i in ng for i in o["inputs"]) for o in ops]
     saved = []
     for o in ops:
         spec = SAVED[o["kind"]]
         lst = []
         if spec is not None:
-            src = o["inputs"] if spec[0] == "in" else o["outputs"]
-            for idx in spec[1:]:
-                t = src[idx]
-                if ts[t]["kind"] != "param" and t not in lst:
-                    lst.append(t)
+            for part in (spec if isinstance(spec[0], tuple) else (spec,)):
+                src = o["inputs"] if part[0] == "in" else o["outputs"]
+                for idx in part[1:]:
+                    t = src[idx]
+                    if ts[t]["kind"] != "param" and t not in lst:
+                        lst.append(t)
         saved.append(lst)
     return Analysis(n, producer, sample, is_loss, ng, has_bwd, saved, [tbytes(t) for t in ts])
 
@@ -320,7 +324,7 @@ def expand(graph, cfg, order=None, an=None):
             b = Item("B", o, k, group=gid)
             b.reads = list(saved_pieces)
             for t in ops[o]["outputs"]:
-                if not an.is_loss[t]:
+                if not an.is_loss[t] and t in an.needs_grad:
                     b.reads.append((n + t, piece(t, k, P)))
                     if ops[o]["kind"] in BATCH_REDUCE and k == 0:
                         for j in range(p_of(t)):

@@ -110,7 +110,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
       b.group = gid;
       b.reads = saved;
       for (int x : op.out)
-        if (!g.t[x].is_loss) {
+        if (!g.t[x].is_loss && g.t[x].needs_grad) {
           b.reads.push_back(pk(n + x, piece(x, k, P)));
           if (batch_reduce(op.kind) && k == 0)
             for (int j = 0; j < piece_count(g, cfg, x); ++j)

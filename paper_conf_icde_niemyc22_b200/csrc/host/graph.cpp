@@ -86,6 +86,21 @@ bool validate_op(const Graph& g, const Op& o, std::string& why) {
       if ((qk.shape[1] / heads) % 8) return (why = "head dim must be a multiple of 8"), false;
       return true;
     }
+    case TS_OP_ATTENTION: {
+      if (!need(3, 2)) return false;
+      if (o.ia.size() < 3 || o.fa.size() < 2) return (why = "attention attrs {heads, seq, seed} {alpha, p}"), false;
+      const int64_t heads = o.ia[0], seq = o.ia[1];
+      const Tensor &q = T(o.in[0]), &c = T(o.out[0]), &l = T(o.out[1]);
+      if (heads < 1 || seq < 1 || q.ndim != 2 || q.shape[1] % heads || q.shape[0] % seq) return (why = "attention [T,h]"), false;
+      if (!same_shape(q, T(o.in[1])) || !same_shape(q, T(o.in[2])) || !same_shape(q, c))
+        return (why = "attention Q/K/V/C shapes"), false;
+      if (l.ndim != 3 || l.shape[0] * seq != q.shape[0] || l.shape[1] != heads || l.shape[2] != seq ||
+          l.dtype != TS_F32)
+        return (why = "attention lse must be f32 [b,a,s]"), false;
+      if ((q.shape[1] / heads) % 8) return (why = "head dim must be a multiple of 8"), false;
+      if (o.fa[1] < 0 || o.fa[1] >= 1) return (why = "attention dropout p"), false;
+      return true;
+    }
     case TS_OP_EMBED: {
       if (!need(5, 1)) return false;
       const Tensor &ids = T(o.in[0]), &tt = T(o.in[1]), &y = T(o.out[0]);
@@ -174,6 +189,7 @@ std::vector<int> saved_of(const Graph& g, const Op& o) {
       break;
     case TS_OP_RELU: case TS_OP_TANH: case TS_OP_SOFTMAX: src = {o.out[0]}; break;
     case TS_OP_ATTN_QK: case TS_OP_ATTN_PV: case TS_OP_EMBED: case TS_OP_XENT: src = {o.in[0], o.in[1]}; break;
+    case TS_OP_ATTENTION: src = {o.in[0], o.in[1], o.in[2], o.out[0], o.out[1]}; break;
     default: break;
   }
   std::vector<int> r;
@@ -252,7 +268,13 @@ ts_status build_graph(const ts_tensor_desc* td, int nt, const ts_op_desc* od, in
       t.rows_per_sample = t.shape[0] / samples;
       t.elems_per_sample = t.numel / samples;
     }
-    if (t.kind == TS_ACT && t.dtype != dtype && !t.is_loss)
+    bool aux = false;
+    if (t.producer >= 0) {
+      const Op& po = g.ops[t.producer];
+      for (size_t i = 0; i < po.out.size(); ++i)
+        if (po.out[i] == t.id && aux_output(po.kind, int(i))) aux = true;
+    }
+    if (t.kind == TS_ACT && t.dtype != dtype && !t.is_loss && !aux)
       return set_error("activation dtype must equal the compute dtype"), TS_ERR_GRAPH;
   }
   // needs_grad: params, and everything downstream of one (in definition order
@@ -264,8 +286,10 @@ ts_status build_graph(const ts_tensor_desc* td, int nt, const ts_op_desc* od, in
       bool any = false;
       for (int x : o.in) any |= g.t[x].needs_grad;
       if (any)
-        for (int x : o.out)
-          if (!g.t[x].needs_grad) g.t[x].needs_grad = changed = true;
+        for (size_t i = 0; i < o.out.size(); ++i) {
+          const int x = o.out[i];
+          if (!aux_output(o.kind, int(i)) && !g.t[x].needs_grad) g.t[x].needs_grad = changed = true;
+        }
     }
   }
   for (auto& o : g.ops) {

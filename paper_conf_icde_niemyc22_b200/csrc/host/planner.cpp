@@ -79,6 +79,20 @@ OpCost op_cost(const Graph& g, int oi) {
       c.bytes_f = 2 * nb(o.in[0]);
       c.bytes_b = 2 * nb(o.in[0]);
       break;
+    case TS_OP_ATTENTION: {
+      // fused: 2 products forward (S = QK^T, C = PV), 7 backward (dQ kernel: S, dP, dQ;
+      // dK/dV kernel: S, dP, dV, dK); no [b,a,s,s] tensor touches HBM
+      const Tensor& q = g.t[o.in[0]];
+      const double heads = double(o.ia[0]), seq = double(o.ia[1]);
+      const double d = double(q.shape[1]) / heads, nbt = double(q.shape[0]) / seq;
+      const double unit = 2.0 * nbt * heads * seq * seq * d;
+      c.flop_f = 2 * unit;
+      c.flop_b = 7 * unit;
+      c.bytes_f = 4 * nb(o.in[0]) + nb(o.out[1]);
+      c.bytes_b = 8 * nb(o.in[0]) + 2 * nb(o.out[1]);
+      c.kern_b = 3;
+      break;
+    }
     case TS_OP_CONV2D: {
       const Tensor &w = g.t[o.in[1]], &y = g.t[o.out[0]];
       const double rsc = double(w.shape[1]) * w.shape[2] * w.shape[3];

@@ -14,7 +14,7 @@ LIB_PATH = os.path.join(_PKG, "libtsplit.so")
 
 OPS = {"linear": 0, "relu": 1, "gelu": 2, "tanh": 3, "layernorm": 4, "add": 5, "dropout": 6,
        "softmax": 7, "attn_qk": 8, "attn_pv": 9, "embed": 10, "cls": 11, "xent": 12,
-       "conv2d": 13, "batchnorm": 14, "maxpool": 15, "avgpool": 16, "flatten": 17}
+       "conv2d": 13, "batchnorm": 14, "maxpool": 15, "avgpool": 16, "flatten": 17, "attention": 18}
 DTYPES = {"f32": 0, "bf16": 1, "i32": 2}
 KINDS = {"param": 0, "input": 1, "label": 2, "act": 3}
 RESIDE, SWAP, RECOMPUTE = 0, 1, 2

@@ -157,3 +157,24 @@ def test_cnn_trace_bit_exact_random_plans(gname, seed):
     for t in brute.act_tensors(g):
         cfg[t] = (r.choice([0, 1, 2]), r.choice([1, 2, 4]), r.choice([1, 2]))
     _compare(g, cfg)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_trace_bit_exact_random_plans_bert_tiny_fused_attention(seed):
+    """Fused attention (two outputs, one auxiliary): schedule, replays of either
+    output, and the allocation trace equal the oracle simulator's."""
+    g = graphs.config_graph("bert_tiny", fused_attention=True)
+    r = random.Random(100 + seed)
+    cfg = sim.default_cfg(g)
+    for t in brute.act_tensors(g):
+        cfg[t] = (r.choice([0, 1, 2]), r.choice([1, 2, 4]), r.choice([1, 2, 3]))
+    _compare(g, cfg)
+
+
+def test_fused_attention_large_default_and_planned():
+    g = graphs.config_graph("bert_large", fused_attention=True)
+    G = tsplit.Graph(g)
+    st = tsplit.Plan.default(G).stats()
+    assert st["peak_extent"] == sim.simulate(g, sim.default_cfg(g)).peak_extent
+    P = tsplit.Plan.plan(G, st["static_bytes"] + (st["peak_extent"] - st["static_bytes"]) // 4)
+    assert P.stats()["peak_extent"] <= st["static_bytes"] + (st["peak_extent"] - st["static_bytes"]) // 4

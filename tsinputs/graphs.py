@@ -69,6 +69,20 @@ class GraphBuilder:
         })
         return out
 
+    def op_multi(self, kind, name, inputs, outs, iattrs=(), fattrs=()):
+        """An op with several outputs: outs = [(name, shape, dtype or None)]."""
+        ids = [self.tensor(n, sh, "act", dtype=dt) for n, sh, dt in outs]
+        self.ops.append({
+            "id": len(self.ops),
+            "kind": kind,
+            "name": name,
+            "inputs": list(inputs),
+            "outputs": ids,
+            "iattrs": [int(v) for v in iattrs],
+            "fattrs": [float(v) for v in fattrs],
+        })
+        return ids
+
     def done(self) -> dict:
         return {
             "name": self.name,
@@ -100,19 +114,25 @@ def mlp(batch=8, hidden=256, depth=3, in_dim=256, classes=10, dtype="f32") -> di
 
 
 def bert(layers=24, hidden=1024, heads=16, seq=512, batch=32, vocab=30522, ffn=None,
-         classes=2, dtype="bf16", attn_dropout=0.1, emb_dropout=0.1, seed=1234) -> dict:
+         classes=2, dtype="bf16", attn_dropout=0.1, emb_dropout=0.1, seed=1234,
+         fused_attention=False) -> dict:
     """Canonical unfused BERT encoder + pooler/classifier head (MRPC-like).
 
     Per layer it emits exactly the tensors SURVEY.md §4 T2 reconciles with
     PAPER.md Table II (L85-112): 3 x [b,a,s,s] (scores, softmax, attention
     dropout), 2 x [T,4h] (FFN1, GELU), 10 x [T,h] (Q, K, V, context, proj, res1,
     LN1, FFN2, res2, LN2), weights 2 x [h,4h] and 4 x [h,h].
+
+    fused_attention=True replaces scores/probs/attn_drop/ctx by
+    one "attention" op: in (Q, K, V), out (ctx [T,h], lse [b,a,s] f32); iattrs
+    {heads, seq, dropout seed}, fattrs {alpha, p}; the same function (same seeds).
     """
     ffn = ffn or 4 * hidden
     assert hidden % heads == 0
     dh = hidden // heads
     T = batch * seq
-    g = GraphBuilder(f"bert_L{layers}_h{hidden}_a{heads}_s{seq}_b{batch}", dtype, batch)
+    g = GraphBuilder(f"bert_L{layers}_h{hidden}_a{heads}_s{seq}_b{batch}" + ("_fa" if fused_attention else ""),
+                     dtype, batch)
     ids = g.tensor("input_ids", (T,), "input", dtype="i32")
     tts = g.tensor("token_type_ids", (T,), "input", dtype="i32")
     labels = g.tensor("labels", (batch,), "label", dtype="i32")
@@ -136,11 +156,17 @@ def bert(layers=24, hidden=1024, heads=16, seq=512, batch=32, vocab=30522, ffn=N
         q = lin("q", x, hidden, hidden)
         k = lin("k", x, hidden, hidden)
         v = lin("v", x, hidden, hidden)
-        s = g.op("attn_qk", p + "scores", [q, k], (batch, heads, seq, seq), iattrs=[heads, seq], fattrs=[alpha])
-        pr = g.op("softmax", p + "probs", [s], (batch, heads, seq, seq))
-        pd = g.op("dropout", p + "attn_drop", [pr], (batch, heads, seq, seq), fattrs=[attn_dropout],
-                  iattrs=[seed + 1 + l])
-        c = g.op("attn_pv", p + "ctx", [pd, v], (T, hidden), iattrs=[heads, seq])
+        if fused_attention:
+            c, _ = g.op_multi("attention", p + "attn", [q, k, v],
+                              [(p + "ctx", (T, hidden), None), (p + "lse", (batch, heads, seq), "f32")],
+                              iattrs=[heads, seq, seed + 1 + l], fattrs=[alpha, attn_dropout])
+        else:
+            s = g.op("attn_qk", p + "scores", [q, k], (batch, heads, seq, seq), iattrs=[heads, seq],
+                     fattrs=[alpha])
+            pr = g.op("softmax", p + "probs", [s], (batch, heads, seq, seq))
+            pd = g.op("dropout", p + "attn_drop", [pr], (batch, heads, seq, seq), fattrs=[attn_dropout],
+                      iattrs=[seed + 1 + l])
+            c = g.op("attn_pv", p + "ctx", [pd, v], (T, hidden), iattrs=[heads, seq])
         o = lin("proj", c, hidden, hidden)
         r1 = g.op("add", p + "res1", [o, x], (T, hidden))
         g1 = g.param(p + "ln1.g", (hidden,))
