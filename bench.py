@@ -46,10 +46,10 @@ WORKLOADS = {
 }
 
 
-def workload_graph(wl, layers=LAYERS):
+def workload_graph(wl, layers=LAYERS, fused=True):
     from tsinputs import graphs
     if wl == "bert_large":
-        return graphs.bert(layers=layers, batch=BATCH)
+        return graphs.bert(layers=layers, batch=BATCH, fused_attention=fused)
     return graphs.config_graph(wl)
 
 
@@ -279,6 +279,8 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="tsplit", choices=["tsplit", "reference"])
     ap.add_argument("--workload", default="bert_large", choices=sorted(WORKLOADS))
+    ap.add_argument("--attention", default="fused", choices=["fused", "unfused"],
+                    help="BERT: one fused attention op per layer (SURVEY f2) or the paper's unfused graph")
     ap.add_argument("--budget-frac", type=float, default=None)
     ap.add_argument("--layers", type=int, default=LAYERS)
     ap.add_argument("--no-unbudgeted", action="store_true")
@@ -323,7 +325,7 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    spec = workload_graph(args.workload, args.layers)
+    spec = workload_graph(args.workload, args.layers, fused=args.attention == "fused")
     G = tsplit.Graph(spec)
     base = tsplit.Plan.default(G)
     bst = base.stats()
@@ -436,6 +438,7 @@ def main():
                        "one FFN1-forward launch from the committed ncu --set full capture"}
     config = {
         "workload": W["name"], "model": W["model"] if cnn else f"bert-large ({args.layers}L h{HID} a{HEADS} s{SEQ})",
+        "attention": None if cnn else args.attention,
         "global_batch": batch * world, "seq_len": W["seq_len"], "parallelism": f"dp{world}",
         "budget_frac_of_unsplit_dynamic_peak": args.budget_frac,
         "budget_bytes": budget, "unsplit_peak_bytes": unsplit_peak, "static_bytes": static,

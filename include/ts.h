@@ -304,6 +304,20 @@ ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K,
 ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void* x, const void* w, const void* dy,
                     void* out, const void* bias, int32_t acc, void* stream, int32_t* used_tc);
 
+/* Fused attention micro-op kernels (unit tests; the session uses the same ones).
+ * Cites: SURVEY.md §8(f) f2; semantics of TS_OP_ATTENTION above.  Q, K, V, C, dC, dQ,
+ * dK, dV: device [nb*seq, heads*d] (row stride heads*d); lse: device fp32 [nb, heads, seq];
+ * ws: device fp32 scratch >= nb*heads*seq floats (backward).  geom = {nb, heads, seq, d,
+ * dropout seed, b0 (global index of the first sample, for the dropout counters), step};
+ * fattr = {alpha, p}.  mode 1: forward (writes C and lse; either may be NULL);
+ * mode 2: backward (reads Q, K, V, C, lse, dC; writes dQ, dK, dV, any may be NULL;
+ * acc bit 0/1/2 adds into dQ/dK/dV).  mode | 0x10 forces the CUDA-core kernels.
+ * dtype TS_BF16 with d = 64 and seq % 64 == 0 runs the tensor-core (mma.sync) kernels.
+ * *used_tc reports the path.  Errors: TS_ERR_ARG, TS_ERR_CUDA. */
+ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const float* fattr, const void* q,
+                       const void* k, const void* v, void* c, float* lse, const void* dc, void* dq, void* dk,
+                       void* dv, int32_t acc, float* ws, void* stream, int32_t* used_tc);
+
 #ifdef __cplusplus
 }
 #endif

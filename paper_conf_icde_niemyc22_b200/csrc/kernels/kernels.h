@@ -95,6 +95,30 @@ void bn_bwd_sums(int dt, const PieceList& dy, const PieceList& x, const void* ga
 // dx (+)= rstd * (dy*gamma - s1/m - xhat*s2/m), m = rows of the whole batch
 void bn_bwd_apply(int dt, const void* dy, const void* x, const float* stats, const void* gamma, void* dx, int acc,
                   int64_t rows, int C, int64_t m_total, cudaStream_t st);
+// ---- fused attention (attention.cu) -----------------------------
+// Q, K, V, C, dC, dQ, dK, dV: [nb*seq, ld] with head a at columns a*d..(a+1)*d;
+// lse [nb, heads, seq] fp32; ws >= nb*heads*seq floats (backward row terms D_i).
+// Dropout: Philox on the [b,a,s,s] element index with b = b0 + local sample.
+struct AttnArgs {
+  int dtype = BF16;
+  int nb = 0, heads = 0, seq = 0, d = 0;
+  int64_t ld = 0;
+  const void *q = nullptr, *k = nullptr, *v = nullptr;
+  void* c = nullptr;       // forward output (may be null: a replay regenerating only lse)
+  float* lse = nullptr;    // forward output (may be null) / backward input
+  const void* dc = nullptr;
+  void *dq = nullptr, *dk = nullptr, *dv = nullptr;
+  int acc_q = 0, acc_k = 0, acc_v = 0;
+  float alpha = 1.f, p = 0.f;
+  uint32_t seed = 0, step = 0, thr = 0;
+  int64_t b0 = 0;
+  float* ws = nullptr;
+};
+bool attention_tc_eligible(const AttnArgs& a);  // bf16, d = 64, seq % 64 == 0 (mma.sync path)
+void attention_fwd(const AttnArgs& a, cudaStream_t st);
+void attention_bwd(const AttnArgs& a, cudaStream_t st);  // needs a.c (= O), a.lse, a.dc
+void attention_simt(const AttnArgs& a, bool bwd, cudaStream_t st);  // CUDA-core kernels only (tests)
+
 // ---- pooling (NHWC) ----------------------------------------------------------------
 void maxpool_fwd(int dt, const void* x, void* y, int n, int H, int W, int C, int P, int Q, int k, int stride,
                  int pad, cudaStream_t st);

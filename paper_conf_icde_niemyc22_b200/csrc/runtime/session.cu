@@ -106,6 +106,7 @@ struct Micro {
   bool replay = false;
   int64_t s0, s1;
   tsk::PieceList all_x, all_dy;  // batch-statistics ops at k = 0: every piece (R13)
+  std::set<int> writes;          // tensor ids (values) this item writes
   std::unordered_map<int, char*> val, grad;
   std::unordered_map<int, int> acc;  // grad key -> accumulate flag
 };
@@ -466,6 +467,54 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       const int acc = A(g.n() + o.in[0]);
       return [=](cudaStream_t st) { tsk::axpy(dt, dy, dx, acc, n_out, st); };
     }
+    case TS_OP_ATTENTION: {
+      const Tensor& q = g.t[o.in[0]];
+      tsk::AttnArgs a;
+      a.dtype = dt;
+      a.heads = int(o.ia[0]);
+      a.seq = int(o.ia[1]);
+      a.nb = int(ns);
+      a.d = int(q.shape[1] / a.heads);
+      a.ld = q.shape[1];
+      a.q = V(o.in[0]);
+      a.k = V(o.in[1]);
+      a.v = V(o.in[2]);
+      a.alpha = float(o.fa[0]);
+      a.p = float(o.fa[1]);
+      a.seed = uint32_t(o.ia[2]);
+      a.b0 = m.s0;
+      a.ws = ws;
+      if (!bwd) {
+        // a replay writes only the output it regenerates
+        a.c = m.writes.count(o.out[0]) ? V(o.out[0]) : nullptr;
+        a.lse = m.writes.count(o.out[1]) ? reinterpret_cast<float*>(V(o.out[1])) : nullptr;
+        nk = 1;
+        return [a, stepp](cudaStream_t st) {
+          tsk::AttnArgs b = a;
+          b.step = *stepp;
+          tsk::attention_fwd(b, st);
+        };
+      }
+      a.c = V(o.out[0]);
+      a.lse = reinterpret_cast<float*>(V(o.out[1]));
+      a.dc = G(o.out[0]);
+      auto gslot = [&](int i, void*& ptr, int& acc) {
+        const Tensor& x = g.t[o.in[i]];
+        if (x.kind == TS_ACT && x.needs_grad) {
+          ptr = G(o.in[i]);
+          acc = A(g.n() + o.in[i]);
+        }
+      };
+      gslot(0, a.dq, a.acc_q);
+      gslot(1, a.dk, a.acc_k);
+      gslot(2, a.dv, a.acc_v);
+      nk = 2;
+      return [a, stepp](cudaStream_t st) {
+        tsk::AttnArgs b = a;
+        b.step = *stepp;
+        tsk::attention_bwd(b, st);
+      };
+    }
     case TS_OP_XENT: {
       const int C = int(g.t[o.in[0]].shape[1]);
       const float inv_b = 1.f / float(B);
@@ -613,6 +662,12 @@ ts_status build_program(ts_session_t* s) {
         }
       }
       m.replay = it.kind == IT_R;
+      for (PieceKey pc : it.writes)
+        if (pk_key(pc) < n) m.writes.insert(pk_key(pc));
+      if (o.kind == TS_OP_ATTENTION) {
+        const uint64_t need = uint64_t(m.s1 - m.s0) * uint64_t(o.ia[0]) * uint64_t(o.ia[1]) * 4;
+        if (need + 4096 > g.ws_bytes) return set_error("attention: workspace too small for the row terms"), TS_ERR_GRAPH;
+      }
       if (batch_reduce(o.kind) && it.k == 0 && it.kind != IT_R) {  // replays reuse the step's statistics
         const int C = int(g.t[o.in[0]].shape[g.t[o.in[0]].ndim - 1]);
         if (!tsk::bn_supported(g.dtype == TS_BF16 ? tsk::BF16 : tsk::F32, C))
@@ -1215,6 +1270,38 @@ ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void
   if (!tc) tsk::conv_simt(mode, a, out, bias, acc, st);
   CU(cudaGetLastError());
   if (used_tc) *used_tc = tc;
+  return TS_OK;
+}
+
+ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const float* fattr, const void* q,
+                       const void* k, const void* v, void* c, float* lse, const void* dc, void* dq, void* dk,
+                       void* dv, int32_t acc, float* ws, void* stream, int32_t* used_tc) {
+  const bool simt_only = (mode & 0x10) != 0;
+  mode &= 0xF;
+  if (!geom || !fattr || (mode != 1 && mode != 2) || (dtype != TS_BF16 && dtype != TS_F32) || !q || !k || !v)
+    return set_error("ts_attention: bad argument"), TS_ERR_ARG;
+  tsk::AttnArgs a;
+  a.dtype = dtype == TS_BF16 ? tsk::BF16 : tsk::F32;
+  a.nb = geom[0]; a.heads = geom[1]; a.seq = geom[2]; a.d = geom[3];
+  a.seed = uint32_t(geom[4]); a.b0 = geom[5]; a.step = uint32_t(geom[6]);
+  a.alpha = fattr[0]; a.p = fattr[1];
+  if (a.nb < 1 || a.heads < 1 || a.seq < 1 || a.d < 1 || a.d > 1024 || a.p < 0.f || a.p >= 1.f)
+    return set_error("ts_attention: bad geometry"), TS_ERR_ARG;
+  a.ld = int64_t(a.heads) * a.d;
+  a.q = q; a.k = k; a.v = v; a.c = c; a.lse = lse; a.dc = dc; a.dq = dq; a.dk = dk; a.dv = dv;
+  a.acc_q = acc & 1; a.acc_k = (acc >> 1) & 1; a.acc_v = (acc >> 2) & 1;
+  a.ws = ws;
+  if (mode == 2 && (!c || !lse || !dc || !ws)) return set_error("ts_attention: backward needs C, lse, dC, ws"), TS_ERR_ARG;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const bool tc = !simt_only && tsk::attention_tc_eligible(a);
+  if (tc) {
+    if (mode == 1) tsk::attention_fwd(a, st);
+    else tsk::attention_bwd(a, st);
+  } else {
+    tsk::attention_simt(a, mode == 2, st);
+  }
+  CU(cudaGetLastError());
+  if (used_tc) *used_tc = tc ? 1 : 0;
   return TS_OK;
 }
 

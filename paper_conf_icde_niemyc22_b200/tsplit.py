@@ -131,6 +131,8 @@ def lib():
             "ts_gemm_f32": (i32, [i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, C.c_float,
                                   vp, vp]),
             "ts_conv2d": (i32, [i32, i32, P(i32), vp, vp, vp, vp, vp, i32, vp, P(i32)]),
+            "ts_attention": (i32, [i32, i32, P(i32), P(C.c_float), vp, vp, vp, vp, vp, vp, vp, vp, vp, i32, vp, vp,
+                                   P(i32)]),
         }
         for name, (res, args) in list(sig.items()) + list(optional.items()):
             if not hasattr(L, name):
@@ -487,4 +489,23 @@ def conv2d(mode: int, geom, x, w, dy, out, bias=None, acc: int = 0, stream=None)
     used = C.c_int32(0)
     st = C.c_void_p(stream if stream is not None else torch.cuda.current_stream().cuda_stream)
     check(lib().ts_conv2d(mode, dt, g, ptr(x), ptr(w), ptr(dy), ptr(out), ptr(bias), acc, st, C.byref(used)))
+    return bool(used.value)
+
+
+def attention(mode: int, geom, alpha: float, p: float, q, k, v, c=None, lse=None, dc=None, dq=None, dk=None,
+              dv=None, acc: int = 0, ws=None, stream=None) -> bool:
+    """One fused-attention kernel call through the C ABI (`ts_attention`) on torch device
+    tensors (marshalling only).  geom = (nb, heads, seq, d, seed, b0, step).  Returns True
+    when the tensor-core kernels ran."""
+    import torch
+    dt = DTYPES["bf16"] if q.dtype == torch.bfloat16 else DTYPES["f32"]
+    g = (C.c_int32 * 7)(*[int(x) for x in geom])
+    fa = (C.c_float * 2)(alpha, p)
+    ptr = (lambda t: C.c_void_p(t.data_ptr()) if t is not None else None)
+    used = C.c_int32(0)
+    st = C.c_void_p(stream if stream is not None else torch.cuda.current_stream().cuda_stream)
+    lse_p = C.cast(C.c_void_p(lse.data_ptr()), C.POINTER(C.c_float)) if lse is not None else None
+    ws_p = C.c_void_p(ws.data_ptr()) if ws is not None else None
+    check(lib().ts_attention(mode, dt, g, fa, ptr(q), ptr(k), ptr(v), ptr(c), lse_p, ptr(dc), ptr(dq), ptr(dk),
+                             ptr(dv), acc, ws_p, st, C.byref(used)))
     return bool(used.value)
