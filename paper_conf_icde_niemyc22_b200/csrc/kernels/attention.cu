@@ -25,17 +25,38 @@ namespace {
 constexpr float kLog2e = 1.4426950408889634f;
 constexpr float kLn2 = 0.6931471805599453f;
 
-__device__ __forceinline__ uint2 philox_pair(uint64_t e, uint32_t seed, uint32_t step) {
-  // words (e & 3) and (e & 3) + 1 of Philox(counter = e >> 2); e is even
-  const uint64_t c = e >> 2;
-  const uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), step, 0u, seed, kPhiloxKey1);
-  return (e & 2) ? make_uint2(r.z, r.w) : make_uint2(r.x, r.y);
-}
 __device__ __forceinline__ uint32_t philox_one(uint64_t e, uint32_t seed, uint32_t step) {
   const uint64_t c = e >> 2;
   const uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), step, 0u, seed, kPhiloxKey1);
   const uint32_t w[4] = {r.x, r.y, r.z, r.w};
   return w[e & 3];
+}
+
+// Keep decisions of one 8-column n-tile of an mma.sync accumulator, for this thread's
+// (row r, cols 2t, 2t+1) and (row r + 8, same cols): the quad's 4 Philox calls (2 rows x
+// 2 four-column groups) are spread one per lane and the words exchanged by shuffles.
+// e0 = element index of (row r of lane 0's quad, column 0 of the n-tile); S = row stride.
+__device__ __forceinline__ void quad_keep(uint64_t e0, uint64_t S, uint32_t seed, uint32_t step, uint32_t thr,
+                                          bool (&k)[4]) {
+  const int lane = threadIdx.x & 31, t = lane & 3;
+  const uint64_t e = e0 + uint64_t(t & 1) * 8ull * S + uint64_t(4 * (t >> 1));
+  const uint64_t c = e >> 2;
+  const uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), step, 0u, seed, kPhiloxKey1);
+  const int src0 = (lane & ~3) | (t & 2), src1 = src0 | 1;
+  const uint32_t ax = __shfl_sync(0xffffffffu, r.x, src0), ay = __shfl_sync(0xffffffffu, r.y, src0);
+  const uint32_t az = __shfl_sync(0xffffffffu, r.z, src0), aw = __shfl_sync(0xffffffffu, r.w, src0);
+  const uint32_t bx = __shfl_sync(0xffffffffu, r.x, src1), by = __shfl_sync(0xffffffffu, r.y, src1);
+  const uint32_t bz = __shfl_sync(0xffffffffu, r.z, src1), bw = __shfl_sync(0xffffffffu, r.w, src1);
+  const bool hi = t & 1;
+  k[0] = (hi ? az : ax) >= thr;
+  k[1] = (hi ? aw : ay) >= thr;
+  k[2] = (hi ? bz : bx) >= thr;
+  k[3] = (hi ? bw : by) >= thr;
+}
+__device__ __forceinline__ float ex2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
 }
 
 // ============================================================ CUDA-core version
@@ -298,8 +319,8 @@ __global__ void __launch_bounds__(128) fa_fwd(AttnArgs A) {
   float m[2] = {-INFINITY, -INFINITY}, l[2] = {0.f, 0.f};
   uint32_t qa[4][4];
   const int r_lo = warp * 16 + (lane >> 2);  // rows of this thread within the CTA tile
-  const uint64_t erow0 = ((uint64_t(A.b0 + b) * A.heads + a) * S + qb * kBM + r_lo) * uint64_t(S);
-  const uint64_t erow1 = erow0 + 8ull * S;
+  // element index of (this quad's row r_lo, key 0) in the [b,a,s,s] probabilities
+  const uint64_t equad = ((uint64_t(A.b0 + b) * A.heads + a) * S + qb * kBM + r_lo) * uint64_t(S);
   for (int kb = 0; kb < nkb; ++kb) {
     if (kb + 1 < nkb) {
       load_tile(sK[(kb + 1) & 1], K + int64_t(kb + 1) * kBN * ld, ld, tid);
@@ -336,7 +357,7 @@ __global__ void __launch_bounds__(128) fa_fwd(AttnArgs A) {
       mx[h] = fmaxf(mx[h], __shfl_xor_sync(0xffffffffu, mx[h], 1));
       mx[h] = fmaxf(mx[h], __shfl_xor_sync(0xffffffffu, mx[h], 2));
     }
-    const float corr0 = exp2f(m[0] - mx[0]), corr1 = exp2f(m[1] - mx[1]);
+    const float corr0 = ex2(m[0] - mx[0]), corr1 = ex2(m[1] - mx[1]);
     m[0] = mx[0];
     m[1] = mx[1];
     l[0] *= corr0;
@@ -351,18 +372,17 @@ __global__ void __launch_bounds__(128) fa_fwd(AttnArgs A) {
     uint32_t pa[4][4];  // P as A fragments of the PV product (k = keys)
 #pragma unroll
     for (int n = 0; n < 8; ++n) {
-      float p0 = exp2f(s[n][0] * sl2 - m[0]), p1 = exp2f(s[n][1] * sl2 - m[0]);
-      float p2 = exp2f(s[n][2] * sl2 - m[1]), p3 = exp2f(s[n][3] * sl2 - m[1]);
+      float p0 = ex2(s[n][0] * sl2 - m[0]), p1 = ex2(s[n][1] * sl2 - m[0]);
+      float p2 = ex2(s[n][2] * sl2 - m[1]), p3 = ex2(s[n][3] * sl2 - m[1]);
       l[0] += p0 + p1;
       l[1] += p2 + p3;
       if (A.p > 0.f) {
-        const int key = kb * kBN + n * 8 + 2 * (lane & 3);
-        const uint2 w0 = philox_pair(erow0 + key, A.seed, A.step);
-        const uint2 w1 = philox_pair(erow1 + key, A.seed, A.step);
-        p0 = w0.x >= A.thr ? p0 : 0.f;
-        p1 = w0.y >= A.thr ? p1 : 0.f;
-        p2 = w1.x >= A.thr ? p2 : 0.f;
-        p3 = w1.y >= A.thr ? p3 : 0.f;
+        bool kp[4];
+        quad_keep(equad + uint64_t(kb * kBN + n * 8), uint64_t(S), A.seed, A.step, A.thr, kp);
+        p0 = kp[0] ? p0 : 0.f;
+        p1 = kp[1] ? p1 : 0.f;
+        p2 = kp[2] ? p2 : 0.f;
+        p3 = kp[3] ? p3 : 0.f;
       }
       const int kk = n >> 1;
       if ((n & 1) == 0) {
@@ -459,8 +479,7 @@ __global__ void __launch_bounds__(128) fa_bwd_dq(AttnArgs A) {
   }
   const float sl2 = A.alpha * kLog2e;
   const float keep_scale = A.p > 0.f ? 1.f / (1.f - A.p) : 1.f;
-  const uint64_t erow0 = ((uint64_t(A.b0 + b) * A.heads + a) * S + q0) * uint64_t(S);
-  const uint64_t erow1 = erow0 + 8ull * S;
+  const uint64_t equad = ((uint64_t(A.b0 + b) * A.heads + a) * S + q0) * uint64_t(S);
   uint32_t qa[4][4], ga[4][4];
   float dq[8][4] = {};
   const int nkb = S / kBN;
@@ -500,19 +519,18 @@ __global__ void __launch_bounds__(128) fa_bwd_dq(AttnArgs A) {
       float v4[4];
 #pragma unroll
       for (int e = 0; e < 4; ++e) {
-        const float pr = exp2f(s[n][e] * sl2 - lse2[e >> 1]);
+        const float pr = ex2(s[n][e] * sl2 - lse2[e >> 1]);
         v4[e] = pr;
       }
       float d0 = dp[n][0] * keep_scale, d1 = dp[n][1] * keep_scale, d2 = dp[n][2] * keep_scale,
             d3 = dp[n][3] * keep_scale;
       if (A.p > 0.f) {
-        const int key = kb * kBN + n * 8 + 2 * (lane & 3);
-        const uint2 w0 = philox_pair(erow0 + key, A.seed, A.step);
-        const uint2 w1 = philox_pair(erow1 + key, A.seed, A.step);
-        d0 = w0.x >= A.thr ? d0 : 0.f;
-        d1 = w0.y >= A.thr ? d1 : 0.f;
-        d2 = w1.x >= A.thr ? d2 : 0.f;
-        d3 = w1.y >= A.thr ? d3 : 0.f;
+        bool kp[4];
+        quad_keep(equad + uint64_t(kb * kBN + n * 8), uint64_t(S), A.seed, A.step, A.thr, kp);
+        d0 = kp[0] ? d0 : 0.f;
+        d1 = kp[1] ? d1 : 0.f;
+        d2 = kp[2] ? d2 : 0.f;
+        d3 = kp[3] ? d3 : 0.f;
       }
       const float s0 = v4[0] * (d0 - Dr[0]), s1 = v4[1] * (d1 - Dr[0]);
       const float s2 = v4[2] * (d2 - Dr[1]), s3 = v4[3] * (d3 - Dr[1]);
@@ -634,28 +652,34 @@ __global__ void __launch_bounds__(128) fa_bwd_dkv(AttnArgs A) {
       }
     // P, Pd, dS -> per-warp staging [query][key]
 #pragma unroll
-    for (int mt = 0; mt < 4; ++mt)
+    for (int mt = 0; mt < 4; ++mt) {
+      float l2[2], Dq[2];
 #pragma unroll
       for (int h = 0; h < 2; ++h) {
-        const int ql = mt * 16 + (lane >> 2) + 8 * h;  // query within the block
-        const int qg = qb * kBM + ql;
-        const float l2 = L[qg] * kLog2e, Dq = D[qg];
+        const int qg = qb * kBM + mt * 16 + (lane >> 2) + 8 * h;
+        l2[h] = L[qg] * kLog2e;
+        Dq[h] = D[qg];
+      }
 #pragma unroll
-        for (int nt = 0; nt < 2; ++nt) {
-          const int kl = nt * 8 + 2 * (lane & 3);  // key within the warp's 16
-          float p0 = exp2f(s[mt][nt][2 * h] * sl2 - l2), p1 = exp2f(s[mt][nt][2 * h + 1] * sl2 - l2);
+      for (int nt = 0; nt < 2; ++nt) {
+        bool kp[4] = {true, true, true, true};
+        if (A.p > 0.f)
+          quad_keep((ehead + qb * kBM + mt * 16 + (lane >> 2)) * uint64_t(S) + uint64_t(kb * kBN + key_w + nt * 8),
+                    uint64_t(S), A.seed, A.step, A.thr, kp);
+        const int kl = nt * 8 + 2 * (lane & 3);  // key within the warp's 16
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const int ql = mt * 16 + (lane >> 2) + 8 * h;  // query within the block
+          float p0 = ex2(s[mt][nt][2 * h] * sl2 - l2[h]), p1 = ex2(s[mt][nt][2 * h + 1] * sl2 - l2[h]);
           float d0 = dp[mt][nt][2 * h] * keep_scale, d1 = dp[mt][nt][2 * h + 1] * keep_scale;
           float pd0 = p0 * keep_scale, pd1 = p1 * keep_scale;
-          if (A.p > 0.f) {
-            const uint64_t e = (ehead + qg) * uint64_t(S) + uint64_t(kb * kBN + key_w + kl);
-            const uint2 w = philox_pair(e, A.seed, A.step);
-            if (w.x < A.thr) d0 = pd0 = 0.f;
-            if (w.y < A.thr) d1 = pd1 = 0.f;
-          }
+          if (!kp[2 * h]) d0 = pd0 = 0.f;
+          if (!kp[2 * h + 1]) d1 = pd1 = 0.f;
           *reinterpret_cast<uint32_t*>(stP + ql * kPS + kl * 2) = pack_bf16(pd0, pd1);
-          *reinterpret_cast<uint32_t*>(stS + ql * kPS + kl * 2) = pack_bf16(p0 * (d0 - Dq), p1 * (d1 - Dq));
+          *reinterpret_cast<uint32_t*>(stS + ql * kPS + kl * 2) = pack_bf16(p0 * (d0 - Dq[h]), p1 * (d1 - Dq[h]));
         }
       }
+    }
     __syncwarp();
     // dV_w += Pd^T dO, dK_w += dS^T Q (k = the 64 queries)
 #pragma unroll

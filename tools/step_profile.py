@@ -1,5 +1,5 @@
 """Per-micro-op cudaEvent breakdown of one BERT-Large step (eager, profiled) for the
-budgeted plan and the all-reside plan.  Usage: python tools/step_profile.py [budget_frac]"""
+budgeted plan and the all-reside plan.  Usage: python tools/step_profile.py [budget_frac] [fused]"""
 import collections
 import json
 import os
@@ -35,7 +35,8 @@ def profile(G, P, spec, params, dev):
 
 def main():
     frac = float(sys.argv[1]) if len(sys.argv) > 1 else 0.25
-    spec = graphs.bert(layers=24, batch=32)
+    fused = len(sys.argv) > 2 and sys.argv[2] == "fused"
+    spec = graphs.bert(layers=24, batch=32, fused_attention=fused)
     G = tsplit.Graph(spec)
     base = tsplit.Plan.default(G)
     st = base.stats()
