@@ -766,6 +766,7 @@ void attention_fwd(const AttnArgs& in, cudaStream_t st) {
   AttnArgs A = in;
   fill_thr(A);
   dim3 grid(A.seq, A.heads, A.nb);
+  if (attention_fwd_tc5(A, st)) return;  // tcgen05 (attention_tc.cu)
   if (tc_eligible(A)) {
     fa_fwd<<<dim3(A.seq / kBM, A.heads, A.nb), 128, 0, st>>>(A);
   } else if (A.dtype == BF16) {

@@ -1,0 +1,291 @@
+// Fused attention forward on the 5th-generation tensor cores (sm_100a), head dim 64,
+// seq a multiple of 128 up to 512 (BERT-Large / scaled BERT) — the same arithmetic as
+// attention.cu's kernels (dropout reading D-RNG).
+//
+// One CTA = 128 queries of one (sample, head).  The whole score row fits TMEM
+// (128 lanes x seq fp32 columns <= 512), so the softmax is exact, not online:
+//   1. one thread issues TMA loads of Q (128 x 64), K and V (seq x 64) into 128B-swizzled
+//      shared memory and the tcgen05.mma products S = Q K^T into TMEM;
+//   2. eight softmax warps (two per TMEM lane quarter, each owning half of the keys)
+//      read S with tcgen05.ld, take the row max (exchanged through shared memory),
+//      form P = exp2(S*alpha*log2e - max) with the Philox keep mask — a thread owns a
+//      row, so one Philox call covers four consecutive keys — and store bf16 P in the
+//      K-major UMMA layout over the dead K / Q buffers;
+//   3. as each key half lands, O += P_half V_half runs on the tensor cores (V is the
+//      MN-major B operand straight from its TMA tile) into TMEM columns 0..63;
+//   4. the first four warps scale O by 1 / (rowsum (1-p)), write C and the log-sum-exp.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <mutex>
+
+#include "common.cuh"
+#include "kernels.h"
+#include "tc_ptx.cuh"
+
+namespace tsk {
+
+namespace {
+
+using namespace tc;
+
+constexpr int kSoftWarps = 8;
+constexpr int kCtlWarp = kSoftWarps;
+constexpr int kThreads = 32 * (kSoftWarps + 1);
+constexpr int kRegion = 64 * 1024;
+constexpr int kSmem = 3 * kRegion + 2048 + 1024;  // PB(+Q) | K(=PA) | V | barriers + exchange
+
+constexpr float kLog2e = 1.4426950408889634f;
+constexpr float kLn2 = 0.6931471805599453f;
+
+__device__ __forceinline__ float ex2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+__device__ __forceinline__ void named_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n)); }
+__device__ __forceinline__ void sts128(uint32_t addr, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d) : "memory");
+}
+__device__ __forceinline__ uint32_t pk2(float lo, float hi) {
+  __nv_bfloat162 h = __floats2bfloat162_rn(lo, hi);
+  return *reinterpret_cast<uint32_t*>(&h);
+}
+
+struct Fa5P {
+  int nb, heads, seq;
+  int64_t ld;
+  float sl2;          // alpha * log2(e)
+  float p, keep_scale;
+  uint32_t seed, step, thr;
+  int64_t b0;
+  void* c;
+  float* lse;
+  int kbox;           // rows per K/V TMA box
+};
+
+__global__ void __launch_bounds__(kThreads, 1)
+    fa5_fwd(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mK,
+            const __grid_constant__ CUtensorMap mV, const Fa5P p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* rPB = smem;              // P keys [seq/2, seq); Q tile at its start until S is done
+  uint8_t* rK = smem + kRegion;     // K; then P keys [0, seq/2)
+  uint8_t* rV = smem + 2 * kRegion;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 3 * kRegion);
+  uint64_t *qk_full = bar, *v_full = bar + 1, *s_full = bar + 2, *p_full = bar + 3, *o_full = bar + 5;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 6);
+  float* red_m = reinterpret_cast<float*>(smem + 3 * kRegion + 256);
+  float* red_l = red_m + 256;
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int qt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
+  const int S = p.seq, half = S / 2;
+  if (threadIdx.x == 0) {
+    mbar_init(qk_full, 1);
+    mbar_init(v_full, 1);
+    mbar_init(s_full, 1);
+    mbar_init(&p_full[0], 128);
+    mbar_init(&p_full[1], 128);
+    mbar_init(o_full, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == kCtlWarp) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(512));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == kCtlWarp) {
+    if (lane == 0) {
+      const int row0 = b * S;
+      mbar_arrive_tx(qk_full, 128 * 128 + uint32_t(S) * 128);
+      tma_load(rPB, &mQ, qk_full, a * 64, row0 + qt * 128, 0, 0);
+      for (int j = 0; j < S; j += p.kbox) tma_load(rK + j * 128, &mK, qk_full, a * 64, row0 + j, 0, 0);
+      mbar_arrive_tx(v_full, uint32_t(S) * 128);
+      for (int j = 0; j < S; j += p.kbox) tma_load(rV + j * 128, &mV, v_full, a * 64, row0 + j, 0, 0);
+      // S = Q K^T: M 128, N 128 per instruction, K = 64 (4 steps of 16)
+      constexpr uint32_t idS = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(128 >> 3) << 17) |
+                               (uint32_t(128 >> 4) << 24);
+      mbar_wait(qk_full, 0);
+      tc_fence_after();
+      const uint32_t sq = smem_u32(rPB), sk = smem_u32(rK);
+      for (int c = 0; c < S / 128; ++c)
+#pragma unroll
+        for (int k = 0; k < 4; ++k)
+          tc_mma(tmem + uint32_t(c * 128), smem_desc(sq + k * 32, 16, 1024),
+                 smem_desc(sk + c * 16384 + k * 32, 16, 1024), idS, k > 0 ? 1u : 0u);
+      tc_commit(s_full);
+      // O = P V: M 128, N 64, K 16 per instruction; A = P (K-major), B = V (MN-major)
+      constexpr uint32_t idO = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | (uint32_t(64 >> 3) << 17) |
+                               (uint32_t(128 >> 4) << 24);
+      mbar_wait(v_full, 0);
+      const uint32_t sv = smem_u32(rV);
+      for (int h = 0; h < 2; ++h) {
+        mbar_wait(&p_full[h], 0);
+        tc_fence_after();
+        const uint32_t sp = smem_u32(h == 0 ? rK : rPB);
+        for (int kk = 0; kk < half; kk += 16) {
+          const uint32_t ad = sp + (kk >> 6) * 16384 + ((kk & 63) >> 4) * 32;
+          const uint32_t bd = sv + uint32_t(h * half + kk) * 128;
+          tc_mma(tmem, smem_desc(ad, 16, 1024), smem_desc(bd, 8192, 1024), idO, (h > 0 || kk > 0) ? 1u : 0u);
+        }
+      }
+      tc_commit(o_full);
+    }
+  } else {
+    // ===== softmax warps: row i, key half g =====
+    const int qq = warp & 3, g = warp >> 2;
+    const int i = qq * 32 + lane;
+    const uint32_t trow = tmem + (uint32_t(qq * 32) << 16);
+    const int c0 = g * half;
+    mbar_wait(s_full, 0);
+    tc_fence_after();
+    float m = -INFINITY;
+    for (int c = c0; c < c0 + half; c += 32) {
+      uint32_t r[32];
+      tmem_ld32(trow + uint32_t(c), r);
+#pragma unroll
+      for (int j = 0; j < 32; ++j) m = fmaxf(m, __uint_as_float(r[j]));
+    }
+    red_m[g * 128 + i] = m;
+    named_sync(1, 32 * kSoftWarps);
+    m = fmaxf(red_m[i], red_m[128 + i]) * p.sl2;
+    const uint64_t erow = ((uint64_t(p.b0 + b) * p.heads + a) * uint64_t(S) + uint64_t(qt * 128 + i)) * uint64_t(S);
+    float l = 0.f;
+    const uint32_t sp = smem_u32(g == 0 ? rK : rPB);
+    for (int c = c0; c < c0 + half; c += 32) {
+      uint32_t r[32];
+      tmem_ld32(trow + uint32_t(c), r);
+      float v[32];
+#pragma unroll
+      for (int j = 0; j < 32; ++j) {
+        v[j] = ex2(__uint_as_float(r[j]) * p.sl2 - m);
+        l += v[j];
+      }
+      if (p.p > 0.f) {
+#pragma unroll
+        for (int u = 0; u < 8; ++u) {
+          const uint64_t cnt = (erow + uint64_t(c + 4 * u)) >> 2;
+          const uint4 w = philox4x32_10(uint32_t(cnt), uint32_t(cnt >> 32), p.step, 0u, p.seed, kPhiloxKey1);
+          if (w.x < p.thr) v[4 * u] = 0.f;
+          if (w.y < p.thr) v[4 * u + 1] = 0.f;
+          if (w.z < p.thr) v[4 * u + 2] = 0.f;
+          if (w.w < p.thr) v[4 * u + 3] = 0.f;
+        }
+      }
+      // 32 keys = 4 sixteen-byte chunks of row i in the K-major SW128 layout
+      const int kl = c - c0;  // key within this half
+      const uint32_t blk = sp + uint32_t(kl >> 6) * 16384u + uint32_t(i) * 128u;
+#pragma unroll
+      for (int q4 = 0; q4 < 4; ++q4) {
+        const int chunk = ((kl & 63) >> 3) + q4;
+        sts128(blk + (uint32_t(chunk ^ (i & 7)) << 4), pk2(v[8 * q4], v[8 * q4 + 1]), pk2(v[8 * q4 + 2], v[8 * q4 + 3]),
+               pk2(v[8 * q4 + 4], v[8 * q4 + 5]), pk2(v[8 * q4 + 6], v[8 * q4 + 7]));
+      }
+    }
+    fence_async_smem();
+    tc_fence_before();
+    mbar_arrive(&p_full[g]);
+    red_l[g * 128 + i] = l;
+    named_sync(1, 32 * kSoftWarps);
+    if (g == 0) {
+      l = red_l[i] + red_l[128 + i];
+      mbar_wait(o_full, 0);
+      tc_fence_after();
+      const float inv = p.keep_scale / l;
+      const int q = qt * 128 + i;
+      bf16* crow = static_cast<bf16*>(p.c) + (int64_t(b) * S + q) * p.ld + a * 64;
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        uint32_t r[32];
+        tmem_ld32(trow + uint32_t(h * 32), r);
+        if (p.c) {
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            uint4 o;
+            o.x = pk2(__uint_as_float(r[8 * j]) * inv, __uint_as_float(r[8 * j + 1]) * inv);
+            o.y = pk2(__uint_as_float(r[8 * j + 2]) * inv, __uint_as_float(r[8 * j + 3]) * inv);
+            o.z = pk2(__uint_as_float(r[8 * j + 4]) * inv, __uint_as_float(r[8 * j + 5]) * inv);
+            o.w = pk2(__uint_as_float(r[8 * j + 6]) * inv, __uint_as_float(r[8 * j + 7]) * inv);
+            *reinterpret_cast<uint4*>(crow + h * 32 + 8 * j) = o;
+          }
+        }
+      }
+      if (p.lse) p.lse[(int64_t(b) * p.heads + a) * S + q] = (m + log2f(l)) * kLn2;
+    }
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  if (warp == kCtlWarp) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
+  }
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    cudaDriverEntryPointQueryResult q;
+    void* f = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(f);
+  });
+  return fn;
+}
+
+// [rows, ld] bf16 as a 4-D map (ld, rows, 1, 1) — tma_load issues the 4-D form —
+// box (64 columns, box_rows rows), 128-byte swizzle
+bool map2(CUtensorMap* m, const void* ptr, int64_t ld, int64_t rows, int box_rows) {
+  auto fn = encode();
+  if (!fn || reinterpret_cast<uintptr_t>(ptr) % 16 || (ld * 2) % 16) return false;
+  cuuint64_t dims[4] = {cuuint64_t(ld), cuuint64_t(rows), 1, 1};
+  cuuint64_t str[3] = {cuuint64_t(ld * 2), cuuint64_t(ld * 2 * rows), cuuint64_t(ld * 2 * rows)};
+  cuuint32_t box[4] = {64, cuuint32_t(box_rows), 1, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(ptr), dims, str, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+}  // namespace
+
+bool attention_fwd_tc5(const AttnArgs& A, cudaStream_t st) {
+  if (A.dtype != BF16 || A.d != 64 || A.seq % 128 || A.seq > 512 || A.nb < 1 || !A.c || !A.lse) return false;
+  const int64_t rows = int64_t(A.nb) * A.seq;
+  const int kbox = A.seq < 256 ? A.seq : 256;
+  CUtensorMap mq, mk, mv;
+  if (!map2(&mq, A.q, A.ld, rows, 128) || !map2(&mk, A.k, A.ld, rows, kbox) || !map2(&mv, A.v, A.ld, rows, kbox))
+    return false;
+  Fa5P p;
+  p.nb = A.nb;
+  p.heads = A.heads;
+  p.seq = A.seq;
+  p.ld = A.ld;
+  p.sl2 = A.alpha * kLog2e;
+  p.p = A.p;
+  p.keep_scale = A.p > 0.f ? 1.f / (1.f - A.p) : 1.f;
+  p.seed = A.seed;
+  p.step = A.step;
+  p.thr = A.thr;
+  p.b0 = A.b0;
+  p.c = A.c;
+  p.lse = A.lse;
+  p.kbox = kbox;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(fa5_fwd, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
+    attr = true;
+  }
+  fa5_fwd<<<dim3(A.seq / 128, A.heads, A.nb), kThreads, kSmem, st>>>(mq, mk, mv, p);
+  return true;
+}
+
+}  // namespace tsk

@@ -493,10 +493,10 @@ def conv2d(mode: int, geom, x, w, dy, out, bias=None, acc: int = 0, stream=None)
 
 
 def attention(mode: int, geom, alpha: float, p: float, q, k, v, c=None, lse=None, dc=None, dq=None, dk=None,
-              dv=None, acc: int = 0, ws=None, stream=None) -> bool:
+              dv=None, acc: int = 0, ws=None, stream=None) -> int:
     """One fused-attention kernel call through the C ABI (`ts_attention`) on torch device
-    tensors (marshalling only).  geom = (nb, heads, seq, d, seed, b0, step).  Returns True
-    when the tensor-core kernels ran."""
+    tensors (marshalling only).  geom = (nb, heads, seq, d, seed, b0, step).  Returns the
+    path: 0 CUDA cores, 1 mma.sync, 2 tcgen05 (forward)."""
     import torch
     dt = DTYPES["bf16"] if q.dtype == torch.bfloat16 else DTYPES["f32"]
     g = (C.c_int32 * 7)(*[int(x) for x in geom])
@@ -508,4 +508,4 @@ def attention(mode: int, geom, alpha: float, p: float, q, k, v, c=None, lse=None
     ws_p = C.c_void_p(ws.data_ptr()) if ws is not None else None
     check(lib().ts_attention(mode, dt, g, fa, ptr(q), ptr(k), ptr(v), ptr(c), lse_p, ptr(dc), ptr(dq), ptr(dk),
                              ptr(dv), acc, ws_p, st, C.byref(used)))
-    return bool(used.value)
+    return used.value

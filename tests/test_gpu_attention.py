@@ -36,10 +36,12 @@ def _inputs(nb, heads, seq, d, seed=0):
     return mk(1.0), mk(1.0), mk(1.0), mk(1.0)
 
 
-@pytest.mark.parametrize("seq", [64, 192, 512])
+@pytest.mark.parametrize("seq", [64, 128, 192, 512])
 @pytest.mark.parametrize("p", [0.0, 0.1])
-@pytest.mark.parametrize("path", ["tc", "simt"])
+@pytest.mark.parametrize("path", ["tc", "mma", "simt"])
 def test_attention_kernels_vs_oracle(seq, p, path):
+    """path tc: the default dispatch (tcgen05 forward where seq % 128 == 0, else mma.sync);
+    mma: the mma.sync forward forced; simt: CUDA cores."""
     nb, heads, d = 2, 3, 64
     alpha, seed, b0, step = 0.125, 77, 5, 3
     q, k, v, dc = _inputs(nb, heads, seq, d)
@@ -51,9 +53,9 @@ def test_attention_kernels_vs_oracle(seq, p, path):
     L = torch.empty((nb, heads, seq), dtype=torch.float32, device="cuda")
     geom = (nb, heads, seq, d, seed, b0, step)
     force = 0x10 if path == "simt" else 0
-    used = tsplit.attention(1 | force, geom, alpha, p, Q, K, V, c=C, lse=L)
+    used = tsplit.attention(1 | force, geom, alpha, p, Q, K, V, c=C, lse=L, acc=0x100 if path == "mma" else 0)
     torch.cuda.synchronize()
-    assert used == (path == "tc")
+    assert used == {"simt": 0, "mma": 1, "tc": 2 if seq % 128 == 0 else 1}[path]
     assert _rel(L.cpu().numpy(), lse_ref) <= 1e-5
     assert _rel(C.float().cpu().numpy(), c_ref) <= 1e-2
     ws = torch.empty(nb * heads * seq, dtype=torch.float32, device="cuda")
