@@ -72,10 +72,11 @@ typedef enum {
   TS_OP_AVGPOOL = 16,  /* global average: in X[N,H,W,C] out [N,C]                       */
   TS_OP_FLATTEN = 17,  /* in X[N,...] out [N, prod(...)] (copy)                          */
   TS_OP_ATTENTION = 18 /* fused attention: in Q[T,h], K[T,h], V[T,h];
-                          out C[T,h] = dropout(softmax(alpha Q_h K_h^T)) V_h (heads merged)
-                          and lse[b,a,s] (f32, auxiliary: read only by its own backward,
-                          never differentiated); iattr {heads, seq, dropout seed},
-                          fattr {alpha, p}; dropout mask = Philox on the [b,a,s,s] index  */
+                          out C[T,h] = dropout(softmax(alpha Q_h K_h^T)) V_h (heads merged),
+                          lse[b,a,s] (f32) and the dropout keep bits [b,a,s,s/32] (i32, key j
+                          at bit j%32) — both auxiliary: read only by its own backward, never
+                          differentiated; iattr {heads, seq (% 32 == 0), dropout seed},
+                          fattr {alpha, p}; keep = Philox on the [b,a,s,s] index (D-RNG)    */
 } ts_op_kind;
 
 typedef struct {
@@ -307,18 +308,20 @@ ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void
 /* Fused attention micro-op kernels (unit tests; the session uses the same ones).
  * Cites: SURVEY.md §8(f) f2; semantics of TS_OP_ATTENTION above.  Q, K, V, C, dC, dQ,
  * dK, dV: device [nb*seq, heads*d] (row stride heads*d); lse: device fp32 [nb, heads, seq];
+ * mask: device keep bits [nb, heads, seq, seq/32] (key j of a row at bit j%32; seq % 32 == 0),
+ * written by the forward (may be NULL there), read by the backward;
  * ws: device fp32 scratch >= nb*heads*seq floats (backward).  geom = {nb, heads, seq, d,
  * dropout seed, b0 (global index of the first sample, for the dropout counters), step};
  * fattr = {alpha, p}.  mode 1: forward (writes C and lse; either may be NULL);
- * mode 2: backward (reads Q, K, V, C, lse, dC; writes dQ, dK, dV, any may be NULL;
+ * mode 2: backward (reads Q, K, V, C, lse, mask, dC; writes dQ, dK, dV, any may be NULL;
  * acc bit 0/1/2 adds into dQ/dK/dV).  mode | 0x10 forces the CUDA-core kernels.
  * dtype TS_BF16 with d = 64 and seq % 64 == 0 runs the tensor-core (mma.sync) kernels.
  * Forward with seq % 128 == 0 and seq <= 512 (and both C and lse requested) runs the
  * tcgen05 kernel (*used_tc = 2) unless acc bit 8 (0x100) asks for the mma.sync one.
  * *used_tc reports the path (0 CUDA cores, 1 mma.sync, 2 tcgen05).  Errors: TS_ERR_ARG, TS_ERR_CUDA. */
 ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const float* fattr, const void* q,
-                       const void* k, const void* v, void* c, float* lse, const void* dc, void* dq, void* dk,
-                       void* dv, int32_t acc, float* ws, void* stream, int32_t* used_tc);
+                       const void* k, const void* v, void* c, float* lse, uint32_t* mask, const void* dc, void* dq,
+                       void* dk, void* dv, int32_t acc, float* ws, void* stream, int32_t* used_tc);
 
 #ifdef __cplusplus
 }

@@ -46,7 +46,7 @@ def forward_op(graph, op, val, row0=0, elem0=0, step=0):
         return ops.attn_qk_fwd(x[0], x[1], ia[0], ia[1], fa[0])
     if k == "attn_pv":
         return ops.attn_pv_fwd(x[0], x[1], ia[0], ia[1])
-    if k == "attention":  # two outputs: (C, lse); dropout offset from the first sample
+    if k == "attention":  # outputs (C, lse, keep-mask words); dropout offset from the first sample
         b0 = row0 // ia[1]
         return ops.attention_fwd(x[0], x[1], x[2], ia[0], ia[1], fa[0], fa[1], ia[2],
                                  b0 * ia[0] * ia[1] * ia[1], step)
@@ -139,7 +139,7 @@ def backward_op(graph, op, val, dy, row0=0, elem0=0, step=0):
 
 # Auxiliary outputs: statistics an op saves for its own backward, never read by another
 # op and never differentiated (the fused attention's row log-sum-exp).
-AUX_OUTPUTS = {"attention": (1,)}
+AUX_OUTPUTS = {"attention": (1, 2)}
 
 
 def grad_outputs(op):

@@ -203,12 +203,23 @@ def attention_fwd(q, k, v, heads, seq, alpha, p, seed, elem0, step=0):
     lse[b,a,i] = log sum_j exp(S_ij) that its backward reads.  The dropout mask is the
     unfused op's: Philox on the element index of the [b,a,s,s] probabilities
     (elem0 = first sample's offset there), so fused and unfused graphs compute the
-    same function."""
+    same function.  Returns (C, lse, mask words)."""
     s = attn_qk_fwd(q, k, heads, seq, alpha)
     m = s.max(axis=-1, keepdims=True)
     lse = (m + np.log(np.exp(s - m).sum(axis=-1, keepdims=True)))[..., 0]
     pd = dropout_fwd(softmax_fwd(s), p, seed, elem0, step)
-    return attn_pv_fwd(pd, v, heads, seq), lse
+    return attn_pv_fwd(pd, v, heads, seq), lse, attention_mask_words(s.shape, p, seed, elem0, step)
+
+
+def attention_mask_words(shape, p, seed, elem0, step=0):
+    """The keep mask of attention_fwd packed 32 keys per int32 word, key 32w + j at bit j
+    ([b,a,s,s/32]); all ones when p = 0.  The fused op stores it for its backward."""
+    keep = np.ones(shape, bool) if p == 0.0 else dropout_keep(shape, elem0, p, seed, step)
+    nw = (shape[-1] + 31) // 32  # keys past the end read as dropped bits 0
+    keep = np.concatenate([keep, np.zeros(shape[:-1] + (nw * 32 - shape[-1],), bool)], axis=-1)
+    bits = keep.reshape(shape[:-1] + (nw, 32)).astype(np.uint64)
+    w = (bits << np.arange(32, dtype=np.uint64)).sum(axis=-1)
+    return w.astype(np.uint32).view(np.int32)
 
 
 def attention_bwd(dc, q, k, v, heads, seq, alpha, p, seed, elem0, step=0):

@@ -51,9 +51,9 @@ SAVED = {
     "maxpool": ("in", 0),
     "avgpool": None,
     "flatten": None,
-    "attention": (("in", 0, 1, 2), ("out", 0, 1)),  # Q, K, V, C, lse (D-SAVED)
+    "attention": (("in", 0, 1, 2), ("out", 0, 1, 2)),  # Q, K, V, C, lse, keep mask (D-SAVED)
 }
-AUX_OUTPUTS = {"attention": (1,)}  # never differentiated (same rule as net.AUX_OUTPUTS)
+AUX_OUTPUTS = {"attention": (1, 2)}  # never differentiated (same rule as net.AUX_OUTPUTS)
 
 # Ops whose statistics span the whole batch ("the merge of
 # micro-tensors can be required by the operation (e.g., batch normalization)"):

@@ -69,6 +69,11 @@ def build(force: bool = False, verbose: bool = False) -> str:
             os.remove(f)
     with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 1)) as ex:
         objs = list(ex.map(lambda s: _compile(s, digest), cpp + cu))
+    # drop objects of older source versions (they would travel to the GPU box with the tree)
+    keep = set(objs)
+    for f in glob.glob(os.path.join(BUILD, "*.o")):
+        if f not in keep:
+            os.remove(f)
     stamp = hashlib.sha1("".join(objs).encode()).hexdigest()
     stamp_file = LIB + ".stamp"
     if os.path.exists(LIB) and os.path.exists(stamp_file) and open(stamp_file).read() == stamp:

@@ -21,8 +21,8 @@ inline uint64_t align_up(uint64_t n) { return (n + kAlign - 1) / kAlign * kAlign
 inline bool batch_reduce(int kind) { return kind == TS_OP_BATCHNORM; }
 inline int dtype_bytes(int d) { return d == TS_BF16 ? 2 : 4; }
 // Auxiliary outputs (statistics an op keeps for its own backward; no gradient): the
-// fused attention's row log-sum-exp.
-inline bool aux_output(int kind, int idx) { return kind == TS_OP_ATTENTION && idx == 1; }
+// fused attention's row log-sum-exp and dropout keep bits.
+inline bool aux_output(int kind, int idx) { return kind == TS_OP_ATTENTION && (idx == 1 || idx == 2); }
 
 void set_error(const std::string& msg);
 

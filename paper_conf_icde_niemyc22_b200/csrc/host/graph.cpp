@@ -87,7 +87,7 @@ bool validate_op(const Graph& g, const Op& o, std::string& why) {
       return true;
     }
     case TS_OP_ATTENTION: {
-      if (!need(3, 2)) return false;
+      if (!need(3, 3)) return false;
       if (o.ia.size() < 3 || o.fa.size() < 2) return (why = "attention attrs {heads, seq, seed} {alpha, p}"), false;
       const int64_t heads = o.ia[0], seq = o.ia[1];
       const Tensor &q = T(o.in[0]), &c = T(o.out[0]), &l = T(o.out[1]);
@@ -99,6 +99,10 @@ bool validate_op(const Graph& g, const Op& o, std::string& why) {
         return (why = "attention lse must be f32 [b,a,s]"), false;
       if ((q.shape[1] / heads) % 8) return (why = "head dim must be a multiple of 8"), false;
       if (o.fa[1] < 0 || o.fa[1] >= 1) return (why = "attention dropout p"), false;
+      const Tensor& mk = T(o.out[2]);
+      if (seq % 32 || mk.ndim != 4 || mk.dtype != TS_I32 || mk.shape[0] != l.shape[0] || mk.shape[1] != heads ||
+          mk.shape[2] != seq || mk.shape[3] != seq / 32)
+        return (why = "attention keep bits must be i32 [b,a,s,s/32] (seq % 32 == 0)"), false;
       return true;
     }
     case TS_OP_EMBED: {
@@ -189,7 +193,7 @@ std::vector<int> saved_of(const Graph& g, const Op& o) {
       break;
     case TS_OP_RELU: case TS_OP_TANH: case TS_OP_SOFTMAX: src = {o.out[0]}; break;
     case TS_OP_ATTN_QK: case TS_OP_ATTN_PV: case TS_OP_EMBED: case TS_OP_XENT: src = {o.in[0], o.in[1]}; break;
-    case TS_OP_ATTENTION: src = {o.in[0], o.in[1], o.in[2], o.out[0], o.out[1]}; break;
+    case TS_OP_ATTENTION: src = {o.in[0], o.in[1], o.in[2], o.out[0], o.out[1], o.out[2]}; break;
     default: break;
   }
   std::vector<int> r;

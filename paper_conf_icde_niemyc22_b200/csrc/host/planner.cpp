@@ -88,8 +88,8 @@ OpCost op_cost(const Graph& g, int oi) {
       const double unit = 2.0 * nbt * heads * seq * seq * d;
       c.flop_f = 2 * unit;
       c.flop_b = 7 * unit;
-      c.bytes_f = 4 * nb(o.in[0]) + nb(o.out[1]);
-      c.bytes_b = 8 * nb(o.in[0]) + 2 * nb(o.out[1]);
+      c.bytes_f = 4 * nb(o.in[0]) + double(g.t[o.out[1]].bytes + g.t[o.out[2]].bytes);
+      c.bytes_b = 8 * nb(o.in[0]) + 2.0 * double(g.t[o.out[1]].bytes + g.t[o.out[2]].bytes);
       c.kern_b = 3;
       break;
     }

@@ -59,6 +59,8 @@ __device__ __forceinline__ float ex2(float x) {
   return y;
 }
 
+__device__ __forceinline__ bool mask_bit(const uint32_t* mrow, int key) { return (mrow[key >> 5] >> (key & 31)) & 1u; }
+
 // ============================================================ CUDA-core version
 template <class T>
 struct AccOf {
@@ -124,6 +126,16 @@ __global__ void attn_fwd_simt(AttnArgs A) {
     }
   }
   if (A.lse && threadIdx.x == 0) A.lse[(int64_t(b) * A.heads + a) * S + i] = float(lse);
+  if (A.mask) {
+    const int nw = (S + 31) / 32;
+    uint32_t* mrow = A.mask + ((int64_t(b) * A.heads + a) * S + i) * nw;
+    for (int w = threadIdx.x; w < nw; w += blockDim.x) {
+      uint32_t bits = 0;
+      for (int j = 0; j < 32 && 32 * w + j < S; ++j)
+        if (A.p <= 0.f || philox_one(e0 + 32 * w + j, A.seed, A.step) >= A.thr) bits |= 1u << j;
+      mrow[w] = bits;
+    }
+  }
 }
 
 // query-major backward: dQ_i and D_i = sum_j P_ij dP_ij (= dO_i . O_i), stored to ws
@@ -142,7 +154,7 @@ __global__ void attn_bwd_q_simt(AttnArgs A) {
   const T* k = static_cast<const T*>(A.k) + int64_t(b) * S * A.ld + a * d;
   const T* v = static_cast<const T*>(A.v) + int64_t(b) * S * A.ld + a * d;
   const Acc lse = A.lse[(int64_t(b) * A.heads + a) * S + i];
-  const uint64_t e0 = ((uint64_t(A.b0 + b) * A.heads + a) * S + i) * uint64_t(S);
+  const uint32_t* mrow = A.mask + ((int64_t(b) * A.heads + a) * S + i) * ((S + 31) / 32);
   const Acc scale = A.p > 0.f ? Acc(1) / (Acc(1) - Acc(A.p)) : Acc(1);
   Acc part = 0;
   for (int j = threadIdx.x; j < S; j += blockDim.x) {
@@ -153,7 +165,7 @@ __global__ void attn_bwd_q_simt(AttnArgs A) {
     }
     const Acc pj = exp(Acc(A.alpha) * sq - lse);
     Acc dpj = dd;
-    if (A.p > 0.f) dpj = philox_one(e0 + j, A.seed, A.step) >= A.thr ? dpj * scale : Acc(0);
+    if (A.p > 0.f) dpj = mask_bit(mrow, j) ? dpj * scale : Acc(0);
     P[j] = pj;
     dP[j] = dpj;
     part += pj * dpj;
@@ -203,10 +215,7 @@ __global__ void attn_bwd_kv_simt(AttnArgs A) {
     }
     const Acc pij = exp(Acc(A.alpha) * sq - Acc(lse[i]));
     bool keep = true;
-    if (A.p > 0.f) {
-      const uint64_t e = ((uint64_t(A.b0 + b) * A.heads + a) * S + i) * uint64_t(S) + j;
-      keep = philox_one(e, A.seed, A.step) >= A.thr;
-    }
+    if (A.p > 0.f) keep = mask_bit(A.mask + ((int64_t(b) * A.heads + a) * S + i) * ((S + 31) / 32), j);
     const Acc dpij = keep ? dd * scale : Acc(0);
     Pd[i] = keep ? pij * scale : Acc(0);
     dS[i] = pij * (dpij - Acc(D[i]));
@@ -370,19 +379,25 @@ __global__ void __launch_bounds__(128) fa_fwd(AttnArgs A) {
       o[n][3] *= corr1;
     }
     uint32_t pa[4][4];  // P as A fragments of the PV product (k = keys)
+    uint32_t mw[2][2] = {{0u, 0u}, {0u, 0u}};  // [word of the 64-key block][row r_lo / r_lo + 8]
 #pragma unroll
     for (int n = 0; n < 8; ++n) {
       float p0 = ex2(s[n][0] * sl2 - m[0]), p1 = ex2(s[n][1] * sl2 - m[0]);
       float p2 = ex2(s[n][2] * sl2 - m[1]), p3 = ex2(s[n][3] * sl2 - m[1]);
       l[0] += p0 + p1;
       l[1] += p2 + p3;
+      bool kp[4] = {true, true, true, true};
       if (A.p > 0.f) {
-        bool kp[4];
         quad_keep(equad + uint64_t(kb * kBN + n * 8), uint64_t(S), A.seed, A.step, A.thr, kp);
         p0 = kp[0] ? p0 : 0.f;
         p1 = kp[1] ? p1 : 0.f;
         p2 = kp[2] ? p2 : 0.f;
         p3 = kp[3] ? p3 : 0.f;
+      }
+      {
+        const int bit = (n & 3) * 8 + 2 * (lane & 3);
+        mw[n >> 2][0] |= (uint32_t(kp[0]) << bit) | (uint32_t(kp[1]) << (bit + 1));
+        mw[n >> 2][1] |= (uint32_t(kp[2]) << bit) | (uint32_t(kp[3]) << (bit + 1));
       }
       const int kk = n >> 1;
       if ((n & 1) == 0) {
@@ -391,6 +406,22 @@ __global__ void __launch_bounds__(128) fa_fwd(AttnArgs A) {
       } else {
         pa[kk][2] = pack_bf16(p0, p1);
         pa[kk][3] = pack_bf16(p2, p3);
+      }
+    }
+    if (A.mask) {  // OR the quad's bits; lane 0 of the quad stores this block's 2 words per row
+#pragma unroll
+      for (int w = 0; w < 2; ++w)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          mw[w][h] |= __shfl_xor_sync(0xffffffffu, mw[w][h], 1);
+          mw[w][h] |= __shfl_xor_sync(0xffffffffu, mw[w][h], 2);
+        }
+      if ((lane & 3) == 0) {
+        uint32_t* m0 = A.mask + ((int64_t(b) * A.heads + a) * S + qb * kBM + r_lo) * (S / 32) + kb * 2;
+        m0[0] = mw[0][0];
+        m0[1] = mw[1][0];
+        m0[8 * (S / 32)] = mw[0][1];
+        m0[8 * (S / 32) + 1] = mw[1][1];
       }
     }
 #pragma unroll
@@ -479,7 +510,8 @@ __global__ void __launch_bounds__(128) fa_bwd_dq(AttnArgs A) {
   }
   const float sl2 = A.alpha * kLog2e;
   const float keep_scale = A.p > 0.f ? 1.f / (1.f - A.p) : 1.f;
-  const uint64_t equad = ((uint64_t(A.b0 + b) * A.heads + a) * S + q0) * uint64_t(S);
+  const uint32_t* mrow0 = A.mask + ((int64_t(b) * A.heads + a) * S + q0) * (S / 32);
+  const uint32_t* mrow1 = mrow0 + 8 * (S / 32);
   uint32_t qa[4][4], ga[4][4];
   float dq[8][4] = {};
   const int nkb = S / kBN;
@@ -525,12 +557,12 @@ __global__ void __launch_bounds__(128) fa_bwd_dq(AttnArgs A) {
       float d0 = dp[n][0] * keep_scale, d1 = dp[n][1] * keep_scale, d2 = dp[n][2] * keep_scale,
             d3 = dp[n][3] * keep_scale;
       if (A.p > 0.f) {
-        bool kp[4];
-        quad_keep(equad + uint64_t(kb * kBN + n * 8), uint64_t(S), A.seed, A.step, A.thr, kp);
-        d0 = kp[0] ? d0 : 0.f;
-        d1 = kp[1] ? d1 : 0.f;
-        d2 = kp[2] ? d2 : 0.f;
-        d3 = kp[3] ? d3 : 0.f;
+        const int key = kb * kBN + n * 8 + 2 * (lane & 3);
+        const uint32_t w0 = mrow0[key >> 5] >> (key & 31), w1 = mrow1[key >> 5] >> (key & 31);
+        d0 = (w0 & 1u) ? d0 : 0.f;
+        d1 = (w0 & 2u) ? d1 : 0.f;
+        d2 = (w1 & 1u) ? d2 : 0.f;
+        d3 = (w1 & 2u) ? d3 : 0.f;
       }
       const float s0 = v4[0] * (d0 - Dr[0]), s1 = v4[1] * (d1 - Dr[0]);
       const float s2 = v4[2] * (d2 - Dr[1]), s3 = v4[3] * (d3 - Dr[1]);
@@ -619,7 +651,6 @@ __global__ void __launch_bounds__(128) fa_bwd_dkv(AttnArgs A) {
   const float sl2 = A.alpha * kLog2e;
   const float keep_scale = A.p > 0.f ? 1.f / (1.f - A.p) : 1.f;
   const int key_w = warp * 16;  // this warp's keys within the block
-  const uint64_t ehead = (uint64_t(A.b0 + b) * A.heads + a) * uint64_t(S);
   float dk[8][4] = {}, dv[8][4] = {};
   uint8_t* stP = sP[warp];
   uint8_t* stS = sS[warp];
@@ -663,10 +694,16 @@ __global__ void __launch_bounds__(128) fa_bwd_dkv(AttnArgs A) {
 #pragma unroll
       for (int nt = 0; nt < 2; ++nt) {
         bool kp[4] = {true, true, true, true};
-        if (A.p > 0.f)
-          quad_keep((ehead + qb * kBM + mt * 16 + (lane >> 2)) * uint64_t(S) + uint64_t(kb * kBN + key_w + nt * 8),
-                    uint64_t(S), A.seed, A.step, A.thr, kp);
         const int kl = nt * 8 + 2 * (lane & 3);  // key within the warp's 16
+        if (A.p > 0.f) {
+          const int key = kb * kBN + key_w + kl;
+          const uint32_t* m0 = A.mask + ((int64_t(b) * A.heads + a) * S + qb * kBM + mt * 16 + (lane >> 2)) * (S / 32);
+          const uint32_t w0 = m0[key >> 5] >> (key & 31), w1 = m0[8 * (S / 32) + (key >> 5)] >> (key & 31);
+          kp[0] = w0 & 1u;
+          kp[1] = w0 & 2u;
+          kp[2] = w1 & 1u;
+          kp[3] = w1 & 2u;
+        }
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           const int ql = mt * 16 + (lane >> 2) + 8 * h;  // query within the block

@@ -61,6 +61,7 @@ struct Fa5P {
   int64_t b0;
   void* c;
   float* lse;
+  uint32_t* mask;
   int kbox;           // rows per K/V TMA box
 };
 
@@ -156,6 +157,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     named_sync(1, 32 * kSoftWarps);
     m = fmaxf(red_m[i], red_m[128 + i]) * p.sl2;
     const uint64_t erow = ((uint64_t(p.b0 + b) * p.heads + a) * uint64_t(S) + uint64_t(qt * 128 + i)) * uint64_t(S);
+    const int64_t mrow = ((int64_t(b) * p.heads + a) * S + qt * 128 + i) * (S / 32);
     float l = 0.f;
     const uint32_t sp = smem_u32(g == 0 ? rK : rPB);
     for (int c = c0; c < c0 + half; c += 32) {
@@ -167,17 +169,22 @@ __global__ void __launch_bounds__(kThreads, 1)
         v[j] = ex2(__uint_as_float(r[j]) * p.sl2 - m);
         l += v[j];
       }
+      uint32_t bits = 0xFFFFFFFFu;
       if (p.p > 0.f) {
+        bits = 0u;
 #pragma unroll
         for (int u = 0; u < 8; ++u) {
           const uint64_t cnt = (erow + uint64_t(c + 4 * u)) >> 2;
           const uint4 w = philox4x32_10(uint32_t(cnt), uint32_t(cnt >> 32), p.step, 0u, p.seed, kPhiloxKey1);
-          if (w.x < p.thr) v[4 * u] = 0.f;
-          if (w.y < p.thr) v[4 * u + 1] = 0.f;
-          if (w.z < p.thr) v[4 * u + 2] = 0.f;
-          if (w.w < p.thr) v[4 * u + 3] = 0.f;
+          bits |= (uint32_t(w.x >= p.thr) | (uint32_t(w.y >= p.thr) << 1) | (uint32_t(w.z >= p.thr) << 2) |
+                   (uint32_t(w.w >= p.thr) << 3))
+                  << (4 * u);
         }
+#pragma unroll
+        for (int j = 0; j < 32; ++j)
+          if (!((bits >> j) & 1u)) v[j] = 0.f;
       }
+      if (p.mask) p.mask[mrow + (c >> 5)] = bits;
       // 32 keys = 4 sixteen-byte chunks of row i in the K-major SW128 layout
       const int kl = c - c0;  // key within this half
       const uint32_t blk = sp + uint32_t(kl >> 6) * 16384u + uint32_t(i) * 128u;
@@ -278,6 +285,7 @@ bool attention_fwd_tc5(const AttnArgs& A, cudaStream_t st) {
   p.b0 = A.b0;
   p.c = A.c;
   p.lse = A.lse;
+  p.mask = A.mask;
   p.kbox = kbox;
   static bool attr = false;
   if (!attr) {

@@ -106,6 +106,7 @@ struct AttnArgs {
   const void *q = nullptr, *k = nullptr, *v = nullptr;
   void* c = nullptr;       // forward output (may be null: a replay regenerating only lse)
   float* lse = nullptr;    // forward output (may be null) / backward input
+  uint32_t* mask = nullptr;  // dropout keep bits [nb, heads, seq, seq/32]: forward output (may be null) / backward input
   const void* dc = nullptr;
   void *dq = nullptr, *dk = nullptr, *dv = nullptr;
   int acc_q = 0, acc_k = 0, acc_v = 0;

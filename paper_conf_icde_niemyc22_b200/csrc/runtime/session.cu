@@ -488,6 +488,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
         // a replay writes only the output it regenerates
         a.c = m.writes.count(o.out[0]) ? V(o.out[0]) : nullptr;
         a.lse = m.writes.count(o.out[1]) ? reinterpret_cast<float*>(V(o.out[1])) : nullptr;
+        a.mask = m.writes.count(o.out[2]) ? reinterpret_cast<uint32_t*>(V(o.out[2])) : nullptr;
         nk = 1;
         return [a, stepp](cudaStream_t st) {
           tsk::AttnArgs b = a;
@@ -497,6 +498,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       }
       a.c = V(o.out[0]);
       a.lse = reinterpret_cast<float*>(V(o.out[1]));
+      a.mask = reinterpret_cast<uint32_t*>(V(o.out[2]));
       a.dc = G(o.out[0]);
       auto gslot = [&](int i, void*& ptr, int& acc) {
         const Tensor& x = g.t[o.in[i]];
@@ -1274,8 +1276,8 @@ ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void
 }
 
 ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const float* fattr, const void* q,
-                       const void* k, const void* v, void* c, float* lse, const void* dc, void* dq, void* dk,
-                       void* dv, int32_t acc, float* ws, void* stream, int32_t* used_tc) {
+                       const void* k, const void* v, void* c, float* lse, uint32_t* mask, const void* dc, void* dq,
+                       void* dk, void* dv, int32_t acc, float* ws, void* stream, int32_t* used_tc) {
   const bool simt_only = (mode & 0x10) != 0;
   mode &= 0xF;
   if (!geom || !fattr || (mode != 1 && mode != 2) || (dtype != TS_BF16 && dtype != TS_F32) || !q || !k || !v)
@@ -1288,10 +1290,12 @@ ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const f
   if (a.nb < 1 || a.heads < 1 || a.seq < 1 || a.d < 1 || a.d > 1024 || a.p < 0.f || a.p >= 1.f)
     return set_error("ts_attention: bad geometry"), TS_ERR_ARG;
   a.ld = int64_t(a.heads) * a.d;
-  a.q = q; a.k = k; a.v = v; a.c = c; a.lse = lse; a.dc = dc; a.dq = dq; a.dk = dk; a.dv = dv;
+  a.q = q; a.k = k; a.v = v; a.c = c; a.lse = lse; a.mask = mask; a.dc = dc; a.dq = dq; a.dk = dk; a.dv = dv;
+  if (a.seq % 32) return set_error("ts_attention: seq must be a multiple of 32"), TS_ERR_ARG;
   a.acc_q = acc & 1; a.acc_k = (acc >> 1) & 1; a.acc_v = (acc >> 2) & 1;
   a.ws = ws;
-  if (mode == 2 && (!c || !lse || !dc || !ws)) return set_error("ts_attention: backward needs C, lse, dC, ws"), TS_ERR_ARG;
+  if (mode == 2 && (!c || !lse || !mask || !dc || !ws))
+    return set_error("ts_attention: backward needs C, lse, mask, dC, ws"), TS_ERR_ARG;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const bool mma_only = (acc & 0x100) != 0;  // tests: skip the tcgen05 forward, keep mma.sync
   a.acc_q = acc & 1; a.acc_k = (acc >> 1) & 1; a.acc_v = (acc >> 2) & 1;

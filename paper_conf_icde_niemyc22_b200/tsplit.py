@@ -131,8 +131,8 @@ def lib():
             "ts_gemm_f32": (i32, [i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, C.c_float,
                                   vp, vp]),
             "ts_conv2d": (i32, [i32, i32, P(i32), vp, vp, vp, vp, vp, i32, vp, P(i32)]),
-            "ts_attention": (i32, [i32, i32, P(i32), P(C.c_float), vp, vp, vp, vp, vp, vp, vp, vp, vp, i32, vp, vp,
-                                   P(i32)]),
+            "ts_attention": (i32, [i32, i32, P(i32), P(C.c_float), vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, i32, vp,
+                                   vp, P(i32)]),
         }
         for name, (res, args) in list(sig.items()) + list(optional.items()):
             if not hasattr(L, name):
@@ -493,7 +493,7 @@ def conv2d(mode: int, geom, x, w, dy, out, bias=None, acc: int = 0, stream=None)
 
 
 def attention(mode: int, geom, alpha: float, p: float, q, k, v, c=None, lse=None, dc=None, dq=None, dk=None,
-              dv=None, acc: int = 0, ws=None, stream=None) -> int:
+              dv=None, acc: int = 0, ws=None, stream=None, mask=None) -> int:
     """One fused-attention kernel call through the C ABI (`ts_attention`) on torch device
     tensors (marshalling only).  geom = (nb, heads, seq, d, seed, b0, step).  Returns the
     path: 0 CUDA cores, 1 mma.sync, 2 tcgen05 (forward)."""
@@ -506,6 +506,6 @@ def attention(mode: int, geom, alpha: float, p: float, q, k, v, c=None, lse=None
     st = C.c_void_p(stream if stream is not None else torch.cuda.current_stream().cuda_stream)
     lse_p = C.cast(C.c_void_p(lse.data_ptr()), C.POINTER(C.c_float)) if lse is not None else None
     ws_p = C.c_void_p(ws.data_ptr()) if ws is not None else None
-    check(lib().ts_attention(mode, dt, g, fa, ptr(q), ptr(k), ptr(v), ptr(c), lse_p, ptr(dc), ptr(dq), ptr(dk),
-                             ptr(dv), acc, ws_p, st, C.byref(used)))
+    check(lib().ts_attention(mode, dt, g, fa, ptr(q), ptr(k), ptr(v), ptr(c), lse_p, ptr(mask), ptr(dc), ptr(dq),
+                             ptr(dk), ptr(dv), acc, ws_p, st, C.byref(used)))
     return used.value

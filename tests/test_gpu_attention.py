@@ -45,27 +45,30 @@ def test_attention_kernels_vs_oracle(seq, p, path):
     nb, heads, d = 2, 3, 64
     alpha, seed, b0, step = 0.125, 77, 5, 3
     q, k, v, dc = _inputs(nb, heads, seq, d)
-    c_ref, lse_ref = O.attention_fwd(q, k, v, heads, seq, alpha, p, seed, b0 * heads * seq * seq, step)
+    c_ref, lse_ref, mask_ref = O.attention_fwd(q, k, v, heads, seq, alpha, p, seed, b0 * heads * seq * seq, step)
     dq_ref, dk_ref, dv_ref = O.attention_bwd(dc, q, k, v, heads, seq, alpha, p, seed, b0 * heads * seq * seq, step)
     dev = lambda a: torch.from_numpy(a).to("cuda").to(torch.bfloat16)  # noqa: E731
     Q, K, V, DC = dev(q), dev(k), dev(v), dev(dc)
     C = torch.empty_like(Q)
     L = torch.empty((nb, heads, seq), dtype=torch.float32, device="cuda")
+    M = torch.empty((nb, heads, seq, seq // 32), dtype=torch.int32, device="cuda")
     geom = (nb, heads, seq, d, seed, b0, step)
     force = 0x10 if path == "simt" else 0
-    used = tsplit.attention(1 | force, geom, alpha, p, Q, K, V, c=C, lse=L, acc=0x100 if path == "mma" else 0)
+    used = tsplit.attention(1 | force, geom, alpha, p, Q, K, V, c=C, lse=L, mask=M, acc=0x100 if path == "mma" else 0)
     torch.cuda.synchronize()
     assert used == {"simt": 0, "mma": 1, "tc": 2 if seq % 128 == 0 else 1}[path]
+    assert np.array_equal(M.cpu().numpy(), mask_ref)  # keep bits: integer decisions, bit-exact
     assert _rel(L.cpu().numpy(), lse_ref) <= 1e-5
     assert _rel(C.float().cpu().numpy(), c_ref) <= 1e-2
     ws = torch.empty(nb * heads * seq, dtype=torch.float32, device="cuda")
     dQ, dK, dV = (torch.full_like(Q, 0.25) for _ in range(3))
-    tsplit.attention(2 | force, geom, alpha, p, Q, K, V, c=C, lse=L, dc=DC, dq=dQ, dk=dK, dv=dV, ws=ws)
+    tsplit.attention(2 | force, geom, alpha, p, Q, K, V, c=C, lse=L, mask=M, dc=DC, dq=dQ, dk=dK, dv=dV, ws=ws)
     torch.cuda.synchronize()
     for got, ref in ((dQ, dq_ref), (dK, dk_ref), (dV, dv_ref)):
         assert _rel(got.float().cpu().numpy(), ref) <= 2e-2
     # accumulate flags (a later backward op adding its share)
-    tsplit.attention(2 | force, geom, alpha, p, Q, K, V, c=C, lse=L, dc=DC, dq=dQ, dk=dK, dv=dV, acc=7, ws=ws)
+    tsplit.attention(2 | force, geom, alpha, p, Q, K, V, c=C, lse=L, mask=M, dc=DC, dq=dQ, dk=dK, dv=dV, acc=7,
+                     ws=ws)
     torch.cuda.synchronize()
     for got, ref in ((dQ, dq_ref), (dK, dk_ref), (dV, dv_ref)):
         assert _rel(got.float().cpu().numpy(), 2 * ref) <= 2e-2
@@ -79,20 +82,21 @@ def test_attention_split_equals_whole():
     Q, K, V, DC = dev(q), dev(k), dev(v), dev(dc)
     C, C2 = torch.empty_like(Q), torch.empty_like(Q)
     L, L2 = (torch.empty((nb, heads, seq), dtype=torch.float32, device="cuda") for _ in range(2))
+    M, M2 = (torch.empty((nb, heads, seq, seq // 32), dtype=torch.int32, device="cuda") for _ in range(2))
     ws = torch.empty(nb * heads * seq, dtype=torch.float32, device="cuda")
     G = [torch.empty_like(Q) for _ in range(6)]
-    tsplit.attention(1, (nb, heads, seq, d, 9, 0, 1), 0.125, 0.1, Q, K, V, c=C, lse=L)
-    tsplit.attention(2, (nb, heads, seq, d, 9, 0, 1), 0.125, 0.1, Q, K, V, c=C, lse=L, dc=DC, dq=G[0], dk=G[1],
-                     dv=G[2], ws=ws)
+    tsplit.attention(1, (nb, heads, seq, d, 9, 0, 1), 0.125, 0.1, Q, K, V, c=C, lse=L, mask=M)
+    tsplit.attention(2, (nb, heads, seq, d, 9, 0, 1), 0.125, 0.1, Q, K, V, c=C, lse=L, mask=M, dc=DC, dq=G[0],
+                     dk=G[1], dv=G[2], ws=ws)
     rows = seq * 2
     for s0 in (0, 2):
         sl = slice(s0 * seq, s0 * seq + rows)
         g2 = (2, heads, seq, d, 9, s0, 1)
-        tsplit.attention(1, g2, 0.125, 0.1, Q[sl], K[sl], V[sl], c=C2[sl], lse=L2[s0:s0 + 2])
-        tsplit.attention(2, g2, 0.125, 0.1, Q[sl], K[sl], V[sl], c=C2[sl], lse=L2[s0:s0 + 2], dc=DC[sl],
-                         dq=G[3][sl], dk=G[4][sl], dv=G[5][sl], ws=ws)
+        tsplit.attention(1, g2, 0.125, 0.1, Q[sl], K[sl], V[sl], c=C2[sl], lse=L2[s0:s0 + 2], mask=M2[s0:s0 + 2])
+        tsplit.attention(2, g2, 0.125, 0.1, Q[sl], K[sl], V[sl], c=C2[sl], lse=L2[s0:s0 + 2], mask=M2[s0:s0 + 2],
+                         dc=DC[sl], dq=G[3][sl], dk=G[4][sl], dv=G[5][sl], ws=ws)
     torch.cuda.synchronize()
-    assert torch.equal(C, C2) and torch.equal(L, L2)
+    assert torch.equal(C, C2) and torch.equal(L, L2) and torch.equal(M, M2)
     for i in range(3):
         assert torch.equal(G[i], G[3 + i])
 

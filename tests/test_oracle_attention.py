@@ -47,8 +47,11 @@ def test_attention_loops_and_lse():
     nb, seq, heads, d = 2, 4, 3, 2
     q, k, v = _qkv(nb, seq, heads, d)
     alpha, p, seed, elem0 = 0.5, 0.25, 3, 96
-    c, lse = O.attention_fwd(q, k, v, heads, seq, alpha, p, seed, elem0)
+    c, lse, mw = O.attention_fwd(q, k, v, heads, seq, alpha, p, seed, elem0)
     keep = O.dropout_keep((nb, heads, seq, seq), elem0, p, seed)
+    # the stored keep bits: key j of a row at bit j % 32 of word j // 32
+    bits = (mw.view(np.uint32)[..., :, None] >> np.arange(32, dtype=np.uint32)) & 1
+    assert np.array_equal(bits.reshape(nb, heads, seq, -1)[..., :seq].astype(bool), keep)
     for b in range(nb):
         for a in range(heads):
             cols = slice(a * d, (a + 1) * d)
@@ -73,6 +76,11 @@ def test_fused_graph_equals_unfused(dtype):
     assert max(rel_errs(pf, pu).values()) <= 1e-12
     lse_ids = [t["id"] for t in gf["tensors"] if t["name"].endswith(".lse")]
     assert lse_ids and all(vals[t].dtype == np.float64 for t in lse_ids)
+    mask_ids = [t["id"] for t in gf["tensors"] if t["name"].endswith(".dmask")]
+    # keep fraction of the attention dropout (p = 0.1) over all layers' bits
+    ones = sum(int(np.unpackbits(vals[t].view(np.uint8)).sum()) for t in mask_ids)
+    total = sum(vals[t].size * 32 for t in mask_ids)
+    assert abs(ones / total - 0.9) < 0.01
 
 
 @pytest.mark.parametrize("seed", range(4))

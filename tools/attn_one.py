@@ -15,12 +15,13 @@ Q = torch.randn(nb * seq, heads * d, device="cuda", dtype=torch.bfloat16)
 K, V, DC = torch.randn_like(Q), torch.randn_like(Q), torch.randn_like(Q)
 C = torch.empty_like(Q)
 L = torch.empty(nb, heads, seq, device="cuda")
+M = torch.empty(nb, heads, seq, seq // 32, device="cuda", dtype=torch.int32)
 ws = torch.empty(nb * heads * seq, device="cuda")
 dq, dk, dv = torch.empty_like(Q), torch.empty_like(Q), torch.empty_like(Q)
 g = (nb, heads, seq, d, 1, 0, 0)
 for _ in range(3):
-    used = tsplit.attention(1, g, 0.125, p, Q, K, V, c=C, lse=L)
+    used = tsplit.attention(1, g, 0.125, p, Q, K, V, c=C, lse=L, mask=M)
     if mode == 2:
-        tsplit.attention(2, g, 0.125, p, Q, K, V, c=C, lse=L, dc=DC, dq=dq, dk=dk, dv=dv, ws=ws)
+        tsplit.attention(2, g, 0.125, p, Q, K, V, c=C, lse=L, mask=M, dc=DC, dq=dq, dk=dk, dv=dv, ws=ws)
 torch.cuda.synchronize()
 print("ok path", used, float(C.float().abs().mean()))

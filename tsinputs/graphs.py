@@ -124,8 +124,9 @@ def bert(layers=24, hidden=1024, heads=16, seq=512, batch=32, vocab=30522, ffn=N
     LN1, FFN2, res2, LN2), weights 2 x [h,4h] and 4 x [h,h].
 
     fused_attention=True replaces scores/probs/attn_drop/ctx by
-    one "attention" op: in (Q, K, V), out (ctx [T,h], lse [b,a,s] f32); iattrs
-    {heads, seq, dropout seed}, fattrs {alpha, p}; the same function (same seeds).
+    one "attention" op: in (Q, K, V), out (ctx [T,h], lse [b,a,s] f32, dropout keep
+    bits [b,a,s,s/32] i32); iattrs {heads, seq, dropout seed}, fattrs {alpha, p}; the
+    same function (same seeds).
     """
     ffn = ffn or 4 * hidden
     assert hidden % heads == 0
@@ -157,9 +158,10 @@ def bert(layers=24, hidden=1024, heads=16, seq=512, batch=32, vocab=30522, ffn=N
         k = lin("k", x, hidden, hidden)
         v = lin("v", x, hidden, hidden)
         if fused_attention:
-            c, _ = g.op_multi("attention", p + "attn", [q, k, v],
-                              [(p + "ctx", (T, hidden), None), (p + "lse", (batch, heads, seq), "f32")],
-                              iattrs=[heads, seq, seed + 1 + l], fattrs=[alpha, attn_dropout])
+            c, _, _ = g.op_multi("attention", p + "attn", [q, k, v],
+                                 [(p + "ctx", (T, hidden), None), (p + "lse", (batch, heads, seq), "f32"),
+                                  (p + "dmask", (batch, heads, seq, seq // 32), "i32")],
+                                 iattrs=[heads, seq, seed + 1 + l], fattrs=[alpha, attn_dropout])
         else:
             s = g.op("attn_qk", p + "scores", [q, k], (batch, heads, seq, seq), iattrs=[heads, seq],
                      fattrs=[alpha])
