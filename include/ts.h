@@ -316,8 +316,8 @@ ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void
  * mode 2: backward (reads Q, K, V, C, lse, mask, dC; writes dQ, dK, dV, any may be NULL;
  * acc bit 0/1/2 adds into dQ/dK/dV).  mode | 0x10 forces the CUDA-core kernels.
  * dtype TS_BF16 with d = 64 and seq % 64 == 0 runs the tensor-core (mma.sync) kernels.
- * Forward with seq % 128 == 0 and seq <= 512 (and both C and lse requested) runs the
- * tcgen05 kernel (*used_tc = 2) unless acc bit 8 (0x100) asks for the mma.sync one.
+ * With seq % 128 == 0 and seq <= 512 the tcgen05 kernels run (*used_tc = 2) unless acc
+ * bit 8 (0x100) asks for the mma.sync ones.
  * *used_tc reports the path (0 CUDA cores, 1 mma.sync, 2 tcgen05).  Errors: TS_ERR_ARG, TS_ERR_CUDA. */
 ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const float* fattr, const void* q,
                        const void* k, const void* v, void* c, float* lse, uint32_t* mask, const void* dc, void* dq,

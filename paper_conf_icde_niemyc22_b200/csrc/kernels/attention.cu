@@ -803,7 +803,7 @@ void attention_fwd(const AttnArgs& in, cudaStream_t st) {
   AttnArgs A = in;
   fill_thr(A);
   dim3 grid(A.seq, A.heads, A.nb);
-  if (attention_fwd_tc5(A, st)) return;  // tcgen05 (attention_tc.cu)
+  if (!A.no_tc5 && attention_fwd_tc5(A, st)) return;  // tcgen05 (attention_tc.cu)
   if (tc_eligible(A)) {
     fa_fwd<<<dim3(A.seq / kBM, A.heads, A.nb), 128, 0, st>>>(A);
   } else if (A.dtype == BF16) {
@@ -817,6 +817,7 @@ void attention_bwd(const AttnArgs& in, cudaStream_t st) {
   AttnArgs A = in;
   fill_thr(A);
   dim3 grid(A.seq, A.heads, A.nb);
+  if (!A.no_tc5 && attention_bwd_tc5(A, st)) return;  // tcgen05 (attention_tc.cu)
   if (tc_eligible(A)) {
     fa_bwd_dq<<<dim3(A.seq / kBM, A.heads, A.nb), 128, 0, st>>>(A);
     static bool attr = false;

@@ -235,6 +235,364 @@ __global__ void __launch_bounds__(kThreads, 1)
   }
 }
 
+// ======================================================================= backward
+// Shared by both backward kernels: 128 row threads (TMEM lane i = thread i), one control
+// thread (TMA + tcgen05.mma).  P is rebuilt from S and the saved log-sum-exp, the keep
+// bits come from the forward's mask (no Philox), D_q = dO_q . O_q.
+struct Fa5B {
+  int heads, seq;
+  int64_t ld;
+  float sl2, alpha, keep_scale;
+  int drop;
+  const float* lse;
+  const uint32_t* mask;
+  float* D;             // [nb, heads, seq] row terms (dq5 writes, dkv5 reads)
+  const bf16* o;        // forward output (dq5: D)
+  const bf16* dout;
+  void *dq, *dk, *dv;
+  int acc_q, acc_k, acc_v;
+};
+
+constexpr int kBwdThreads = 32 * 5;
+constexpr uint32_t kIdN128 = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(128 >> 3) << 17) | (uint32_t(128 >> 4) << 24);
+constexpr uint32_t kIdN64MN = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | (uint32_t(64 >> 3) << 17) |
+                              (uint32_t(128 >> 4) << 24);
+
+__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+// 16 values of row i at keys [kl, kl+16) (two 16-byte chunks) of a K-major SW128 operand
+__device__ __forceinline__ void st_row16(uint32_t base, int i, int kl, const float* v) {
+  const uint32_t blk = base + uint32_t(kl >> 6) * 16384u + uint32_t(i) * 128u;
+#pragma unroll
+  for (int q2 = 0; q2 < 2; ++q2) {
+    const int chunk = ((kl & 63) >> 3) + q2;
+    sts128(blk + (uint32_t(chunk ^ (i & 7)) << 4), pk2(v[8 * q2], v[8 * q2 + 1]), pk2(v[8 * q2 + 2], v[8 * q2 + 3]),
+           pk2(v[8 * q2 + 4], v[8 * q2 + 5]), pk2(v[8 * q2 + 6], v[8 * q2 + 7]));
+  }
+}
+// store 32 bf16 values of row i at keys [kl, kl+32) of a K-major SW128 operand (64-key blocks of 16 KB)
+__device__ __forceinline__ void st_row32(uint32_t base, int i, int kl, const float* v) {
+  const uint32_t blk = base + uint32_t(kl >> 6) * 16384u + uint32_t(i) * 128u;
+#pragma unroll
+  for (int q4 = 0; q4 < 4; ++q4) {
+    const int chunk = ((kl & 63) >> 3) + q4;
+    sts128(blk + (uint32_t(chunk ^ (i & 7)) << 4), pk2(v[8 * q4], v[8 * q4 + 1]), pk2(v[8 * q4 + 2], v[8 * q4 + 3]),
+           pk2(v[8 * q4 + 4], v[8 * q4 + 5]), pk2(v[8 * q4 + 6], v[8 * q4 + 7]));
+  }
+}
+__device__ __forceinline__ void store_row64(bf16* dst, const uint32_t (&r0)[32], const uint32_t (&r1)[32], float sc,
+                                            int acc) {
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    const uint32_t* r = h ? r1 : r0;
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      float f[8];
+#pragma unroll
+      for (int e = 0; e < 8; ++e) f[e] = __uint_as_float(r[8 * j + e]) * sc;
+      uint4* pp = reinterpret_cast<uint4*>(dst + h * 32 + 8 * j);
+      if (acc) {
+        const uint4 old = *pp;
+        const __nv_bfloat162* o2 = reinterpret_cast<const __nv_bfloat162*>(&old);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 x = __bfloat1622float2(o2[e]);
+          f[2 * e] += x.x;
+          f[2 * e + 1] += x.y;
+        }
+      }
+      *pp = make_uint4(pk2(f[0], f[1]), pk2(f[2], f[3]), pk2(f[4], f[5]), pk2(f[6], f[7]));
+    }
+  }
+}
+
+// dQ for 128 queries of one (sample, head); all of K and V in shared memory.
+// smem: Q 16K | dO 16K | K seq*128 | V seq*128 | dS 32K | barriers
+__global__ void __launch_bounds__(kBwdThreads, 1)
+    fa5_bwd_dq(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mdO,
+               const __grid_constant__ CUtensorMap mK, const __grid_constant__ CUtensorMap mV, const Fa5B p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int S = p.seq, nkt = S / 128;
+  uint8_t* sQ = smem;
+  uint8_t* sdO = smem + 16384;
+  uint8_t* sK = smem + 32768;
+  uint8_t* sV = sK + S * 128;
+  uint8_t* sdS = sV + S * 128;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sdS + 32768);
+  uint64_t *ld_full = bar, *s_full = bar + 1, *ds_full = bar + 2, *dq_done = bar + 3;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 4);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int qt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
+  if (threadIdx.x == 0) {
+    mbar_init(ld_full, 1);
+    mbar_init(s_full, 1);
+    mbar_init(ds_full, 128);
+    mbar_init(dq_done, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 4) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(512));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;  // S: 0..127, dP: 128..255, dQ: 256..319
+  if (warp == 4) {
+    if (lane == 0) {
+      const int row0 = b * S;
+      mbar_arrive_tx(ld_full, 32768u + uint32_t(S) * 256u);
+      tma_load(sQ, &mQ, ld_full, a * 64, row0 + qt * 128, 0, 0);
+      tma_load(sdO, &mdO, ld_full, a * 64, row0 + qt * 128, 0, 0);
+      for (int j = 0; j < S; j += 128) {
+        tma_load(sK + j * 128, &mK, ld_full, a * 64, row0 + j, 0, 0);
+        tma_load(sV + j * 128, &mV, ld_full, a * 64, row0 + j, 0, 0);
+      }
+      mbar_wait(ld_full, 0);
+      tc_fence_after();
+      const uint32_t q = smem_u32(sQ), g = smem_u32(sdO), k = smem_u32(sK), v = smem_u32(sV), ds = smem_u32(sdS);
+      auto issue_s = [&](int kt) {
+#pragma unroll
+        for (int kk = 0; kk < 4; ++kk) {
+          tc_mma(tmem, smem_desc(q + kk * 32, 16, 1024), smem_desc(k + kt * 16384 + kk * 32, 16, 1024), kIdN128,
+                 kk > 0 ? 1u : 0u);
+          tc_mma(tmem + 128, smem_desc(g + kk * 32, 16, 1024), smem_desc(v + kt * 16384 + kk * 32, 16, 1024),
+                 kIdN128, kk > 0 ? 1u : 0u);
+        }
+        tc_commit(s_full);
+      };
+      issue_s(0);
+      for (int kt = 0; kt < nkt; ++kt) {
+        mbar_wait(ds_full, kt & 1);
+        tc_fence_after();
+        // dQ += dS K_kt: A = dS (K-major, 2 blocks of 64 keys), B = K rows of this tile (MN-major)
+        for (int kk = 0; kk < 128; kk += 16)
+          tc_mma(tmem + 256, smem_desc(ds + (kk >> 6) * 16384 + ((kk & 63) >> 4) * 32, 16, 1024),
+                 smem_desc(k + uint32_t(kt * 128 + kk) * 128, 8192, 1024), kIdN64MN, (kt > 0 || kk > 0) ? 1u : 0u);
+        tc_commit(dq_done);
+        if (kt + 1 < nkt) issue_s(kt + 1);
+      }
+    }
+  } else {
+    const int i = warp * 32 + lane;
+    const int q = qt * 128 + i;
+    const int64_t hrow = (int64_t(b) * p.heads + a) * S + q;
+    const uint32_t trow = tmem + (uint32_t(warp * 32) << 16);
+    // D_q = dO_q . O_q (fp32 over the bf16 row)
+    float D = 0.f;
+    {
+      const bf16* orow = p.o + (int64_t(b) * S + q) * p.ld + a * 64;
+      const bf16* grow = p.dout + (int64_t(b) * S + q) * p.ld + a * 64;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const uint4 x = *reinterpret_cast<const uint4*>(orow + 8 * j);
+        const uint4 y = *reinterpret_cast<const uint4*>(grow + 8 * j);
+        const __nv_bfloat162* x2 = reinterpret_cast<const __nv_bfloat162*>(&x);
+        const __nv_bfloat162* y2 = reinterpret_cast<const __nv_bfloat162*>(&y);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 u = __bfloat1622float2(x2[e]), w = __bfloat1622float2(y2[e]);
+          D += u.x * w.x + u.y * w.y;
+        }
+      }
+      p.D[hrow] = D;
+    }
+    const float l2 = p.lse[hrow] * kLog2e;
+    const uint32_t* mrow = p.mask + hrow * (S / 32);
+    const uint32_t ds = smem_u32(sdS);
+    for (int kt = 0; kt < nkt; ++kt) {
+      mbar_wait(s_full, kt & 1);
+      if (kt > 0) mbar_wait(dq_done, (kt - 1) & 1);  // dS buffer free
+      tc_fence_after();
+#pragma unroll 1
+      for (int c = 0; c < 128; c += 32) {
+        uint32_t rs[32], rp[32];
+        tmem_ld32(trow + uint32_t(c), rs);
+        tmem_ld32(trow + uint32_t(128 + c), rp);
+        const uint32_t bits = p.drop ? mrow[(kt * 128 + c) >> 5] : 0xFFFFFFFFu;
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
+          const float dp = ((bits >> j) & 1u) ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
+          rs[j] = __float_as_uint(pr * (dp - D));
+        }
+        st_row32(ds, i, c, reinterpret_cast<const float*>(rs));
+      }
+      fence_async_smem();
+      tc_fence_before();
+      mbar_arrive(ds_full);
+    }
+    mbar_wait(dq_done, (nkt - 1) & 1);
+    tc_fence_after();
+    uint32_t r0[32], r1[32];
+    tmem_ld32(trow + 256u, r0);
+    tmem_ld32(trow + 288u, r1);
+    if (p.dq) store_row64(static_cast<bf16*>(p.dq) + (int64_t(b) * S + q) * p.ld + a * 64, r0, r1, p.alpha, p.acc_q);
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
+  }
+}
+
+// dK, dV for 128 keys of one (sample, head); loops over query tiles (double-buffered Q, dO).
+// smem: K 16K | V 16K | Q/dO 2 x 32K | Pd^T 32K | dS^T 32K | lse, D (seq floats each) | barriers
+__global__ void __launch_bounds__(kBwdThreads, 1)
+    fa5_bwd_dkv(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mdO,
+                const __grid_constant__ CUtensorMap mK, const __grid_constant__ CUtensorMap mV, const Fa5B p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  const int S = p.seq, nqt = S / 128;
+  uint8_t* sK = smem;
+  uint8_t* sV = smem + 16384;
+  uint8_t* sQ[2] = {smem + 32768, smem + 65536};
+  uint8_t* sG[2] = {smem + 49152, smem + 81920};
+  uint8_t* sPd = smem + 98304;
+  uint8_t* sdS = smem + 131072;
+  float* s_l2 = reinterpret_cast<float*>(smem + 163840);
+  float* s_D = s_l2 + S;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 163840 + 8 * S);
+  uint64_t *ld_kv = bar, *qd_full = bar + 1, *s_full = bar + 3, *ps_full = bar + 4, *acc_done = bar + 5;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 6);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int kt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
+  const int64_t hbase = (int64_t(b) * p.heads + a) * S;
+  for (int t = threadIdx.x; t < S; t += blockDim.x) {
+    s_l2[t] = p.lse[hbase + t] * kLog2e;
+    s_D[t] = p.D[hbase + t];
+  }
+  if (threadIdx.x == 0) {
+    mbar_init(ld_kv, 1);
+    mbar_init(&qd_full[0], 1);
+    mbar_init(&qd_full[1], 1);
+    mbar_init(s_full, 1);
+    mbar_init(ps_full, 128);
+    mbar_init(acc_done, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 4) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(512));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;  // S^T 0..127, dP^T 128..255, dV 256..319, dK 320..383
+  if (warp == 4) {
+    if (lane == 0) {
+      const int row0 = b * S;
+      mbar_arrive_tx(ld_kv, 32768u);
+      tma_load(sK, &mK, ld_kv, a * 64, row0 + kt * 128, 0, 0);
+      tma_load(sV, &mV, ld_kv, a * 64, row0 + kt * 128, 0, 0);
+      auto load_qd = [&](int t) {
+        mbar_arrive_tx(&qd_full[t & 1], 32768u);
+        tma_load(sQ[t & 1], &mQ, &qd_full[t & 1], a * 64, row0 + t * 128, 0, 0);
+        tma_load(sG[t & 1], &mdO, &qd_full[t & 1], a * 64, row0 + t * 128, 0, 0);
+      };
+      load_qd(0);
+      if (nqt > 1) load_qd(1);
+      const uint32_t k = smem_u32(sK), v = smem_u32(sV), pd = smem_u32(sPd), ds = smem_u32(sdS);
+      auto issue_s = [&](int t) {
+        mbar_wait(&qd_full[t & 1], (t >> 1) & 1);
+        tc_fence_after();
+        const uint32_t q = smem_u32(sQ[t & 1]), g = smem_u32(sG[t & 1]);
+#pragma unroll
+        for (int kk = 0; kk < 4; ++kk) {
+          tc_mma(tmem, smem_desc(k + kk * 32, 16, 1024), smem_desc(q + kk * 32, 16, 1024), kIdN128, kk > 0 ? 1u : 0u);
+          tc_mma(tmem + 128, smem_desc(v + kk * 32, 16, 1024), smem_desc(g + kk * 32, 16, 1024), kIdN128,
+                 kk > 0 ? 1u : 0u);
+        }
+        tc_commit(s_full);
+      };
+      mbar_wait(ld_kv, 0);
+      issue_s(0);
+      for (int t = 0; t < nqt; ++t) {
+        mbar_wait(ps_full, t & 1);
+        tc_fence_after();
+        const uint32_t q = smem_u32(sQ[t & 1]), g = smem_u32(sG[t & 1]);
+        // dV += Pd^T dO_t, dK += dS^T Q_t: A K-major over the tile's queries, B = dO / Q rows (MN-major)
+        for (int kq = 0; kq < 128; kq += 16) {
+          const uint32_t aoff = (kq >> 6) * 16384 + ((kq & 63) >> 4) * 32;
+          const uint32_t acc = (t > 0 || kq > 0) ? 1u : 0u;
+          tc_mma(tmem + 256, smem_desc(pd + aoff, 16, 1024), smem_desc(g + uint32_t(kq) * 128, 8192, 1024), kIdN64MN,
+                 acc);
+          tc_mma(tmem + 320, smem_desc(ds + aoff, 16, 1024), smem_desc(q + uint32_t(kq) * 128, 8192, 1024), kIdN64MN,
+                 acc);
+        }
+        tc_commit(acc_done);
+        if (t + 1 < nqt) issue_s(t + 1);
+        if (t + 2 < nqt) {
+          mbar_wait(acc_done, t & 1);  // the products that read buffer t & 1 are done
+          load_qd(t + 2);
+        }
+      }
+    }
+  } else {
+    const int i = warp * 32 + lane;
+    const int key = kt * 128 + i;
+    const uint32_t trow = tmem + (uint32_t(warp * 32) << 16);
+    const uint32_t pd = smem_u32(sPd), ds = smem_u32(sdS);
+    const uint32_t* mcol = p.mask + hbase * (S / 32) + (key >> 5);
+    const int kb = key & 31;
+    for (int t = 0; t < nqt; ++t) {
+      mbar_wait(s_full, t & 1);
+      if (t > 0) mbar_wait(acc_done, (t - 1) & 1);  // Pd^T / dS^T buffers free
+      tc_fence_after();
+#pragma unroll 1
+      for (int c = 0; c < 128; c += 16) {
+        uint32_t rs[16], rp[16];
+        tmem_ld16(trow + uint32_t(c), rs);
+        tmem_ld16(trow + uint32_t(128 + c), rp);
+        const uint32_t* mq = mcol + int64_t(t * 128 + c) * (S / 32);
+        // in place: rp <- Pd^T, rs <- dS^T (fp32 bits)
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+          const int qq = t * 128 + c + j;
+          const bool keep = !p.drop || ((mq[j * (S / 32)] >> kb) & 1u);
+          const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - s_l2[qq]);
+          const float dp = keep ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
+          rp[j] = __float_as_uint(keep ? pr * p.keep_scale : 0.f);
+          rs[j] = __float_as_uint(pr * (dp - s_D[qq]));
+        }
+        st_row16(pd, i, c, reinterpret_cast<const float*>(rp));
+        st_row16(ds, i, c, reinterpret_cast<const float*>(rs));
+      }
+      fence_async_smem();
+      tc_fence_before();
+      mbar_arrive(ps_full);
+    }
+    mbar_wait(acc_done, (nqt - 1) & 1);
+    tc_fence_after();
+    const int64_t off = (int64_t(b) * S + key) * p.ld + a * 64;
+    uint32_t r0[32], r1[32];
+    tmem_ld32(trow + 256u, r0);
+    tmem_ld32(trow + 288u, r1);
+    if (p.dv) store_row64(static_cast<bf16*>(p.dv) + off, r0, r1, 1.f, p.acc_v);
+    tmem_ld32(trow + 320u, r0);
+    tmem_ld32(trow + 352u, r1);
+    if (p.dk) store_row64(static_cast<bf16*>(p.dk) + off, r0, r1, p.alpha, p.acc_k);
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 4) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
+  }
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 encode() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   static std::once_flag once;
@@ -293,6 +651,47 @@ bool attention_fwd_tc5(const AttnArgs& A, cudaStream_t st) {
     attr = true;
   }
   fa5_fwd<<<dim3(A.seq / 128, A.heads, A.nb), kThreads, kSmem, st>>>(mq, mk, mv, p);
+  return true;
+}
+
+bool attention_bwd_tc5(const AttnArgs& A, cudaStream_t st) {
+  if (A.dtype != BF16 || A.d != 64 || A.seq % 128 || A.seq > 512 || A.nb < 1 || !A.c || !A.lse || !A.mask ||
+      !A.dc || !A.ws)
+    return false;
+  const int64_t rows = int64_t(A.nb) * A.seq;
+  CUtensorMap mq, mg, mk, mv;
+  if (!map2(&mq, A.q, A.ld, rows, 128) || !map2(&mg, A.dc, A.ld, rows, 128) || !map2(&mk, A.k, A.ld, rows, 128) ||
+      !map2(&mv, A.v, A.ld, rows, 128))
+    return false;
+  Fa5B p;
+  p.heads = A.heads;
+  p.seq = A.seq;
+  p.ld = A.ld;
+  p.sl2 = A.alpha * kLog2e;
+  p.alpha = A.alpha;
+  p.keep_scale = A.p > 0.f ? 1.f / (1.f - A.p) : 1.f;
+  p.drop = A.p > 0.f;
+  p.lse = A.lse;
+  p.mask = A.mask;
+  p.D = A.ws;
+  p.o = static_cast<const bf16*>(A.c);
+  p.dout = static_cast<const bf16*>(A.dc);
+  p.dq = A.dq;
+  p.dk = A.dk;
+  p.dv = A.dv;
+  p.acc_q = A.acc_q;
+  p.acc_k = A.acc_k;
+  p.acc_v = A.acc_v;
+  const int smem_q = 32768 + 2 * A.seq * 128 + 32768 + 256 + 1024;
+  const int smem_kv = 163840 + 8 * A.seq + 256 + 1024;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(fa5_bwd_dq, cudaFuncAttributeMaxDynamicSharedMemorySize, 32768 + 2 * 512 * 128 + 32768 + 1280);
+    cudaFuncSetAttribute(fa5_bwd_dkv, cudaFuncAttributeMaxDynamicSharedMemorySize, 163840 + 8 * 512 + 1280);
+    attr = true;
+  }
+  fa5_bwd_dq<<<dim3(A.seq / 128, A.heads, A.nb), kBwdThreads, smem_q, st>>>(mq, mg, mk, mv, p);
+  fa5_bwd_dkv<<<dim3(A.seq / 128, A.heads, A.nb), kBwdThreads, smem_kv, st>>>(mq, mg, mk, mv, p);
   return true;
 }
 

@@ -114,6 +114,7 @@ struct AttnArgs {
   uint32_t seed = 0, step = 0, thr = 0;
   int64_t b0 = 0;
   float* ws = nullptr;
+  int no_tc5 = 0;  // tests: skip the tcgen05 kernels (mma.sync path instead)
 };
 bool attention_tc_eligible(const AttnArgs& a);  // bf16, d = 64, seq % 64 == 0 (mma.sync path)
 void attention_fwd(const AttnArgs& a, cudaStream_t st);
@@ -122,6 +123,8 @@ void attention_simt(const AttnArgs& a, bool bwd, cudaStream_t st);  // CUDA-core
 // tcgen05 forward (attention_tc.cu): bf16, d = 64, seq % 128 == 0, seq <= 512, C and lse both
 // written; false = not eligible (nothing launched).  a.thr must be set.
 bool attention_fwd_tc5(const AttnArgs& a, cudaStream_t st);
+// tcgen05 backward (same eligibility; needs c, lse, mask, dc, ws)
+bool attention_bwd_tc5(const AttnArgs& a, cudaStream_t st);
 
 // ---- pooling (NHWC) ----------------------------------------------------------------
 void maxpool_fwd(int dt, const void* x, void* y, int n, int H, int W, int C, int P, int Q, int k, int stride,

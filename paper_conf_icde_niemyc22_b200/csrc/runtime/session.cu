@@ -1297,19 +1297,11 @@ ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const f
   if (mode == 2 && (!c || !lse || !mask || !dc || !ws))
     return set_error("ts_attention: backward needs C, lse, mask, dC, ws"), TS_ERR_ARG;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  const bool mma_only = (acc & 0x100) != 0;  // tests: skip the tcgen05 forward, keep mma.sync
+  const bool mma_only = (acc & 0x100) != 0;  // tests: skip the tcgen05 kernels, keep mma.sync
   a.acc_q = acc & 1; a.acc_k = (acc >> 1) & 1; a.acc_v = (acc >> 2) & 1;
+  a.no_tc5 = mma_only ? 1 : 0;
   const bool tc = !simt_only && tsk::attention_tc_eligible(a);
-  if (tc && mode == 1 && !mma_only) {
-    tsk::AttnArgs b = a;
-    const double t = double(b.p) * 4294967296.0;
-    b.thr = b.p <= 0.f ? 0u : (t >= 4294967295.0 ? 0xFFFFFFFFu : uint32_t(t));
-    if (tsk::attention_fwd_tc5(b, st)) {
-      CU(cudaGetLastError());
-      if (used_tc) *used_tc = 2;
-      return TS_OK;
-    }
-  }
+  const bool tc5 = tc && !mma_only && a.seq % 128 == 0 && a.seq <= 512 && a.c && a.lse;
   if (tc) {
     if (mode == 1) tsk::attention_fwd(a, st);
     else tsk::attention_bwd(a, st);
@@ -1317,7 +1309,7 @@ ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const f
     tsk::attention_simt(a, mode == 2, st);
   }
   CU(cudaGetLastError());
-  if (used_tc) *used_tc = tc ? 1 : 0;
+  if (used_tc) *used_tc = tc5 ? 2 : (tc ? 1 : 0);
   return TS_OK;
 }
 

@@ -62,13 +62,15 @@ def test_attention_kernels_vs_oracle(seq, p, path):
     assert _rel(C.float().cpu().numpy(), c_ref) <= 1e-2
     ws = torch.empty(nb * heads * seq, dtype=torch.float32, device="cuda")
     dQ, dK, dV = (torch.full_like(Q, 0.25) for _ in range(3))
-    tsplit.attention(2 | force, geom, alpha, p, Q, K, V, c=C, lse=L, mask=M, dc=DC, dq=dQ, dk=dK, dv=dV, ws=ws)
+    mma = 0x100 if path == "mma" else 0
+    tsplit.attention(2 | force, geom, alpha, p, Q, K, V, c=C, lse=L, mask=M, dc=DC, dq=dQ, dk=dK, dv=dV, ws=ws,
+                     acc=mma)
     torch.cuda.synchronize()
     for got, ref in ((dQ, dq_ref), (dK, dk_ref), (dV, dv_ref)):
         assert _rel(got.float().cpu().numpy(), ref) <= 2e-2
     # accumulate flags (a later backward op adding its share)
-    tsplit.attention(2 | force, geom, alpha, p, Q, K, V, c=C, lse=L, mask=M, dc=DC, dq=dQ, dk=dK, dv=dV, acc=7,
-                     ws=ws)
+    tsplit.attention(2 | force, geom, alpha, p, Q, K, V, c=C, lse=L, mask=M, dc=DC, dq=dQ, dk=dK, dv=dV,
+                     acc=7 | mma, ws=ws)
     torch.cuda.synchronize()
     for got, ref in ((dQ, dq_ref), (dK, dk_ref), (dV, dv_ref)):
         assert _rel(got.float().cpu().numpy(), 2 * ref) <= 2e-2
