@@ -409,15 +409,18 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
     const uint32_t* mrow = p.mask + hrow * (S / 32);
     const uint32_t ds = smem_u32(sdS);
     for (int kt = 0; kt < nkt; ++kt) {
+      // this key tile's 4 keep words of the row, fetched before waiting for the products
+      uint4 mw = make_uint4(~0u, ~0u, ~0u, ~0u);
+      if (p.drop) mw = *reinterpret_cast<const uint4*>(mrow + kt * 4);
       mbar_wait(s_full, kt & 1);
       if (kt > 0) mbar_wait(dq_done, (kt - 1) & 1);  // dS buffer free
       tc_fence_after();
-#pragma unroll 1
+#pragma unroll
       for (int c = 0; c < 128; c += 32) {
         uint32_t rs[32], rp[32];
         tmem_ld32(trow + uint32_t(c), rs);
         tmem_ld32(trow + uint32_t(128 + c), rp);
-        const uint32_t bits = p.drop ? mrow[(kt * 128 + c) >> 5] : 0xFFFFFFFFu;
+        const uint32_t bits = c == 0 ? mw.x : c == 32 ? mw.y : c == 64 ? mw.z : mw.w;
 #pragma unroll
         for (int j = 0; j < 32; ++j) {
           const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
@@ -462,7 +465,8 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
   uint8_t* sdS = smem + 131072;
   float* s_l2 = reinterpret_cast<float*>(smem + 163840);
   float* s_D = s_l2 + S;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 163840 + 8 * S);
+  uint32_t* s_mask = reinterpret_cast<uint32_t*>(s_D + S);  // [128 queries][4 words of this key tile]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 163840 + 8 * S + 2048);
   uint64_t *ld_kv = bar, *qd_full = bar + 1, *s_full = bar + 3, *ps_full = bar + 4, *acc_done = bar + 5;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 6);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -544,9 +548,14 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
     const int key = kt * 128 + i;
     const uint32_t trow = tmem + (uint32_t(warp * 32) << 16);
     const uint32_t pd = smem_u32(sPd), ds = smem_u32(sdS);
-    const uint32_t* mcol = p.mask + hbase * (S / 32) + (key >> 5);
-    const int kb = key & 31;
+    const int kb = key & 31, kw = i >> 5;
     for (int t = 0; t < nqt; ++t) {
+      // stage this query tile's keep words for the key tile (query i's 4 words, one 16-byte load)
+      uint4 mw = make_uint4(~0u, ~0u, ~0u, ~0u);
+      if (p.drop) mw = *reinterpret_cast<const uint4*>(p.mask + (hbase + t * 128 + i) * (S / 32) + kt * 4);
+      named_sync(2, 128);  // previous tile's readers are done with s_mask
+      *reinterpret_cast<uint4*>(s_mask + i * 4) = mw;
+      named_sync(2, 128);
       mbar_wait(s_full, t & 1);
       if (t > 0) mbar_wait(acc_done, (t - 1) & 1);  // Pd^T / dS^T buffers free
       tc_fence_after();
@@ -555,12 +564,11 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
         uint32_t rs[16], rp[16];
         tmem_ld16(trow + uint32_t(c), rs);
         tmem_ld16(trow + uint32_t(128 + c), rp);
-        const uint32_t* mq = mcol + int64_t(t * 128 + c) * (S / 32);
         // in place: rp <- Pd^T, rs <- dS^T (fp32 bits)
 #pragma unroll
         for (int j = 0; j < 16; ++j) {
           const int qq = t * 128 + c + j;
-          const bool keep = !p.drop || ((mq[j * (S / 32)] >> kb) & 1u);
+          const bool keep = (s_mask[(c + j) * 4 + kw] >> kb) & 1u;
           const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - s_l2[qq]);
           const float dp = keep ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
           rp[j] = __float_as_uint(keep ? pr * p.keep_scale : 0.f);
@@ -683,11 +691,11 @@ bool attention_bwd_tc5(const AttnArgs& A, cudaStream_t st) {
   p.acc_k = A.acc_k;
   p.acc_v = A.acc_v;
   const int smem_q = 32768 + 2 * A.seq * 128 + 32768 + 256 + 1024;
-  const int smem_kv = 163840 + 8 * A.seq + 256 + 1024;
+  const int smem_kv = 163840 + 8 * A.seq + 2048 + 256 + 1024;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(fa5_bwd_dq, cudaFuncAttributeMaxDynamicSharedMemorySize, 32768 + 2 * 512 * 128 + 32768 + 1280);
-    cudaFuncSetAttribute(fa5_bwd_dkv, cudaFuncAttributeMaxDynamicSharedMemorySize, 163840 + 8 * 512 + 1280);
+    cudaFuncSetAttribute(fa5_bwd_dkv, cudaFuncAttributeMaxDynamicSharedMemorySize, 163840 + 8 * 512 + 2048 + 1280);
     attr = true;
   }
   fa5_bwd_dq<<<dim3(A.seq / 128, A.heads, A.nb), kBwdThreads, smem_q, st>>>(mq, mg, mk, mv, p);
