@@ -263,6 +263,9 @@ ts_status ts_session_gemm_times(const ts_session_t* s, double* flop, float* ms, 
 /* Kind of each record of ts_session_gemm_times: 0 GEMM (linear / attention), 1 conv
  * fprop, 2 conv dgrad, 3 conv wgrad (implicit GEMM); tc[i] = 1 when the tcgen05 path ran. */
 ts_status ts_session_gemm_kinds(const ts_session_t* s, int32_t* kind, int32_t* tc, uint64_t cap, uint64_t* n);
+/* Shape of each record: int32 quadruples (M, N, K, flags); flags bit0 A MN-major, bit1 B
+ * MN-major, bit2 fp32 C, bit3 beta != 0 (GEMMs; convs report their implicit-GEMM M, N, K). */
+ts_status ts_session_gemm_shapes(const ts_session_t* s, int32_t* mnkf, uint64_t cap, uint64_t* n);
 
 /* ---- data parallelism (north_star: DP over NVLink with NCCL) -------------------
  * The session allreduces the fp32 gradient region (sum) with this communicator

@@ -237,14 +237,30 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
           const bool full_chunk = col0 + 32 <= p.N;
           if (p.bias) {
+            if (full_chunk && !p.bias_f32 && (reinterpret_cast<uintptr_t>(p.bias) & 15) == 0) {
+              // 32 bias values as four 16-byte loads (the same address across the warp: one broadcast each)
+              const uint4* bp = reinterpret_cast<const uint4*>(reinterpret_cast<const bf16*>(p.bias) + col0);
 #pragma unroll
-            for (int i = 0; i < 32; ++i)
-              if (full_chunk || col0 + i < p.N)
-                v[i] += p.bias_f32 ? reinterpret_cast<const float*>(p.bias)[col0 + i]
-                                   : to_f(reinterpret_cast<const bf16*>(p.bias)[col0 + i]);
+              for (int j = 0; j < 4; ++j) {
+                const uint4 u = __ldg(bp + j);
+                const __nv_bfloat162* b2 = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+                for (int h = 0; h < 4; ++h) {
+                  const float2 f = __bfloat1622float2(b2[h]);
+                  v[8 * j + 2 * h] += f.x;
+                  v[8 * j + 2 * h + 1] += f.y;
+                }
+              }
+            } else {
+#pragma unroll
+              for (int i = 0; i < 32; ++i)
+                if (full_chunk || col0 + i < p.N)
+                  v[i] += p.bias_f32 ? reinterpret_cast<const float*>(p.bias)[col0 + i]
+                                     : to_f(reinterpret_cast<const bf16*>(p.bias)[col0 + i]);
+            }
           }
           if (p.tma_store) {
-            if (!p.c_f32 && p.beta != 0.f && row_ok) {  // bf16 accumulate: read the old row chunk
+            if (!p.c_f32 && p.beta != 0.f && !p.reduce_add && row_ok) {  // bf16 accumulate: read the old row chunk
               const bf16* cp = reinterpret_cast<const bf16*>(p.C) + cbase + col0;
 #pragma unroll
               for (int i = 0; i < 32; ++i)
@@ -450,7 +466,9 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
                     ? 1 : 0;
   if (g.beta != 0.f && g.beta != 1.f) p.tma_store = 0;
   if (!p.tma_store) mc = ma;  // unused
-  p.reduce_add = (p.tma_store && p.c_f32 && g.beta == 1.f) ? 1 : 0;
+  // beta = 1 accumulates with a TMA reduce-add of the new tile (fp32, or bf16 gradients that
+  // several backward ops add into: the old values never pass through registers)
+  p.reduce_add = (p.tma_store && g.beta == 1.f) ? 1 : 0;
   // split-K for products with few output tiles and a long reduction (dW = dY^T X):
   // partial tiles are reduce-added in fp32 (the zero-init comes first when beta == 0)
   p.ksplit = 1;
@@ -498,6 +516,7 @@ void gemm(const GemmArgs& g, cudaStream_t st) {
     rec.N = g.N;
     rec.K = g.K;
     rec.batch = g.nb1 * g.nb2;
+    rec.flags = (g.a.mn_major ? 1 : 0) | (g.b.mn_major ? 2 : 0) | (g.c_dtype == F32 ? 4 : 0) | (g.beta != 0.f ? 8 : 0);
     g_sink->push_back(rec);
   }
 }

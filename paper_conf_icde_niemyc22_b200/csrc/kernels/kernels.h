@@ -44,7 +44,8 @@ struct GemmRecord {
   cudaEvent_t start, stop;
   double flop;
   int M, N, K, batch, tc;
-  int kind;  // 0 GEMM, 1 conv fprop, 2 conv dgrad, 3 conv wgrad
+  int kind;   // 0 GEMM, 1 conv fprop, 2 conv dgrad, 3 conv wgrad
+  int flags;  // GEMM: bit0 A MN-major, bit1 B MN-major, bit2 fp32 C, bit3 beta != 0
 };
 void gemm_records_enable(std::vector<GemmRecord>* sink);
 std::vector<GemmRecord>* gemm_records_sink();

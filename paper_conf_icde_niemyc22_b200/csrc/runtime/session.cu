@@ -10,6 +10,7 @@
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <array>
 #include <cstring>
 #include <functional>
 #include <map>
@@ -91,6 +92,7 @@ struct ts_session_s {
   std::vector<tsk::GemmRecord> gemm_recs;
   std::vector<double> gemm_flop, gemm_ms;
   std::vector<int> gemm_batch, gemm_kind, gemm_tc;
+  std::vector<std::array<int, 4>> gemm_shape;  // M, N, K, flags
 };
 
 namespace {
@@ -858,6 +860,7 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
     s->gemm_batch.clear();
     s->gemm_kind.clear();
     s->gemm_tc.clear();
+    s->gemm_shape.clear();
     for (auto& r : s->gemm_recs) {
       float ms = 0.f;
       cudaEventElapsedTime(&ms, r.start, r.stop);
@@ -866,6 +869,7 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
       s->gemm_batch.push_back(r.batch);
       s->gemm_kind.push_back(r.kind);
       s->gemm_tc.push_back(r.tc);
+      s->gemm_shape.push_back({r.M, r.N, r.K, r.flags});
     }
     s->item_ms.assign(s->prog.size(), 0.f);
     for (auto& c : s->prog)
@@ -1056,6 +1060,15 @@ ts_status ts_session_gemm_times(const ts_session_t* s, double* flop, float* ms, 
     if (ms) ms[i] = float(s->gemm_ms[i]);
     if (batch) batch[i] = s->gemm_batch[i];
   }
+  return TS_OK;
+}
+
+ts_status ts_session_gemm_shapes(const ts_session_t* s, int32_t* mnkf, uint64_t cap, uint64_t* n) {
+  if (!s || !n) return set_error("null argument"), TS_ERR_ARG;
+  *n = s->gemm_shape.size();
+  for (uint64_t i = 0; i < s->gemm_shape.size() && i < cap; ++i)
+    for (int j = 0; j < 4; ++j)
+      if (mnkf) mnkf[4 * i + j] = s->gemm_shape[i][j];
   return TS_OK;
 }
 

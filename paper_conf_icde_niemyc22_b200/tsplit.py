@@ -120,6 +120,7 @@ def lib():
             "ts_session_item_times": (i32, [vp, P(C.c_float), u64, P(u64)]),
             "ts_session_gemm_times": (i32, [vp, P(C.c_double), P(C.c_float), P(i32), u64, P(u64)]),
             "ts_session_gemm_kinds": (i32, [vp, P(i32), P(i32), u64, P(u64)]),
+            "ts_session_gemm_shapes": (i32, [vp, P(i32), u64, P(u64)]),
             "ts_profile_measure": (i32, [vp, vp, u64, P(vp), i32, i32, P(vp)]),
             "ts_profile_get": (i32, [vp, i32, i32, P(C.c_double), P(C.c_double)]),
             "ts_profile_pcie": (i32, [vp, P(C.c_double), P(C.c_double)]),
@@ -442,6 +443,14 @@ class Session:
         t = (C.c_int32 * n.value)()
         check(lib().ts_session_gemm_kinds(self.h, k, t, n.value, C.byref(n)))
         return list(zip(k, t))
+
+    def gemm_shapes(self):
+        """[(M, N, K, flags)] per record of gemm_times."""
+        n = C.c_uint64()
+        check(lib().ts_session_gemm_shapes(self.h, None, 0, C.byref(n)))
+        b = (C.c_int32 * (4 * n.value))()
+        check(lib().ts_session_gemm_shapes(self.h, b, len(b), C.byref(n)))
+        return [tuple(b[4 * i:4 * i + 4]) for i in range(n.value)]
 
     def launches(self) -> int:
         n = C.c_int64()
