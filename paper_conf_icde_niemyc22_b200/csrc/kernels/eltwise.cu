@@ -185,6 +185,37 @@ __global__ void scale_kernel(float* x, int64_t n, float s) {
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
     x[i] *= s;
 }
+// One launch for the whole optimiser step: block b updates chunk b of one parameter
+// (fp32 master -= lr * grad) and, for bf16 graphs, writes the bf16 copy from the
+// value still in registers (no second pass over the masters, no per-tensor launches).
+__global__ void __launch_bounds__(256) sgd_fused_kernel(const SgdChunk* __restrict__ chunks, char* slab, float lr) {
+  const SgdChunk c = chunks[blockIdx.x];
+  float* m = reinterpret_cast<float*>(slab + c.m_off);
+  const float* g = reinterpret_cast<const float*>(slab + c.g_off);
+  bf16* cp = c.c_off != ~0ull ? reinterpret_cast<bf16*>(slab + c.c_off) : nullptr;
+  const int64_t nv = c.n / 4;
+  for (int64_t v = threadIdx.x; v < nv; v += blockDim.x) {
+    float4 mv = reinterpret_cast<float4*>(m)[v];
+    const float4 gv = reinterpret_cast<const float4*>(g)[v];
+    mv.x -= lr * gv.x;
+    mv.y -= lr * gv.y;
+    mv.z -= lr * gv.z;
+    mv.w -= lr * gv.w;
+    reinterpret_cast<float4*>(m)[v] = mv;
+    if (cp) {
+      __nv_bfloat162 lo = __floats2bfloat162_rn(mv.x, mv.y), hi = __floats2bfloat162_rn(mv.z, mv.w);
+      uint2 u;
+      u.x = *reinterpret_cast<uint32_t*>(&lo);
+      u.y = *reinterpret_cast<uint32_t*>(&hi);
+      reinterpret_cast<uint2*>(cp)[v] = u;
+    }
+  }
+  for (int64_t i = nv * 4 + threadIdx.x; i < c.n; i += blockDim.x) {
+    m[i] -= lr * g[i];
+    if (cp) cp[i] = __float2bfloat16_rn(m[i]);
+  }
+}
+
 int grid_for(int64_t n) {
   int64_t g = (n + 255) / 256;
   return int(g < 148 * 8 ? (g > 0 ? g : 1) : 148 * 8);
@@ -226,6 +257,9 @@ void dropout(int dt, const void* x, void* y, int acc, int64_t n, int64_t elem0, 
 }
 void sgd_update(float* master, const float* grad, int64_t n, float lr, float gscale, cudaStream_t st) {
   sgd_kernel<<<grid_for(n), 256, 0, st>>>(master, grad, n, lr * gscale);
+}
+void sgd_fused(const SgdChunk* chunks, int n_chunks, char* slab, float lr, float gscale, cudaStream_t st) {
+  if (n_chunks > 0) sgd_fused_kernel<<<n_chunks, 256, 0, st>>>(chunks, slab, lr * gscale);
 }
 void cast_f32_bf16(const float* src, void* dst, int64_t n, cudaStream_t st) {
   cast_kernel<<<grid_for(n), 256, 0, st>>>(src, reinterpret_cast<bf16*>(dst), n);

@@ -176,6 +176,13 @@ void xent_bwd(int dt, const void* z, const int* labels, void* dz, int acc, int64
               cudaStream_t st);
 // ---- optimiser / static region ------------------------------------------------
 void sgd_update(float* master, const float* grad, int64_t n, float lr, float gscale, cudaStream_t st);
+// multi-tensor SGD + bf16 copy refresh: chunk table in device memory (offsets into the slab;
+// c_off = ~0 for no copy); chunk starts are 16-byte aligned
+struct SgdChunk {
+  uint64_t m_off, g_off, c_off;
+  int64_t n;
+};
+void sgd_fused(const SgdChunk* chunks, int n_chunks, char* slab, float lr, float gscale, cudaStream_t st);
 void cast_f32_bf16(const float* src, void* dst, int64_t n, cudaStream_t st);
 void scale_f32(float* x, int64_t n, float s, cudaStream_t st);
 

@@ -318,7 +318,35 @@ __global__ void __launch_bounds__(256) ln_bwd_dgb(const T* __restrict__ dy, cons
   const int c0 = blockIdx.x * 256 + lane * 8;
   float pg[8] = {0, 0, 0, 0, 0, 0, 0, 0}, pb[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   if (c0 < H) {
-    for (int64_t r = int64_t(blockIdx.y) * 8 + w; r < rows; r += int64_t(G) * 8) {
+    const int64_t rstep = int64_t(G) * 8;
+    int64_t r0 = int64_t(blockIdx.y) * 8 + w;
+    if (sizeof(T) == 2) {
+      // two rows in flight per thread (HBM latency hiding); same per-column summation order
+      for (; r0 + rstep < rows; r0 += 2 * rstep) {
+        uint4 ux[2], ud[2];
+        float mr[2], rr[2];
+#pragma unroll
+        for (int k = 0; k < 2; ++k) {
+          const int64_t r = r0 + k * rstep;
+          ux[k] = __ldcs(reinterpret_cast<const uint4*>(x + r * H + c0));
+          ud[k] = __ldcs(reinterpret_cast<const uint4*>(dy + r * H + c0));
+          mr[k] = stats[2 * r];
+          rr[k] = stats[2 * r + 1];
+        }
+#pragma unroll
+        for (int k = 0; k < 2; ++k) {
+          const T* tx = reinterpret_cast<const T*>(&ux[k]);
+          const T* td = reinterpret_cast<const T*>(&ud[k]);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const float d = to_f(td[i]);
+            pg[i] += d * ((to_f(tx[i]) - mr[k]) * rr[k]);
+            pb[i] += d;
+          }
+        }
+      }
+    }
+    for (int64_t r = r0; r < rows; r += rstep) {
       const float mean = stats[2 * r], rstd = stats[2 * r + 1];
       constexpr int VV = 16 / sizeof(T);
 #pragma unroll
@@ -393,7 +421,23 @@ __global__ void __launch_bounds__(256) colsum_kernel(const T* __restrict__ x, in
   const int c0 = blockIdx.x * 256 + lane * 8;
   float accv[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   const bool vec = (N % 8 == 0) && c0 + 8 <= N && (reinterpret_cast<uintptr_t>(x) % 16 == 0);
-  for (int64_t r = int64_t(blockIdx.y) * 8 + w; r < rows; r += int64_t(G) * 8) {
+  const int64_t rstep = int64_t(G) * 8;
+  int64_t r0 = int64_t(blockIdx.y) * 8 + w;
+  if (vec && !filter && sizeof(T) == 2) {
+    // four rows in flight per thread (HBM latency hiding); fixed summation order per column
+    for (; r0 + 3 * rstep < rows; r0 += 4 * rstep) {
+      uint4 u[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) u[k] = __ldcs(reinterpret_cast<const uint4*>(x + (r0 + k * rstep) * N + c0));
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        const T* t = reinterpret_cast<const T*>(&u[k]);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) accv[i] += to_f(t[i]);
+      }
+    }
+  }
+  for (int64_t r = r0; r < rows; r += rstep) {
     if (filter && filter[r] != fval) continue;
     const T* xr = x + r * N;
     if (vec) {
@@ -428,8 +472,15 @@ __global__ void __launch_bounds__(256) colsum_kernel(const T* __restrict__ x, in
   if (!last) return;
   __threadfence();
   if (c < N) {
-    double t = 0.0;
-    for (int b = 0; b < G; ++b) t += double(__ldcg(&ws[int64_t(b) * N + c]));
+    // eight independent fp64 chains (the loads overlap), combined in a fixed order
+    double t8[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    int b = 0;
+    for (; b + 8 <= G; b += 8) {
+#pragma unroll
+      for (int k = 0; k < 8; ++k) t8[k] += double(__ldcg(&ws[int64_t(b + k) * N + c]));
+    }
+    for (; b < G; ++b) t8[0] += double(__ldcg(&ws[int64_t(b) * N + c]));
+    const double t = ((t8[0] + t8[1]) + (t8[2] + t8[3])) + ((t8[4] + t8[5]) + (t8[6] + t8[7]));
     out[c] = acc ? float(double(out[c]) + t) : float(t);
   }
   if (threadIdx.x == 0) tickets[blockIdx.x] = 0u;  // re-arm for the next launch / graph replay
@@ -745,13 +796,21 @@ bool ln_bwd_split_t(const void* dy, const void* x, const void* g, void* dx, int 
   const int nch = (H + 32 * V - 1) / (32 * V);
   if (H % 8 || nch > 4 || !al16(dy) || !al16(x) || !al16(g) || !al16(dx)) return false;
   const int cb = (H + 255) / 256;
-  int G = int((rows + 7) / 8);
-  int cap = (2 * 148) / cb;
-  if (cap > 64) cap = 64;
+  int G = int((rows + 15) / 16);
+  int cap = (4 * 148) / cb;  // ~4 blocks per SM
+  if (sizeof(T) == 4) {
+    G = int((rows + 7) / 8);
+    cap = (2 * 148) / cb;
+  }
+  const uint64_t stats_bytes = uint64_t(rows) * 8;
+  if (stats_bytes + kTicketBytes + uint64_t(2 * H * 4) > ws_bytes) return false;
+  const int64_t ws_rows = int64_t((ws_bytes - kTicketBytes - stats_bytes) / (uint64_t(2 * H) * 4));
+  if (cap > ws_rows) cap = int(ws_rows);
+  if (cap > 1024) cap = 1024;
+  if (sizeof(T) == 4 && cap > 64) cap = 64;  // fp32 graphs: few long partials (see column_sum)
   if (cap < 1) cap = 1;
   if (G > cap) G = cap;
-  const uint64_t stats_bytes = uint64_t(rows) * 8, part_bytes = uint64_t(G) * 2 * H * 4;
-  if (stats_bytes + part_bytes + kTicketBytes > ws_bytes) return false;
+  const uint64_t part_bytes = uint64_t(G) * 2 * H * 4;
   float* part = ws;
   float* stats = ws + (part_bytes / 4);
   auto DY = (const T*)dy;
@@ -796,10 +855,19 @@ void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64
 void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, uint64_t ws_bytes, float* out, int acc,
                 const int* filter, int fval, cudaStream_t st) {
   const int cb = (N + 255) / 256;
-  int G = int((rows + 7) / 8);
-  int cap = 296 / cb;
+  int G = int((rows + 31) / 32);
+  int cap = 592 / cb;  // ~4 blocks of 256 threads per SM
+  if (dt == F32) {     // fp32 graphs keep the round-1 partition (see below)
+    G = int((rows + 7) / 8);
+    cap = 296 / cb;
+  }
+  const int64_t ws_rows = int64_t((ws_bytes - kTicketBytes) / (uint64_t(N) * 4));
+  if (cap > ws_rows) cap = int(ws_rows);
+  if (cap > 1024) cap = 1024;
+  // fp32 graphs (tiny parity configs) keep few, long fp32 partials: their split-vs-unsplit
+  // bar (1e-6, R17) is set by how many rows each fp32 partial sums
+  if (dt == F32 && cap > 64) cap = 64;
   if (cap < 1) cap = 1;
-  if (cap > 64) cap = 64;
   if (G > cap) G = cap;
   if (G < 1) G = 1;
   // completion tickets live in the last 4 KB of the workspace, which no other kernel uses

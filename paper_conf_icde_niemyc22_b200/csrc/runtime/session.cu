@@ -71,6 +71,8 @@ struct ts_session_s {
   std::vector<std::vector<int>> buckets_after;  // per program command: buckets to launch after it
   std::vector<cudaEvent_t> ev_bucket;
   cudaEvent_t ev_comm_done = nullptr;
+  tsk::SgdChunk* sgd_chunks = nullptr;  // device table for the fused optimiser step
+  int n_sgd_chunks = 0;
   int world = 1;
   float lr = 0.f;
   uint32_t step = 0;
@@ -721,6 +723,25 @@ ts_status build_program(ts_session_t* s) {
     }
     CU(cudaEventCreateWithFlags(&s->ev_comm_done, cudaEventDisableTiming));
   }
+  // optimiser chunk table: 64K-element chunks of every parameter (master, grad, bf16 copy)
+  {
+    std::vector<tsk::SgdChunk> ch;
+    for (auto& t : g.t)
+      if (t.kind == TS_PARAM)
+        for (int64_t e = 0; e < t.numel; e += 65536) {
+          tsk::SgdChunk c;
+          c.m_off = g.master_off[t.id] + uint64_t(e) * 4;
+          c.g_off = g.grad_off[t.id] + uint64_t(e) * 4;
+          c.c_off = g.dtype == TS_BF16 ? g.copy_off[t.id] + uint64_t(e) * 2 : ~0ull;
+          c.n = std::min<int64_t>(65536, t.numel - e);
+          ch.push_back(c);
+        }
+    s->n_sgd_chunks = int(ch.size());
+    if (!ch.empty()) {
+      CU(cudaMalloc(&s->sgd_chunks, ch.size() * sizeof(tsk::SgdChunk)));
+      CU(cudaMemcpy(s->sgd_chunks, ch.data(), ch.size() * sizeof(tsk::SgdChunk), cudaMemcpyHostToDevice));
+    }
+  }
   CU(cudaEventCreateWithFlags(&s->ev_mark, cudaEventDisableTiming));
   CU(cudaEventCreateWithFlags(&s->ev_join_d2h, cudaEventDisableTiming));
   CU(cudaEventCreateWithFlags(&s->ev_join_h2d, cudaEventDisableTiming));
@@ -780,15 +801,8 @@ void issue_step(ts_session_t* s) {
     cudaEventRecord(s->ev_comm_done, s->comm);
     cudaStreamWaitEvent(cs, s->ev_comm_done, 0);
   }
-  if (s->lr != 0.f && gend > gbeg) {
-    tsk::sgd_update(reinterpret_cast<float*>(s->slab + mbeg), reinterpret_cast<const float*>(s->slab + gbeg),
-                    int64_t((gend - gbeg) / 4), s->lr, 1.f / float(s->world), cs);
-    if (g.dtype == TS_BF16)
-      for (auto& t : g.t)
-        if (t.kind == TS_PARAM)
-          tsk::cast_f32_bf16(reinterpret_cast<float*>(s->slab + g.master_off[t.id]), s->slab + g.copy_off[t.id],
-                             t.numel, cs);
-  }
+  if (s->lr != 0.f && gend > gbeg) tsk::sgd_fused(s->sgd_chunks, s->n_sgd_chunks, s->slab, s->lr, 1.f / float(s->world), cs);
+  (void)mbeg;
   if (d2h_used) {
     cudaEventRecord(s->ev_join_d2h, s->d2h);
     cudaStreamWaitEvent(cs, s->ev_join_d2h, 0);
@@ -950,6 +964,7 @@ void ts_session_destroy(ts_session_t* s) {
   for (auto e : s->ev_bucket)
     if (e) cudaEventDestroy(e);
   if (s->ev_comm_done) cudaEventDestroy(s->ev_comm_done);
+  if (s->sgd_chunks) cudaFree(s->sgd_chunks);
   if (s->comm) cudaStreamDestroy(s->comm);
   if (s->ev_mark) cudaEventDestroy(s->ev_mark);
   if (s->ev_join_d2h) cudaEventDestroy(s->ev_join_d2h);
