@@ -335,15 +335,19 @@ def main():
     arrays = gen.make_inputs(spec, seed=rank)
     dev_inputs = tsplit.inputs_to_device(G, arrays, device=f"cuda:{local}")
     t0 = time.time()
-    blob, pcie = None, None
+    blob, pcie, pst0 = None, None, None
     if rank == 0:
         # profile every op (and split widths) on the GPU before planning
         prof = tsplit.Profile.measure(G, dev_inputs, max_p=4, device=local) if not args.analytic_profile else None
         pcie = prof.pcie() if prof else None
-        blob = tsplit.Plan.plan(G, budget, prof).serialize()
+        plan0 = tsplit.Plan.plan(G, budget, prof)
+        pst0 = plan0.stats()  # predicted time with the measured profile
+        blob = plan0.serialize()
     plan_s = time.time() - t0
     plan = tsplit.Plan.deserialize(G, bcast_bytes(blob))
     pst = plan.stats()
+    if pst0 is not None:
+        pst["predicted_s"] = pst0["predicted_s"]
 
     comm = None
     if world > 1:

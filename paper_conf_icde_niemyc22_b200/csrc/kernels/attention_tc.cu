@@ -29,11 +29,12 @@ namespace {
 
 using namespace tc;
 
-constexpr int kSoftWarps = 8;
+constexpr int kSoftWarps = 16;  // four per TMEM lane quarter, each owning a quarter of the keys
+constexpr int kGroups = kSoftWarps / 4;
 constexpr int kCtlWarp = kSoftWarps;
 constexpr int kThreads = 32 * (kSoftWarps + 1);
 constexpr int kRegion = 64 * 1024;
-constexpr int kSmem = 3 * kRegion + 2048 + 1024;  // PB(+Q) | K(=PA) | V | barriers + exchange
+constexpr int kSmem = 3 * kRegion + 5120 + 1024;  // PB(+Q) | K(=PA) | V | barriers + exchange (+align)
 
 constexpr float kLog2e = 1.4426950408889634f;
 constexpr float kLn2 = 0.6931471805599453f;
@@ -77,7 +78,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint64_t *qk_full = bar, *v_full = bar + 1, *s_full = bar + 2, *p_full = bar + 3, *o_full = bar + 5;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 6);
   float* red_m = reinterpret_cast<float*>(smem + 3 * kRegion + 256);
-  float* red_l = red_m + 256;
+  float* red_l = red_m + 128 * kGroups;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int qt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
@@ -86,8 +87,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     mbar_init(qk_full, 1);
     mbar_init(v_full, 1);
     mbar_init(s_full, 1);
-    mbar_init(&p_full[0], 128);
-    mbar_init(&p_full[1], 128);
+    mbar_init(&p_full[0], 128 * kGroups / 2);
+    mbar_init(&p_full[1], 128 * kGroups / 2);
     mbar_init(o_full, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -139,15 +140,17 @@ __global__ void __launch_bounds__(kThreads, 1)
       tc_commit(o_full);
     }
   } else {
-    // ===== softmax warps: row i, key half g =====
+    // ===== softmax warps: row i, key group g (S / kGroups keys) =====
     const int qq = warp & 3, g = warp >> 2;
     const int i = qq * 32 + lane;
     const uint32_t trow = tmem + (uint32_t(qq * 32) << 16);
-    const int c0 = g * half;
+    const int gw = S / kGroups;
+    const int c0 = g * gw;
+    const int hf = c0 / half;  // which P half (MMA batch) this group fills
     mbar_wait(s_full, 0);
     tc_fence_after();
     float m = -INFINITY;
-    for (int c = c0; c < c0 + half; c += 32) {
+    for (int c = c0; c < c0 + gw; c += 32) {
       uint32_t r[32];
       tmem_ld32(trow + uint32_t(c), r);
 #pragma unroll
@@ -155,12 +158,14 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     red_m[g * 128 + i] = m;
     named_sync(1, 32 * kSoftWarps);
-    m = fmaxf(red_m[i], red_m[128 + i]) * p.sl2;
+#pragma unroll
+    for (int gg = 0; gg < kGroups; ++gg) m = fmaxf(m, red_m[gg * 128 + i]);
+    m *= p.sl2;
     const uint64_t erow = ((uint64_t(p.b0 + b) * p.heads + a) * uint64_t(S) + uint64_t(qt * 128 + i)) * uint64_t(S);
     const int64_t mrow = ((int64_t(b) * p.heads + a) * S + qt * 128 + i) * (S / 32);
     float l = 0.f;
-    const uint32_t sp = smem_u32(g == 0 ? rK : rPB);
-    for (int c = c0; c < c0 + half; c += 32) {
+    const uint32_t sp = smem_u32(hf == 0 ? rK : rPB);
+    for (int c = c0; c < c0 + gw; c += 32) {
       uint32_t r[32];
       tmem_ld32(trow + uint32_t(c), r);
       float v[32];
@@ -186,7 +191,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       if (p.mask) p.mask[mrow + (c >> 5)] = bits;
       // 32 keys = 4 sixteen-byte chunks of row i in the K-major SW128 layout
-      const int kl = c - c0;  // key within this half
+      const int kl = c - hf * half;  // key within this half
       const uint32_t blk = sp + uint32_t(kl >> 6) * 16384u + uint32_t(i) * 128u;
 #pragma unroll
       for (int q4 = 0; q4 < 4; ++q4) {
@@ -197,11 +202,13 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     fence_async_smem();
     tc_fence_before();
-    mbar_arrive(&p_full[g]);
+    mbar_arrive(&p_full[hf]);
     red_l[g * 128 + i] = l;
     named_sync(1, 32 * kSoftWarps);
     if (g == 0) {
-      l = red_l[i] + red_l[128 + i];
+      l = 0.f;
+#pragma unroll
+      for (int gg = 0; gg < kGroups; ++gg) l += red_l[gg * 128 + i];
       mbar_wait(o_full, 0);
       tc_fence_after();
       const float inv = p.keep_scale / l;

@@ -95,7 +95,7 @@ __device__ __forceinline__ void ew_vec(const T* __restrict__ a, const T* __restr
 template <class T, int OP, int V>
 __global__ void __launch_bounds__(256) ew_kernel(const T* __restrict__ a, const T* __restrict__ b, T* y, int64_t n,
                                                  int acc, EwP q) {
-  constexpr int U = 1;
+  constexpr int U = 2;  // two 16-byte vectors in flight per thread (HBM latency)
   const int64_t nv = n / V;
   const int64_t stride = int64_t(gridDim.x) * blockDim.x;
   for (int64_t v0 = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; v0 < nv; v0 += stride * U) {

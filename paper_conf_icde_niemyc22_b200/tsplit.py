@@ -191,8 +191,11 @@ class Graph:
         self.names = {t["name"]: t["id"] for t in ts}
 
     def __del__(self):
-        if getattr(self, "h", None):
-            lib().ts_graph_destroy(self.h)
+        try:
+            if getattr(self, "h", None):
+                lib().ts_graph_destroy(self.h)
+        except Exception:  # interpreter teardown: the library may already be gone
+            pass
 
     def schedule(self):
         n = C.c_int32()
@@ -252,8 +255,11 @@ class Profile:
         check(lib().ts_profile_set_pcie(self.h, d2h, h2d))
 
     def __del__(self):
-        if getattr(self, "h", None):
-            lib().ts_profile_destroy(self.h)
+        try:
+            if getattr(self, "h", None):
+                lib().ts_profile_destroy(self.h)
+        except Exception:  # interpreter teardown: the library may already be gone
+            pass
 
 
 class Plan:
@@ -280,8 +286,11 @@ class Plan:
         return cls(graph, h)
 
     def __del__(self):
-        if getattr(self, "h", None):
-            lib().ts_plan_destroy(self.h)
+        try:
+            if getattr(self, "h", None):
+                lib().ts_plan_destroy(self.h)
+        except Exception:  # interpreter teardown: the library may already be gone
+            pass
 
     def get(self, tid):
         c = TensorCfg()
@@ -365,8 +374,11 @@ class Session:
         self.input_ids = [t["id"] for t in spec["tensors"] if t["kind"] in ("input", "label")]
 
     def __del__(self):
-        if getattr(self, "h", None):
-            lib().ts_session_destroy(self.h)
+        try:
+            if getattr(self, "h", None):
+                lib().ts_session_destroy(self.h)
+        except Exception:  # interpreter teardown: the library may already be gone
+            pass
 
     def set_params(self, params: dict):
         for t in self.graph.spec["tensors"]:
