@@ -260,29 +260,14 @@ struct Fa5B {
   int acc_q, acc_k, acc_v;
 };
 
-constexpr int kBwdThreads = 32 * 5;
+// 16 compute warps (four per TMEM lane quarter, each owning 32 of a tile's 128 columns) + 1 control warp
+constexpr int kBwdCW = 16;
+constexpr int kBwdCtl = kBwdCW;
+constexpr int kBwdThreads = 32 * (kBwdCW + 1);
 constexpr uint32_t kIdN128 = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(128 >> 3) << 17) | (uint32_t(128 >> 4) << 24);
 constexpr uint32_t kIdN64MN = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | (uint32_t(64 >> 3) << 17) |
                               (uint32_t(128 >> 4) << 24);
 
-__device__ __forceinline__ void tmem_ld16(uint32_t taddr, uint32_t (&r)[16]) {
-  asm volatile(
-      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
-      : "r"(taddr));
-  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-}
-// 16 values of row i at keys [kl, kl+16) (two 16-byte chunks) of a K-major SW128 operand
-__device__ __forceinline__ void st_row16(uint32_t base, int i, int kl, const float* v) {
-  const uint32_t blk = base + uint32_t(kl >> 6) * 16384u + uint32_t(i) * 128u;
-#pragma unroll
-  for (int q2 = 0; q2 < 2; ++q2) {
-    const int chunk = ((kl & 63) >> 3) + q2;
-    sts128(blk + (uint32_t(chunk ^ (i & 7)) << 4), pk2(v[8 * q2], v[8 * q2 + 1]), pk2(v[8 * q2 + 2], v[8 * q2 + 3]),
-           pk2(v[8 * q2 + 4], v[8 * q2 + 5]), pk2(v[8 * q2 + 6], v[8 * q2 + 7]));
-  }
-}
 // store 32 bf16 values of row i at keys [kl, kl+32) of a K-major SW128 operand (64-key blocks of 16 KB)
 __device__ __forceinline__ void st_row32(uint32_t base, int i, int kl, const float* v) {
   const uint32_t blk = base + uint32_t(kl >> 6) * 16384u + uint32_t(i) * 128u;
@@ -293,34 +278,51 @@ __device__ __forceinline__ void st_row32(uint32_t base, int i, int kl, const flo
            pk2(v[8 * q4 + 4], v[8 * q4 + 5]), pk2(v[8 * q4 + 6], v[8 * q4 + 7]));
   }
 }
-__device__ __forceinline__ void store_row64(bf16* dst, const uint32_t (&r0)[32], const uint32_t (&r1)[32], float sc,
-                                            int acc) {
+__device__ __forceinline__ void tmem_ld32_nw(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+        "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+        "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+// 32 columns of one row (scaled by sc, optionally added to the bf16 values already there)
+__device__ __forceinline__ void store_row32(bf16* dst, const uint32_t (&r)[32], float sc, int acc) {
 #pragma unroll
-  for (int h = 0; h < 2; ++h) {
-    const uint32_t* r = h ? r1 : r0;
+  for (int j = 0; j < 4; ++j) {
+    float f[8];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      float f[8];
+    for (int e = 0; e < 8; ++e) f[e] = __uint_as_float(r[8 * j + e]) * sc;
+    uint4* pp = reinterpret_cast<uint4*>(dst + 8 * j);
+    if (acc) {
+      const uint4 old = *pp;
+      const __nv_bfloat162* o2 = reinterpret_cast<const __nv_bfloat162*>(&old);
 #pragma unroll
-      for (int e = 0; e < 8; ++e) f[e] = __uint_as_float(r[8 * j + e]) * sc;
-      uint4* pp = reinterpret_cast<uint4*>(dst + h * 32 + 8 * j);
-      if (acc) {
-        const uint4 old = *pp;
-        const __nv_bfloat162* o2 = reinterpret_cast<const __nv_bfloat162*>(&old);
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const float2 x = __bfloat1622float2(o2[e]);
-          f[2 * e] += x.x;
-          f[2 * e + 1] += x.y;
-        }
+      for (int e = 0; e < 4; ++e) {
+        const float2 x = __bfloat1622float2(o2[e]);
+        f[2 * e] += x.x;
+        f[2 * e + 1] += x.y;
       }
-      *pp = make_uint4(pk2(f[0], f[1]), pk2(f[2], f[3]), pk2(f[4], f[5]), pk2(f[6], f[7]));
     }
+    *pp = make_uint4(pk2(f[0], f[1]), pk2(f[2], f[3]), pk2(f[4], f[5]), pk2(f[6], f[7]));
   }
 }
 
+// Both backward kernels put queries on the TMEM lanes of the score tiles (S = Q K^T and
+// dP = dO V^T, M = 128 queries), so a thread's row constants — lse, D = dO.O and the keep
+// word of its 32 keys — are per-thread scalars loaded once per tile.  16 compute warps
+// (four per lane quarter, each owning 32 of the tile's 128 key columns) and one control
+// thread.  The control thread issues the next tile's S, dP as soon as every compute warp has
+// copied the current ones out of TMEM (s_free), and the bf16 operands the compute warps
+// write (dS; P^T as well for dK/dV) are double-buffered in shared memory, so the tensor
+// core works on tile t+1 while the compute warps are still on tile t.
+//
 // dQ for 128 queries of one (sample, head); all of K and V in shared memory.
-// smem: Q 16K | dO 16K | K seq*128 | V seq*128 | dS 32K | barriers
+// smem: Q 16K | dO 16K | K seq*128 | V seq*128 | dS 2 x 32K | barriers
+// TMEM: S 0..127, dP 128..255, dQ 256..319
 __global__ void __launch_bounds__(kBwdThreads, 1)
     fa5_bwd_dq(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mdO,
                const __grid_constant__ CUtensorMap mK, const __grid_constant__ CUtensorMap mV, const Fa5B p) {
@@ -331,20 +333,32 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
   uint8_t* sdO = smem + 16384;
   uint8_t* sK = smem + 32768;
   uint8_t* sV = sK + S * 128;
-  uint8_t* sdS = sV + S * 128;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sdS + 32768);
-  uint64_t *ld_full = bar, *s_full = bar + 1, *ds_full = bar + 2, *dq_done = bar + 3;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 4);
+  uint8_t* sdS = sV + S * 128;  // two 32 KB buffers
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sdS + 65536);
+  uint64_t *ld_full = bar, *s_full = bar + 1, *s_free = bar + 2, *ds_full = bar + 3 /*[2]*/, *dq_done = bar + 5 /*[2]*/;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 7);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int qt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
+  // the D-row loads of the compute warps go out before the setup (their latency overlaps it)
+  uint4 x0, x1, y0, y1;
+  if (warp < kBwdCW) {
+    const int64_t roff = (int64_t(b) * S + qt * 128 + (warp & 3) * 32 + lane) * p.ld + a * 64 + (warp >> 2) * 16;
+    x0 = *reinterpret_cast<const uint4*>(p.o + roff);
+    x1 = *reinterpret_cast<const uint4*>(p.o + roff + 8);
+    y0 = *reinterpret_cast<const uint4*>(p.dout + roff);
+    y1 = *reinterpret_cast<const uint4*>(p.dout + roff + 8);
+  }
   if (threadIdx.x == 0) {
     mbar_init(ld_full, 1);
     mbar_init(s_full, 1);
-    mbar_init(ds_full, 128);
-    mbar_init(dq_done, 1);
+    mbar_init(s_free, 32 * kBwdCW);
+    mbar_init(&ds_full[0], 32 * kBwdCW);
+    mbar_init(&ds_full[1], 32 * kBwdCW);
+    mbar_init(&dq_done[0], 1);
+    mbar_init(&dq_done[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 4) {
+  if (warp == kBwdCtl) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(512));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -352,8 +366,8 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  const uint32_t tmem = *tmem_slot;  // S: 0..127, dP: 128..255, dQ: 256..319
-  if (warp == 4) {
+  const uint32_t tmem = *tmem_slot;
+  if (warp == kBwdCtl) {
     if (lane == 0) {
       const int row0 = b * S;
       mbar_arrive_tx(ld_full, 32768u + uint32_t(S) * 256u);
@@ -366,7 +380,20 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
       mbar_wait(ld_full, 0);
       tc_fence_after();
       const uint32_t q = smem_u32(sQ), g = smem_u32(sdO), k = smem_u32(sK), v = smem_u32(sV), ds = smem_u32(sdS);
-      auto issue_s = [&](int kt) {
+      auto issue_dq = [&](int kt) {  // dQ += dS_kt K_kt: A = dS (K-major), B = K rows of the tile (MN-major)
+        mbar_wait(&ds_full[kt & 1], (kt >> 1) & 1);
+        tc_fence_after();
+        const uint32_t dsb = ds + uint32_t(kt & 1) * 32768u;
+        for (int kk = 0; kk < 128; kk += 16)
+          tc_mma(tmem + 256, smem_desc(dsb + (kk >> 6) * 16384 + ((kk & 63) >> 4) * 32, 16, 1024),
+                 smem_desc(k + uint32_t(kt * 128 + kk) * 128, 8192, 1024), kIdN64MN, (kt > 0 || kk > 0) ? 1u : 0u);
+        tc_commit(&dq_done[kt & 1]);
+      };
+      for (int kt = 0; kt < nkt; ++kt) {
+        if (kt > 0) {
+          mbar_wait(s_free, (kt - 1) & 1);  // S, dP of tile kt-1 are in registers
+          tc_fence_after();
+        }
 #pragma unroll
         for (int kk = 0; kk < 4; ++kk) {
           tc_mma(tmem, smem_desc(q + kk * 32, 16, 1024), smem_desc(k + kt * 16384 + kk * 32, 16, 1024), kIdN128,
@@ -375,89 +402,90 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
                  kIdN128, kk > 0 ? 1u : 0u);
         }
         tc_commit(s_full);
-      };
-      issue_s(0);
-      for (int kt = 0; kt < nkt; ++kt) {
-        mbar_wait(ds_full, kt & 1);
-        tc_fence_after();
-        // dQ += dS K_kt: A = dS (K-major, 2 blocks of 64 keys), B = K rows of this tile (MN-major)
-        for (int kk = 0; kk < 128; kk += 16)
-          tc_mma(tmem + 256, smem_desc(ds + (kk >> 6) * 16384 + ((kk & 63) >> 4) * 32, 16, 1024),
-                 smem_desc(k + uint32_t(kt * 128 + kk) * 128, 8192, 1024), kIdN64MN, (kt > 0 || kk > 0) ? 1u : 0u);
-        tc_commit(dq_done);
-        if (kt + 1 < nkt) issue_s(kt + 1);
+        if (kt > 0) issue_dq(kt - 1);
       }
+      issue_dq(nkt - 1);
     }
   } else {
-    const int i = warp * 32 + lane;
+    const int qw = warp & 3, cg = warp >> 2;  // TMEM lane quarter, 32-column group
+    const int i = qw * 32 + lane;
     const int q = qt * 128 + i;
     const int64_t hrow = (int64_t(b) * p.heads + a) * S + q;
-    const uint32_t trow = tmem + (uint32_t(warp * 32) << 16);
-    // D_q = dO_q . O_q (fp32 over the bf16 row)
-    float D = 0.f;
+    const uint32_t trow = tmem + (uint32_t(qw * 32) << 16);
+    // D_q = dO_q . O_q in fp32 over the bf16 row: group cg sums dims [16cg, 16cg+16), the four
+    // partials meet in the (still unused) second dS buffer.  Nothing writes that buffer before
+    // tile 1, which needs every thread's s_free arrival of tile 0, i.e. after these reads.
+    float* red = reinterpret_cast<float*>(sdS + 32768);
     {
-      const bf16* orow = p.o + (int64_t(b) * S + q) * p.ld + a * 64;
-      const bf16* grow = p.dout + (int64_t(b) * S + q) * p.ld + a * 64;
+      const __nv_bfloat162* xa = reinterpret_cast<const __nv_bfloat162*>(&x0);
+      const __nv_bfloat162* xb = reinterpret_cast<const __nv_bfloat162*>(&x1);
+      const __nv_bfloat162* ya = reinterpret_cast<const __nv_bfloat162*>(&y0);
+      const __nv_bfloat162* yb = reinterpret_cast<const __nv_bfloat162*>(&y1);
+      float part = 0.f;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        const uint4 x = *reinterpret_cast<const uint4*>(orow + 8 * j);
-        const uint4 y = *reinterpret_cast<const uint4*>(grow + 8 * j);
-        const __nv_bfloat162* x2 = reinterpret_cast<const __nv_bfloat162*>(&x);
-        const __nv_bfloat162* y2 = reinterpret_cast<const __nv_bfloat162*>(&y);
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-          const float2 u = __bfloat1622float2(x2[e]), w = __bfloat1622float2(y2[e]);
-          D += u.x * w.x + u.y * w.y;
-        }
+      for (int e = 0; e < 4; ++e) {
+        const float2 u = __bfloat1622float2(xa[e]), w = __bfloat1622float2(ya[e]);
+        part += u.x * w.x + u.y * w.y;
       }
-      p.D[hrow] = D;
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float2 u = __bfloat1622float2(xb[e]), w = __bfloat1622float2(yb[e]);
+        part += u.x * w.x + u.y * w.y;
+      }
+      red[cg * 128 + i] = part;
     }
+    named_sync(2, 32 * kBwdCW);
+    const float D = (red[i] + red[128 + i]) + (red[256 + i] + red[384 + i]);
+    if (cg == 0) p.D[hrow] = D;
     const float l2 = p.lse[hrow] * kLog2e;
     const uint32_t* mrow = p.mask + hrow * (S / 32);
     const uint32_t ds = smem_u32(sdS);
     for (int kt = 0; kt < nkt; ++kt) {
-      // this key tile's 4 keep words of the row, fetched before waiting for the products
-      uint4 mw = make_uint4(~0u, ~0u, ~0u, ~0u);
-      if (p.drop) mw = *reinterpret_cast<const uint4*>(mrow + kt * 4);
+      // this key tile's keep word of the row for the group's 32 keys, fetched before waiting
+      const uint32_t bits = p.drop ? mrow[kt * 4 + cg] : ~0u;
       mbar_wait(s_full, kt & 1);
-      if (kt > 0) mbar_wait(dq_done, (kt - 1) & 1);  // dS buffer free
       tc_fence_after();
+      uint32_t rs[32], rp[32];
+      tmem_ld32_nw(trow + uint32_t(cg * 32), rs);
+      tmem_ld32_nw(trow + uint32_t(128 + cg * 32), rp);
+      tmem_wait_ld();
+      tc_fence_before();
+      mbar_arrive(s_free);
 #pragma unroll
-      for (int c = 0; c < 128; c += 32) {
-        uint32_t rs[32], rp[32];
-        tmem_ld32(trow + uint32_t(c), rs);
-        tmem_ld32(trow + uint32_t(128 + c), rp);
-        const uint32_t bits = c == 0 ? mw.x : c == 32 ? mw.y : c == 64 ? mw.z : mw.w;
-#pragma unroll
-        for (int j = 0; j < 32; ++j) {
-          const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
-          const float dp = ((bits >> j) & 1u) ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
-          rs[j] = __float_as_uint(pr * (dp - D));
-        }
-        st_row32(ds, i, c, reinterpret_cast<const float*>(rs));
+      for (int j = 0; j < 32; ++j) {
+        const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
+        const float dp = ((bits >> j) & 1u) ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
+        rs[j] = __float_as_uint(pr * (dp - D));
       }
+      if (kt >= 2) mbar_wait(&dq_done[kt & 1], ((kt - 2) >> 1) & 1);  // dS buffer kt&1 free
+      st_row32(ds + uint32_t(kt & 1) * 32768u, i, cg * 32, reinterpret_cast<const float*>(rs));
       fence_async_smem();
       tc_fence_before();
-      mbar_arrive(ds_full);
+      mbar_arrive(&ds_full[kt & 1]);
     }
-    mbar_wait(dq_done, (nkt - 1) & 1);
+    mbar_wait(&dq_done[(nkt - 1) & 1], ((nkt - 1) >> 1) & 1);
     tc_fence_after();
-    uint32_t r0[32], r1[32];
-    tmem_ld32(trow + 256u, r0);
-    tmem_ld32(trow + 288u, r1);
-    if (p.dq) store_row64(static_cast<bf16*>(p.dq) + (int64_t(b) * S + q) * p.ld + a * 64, r0, r1, p.alpha, p.acc_q);
+    if (cg < 2) {
+      uint32_t r0[32];
+      tmem_ld32(trow + 256u + uint32_t(cg * 32), r0);
+      if (p.dq)
+        store_row32(static_cast<bf16*>(p.dq) + (int64_t(b) * S + q) * p.ld + a * 64 + cg * 32, r0, p.alpha, p.acc_q);
+    }
   }
   __syncwarp();
   tc_fence_before();
   __syncthreads();
-  if (warp == 4) {
+  if (warp == kBwdCtl) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
   }
 }
 
-// dK, dV for 128 keys of one (sample, head); loops over query tiles (double-buffered Q, dO).
-// smem: K 16K | V 16K | Q/dO 2 x 32K | Pd^T 32K | dS^T 32K | lse, D (seq floats each) | barriers
+// dK, dV for 128 keys of one (sample, head); loops over 128-query tiles (double-buffered Q, dO).
+// P_d (dropped, scaled P) and dS are written query-major ([query][key] rows, SW128), which is
+// the MN-major layout of the A operands P_d^T and dS^T of dV += P_d^T dO and dK += dS^T Q.
+// smem: K 16K | V 16K | Q 2 x 16K | dO 2 x 16K | P_d 2 x 32K | dS 2 x 32K | barriers
+// TMEM: S 0..127, dP 128..255 (lanes = queries), dV 256..319, dK 320..383 (lanes = keys)
 __global__ void __launch_bounds__(kBwdThreads, 1)
     fa5_bwd_dkv(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mdO,
                 const __grid_constant__ CUtensorMap mK, const __grid_constant__ CUtensorMap mV, const Fa5B p) {
@@ -466,33 +494,30 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
   const int S = p.seq, nqt = S / 128;
   uint8_t* sK = smem;
   uint8_t* sV = smem + 16384;
-  uint8_t* sQ[2] = {smem + 32768, smem + 65536};
-  uint8_t* sG[2] = {smem + 49152, smem + 81920};
-  uint8_t* sPd = smem + 98304;
-  uint8_t* sdS = smem + 131072;
-  float* s_l2 = reinterpret_cast<float*>(smem + 163840);
-  float* s_D = s_l2 + S;
-  uint32_t* s_mask = reinterpret_cast<uint32_t*>(s_D + S);  // [128 queries][4 words of this key tile]
-  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 163840 + 8 * S + 2048);
-  uint64_t *ld_kv = bar, *qd_full = bar + 1, *s_full = bar + 3, *ps_full = bar + 4, *acc_done = bar + 5;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 6);
+  uint8_t* sQ = smem + 32768;    // two 16 KB buffers
+  uint8_t* sG = smem + 65536;    // two 16 KB buffers
+  uint8_t* sPd = smem + 98304;   // two 32 KB buffers
+  uint8_t* sdS = smem + 163840;  // two 32 KB buffers
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 229376);
+  uint64_t *ld_kv = bar, *qd_full = bar + 1 /*[2]*/, *s_full = bar + 3, *s_free = bar + 4, *ps_full = bar + 5 /*[2]*/,
+           *acc_done = bar + 7 /*[2]*/;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 9);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int kt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
   const int64_t hbase = (int64_t(b) * p.heads + a) * S;
-  for (int t = threadIdx.x; t < S; t += blockDim.x) {
-    s_l2[t] = p.lse[hbase + t] * kLog2e;
-    s_D[t] = p.D[hbase + t];
-  }
   if (threadIdx.x == 0) {
     mbar_init(ld_kv, 1);
     mbar_init(&qd_full[0], 1);
     mbar_init(&qd_full[1], 1);
     mbar_init(s_full, 1);
-    mbar_init(ps_full, 128);
-    mbar_init(acc_done, 1);
+    mbar_init(s_free, 32 * kBwdCW);
+    mbar_init(&ps_full[0], 32 * kBwdCW);
+    mbar_init(&ps_full[1], 32 * kBwdCW);
+    mbar_init(&acc_done[0], 1);
+    mbar_init(&acc_done[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == 4) {
+  if (warp == kBwdCtl) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(512));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -500,8 +525,8 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
-  const uint32_t tmem = *tmem_slot;  // S^T 0..127, dP^T 128..255, dV 256..319, dK 320..383
-  if (warp == 4) {
+  const uint32_t tmem = *tmem_slot;
+  if (warp == kBwdCtl) {
     if (lane == 0) {
       const int row0 = b * S;
       mbar_arrive_tx(ld_kv, 32768u);
@@ -509,100 +534,112 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
       tma_load(sV, &mV, ld_kv, a * 64, row0 + kt * 128, 0, 0);
       auto load_qd = [&](int t) {
         mbar_arrive_tx(&qd_full[t & 1], 32768u);
-        tma_load(sQ[t & 1], &mQ, &qd_full[t & 1], a * 64, row0 + t * 128, 0, 0);
-        tma_load(sG[t & 1], &mdO, &qd_full[t & 1], a * 64, row0 + t * 128, 0, 0);
+        tma_load(sQ + (t & 1) * 16384, &mQ, &qd_full[t & 1], a * 64, row0 + t * 128, 0, 0);
+        tma_load(sG + (t & 1) * 16384, &mdO, &qd_full[t & 1], a * 64, row0 + t * 128, 0, 0);
       };
       load_qd(0);
       if (nqt > 1) load_qd(1);
-      const uint32_t k = smem_u32(sK), v = smem_u32(sV), pd = smem_u32(sPd), ds = smem_u32(sdS);
-      auto issue_s = [&](int t) {
+      const uint32_t k = smem_u32(sK), v = smem_u32(sV);
+      // dV += P_d^T dO_t, dK += dS^T Q_t: A MN-major (keys contiguous, 64-key blocks 16 KB apart,
+      // K step of 16 queries = 2 KB), B = dO / Q tile rows (MN-major)
+      constexpr uint32_t idAcc = kIdN64MN | (1u << 15);
+      auto issue_acc = [&](int t) {
+        mbar_wait(&ps_full[t & 1], (t >> 1) & 1);
+        tc_fence_after();
+        const uint32_t pd = smem_u32(sPd) + uint32_t(t & 1) * 32768u, ds = smem_u32(sdS) + uint32_t(t & 1) * 32768u;
+        const uint32_t q = smem_u32(sQ) + uint32_t(t & 1) * 16384u, g = smem_u32(sG) + uint32_t(t & 1) * 16384u;
+        for (int kq = 0; kq < 128; kq += 16) {
+          const uint32_t acc = (t > 0 || kq > 0) ? 1u : 0u;
+          tc_mma(tmem + 256, smem_desc(pd + uint32_t(kq) * 128, 16384, 1024),
+                 smem_desc(g + uint32_t(kq) * 128, 8192, 1024), idAcc, acc);
+          tc_mma(tmem + 320, smem_desc(ds + uint32_t(kq) * 128, 16384, 1024),
+                 smem_desc(q + uint32_t(kq) * 128, 8192, 1024), idAcc, acc);
+        }
+        tc_commit(&acc_done[t & 1]);
+      };
+      mbar_wait(ld_kv, 0);
+      for (int t = 0; t < nqt; ++t) {
+        if (t > 0) mbar_wait(s_free, (t - 1) & 1);  // S, dP of tile t-1 are in registers
         mbar_wait(&qd_full[t & 1], (t >> 1) & 1);
         tc_fence_after();
-        const uint32_t q = smem_u32(sQ[t & 1]), g = smem_u32(sG[t & 1]);
+        const uint32_t q = smem_u32(sQ) + uint32_t(t & 1) * 16384u, g = smem_u32(sG) + uint32_t(t & 1) * 16384u;
+        // S = Q_t K^T, dP = dO_t V^T (M = 128 queries, N = 128 keys)
 #pragma unroll
         for (int kk = 0; kk < 4; ++kk) {
-          tc_mma(tmem, smem_desc(k + kk * 32, 16, 1024), smem_desc(q + kk * 32, 16, 1024), kIdN128, kk > 0 ? 1u : 0u);
-          tc_mma(tmem + 128, smem_desc(v + kk * 32, 16, 1024), smem_desc(g + kk * 32, 16, 1024), kIdN128,
+          tc_mma(tmem, smem_desc(q + kk * 32, 16, 1024), smem_desc(k + kk * 32, 16, 1024), kIdN128, kk > 0 ? 1u : 0u);
+          tc_mma(tmem + 128, smem_desc(g + kk * 32, 16, 1024), smem_desc(v + kk * 32, 16, 1024), kIdN128,
                  kk > 0 ? 1u : 0u);
         }
         tc_commit(s_full);
-      };
-      mbar_wait(ld_kv, 0);
-      issue_s(0);
-      for (int t = 0; t < nqt; ++t) {
-        mbar_wait(ps_full, t & 1);
-        tc_fence_after();
-        const uint32_t q = smem_u32(sQ[t & 1]), g = smem_u32(sG[t & 1]);
-        // dV += Pd^T dO_t, dK += dS^T Q_t: A K-major over the tile's queries, B = dO / Q rows (MN-major)
-        for (int kq = 0; kq < 128; kq += 16) {
-          const uint32_t aoff = (kq >> 6) * 16384 + ((kq & 63) >> 4) * 32;
-          const uint32_t acc = (t > 0 || kq > 0) ? 1u : 0u;
-          tc_mma(tmem + 256, smem_desc(pd + aoff, 16, 1024), smem_desc(g + uint32_t(kq) * 128, 8192, 1024), kIdN64MN,
-                 acc);
-          tc_mma(tmem + 320, smem_desc(ds + aoff, 16, 1024), smem_desc(q + uint32_t(kq) * 128, 8192, 1024), kIdN64MN,
-                 acc);
-        }
-        tc_commit(acc_done);
-        if (t + 1 < nqt) issue_s(t + 1);
-        if (t + 2 < nqt) {
-          mbar_wait(acc_done, t & 1);  // the products that read buffer t & 1 are done
-          load_qd(t + 2);
+        if (t > 0) {
+          issue_acc(t - 1);
+          if (t + 1 < nqt) {
+            mbar_wait(&acc_done[(t - 1) & 1], ((t - 1) >> 1) & 1);  // Q/dO buffer (t+1)&1 is free
+            load_qd(t + 1);
+          }
         }
       }
+      issue_acc(nqt - 1);
     }
   } else {
-    const int i = warp * 32 + lane;
-    const int key = kt * 128 + i;
-    const uint32_t trow = tmem + (uint32_t(warp * 32) << 16);
-    const uint32_t pd = smem_u32(sPd), ds = smem_u32(sdS);
-    const int kb = key & 31, kw = i >> 5;
+    const int qw = warp & 3, cg = warp >> 2;  // TMEM lane quarter, 32-key group
+    const int i = qw * 32 + lane;
+    const uint32_t trow = tmem + (uint32_t(qw * 32) << 16);
+    // row constants of query tile t (lse, D, keep word), prefetched one tile ahead
+    auto row_consts = [&](int t, float& l2, float& D, uint32_t& bits) {
+      const int64_t hrow = hbase + t * 128 + i;
+      l2 = p.lse[hrow] * kLog2e;
+      D = p.D[hrow];
+      bits = p.drop ? p.mask[hrow * (S / 32) + kt * 4 + cg] : ~0u;
+    };
+    float nl2, nD;
+    uint32_t nbits;
+    row_consts(0, nl2, nD, nbits);
     for (int t = 0; t < nqt; ++t) {
-      // stage this query tile's keep words for the key tile (query i's 4 words, one 16-byte load)
-      uint4 mw = make_uint4(~0u, ~0u, ~0u, ~0u);
-      if (p.drop) mw = *reinterpret_cast<const uint4*>(p.mask + (hbase + t * 128 + i) * (S / 32) + kt * 4);
-      named_sync(2, 128);  // previous tile's readers are done with s_mask
-      *reinterpret_cast<uint4*>(s_mask + i * 4) = mw;
-      named_sync(2, 128);
+      const float l2 = nl2, D = nD;
+      const uint32_t bits = nbits;
+      if (t + 1 < nqt) row_consts(t + 1, nl2, nD, nbits);
       mbar_wait(s_full, t & 1);
-      if (t > 0) mbar_wait(acc_done, (t - 1) & 1);  // Pd^T / dS^T buffers free
       tc_fence_after();
-#pragma unroll 1
-      for (int c = 0; c < 128; c += 16) {
-        uint32_t rs[16], rp[16];
-        tmem_ld16(trow + uint32_t(c), rs);
-        tmem_ld16(trow + uint32_t(128 + c), rp);
-        // in place: rp <- Pd^T, rs <- dS^T (fp32 bits)
+      uint32_t rs[32], rp[32];
+      tmem_ld32_nw(trow + uint32_t(cg * 32), rs);
+      tmem_ld32_nw(trow + uint32_t(128 + cg * 32), rp);
+      tmem_wait_ld();
+      tc_fence_before();
+      mbar_arrive(s_free);
+      // in place: rp <- P_d, rs <- dS (fp32 bits)
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const int qq = t * 128 + c + j;
-          const bool keep = (s_mask[(c + j) * 4 + kw] >> kb) & 1u;
-          const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - s_l2[qq]);
-          const float dp = keep ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
-          rp[j] = __float_as_uint(keep ? pr * p.keep_scale : 0.f);
-          rs[j] = __float_as_uint(pr * (dp - s_D[qq]));
-        }
-        st_row16(pd, i, c, reinterpret_cast<const float*>(rp));
-        st_row16(ds, i, c, reinterpret_cast<const float*>(rs));
+      for (int j = 0; j < 32; ++j) {
+        const bool keep = (bits >> j) & 1u;
+        const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
+        const float dp = keep ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
+        rp[j] = __float_as_uint(keep ? pr * p.keep_scale : 0.f);
+        rs[j] = __float_as_uint(pr * (dp - D));
       }
+      if (t >= 2) mbar_wait(&acc_done[t & 1], ((t - 2) >> 1) & 1);  // P_d / dS buffers t&1 free
+      st_row32(smem_u32(sPd) + uint32_t(t & 1) * 32768u, i, cg * 32, reinterpret_cast<const float*>(rp));
+      st_row32(smem_u32(sdS) + uint32_t(t & 1) * 32768u, i, cg * 32, reinterpret_cast<const float*>(rs));
       fence_async_smem();
       tc_fence_before();
-      mbar_arrive(ps_full);
+      mbar_arrive(&ps_full[t & 1]);
     }
-    mbar_wait(acc_done, (nqt - 1) & 1);
+    mbar_wait(&acc_done[(nqt - 1) & 1], ((nqt - 1) >> 1) & 1);
     tc_fence_after();
-    const int64_t off = (int64_t(b) * S + key) * p.ld + a * 64;
-    uint32_t r0[32], r1[32];
-    tmem_ld32(trow + 256u, r0);
-    tmem_ld32(trow + 288u, r1);
-    if (p.dv) store_row64(static_cast<bf16*>(p.dv) + off, r0, r1, 1.f, p.acc_v);
-    tmem_ld32(trow + 320u, r0);
-    tmem_ld32(trow + 352u, r1);
-    if (p.dk) store_row64(static_cast<bf16*>(p.dk) + off, r0, r1, p.alpha, p.acc_k);
+    // accumulator lanes are keys: group 0/1 store dV columns 0-31 / 32-63, group 2/3 dK
+    const int key = kt * 128 + i;
+    const int64_t off = (int64_t(b) * S + key) * p.ld + a * 64 + (cg & 1) * 32;
+    uint32_t r0[32];
+    tmem_ld32(trow + 256u + uint32_t(cg * 32), r0);
+    if (cg < 2) {
+      if (p.dv) store_row32(static_cast<bf16*>(p.dv) + off, r0, 1.f, p.acc_v);
+    } else {
+      if (p.dk) store_row32(static_cast<bf16*>(p.dk) + off, r0, p.alpha, p.acc_k);
+    }
   }
   __syncwarp();
   tc_fence_before();
   __syncthreads();
-  if (warp == 4) {
+  if (warp == kBwdCtl) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
   }
@@ -697,12 +734,12 @@ bool attention_bwd_tc5(const AttnArgs& A, cudaStream_t st) {
   p.acc_q = A.acc_q;
   p.acc_k = A.acc_k;
   p.acc_v = A.acc_v;
-  const int smem_q = 32768 + 2 * A.seq * 128 + 32768 + 256 + 1024;
-  const int smem_kv = 163840 + 8 * A.seq + 2048 + 256 + 1024;
+  const int smem_q = 32768 + 2 * A.seq * 128 + 65536 + 256 + 1024;
+  const int smem_kv = 229376 + 256 + 1024;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(fa5_bwd_dq, cudaFuncAttributeMaxDynamicSharedMemorySize, 32768 + 2 * 512 * 128 + 32768 + 1280);
-    cudaFuncSetAttribute(fa5_bwd_dkv, cudaFuncAttributeMaxDynamicSharedMemorySize, 163840 + 8 * 512 + 2048 + 1280);
+    cudaFuncSetAttribute(fa5_bwd_dq, cudaFuncAttributeMaxDynamicSharedMemorySize, 32768 + 2 * 512 * 128 + 65536 + 1280);
+    cudaFuncSetAttribute(fa5_bwd_dkv, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_kv);
     attr = true;
   }
   fa5_bwd_dq<<<dim3(A.seq / 128, A.heads, A.nb), kBwdThreads, smem_q, st>>>(mq, mg, mk, mv, p);
