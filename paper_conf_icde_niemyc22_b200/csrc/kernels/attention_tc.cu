@@ -29,13 +29,6 @@ namespace {
 
 using namespace tc;
 
-constexpr int kSoftWarps = 16;  // four per TMEM lane quarter, each owning a quarter of the keys
-constexpr int kGroups = kSoftWarps / 4;
-constexpr int kCtlWarp = kSoftWarps;
-constexpr int kThreads = 32 * (kSoftWarps + 1);
-constexpr int kRegion = 64 * 1024;
-constexpr int kSmem = 3 * kRegion + 5120 + 1024;  // PB(+Q) | K(=PA) | V | barriers + exchange (+align)
-
 constexpr float kLog2e = 1.4426950408889634f;
 constexpr float kLn2 = 0.6931471805599453f;
 
@@ -63,184 +56,7 @@ struct Fa5P {
   void* c;
   float* lse;
   uint32_t* mask;
-  int kbox;           // rows per K/V TMA box
 };
-
-__global__ void __launch_bounds__(kThreads, 1)
-    fa5_fwd(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mK,
-            const __grid_constant__ CUtensorMap mV, const Fa5P p) {
-  extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint8_t* rPB = smem;              // P keys [seq/2, seq); Q tile at its start until S is done
-  uint8_t* rK = smem + kRegion;     // K; then P keys [0, seq/2)
-  uint8_t* rV = smem + 2 * kRegion;
-  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 3 * kRegion);
-  uint64_t *qk_full = bar, *v_full = bar + 1, *s_full = bar + 2, *p_full = bar + 3, *o_full = bar + 5;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 6);
-  float* red_m = reinterpret_cast<float*>(smem + 3 * kRegion + 256);
-  float* red_l = red_m + 128 * kGroups;
-
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int qt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
-  const int S = p.seq, half = S / 2;
-  if (threadIdx.x == 0) {
-    mbar_init(qk_full, 1);
-    mbar_init(v_full, 1);
-    mbar_init(s_full, 1);
-    mbar_init(&p_full[0], 128 * kGroups / 2);
-    mbar_init(&p_full[1], 128 * kGroups / 2);
-    mbar_init(o_full, 1);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  if (warp == kCtlWarp) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                 "r"(512));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
-  }
-  tc_fence_before();
-  __syncthreads();
-  tc_fence_after();
-  const uint32_t tmem = *tmem_slot;
-
-  if (warp == kCtlWarp) {
-    if (lane == 0) {
-      const int row0 = b * S;
-      mbar_arrive_tx(qk_full, 128 * 128 + uint32_t(S) * 128);
-      tma_load(rPB, &mQ, qk_full, a * 64, row0 + qt * 128, 0, 0);
-      for (int j = 0; j < S; j += p.kbox) tma_load(rK + j * 128, &mK, qk_full, a * 64, row0 + j, 0, 0);
-      mbar_arrive_tx(v_full, uint32_t(S) * 128);
-      for (int j = 0; j < S; j += p.kbox) tma_load(rV + j * 128, &mV, v_full, a * 64, row0 + j, 0, 0);
-      // S = Q K^T: M 128, N 128 per instruction, K = 64 (4 steps of 16)
-      constexpr uint32_t idS = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(128 >> 3) << 17) |
-                               (uint32_t(128 >> 4) << 24);
-      mbar_wait(qk_full, 0);
-      tc_fence_after();
-      const uint32_t sq = smem_u32(rPB), sk = smem_u32(rK);
-      for (int c = 0; c < S / 128; ++c)
-#pragma unroll
-        for (int k = 0; k < 4; ++k)
-          tc_mma(tmem + uint32_t(c * 128), smem_desc(sq + k * 32, 16, 1024),
-                 smem_desc(sk + c * 16384 + k * 32, 16, 1024), idS, k > 0 ? 1u : 0u);
-      tc_commit(s_full);
-      // O = P V: M 128, N 64, K 16 per instruction; A = P (K-major), B = V (MN-major)
-      constexpr uint32_t idO = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | (uint32_t(64 >> 3) << 17) |
-                               (uint32_t(128 >> 4) << 24);
-      mbar_wait(v_full, 0);
-      const uint32_t sv = smem_u32(rV);
-      for (int h = 0; h < 2; ++h) {
-        mbar_wait(&p_full[h], 0);
-        tc_fence_after();
-        const uint32_t sp = smem_u32(h == 0 ? rK : rPB);
-        for (int kk = 0; kk < half; kk += 16) {
-          const uint32_t ad = sp + (kk >> 6) * 16384 + ((kk & 63) >> 4) * 32;
-          const uint32_t bd = sv + uint32_t(h * half + kk) * 128;
-          tc_mma(tmem, smem_desc(ad, 16, 1024), smem_desc(bd, 8192, 1024), idO, (h > 0 || kk > 0) ? 1u : 0u);
-        }
-      }
-      tc_commit(o_full);
-    }
-  } else {
-    // ===== softmax warps: row i, key group g (S / kGroups keys) =====
-    const int qq = warp & 3, g = warp >> 2;
-    const int i = qq * 32 + lane;
-    const uint32_t trow = tmem + (uint32_t(qq * 32) << 16);
-    const int gw = S / kGroups;
-    const int c0 = g * gw;
-    const int hf = c0 / half;  // which P half (MMA batch) this group fills
-    mbar_wait(s_full, 0);
-    tc_fence_after();
-    float m = -INFINITY;
-    for (int c = c0; c < c0 + gw; c += 32) {
-      uint32_t r[32];
-      tmem_ld32(trow + uint32_t(c), r);
-#pragma unroll
-      for (int j = 0; j < 32; ++j) m = fmaxf(m, __uint_as_float(r[j]));
-    }
-    red_m[g * 128 + i] = m;
-    named_sync(1, 32 * kSoftWarps);
-#pragma unroll
-    for (int gg = 0; gg < kGroups; ++gg) m = fmaxf(m, red_m[gg * 128 + i]);
-    m *= p.sl2;
-    const uint64_t erow = ((uint64_t(p.b0 + b) * p.heads + a) * uint64_t(S) + uint64_t(qt * 128 + i)) * uint64_t(S);
-    const int64_t mrow = ((int64_t(b) * p.heads + a) * S + qt * 128 + i) * (S / 32);
-    float l = 0.f;
-    const uint32_t sp = smem_u32(hf == 0 ? rK : rPB);
-    for (int c = c0; c < c0 + gw; c += 32) {
-      uint32_t r[32];
-      tmem_ld32(trow + uint32_t(c), r);
-      float v[32];
-#pragma unroll
-      for (int j = 0; j < 32; ++j) {
-        v[j] = ex2(__uint_as_float(r[j]) * p.sl2 - m);
-        l += v[j];
-      }
-      uint32_t bits = 0xFFFFFFFFu;
-      if (p.p > 0.f) {
-        bits = 0u;
-#pragma unroll
-        for (int u = 0; u < 8; ++u) {
-          const uint64_t cnt = (erow + uint64_t(c + 4 * u)) >> 2;
-          const uint4 w = philox4x32_10(uint32_t(cnt), uint32_t(cnt >> 32), p.step, 0u, p.seed, kPhiloxKey1);
-          bits |= (uint32_t(w.x >= p.thr) | (uint32_t(w.y >= p.thr) << 1) | (uint32_t(w.z >= p.thr) << 2) |
-                   (uint32_t(w.w >= p.thr) << 3))
-                  << (4 * u);
-        }
-#pragma unroll
-        for (int j = 0; j < 32; ++j)
-          if (!((bits >> j) & 1u)) v[j] = 0.f;
-      }
-      if (p.mask) p.mask[mrow + (c >> 5)] = bits;
-      // 32 keys = 4 sixteen-byte chunks of row i in the K-major SW128 layout
-      const int kl = c - hf * half;  // key within this half
-      const uint32_t blk = sp + uint32_t(kl >> 6) * 16384u + uint32_t(i) * 128u;
-#pragma unroll
-      for (int q4 = 0; q4 < 4; ++q4) {
-        const int chunk = ((kl & 63) >> 3) + q4;
-        sts128(blk + (uint32_t(chunk ^ (i & 7)) << 4), pk2(v[8 * q4], v[8 * q4 + 1]), pk2(v[8 * q4 + 2], v[8 * q4 + 3]),
-               pk2(v[8 * q4 + 4], v[8 * q4 + 5]), pk2(v[8 * q4 + 6], v[8 * q4 + 7]));
-      }
-    }
-    fence_async_smem();
-    tc_fence_before();
-    mbar_arrive(&p_full[hf]);
-    red_l[g * 128 + i] = l;
-    named_sync(1, 32 * kSoftWarps);
-    if (g == 0) {
-      l = 0.f;
-#pragma unroll
-      for (int gg = 0; gg < kGroups; ++gg) l += red_l[gg * 128 + i];
-      mbar_wait(o_full, 0);
-      tc_fence_after();
-      const float inv = p.keep_scale / l;
-      const int q = qt * 128 + i;
-      bf16* crow = static_cast<bf16*>(p.c) + (int64_t(b) * S + q) * p.ld + a * 64;
-#pragma unroll
-      for (int h = 0; h < 2; ++h) {
-        uint32_t r[32];
-        tmem_ld32(trow + uint32_t(h * 32), r);
-        if (p.c) {
-#pragma unroll
-          for (int j = 0; j < 4; ++j) {
-            uint4 o;
-            o.x = pk2(__uint_as_float(r[8 * j]) * inv, __uint_as_float(r[8 * j + 1]) * inv);
-            o.y = pk2(__uint_as_float(r[8 * j + 2]) * inv, __uint_as_float(r[8 * j + 3]) * inv);
-            o.z = pk2(__uint_as_float(r[8 * j + 4]) * inv, __uint_as_float(r[8 * j + 5]) * inv);
-            o.w = pk2(__uint_as_float(r[8 * j + 6]) * inv, __uint_as_float(r[8 * j + 7]) * inv);
-            *reinterpret_cast<uint4*>(crow + h * 32 + 8 * j) = o;
-          }
-        }
-      }
-      if (p.lse) p.lse[(int64_t(b) * p.heads + a) * S + q] = (m + log2f(l)) * kLn2;
-    }
-  }
-  __syncwarp();
-  tc_fence_before();
-  __syncthreads();
-  if (warp == kCtlWarp) {
-    tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
-  }
-}
 
 // ======================================================================= backward
 // Shared by both backward kernels: 128 row threads (TMEM lane i = thread i), one control
@@ -645,6 +461,298 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
   }
 }
 
+// ======================================================================= forward
+// Persistent, warp-specialised forward.  A work item is a pair of 128-query tiles of one
+// (sample, head); K and V stream through a 4-stage TMA ring in 64-key chunks, so any seq
+// that is a multiple of 128 works.  Per tile t of the pair, two softmax warpgroups (key
+// halves h = 0, 1 of every chunk) run an online softmax over the chunks: S_t = Q_t K_j^T
+// lands in one of two TMEM buffers (lanes = queries), so the tensor core computes chunk j+1
+// while the softmax warps work on chunk j; a thread owns one row and 32 keys of the chunk,
+// copies them to registers and releases the buffer at once.  The chunk max is exchanged
+// between the halves through shared memory; the running max only moves when it grows by
+// more than 8 (log2 units) — then the warp rescales its half of the O_t rows in TMEM after
+// the previous P V product has landed — otherwise the stale max is kept (exponentials
+// stay <= 2^8; exact after the final 1/l).  P (dropout applied: Philox keep bits, one call
+// per four keys of a row, reading D-RNG) goes to shared memory in the K-major SW128 layout and
+// O_t += P V_j runs on the tensor cores.  One thread issues TMA, one issues tcgen05.mma;
+// the next item's Q and the next chunks' K / V load while the current item computes.
+//   TMEM: S_0 [0,64) [64,128)  S_1 [128,192) [192,256)  O_0 [256,320)  O_1 [320,384)
+//   smem: Q 2 x 16K | K,V ring 4 x 16K | P 2 x 16K | barriers, row exchange
+constexpr int kFwdSoftWarps = 16;  // (tile t, key half h, lane quarter): warp = 8t + 4h + quarter
+constexpr int kFwdTma = kFwdSoftWarps, kFwdMma = kFwdSoftWarps + 1;
+constexpr int kFwdThreads = 32 * (kFwdSoftWarps + 2);
+constexpr int kFwdKC = 64;  // keys per chunk
+constexpr int kFwdStages = 4;
+constexpr int kFwdSmemQ = 0, kFwdSmemKV = 32768, kFwdSmemP = kFwdSmemKV + kFwdStages * 16384;
+constexpr int kFwdSmemBar = kFwdSmemP + 32768;
+constexpr int kFwdSmem = kFwdSmemBar + 512 + 6144 + 1024;  // barriers | exchange: maxima [t][h][2][128], sums [t][h][128] | align
+constexpr float kRescaleThr = 8.f;
+
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
+      "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15]), "r"(r[16]), "r"(r[17]), "r"(r[18]),
+      "r"(r[19]), "r"(r[20]), "r"(r[21]), "r"(r[22]), "r"(r[23]), "r"(r[24]), "r"(r[25]), "r"(r[26]), "r"(r[27]),
+      "r"(r[28]), "r"(r[29]), "r"(r[30]), "r"(r[31]));
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void sts32(uint32_t addr, float v) {
+  asm volatile("st.shared.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+}
+__device__ __forceinline__ float lds32(uint32_t addr) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(addr) : "memory");
+  return v;
+}
+
+__global__ void __launch_bounds__(kFwdThreads, 1)
+    fa5_fwd(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mK,
+            const __grid_constant__ CUtensorMap mV, const Fa5P p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + kFwdSmemBar);
+  uint64_t *q_full = bar, *q_empty = bar + 2, *kv_full = bar + 3, *kv_empty = bar + 3 + kFwdStages;
+  // per tile: s_full[2], s_free[2], p_full, p_free, o_full, o_free
+  uint64_t* tb = bar + 3 + 2 * kFwdStages;
+  auto s_full = [&](int t, int b) { return tb + 8 * t + b; };
+  auto s_free = [&](int t, int b) { return tb + 8 * t + 2 + b; };
+  auto p_full = [&](int t) { return tb + 8 * t + 4; };
+  auto p_free = [&](int t) { return tb + 8 * t + 5; };
+  auto o_full = [&](int t) { return tb + 8 * t + 6; };
+  auto o_free = [&](int t) { return tb + 8 * t + 7; };
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tb + 16);
+  const uint32_t xch = smem_u32(smem + kFwdSmemBar + 512);  // floats: maxima [t][h][2][128] | sums [t][h][128]
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int S = p.seq, nqt = S / 128, npair = (nqt + 1) / 2, nkc = S / kFwdKC;
+  const int items = p.nb * p.heads * npair;
+  if (threadIdx.x == 0) {
+    mbar_init(&q_full[0], 1);
+    mbar_init(&q_full[1], 1);
+    mbar_init(q_empty, 1);
+    for (int s = 0; s < kFwdStages; ++s) {
+      mbar_init(&kv_full[s], 1);
+      mbar_init(&kv_empty[s], 1);
+    }
+    for (int t = 0; t < 2; ++t) {
+      for (int b = 0; b < 2; ++b) {
+        mbar_init(s_full(t, b), 1);
+        mbar_init(s_free(t, b), 256);
+      }
+      mbar_init(p_full(t), 256);
+      mbar_init(p_free(t), 1);
+      mbar_init(o_full(t), 1);
+      mbar_init(o_free(t), 256);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == kFwdMma) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                 "r"(512));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == kFwdTma) {
+    if (lane == 0) {
+      int it = 0, kc = 0;  // items done by this CTA, K/V chunks loaded
+      for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
+        const int pair = item % npair, ah = item / npair, a = ah % p.heads, b = ah / p.heads;
+        const int row0 = b * S;
+        const int nt = min(2, nqt - 2 * pair);
+        if (it > 0) mbar_wait(q_empty, (it - 1) & 1);
+        for (int t = 0; t < nt; ++t) {
+          mbar_arrive_tx(&q_full[t], 16384u);
+          tma_load(smem + kFwdSmemQ + t * 16384, &mQ, &q_full[t], a * 64, row0 + (2 * pair + t) * 128, 0, 0);
+        }
+        for (int j = 0; j < nkc; ++j, ++kc) {
+          const int s = kc % kFwdStages;
+          if (kc >= kFwdStages) mbar_wait(&kv_empty[s], ((kc / kFwdStages) - 1) & 1);
+          uint8_t* st = smem + kFwdSmemKV + s * 16384;
+          mbar_arrive_tx(&kv_full[s], 16384u);
+          tma_load(st, &mK, &kv_full[s], a * 64, row0 + j * kFwdKC, 0, 0);
+          tma_load(st + 8192, &mV, &kv_full[s], a * 64, row0 + j * kFwdKC, 0, 0);
+        }
+      }
+    }
+  } else if (warp == kFwdMma) {
+    if (lane == 0) {
+      constexpr uint32_t idS = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(kFwdKC >> 3) << 17) |
+                               (uint32_t(128 >> 4) << 24);
+      constexpr uint32_t idO = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | (uint32_t(64 >> 3) << 17) |
+                               (uint32_t(128 >> 4) << 24);
+      int kc = 0;
+      uint32_t cs[2] = {0, 0};   // S chunks issued per tile (running: buffer cs & 1)
+      uint32_t np[2] = {0, 0};   // p_full completions consumed per tile
+      uint32_t nit[2] = {0, 0};  // items per tile (q_full / o_free phases)
+      auto issue_s = [&](int t, int s) {
+        const uint32_t c = cs[t]++, bsel = c & 1;
+        if (c >= 2) mbar_wait(s_free(t, bsel), ((c >> 1) - 1) & 1);  // the buffer's previous chunk is read
+        tc_fence_after();
+        const uint32_t q = smem_u32(smem + kFwdSmemQ + t * 16384), k = smem_u32(smem + kFwdSmemKV + s * 16384);
+#pragma unroll
+        for (int kk = 0; kk < 4; ++kk)
+          tc_mma(tmem + uint32_t(t * 128 + bsel * 64), smem_desc(q + kk * 32, 16, 1024),
+                 smem_desc(k + kk * 32, 16, 1024), idS, kk > 0 ? 1u : 0u);
+        tc_commit(s_full(t, bsel));
+      };
+      for (int item = blockIdx.x; item < items; item += gridDim.x) {
+        const int pair = item % npair;
+        const int nt = min(2, nqt - 2 * pair);
+        {
+          const int s = kc % kFwdStages;
+          mbar_wait(&kv_full[s], (kc / kFwdStages) & 1);
+          for (int t = 0; t < nt; ++t) {
+            mbar_wait(&q_full[t], nit[t] & 1);
+            issue_s(t, s);
+          }
+        }
+        for (int j = 0; j < nkc; ++j, ++kc) {
+          const int s = kc % kFwdStages;
+          const uint32_t v = smem_u32(smem + kFwdSmemKV + s * 16384 + 8192);
+          const bool more = j + 1 < nkc;
+          if (more) mbar_wait(&kv_full[(kc + 1) % kFwdStages], ((kc + 1) / kFwdStages) & 1);
+          for (int t = 0; t < nt; ++t) {
+            if (more) issue_s(t, (kc + 1) % kFwdStages);  // chunk j+1 into the other S buffer
+            mbar_wait(p_full(t), np[t] & 1);
+            ++np[t];
+            if (j == 0 && nit[t] > 0) mbar_wait(o_free(t), (nit[t] - 1) & 1);
+            tc_fence_after();
+            const uint32_t pb = smem_u32(smem + kFwdSmemP + t * 16384);
+#pragma unroll
+            for (int kk = 0; kk < kFwdKC; kk += 16)
+              tc_mma(tmem + 256 + uint32_t(t * 64), smem_desc(pb + (kk >> 4) * 32, 16, 1024),
+                     smem_desc(v + uint32_t(kk) * 128, 8192, 1024), idO, (j > 0 || kk > 0) ? 1u : 0u);
+            tc_commit(p_free(t));
+            if (!more) tc_commit(o_full(t));
+          }
+          tc_commit(&kv_empty[s]);
+        }
+        for (int t = 0; t < nt; ++t) ++nit[t];
+        tc_commit(q_empty);
+      }
+    }
+  } else {
+    // ===== softmax warps: tile t, key half h (32 keys of each chunk), row i
+    const int t = warp >> 3, h = (warp >> 2) & 1, qq = warp & 3;
+    const int i = qq * 32 + lane;
+    const uint32_t srow = tmem + (uint32_t(qq * 32) << 16) + uint32_t(t * 128 + 32 * h);
+    const uint32_t orow = tmem + (uint32_t(qq * 32) << 16) + 256u + uint32_t(t * 64 + 32 * h);
+    const uint32_t pbuf = smem_u32(smem + kFwdSmemP + t * 16384);
+    const uint32_t xm = xch + uint32_t(t * 2) * 1024u;         // [h][2][128] floats
+    const uint32_t xl = xch + 4096u + uint32_t(t) * 1024u;     // [h][128] floats
+    const int bar_id = 1 + t;                                  // named barrier of the tile's 256 threads
+    uint32_t cs = 0, npw = 0, nit = 0;  // S chunks read, P tiles written, items (this tile)
+    for (int item = blockIdx.x; item < items; item += gridDim.x) {
+      const int pair = item % npair, ah = item / npair, a = ah % p.heads, b = ah / p.heads;
+      const int nt = min(2, nqt - 2 * pair);
+      if (t >= nt) continue;
+      const int q = (2 * pair + t) * 128 + i;
+      const uint64_t erow = ((uint64_t(p.b0 + b) * p.heads + a) * uint64_t(S) + uint64_t(q)) * uint64_t(S);
+      uint32_t* mrow = p.mask ? p.mask + ((int64_t(b) * p.heads + a) * S + q) * (S / 32) : nullptr;
+      float mrun = -INFINITY, l = 0.f;
+      for (int j = 0; j < nkc; ++j, ++cs) {
+        const uint32_t bsel = cs & 1;
+        mbar_wait(s_full(t, bsel), (cs >> 1) & 1);
+        tc_fence_after();
+        uint32_t r[32];
+        tmem_ld32(srow + bsel * 64u, r);
+        tc_fence_before();
+        mbar_arrive(s_free(t, bsel));
+        // chunk max over the 64 keys (this half's 32, exchanged with the other half)
+        float m = -INFINITY;
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj) m = fmaxf(m, __uint_as_float(r[jj]));
+        sts32(xm + uint32_t((h * 2 + (j & 1)) * 128 + i) * 4u, m);
+        named_sync(bar_id, 256);
+        m = fmaxf(m, lds32(xm + uint32_t(((h ^ 1) * 2 + (j & 1)) * 128 + i) * 4u)) * p.sl2;
+        // the running max moves when it grows by more than kRescaleThr; the O_t row rescale is a
+        // warp-collective TMEM access, so the warp takes it when any of its rows needs it
+        const bool grow = m > mrun + kRescaleThr;
+        const float f = grow ? ex2(mrun - m) : 1.f;
+        l *= f;
+        if (j > 0 && __any_sync(0xffffffffu, grow)) {
+          mbar_wait(p_free(t), (npw - 1) & 1);  // P V of chunk j-1 has landed in O_t
+          tc_fence_after();
+          uint32_t o[32];
+          tmem_ld32(orow, o);
+#pragma unroll
+          for (int jj = 0; jj < 32; ++jj) o[jj] = __float_as_uint(__uint_as_float(o[jj]) * f);
+          tmem_st32(orow, o);
+          tmem_wait_st();
+        }
+        if (grow) mrun = m;
+        // P = 2^(S alpha log2e - mrun) with the keep bits, bf16 into the K-major P tile
+        const int key = j * kFwdKC + 32 * h;
+        float* v = reinterpret_cast<float*>(r);
+#pragma unroll
+        for (int jj = 0; jj < 32; ++jj) {
+          v[jj] = ex2(fmaf(v[jj], p.sl2, -mrun));
+          l += v[jj];
+        }
+        uint32_t bits = 0xFFFFFFFFu;
+        if (p.p > 0.f) {
+          bits = 0u;
+#pragma unroll
+          for (int u = 0; u < 8; ++u) {
+            const uint64_t cnt = (erow + uint64_t(key + 4 * u)) >> 2;
+            const uint4 w = philox4x32_10(uint32_t(cnt), uint32_t(cnt >> 32), p.step, 0u, p.seed, kPhiloxKey1);
+            bits |= (uint32_t(w.x >= p.thr) | (uint32_t(w.y >= p.thr) << 1) | (uint32_t(w.z >= p.thr) << 2) |
+                     (uint32_t(w.w >= p.thr) << 3))
+                    << (4 * u);
+          }
+#pragma unroll
+          for (int jj = 0; jj < 32; ++jj)
+            if (!((bits >> jj) & 1u)) v[jj] = 0.f;
+        }
+        if (mrow) mrow[key >> 5] = bits;
+        if (npw > 0) mbar_wait(p_free(t), (npw - 1) & 1);  // the previous P V has read the P tile
+        st_row32(pbuf, i, 32 * h, v);
+        ++npw;
+        fence_async_smem();
+        tc_fence_before();
+        mbar_arrive(p_full(t));
+      }
+      // epilogue: O_t row / l (keep_scale folded in), C and the log-sum-exp
+      sts32(xl + uint32_t(h * 128 + i) * 4u, l);
+      named_sync(bar_id, 256);
+      const float lt = l + lds32(xl + uint32_t((h ^ 1) * 128 + i) * 4u);
+      mbar_wait(o_full(t), nit & 1);
+      ++nit;
+      tc_fence_after();
+      uint32_t o[32];
+      tmem_ld32(orow, o);
+      tc_fence_before();
+      mbar_arrive(o_free(t));
+      const float inv = p.keep_scale / lt;
+      bf16* crow = static_cast<bf16*>(p.c) + (int64_t(b) * S + q) * p.ld + a * 64 + 32 * h;
+#pragma unroll
+      for (int jj = 0; jj < 4; ++jj) {
+        uint4 ov;
+        ov.x = pk2(__uint_as_float(o[8 * jj]) * inv, __uint_as_float(o[8 * jj + 1]) * inv);
+        ov.y = pk2(__uint_as_float(o[8 * jj + 2]) * inv, __uint_as_float(o[8 * jj + 3]) * inv);
+        ov.z = pk2(__uint_as_float(o[8 * jj + 4]) * inv, __uint_as_float(o[8 * jj + 5]) * inv);
+        ov.w = pk2(__uint_as_float(o[8 * jj + 6]) * inv, __uint_as_float(o[8 * jj + 7]) * inv);
+        *reinterpret_cast<uint4*>(crow + 8 * jj) = ov;
+      }
+      if (h == 0 && p.lse) p.lse[(int64_t(b) * p.heads + a) * S + q] = (mrun + log2f(lt)) * kLn2;
+      named_sync(bar_id, 256);  // the sum slots are reused by the next item
+    }
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  if (warp == kFwdMma) {
+    tc_fence_after();
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
+  }
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 encode() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   static std::once_flag once;
@@ -675,11 +783,11 @@ bool map2(CUtensorMap* m, const void* ptr, int64_t ld, int64_t rows, int box_row
 }  // namespace
 
 bool attention_fwd_tc5(const AttnArgs& A, cudaStream_t st) {
-  if (A.dtype != BF16 || A.d != 64 || A.seq % 128 || A.seq > 512 || A.nb < 1 || !A.c || !A.lse) return false;
+  if (A.dtype != BF16 || A.d != 64 || A.seq % 128 || A.nb < 1 || !A.c || !A.lse) return false;
   const int64_t rows = int64_t(A.nb) * A.seq;
-  const int kbox = A.seq < 256 ? A.seq : 256;
   CUtensorMap mq, mk, mv;
-  if (!map2(&mq, A.q, A.ld, rows, 128) || !map2(&mk, A.k, A.ld, rows, kbox) || !map2(&mv, A.v, A.ld, rows, kbox))
+  if (!map2(&mq, A.q, A.ld, rows, 128) || !map2(&mk, A.k, A.ld, rows, kFwdKC) ||
+      !map2(&mv, A.v, A.ld, rows, kFwdKC))
     return false;
   Fa5P p;
   p.nb = A.nb;
@@ -696,13 +804,15 @@ bool attention_fwd_tc5(const AttnArgs& A, cudaStream_t st) {
   p.c = A.c;
   p.lse = A.lse;
   p.mask = A.mask;
-  p.kbox = kbox;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(fa5_fwd, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem);
-    attr = true;
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaFuncSetAttribute(fa5_fwd, cudaFuncAttributeMaxDynamicSharedMemorySize, kFwdSmem);
   }
-  fa5_fwd<<<dim3(A.seq / 128, A.heads, A.nb), kThreads, kSmem, st>>>(mq, mk, mv, p);
+  const int items = A.nb * A.heads * ((A.seq / 128 + 1) / 2);
+  fa5_fwd<<<items < sms ? items : sms, kFwdThreads, kFwdSmem, st>>>(mq, mk, mv, p);
   return true;
 }
 

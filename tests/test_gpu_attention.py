@@ -36,7 +36,7 @@ def _inputs(nb, heads, seq, d, seed=0):
     return mk(1.0), mk(1.0), mk(1.0), mk(1.0)
 
 
-@pytest.mark.parametrize("seq", [64, 128, 192, 512])
+@pytest.mark.parametrize("seq", [64, 128, 192, 384, 512])
 @pytest.mark.parametrize("p", [0.0, 0.1])
 @pytest.mark.parametrize("path", ["tc", "mma", "simt"])
 def test_attention_kernels_vs_oracle(seq, p, path):
@@ -74,6 +74,35 @@ def test_attention_kernels_vs_oracle(seq, p, path):
     torch.cuda.synchronize()
     for got, ref in ((dQ, dq_ref), (dK, dk_ref), (dV, dv_ref)):
         assert _rel(got.float().cpu().numpy(), 2 * ref) <= 2e-2
+
+
+@pytest.mark.parametrize("nb,heads,seq,ramp", [(8, 16, 512, 3.0), (3, 5, 384, 6.0), (2, 2, 1024, 4.0)])
+def test_tc_forward_online_rescale_persistent(nb, heads, seq, ramp):
+    """The tcgen05 forward streams K/V in 128-key chunks with an online softmax whose running
+    max moves only when it grows by > 8 (log2 units).  Keys scaled by a ramp along the sequence
+    make later chunks' maxima jump past that threshold (O-row rescale path); (8, 16, 512) has
+    256 work items, more than the persistent grid, so CTAs loop over items; seq 384 has an odd
+    tile count (single-tile items); seq 1024 exceeds the old whole-row-in-TMEM limit."""
+    d, alpha, p, seed, b0, step = 64, 0.5, 0.1, 11, 2, 4
+    q, k, v, dc = _inputs(nb, heads, seq, d, seed=5)
+    pos = np.tile(np.arange(seq), nb)[:, None]
+    k = gen.snap_bf16((k * (1.0 + ramp * pos / seq)).astype(np.float32))
+    c_ref, lse_ref, mask_ref = O.attention_fwd(q, k, v, heads, seq, alpha, p, seed, b0 * heads * seq * seq, step)
+    # the ramp really crosses the rescale threshold somewhere: chunk maxima grow by > 8 / log2(e)
+    s = np.einsum("qhd,khd->hqk", q.reshape(nb * seq, heads, d)[:seq], k.reshape(nb * seq, heads, d)[:seq]) * alpha
+    cm = s.reshape(heads, seq, seq // 128, 128).max(-1)
+    assert (np.diff(np.maximum.accumulate(cm, axis=-1), axis=-1) > 8 / np.log2(np.e)).any()
+    dev = lambda a: torch.from_numpy(a).to("cuda").to(torch.bfloat16)  # noqa: E731
+    Q, K, V = dev(q), dev(k), dev(v)
+    C = torch.empty_like(Q)
+    L = torch.empty((nb, heads, seq), dtype=torch.float32, device="cuda")
+    M = torch.empty((nb, heads, seq, seq // 32), dtype=torch.int32, device="cuda")
+    used = tsplit.attention(1, (nb, heads, seq, d, seed, b0, step), alpha, p, Q, K, V, c=C, lse=L, mask=M)
+    torch.cuda.synchronize()
+    assert used == 2
+    assert np.array_equal(M.cpu().numpy(), mask_ref)
+    assert _rel(L.cpu().numpy(), lse_ref) <= 1e-5
+    assert _rel(C.float().cpu().numpy(), c_ref) <= 1e-2
 
 
 def test_attention_split_equals_whole():
