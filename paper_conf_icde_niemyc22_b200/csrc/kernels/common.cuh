@@ -18,6 +18,42 @@ __device__ __forceinline__ float from_f<float>(float x) { return x; }
 template <>
 __device__ __forceinline__ bf16 from_f<bf16>(float x) { return __float2bfloat16_rn(x); }
 
+// erf-GELU (R16) shared by the elementwise kernels and the GEMM epilogue (one definition, so a
+// fused epilogue computes bit-for-bit what the separate kernel would).  erf by Abramowitz &
+// Stegun 7.1.26 (|error| <= 1.5e-7) on the MUFU unit: t = rcp.approx(1 + p|z|) and
+// exp(-z^2) = ex2.approx(-x^2 log2(e) / 2), which the derivative's normal pdf reuses — about
+// 13 FP32 instructions and 2 MUFU per element (the CUDA erff costs ~22 with selects, an IEEE
+// reciprocal far more; both made the GELU passes ALU-bound).
+__device__ __forceinline__ float ex2_approx(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+__device__ __forceinline__ float rcp_approx(float x) {
+  float y;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+// erf(x / sqrt 2) given e = exp(-x^2 / 2)
+__device__ __forceinline__ float erf_gelu(float x, float e) {
+  const float t = rcp_approx(fmaf(0.3275911f * 0.70710678118654752f, fabsf(x), 1.f));
+  float p = fmaf(1.061405429f, t, -1.453152027f);
+  p = fmaf(p, t, 1.421413741f);
+  p = fmaf(p, t, -0.284496736f);
+  p = fmaf(p, t, 0.254829592f);
+  return copysignf(fmaf(-p * t, e, 1.f), x);
+}
+__device__ __forceinline__ float gelu_f(float x) {
+  const float e = ex2_approx(x * x * -0.72134752044448170f);  // exp(-x^2/2) = 2^(-x^2 log2(e)/2)
+  return 0.5f * x * (1.f + erf_gelu(x, e));
+}
+__device__ __forceinline__ float gelu_d(float x) {
+  const float e = ex2_approx(x * x * -0.72134752044448170f);
+  const float cdf = 0.5f * (1.f + erf_gelu(x, e));
+  return fmaf(x * 0.39894228040143268f, e, cdf);
+}
+__device__ __forceinline__ float bf16_round(float x) { return __bfloat162float(__float2bfloat16_rn(x)); }
+
 // Philox4x32-10 (Salmon et al. SC'11); reading D-RNG: element idx uses
 // word (idx & 3) of Philox(counter = (idx>>2 lo, idx>>2 hi, step, 0), key = (seed, 0x5453504C)).
 __device__ __forceinline__ uint4 philox4x32_10(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3,

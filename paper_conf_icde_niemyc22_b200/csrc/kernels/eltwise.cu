@@ -17,21 +17,7 @@ struct EwP {
   uint32_t seed, step, thr;
 };
 
-// erf-GELU (R16).  The forward uses the CUDA math library's erff (<= 2 ulp, one MUFU
-// exponential); the derivative needs the normal pdf exp(-x^2/2) too, which is one ex2.approx.
-// The previous Abramowitz & Stegun form used an IEEE reciprocal (__frcp_rn, a multi-instruction
-// sequence) and made the GELU kernels ALU-bound at ~half of HBM bandwidth (ncu: 76% SM, 30% DRAM).
-__device__ __forceinline__ float ex2f(float x) {
-  float y;
-  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
-  return y;
-}
-__device__ __forceinline__ float gelu_f(float x) { return 0.5f * x * (1.f + erff(x * 0.70710678118654752f)); }
-__device__ __forceinline__ float gelu_d(float x) {
-  const float cdf = 0.5f * (1.f + erff(x * 0.70710678118654752f));
-  const float pdf = ex2f(x * x * -0.72134752044448170f);  // exp(-x^2/2) = 2^(-x^2 log2(e)/2)
-  return fmaf(x * 0.39894228040143268f, pdf, cdf);
-}
+// GELU: gelu_f / gelu_d from common.cuh (shared with the GEMM epilogue).
 
 template <int OP>
 __device__ __forceinline__ float ew_apply(float a, float b, int64_t idx, uint32_t word, const EwP& q) {

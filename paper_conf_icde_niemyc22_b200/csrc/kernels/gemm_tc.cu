@@ -27,8 +27,10 @@ namespace {
 using namespace tc;
 
 constexpr int BM = 128, BK = 64;
-constexpr int kEpiWarps = 8;   // two per TMEM lane quarter, alternating 32-column chunks
-constexpr int kThreads = 64 + 32 * kEpiWarps;  // warp0 TMA, warp1 MMA, warps 2.. epilogue
+// epilogue warps EW: 8 (two per TMEM lane quarter) for plain epilogues; 16 for the fused GELU
+// forward epilogue, whose ALU work needs four warps per scheduler to hide its latency
+template <int EW>
+constexpr int num_threads() { return 64 + 32 * EW; }  // warp0 TMA, warp1 MMA, warps 2.. epilogue
 
 struct TcParams {
   int M, N, K, nb1, nb2;
@@ -44,18 +46,21 @@ struct TcParams {
   int bias_f32;
   int tma_store;   // 1: stage in smem and TMA-store; 0: direct per-thread stores
   int reduce_add;  // 1: TMA reduce-add into an fp32 C (beta = 1 or split-K)
+  int epi;         // GemmArgs::epi (bf16 TMA-store path only): 1 GELU fwd (2nd output via tmC2), 2 GELU bwd
+  const bf16* aux; // epi 2: U, row-major with leading dimension ldaux
+  int64_t ldaux;
 };
 // epilogue staging: per warp, 32x32 output blocks (two for bf16; one for fp32, whose
 // products have long K and keep the smem for a deeper operand pipeline)
-template <bool F32OUT>
-constexpr int staging_bufs() { return F32OUT ? 1 : 2; }
+template <bool F32OUT, int EW>
+constexpr int staging_nbuf() { return (!F32OUT && EW == 8) ? 2 : 1; }
 constexpr int kSmemLimit = 232448;  // 227 KB opt-in dynamic shared memory per CTA
-template <bool F32OUT>
-constexpr int staging_bytes() { return kEpiWarps * staging_bufs<F32OUT>() * 32 * 32 * (F32OUT ? 4 : 2); }
-template <int BN, bool F32OUT>
+template <bool F32OUT, int EW>
+constexpr int staging_bytes() { return EW * staging_nbuf<F32OUT, EW>() * 32 * 32 * (F32OUT ? 4 : 2); }
+template <int BN, bool F32OUT, int EW>
 constexpr int num_stages() {
   constexpr int stage = (BM + BN) * BK * 2;
-  constexpr int n = (kSmemLimit - staging_bytes<F32OUT>() - 2048) / stage;
+  constexpr int n = (kSmemLimit - staging_bytes<F32OUT, EW>() - 2048) / stage;
   return n > 8 ? 8 : n;
 }
 
@@ -79,14 +84,15 @@ __device__ __forceinline__ void decode_tile(const TcParams& p, int tile, int& b1
   n0 = nt;  // scaled by BN by the caller
 }
 
-template <int BN, bool F32OUT>
-__global__ void __launch_bounds__(kThreads, 1)
+template <int BN, bool F32OUT, int EW>
+__global__ void __launch_bounds__(num_threads<EW>(), 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   const __grid_constant__ CUtensorMap tmC, const TcParams p) {
+                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmC2,
+                   const TcParams p) {
   constexpr int A_BYTES = BM * BK * 2;
   constexpr int B_BYTES = BN * BK * 2;
   constexpr int STAGE = A_BYTES + B_BYTES;
-  constexpr int STAGES = num_stages<BN, F32OUT>();
+  constexpr int STAGES = num_stages<BN, F32OUT, EW>();
   constexpr uint32_t TMEM_COLS = 2 * BN;
   constexpr int BUF = 32 * 32 * (F32OUT ? 4 : 2);
   // instruction descriptor: D f32, A/B bf16, M = 128, N = BN
@@ -110,7 +116,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int s = 0; s < 2; ++s) {
       mbar_init(&tfull[s], 1);
-      mbar_init(&tempty[s], 32 * kEpiWarps);
+      mbar_init(&tempty[s], 32 * EW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
@@ -209,9 +215,11 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else {
     // ===== epilogue: TMEM -> registers (alpha, bias) -> swizzled smem -> TMA store =====
     const int q = warp & 3;        // TMEM lane quarter this warp may access
-    const int ew = warp - 2;       // epilogue warp index 0..7
-    const int half = ew >> 2;      // which alternate 32-column chunks this warp stores
-    uint8_t* wbuf = cstage + ew * staging_bufs<F32OUT>() * BUF;
+    const int ew = warp - 2;       // epilogue warp index
+    const int half = ew >> 2;      // column group: chunks half, half + kGrp, ... of each tile
+    constexpr int kGrp = EW / 4;
+    constexpr int NBUF = staging_nbuf<F32OUT, EW>();
+    uint8_t* wbuf = cstage + ew * NBUF * BUF;
     int nbuf = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -227,7 +235,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const bool row_ok = row < p.M;
       const int64_t cbase = int64_t(b1) * p.cbs1 + int64_t(b2) * p.cbs2 + int64_t(row) * p.ldc;
 #pragma unroll 1
-      for (int c = half; c < BN / 32; c += 2) {
+      for (int c = half; c < BN / 32; c += kGrp) {
         uint32_t r[32];
         tmem_ld32(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * BN + c * 32), r);
         const int col0 = n0 + c * 32;
@@ -266,36 +274,65 @@ __global__ void __launch_bounds__(kThreads, 1)
               for (int i = 0; i < 32; ++i)
                 if (full_chunk || col0 + i < p.N) v[i] += p.beta * to_f(cp[i]);
             }
-            uint8_t* buf = wbuf + nbuf * BUF;
-            if (lane == 0) {  // the store that last used `buf` has read it
-              if constexpr (F32OUT) bulk_wait_read0();
-              else bulk_wait_read1();
-            }
-            __syncwarp();
-            if constexpr (F32OUT) {
+            if constexpr (!F32OUT) {
+              if (p.epi == 2) {  // dU = bf16(dH) * gelu'(U): U's row chunk straight from global
+                const bf16* up = p.aux + int64_t(row) * p.ldaux + col0;
+                if (row_ok && full_chunk) {
+                  uint4 u[4];
 #pragma unroll
-              for (int j = 0; j < 8; ++j) {  // 128 B row, SWIZZLE_128B
-                float4 o = make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
-                *reinterpret_cast<float4*>(buf + lane * 128 + ((j ^ (lane & 7)) << 4)) = o;
-              }
-            } else {
+                  for (int j = 0; j < 4; ++j) u[j] = __ldg(reinterpret_cast<const uint4*>(up) + j);
+                  const bf16* ub = reinterpret_cast<const bf16*>(u);
 #pragma unroll
-              for (int j = 0; j < 4; ++j) {  // 64 B row, SWIZZLE_64B
-                uint4 o;
-                __nv_bfloat162* o2 = reinterpret_cast<__nv_bfloat162*>(&o);
+                  for (int i = 0; i < 32; ++i) v[i] = bf16_round(v[i]) * gelu_d(to_f(ub[i]));
+                } else if (row_ok) {
 #pragma unroll
-                for (int h = 0; h < 4; ++h) o2[h] = __floats2bfloat162_rn(v[8 * j + 2 * h], v[8 * j + 2 * h + 1]);
-                *reinterpret_cast<uint4*>(buf + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4)) = o;
+                  for (int i = 0; i < 32; ++i)
+                    if (col0 + i < p.N) v[i] = bf16_round(v[i]) * gelu_d(to_f(up[i]));
+                }
               }
             }
-            fence_async_smem();
-            __syncwarp();
-            if (lane == 0) {
-              if (p.reduce_add) tma_reduce_add(&tmC, buf, col0, m0 + q * 32, b1, b2);
-              else tma_store(&tmC, buf, col0, m0 + q * 32, b1, b2);
-              bulk_commit();
+            // stage 32 rows x 32 columns in swizzled smem, then one TMA store (or reduce-add)
+            auto stage_store = [&](const float* vals, const CUtensorMap* map, bool radd) {
+              uint8_t* buf = wbuf + nbuf * BUF;
+              if (lane == 0) {  // the store that last used `buf` has read it
+                if constexpr (NBUF == 1) bulk_wait_read0();
+                else bulk_wait_read1();
+              }
+              __syncwarp();
+              if constexpr (F32OUT) {
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {  // 128 B row, SWIZZLE_128B
+                  float4 o = make_float4(vals[4 * j], vals[4 * j + 1], vals[4 * j + 2], vals[4 * j + 3]);
+                  *reinterpret_cast<float4*>(buf + lane * 128 + ((j ^ (lane & 7)) << 4)) = o;
+                }
+              } else {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {  // 64 B row, SWIZZLE_64B
+                  uint4 o;
+                  __nv_bfloat162* o2 = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+                  for (int h = 0; h < 4; ++h)
+                    o2[h] = __floats2bfloat162_rn(vals[8 * j + 2 * h], vals[8 * j + 2 * h + 1]);
+                  *reinterpret_cast<uint4*>(buf + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4)) = o;
+                }
+              }
+              fence_async_smem();
+              __syncwarp();
+              if (lane == 0) {
+                if (radd) tma_reduce_add(map, buf, col0, m0 + q * 32, b1, b2);
+                else tma_store(map, buf, col0, m0 + q * 32, b1, b2);
+                bulk_commit();
+              }
+              nbuf = (nbuf + 1) % NBUF;
+            };
+            stage_store(v, &tmC, p.reduce_add);
+            if constexpr (!F32OUT) {
+              if (p.epi == 1) {  // second output: gelu of the stored (bf16) U
+#pragma unroll
+                for (int i = 0; i < 32; ++i) v[i] = gelu_f(bf16_round(v[i]));
+                stage_store(v, &tmC2, false);
+              }
             }
-            if constexpr (!F32OUT) nbuf ^= 1;
           } else if (row_ok) {
             if (p.c_f32) {
               float* cp = reinterpret_cast<float*>(p.C) + cbase + col0;
@@ -375,17 +412,18 @@ bool make_operand_map(CUtensorMap* map, const GemmOperand& op, int64_t d0, int64
 int g_num_sms = 0;
 std::atomic<int64_t> g_launches{0};
 
-template <int BN, bool F32OUT>
-void launch(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, const TcParams& p, cudaStream_t st) {
+template <int BN, bool F32OUT, int EW = 8>
+void launch(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, const CUtensorMap& c2, const TcParams& p,
+            cudaStream_t st) {
   constexpr int STAGE = (BM + BN) * BK * 2;
-  const int smem = num_stages<BN, F32OUT>() * STAGE + 1024 + staging_bytes<F32OUT>() + 1024;
+  const int smem = num_stages<BN, F32OUT, EW>() * STAGE + 1024 + staging_bytes<F32OUT, EW>() + 1024;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(gemm_tc_kernel<BN, F32OUT>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(gemm_tc_kernel<BN, F32OUT, EW>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
   int grid = p.num_units < g_num_sms ? p.num_units : g_num_sms;
-  gemm_tc_kernel<BN, F32OUT><<<grid, kThreads, smem, st>>>(a, b, c, p);
+  gemm_tc_kernel<BN, F32OUT, EW><<<grid, num_threads<EW>(), smem, st>>>(a, b, c, c2, p);
   g_launches++;
 }
 
@@ -466,6 +504,19 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
                     ? 1 : 0;
   if (g.beta != 0.f && g.beta != 1.f) p.tma_store = 0;
   if (!p.tma_store) mc = ma;  // unused
+  // fused GELU epilogues need the bf16 TMA-store path (and no accumulation into C)
+  p.epi = g.epi;
+  p.aux = static_cast<const bf16*>(g.aux);
+  p.ldaux = g.ldaux;
+  CUtensorMap mc2 = mc;
+  if (g.epi) {
+    if (!p.tma_store || p.c_f32 || g.beta != 0.f || !g.aux) return false;
+    if (g.epi == 1 && !make_map(&mc2, g.aux, g.ldaux, 0, 0, g.N, g.M, 1, 1, 32, 32, 2,
+                                CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, CU_TENSOR_MAP_SWIZZLE_64B))
+      return false;
+    if (g.epi == 2 && ((reinterpret_cast<uintptr_t>(g.aux) | uintptr_t(g.ldaux * 2)) & 15)) return false;
+    if (g.nb1 * g.nb2 != 1) return false;
+  }
   // beta = 1 accumulates with a TMA reduce-add of the new tile (fp32, or bf16 gradients that
   // several backward ops add into: the old values never pass through registers)
   p.reduce_add = (p.tma_store && g.beta == 1.f) ? 1 : 0;
@@ -482,15 +533,18 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   p.num_units = p.num_tiles * p.ksplit;
   if (p.c_f32) {
     switch (best_bn) {
-      case 256: launch<256, true>(ma, mb, mc, p, st); break;
-      case 128: launch<128, true>(ma, mb, mc, p, st); break;
-      default: launch<64, true>(ma, mb, mc, p, st); break;
+      case 256: launch<256, true>(ma, mb, mc, mc2, p, st); break;
+      case 128: launch<128, true>(ma, mb, mc, mc2, p, st); break;
+      default: launch<64, true>(ma, mb, mc, mc2, p, st); break;
     }
   } else {
     switch (best_bn) {
-      case 256: launch<256, false>(ma, mb, mc, p, st); break;
-      case 128: launch<128, false>(ma, mb, mc, p, st); break;
-      default: launch<64, false>(ma, mb, mc, p, st); break;
+      case 256:
+        if (p.epi == 1) launch<256, false, 16>(ma, mb, mc, mc2, p, st);
+        else launch<256, false>(ma, mb, mc, mc2, p, st);
+        break;
+      case 128: launch<128, false>(ma, mb, mc, mc2, p, st); break;
+      default: launch<64, false>(ma, mb, mc, mc2, p, st); break;
     }
   }
   return true;
@@ -508,7 +562,14 @@ void gemm(const GemmArgs& g, cudaStream_t st) {
     cudaEventRecord(rec.start, st);
   }
   rec.tc = gemm_tc(g, st) ? 1 : 0;
-  if (!rec.tc) gemm_simt(g, st);
+  if (!rec.tc) {
+    GemmArgs plain = g;
+    plain.epi = 0;
+    gemm_simt(plain, st);
+    // the fused epilogue's effect, unfused: gelu of the stored U / dU = dH * gelu'(U) in place
+    if (g.epi == 1) gelu_fwd(BF16, g.c, g.aux, int64_t(g.M) * g.N, st);
+    if (g.epi == 2) gelu_bwd(BF16, g.c, g.aux, g.c, 0, int64_t(g.M) * g.N, st);
+  }
   if (g_sink) {
     cudaEventRecord(rec.stop, st);
     rec.flop = 2.0 * g.M * double(g.N) * g.K * g.nb1 * g.nb2;

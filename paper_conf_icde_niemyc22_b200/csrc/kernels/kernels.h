@@ -30,6 +30,13 @@ struct GemmArgs {
   float alpha = 1.f, beta = 0.f;
   const void* bias = nullptr;
   int bias_dtype = BF16;
+  // fused epilogue (bf16 C, beta = 0): 1 = GELU forward, C = U = alpha AB + bias and
+  // aux = gelu(U) (the linear -> gelu pair of one micro-op); 2 = GELU backward, C = dU =
+  // bf16(alpha AB) * gelu'(aux) with aux = U (the dX product of the layer after a gelu).
+  // Values pass through bf16 exactly where the separate kernels would store them.
+  int epi = 0;
+  void* aux = nullptr;
+  int64_t ldaux = 0;
 };
 
 // Returns false (and leaves nothing launched) when the shape/alignment does not

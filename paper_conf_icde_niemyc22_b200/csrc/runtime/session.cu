@@ -11,6 +11,7 @@
 
 #include <algorithm>
 #include <array>
+#include <cstdlib>
 #include <cstring>
 #include <functional>
 #include <map>
@@ -115,8 +116,19 @@ struct Micro {
   std::unordered_map<int, int> acc;  // grad key -> accumulate flag
 };
 
+// Peephole fusion of a linear micro-op with the gelu micro-op next to it (build_program
+// decides when it is safe): mode 1 = forward, the GEMM epilogue also writes gelu(U) to `y`;
+// mode 2 = backward, the dX product writes dU = dH * gelu'(U) to `du` (reading `u`) instead of dH.
+struct Fuse {
+  int mode = 0;
+  char* y = nullptr;
+  char* du = nullptr;
+  char* u = nullptr;
+};
+
 // Lower one micro-op to kernel launches (DESIGN.md §3 op table).
-std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bwd, int& nk) {
+std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bwd, int& nk,
+                                        const Fuse* fz = nullptr) {
   const Graph& g = *s->g;
   const Op& o = g.ops[m.op];
   const int dt = g.dtype == TS_BF16 ? tsk::BF16 : tsk::F32;
@@ -145,6 +157,9 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
         a.b = {param_w(s, w), K, false, 0, 0};
         a.c = V(o.out[0]); a.ldc = N; a.c_dtype = dt;
         a.bias = param_w(s, bb); a.bias_dtype = dt;
+        if (fz && fz->mode == 1) {
+          a.epi = 1; a.aux = fz->y; a.ldaux = N;
+        }
         nk = 1;
         return [a](cudaStream_t st) { tsk::gemm(a, st); };
       }
@@ -156,6 +171,9 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
         a.a = {dY, N, false, 0, 0};
         a.b = {param_w(s, w), K, true, 0, 0};
         a.c = G(o.in[0]); a.ldc = K; a.c_dtype = dt; a.beta = A(g.n() + o.in[0]) ? 1.f : 0.f;
+        if (fz && fz->mode == 2) {
+          a.c = fz->du; a.beta = 0.f; a.epi = 2; a.aux = fz->u; a.ldaux = K;
+        }
         gs.push_back(a);
       }
       tsk::GemmArgs d;
@@ -167,6 +185,8 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       float* db = param_g(s, bb);
       int dacc = A(bb);
       const uint64_t wsb = g.ws_bytes;
+      // fused backward: dW (the last reader of X = H) first, then dX may overwrite H's range with dU
+      if (fz && fz->mode == 2 && gs.size() == 2) std::swap(gs[0], gs[1]);
       nk = int(gs.size()) + 1;
       return [gs, dY, R, N, db, dacc, ws, wsb, dt](cudaStream_t st) {
         for (auto& a : gs) tsk::gemm(a, st);
@@ -586,6 +606,15 @@ ts_status build_program(ts_session_t* s) {
   std::map<int, int> param_first_item;
   s->ev_d2h.assign(s->ex.items.size(), nullptr);
   s->ev_h2d.assign(s->ex.items.size(), nullptr);
+  // per item: the trace's ALLOC / FREE events (for the linear + gelu fusion check)
+  std::vector<std::vector<const Event*>> allocs_of(s->ex.items.size()), frees_of(s->ex.items.size());
+  for (auto& e : tr)
+    if (e.item >= 0 && size_t(e.item) < s->ex.items.size())  // (the loss is freed after the last item)
+      (e.kind == 0 ? allocs_of : frees_of)[e.item].push_back(&e);
+  std::set<int> fused_away;  // gelu items whose work the previous linear item's GEMM does
+  // TSPLIT_NO_FUSION=1 lowers every micro-op on its own (tests compare the two programs)
+  const char* nf = std::getenv("TSPLIT_NO_FUSION");
+  const bool fusion_on = !(nf && nf[0] == '1');
   auto overlaps = [](uint64_t a0, uint64_t al, uint64_t b0, uint64_t bl) { return a0 < b0 + bl && b0 < a0 + al; };
   for (size_t i = 0; i < s->ex.items.size(); ++i) {
     const Item& it = s->ex.items[i];
@@ -692,8 +721,61 @@ ts_status build_program(ts_session_t* s) {
         if (!list(o.in[0], m.all_x)) return set_error("batchnorm: too many pieces"), TS_ERR_GRAPH;
         if (bwd && !list(n + o.out[0], m.all_dy)) return set_error("batchnorm: too many pieces"), TS_ERR_GRAPH;
       }
+      // linear + gelu peephole fusion (bf16): the next item is the gelu micro-op over the same
+      // samples; its output (forward) / input gradient (backward) range must already be free
+      // while this item runs — it is allocated at the next item and no range freed after this
+      // item overlaps it — and the next item must have no copy fences of its own.
+      Fuse fz;
+      if (fusion_on && g.dtype == TS_BF16 && o.kind == TS_OP_LINEAR && i + 1 < s->ex.items.size()) {
+        const Item& nx = s->ex.items[i + 1];
+        const Op& go = g.ops[nx.op];
+        const bool same = nx.kind == it.kind && nx.k == it.k && s->ex.P[nx.op] == m.P && nx.group == it.group &&
+                          go.kind == TS_OP_GELU && s->sim.wait_so[i + 1].empty();
+        // `ok_key`: a tensor freed after this item that the fused product may overwrite because
+        // its last reader runs first (backward: the gelu output H, read only by the dW product)
+        auto free_while_here = [&](int key, uint64_t& off, uint64_t& bytes, int ok_key) -> bool {
+          const Event* a = nullptr;
+          for (const Event* e : allocs_of[i + 1])
+            if (e->key == key) a = e;
+          if (!a) return false;
+          for (const Event* f : frees_of[i])
+            if (f->key != ok_key && overlaps(a->offset, align_up(a->bytes), f->offset, align_up(f->bytes)))
+              return false;
+          off = a->offset;
+          bytes = a->bytes;
+          return true;
+        };
+        auto sub_view = [&](int t, uint64_t piece_off) -> char* {
+          const Tensor& x = g.t[t];
+          int p = piece_count(g, s->cfg, t);
+          int j = int(m.s0 * p / B);
+          int64_t first = int64_t(j) * B / p;
+          return s->slab + piece_off + (m.s0 - first) * x.elems_per_sample * es;
+        };
+        uint64_t off = 0, bytes = 0;
+        if (same && !bwd && go.in[0] == o.out[0] && free_while_here(go.out[0], off, bytes, -1)) {
+          fz.mode = 1;
+          fz.y = sub_view(go.out[0], off);
+        } else if (same && bwd && go.out[0] == o.in[0] && g.t[go.out[0]].consumers.size() == 1 &&
+                   m.grad.count(o.in[0]) && m.acc.count(n + o.in[0]) && m.acc.at(n + o.in[0]) == 0 &&
+                   !grad_first_op.count(n + go.in[0]) && free_while_here(n + go.in[0], off, bytes, o.in[0])) {
+          const int u = go.in[0];
+          const int pu = piece_count(g, s->cfg, u);
+          const PieceKey upc = pk(u, int(m.s0 * pu / B));
+          if (where.count(upc) && !si_live.count(upc)) {
+            fz.mode = 2;
+            fz.du = sub_view(u, off);
+            fz.u = view(u);
+          }
+        }
+      }
       int nk = 0;
-      cmd.fn = lower(s, m, bwd, nk);
+      if (fused_away.count(int(i))) {
+        cmd.fn = [](cudaStream_t) {};
+      } else {
+        cmd.fn = lower(s, m, bwd, nk, fz.mode ? &fz : nullptr);
+        if (fz.mode) fused_away.insert(int(i) + 1);
+      }
       s->launches += nk;
       if (bwd)
         for (int t : o.in)
