@@ -486,6 +486,88 @@ __global__ void __launch_bounds__(256) colsum_kernel(const T* __restrict__ x, in
   if (threadIdx.x == 0) tickets[blockIdx.x] = 0u;  // re-arm for the next launch / graph replay
 }
 
+// bf16 column sums (bias gradients) at HBM rate: block (cb, g) owns 256 columns (32 lanes x
+// one 16-byte vector) and rows g*8+w, g*8+w+8G, ...; eight rows are in flight per thread.  The
+// eight warps combine in a fixed order into the partial row ws[g]; the last block of a column
+// block (atomic ticket) reduces the G partials with all its warps — warp w takes partial rows
+// w, w+8, ... (two float4 per lane), the warps combine in fp64 in order — so the result is
+// deterministic for a given shape and the tail is a few dependent loads, not G of them.
+__global__ void __launch_bounds__(256) colsum_bf16_kernel(const bf16* __restrict__ x, int64_t rows, int N, int G,
+                                                          float* __restrict__ ws, unsigned* __restrict__ tickets,
+                                                          float* out, int acc) {
+  __shared__ float red[8][256];
+  __shared__ double redd[8][256];
+  __shared__ bool last;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int c0 = blockIdx.x * 256 + lane * 8;
+  const bool colok = c0 < N;
+  float a[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  const int64_t rstep = int64_t(G) * 8;
+  int64_t r = int64_t(blockIdx.y) * 8 + w;
+  if (colok) {
+    for (; r + 7 * rstep < rows; r += 8 * rstep) {
+      uint4 u[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) u[k] = __ldcs(reinterpret_cast<const uint4*>(x + (r + k * rstep) * N + c0));
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u[k]);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 f = __bfloat1622float2(h[e]);
+          a[2 * e] += f.x;
+          a[2 * e + 1] += f.y;
+        }
+      }
+    }
+    for (; r < rows; r += rstep) {
+      const uint4 u = __ldcs(reinterpret_cast<const uint4*>(x + r * N + c0));
+      const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float2 f = __bfloat1622float2(h[e]);
+        a[2 * e] += f.x;
+        a[2 * e + 1] += f.y;
+      }
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) red[w][lane * 8 + i] = a[i];
+  __syncthreads();
+  const int c = blockIdx.x * 256 + threadIdx.x;
+  if (c < N) {
+    float t = 0.f;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) t += red[k][threadIdx.x];
+    ws[int64_t(blockIdx.y) * N + c] = t;
+  }
+  __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) last = atomicAdd(&tickets[blockIdx.x], 1u) == unsigned(G - 1);
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  double d[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  if (colok) {
+    for (int b = w; b < G; b += 8) {
+      const float4 u0 = __ldcg(reinterpret_cast<const float4*>(ws + int64_t(b) * N + c0));
+      const float4 u1 = __ldcg(reinterpret_cast<const float4*>(ws + int64_t(b) * N + c0 + 4));
+      d[0] += u0.x; d[1] += u0.y; d[2] += u0.z; d[3] += u0.w;
+      d[4] += u1.x; d[5] += u1.y; d[6] += u1.z; d[7] += u1.w;
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 8; ++i) redd[w][lane * 8 + i] = d[i];
+  __syncthreads();
+  if (c < N) {
+    double t = 0.0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) t += redd[k][threadIdx.x];
+    out[c] = acc ? float(double(out[c]) + t) : float(t);
+  }
+  if (threadIdx.x == 0) tickets[blockIdx.x] = 0u;  // re-arm for the next launch / graph replay
+}
+
 // ------------------------------------------------------------------ softmax
 template <class T, int NCH>
 __global__ void __launch_bounds__(kWarps * 32) softmax_fwd_kernel(const T* __restrict__ x, T* __restrict__ y,
@@ -789,12 +871,198 @@ void ln_bwd_t(const void* dy, const void* x, const void* g, void* dx, int acc, f
   ln_bwd_kernel<T><<<G, kWarps * 32, smem, st>>>(DY, X, Gm, DX, acc, ws, rows, H, eps);
 }
 
+// Fused bf16 LayerNorm backward (rows of NCH x 256 columns): x and dy are read once.  A
+// persistent grid of G blocks; warp w of block b takes rows b*8+w, b*8+w+8G, ...: dx (+)=
+// rstd*(g dy - mean(g dy) - xhat mean(g dy xhat)) from registers, and the row's dy*xhat and dy
+// are added into the warp's private shared-memory partial row (lanes own disjoint columns, so
+// no atomics).  The block's eight warps combine in a fixed order into ws[b][2H] (dgamma | dbeta
+// partials), reduced over the G blocks by reduce_partials2 — deterministic for a given shape.
+template <int NCH>
+__global__ void __launch_bounds__(256, 2) ln_bwd_fused_bf16(const bf16* __restrict__ dy, const bf16* __restrict__ x,
+                                                             const bf16* __restrict__ g, bf16* dx, int acc,
+                                                             int64_t rows, int H, float eps, float* __restrict__ ws) {
+  extern __shared__ float sp[];  // [8 warps][2][H]
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  float* pg = sp + w * 2 * H;
+  float* pb = pg + H;
+  uint4 gv[NCH];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int col = (c * 32 + lane) * 8;
+    gv[c] = col < H ? *reinterpret_cast<const uint4*>(g + col) : make_uint4(0, 0, 0, 0);
+    if (col < H) {
+#pragma unroll
+      for (int i = 0; i < 8; i += 4) {
+        *reinterpret_cast<float4*>(pg + col + i) = make_float4(0.f, 0.f, 0.f, 0.f);
+        *reinterpret_cast<float4*>(pb + col + i) = make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    }
+  }
+  const float invH = 1.f / float(H);
+  for (int64_t r = int64_t(blockIdx.x) * 8 + w; r < rows; r += int64_t(gridDim.x) * 8) {
+    uint4 xu[NCH], du[NCH], ou[NCH];
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      const int col = (c * 32 + lane) * 8;
+      if (col < H) {
+        xu[c] = __ldcs(reinterpret_cast<const uint4*>(x + r * H + col));
+        du[c] = __ldcs(reinterpret_cast<const uint4*>(dy + r * H + col));
+        if (acc) ou[c] = *reinterpret_cast<const uint4*>(dx + r * H + col);
+      }
+    }
+    float s = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c)
+      if ((c * 32 + lane) * 8 < H) {
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&xu[c]);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 f = __bfloat1622float2(h[e]);
+          s += f.x + f.y;
+        }
+      }
+    const float mean = warp_sum(s) * invH;
+    float q = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c)
+      if ((c * 32 + lane) * 8 < H) {
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&xu[c]);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 f = __bfloat1622float2(h[e]);
+          q += (f.x - mean) * (f.x - mean) + (f.y - mean) * (f.y - mean);
+        }
+      }
+    const float rstd = rsqrtf(warp_sum(q) * invH + eps);
+    float s1 = 0.f, s2 = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c)
+      if ((c * 32 + lane) * 8 < H) {
+        const __nv_bfloat162* hx = reinterpret_cast<const __nv_bfloat162*>(&xu[c]);
+        const __nv_bfloat162* hd = reinterpret_cast<const __nv_bfloat162*>(&du[c]);
+        const __nv_bfloat162* hg = reinterpret_cast<const __nv_bfloat162*>(&gv[c]);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 fx = __bfloat1622float2(hx[e]), fd = __bfloat1622float2(hd[e]), fg = __bfloat1622float2(hg[e]);
+          const float a0 = fd.x * fg.x, a1 = fd.y * fg.y;
+          s1 += a0 + a1;
+          s2 += a0 * ((fx.x - mean) * rstd) + a1 * ((fx.y - mean) * rstd);
+        }
+      }
+    s1 = warp_sum(s1) * invH;
+    s2 = warp_sum(s2) * invH;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      const int col = (c * 32 + lane) * 8;
+      if (col < H) {
+        const __nv_bfloat162* hx = reinterpret_cast<const __nv_bfloat162*>(&xu[c]);
+        const __nv_bfloat162* hd = reinterpret_cast<const __nv_bfloat162*>(&du[c]);
+        const __nv_bfloat162* hg = reinterpret_cast<const __nv_bfloat162*>(&gv[c]);
+        const __nv_bfloat162* ho = reinterpret_cast<const __nv_bfloat162*>(&ou[c]);
+        float o[8], xh[8], dd[8];
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 fx = __bfloat1622float2(hx[e]), fd = __bfloat1622float2(hd[e]), fg = __bfloat1622float2(hg[e]);
+          xh[2 * e] = (fx.x - mean) * rstd;
+          xh[2 * e + 1] = (fx.y - mean) * rstd;
+          dd[2 * e] = fd.x;
+          dd[2 * e + 1] = fd.y;
+          o[2 * e] = rstd * (fd.x * fg.x - s1 - xh[2 * e] * s2);
+          o[2 * e + 1] = rstd * (fd.y * fg.y - s1 - xh[2 * e + 1] * s2);
+          if (acc) {
+            const float2 fo = __bfloat1622float2(ho[e]);
+            o[2 * e] += fo.x;
+            o[2 * e + 1] += fo.y;
+          }
+        }
+        uint4 st;
+        __nv_bfloat162* hs = reinterpret_cast<__nv_bfloat162*>(&st);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) hs[e] = __floats2bfloat162_rn(o[2 * e], o[2 * e + 1]);
+        *reinterpret_cast<uint4*>(dx + r * H + col) = st;
+#pragma unroll
+        for (int i = 0; i < 8; i += 4) {
+          float4 a = *reinterpret_cast<float4*>(pg + col + i);
+          float4 b = *reinterpret_cast<float4*>(pb + col + i);
+          a.x += dd[i] * xh[i]; a.y += dd[i + 1] * xh[i + 1]; a.z += dd[i + 2] * xh[i + 2]; a.w += dd[i + 3] * xh[i + 3];
+          b.x += dd[i]; b.y += dd[i + 1]; b.z += dd[i + 2]; b.w += dd[i + 3];
+          *reinterpret_cast<float4*>(pg + col + i) = a;
+          *reinterpret_cast<float4*>(pb + col + i) = b;
+        }
+      }
+    }
+  }
+  __syncthreads();
+  for (int c = threadIdx.x; c < 2 * H; c += blockDim.x) {
+    float t = 0.f;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) t += sp[k * 2 * H + c];
+    ws[int64_t(blockIdx.x) * 2 * H + c] = t;
+  }
+}
+
+// out0[c] (+)= sum_b ws[b][c], out1[c] (+)= sum_b ws[b][H + c] (c < H): block = 256 columns of the
+// 2H-wide partial rows x 8 warps over the G rows, combined in fp64 in warp order.
+__global__ void __launch_bounds__(256) reduce_partials2(const float* __restrict__ ws, int G, int H, float* out0,
+                                                        float* out1, int acc) {
+  __shared__ double red[8][32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int c = blockIdx.x * 32 + lane;
+  double s = 0.0;
+  if (c < 2 * H) {
+    int b = w;
+    // sixteen partial rows in flight per thread (the reduce is latency-bound, not bandwidth-bound)
+    for (; b + 8 * 15 < G; b += 8 * 16) {
+      float a[16];
+#pragma unroll
+      for (int k = 0; k < 16; ++k) a[k] = __ldcg(ws + int64_t(b + 8 * k) * 2 * H + c);
+#pragma unroll
+      for (int k = 0; k < 16; ++k) s += double(a[k]);
+    }
+    for (; b < G; b += 8) s += double(__ldcg(ws + int64_t(b) * 2 * H + c));
+  }
+  red[w][lane] = s;
+  __syncthreads();
+  if (w == 0 && c < 2 * H) {
+    double t = 0.0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) t += red[k][lane];
+    float* o = c < H ? out0 + c : out1 + (c - H);
+    *o = acc ? float(double(*o) + t) : float(t);
+  }
+}
+
 template <class T>
 bool ln_bwd_split_t(const void* dy, const void* x, const void* g, void* dx, int acc, float* ws, uint64_t ws_bytes,
                     float* dgamma, float* dbeta, int pacc, int64_t rows, int H, float eps, cudaStream_t st) {
   constexpr int V = Vec<T>::N;
   const int nch = (H + 32 * V - 1) / (32 * V);
   if (H % 8 || nch > 4 || !al16(dy) || !al16(x) || !al16(g) || !al16(dx)) return false;
+  if (sizeof(T) == 2 && rows >= 64) {  // bf16: one fused pass (x, dy read once)
+    int G = 2 * 148;
+    if (G > rows / 8) G = int(rows / 8);
+    if (uint64_t(G) * 2 * H * 4 + kTicketBytes > ws_bytes) G = int((ws_bytes - kTicketBytes) / (uint64_t(2 * H) * 4));
+    if (G >= 1) {
+      const int smem = 8 * 2 * H * 4;
+      static int attr_done[5] = {0, 0, 0, 0, 0};
+      auto DY = static_cast<const bf16*>(dy);
+      auto X = static_cast<const bf16*>(x);
+      auto Gm = static_cast<const bf16*>(g);
+      auto DX = static_cast<bf16*>(dx);
+      auto go = [&](auto kern) {
+        if (!attr_done[nch]) {
+          cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * 2 * 1024 * 4);
+          attr_done[nch] = 1;
+        }
+        kern<<<G, 256, smem, st>>>(DY, X, Gm, DX, acc, rows, H, eps, ws);
+      };
+      if (nch == 1) go(ln_bwd_fused_bf16<1>);
+      else if (nch == 2) go(ln_bwd_fused_bf16<2>);
+      else go(ln_bwd_fused_bf16<4>);
+      reduce_partials2<<<(2 * H + 31) / 32, 256, 0, st>>>(ws, G, H, dgamma, dbeta, pacc);
+      return true;
+    }
+  }
   const int cb = (H + 255) / 256;
   int G = int((rows + 15) / 16);
   int cap = (4 * 148) / cb;  // ~4 blocks per SM
@@ -855,6 +1123,17 @@ void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64
 void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, uint64_t ws_bytes, float* out, int acc,
                 const int* filter, int fval, cudaStream_t st) {
   const int cb = (N + 255) / 256;
+  if (dt == BF16 && !filter && N % 8 == 0 && (reinterpret_cast<uintptr_t>(x) % 16) == 0 && rows >= 64) {
+    // ~2 blocks of 256 threads per SM, at least 32 rows per block
+    int G = int(296 / cb);
+    if (G > rows / 32) G = int(rows / 32);
+    const int64_t ws_rows = int64_t((ws_bytes - kTicketBytes) / (uint64_t(N) * 4));
+    if (G > ws_rows) G = int(ws_rows);
+    if (G < 1) G = 1;
+    unsigned* tickets = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(ws) + ws_bytes - kTicketBytes);
+    colsum_bf16_kernel<<<dim3(cb, G), 256, 0, st>>>(static_cast<const bf16*>(x), rows, N, G, ws, tickets, out, acc);
+    return;
+  }
   int G = int((rows + 31) / 32);
   int cap = 592 / cb;  // ~4 blocks of 256 threads per SM
   if (dt == F32) {     // fp32 graphs keep the round-1 partition (see below)
