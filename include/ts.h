@@ -124,6 +124,7 @@ typedef struct {
   int64_t n_split_tensors; /* tensors with p_num > 1                                     */
   int64_t n_swap_tensors;
   int64_t n_recompute_tensors;
+  uint64_t recompute_cache_bytes; /* D-LRU recompute cache limit (0 = memory-centric, Fig. 11) */
 } ts_plan_stats_t;
 
 typedef struct {
@@ -197,6 +198,14 @@ ts_status ts_plan_get(const ts_plan_t* p, int32_t tensor_id, ts_tensor_cfg* out)
  * re-simulated.  Only TS_ACT tensors accept opt != RESIDE or p_num > 1. */
 ts_status ts_plan_set(ts_plan_t* p, const ts_tensor_cfg* cfg);
 ts_status ts_plan_stats(const ts_plan_t* p, ts_plan_stats_t* out);
+/* LRU-based recomputation ("execute as the speed-centric manner and abandon the
+ * least recently used intermediate tensor once the available memory is not enough";
+ * DESIGN.md reading D-LRU).  `cache_bytes` caps the regenerated micro-tensors kept
+ * resident across backward groups (checked at the end of each group, least recently used
+ * abandoned first); 0 = memory-centric (every backward group regenerates what it reads).
+ * ts_plan chooses it (fastest feasible of a small candidate set); this forces one.  The
+ * plan is re-expanded and re-simulated; the caller checks the new peak against its budget. */
+ts_status ts_plan_set_recompute_cache(ts_plan_t* p, uint64_t cache_bytes);
 /* Simulated allocation trace (R3, R11); *n = total events (buf may be NULL). */
 ts_status ts_plan_trace(const ts_plan_t* p, ts_alloc_event* buf, uint64_t cap, uint64_t* n);
 /* Augmented schedule as int32 quadruples (kind, op, k, aux) — kind 0 F, 1 B, 2 R,

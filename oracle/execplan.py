@@ -18,8 +18,8 @@ from . import ops as O
 F = np.float64
 
 
-def execute(graph, cfg, params, inputs, step=0):
-    items, f_alloc, f_free, fwd_end, an = sim.expand(graph, cfg)
+def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
+    items, f_alloc, f_free, fwd_end, an = sim.expand(graph, cfg, cache_bytes=cache_bytes)
     ts, ops = graph["tensors"], graph["ops"]
     n, B = an.n, graph["samples"]
     pval = {t["id"]: np.asarray(params[t["name"]], F) for t in ts if t["kind"] == "param"}

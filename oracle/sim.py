@@ -22,6 +22,7 @@ DESIGN.md §4 fixes:
 
 from __future__ import annotations
 
+from collections import OrderedDict
 from dataclasses import dataclass, field
 
 DTYPE_BYTES = {"f32": 4, "bf16": 2, "i32": 4}
@@ -241,9 +242,17 @@ def default_cfg(graph):
     return {t["id"]: (RESIDE, 1, 1) for t in graph["tensors"]}
 
 
-def expand(graph, cfg, order=None, an=None):
+def expand(graph, cfg, order=None, an=None, cache_bytes=0):
     """Augmented schedule: returns (items, alloc_at, free_after, fwd_end) where
-    alloc_at / free_after map item index -> ordered list of (key, piece)."""
+    alloc_at / free_after map item index -> ordered list of (key, piece).
+
+    cache_bytes > 0 selects the LRU-based recomputation of P:L294 (DESIGN.md reading
+    D-LRU): "execute as the speed-centric manner and abandon the least recently used
+    intermediate tensor once the available memory is not enough".  A regenerated piece
+    stays resident for later backward groups (a later group that reads it replays
+    nothing); at the end of every group the least recently used regenerated pieces
+    are abandoned until the resident ones total <= cache_bytes.  cache_bytes = 0 is
+    the memory-centric strategy (Fig. 11: everything regenerated per group)."""
     an = an or analyze(graph)
     order = order if order is not None else schedule(graph)
     ts, ops = graph["tensors"], graph["ops"]
@@ -289,6 +298,10 @@ def expand(graph, cfg, order=None, an=None):
             items.append(it)
     fwd_end = len(items)
 
+    def piece_nbytes(t):
+        return an.bytes_[t] // p_of(t)
+
+    cache = OrderedDict()  # regenerated pieces still resident, least recently used first
     gid = 0
     for o in reversed(order):
         if not an.has_bwd[o]:
@@ -301,6 +314,10 @@ def expand(graph, cfg, order=None, an=None):
             def need(t, j):
                 if ts[t]["kind"] != "act" or opt_of(t) != RECOMPUTE or (t, j) in live_temp:
                     return
+                if (t, j) in cache:  # D-LRU hit: resident since an earlier group
+                    cache.move_to_end((t, j))
+                    live_temp.add((t, j))
+                    return
                 po = an.producer[t]
                 Q = P_op(po)
                 pt = p_of(t)
@@ -312,6 +329,7 @@ def expand(graph, cfg, order=None, an=None):
                     r.writes = [(t, j)]
                     group.append(r)
                 live_temp.add((t, j))
+                cache[(t, j)] = piece_nbytes(t)
 
             saved_pieces = [(t, piece(t, k, P)) for t in an.saved[o]]
             if ops[o]["kind"] in BATCH_REDUCE and k == 0:
@@ -338,6 +356,9 @@ def expand(graph, cfg, order=None, an=None):
             group.append(b)
             items.extend(group)
             gid += 1
+            # abandon least recently used regenerated pieces beyond the cache limit
+            while cache and sum(cache.values()) > cache_bytes:
+                cache.popitem(last=False)
 
     # ---- lifetimes -------------------------------------------------------------
     touches = {}
@@ -384,15 +405,23 @@ def expand(graph, cfg, order=None, an=None):
             pos = max(min(bw) - lead, fwd_end)
             swap_in_before.setdefault(pos, []).append(pc)
             free_after.setdefault(max(bw), []).append(pc)
-        else:  # RECOMPUTE: forward lifetime, then per-group temporaries
+        else:  # RECOMPUTE: forward lifetime, then one residency per regeneration
             free_after.setdefault(max(fw), []).append(pc)
-            by_group = {}
+            # a residency starts at the replay writing the piece and ends at its last
+            # touch before the next replay of it (memory-centric: one per group)
+            # (a regeneration may be several replays of one group, when the producer has
+            # more micro-ops than the piece: the group's first one starts the residency)
+            seen, starts = set(), []
             for i in bw:
-                by_group.setdefault(items[i].group, []).append(i)
-            for g, gi in by_group.items():
-                alloc_at.setdefault(min(gi), []).append(pc)
-                free_after.setdefault(max(gi), []).append(pc)
-                temp_spans.append((pc, min(gi), max(gi)))
+                if items[i].kind == "R" and pc in items[i].writes and items[i].group not in seen:
+                    seen.add(items[i].group)
+                    starts.append(i)
+            for a, st in enumerate(starts):
+                end = starts[a + 1] if a + 1 < len(starts) else None
+                span = [i for i in bw if i >= st and (end is None or i < end)]
+                alloc_at.setdefault(st, []).append(pc)
+                free_after.setdefault(max(span), []).append(pc)
+                temp_spans.append((pc, st, max(span)))
 
     # ---- final item list with SO / SI items -----------------------------------
     final = []
@@ -435,9 +464,9 @@ class SimResult:
     h2d_bytes: int
 
 
-def simulate(graph, cfg=None, order=None, capacity=INF):
+def simulate(graph, cfg=None, order=None, capacity=INF, cache_bytes=0):
     cfg = cfg or default_cfg(graph)
-    items, f_alloc, f_free, fwd_end, an = expand(graph, cfg, order)
+    items, f_alloc, f_free, fwd_end, an = expand(graph, cfg, order, cache_bytes=cache_bytes)
     ts = graph["tensors"]
     n = an.n
     base = static_bytes(graph)

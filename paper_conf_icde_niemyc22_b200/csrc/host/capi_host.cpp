@@ -159,6 +159,16 @@ ts_status ts_plan_stats(const ts_plan_t* p, ts_plan_stats_t* out) {
     out->n_swap_tensors += c.opt == TS_SWAP;
     out->n_recompute_tensors += c.opt == TS_RECOMPUTE;
   }
+  out->recompute_cache_bytes = s.cache;
+  return TS_OK;
+}
+
+ts_status ts_plan_set_recompute_cache(ts_plan_t* p, uint64_t cache_bytes) {
+  if (!p) return set_error("null argument"), TS_ERR_ARG;
+  p->st.cache = cache_bytes;
+  Profile pr;
+  profile_analytic(*p->graph, default_hw(), pr);
+  plan_refresh(*p->graph, p->st, &pr);
   return TS_OK;
 }
 
@@ -212,11 +222,12 @@ ts_status ts_plan_grad_buckets(const ts_plan_t* p, uint64_t bucket_bytes, int64_
   return TS_OK;
 }
 
-// Serialized form: magic, n_tensors, budget, then (opt, p, dim, lead) per tensor.
+// Serialized form: magic, n_tensors, budget, then (opt, p, dim, lead) per tensor, then the
+// D-LRU recompute cache limit.
 ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n) {
   if (!p || !n) return set_error("null argument"), TS_ERR_ARG;
   const int nt = p->graph->n();
-  uint64_t need = 16 + 16ull * nt;
+  uint64_t need = 16 + 16ull * nt + 8;
   *n = need;
   if (!buf) return TS_OK;
   if (cap < need) return set_error("buffer too small"), TS_ERR_ARG;
@@ -231,6 +242,7 @@ ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_
     w[4 + 4 * t + 2] = c.dim;
     w[4 + 4 * t + 3] = c.lead;
   }
+  std::memcpy(w + 4 + 4 * nt, &p->st.cache, 8);
   return TS_OK;
 }
 
@@ -238,7 +250,7 @@ ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, 
   if (!g || !buf || !out) return set_error("null argument"), TS_ERR_ARG;
   auto* r = static_cast<const int32_t*>(buf);
   const int nt = g->g.n();
-  if (n < 16 || r[0] != 0x54535031 || r[1] != nt || n < 16 + 16ull * nt)
+  if (n < 16 || r[0] != 0x54535031 || r[1] != nt || n < 16 + 16ull * nt + 8)
     return set_error("not a plan for this graph"), TS_ERR_ARG;
   std::unique_ptr<ts_plan_t> p(new_plan(g));
   std::memcpy(&p->budget, r + 2, 8);
@@ -249,6 +261,7 @@ ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, 
     c.dim = r[4 + 4 * t + 2];
     c.lead = r[4 + 4 * t + 3];
   }
+  std::memcpy(&p->st.cache, r + 4 + 4 * nt, 8);
   Profile pr;
   profile_analytic(g->g, default_hw(), pr);
   plan_refresh(g->g, p->st, &pr);

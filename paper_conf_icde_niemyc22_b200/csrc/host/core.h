@@ -113,7 +113,8 @@ struct SimResult {
 
 int piece_count(const Graph& g, const std::vector<Cfg>& cfg, int key);
 uint64_t piece_bytes(const Graph& g, const std::vector<Cfg>& cfg, int key);
-void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex);
+// cache_bytes: D-LRU recompute cache limit (0 = memory-centric, Fig. 11)
+void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t cache_bytes = 0);
 // capacity = kInf for planning; the runtime uses the slab size (identical trace if it fits).
 bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, uint64_t capacity,
               SimResult& r, std::vector<std::vector<std::pair<PieceKey, uint64_t>>>* placements = nullptr);
@@ -157,6 +158,7 @@ ts_hw default_hw();
 
 struct PlanState {
   std::vector<Cfg> cfg;
+  uint64_t cache = 0;  // D-LRU recompute cache limit (bytes); 0 = memory-centric
   Expansion ex;
   SimResult sim;
   double predicted_s = 0, flop = 0;

@@ -4,7 +4,10 @@
 //                        best-fit allocation over one pre-allocated pool
 //   P:L281             — swap-out begins at generation, swap-in at the previous op
 //   P:L291             — compute / D2H / H2D streams, pre-allocated pool
-//   P:L293-294 Fig. 11 — memory-centric recompute (regenerate for every backward use)
+//   P:L293-294 Fig. 11 — memory-centric recompute (regenerate for every backward use);
+//                        with cache_bytes > 0 the LRU-based hybrid (reading D-LRU): regenerated
+//                        pieces stay resident for later groups, least recently used ones are
+//                        abandoned at the end of a group beyond cache_bytes
 //   P:L56, P:L134      — allocate at the beginning, free at the end of an operation
 #include <algorithm>
 #include <functional>
@@ -27,7 +30,7 @@ uint64_t piece_bytes(const Graph& g, const std::vector<Cfg>& cfg, int key) {
   return g.t[t].bytes / uint64_t(piece_count(g, cfg, key));
 }
 
-void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
+void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t cache_bytes) {
   const int n = g.n();
   ex = Expansion();
   ex.P.assign(g.ops.size(), 1);
@@ -66,6 +69,13 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
   }
   ex.fwd_end = (int)items.size();
   // ---- backward phase: reverse order, replays inline --------------------------
+  // D-LRU cache: regenerated pieces still resident, least recently used first
+  std::vector<std::pair<PieceKey, uint64_t>> cache;
+  auto cache_find = [&](PieceKey pc) {
+    for (size_t i = 0; i < cache.size(); ++i)
+      if (cache[i].first == pc) return int(i);
+    return -1;
+  };
   int gid = 0;
   for (auto rit = g.order.rbegin(); rit != g.order.rend(); ++rit) {
     const Op& op = g.ops[*rit];
@@ -78,6 +88,14 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
         const Tensor& x = g.t[t];
         if (x.kind != TS_ACT || cfg[t].opt != TS_RECOMPUTE) return;
         if (regenerated.count(pk(t, j))) return;
+        int ci = cache_find(pk(t, j));
+        if (ci >= 0) {  // D-LRU hit: resident since an earlier group; now most recently used
+          auto e = cache[ci];
+          cache.erase(cache.begin() + ci);
+          cache.push_back(e);
+          regenerated.insert(pk(t, j));
+          return;
+        }
         const Op& po = g.ops[x.producer];
         int Q = ex.P[po.id];
         int pt = piece_count(g, cfg, t);
@@ -95,6 +113,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
           group.push_back(std::move(r));
         }
         regenerated.insert(pk(t, j));
+        cache.push_back({pk(t, j), piece_bytes(g, cfg, t)});
       };
       std::vector<PieceKey> saved;
       for (int t : op.saved) saved.push_back(pk(t, piece(t, k, P)));
@@ -125,6 +144,13 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
       group.push_back(std::move(b));
       for (auto& it : group) items.push_back(std::move(it));
       ++gid;
+      // abandon the least recently used regenerated pieces beyond the cache limit
+      uint64_t used = 0;
+      for (auto& e : cache) used += e.second;
+      while (!cache.empty() && used > cache_bytes) {
+        used -= cache.front().second;
+        cache.erase(cache.begin());
+      }
     }
   }
   const int nitems = (int)items.size();
@@ -168,18 +194,25 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex) {
       int pos = std::max(first_bw - std::max(1, cfg[key].lead), ex.fwd_end);
       si_before[pos].push_back(pc);
       free_after[lastt].push_back(pc);
-    } else {  // recompute: forward lifetime, then one temporary per backward group
+    } else {  // recompute: forward lifetime, then one residency per regeneration
       free_after[last_fw].push_back(pc);
-      std::map<int, std::pair<int, int>> span;
+      // a residency starts at the group's first replay writing the piece and ends at its
+      // last touch before the next regeneration (memory-centric: one per group)
+      std::vector<int> starts;
+      std::set<int> seen;
       for (int i : idx)
-        if (i >= ex.fwd_end) {
-          auto it = span.find(items[i].group);
-          if (it == span.end()) span[items[i].group] = {i, i};
-          else it->second.second = i;
+        if (i >= ex.fwd_end && items[i].kind == IT_R && !seen.count(items[i].group) &&
+            std::find(items[i].writes.begin(), items[i].writes.end(), pc) != items[i].writes.end()) {
+          seen.insert(items[i].group);
+          starts.push_back(i);
         }
-      for (auto& [gg, se] : span) {
-        alloc_at[se.first].push_back(pc);
-        free_after[se.second].push_back(pc);
+      for (size_t a = 0; a < starts.size(); ++a) {
+        const int st = starts[a], end = a + 1 < starts.size() ? starts[a + 1] : nitems;
+        int last = st;
+        for (int i : idx)
+          if (i >= st && i < end) last = std::max(last, i);
+        alloc_at[st].push_back(pc);
+        free_after[last].push_back(pc);
       }
     }
   }

@@ -243,7 +243,7 @@ double flops_of(const Graph& g, const PlanState& ps) {
 }  // namespace
 
 void plan_refresh(const Graph& g, PlanState& ps, const Profile* pr) {
-  expand(g, ps.cfg, ps.ex);
+  expand(g, ps.cfg, ps.ex, ps.cache);
   simulate(g, ps.cfg, ps.ex, kInf, ps.sim);
   ps.flop = flops_of(g, ps);
   if (pr) {
@@ -290,6 +290,7 @@ void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& 
   const int n = g.n();
   auto try_cfg = [&](const std::vector<Cfg>& cfg, PlanState& out) {
     out.cfg = cfg;
+    out.cache = ps.cache;
     plan_refresh(g, out, &pr);
     return max_top(out) <= budget;
   };
@@ -302,6 +303,7 @@ void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& 
     std::vector<Cfg> cfg = ps.cfg;
     cfg[t] = Cfg();
     tmp.cfg = cfg;
+    tmp.cache = ps.cache;
     plan_refresh(g, tmp, &pr);
     order.push_back({ps.predicted_s - tmp.predicted_s, t});
   }
@@ -333,6 +335,32 @@ void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& 
   }
 }
 
+// LRU-based recomputation (reading D-LRU): the greedy plan is made memory-centric;
+// then the recompute cache limit is chosen as the fastest feasible of {unbounded, the
+// plan's headroom x 8, x 4, x 2, x 1, x 1/2} (headroom = budget - simulated peak, so the
+// cached pieces only use memory the memory-centric plan leaves free), and with a cache the
+// D-R8c post-pass runs again (decisions that no longer pay can be reverted).
+void plan_lru(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps) {
+  bool any = false;
+  for (const Cfg& c : ps.cfg) any |= c.opt == TS_RECOMPUTE;
+  if (!any) return;
+  const uint64_t head = budget > max_top(ps) ? budget - max_top(ps) : 0;
+  PlanState best = ps;
+  const uint64_t caps[] = {~uint64_t(0), 8 * head, 4 * head, 2 * head, head, head / 2};
+  for (uint64_t cap : caps) {
+    if (cap == 0) continue;
+    PlanState cand;
+    cand.cfg = ps.cfg;
+    cand.cache = cap;
+    plan_refresh(g, cand, &pr);
+    if (max_top(cand) <= budget && cand.predicted_s < best.predicted_s - 1e-9) best = std::move(cand);
+  }
+  if (best.cache != ps.cache) {
+    ps = std::move(best);
+    plan_refine(g, budget, pr, ps);
+  }
+}
+
 ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps) {
   const int n = g.n();
   ps.cfg.assign(n, Cfg());
@@ -355,6 +383,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       }
     if (bi < 0) {
       plan_refine(g, budget, pr, ps);
+      plan_lru(g, budget, pr, ps);
       return TS_OK;
     }
     // bottleneck op and phase

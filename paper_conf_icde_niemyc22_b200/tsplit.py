@@ -43,7 +43,7 @@ class PlanStats(C.Structure):
                 ("d2h_bytes", C.c_uint64), ("h2d_bytes", C.c_uint64), ("n_items", C.c_int64),
                 ("n_compute", C.c_int64), ("n_replay", C.c_int64), ("predicted_s", C.c_double),
                 ("compute_flop", C.c_double), ("n_split_tensors", C.c_int64), ("n_swap_tensors", C.c_int64),
-                ("n_recompute_tensors", C.c_int64)]
+                ("n_recompute_tensors", C.c_int64), ("recompute_cache_bytes", C.c_uint64)]
 
 
 class AllocEvent(C.Structure):
@@ -97,6 +97,7 @@ def lib():
             "ts_plan_get": (i32, [vp, i32, P(TensorCfg)]),
             "ts_plan_set": (i32, [vp, P(TensorCfg)]),
             "ts_plan_stats": (i32, [vp, P(PlanStats)]),
+            "ts_plan_set_recompute_cache": (i32, [vp, C.c_uint64]),
             "ts_plan_trace": (i32, [vp, P(AllocEvent), u64, P(u64)]),
             "ts_plan_items": (i32, [vp, P(i32), u64, P(u64)]),
             "ts_plan_grad_buckets": (i32, [vp, u64, P(i64), u64, P(u64)]),
@@ -300,6 +301,10 @@ class Plan:
     def set(self, tid, opt=RESIDE, p_num=1, prefetch_lead=1, dim=0):
         c = TensorCfg(tid, opt, p_num, dim, prefetch_lead)
         check(lib().ts_plan_set(self.h, C.byref(c)))
+
+    def set_recompute_cache(self, cache_bytes: int):
+        """D-LRU recompute cache limit in bytes (0 = memory-centric; 2**64-1 = unbounded)."""
+        check(lib().ts_plan_set_recompute_cache(self.h, C.c_uint64(cache_bytes)))
 
     def stats(self):
         s = PlanStats()

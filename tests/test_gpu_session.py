@@ -209,3 +209,31 @@ def test_linear_gelu_fusion_equals_unfused(fused_attention, plan):
     params, inputs = gen.init_params(g), gen.make_inputs(g)
     _, ogb, _, _ = net.train_step(g, params, inputs, storage="bf16")
     assert global_rel_err(g1, ogb) <= 2e-2
+
+
+@pytest.mark.parametrize("cache", [1 << 20, 2 ** 64 - 1])
+def test_lru_recompute_cache_session(cache):
+    """D-LRU recompute cache on the GPU: fewer replays, the runtime's allocation trace is
+    the simulator's (regenerated pieces held across backward groups), and the gradients
+    equal the memory-centric plan's (fp32: 1e-6) and the oracle's (1e-5)."""
+    g = graphs.config_graph("bert_tiny", dtype="f32", fused_attention=True)
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    cfg = {names[f"l{i}.{x}"]: (tsplit.RECOMPUTE, 1, 1) for i in (0, 1) for x in ("ffn1", "gelu", "ln1", "q", "k")}
+    cfg[names["l0.v"]] = (tsplit.RECOMPUTE, 2, 1)
+    G = tsplit.Graph(g)
+    out = []
+    for c in (0, cache):
+        P = tsplit.Plan.default(G)
+        for t, (o, p, lead) in cfg.items():
+            P.set(t, o, p, lead)
+        P.set_recompute_cache(c)
+        S = tsplit.Session(G, P)
+        params, inputs = gen.init_params(g), gen.make_inputs(g)
+        S.set_params(params)
+        loss = S.step(tsplit.inputs_to_device(G, inputs))
+        assert S.trace() == [tuple(e) for e in sim.simulate(g, {**sim.default_cfg(g), **cfg}, cache_bytes=c).trace]
+        out.append((loss, S.grads(), P.stats()["n_replay"]))
+    assert out[1][2] < out[0][2]
+    assert max(rel_errs(out[1][1], out[0][1]).values()) <= 1e-6
+    ol, og = _oracle(g)
+    assert max(rel_errs(out[1][1], og).values()) <= 1e-5

@@ -17,11 +17,13 @@ def _apply(plan, cfg, acts):
         plan.set(t, o, p, lead)
 
 
-def _compare(g, cfg):
+def _compare(g, cfg, cache=0):
     G = tsplit.Graph(g)
     plan = tsplit.Plan.default(G)
     _apply(plan, cfg, brute.act_tensors(g))
-    ref = sim.simulate(g, cfg)
+    if cache:
+        plan.set_recompute_cache(cache)
+    ref = sim.simulate(g, cfg, cache_bytes=cache)
     got = plan.trace()
     assert len(got) == len(ref.trace)
     for a, b in zip(got, ref.trace):
@@ -178,3 +180,35 @@ def test_fused_attention_large_default_and_planned():
     assert st["peak_extent"] == sim.simulate(g, sim.default_cfg(g)).peak_extent
     P = tsplit.Plan.plan(G, st["static_bytes"] + (st["peak_extent"] - st["static_bytes"]) // 4)
     assert P.stats()["peak_extent"] <= st["static_bytes"] + (st["peak_extent"] - st["static_bytes"]) // 4
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_trace_bit_exact_lru_recompute_cache(seed):
+    """D-LRU: the C++ expansion with a recompute cache limit reproduces the oracle's
+    items, replay count and allocation trace bit for bit (bf16 BERT-tiny, random plans)."""
+    g = graphs.config_graph("bert_tiny")
+    rnd = random.Random(100 + seed)
+    acts = brute.act_tensors(g)
+    cfg = sim.default_cfg(g)
+    for t in acts:
+        cfg[t] = (rnd.choice([sim.RESIDE, sim.RECOMPUTE, sim.RECOMPUTE, sim.SWAP]), rnd.choice([1, 1, 2, 4]), 1)
+    for cache in (1 << 16, 1 << 20, 2 ** 64 - 1):
+        _compare(g, cfg, cache)
+
+
+def test_planner_lru_cache_feasible_and_not_slower():
+    """ts_plan's D-LRU post-pass keeps the plan within the budget and never predicts a
+    slower step than the memory-centric plan it starts from; the plan serializes with it."""
+    g = graphs.config_graph("bert_large", layers=4)
+    G = tsplit.Graph(g)
+    st = tsplit.Plan.default(G).stats()
+    budget = st["static_bytes"] + int(0.25 * (st["peak_extent"] - st["static_bytes"]))
+    P = tsplit.Plan.plan(G, budget)
+    s = P.stats()
+    assert s["peak_extent"] <= budget
+    mc = tsplit.Plan.deserialize(G, P.serialize())
+    assert mc.stats()["recompute_cache_bytes"] == s["recompute_cache_bytes"]
+    assert mc.trace() == P.trace()
+    mc.set_recompute_cache(0)
+    assert s["predicted_s"] <= mc.stats()["predicted_s"] + 1e-12
+    assert s["n_replay"] <= mc.stats()["n_replay"]

@@ -264,3 +264,64 @@ def test_pool_best_fit_and_tail_rule():
     x = q.alloc(512); y = q.alloc(256)
     q.release(x, 512)           # hole 512 at 0, tail 256 at 768
     assert q.alloc(200) == 0    # tail is used only when nothing else fits
+
+
+# ------------------------------------------------------------- D-LRU recompute cache
+def _chain(N):
+    b = graphs.GraphBuilder("chain", "f32", 2)
+    X = b.tensor("X", (2, 4), "input")
+    Y = b.tensor("labels", (2,), "label", dtype="i32")
+    W = b.param("W", (4, 4)); bb = b.param("b", (4,))
+    a = b.op("linear", "op1", [X, W, bb], (2, 4))
+    acts = [a]
+    for i in range(2, N + 1):
+        a = b.op("gelu", f"op{i}", [a], (2, 4))
+        acts.append(a)
+    b.op("xent", "loss", [a, Y], (1,), out_dtype="f32")
+    g = b.done()
+    cfg = sim.default_cfg(g)
+    for t in acts:
+        cfg[t] = (sim.RECOMPUTE, 1, 1)
+    return g, cfg
+
+
+@pytest.mark.parametrize("N", [1, 2, 3, 5, 8])
+def test_lru_recompute_counts_on_the_fig11_chain(N):
+    """the speed-centric strategy recomputes the N ancestors once (O(N)); the
+    memory-centric one N(N+1)/2 times; the LRU hybrid keeps the most recently used
+    regenerated tensors up to the memory limit.  On the chain, backward group i needs
+    op_{N-i}'s output: with room for K regenerated tensors (K >= 2) every miss replays
+    the chain up to the needed tensor and the K - 1 tensors before it stay for the next
+    K - 1 groups, so the replays are N + (N - K) + (N - 2K) + ...; with K = 1 the one kept
+    tensor is always the one just consumed, i.e. memory-centric again."""
+    g, cfg = _chain(N)
+    piece = 2 * 4 * 4  # one [2, 4] fp32 activation
+    assert sim.simulate(g, cfg, cache_bytes=0).n_replay == N * (N + 1) // 2
+    assert sim.simulate(g, cfg, cache_bytes=piece).n_replay == N * (N + 1) // 2
+    assert sim.simulate(g, cfg, cache_bytes=2 ** 64 - 1).n_replay == N
+    for K in (2, 3):
+        want = sum(N - K * i for i in range(N) if N - K * i >= 1)
+        assert sim.simulate(g, cfg, cache_bytes=K * piece).n_replay == want
+    # caching trades memory for replays: the unbounded cache holds the whole chain at once
+    if N >= 3:
+        assert sim.simulate(g, cfg, cache_bytes=2 ** 64 - 1).peak_live > sim.simulate(g, cfg).peak_live
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_t1_lru_plans_compute_the_unsplit_gradients(seed):
+    """T1 with the recompute cache: any plan and any cache limit give the unsplit
+    gradients (fp64, 1e-12), and the simulator finds every read resident."""
+    g = graphs.mlp(batch=4, hidden=8, depth=3, in_dim=8, classes=3)
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    ref_loss, ref_g, _, _ = net.train_step(g, params, inputs)
+    rnd = random.Random(seed)
+    acts = brute.act_tensors(g)
+    for _ in range(4):
+        cfg = sim.default_cfg(g)
+        for t in acts:
+            cfg[t] = (rnd.choice([sim.RESIDE, sim.RECOMPUTE, sim.RECOMPUTE, sim.SWAP]), rnd.choice([1, 2, 4]), 1)
+        cache = rnd.choice([0, 64, 256, 1024, 2 ** 64 - 1])
+        loss, grads = execplan.execute(g, cfg, params, inputs, cache_bytes=cache)
+        sim.simulate(g, cfg, cache_bytes=cache)
+        assert abs(loss - ref_loss) <= 1e-12 * abs(ref_loss)
+        assert max(rel_errs(grads, ref_g).values()) <= 1e-12
