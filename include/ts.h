@@ -193,6 +193,13 @@ ts_status ts_plan_default(const ts_graph_t* g, ts_plan_t** out);
  * may be NULL (analytic model with B200 defaults).  Returns TS_ERR_INFEASIBLE
  * when no candidate remains. */
 ts_status ts_plan(const ts_graph_t* g, uint64_t budget_bytes, const ts_profile_t* profile, ts_plan_t** out);
+/* ts_plan with planner options (the breakdown of P:L457-467):
+ *   TS_PLAN_NO_SPLIT        "TSPLIT w/o Split": Alg. 2 without split candidates (steps 1, 3 only)
+ *   TS_PLAN_MEMORY_CENTRIC  no LRU recompute cache (every backward group regenerates, Fig. 11) */
+#define TS_PLAN_NO_SPLIT 1u
+#define TS_PLAN_MEMORY_CENTRIC 2u
+ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profile_t* profile, uint32_t flags,
+                     ts_plan_t** out);
 ts_status ts_plan_get(const ts_plan_t* p, int32_t tensor_id, ts_tensor_cfg* out);
 /* Forced configuration (Fig. 9 set_config); the plan is re-expanded and
  * re-simulated.  Only TS_ACT tensors accept opt != RESIDE or p_num > 1. */

@@ -90,7 +90,13 @@ ts_status ts_plan_default(const ts_graph_t* g, ts_plan_t** out) {
 }
 
 ts_status ts_plan(const ts_graph_t* g, uint64_t budget_bytes, const ts_profile_t* profile, ts_plan_t** out) {
+  return ts_plan_ex(g, budget_bytes, profile, 0u, out);
+}
+
+ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profile_t* profile, uint32_t flags,
+                     ts_plan_t** out) {
   if (!g || !out) return set_error("null argument"), TS_ERR_ARG;
+  if (flags & ~(TS_PLAN_NO_SPLIT | TS_PLAN_MEMORY_CENTRIC)) return set_error("unknown planner flags"), TS_ERR_ARG;
   std::unique_ptr<ts_plan_t> p(new_plan(g));
   Profile local;
   const Profile* pr = profile ? &profile->pr : nullptr;
@@ -98,7 +104,7 @@ ts_status ts_plan(const ts_graph_t* g, uint64_t budget_bytes, const ts_profile_t
     profile_analytic(g->g, default_hw(), local);
     pr = &local;
   }
-  ts_status st = plan_greedy(g->g, budget_bytes, *pr, p->st);
+  ts_status st = plan_greedy(g->g, budget_bytes, *pr, p->st, flags);
   if (st != TS_OK) return st;
   p->budget = budget_bytes;
   *out = p.release();

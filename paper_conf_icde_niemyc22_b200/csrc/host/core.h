@@ -164,7 +164,7 @@ struct PlanState {
   double predicted_s = 0, flop = 0;
 };
 void plan_refresh(const Graph& g, PlanState& ps, const Profile* pr);
-ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps);
+ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps, uint32_t flags = 0);
 void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps);
 
 }  // namespace ts

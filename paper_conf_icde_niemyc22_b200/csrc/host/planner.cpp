@@ -361,7 +361,7 @@ void plan_lru(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps)
   }
 }
 
-ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps) {
+ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps, uint32_t flags) {
   const int n = g.n();
   ps.cfg.assign(n, Cfg());
   if (g.static_bytes > budget) {
@@ -383,7 +383,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       }
     if (bi < 0) {
       plan_refine(g, budget, pr, ps);
-      plan_lru(g, budget, pr, ps);
+      if (!(flags & TS_PLAN_MEMORY_CENTRIC)) plan_lru(g, budget, pr, ps);
       return TS_OK;
     }
     // bottleneck op and phase
@@ -543,14 +543,16 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       step1 = sw;
       step1.insert(step1.end(), rc.begin(), rc.end());
     }
-    // step 2: split options on the bottleneck op's own activations (Eq. 6)
+    // step 2: split options on the bottleneck op's own activations (Eq. 6); the
+    // "TSPLIT w/o Split" ablation of P:L463 plans with steps 1 and 3 only
+    const bool no_split = flags & TS_PLAN_NO_SPLIT;
     std::vector<int> split_cands;
     for (int x : g.ops[bop].in)
       if (g.t[x].kind == TS_ACT && !g.t[x].is_loss) split_cands.push_back(x);
     for (int x : g.ops[bop].out)
       if (g.t[x].kind == TS_ACT && !g.t[x].is_loss) split_cands.push_back(x);
     for (int t : split_cands)
-      for (int p = 2; p <= 16; p *= 2) {
+      for (int p = 2; p <= 16 && !no_split; p *= 2) {
         if (p <= ps.cfg[t].p || g.samples % p) continue;
         for (int opt : {TS_RESIDE, TS_SWAP, TS_RECOMPUTE}) {
           if (opt != TS_RESIDE && first_bw[t] < 0) continue;
@@ -567,7 +569,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
     for (int t : live) {
       const Tensor& x = g.t[t];
       if (x.kind != TS_ACT || x.is_loss || own.count(t) || ps.cfg[t].opt != TS_RECOMPUTE) continue;
-      for (int p = ps.cfg[t].p * 2; p <= 16; p *= 2) {
+      for (int p = ps.cfg[t].p * 2; p <= 16 && !no_split; p *= 2) {
         if (g.samples % p) break;
         Cand2 c;
         c.birth = birth[t];
@@ -580,7 +582,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
     // p at once.  Under op-major execution (R10) an input piece is released while the
     // output is produced only when both sides are split, so single-tensor splits can
     // show no gain (dM = 0) where the joint one does (e.g. VGG conv1 -> relu1).
-    for (int p = 2; p <= 16; p *= 2) {
+    for (int p = 2; p <= 16 && !no_split; p *= 2) {
       if (g.samples % p) continue;
       Cand2 c;
       for (int t : split_cands)

@@ -94,6 +94,7 @@ def lib():
             "ts_profile_destroy": (None, [vp]),
             "ts_plan_default": (i32, [vp, P(vp)]),
             "ts_plan": (i32, [vp, u64, vp, P(vp)]),
+            "ts_plan_ex": (i32, [vp, C.c_uint64, vp, C.c_uint32, P(vp)]),
             "ts_plan_get": (i32, [vp, i32, P(TensorCfg)]),
             "ts_plan_set": (i32, [vp, P(TensorCfg)]),
             "ts_plan_stats": (i32, [vp, P(PlanStats)]),
@@ -274,9 +275,12 @@ class Plan:
         return cls(graph, h)
 
     @classmethod
-    def plan(cls, graph, budget_bytes, profile: Profile | None = None):
+    def plan(cls, graph, budget_bytes, profile: Profile | None = None, no_split=False, memory_centric=False):
+        """ts_plan / ts_plan_ex: no_split = the "TSPLIT w/o Split" ablation (P:L463),
+        memory_centric = no LRU recompute cache (Fig. 11 strategy only)."""
         h = C.c_void_p()
-        check(lib().ts_plan(graph.h, int(budget_bytes), profile.h if profile else None, C.byref(h)))
+        flags = (1 if no_split else 0) | (2 if memory_centric else 0)
+        check(lib().ts_plan_ex(graph.h, int(budget_bytes), profile.h if profile else None, flags, C.byref(h)))
         return cls(graph, h)
 
     @classmethod
