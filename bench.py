@@ -336,11 +336,21 @@ def main():
     dev_inputs = tsplit.inputs_to_device(G, arrays, device=f"cuda:{local}")
     t0 = time.time()
     blob, pcie, pst0 = None, None, None
+    plan_profile = "measured (rank 0)"
     if rank == 0:
         # profile every op (and split widths) on the GPU before planning
         prof = tsplit.Profile.measure(G, dev_inputs, max_p=4, device=local) if not args.analytic_profile else None
         pcie = prof.pcie() if prof else None
-        plan0 = tsplit.Plan.plan(G, budget, prof)
+        plan_profile = "measured" if prof else "analytic"
+        try:
+            plan0 = tsplit.Plan.plan(G, budget, prof)
+        except tsplit.TsError as e:
+            # Alg. 2 is a path-dependent greedy heuristic: when the measured profile leads it
+            # into a dead end, plan with the analytic cost model instead (reported in config)
+            if prof is None or e.status != "ERR_INFEASIBLE":
+                raise
+            plan_profile = f"analytic (the measured-profile plan was infeasible: {str(e)[:80]})"
+            plan0 = tsplit.Plan.plan(G, budget, None)
         pst0 = plan0.stats()  # predicted time with the measured profile
         blob = plan0.serialize()
     plan_s = time.time() - t0
@@ -451,7 +461,8 @@ def main():
                  "recompute_tensors": pst["n_recompute_tensors"], "replays": pst["n_replay"],
                  "d2h_bytes": pst["d2h_bytes"], "h2d_bytes": pst["h2d_bytes"],
                  "step_flop": pst["compute_flop"], "predicted_ms": pst["predicted_s"] * 1e3,
-                 "profile_and_planning_s": round(plan_s, 2),
+                 "profile_and_planning_s": round(plan_s, 2), "planned_with": plan_profile,
+                 "recompute_cache_bytes": pst["recompute_cache_bytes"],
                  "measured_pcie_gbs": [round(x / 1e9, 1) for x in pcie] if pcie else None},
         "l2": "no flush needed: every step streams >10 GB of activations through a 126 MB L2"
               if not cnn else "no flush needed: every step streams several GB of activations through a 126 MB L2",

@@ -32,10 +32,11 @@ def round_bf16(x):
 
 
 # ---------------------------------------------------------------------------
-# Philox4x32-10 counter-based RNG (Salmon et al., SC'11), SURVEY.md §8(c) R15.
-# Element idx draws word (idx & 3) of Philox(counter = (c_lo, c_hi, step, 0),
-# key = (seed, 0x5453504C)) with c = idx >> 2 (one Philox call feeds four
-# consecutive elements), and keep = (word >= floor(p * 2^32)).  Pure integer
+# Philox4x32-10 counter-based RNG (Salmon et al., SC'11), SURVEY.md §8(c) R15,
+# DESIGN.md reading D-RNG.  Element idx draws the 16-bit half (idx & 1, low half
+# first) of word ((idx >> 1) & 3) of Philox(counter = (c_lo, c_hi, step, 0),
+# key = (seed, 0x5453504C)) with c = idx >> 3 (one Philox call feeds eight
+# consecutive elements), and keep = (half >= floor(p * 2^16)).  Pure integer
 # maths, so both sides of the parity test take the identical keep/drop decision.
 # ---------------------------------------------------------------------------
 _M0, _M1 = np.uint64(0xD2511F53), np.uint64(0xCD9E8D57)
@@ -60,21 +61,22 @@ def philox4x32_10(c, k0, k1):
 
 
 def philox_word(idx: np.ndarray, seed: int, step: int = 0) -> np.ndarray:
-    """The 32-bit random word of element idx (see above)."""
+    """The 16-bit random draw of element idx (see above)."""
     idx = idx.astype(np.uint64)
-    ctr = idx >> np.uint64(2)
+    ctr = idx >> np.uint64(3)
     c0 = ctr & _MASK32
     c1 = ctr >> np.uint64(32)
     c2 = np.full_like(c0, np.uint64(step & 0xFFFFFFFF))
     c3 = np.zeros_like(c0)
     words = np.stack(philox4x32_10((c0, c1, c2, c3), seed, PHILOX_KEY1))
-    return words[(idx & np.uint64(3)).astype(np.int64), np.arange(idx.shape[0])]
+    w = words[((idx >> np.uint64(1)) & np.uint64(3)).astype(np.int64), np.arange(idx.shape[0])]
+    return (w >> (np.uint64(16) * (idx & np.uint64(1)))) & np.uint64(0xFFFF)
 
 
 def dropout_keep(shape, elem0: int, p: float, seed: int, step: int = 0) -> np.ndarray:
     n = int(np.prod(shape))
     w = philox_word(np.arange(elem0, elem0 + n, dtype=np.uint64), seed, step)
-    thr = np.uint64(int(np.floor(p * 4294967296.0)))
+    thr = np.uint64(min(int(np.floor(p * 65536.0)), 65535))
     return (w >= thr).reshape(shape)
 
 

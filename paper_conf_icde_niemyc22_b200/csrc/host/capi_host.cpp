@@ -1,5 +1,6 @@
 // C ABI: graph, profile and plan entry points (host only; no CUDA calls).
 #include <cstring>
+#include <string>
 #include <memory>
 #include <new>
 
@@ -105,6 +106,16 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
     pr = &local;
   }
   ts_status st = plan_greedy(g->g, budget_bytes, *pr, p->st, flags);
+  // Alg. 2 is greedy and path-dependent: when it runs out of candidates, plan again for a
+  // slightly tighter budget (different early decisions); any plan found fits the real one
+  const std::string first_error = st == TS_OK ? std::string() : std::string(ts_last_error());
+  for (int k = 1; st == TS_ERR_INFEASIBLE && k <= 6; ++k) {
+    const uint64_t tight = g->g.static_bytes + uint64_t(double(budget_bytes - g->g.static_bytes) * (1.0 - 0.03 * k));
+    if (tight <= g->g.static_bytes) break;
+    p->st = PlanState();
+    st = plan_greedy(g->g, tight, *pr, p->st, flags);
+  }
+  if (st == TS_ERR_INFEASIBLE) set_error(first_error);
   if (st != TS_OK) return st;
   p->budget = budget_bytes;
   *out = p.release();

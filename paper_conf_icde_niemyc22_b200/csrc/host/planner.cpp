@@ -340,13 +340,19 @@ void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& 
 // plan's headroom x 8, x 4, x 2, x 1, x 1/2} (headroom = budget - simulated peak, so the
 // cached pieces only use memory the memory-centric plan leaves free), and with a cache the
 // D-R8c post-pass runs again (decisions that no longer pay can be reverted).
+// (plus rbytes / 2^k down to 1 MiB: the plan's peak is usually set in the forward pass, so a
+// cache far larger than the headroom can still fit the backward)
 void plan_lru(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps) {
   bool any = false;
   for (const Cfg& c : ps.cfg) any |= c.opt == TS_RECOMPUTE;
   if (!any) return;
   const uint64_t head = budget > max_top(ps) ? budget - max_top(ps) : 0;
+  uint64_t rbytes = 0;  // every recompute-opt tensor: an upper bound on what can be cached
+  for (int t = 0; t < g.n(); ++t)
+    if (ps.cfg[t].opt == TS_RECOMPUTE) rbytes += g.t[t].bytes;
   PlanState best = ps;
-  const uint64_t caps[] = {~uint64_t(0), 8 * head, 4 * head, 2 * head, head, head / 2};
+  std::vector<uint64_t> caps = {~uint64_t(0), 8 * head, 4 * head, 2 * head, head, head / 2};
+  for (uint64_t c = rbytes / 2; c > (uint64_t(1) << 20) && caps.size() < 24; c /= 2) caps.push_back(c);
   for (uint64_t cap : caps) {
     if (cap == 0) continue;
     PlanState cand;
@@ -528,6 +534,26 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       c.analytic = double(bw_ops[t].size()) * rc_time(rc_time, t, 0) / dm;
       step1.push_back(with_feeders(c, t));
     }
+    // a swapped tensor live at a backward bottleneck only because its prefetch lands early
+    // (long lead): shorten the lead to the previous computation or recompute it
+    if (bwd_phase)
+      for (int t : live) {
+        const Tensor& x = g.t[t];
+        if (x.kind != TS_ACT || x.is_loss || ps.cfg[t].opt != TS_SWAP || own.count(t)) continue;
+        if (first_bw[t] <= bi) continue;
+        const double dm = double(x.bytes);
+        Cand2 c;
+        c.birth = birth[t];
+        c.tensor = t;
+        if (ps.cfg[t].lead > 1) {
+          c.ch = {{t, TS_SWAP, ps.cfg[t].p, 1}};
+          c.analytic = swap_cost(t, dm) / dm;
+          step1.push_back(c);
+        }
+        c.ch = {{t, TS_RECOMPUTE, ps.cfg[t].p, 1}};
+        c.analytic = double(bw_ops[t].size()) * rc_time(rc_time, t, 0) / dm;
+        step1.push_back(with_feeders(c, t));
+      }
     // shortlist by the analytic ratio, keeping the best swaps and the best recomputes
     {
       auto by = [](const Cand2& a, const Cand2& b) {

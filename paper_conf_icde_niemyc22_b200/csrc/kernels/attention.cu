@@ -26,32 +26,30 @@ constexpr float kLog2e = 1.4426950408889634f;
 constexpr float kLn2 = 0.6931471805599453f;
 
 __device__ __forceinline__ uint32_t philox_one(uint64_t e, uint32_t seed, uint32_t step) {
-  const uint64_t c = e >> 2;
-  const uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), step, 0u, seed, kPhiloxKey1);
-  const uint32_t w[4] = {r.x, r.y, r.z, r.w};
-  return w[e & 3];
+  return philox_u16(e, seed, step);  // the element's 16-bit draw (D-RNG)
 }
 
 // Keep decisions of one 8-column n-tile of an mma.sync accumulator, for this thread's
-// (row r, cols 2t, 2t+1) and (row r + 8, same cols): the quad's 4 Philox calls (2 rows x
-// 2 four-column groups) are spread one per lane and the words exchanged by shuffles.
+// (row r, cols 2t, 2t+1) and (row r + 8, same cols): one Philox call covers the eight keys
+// of a row (D-RNG), so lanes t = 0 / 1 of the quad draw rows r / r + 8 and every lane takes
+// word t (its two keys' halves) of both by shuffles.
 // e0 = element index of (row r of lane 0's quad, column 0 of the n-tile); S = row stride.
 __device__ __forceinline__ void quad_keep(uint64_t e0, uint64_t S, uint32_t seed, uint32_t step, uint32_t thr,
                                           bool (&k)[4]) {
   const int lane = threadIdx.x & 31, t = lane & 3;
-  const uint64_t e = e0 + uint64_t(t & 1) * 8ull * S + uint64_t(4 * (t >> 1));
-  const uint64_t c = e >> 2;
+  const uint64_t c = (e0 + uint64_t(t & 1) * 8ull * S) >> 3;
   const uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), step, 0u, seed, kPhiloxKey1);
-  const int src0 = (lane & ~3) | (t & 2), src1 = src0 | 1;
-  const uint32_t ax = __shfl_sync(0xffffffffu, r.x, src0), ay = __shfl_sync(0xffffffffu, r.y, src0);
-  const uint32_t az = __shfl_sync(0xffffffffu, r.z, src0), aw = __shfl_sync(0xffffffffu, r.w, src0);
-  const uint32_t bx = __shfl_sync(0xffffffffu, r.x, src1), by = __shfl_sync(0xffffffffu, r.y, src1);
-  const uint32_t bz = __shfl_sync(0xffffffffu, r.z, src1), bw = __shfl_sync(0xffffffffu, r.w, src1);
-  const bool hi = t & 1;
-  k[0] = (hi ? az : ax) >= thr;
-  k[1] = (hi ? aw : ay) >= thr;
-  k[2] = (hi ? bz : bx) >= thr;
-  k[3] = (hi ? bw : by) >= thr;
+  const int src0 = lane & ~3, src1 = src0 | 1;
+  const uint32_t a0 = __shfl_sync(0xffffffffu, r.x, src0), a1 = __shfl_sync(0xffffffffu, r.y, src0);
+  const uint32_t a2 = __shfl_sync(0xffffffffu, r.z, src0), a3 = __shfl_sync(0xffffffffu, r.w, src0);
+  const uint32_t b0 = __shfl_sync(0xffffffffu, r.x, src1), b1 = __shfl_sync(0xffffffffu, r.y, src1);
+  const uint32_t b2 = __shfl_sync(0xffffffffu, r.z, src1), b3 = __shfl_sync(0xffffffffu, r.w, src1);
+  const uint32_t wa = t == 0 ? a0 : t == 1 ? a1 : t == 2 ? a2 : a3;
+  const uint32_t wb = t == 0 ? b0 : t == 1 ? b1 : t == 2 ? b2 : b3;
+  k[0] = (wa & 0xFFFFu) >= thr;
+  k[1] = (wa >> 16) >= thr;
+  k[2] = (wb & 0xFFFFu) >= thr;
+  k[3] = (wb >> 16) >= thr;
 }
 __device__ __forceinline__ float ex2(float x) {
   float y;
@@ -774,10 +772,7 @@ bool tc_eligible(const AttnArgs& A) {
          reinterpret_cast<uintptr_t>(A.v) % 16 == 0;
 }
 
-void fill_thr(AttnArgs& A) {
-  const double t = double(A.p) * 4294967296.0;
-  A.thr = A.p <= 0.f ? 0u : (t >= 4294967295.0 ? 0xFFFFFFFFu : uint32_t(t));
-}
+void fill_thr(AttnArgs& A) { A.thr = dropout_thr16(A.p); }
 
 }  // namespace
 

@@ -63,7 +63,7 @@ struct Fa5P {
 // thread (TMA + tcgen05.mma).  P is rebuilt from S and the saved log-sum-exp, the keep
 // bits come from the forward's mask (no Philox), D_q = dO_q . O_q.
 struct Fa5B {
-  int heads, seq;
+  int nb, heads, seq;
   int64_t ld;
   float sl2, alpha, keep_scale;
   int drop;
@@ -136,45 +136,52 @@ __device__ __forceinline__ void store_row32(bf16* dst, const uint32_t (&r)[32], 
 // write (dS; P^T as well for dK/dV) are double-buffered in shared memory, so the tensor
 // core works on tile t+1 while the compute warps are still on tile t.
 //
-// dQ for 128 queries of one (sample, head); all of K and V in shared memory.
-// smem: Q 16K | dO 16K | K seq*128 | V seq*128 | dS 2 x 32K | barriers
-// TMEM: S 0..127, dP 128..255, dQ 256..319
-__global__ void __launch_bounds__(kBwdThreads, 1)
+// dQ, persistent: a work item is 128 queries of one (sample, head); K and V stream through a
+// 3-stage TMA ring one 128-key tile at a time (so the next item's loads run ahead), Q / dO
+// are double-buffered per item, and dQ accumulates in one of two TMEM buffers so an item's
+// epilogue overlaps the next item's products.  One TMA thread, one MMA thread, 16 compute
+// warps.  D_q = dO_q . O_q is formed by the first column group of each item (and stored for
+// the dK/dV kernel).
+// smem: Q 2 x 16K | dO 2 x 16K | K,V ring 3 x 32K | dS 2 x 32K | D 2 x 512 B | barriers
+// TMEM: S 0..127, dP 128..255, dQ 256..319 / 320..383
+constexpr int kDqStages = 3;
+constexpr int kDqThreads = 32 * (kBwdCW + 2);
+constexpr int kDqSmemQ = 0, kDqSmemG = 32768, kDqSmemKV = 65536, kDqSmemDS = kDqSmemKV + kDqStages * 32768;
+constexpr int kDqSmemD = kDqSmemDS + 65536, kDqSmemBar = kDqSmemD + 1024;
+constexpr int kDqSmem = kDqSmemBar + 256 + 1024;
+__global__ void __launch_bounds__(kDqThreads, 1)
     fa5_bwd_dq(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mdO,
                const __grid_constant__ CUtensorMap mK, const __grid_constant__ CUtensorMap mV, const Fa5B p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  const int S = p.seq, nkt = S / 128;
-  uint8_t* sQ = smem;
-  uint8_t* sdO = smem + 16384;
-  uint8_t* sK = smem + 32768;
-  uint8_t* sV = sK + S * 128;
-  uint8_t* sdS = sV + S * 128;  // two 32 KB buffers
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sdS + 65536);
-  uint64_t *ld_full = bar, *s_full = bar + 1, *s_free = bar + 2, *ds_full = bar + 3 /*[2]*/, *dq_done = bar + 5 /*[2]*/;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 7);
+  const int S = p.seq, nkt = S / 128, nqt = S / 128;
+  const int items = p.nb * p.heads * nqt;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + kDqSmemBar);
+  uint64_t *qd_full = bar /*[2]*/, *qd_empty = bar + 2 /*[2]*/, *kv_full = bar + 4 /*[3]*/,
+           *kv_empty = bar + 7 /*[3]*/, *s_full = bar + 10, *s_free = bar + 11, *ds_full = bar + 12 /*[2]*/,
+           *ds_free = bar + 14 /*[2]*/, *dq_full = bar + 16 /*[2]*/, *dq_empty = bar + 18 /*[2]*/;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 20);
+  float* sD = reinterpret_cast<float*>(smem + kDqSmemD);  // [2][128]
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int qt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
-  // the D-row loads of the compute warps go out before the setup (their latency overlaps it)
-  uint4 x0, x1, y0, y1;
-  if (warp < kBwdCW) {
-    const int64_t roff = (int64_t(b) * S + qt * 128 + (warp & 3) * 32 + lane) * p.ld + a * 64 + (warp >> 2) * 16;
-    x0 = *reinterpret_cast<const uint4*>(p.o + roff);
-    x1 = *reinterpret_cast<const uint4*>(p.o + roff + 8);
-    y0 = *reinterpret_cast<const uint4*>(p.dout + roff);
-    y1 = *reinterpret_cast<const uint4*>(p.dout + roff + 8);
-  }
+  constexpr int kTma = kBwdCW, kMma = kBwdCW + 1;
   if (threadIdx.x == 0) {
-    mbar_init(ld_full, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&qd_full[i], 1);
+      mbar_init(&qd_empty[i], 1);
+      mbar_init(&ds_full[i], 32 * kBwdCW);
+      mbar_init(&ds_free[i], 1);
+      mbar_init(&dq_full[i], 1);
+      mbar_init(&dq_empty[i], 32 * kBwdCW);
+    }
+    for (int i = 0; i < kDqStages; ++i) {
+      mbar_init(&kv_full[i], 1);
+      mbar_init(&kv_empty[i], 1);
+    }
     mbar_init(s_full, 1);
     mbar_init(s_free, 32 * kBwdCW);
-    mbar_init(&ds_full[0], 32 * kBwdCW);
-    mbar_init(&ds_full[1], 32 * kBwdCW);
-    mbar_init(&dq_done[0], 1);
-    mbar_init(&dq_done[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == kBwdCtl) {
+  if (warp == kMma) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(512));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -183,115 +190,144 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
-  if (warp == kBwdCtl) {
+  if (warp == kTma) {
     if (lane == 0) {
-      const int row0 = b * S;
-      mbar_arrive_tx(ld_full, 32768u + uint32_t(S) * 256u);
-      tma_load(sQ, &mQ, ld_full, a * 64, row0 + qt * 128, 0, 0);
-      tma_load(sdO, &mdO, ld_full, a * 64, row0 + qt * 128, 0, 0);
-      for (int j = 0; j < S; j += 128) {
-        tma_load(sK + j * 128, &mK, ld_full, a * 64, row0 + j, 0, 0);
-        tma_load(sV + j * 128, &mV, ld_full, a * 64, row0 + j, 0, 0);
+      int it = 0, kc = 0;
+      for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
+        const int qt = item % nqt, ah = item / nqt, a = ah % p.heads, b = ah / p.heads;
+        const int row0 = b * S, buf = it & 1;
+        if (it >= 2) mbar_wait(&qd_empty[buf], ((it >> 1) - 1) & 1);
+        mbar_arrive_tx(&qd_full[buf], 32768u);
+        tma_load(smem + kDqSmemQ + buf * 16384, &mQ, &qd_full[buf], a * 64, row0 + qt * 128, 0, 0);
+        tma_load(smem + kDqSmemG + buf * 16384, &mdO, &qd_full[buf], a * 64, row0 + qt * 128, 0, 0);
+        for (int kt = 0; kt < nkt; ++kt, ++kc) {
+          const int st = kc % kDqStages;
+          if (kc >= kDqStages) mbar_wait(&kv_empty[st], ((kc / kDqStages) - 1) & 1);
+          mbar_arrive_tx(&kv_full[st], 32768u);
+          tma_load(smem + kDqSmemKV + st * 32768, &mK, &kv_full[st], a * 64, row0 + kt * 128, 0, 0);
+          tma_load(smem + kDqSmemKV + st * 32768 + 16384, &mV, &kv_full[st], a * 64, row0 + kt * 128, 0, 0);
+        }
       }
-      mbar_wait(ld_full, 0);
-      tc_fence_after();
-      const uint32_t q = smem_u32(sQ), g = smem_u32(sdO), k = smem_u32(sK), v = smem_u32(sV), ds = smem_u32(sdS);
-      auto issue_dq = [&](int kt) {  // dQ += dS_kt K_kt: A = dS (K-major), B = K rows of the tile (MN-major)
-        mbar_wait(&ds_full[kt & 1], (kt >> 1) & 1);
-        tc_fence_after();
-        const uint32_t dsb = ds + uint32_t(kt & 1) * 32768u;
-        for (int kk = 0; kk < 128; kk += 16)
-          tc_mma(tmem + 256, smem_desc(dsb + (kk >> 6) * 16384 + ((kk & 63) >> 4) * 32, 16, 1024),
-                 smem_desc(k + uint32_t(kt * 128 + kk) * 128, 8192, 1024), kIdN64MN, (kt > 0 || kk > 0) ? 1u : 0u);
-        tc_commit(&dq_done[kt & 1]);
-      };
-      for (int kt = 0; kt < nkt; ++kt) {
-        if (kt > 0) {
-          mbar_wait(s_free, (kt - 1) & 1);  // S, dP of tile kt-1 are in registers
+    }
+  } else if (warp == kMma) {
+    if (lane == 0) {
+      int it = 0, kc = 0;  // items, key tiles (running)
+      uint32_t ns = 0;     // S / dP tiles issued
+      for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
+        const int buf = it & 1, acc = it & 1;
+        mbar_wait(&qd_full[buf], (it >> 1) & 1);
+        const uint32_t q = smem_u32(smem + kDqSmemQ + buf * 16384), g = smem_u32(smem + kDqSmemG + buf * 16384);
+        auto issue_dq = [&](int kcp, int first) {  // dQ += dS K of running tile kcp
+          mbar_wait(&ds_full[kcp & 1], (kcp >> 1) & 1);
           tc_fence_after();
-        }
+          const uint32_t dsb = smem_u32(smem + kDqSmemDS + (kcp & 1) * 32768);
+          const uint32_t k = smem_u32(smem + kDqSmemKV + (kcp % kDqStages) * 32768);
+          for (int kk = 0; kk < 128; kk += 16)
+            tc_mma(tmem + 256 + uint32_t(acc * 64), smem_desc(dsb + (kk >> 6) * 16384 + ((kk & 63) >> 4) * 32, 16, 1024),
+                   smem_desc(k + uint32_t(kk) * 128, 8192, 1024), kIdN64MN, (first && kk == 0) ? 0u : 1u);
+          tc_commit(&ds_free[kcp & 1]);
+          tc_commit(&kv_empty[kcp % kDqStages]);
+        };
+        for (int kt = 0; kt < nkt; ++kt, ++kc) {
+          const int st = kc % kDqStages;
+          mbar_wait(&kv_full[st], (kc / kDqStages) & 1);
+          if (ns > 0) mbar_wait(s_free, (ns - 1) & 1);  // the previous S, dP are in registers
+          tc_fence_after();
+          const uint32_t k = smem_u32(smem + kDqSmemKV + st * 32768), v = k + 16384;
 #pragma unroll
-        for (int kk = 0; kk < 4; ++kk) {
-          tc_mma(tmem, smem_desc(q + kk * 32, 16, 1024), smem_desc(k + kt * 16384 + kk * 32, 16, 1024), kIdN128,
-                 kk > 0 ? 1u : 0u);
-          tc_mma(tmem + 128, smem_desc(g + kk * 32, 16, 1024), smem_desc(v + kt * 16384 + kk * 32, 16, 1024),
-                 kIdN128, kk > 0 ? 1u : 0u);
+          for (int kk = 0; kk < 4; ++kk) {
+            tc_mma(tmem, smem_desc(q + kk * 32, 16, 1024), smem_desc(k + kk * 32, 16, 1024), kIdN128, kk > 0 ? 1u : 0u);
+            tc_mma(tmem + 128, smem_desc(g + kk * 32, 16, 1024), smem_desc(v + kk * 32, 16, 1024), kIdN128,
+                   kk > 0 ? 1u : 0u);
+          }
+          tc_commit(s_full);
+          ++ns;
+          if (kt == nkt - 1) tc_commit(&qd_empty[buf]);  // every product reading Q, dO of this item issued
+          if (kt > 0) {
+            if (kt == 1 && it >= 2) mbar_wait(&dq_empty[acc], ((it >> 1) - 1) & 1);  // epilogue of item it-2 read dQ
+            issue_dq(kc - 1, kt == 1);
+          }
         }
-        tc_commit(s_full);
-        if (kt > 0) issue_dq(kt - 1);
+        if (nkt == 1 && it >= 2) mbar_wait(&dq_empty[acc], ((it >> 1) - 1) & 1);
+        issue_dq(kc - 1, nkt == 1);
+        tc_commit(&dq_full[acc]);
       }
-      issue_dq(nkt - 1);
     }
   } else {
     const int qw = warp & 3, cg = warp >> 2;  // TMEM lane quarter, 32-column group
     const int i = qw * 32 + lane;
-    const int q = qt * 128 + i;
-    const int64_t hrow = (int64_t(b) * p.heads + a) * S + q;
     const uint32_t trow = tmem + (uint32_t(qw * 32) << 16);
-    // D_q = dO_q . O_q in fp32 over the bf16 row: group cg sums dims [16cg, 16cg+16), the four
-    // partials meet in the (still unused) second dS buffer.  Nothing writes that buffer before
-    // tile 1, which needs every thread's s_free arrival of tile 0, i.e. after these reads.
-    float* red = reinterpret_cast<float*>(sdS + 32768);
-    {
-      const __nv_bfloat162* xa = reinterpret_cast<const __nv_bfloat162*>(&x0);
-      const __nv_bfloat162* xb = reinterpret_cast<const __nv_bfloat162*>(&x1);
-      const __nv_bfloat162* ya = reinterpret_cast<const __nv_bfloat162*>(&y0);
-      const __nv_bfloat162* yb = reinterpret_cast<const __nv_bfloat162*>(&y1);
-      float part = 0.f;
+    int it = 0, kc = 0;
+    for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
+      const int qt = item % nqt, ah = item / nqt, a = ah % p.heads, b = ah / p.heads;
+      const int q = qt * 128 + i;
+      const int64_t hrow = (int64_t(b) * p.heads + a) * S + q;
+      float* sd = sD + (it & 1) * 128;
+      if (cg == 0) {  // D_q = dO_q . O_q in fp32 over the bf16 row
+        const bf16* orow = p.o + (int64_t(b) * S + q) * p.ld + a * 64;
+        const bf16* grow = p.dout + (int64_t(b) * S + q) * p.ld + a * 64;
+        uint4 x[8], y[8];
 #pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const float2 u = __bfloat1622float2(xa[e]), w = __bfloat1622float2(ya[e]);
-        part += u.x * w.x + u.y * w.y;
-      }
+        for (int j = 0; j < 8; ++j) {
+          x[j] = *reinterpret_cast<const uint4*>(orow + 8 * j);
+          y[j] = *reinterpret_cast<const uint4*>(grow + 8 * j);
+        }
+        float D = 0.f;
 #pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const float2 u = __bfloat1622float2(xb[e]), w = __bfloat1622float2(yb[e]);
-        part += u.x * w.x + u.y * w.y;
+        for (int j = 0; j < 8; ++j) {
+          const __nv_bfloat162* x2 = reinterpret_cast<const __nv_bfloat162*>(&x[j]);
+          const __nv_bfloat162* y2 = reinterpret_cast<const __nv_bfloat162*>(&y[j]);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const float2 u = __bfloat1622float2(x2[e]), w = __bfloat1622float2(y2[e]);
+            D += u.x * w.x + u.y * w.y;
+          }
+        }
+        sd[i] = D;
+        p.D[hrow] = D;
       }
-      red[cg * 128 + i] = part;
-    }
-    named_sync(2, 32 * kBwdCW);
-    const float D = (red[i] + red[128 + i]) + (red[256 + i] + red[384 + i]);
-    if (cg == 0) p.D[hrow] = D;
-    const float l2 = p.lse[hrow] * kLog2e;
-    const uint32_t* mrow = p.mask + hrow * (S / 32);
-    const uint32_t ds = smem_u32(sdS);
-    for (int kt = 0; kt < nkt; ++kt) {
-      // this key tile's keep word of the row for the group's 32 keys, fetched before waiting
-      const uint32_t bits = p.drop ? mrow[kt * 4 + cg] : ~0u;
-      mbar_wait(s_full, kt & 1);
+      named_sync(2, 32 * kBwdCW);
+      const float D = sd[i];
+      const float l2 = p.lse[hrow] * kLog2e;
+      const uint32_t* mrow = p.mask + hrow * (S / 32);
+      for (int kt = 0; kt < nkt; ++kt, ++kc) {
+        const uint32_t bits = p.drop ? mrow[kt * 4 + cg] : ~0u;
+        mbar_wait(s_full, kc & 1);
+        tc_fence_after();
+        uint32_t rs[32], rp[32];
+        tmem_ld32_nw(trow + uint32_t(cg * 32), rs);
+        tmem_ld32_nw(trow + uint32_t(128 + cg * 32), rp);
+        tmem_wait_ld();
+        tc_fence_before();
+        mbar_arrive(s_free);
+#pragma unroll
+        for (int j = 0; j < 32; ++j) {
+          const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
+          const float dp = ((bits >> j) & 1u) ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
+          rs[j] = __float_as_uint(pr * (dp - D));
+        }
+        if (kc >= 2) mbar_wait(&ds_free[kc & 1], ((kc >> 1) - 1) & 1);  // the dQ product of tile kc-2 read it
+        st_row32(smem_u32(smem + kDqSmemDS + (kc & 1) * 32768), i, cg * 32, reinterpret_cast<const float*>(rs));
+        fence_async_smem();
+        tc_fence_before();
+        mbar_arrive(&ds_full[kc & 1]);
+      }
+      mbar_wait(&dq_full[it & 1], (it >> 1) & 1);
       tc_fence_after();
-      uint32_t rs[32], rp[32];
-      tmem_ld32_nw(trow + uint32_t(cg * 32), rs);
-      tmem_ld32_nw(trow + uint32_t(128 + cg * 32), rp);
-      tmem_wait_ld();
-      tc_fence_before();
-      mbar_arrive(s_free);
-#pragma unroll
-      for (int j = 0; j < 32; ++j) {
-        const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
-        const float dp = ((bits >> j) & 1u) ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
-        rs[j] = __float_as_uint(pr * (dp - D));
+      if (cg < 2) {
+        uint32_t r0[32];
+        tmem_ld32(trow + 256u + uint32_t((it & 1) * 64 + cg * 32), r0);
+        if (p.dq)
+          store_row32(static_cast<bf16*>(p.dq) + (int64_t(b) * S + q) * p.ld + a * 64 + cg * 32, r0, p.alpha, p.acc_q);
       }
-      if (kt >= 2) mbar_wait(&dq_done[kt & 1], ((kt - 2) >> 1) & 1);  // dS buffer kt&1 free
-      st_row32(ds + uint32_t(kt & 1) * 32768u, i, cg * 32, reinterpret_cast<const float*>(rs));
-      fence_async_smem();
       tc_fence_before();
-      mbar_arrive(&ds_full[kt & 1]);
-    }
-    mbar_wait(&dq_done[(nkt - 1) & 1], ((nkt - 1) >> 1) & 1);
-    tc_fence_after();
-    if (cg < 2) {
-      uint32_t r0[32];
-      tmem_ld32(trow + 256u + uint32_t(cg * 32), r0);
-      if (p.dq)
-        store_row32(static_cast<bf16*>(p.dq) + (int64_t(b) * S + q) * p.ld + a * 64 + cg * 32, r0, p.alpha, p.acc_q);
+      mbar_arrive(&dq_empty[it & 1]);
     }
   }
   __syncwarp();
   tc_fence_before();
   __syncthreads();
-  if (warp == kBwdCtl) {
+  if (warp == kMma) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
   }
@@ -699,12 +735,13 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
         if (p.p > 0.f) {
           bits = 0u;
 #pragma unroll
-          for (int u = 0; u < 8; ++u) {
-            const uint64_t cnt = (erow + uint64_t(key + 4 * u)) >> 2;
-            const uint4 w = philox4x32_10(uint32_t(cnt), uint32_t(cnt >> 32), p.step, 0u, p.seed, kPhiloxKey1);
-            bits |= (uint32_t(w.x >= p.thr) | (uint32_t(w.y >= p.thr) << 1) | (uint32_t(w.z >= p.thr) << 2) |
-                     (uint32_t(w.w >= p.thr) << 3))
-                    << (4 * u);
+          // one Philox call per eight keys of the row (D-RNG); erow + key is a multiple of 32,
+          // so the four counters share the high word
+          const uint64_t cnt0 = (erow + uint64_t(key)) >> 3;
+          for (int u = 0; u < 4; ++u) {
+            const uint4 w = philox4x32_10(uint32_t(cnt0) + uint32_t(u), uint32_t(cnt0 >> 32), p.step, 0u, p.seed,
+                                          kPhiloxKey1);
+            bits |= keep_bits8(w, p.thr) << (8 * u);
           }
 #pragma unroll
           for (int jj = 0; jj < 32; ++jj)
@@ -844,15 +881,18 @@ bool attention_bwd_tc5(const AttnArgs& A, cudaStream_t st) {
   p.acc_q = A.acc_q;
   p.acc_k = A.acc_k;
   p.acc_v = A.acc_v;
-  const int smem_q = 32768 + 2 * A.seq * 128 + 65536 + 256 + 1024;
   const int smem_kv = 229376 + 256 + 1024;
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(fa5_bwd_dq, cudaFuncAttributeMaxDynamicSharedMemorySize, 32768 + 2 * 512 * 128 + 65536 + 1280);
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaFuncSetAttribute(fa5_bwd_dq, cudaFuncAttributeMaxDynamicSharedMemorySize, kDqSmem);
     cudaFuncSetAttribute(fa5_bwd_dkv, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_kv);
-    attr = true;
   }
-  fa5_bwd_dq<<<dim3(A.seq / 128, A.heads, A.nb), kBwdThreads, smem_q, st>>>(mq, mg, mk, mv, p);
+  p.nb = A.nb;
+  const int items_q = A.nb * A.heads * (A.seq / 128);
+  fa5_bwd_dq<<<items_q < sms ? items_q : sms, kDqThreads, kDqSmem, st>>>(mq, mg, mk, mv, p);
   fa5_bwd_dkv<<<dim3(A.seq / 128, A.heads, A.nb), kBwdThreads, smem_kv, st>>>(mq, mg, mk, mv, p);
   return true;
 }

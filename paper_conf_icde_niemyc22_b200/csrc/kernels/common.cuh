@@ -54,8 +54,10 @@ __device__ __forceinline__ float gelu_d(float x) {
 }
 __device__ __forceinline__ float bf16_round(float x) { return __bfloat162float(__float2bfloat16_rn(x)); }
 
-// Philox4x32-10 (Salmon et al. SC'11); reading D-RNG: element idx uses
-// word (idx & 3) of Philox(counter = (idx>>2 lo, idx>>2 hi, step, 0), key = (seed, 0x5453504C)).
+// Philox4x32-10 (Salmon et al. SC'11); reading D-RNG: element idx takes the 16-bit half
+// (idx & 1) of word ((idx >> 1) & 3) of Philox(counter = (idx>>3 lo, idx>>3 hi, step, 0),
+// key = (seed, 0x5453504C)), and is kept when that half >= floor(p * 2^16): one call covers
+// eight consecutive elements.
 __device__ __forceinline__ uint4 philox4x32_10(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3,
                                                uint32_t k0, uint32_t k1) {
 #pragma unroll
@@ -73,6 +75,27 @@ __device__ __forceinline__ uint4 philox4x32_10(uint32_t c0, uint32_t c1, uint32_
   return make_uint4(c0, c1, c2, c3);
 }
 constexpr uint32_t kPhiloxKey1 = 0x5453504Cu;
+// keep bits of the eight elements of one Philox call (bit i = element 8c + i)
+__device__ __forceinline__ uint32_t keep_bits8(const uint4& w, uint32_t thr16) {
+  return uint32_t((w.x & 0xFFFFu) >= thr16) | (uint32_t((w.x >> 16) >= thr16) << 1) |
+         (uint32_t((w.y & 0xFFFFu) >= thr16) << 2) | (uint32_t((w.y >> 16) >= thr16) << 3) |
+         (uint32_t((w.z & 0xFFFFu) >= thr16) << 4) | (uint32_t((w.z >> 16) >= thr16) << 5) |
+         (uint32_t((w.w & 0xFFFFu) >= thr16) << 6) | (uint32_t((w.w >> 16) >= thr16) << 7);
+}
+// the 16-bit draw of element idx (one call per element: tails and reference kernels)
+__device__ __forceinline__ uint32_t philox_u16(uint64_t idx, uint32_t seed, uint32_t step) {
+  const uint64_t c = idx >> 3;
+  const uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), step, 0u, seed, kPhiloxKey1);
+  const uint32_t q = uint32_t(idx >> 1) & 3u;
+  const uint32_t word = q == 0 ? r.x : q == 1 ? r.y : q == 2 ? r.z : r.w;
+  return (idx & 1) ? (word >> 16) : (word & 0xFFFFu);
+}
+// floor(p * 2^16) (p in [0, 1))
+inline uint32_t dropout_thr16(float p) {
+  if (p <= 0.f) return 0u;
+  const double t = double(p) * 65536.0;
+  return t >= 65535.0 ? 65535u : uint32_t(t);
+}
 
 __device__ __forceinline__ float warp_sum(float v) {
 #pragma unroll

@@ -38,27 +38,21 @@ __device__ __forceinline__ float ew_apply(float a, float b, int64_t idx, uint32_
 template <class T, int OP, int V>
 __device__ __forceinline__ void ew_vec(const T* __restrict__ a, const T* __restrict__ b, T* y, int64_t v, int acc,
                                        const EwP& q, const T* av, const T* bv, T* yv) {
-  uint32_t words[V];
+  uint32_t words[V];  // DROP: the element's 16-bit draw (D-RNG)
   if constexpr (OP == DROP) {
     const int64_t i0 = q.elem0 + v * V;
-    if ((i0 & 3) == 0 && V % 4 == 0) {
+    if ((i0 & 7) == 0 && V % 8 == 0) {
 #pragma unroll
-      for (int j = 0; j < V; j += 4) {
-        uint64_t c = uint64_t(i0 + j) >> 2;
-        uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
-        words[j] = r.x;
-        words[j + 1] = r.y;
-        words[j + 2] = r.z;
-        words[j + 3] = r.w;
+      for (int j = 0; j < V; j += 8) {
+        const uint64_t c = uint64_t(i0 + j) >> 3;
+        const uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
+        const uint32_t w4[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+        for (int e = 0; e < 8; ++e) words[j + e] = (e & 1) ? (w4[e >> 1] >> 16) : (w4[e >> 1] & 0xFFFFu);
       }
     } else {
 #pragma unroll
-      for (int j = 0; j < V; ++j) {
-        uint64_t e = uint64_t(i0 + j), c = e >> 2;
-        uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
-        uint32_t w[4] = {r.x, r.y, r.z, r.w};
-        words[j] = w[e & 3];
-      }
+      for (int j = 0; j < V; ++j) words[j] = philox_u16(uint64_t(i0 + j), q.seed, q.step);
     }
   }
 #pragma unroll
@@ -112,12 +106,7 @@ __global__ void __launch_bounds__(256) ew_kernel(const T* __restrict__ a, const 
   // scalar tail
   for (int64_t i = nv * V + int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
     uint32_t w = 0;
-    if constexpr (OP == DROP) {
-      uint64_t e = uint64_t(q.elem0 + i), c = e >> 2;
-      uint4 r = philox4x32_10(uint32_t(c), uint32_t(c >> 32), q.step, 0u, q.seed, kPhiloxKey1);
-      uint32_t ww[4] = {r.x, r.y, r.z, r.w};
-      w = ww[e & 3];
-    }
+    if constexpr (OP == DROP) w = philox_u16(uint64_t(q.elem0 + i), q.seed, q.step);
     float r = ew_apply<OP>(to_f(a[i]), b ? to_f(b[i]) : 0.f, i, w, q);
     if (acc) r += to_f(y[i]);
     y[i] = from_f<T>(r);
@@ -230,8 +219,7 @@ void dropout(int dt, const void* x, void* y, int acc, int64_t n, int64_t elem0, 
   q.scale = p > 0.f ? 1.f / (1.f - p) : 1.f;
   q.seed = seed;
   q.step = step;
-  double t = double(p) * 4294967296.0;
-  q.thr = t >= 4294967295.0 ? 0xFFFFFFFFu : uint32_t(t);
+  q.thr = dropout_thr16(p);
   ew<DROP>(dt, x, nullptr, y, n, acc, q, st);
 }
 void sgd_update(float* master, const float* grad, int64_t n, float lr, float gscale, cudaStream_t st) {

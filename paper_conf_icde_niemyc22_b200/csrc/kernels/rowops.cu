@@ -84,6 +84,80 @@ __global__ void __launch_bounds__(kWarps * 32) ln_fwd_kernel(const T* __restrict
   }
 }
 
+// bf16 LayerNorm forward at HBM rate: a persistent grid (~2 blocks per SM), gamma/beta held
+// packed in registers, and every warp loads its next row before normalising the current one
+// (two rows of loads in flight), one row per warp at a time held in registers.
+template <int NCH>
+__global__ void __launch_bounds__(256) ln_fwd_bf16(const bf16* __restrict__ x, const bf16* __restrict__ g,
+                                                   const bf16* __restrict__ b, bf16* __restrict__ y, int64_t rows,
+                                                   int H, float eps) {
+  const int lane = threadIdx.x & 31;
+  const float invH = 1.f / float(H);
+  uint4 gv[NCH], bv[NCH], cur[NCH];
+#pragma unroll
+  for (int c = 0; c < NCH; ++c) {
+    const int col = (c * 32 + lane) * 8;
+    gv[c] = col < H ? *reinterpret_cast<const uint4*>(g + col) : make_uint4(0, 0, 0, 0);
+    bv[c] = col < H ? *reinterpret_cast<const uint4*>(b + col) : make_uint4(0, 0, 0, 0);
+  }
+  const int64_t stride = int64_t(gridDim.x) * 8;
+  int64_t r = int64_t(blockIdx.x) * 8 + (threadIdx.x >> 5);
+  auto load = [&](int64_t row, uint4 (&v)[NCH]) {
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      const int col = (c * 32 + lane) * 8;
+      v[c] = (row < rows && col < H) ? __ldcs(reinterpret_cast<const uint4*>(x + row * H + col)) : make_uint4(0, 0, 0, 0);
+    }
+  };
+  load(r, cur);
+  for (; r < rows; r += stride) {
+    uint4 nxt[NCH];
+    load(r + stride, nxt);
+    float s = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&cur[c]);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float2 f = __bfloat1622float2(h[e]);
+        s += f.x + f.y;
+      }
+    }
+    const float mean = warp_sum(s) * invH;
+    float q = 0.f;
+#pragma unroll
+    for (int c = 0; c < NCH; ++c)
+      if ((c * 32 + lane) * 8 < H) {
+        const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&cur[c]);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 f = __bfloat1622float2(h[e]);
+          q += (f.x - mean) * (f.x - mean) + (f.y - mean) * (f.y - mean);
+        }
+      }
+    const float rstd = rsqrtf(warp_sum(q) * invH + eps);
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) {
+      const int col = (c * 32 + lane) * 8;
+      if (col < H) {
+        const __nv_bfloat162* hx = reinterpret_cast<const __nv_bfloat162*>(&cur[c]);
+        const __nv_bfloat162* hg = reinterpret_cast<const __nv_bfloat162*>(&gv[c]);
+        const __nv_bfloat162* hb = reinterpret_cast<const __nv_bfloat162*>(&bv[c]);
+        uint4 o;
+        __nv_bfloat162* ho = reinterpret_cast<__nv_bfloat162*>(&o);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 fx = __bfloat1622float2(hx[e]), fg = __bfloat1622float2(hg[e]), fb = __bfloat1622float2(hb[e]);
+          ho[e] = __floats2bfloat162_rn((fx.x - mean) * rstd * fg.x + fb.x, (fx.y - mean) * rstd * fg.y + fb.y);
+        }
+        *reinterpret_cast<uint4*>(y + r * H + col) = o;
+      }
+    }
+#pragma unroll
+    for (int c = 0; c < NCH; ++c) cur[c] = nxt[c];
+  }
+}
+
 // generic (unaligned / long rows): three passes over global memory
 template <class T>
 __global__ void ln_fwd_generic(const T* x, const T* g, const T* b, T* y, int64_t rows, int H, float eps) {
@@ -788,6 +862,19 @@ void ln_fwd_t(const void* x, const void* g, const void* b, void* y, int64_t rows
   auto B = (const T*)b;
   auto Y = (T*)y;
   int grid = grid_rows(rows);
+  if (vec && sizeof(T) == 2 && nch <= 4) {
+    int gb = 2 * 148;
+    if (gb > (rows + 7) / 8) gb = int((rows + 7) / 8);
+    auto Xb = reinterpret_cast<const bf16*>(x);
+    auto Gb = reinterpret_cast<const bf16*>(g);
+    auto Bb = reinterpret_cast<const bf16*>(b);
+    auto Yb = reinterpret_cast<bf16*>(y);
+    switch (nch) {
+      case 1: ln_fwd_bf16<1><<<gb, 256, 0, st>>>(Xb, Gb, Bb, Yb, rows, H, eps); return;
+      case 2: ln_fwd_bf16<2><<<gb, 256, 0, st>>>(Xb, Gb, Bb, Yb, rows, H, eps); return;
+      default: ln_fwd_bf16<4><<<gb, 256, 0, st>>>(Xb, Gb, Bb, Yb, rows, H, eps); return;
+    }
+  }
   if (vec && nch <= 8) {
     switch (nch) {
       case 1: ln_fwd_kernel<T, 1><<<grid, kWarps * 32, 0, st>>>(X, G, B, Y, rows, H, eps); return;

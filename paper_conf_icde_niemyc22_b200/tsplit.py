@@ -256,6 +256,22 @@ class Profile:
     def set_pcie(self, d2h, h2d):
         check(lib().ts_profile_set_pcie(self.h, d2h, h2d))
 
+    def to_dict(self) -> dict:
+        """Every (op, p_num) entry and the PCIe bandwidths (to replay a measured profile)."""
+        ops = {}
+        for o in range(len(self.graph.spec["ops"])):
+            ops[o] = {p: self.get(o, p) for p in (1, 2, 4, 8, 16)}
+        return {"ops": ops, "pcie": self.pcie()}
+
+    @classmethod
+    def from_dict(cls, graph, d: dict):
+        pr = cls(graph)
+        for o, row in d["ops"].items():
+            for p, (f, b) in row.items():
+                pr.set(int(o), int(p), f, b)
+        pr.set_pcie(*d["pcie"])
+        return pr
+
     def __del__(self):
         try:
             if getattr(self, "h", None):

@@ -148,6 +148,19 @@ def test_philox_known_answers():
     assert [int(o[0]) for o in out] == [0xd16cfe09, 0x94fdcceb, 0x5001e420, 0x24126ea1]
 
 
+def test_dropout_draws_are_the_philox_halves():
+    """D-RNG: elements 8c .. 8c+7 take the low / high 16-bit halves of the four words of
+    Philox call c in order (checked against the pinned philox4x32_10 on counters 0 and 5)."""
+    u = lambda *v: tuple(np.array([x], np.uint64) for x in v)
+    for c in (0, 5):
+        w = [int(o[0]) for o in ops.philox4x32_10(u(c, 0, 3, 0), 42, ops.PHILOX_KEY1)]
+        halves = [h for x in w for h in (x & 0xFFFF, x >> 16)]
+        got = ops.philox_word(np.arange(8 * c, 8 * c + 8, dtype=np.uint64), 42, 3)
+        assert [int(v) for v in got] == halves
+        keep = ops.dropout_keep((8,), 8 * c, 0.3, 42, 3)
+        assert list(keep) == [h >= int(0.3 * 65536) for h in halves]
+
+
 def test_dropout_rate_and_split_invariance():
     keep = ops.dropout_keep((1 << 16,), 0, 0.1, 42)
     assert abs(keep.mean() - 0.9) < 0.01
