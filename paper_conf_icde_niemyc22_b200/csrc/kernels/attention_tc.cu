@@ -78,8 +78,6 @@ struct Fa5B {
 
 // 16 compute warps (four per TMEM lane quarter, each owning 32 of a tile's 128 columns) + 1 control warp
 constexpr int kBwdCW = 16;
-constexpr int kBwdCtl = kBwdCW;
-constexpr int kBwdThreads = 32 * (kBwdCW + 1);
 constexpr uint32_t kIdN128 = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(128 >> 3) << 17) | (uint32_t(128 >> 4) << 24);
 constexpr uint32_t kIdN64MN = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | (uint32_t(64 >> 3) << 17) |
                               (uint32_t(128 >> 4) << 24);
@@ -136,12 +134,45 @@ __device__ __forceinline__ void store_row32(bf16* dst, const uint32_t (&r)[32], 
 // write (dS; P^T as well for dK/dV) are double-buffered in shared memory, so the tensor
 // core works on tile t+1 while the compute warps are still on tile t.
 //
+// D[b, a, q] = dO_q . O_q over the 64 dims of head a (fp32 over the bf16 rows), the row term
+// of both backward kernels; 8 lanes per (row, head), 16-byte loads, three shuffles.
+__global__ void __launch_bounds__(256) attn_row_dot(const bf16* __restrict__ o, const bf16* __restrict__ g,
+                                                    float* __restrict__ D, int64_t rows, int heads, int seq,
+                                                    int64_t ld) {
+  const int64_t t = int64_t(blockIdx.x) * 256 + threadIdx.x;
+  const int64_t pair = t >> 3;  // (row, head)
+  const int part = int(t & 7);
+  const bool ok = pair < rows * heads;
+  float d = 0.f;
+  int64_t row = 0;
+  int a = 0;
+  if (ok) {
+    row = pair / heads;
+    a = int(pair - row * heads);
+    const int64_t off = row * ld + a * 64 + part * 8;
+    const uint4 x = *reinterpret_cast<const uint4*>(o + off), y = *reinterpret_cast<const uint4*>(g + off);
+    const __nv_bfloat162* x2 = reinterpret_cast<const __nv_bfloat162*>(&x);
+    const __nv_bfloat162* y2 = reinterpret_cast<const __nv_bfloat162*>(&y);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const float2 u = __bfloat1622float2(x2[e]), w = __bfloat1622float2(y2[e]);
+      d += u.x * w.x + u.y * w.y;
+    }
+  }
+  d += __shfl_xor_sync(0xffffffffu, d, 1);
+  d += __shfl_xor_sync(0xffffffffu, d, 2);
+  d += __shfl_xor_sync(0xffffffffu, d, 4);
+  if (ok && part == 0) {
+    const int64_t b = row / seq, q = row - b * seq;
+    D[(b * heads + a) * seq + q] = d;
+  }
+}
+
 // dQ, persistent: a work item is 128 queries of one (sample, head); K and V stream through a
 // 3-stage TMA ring one 128-key tile at a time (so the next item's loads run ahead), Q / dO
 // are double-buffered per item, and dQ accumulates in one of two TMEM buffers so an item's
 // epilogue overlaps the next item's products.  One TMA thread, one MMA thread, 16 compute
-// warps.  D_q = dO_q . O_q is formed by the first column group of each item (and stored for
-// the dK/dV kernel).
+// warps.  D_q = dO_q . O_q comes from attn_row_dot (launched first).
 // smem: Q 2 x 16K | dO 2 x 16K | K,V ring 3 x 32K | dS 2 x 32K | D 2 x 512 B | barriers
 // TMEM: S 0..127, dP 128..255, dQ 256..319 / 320..383
 constexpr int kDqStages = 3;
@@ -161,7 +192,6 @@ __global__ void __launch_bounds__(kDqThreads, 1)
            *kv_empty = bar + 7 /*[3]*/, *s_full = bar + 10, *s_free = bar + 11, *ds_full = bar + 12 /*[2]*/,
            *ds_free = bar + 14 /*[2]*/, *dq_full = bar + 16 /*[2]*/, *dq_empty = bar + 18 /*[2]*/;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 20);
-  float* sD = reinterpret_cast<float*>(smem + kDqSmemD);  // [2][128]
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   constexpr int kTma = kBwdCW, kMma = kBwdCW + 1;
   if (threadIdx.x == 0) {
@@ -262,32 +292,7 @@ __global__ void __launch_bounds__(kDqThreads, 1)
       const int qt = item % nqt, ah = item / nqt, a = ah % p.heads, b = ah / p.heads;
       const int q = qt * 128 + i;
       const int64_t hrow = (int64_t(b) * p.heads + a) * S + q;
-      float* sd = sD + (it & 1) * 128;
-      if (cg == 0) {  // D_q = dO_q . O_q in fp32 over the bf16 row
-        const bf16* orow = p.o + (int64_t(b) * S + q) * p.ld + a * 64;
-        const bf16* grow = p.dout + (int64_t(b) * S + q) * p.ld + a * 64;
-        uint4 x[8], y[8];
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          x[j] = *reinterpret_cast<const uint4*>(orow + 8 * j);
-          y[j] = *reinterpret_cast<const uint4*>(grow + 8 * j);
-        }
-        float D = 0.f;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const __nv_bfloat162* x2 = reinterpret_cast<const __nv_bfloat162*>(&x[j]);
-          const __nv_bfloat162* y2 = reinterpret_cast<const __nv_bfloat162*>(&y[j]);
-#pragma unroll
-          for (int e = 0; e < 4; ++e) {
-            const float2 u = __bfloat1622float2(x2[e]), w = __bfloat1622float2(y2[e]);
-            D += u.x * w.x + u.y * w.y;
-          }
-        }
-        sd[i] = D;
-        p.D[hrow] = D;
-      }
-      named_sync(2, 32 * kBwdCW);
-      const float D = sd[i];
+      const float D = p.D[hrow];  // attn_row_dot
       const float l2 = p.lse[hrow] * kLog2e;
       const uint32_t* mrow = p.mask + hrow * (S / 32);
       for (int kt = 0; kt < nkt; ++kt, ++kc) {
@@ -333,43 +338,51 @@ __global__ void __launch_bounds__(kDqThreads, 1)
   }
 }
 
-// dK, dV for 128 keys of one (sample, head); loops over 128-query tiles (double-buffered Q, dO).
-// P_d (dropped, scaled P) and dS are written query-major ([query][key] rows, SW128), which is
-// the MN-major layout of the A operands P_d^T and dS^T of dV += P_d^T dO and dK += dS^T Q.
-// smem: K 16K | V 16K | Q 2 x 16K | dO 2 x 16K | P_d 2 x 32K | dS 2 x 32K | barriers
-// TMEM: S 0..127, dP 128..255 (lanes = queries), dV 256..319, dK 320..383 (lanes = keys)
-__global__ void __launch_bounds__(kBwdThreads, 1)
+// dK, dV, persistent: a work item is 128 keys of one (sample, head); K and V are
+// double-buffered per item, Q and dO stream through a 3-stage TMA ring one 128-query tile at
+// a time, and dK / dV accumulate in one of two TMEM buffer pairs so an item's epilogue
+// overlaps the next item's products.  P_d (dropped, scaled P) and dS are written query-major
+// ([query][key] rows, SW128) — the MN-major layout of the A operands P_d^T and dS^T of
+// dV += P_d^T dO and dK += dS^T Q.  One TMA thread, one MMA thread, 16 compute warps.
+// smem: K,V 2 x 32K | Q,dO ring 3 x 32K | P_d 32K | dS 32K | barriers
+// TMEM: S 0..127, dP 128..255 (lanes = queries); dV, dK 256..383 / 384..511 (lanes = keys)
+constexpr int kKvStages = 3;
+constexpr int kKvThreads = 32 * (kBwdCW + 2);
+constexpr int kKvSmemKV = 0, kKvSmemQG = 65536, kKvSmemPd = kKvSmemQG + kKvStages * 32768;
+constexpr int kKvSmemDS = kKvSmemPd + 32768, kKvSmemBar = kKvSmemDS + 32768;
+constexpr int kKvSmem = kKvSmemBar + 256 + 1024;
+__global__ void __launch_bounds__(kKvThreads, 1)
     fa5_bwd_dkv(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mdO,
                 const __grid_constant__ CUtensorMap mK, const __grid_constant__ CUtensorMap mV, const Fa5B p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  const int S = p.seq, nqt = S / 128;
-  uint8_t* sK = smem;
-  uint8_t* sV = smem + 16384;
-  uint8_t* sQ = smem + 32768;    // two 16 KB buffers
-  uint8_t* sG = smem + 65536;    // two 16 KB buffers
-  uint8_t* sPd = smem + 98304;   // two 32 KB buffers
-  uint8_t* sdS = smem + 163840;  // two 32 KB buffers
-  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + 229376);
-  uint64_t *ld_kv = bar, *qd_full = bar + 1 /*[2]*/, *s_full = bar + 3, *s_free = bar + 4, *ps_full = bar + 5 /*[2]*/,
-           *acc_done = bar + 7 /*[2]*/;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 9);
+  const int S = p.seq, nqt = S / 128, nkt = S / 128;
+  const int items = p.nb * p.heads * nkt;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + kKvSmemBar);
+  uint64_t *kv_full = bar /*[2]*/, *kv_empty = bar + 2 /*[2]*/, *qd_full = bar + 4 /*[3]*/, *qd_empty = bar + 7 /*[3]*/,
+           *s_full = bar + 10, *s_free = bar + 11, *ps_full = bar + 12, *ps_free = bar + 13,
+           *acc_full = bar + 14 /*[2]*/, *acc_empty = bar + 16 /*[2]*/;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 18);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int kt = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
-  const int64_t hbase = (int64_t(b) * p.heads + a) * S;
+  constexpr int kTma = kBwdCW, kMma = kBwdCW + 1;
   if (threadIdx.x == 0) {
-    mbar_init(ld_kv, 1);
-    mbar_init(&qd_full[0], 1);
-    mbar_init(&qd_full[1], 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&kv_full[i], 1);
+      mbar_init(&kv_empty[i], 1);
+      mbar_init(&acc_full[i], 1);
+      mbar_init(&acc_empty[i], 32 * kBwdCW);
+    }
+    for (int i = 0; i < kKvStages; ++i) {
+      mbar_init(&qd_full[i], 1);
+      mbar_init(&qd_empty[i], 1);
+    }
     mbar_init(s_full, 1);
     mbar_init(s_free, 32 * kBwdCW);
-    mbar_init(&ps_full[0], 32 * kBwdCW);
-    mbar_init(&ps_full[1], 32 * kBwdCW);
-    mbar_init(&acc_done[0], 1);
-    mbar_init(&acc_done[1], 1);
+    mbar_init(ps_full, 32 * kBwdCW);
+    mbar_init(ps_free, 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (warp == kBwdCtl) {
+  if (warp == kMma) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
                  "r"(512));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
@@ -378,120 +391,142 @@ __global__ void __launch_bounds__(kBwdThreads, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
-  if (warp == kBwdCtl) {
+  if (warp == kTma) {
     if (lane == 0) {
-      const int row0 = b * S;
-      mbar_arrive_tx(ld_kv, 32768u);
-      tma_load(sK, &mK, ld_kv, a * 64, row0 + kt * 128, 0, 0);
-      tma_load(sV, &mV, ld_kv, a * 64, row0 + kt * 128, 0, 0);
-      auto load_qd = [&](int t) {
-        mbar_arrive_tx(&qd_full[t & 1], 32768u);
-        tma_load(sQ + (t & 1) * 16384, &mQ, &qd_full[t & 1], a * 64, row0 + t * 128, 0, 0);
-        tma_load(sG + (t & 1) * 16384, &mdO, &qd_full[t & 1], a * 64, row0 + t * 128, 0, 0);
-      };
-      load_qd(0);
-      if (nqt > 1) load_qd(1);
-      const uint32_t k = smem_u32(sK), v = smem_u32(sV);
+      int it = 0, qc = 0;
+      for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
+        const int kt = item % nkt, ah = item / nkt, a = ah % p.heads, b = ah / p.heads;
+        const int row0 = b * S, kb = it & 1;
+        if (it >= 2) mbar_wait(&kv_empty[kb], ((it >> 1) - 1) & 1);
+        mbar_arrive_tx(&kv_full[kb], 32768u);
+        tma_load(smem + kKvSmemKV + kb * 32768, &mK, &kv_full[kb], a * 64, row0 + kt * 128, 0, 0);
+        tma_load(smem + kKvSmemKV + kb * 32768 + 16384, &mV, &kv_full[kb], a * 64, row0 + kt * 128, 0, 0);
+        for (int t = 0; t < nqt; ++t, ++qc) {
+          const int st = qc % kKvStages;
+          if (qc >= kKvStages) mbar_wait(&qd_empty[st], ((qc / kKvStages) - 1) & 1);
+          mbar_arrive_tx(&qd_full[st], 32768u);
+          tma_load(smem + kKvSmemQG + st * 32768, &mQ, &qd_full[st], a * 64, row0 + t * 128, 0, 0);
+          tma_load(smem + kKvSmemQG + st * 32768 + 16384, &mdO, &qd_full[st], a * 64, row0 + t * 128, 0, 0);
+        }
+      }
+    }
+  } else if (warp == kMma) {
+    if (lane == 0) {
       // dV += P_d^T dO_t, dK += dS^T Q_t: A MN-major (keys contiguous, 64-key blocks 16 KB apart,
       // K step of 16 queries = 2 KB), B = dO / Q tile rows (MN-major)
       constexpr uint32_t idAcc = kIdN64MN | (1u << 15);
-      auto issue_acc = [&](int t) {
-        mbar_wait(&ps_full[t & 1], (t >> 1) & 1);
-        tc_fence_after();
-        const uint32_t pd = smem_u32(sPd) + uint32_t(t & 1) * 32768u, ds = smem_u32(sdS) + uint32_t(t & 1) * 32768u;
-        const uint32_t q = smem_u32(sQ) + uint32_t(t & 1) * 16384u, g = smem_u32(sG) + uint32_t(t & 1) * 16384u;
-        for (int kq = 0; kq < 128; kq += 16) {
-          const uint32_t acc = (t > 0 || kq > 0) ? 1u : 0u;
-          tc_mma(tmem + 256, smem_desc(pd + uint32_t(kq) * 128, 16384, 1024),
-                 smem_desc(g + uint32_t(kq) * 128, 8192, 1024), idAcc, acc);
-          tc_mma(tmem + 320, smem_desc(ds + uint32_t(kq) * 128, 16384, 1024),
-                 smem_desc(q + uint32_t(kq) * 128, 8192, 1024), idAcc, acc);
-        }
-        tc_commit(&acc_done[t & 1]);
-      };
-      mbar_wait(ld_kv, 0);
-      for (int t = 0; t < nqt; ++t) {
-        if (t > 0) mbar_wait(s_free, (t - 1) & 1);  // S, dP of tile t-1 are in registers
-        mbar_wait(&qd_full[t & 1], (t >> 1) & 1);
-        tc_fence_after();
-        const uint32_t q = smem_u32(sQ) + uint32_t(t & 1) * 16384u, g = smem_u32(sG) + uint32_t(t & 1) * 16384u;
-        // S = Q_t K^T, dP = dO_t V^T (M = 128 queries, N = 128 keys)
+      const uint32_t pd = smem_u32(smem + kKvSmemPd), ds = smem_u32(smem + kKvSmemDS);
+      int it = 0, qc = 0;
+      for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
+        const int kb = it & 1, ab = it & 1;
+        mbar_wait(&kv_full[kb], (it >> 1) & 1);
+        const uint32_t k = smem_u32(smem + kKvSmemKV + kb * 32768), v = k + 16384;
+        auto issue_acc = [&](int qcp, int first) {
+          mbar_wait(ps_full, qcp & 1);
+          tc_fence_after();
+          const uint32_t q = smem_u32(smem + kKvSmemQG + (qcp % kKvStages) * 32768), g = q + 16384;
+          for (int kq = 0; kq < 128; kq += 16) {
+            const uint32_t acc = (first && kq == 0) ? 0u : 1u;
+            tc_mma(tmem + 256 + uint32_t(ab * 128), smem_desc(pd + uint32_t(kq) * 128, 16384, 1024),
+                   smem_desc(g + uint32_t(kq) * 128, 8192, 1024), idAcc, acc);
+            tc_mma(tmem + 320 + uint32_t(ab * 128), smem_desc(ds + uint32_t(kq) * 128, 16384, 1024),
+                   smem_desc(q + uint32_t(kq) * 128, 8192, 1024), idAcc, acc);
+          }
+          tc_commit(ps_free);
+          tc_commit(&qd_empty[qcp % kKvStages]);
+        };
+        for (int t = 0; t < nqt; ++t, ++qc) {
+          const int st = qc % kKvStages;
+          mbar_wait(&qd_full[st], (qc / kKvStages) & 1);
+          if (qc > 0) mbar_wait(s_free, (qc - 1) & 1);  // the previous S, dP are in registers
+          tc_fence_after();
+          const uint32_t q = smem_u32(smem + kKvSmemQG + st * 32768), g = q + 16384;
+          // S = Q_t K^T, dP = dO_t V^T (M = 128 queries, N = 128 keys)
 #pragma unroll
-        for (int kk = 0; kk < 4; ++kk) {
-          tc_mma(tmem, smem_desc(q + kk * 32, 16, 1024), smem_desc(k + kk * 32, 16, 1024), kIdN128, kk > 0 ? 1u : 0u);
-          tc_mma(tmem + 128, smem_desc(g + kk * 32, 16, 1024), smem_desc(v + kk * 32, 16, 1024), kIdN128,
-                 kk > 0 ? 1u : 0u);
-        }
-        tc_commit(s_full);
-        if (t > 0) {
-          issue_acc(t - 1);
-          if (t + 1 < nqt) {
-            mbar_wait(&acc_done[(t - 1) & 1], ((t - 1) >> 1) & 1);  // Q/dO buffer (t+1)&1 is free
-            load_qd(t + 1);
+          for (int kk = 0; kk < 4; ++kk) {
+            tc_mma(tmem, smem_desc(q + kk * 32, 16, 1024), smem_desc(k + kk * 32, 16, 1024), kIdN128, kk > 0 ? 1u : 0u);
+            tc_mma(tmem + 128, smem_desc(g + kk * 32, 16, 1024), smem_desc(v + kk * 32, 16, 1024), kIdN128,
+                   kk > 0 ? 1u : 0u);
+          }
+          tc_commit(s_full);
+          if (t == nqt - 1) tc_commit(&kv_empty[kb]);  // every product reading K, V of this item issued
+          if (t > 0) {
+            if (t == 1 && it >= 2) mbar_wait(&acc_empty[ab], ((it >> 1) - 1) & 1);
+            issue_acc(qc - 1, t == 1);
           }
         }
+        if (nqt == 1 && it >= 2) mbar_wait(&acc_empty[ab], ((it >> 1) - 1) & 1);
+        issue_acc(qc - 1, nqt == 1);
+        tc_commit(&acc_full[ab]);
       }
-      issue_acc(nqt - 1);
     }
   } else {
     const int qw = warp & 3, cg = warp >> 2;  // TMEM lane quarter, 32-key group
     const int i = qw * 32 + lane;
     const uint32_t trow = tmem + (uint32_t(qw * 32) << 16);
-    // row constants of query tile t (lse, D, keep word), prefetched one tile ahead
-    auto row_consts = [&](int t, float& l2, float& D, uint32_t& bits) {
-      const int64_t hrow = hbase + t * 128 + i;
-      l2 = p.lse[hrow] * kLog2e;
-      D = p.D[hrow];
-      bits = p.drop ? p.mask[hrow * (S / 32) + kt * 4 + cg] : ~0u;
-    };
-    float nl2, nD;
-    uint32_t nbits;
-    row_consts(0, nl2, nD, nbits);
-    for (int t = 0; t < nqt; ++t) {
-      const float l2 = nl2, D = nD;
-      const uint32_t bits = nbits;
-      if (t + 1 < nqt) row_consts(t + 1, nl2, nD, nbits);
-      mbar_wait(s_full, t & 1);
-      tc_fence_after();
-      uint32_t rs[32], rp[32];
-      tmem_ld32_nw(trow + uint32_t(cg * 32), rs);
-      tmem_ld32_nw(trow + uint32_t(128 + cg * 32), rp);
-      tmem_wait_ld();
-      tc_fence_before();
-      mbar_arrive(s_free);
-      // in place: rp <- P_d, rs <- dS (fp32 bits)
+    const uint32_t pd = smem_u32(smem + kKvSmemPd), ds = smem_u32(smem + kKvSmemDS);
+    int it = 0, qc = 0;
+    for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
+      const int kt = item % nkt, ah = item / nkt, a = ah % p.heads, b = ah / p.heads;
+      const int64_t hbase = (int64_t(b) * p.heads + a) * S;
+      // row constants of query tile t (lse, D, keep word), prefetched one tile ahead
+      auto row_consts = [&](int t, float& l2, float& D, uint32_t& bits) {
+        const int64_t hrow = hbase + t * 128 + i;
+        l2 = p.lse[hrow] * kLog2e;
+        D = p.D[hrow];
+        bits = p.drop ? p.mask[hrow * (S / 32) + kt * 4 + cg] : ~0u;
+      };
+      float nl2, nD;
+      uint32_t nbits;
+      row_consts(0, nl2, nD, nbits);
+      for (int t = 0; t < nqt; ++t, ++qc) {
+        const float l2 = nl2, D = nD;
+        const uint32_t bits = nbits;
+        if (t + 1 < nqt) row_consts(t + 1, nl2, nD, nbits);
+        mbar_wait(s_full, qc & 1);
+        tc_fence_after();
+        uint32_t rs[32], rp[32];
+        tmem_ld32_nw(trow + uint32_t(cg * 32), rs);
+        tmem_ld32_nw(trow + uint32_t(128 + cg * 32), rp);
+        tmem_wait_ld();
+        tc_fence_before();
+        mbar_arrive(s_free);
+        // in place: rp <- P_d, rs <- dS (fp32 bits)
 #pragma unroll
-      for (int j = 0; j < 32; ++j) {
-        const bool keep = (bits >> j) & 1u;
-        const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
-        const float dp = keep ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
-        rp[j] = __float_as_uint(keep ? pr * p.keep_scale : 0.f);
-        rs[j] = __float_as_uint(pr * (dp - D));
+        for (int j = 0; j < 32; ++j) {
+          const bool keep = (bits >> j) & 1u;
+          const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
+          const float dp = keep ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
+          rp[j] = __float_as_uint(keep ? pr * p.keep_scale : 0.f);
+          rs[j] = __float_as_uint(pr * (dp - D));
+        }
+        if (qc > 0) mbar_wait(ps_free, (qc - 1) & 1);  // the previous tile's dV, dK products read P_d / dS
+        st_row32(pd, i, cg * 32, reinterpret_cast<const float*>(rp));
+        st_row32(ds, i, cg * 32, reinterpret_cast<const float*>(rs));
+        fence_async_smem();
+        tc_fence_before();
+        mbar_arrive(ps_full);
       }
-      if (t >= 2) mbar_wait(&acc_done[t & 1], ((t - 2) >> 1) & 1);  // P_d / dS buffers t&1 free
-      st_row32(smem_u32(sPd) + uint32_t(t & 1) * 32768u, i, cg * 32, reinterpret_cast<const float*>(rp));
-      st_row32(smem_u32(sdS) + uint32_t(t & 1) * 32768u, i, cg * 32, reinterpret_cast<const float*>(rs));
-      fence_async_smem();
+      mbar_wait(&acc_full[it & 1], (it >> 1) & 1);
+      tc_fence_after();
+      // accumulator lanes are keys: group 0/1 store dV columns 0-31 / 32-63, group 2/3 dK
+      const int key = kt * 128 + i;
+      const int64_t off = (int64_t(b) * S + key) * p.ld + a * 64 + (cg & 1) * 32;
+      uint32_t r0[32];
+      tmem_ld32(trow + 256u + uint32_t((it & 1) * 128 + cg * 32), r0);
       tc_fence_before();
-      mbar_arrive(&ps_full[t & 1]);
-    }
-    mbar_wait(&acc_done[(nqt - 1) & 1], ((nqt - 1) >> 1) & 1);
-    tc_fence_after();
-    // accumulator lanes are keys: group 0/1 store dV columns 0-31 / 32-63, group 2/3 dK
-    const int key = kt * 128 + i;
-    const int64_t off = (int64_t(b) * S + key) * p.ld + a * 64 + (cg & 1) * 32;
-    uint32_t r0[32];
-    tmem_ld32(trow + 256u + uint32_t(cg * 32), r0);
-    if (cg < 2) {
-      if (p.dv) store_row32(static_cast<bf16*>(p.dv) + off, r0, 1.f, p.acc_v);
-    } else {
-      if (p.dk) store_row32(static_cast<bf16*>(p.dk) + off, r0, p.alpha, p.acc_k);
+      mbar_arrive(&acc_empty[it & 1]);
+      if (cg < 2) {
+        if (p.dv) store_row32(static_cast<bf16*>(p.dv) + off, r0, 1.f, p.acc_v);
+      } else {
+        if (p.dk) store_row32(static_cast<bf16*>(p.dk) + off, r0, p.alpha, p.acc_k);
+      }
     }
   }
   __syncwarp();
   tc_fence_before();
   __syncthreads();
-  if (warp == kBwdCtl) {
+  if (warp == kMma) {
     tc_fence_after();
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
   }
@@ -734,10 +769,10 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
         uint32_t bits = 0xFFFFFFFFu;
         if (p.p > 0.f) {
           bits = 0u;
-#pragma unroll
           // one Philox call per eight keys of the row (D-RNG); erow + key is a multiple of 32,
           // so the four counters share the high word
           const uint64_t cnt0 = (erow + uint64_t(key)) >> 3;
+#pragma unroll
           for (int u = 0; u < 4; ++u) {
             const uint4 w = philox4x32_10(uint32_t(cnt0) + uint32_t(u), uint32_t(cnt0 >> 32), p.step, 0u, p.seed,
                                           kPhiloxKey1);
@@ -881,19 +916,24 @@ bool attention_bwd_tc5(const AttnArgs& A, cudaStream_t st) {
   p.acc_q = A.acc_q;
   p.acc_k = A.acc_k;
   p.acc_v = A.acc_v;
-  const int smem_kv = 229376 + 256 + 1024;
   static int sms = 0;
   if (!sms) {
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaFuncSetAttribute(fa5_bwd_dq, cudaFuncAttributeMaxDynamicSharedMemorySize, kDqSmem);
-    cudaFuncSetAttribute(fa5_bwd_dkv, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_kv);
+    cudaFuncSetAttribute(fa5_bwd_dkv, cudaFuncAttributeMaxDynamicSharedMemorySize, kKvSmem);
   }
   p.nb = A.nb;
+  {
+    const int64_t threads = rows * A.heads * 8;
+    attn_row_dot<<<int((threads + 255) / 256), 256, 0, st>>>(static_cast<const bf16*>(A.c),
+                                                           static_cast<const bf16*>(A.dc), A.ws, rows, A.heads,
+                                                           A.seq, A.ld);
+  }
   const int items_q = A.nb * A.heads * (A.seq / 128);
   fa5_bwd_dq<<<items_q < sms ? items_q : sms, kDqThreads, kDqSmem, st>>>(mq, mg, mk, mv, p);
-  fa5_bwd_dkv<<<dim3(A.seq / 128, A.heads, A.nb), kBwdThreads, smem_kv, st>>>(mq, mg, mk, mv, p);
+  fa5_bwd_dkv<<<items_q < sms ? items_q : sms, kKvThreads, kKvSmem, st>>>(mq, mg, mk, mv, p);
   return true;
 }
 
