@@ -579,12 +579,12 @@ __global__ void __launch_bounds__(256) colsum_bf16_kernel(const bf16* __restrict
   const int64_t rstep = int64_t(G) * 8;
   int64_t r = int64_t(blockIdx.y) * 8 + w;
   if (colok) {
-    for (; r + 7 * rstep < rows; r += 8 * rstep) {
-      uint4 u[8];
+    for (; r + 15 * rstep < rows; r += 16 * rstep) {
+      uint4 u[16];
 #pragma unroll
-      for (int k = 0; k < 8; ++k) u[k] = __ldcs(reinterpret_cast<const uint4*>(x + (r + k * rstep) * N + c0));
+      for (int k = 0; k < 16; ++k) u[k] = __ldcs(reinterpret_cast<const uint4*>(x + (r + k * rstep) * N + c0));
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
+      for (int k = 0; k < 16; ++k) {
         const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u[k]);
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
@@ -623,7 +623,21 @@ __global__ void __launch_bounds__(256) colsum_bf16_kernel(const bf16* __restrict
   __threadfence();
   double d[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   if (colok) {
-    for (int b = w; b < G; b += 8) {
+    int b = w;
+    for (; b + 8 * 7 < G; b += 8 * 8) {  // eight partial rows in flight per thread
+      float4 u[8][2];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        u[k][0] = __ldcg(reinterpret_cast<const float4*>(ws + int64_t(b + 8 * k) * N + c0));
+        u[k][1] = __ldcg(reinterpret_cast<const float4*>(ws + int64_t(b + 8 * k) * N + c0 + 4));
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        d[0] += u[k][0].x; d[1] += u[k][0].y; d[2] += u[k][0].z; d[3] += u[k][0].w;
+        d[4] += u[k][1].x; d[5] += u[k][1].y; d[6] += u[k][1].z; d[7] += u[k][1].w;
+      }
+    }
+    for (; b < G; b += 8) {
       const float4 u0 = __ldcg(reinterpret_cast<const float4*>(ws + int64_t(b) * N + c0));
       const float4 u1 = __ldcg(reinterpret_cast<const float4*>(ws + int64_t(b) * N + c0 + 4));
       d[0] += u0.x; d[1] += u0.y; d[2] += u0.z; d[3] += u0.w;
@@ -1211,8 +1225,10 @@ void column_sum(int dt, const void* x, int64_t rows, int N, float* ws, uint64_t 
                 const int* filter, int fval, cudaStream_t st) {
   const int cb = (N + 255) / 256;
   if (dt == BF16 && !filter && N % 8 == 0 && (reinterpret_cast<uintptr_t>(x) % 16) == 0 && rows >= 64) {
-    // ~2 blocks of 256 threads per SM, at least 32 rows per block
-    int G = int(296 / cb);
+    // ~512 blocks (~3.5 per SM; a [16384, 1024] input gives 16 rows per thread, one round of
+    // loads in flight), at least one block per SM, at least 32 rows per block
+    int G = 512 / cb;
+    if (G * cb < 148) G = (148 + cb - 1) / cb;
     if (G > rows / 32) G = int(rows / 32);
     const int64_t ws_rows = int64_t((ws_bytes - kTicketBytes) / (uint64_t(N) * 4));
     if (G > ws_rows) G = int(ws_rows);
