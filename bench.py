@@ -491,6 +491,21 @@ def main():
                 "h2d_bytes_per_step": h2d_bytes, "d2h_bytes_per_step": 4},
         "roofline": roof,
     }
+    # north_star's governing roofline of the whole budgeted step: the slower of the plan's
+    # FLOP (recompute included) at the sustained tensor peak and its swap bytes at the
+    # measured pinned PCIe bandwidth of this GPU (SURVEY.md §8(d) "Roofline")
+    bw = pcie if pcie else (55e9, 55e9)
+    t_tc = pst["compute_flop"] / (peak * 1e12) if peak else 0.0
+    t_pcie = max(pst["d2h_bytes"] / bw[0], pst["h2d_bytes"] / bw[1])
+    t_roof = max(t_tc, t_pcie)
+    step_s = dt / args.steps
+    line["roofline_step"] = {
+        "bound": "tensor" if t_tc >= t_pcie else "pcie", "t_roof_ms": t_roof * 1e3,
+        "t_tensor_ms": t_tc * 1e3, "t_pcie_ms": t_pcie * 1e3, "ms_per_step": step_s * 1e3,
+        "frac": t_roof / step_s, "plan_flop": pst["compute_flop"], "unsplit_flop": bst["compute_flop"],
+        "pcie_gbs": [round(x / 1e9, 1) for x in bw], "pcie_source": "measured" if pcie else "fallback 55 GB/s",
+        "how": "t_roof = max(plan FLOP / bf16_tflops_sustained, max(D2H bytes / B_d2h, H2D bytes / B_h2d)); "
+               "frac = t_roof / measured step time"}
     if not cnn:
         line["roofline_attention_gemm"] = {
             "bound": "hbm", "kernel": "gemm_tc on per-(sample, head) attention products",

@@ -302,6 +302,17 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch,
                        const void* B, int64_t ldb, int64_t strideB, int32_t tb,
                        void* C, int64_t ldc, int64_t strideC, int32_t c_dtype,
                        float alpha, float beta, const void* bias_bf16, void* stream);
+/* Tile-selection override for the tcgen05 GEMM (tests and microbenchmarks; process-
+ * wide, not thread-safe against concurrent launches): mode 0 = cost model (default),
+ * 1 = single-CTA 128-row tiles only, 2 = CTA-pair (cta_group::2, 256-row) tiles
+ * whenever M > 128 and N > 64; + 4 = never run the last partial wave as half-width
+ * units.  TS_ERR_ARG for any other value. */
+ts_status ts_gemm_set_mode(int32_t mode);
+/* Configuration of the last tcgen05 GEMM launch: out8 = {tile width, CTAs per tile
+ * (1 or 2), split-K factor, work units, SMs, co-resident CTA pairs, first half-width
+ * tail unit (= work units when the tail wave is not split), 0}.  Host memory, 8 int32
+ * written; TS_ERR_ARG when out8 is NULL. */
+ts_status ts_gemm_last_config(int32_t* out8);
 ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K,
                       const float* A, int64_t lda, int32_t ta,
                       const float* B, int64_t ldb, int32_t tb,

@@ -34,9 +34,11 @@ constexpr int num_threads() { return 64 + 32 * EW; }  // warp0 TMA, warp1 MMA, w
 
 struct TcParams {
   int M, N, K, nb1, nb2;
+  int bm;  // output rows per work unit: BM (one CTA) or 2 BM (a CTA pair, cta_group::2)
   int tiles_m, tiles_n, num_tiles, num_kb;
   int n_fastest;  // 1: consecutive tiles walk N (A, the larger operand, is streamed once)
   int ksplit, kb_per_split, num_units;  // work unit = (tile, K slice)
+  int split_from;  // units >= split_from are half-width tail units (2 per tile, ksplit == 1)
   int a_mn, b_mn;
   void* C;
   int64_t ldc, cbs1, cbs2;
@@ -64,6 +66,22 @@ constexpr int num_stages() {
   return n > 8 ? 8 : n;
 }
 
+// Work unit -> (tile, K slice, half).  The last partial wave's tiles (tiles >= split_from)
+// run as two half-width units each (half = 0 / 1 selects the columns), so the tail wave
+// of e.g. 512 tiles on 148 SMs costs half a wave instead of a whole one.
+__device__ __forceinline__ void decode_unit(const TcParams& p, int unit, int& tile, int& ks, int& hsel) {
+  if (unit < p.split_from) {
+    tile = unit / p.ksplit;
+    ks = unit - tile * p.ksplit;
+    hsel = -1;
+  } else {
+    const int j = unit - p.split_from;
+    tile = p.split_from + (j >> 1);
+    ks = 0;
+    hsel = j & 1;
+  }
+}
+
 __device__ __forceinline__ void decode_tile(const TcParams& p, int tile, int& b1, int& b2, int& m0, int& n0) {
   int per = p.tiles_m * p.tiles_n;
   int bb = tile / per;
@@ -80,24 +98,36 @@ __device__ __forceinline__ void decode_tile(const TcParams& p, int tile, int& b1
   }
   b1 = bb % p.nb1;
   b2 = bb / p.nb1;
-  m0 = mt * BM;
+  m0 = mt * p.bm;
   n0 = nt;  // scaled by BN by the caller
 }
 
-template <int BN, bool F32OUT, int EW>
+// CG = 1: one CTA per 128 x BN output tile.  CG = 2: a CTA pair (2-CTA cluster on one
+// TPC) computes a 256 x BN tile with tcgen05.mma.cta_group::2 issued by the leader
+// (rank 0): each CTA stages its own 128 rows of A and half (BN/2 rows) of B, so the
+// pair reads B once for 256 rows and each SM's smem feeds half the B bytes per MMA;
+// both CTAs' TMA bytes complete on the leader's full barrier, MMA commits multicast
+// to both CTAs' empty/tfull barriers, and each CTA's epilogue drains its own TMEM
+// (128 lanes x BN columns) and arrives on the leader's tempty barrier.
+template <int BN, bool F32OUT, int EW, int CG>
 __global__ void __launch_bounds__(num_threads<EW>(), 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmC2,
                    const TcParams p) {
+  constexpr int BNL = BN / CG;  // B rows staged by this CTA
   constexpr int A_BYTES = BM * BK * 2;
-  constexpr int B_BYTES = BN * BK * 2;
+  constexpr int B_BYTES = BNL * BK * 2;
   constexpr int STAGE = A_BYTES + B_BYTES;
-  constexpr int STAGES = num_stages<BN, F32OUT, EW>();
+  constexpr int STAGES = num_stages<BNL, F32OUT, EW>();
   constexpr uint32_t TMEM_COLS = 2 * BN;
   constexpr int BUF = 32 * 32 * (F32OUT ? 4 : 2);
-  // instruction descriptor: D f32, A/B bf16, M = 128, N = BN
+  // instruction descriptor: D f32, A/B bf16, M = 128 CG, N = BN
   const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(p.a_mn) << 15) |
-                         (uint32_t(p.b_mn) << 16) | (uint32_t(BN >> 3) << 17) | (uint32_t(BM >> 4) << 24);
+                         (uint32_t(p.b_mn) << 16) | (uint32_t(BN >> 3) << 17) | (uint32_t((BM * CG) >> 4) << 24);
+  // half-width tail units: N = BN / 2
+  const uint32_t idesc_h = (idesc & ~(0x3Fu << 17)) | (uint32_t(BN >> 4) << 17);
+  const uint32_t rank = CG == 2 ? cluster_ctarank() : 0u;  // rows rank*128.. of the unit
+  const int cid = blockIdx.x / CG, ncl = gridDim.x / CG;     // cluster = consecutive blocks
 
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -116,19 +146,26 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
     }
     for (int s = 0; s < 2; ++s) {
       mbar_init(&tfull[s], 1);
-      mbar_init(&tempty[s], 32 * EW);
+      mbar_init(&tempty[s], EW * CG);  // one arrive per epilogue warp of each CTA
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
   }
   if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                 "r"(TMEM_COLS));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    if constexpr (CG == 1) {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                   "r"(TMEM_COLS));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    } else {
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
+                   "r"(TMEM_COLS));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    }
   }
   tc_fence_before();
   __syncthreads();
+  if constexpr (CG == 2) cluster_sync();  // peer barriers initialised before any remote signal
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
@@ -137,30 +174,52 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
       // ===== TMA producer =====
       int stage = 0;
       uint32_t phase = 0;
-      for (int unit = blockIdx.x; unit < p.num_units; unit += gridDim.x) {
-        const int tile = unit / p.ksplit, ks = unit - tile * p.ksplit;
+      for (int unit = cid; unit < p.num_units; unit += ncl) {
+        int tile, ks, hsel;
+        decode_unit(p, unit, tile, ks, hsel);
         int b1, b2, m0, nt;
         decode_tile(p, tile, b1, b2, m0, nt);
-        int n0 = nt * BN;
+        m0 += int(rank) * BM;
+        // a half-width unit stages B rows [n0 + hsel BN/2 + rank BN/(2 CG), +BNL) (the box
+        // is fixed; the MMA reads only the first BN/(2 CG) rows of each CTA's half)
+        const int n0 = nt * BN + (hsel < 0 ? int(rank) * BNL : hsel * (BN / 2) + int(rank) * (BNL / 2));
         const int kb0 = ks * p.kb_per_split;
         const int kb1 = min(p.num_kb, kb0 + p.kb_per_split);
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * STAGE;
           uint8_t* sb = sa + A_BYTES;
-          mbar_arrive_tx(&full[stage], STAGE);
           const int k0 = kb * BK;
-          if (!p.a_mn) {
-            tma_load(sa, &tmA, &full[stage], k0, m0, b1, b2);
-          } else {
+          if constexpr (CG == 1) {
+            mbar_arrive_tx(&full[stage], STAGE);
+            if (!p.a_mn) {
+              tma_load(sa, &tmA, &full[stage], k0, m0, b1, b2);
+            } else {
 #pragma unroll
-            for (int i = 0; i < BM / 64; ++i) tma_load(sa + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, b1, b2);
-          }
-          if (!p.b_mn) {
-            tma_load(sb, &tmB, &full[stage], k0, n0, b1, b2);
-          } else {
+              for (int i = 0; i < BM / 64; ++i) tma_load(sa + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, b1, b2);
+            }
+            if (!p.b_mn) {
+              tma_load(sb, &tmB, &full[stage], k0, n0, b1, b2);
+            } else {
 #pragma unroll
-            for (int i = 0; i < BN / 64; ++i) tma_load(sb + i * 8192, &tmB, &full[stage], n0 + 64 * i, k0, b1, b2);
+              for (int i = 0; i < BNL / 64; ++i) tma_load(sb + i * 8192, &tmB, &full[stage], n0 + 64 * i, k0, b1, b2);
+            }
+          } else {
+            // both CTAs' bytes complete on the leader's barrier; only the leader arrives
+            if (rank == 0) mbar_arrive_tx(&full[stage], 2 * STAGE);
+            const uint32_t fb = mapa_shared(smem_u32(&full[stage]), 0);
+            if (!p.a_mn) {
+              tma_load_2sm(sa, &tmA, fb, k0, m0, b1, b2);
+            } else {
+#pragma unroll
+              for (int i = 0; i < BM / 64; ++i) tma_load_2sm(sa + i * 8192, &tmA, fb, m0 + 64 * i, k0, b1, b2);
+            }
+            if (!p.b_mn) {
+              tma_load_2sm(sb, &tmB, fb, k0, n0, b1, b2);
+            } else {
+#pragma unroll
+              for (int i = 0; i < BNL / 64; ++i) tma_load_2sm(sb + i * 8192, &tmB, fb, n0 + 64 * i, k0, b1, b2);
+            }
           }
           if (++stage == STAGES) {
             stage = 0;
@@ -170,8 +229,8 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
-      // ===== MMA issuer (single thread) =====
+    if (lane == 0 && rank == 0) {
+      // ===== MMA issuer (single thread; the pair leader for CG = 2) =====
       int stage = 0;
       uint32_t phase = 0;
       int acc = 0;
@@ -181,8 +240,10 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
       // (SBO), K step of 16 = +2048 B.
       const uint32_t a_lbo = p.a_mn ? 8192 : 16, b_lbo = p.b_mn ? 8192 : 16;
       const uint32_t a_kstep = p.a_mn ? 2048 : 32, b_kstep = p.b_mn ? 2048 : 32;
-      for (int unit = blockIdx.x; unit < p.num_units; unit += gridDim.x) {
-        const int ks = unit % p.ksplit;
+      for (int unit = cid; unit < p.num_units; unit += ncl) {
+        int tile, ks, hsel;
+        decode_unit(p, unit, tile, ks, hsel);
+        const uint32_t id = hsel < 0 ? idesc : idesc_h;
         const int kb0 = ks * p.kb_per_split;
         const int kb1 = min(p.num_kb, kb0 + p.kb_per_split);
         mbar_wait(&tempty[acc], acc_phase ^ 1);
@@ -197,15 +258,18 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
           for (int k = 0; k < BK / 16; ++k) {
             uint64_t ad = smem_desc(sa + k * a_kstep, a_lbo, 1024);
             uint64_t bd = smem_desc(sb + k * b_kstep, b_lbo, 1024);
-            tc_mma(tmem_d, ad, bd, idesc, (kb > kb0 || k > 0) ? 1u : 0u);
+            if constexpr (CG == 1) tc_mma(tmem_d, ad, bd, id, (kb > kb0 || k > 0) ? 1u : 0u);
+            else tc_mma2(tmem_d, ad, bd, id, (kb > kb0 || k > 0) ? 1u : 0u);
           }
-          tc_commit(&empty[stage]);
+          if constexpr (CG == 1) tc_commit(&empty[stage]);
+          else tc_commit2(&empty[stage], 3);
           if (++stage == STAGES) {
             stage = 0;
             phase ^= 1;
           }
         }
-        tc_commit(&tfull[acc]);
+        if constexpr (CG == 1) tc_commit(&tfull[acc]);
+        else tc_commit2(&tfull[acc], 3);
         if (++acc == 2) {
           acc = 0;
           acc_phase ^= 1;
@@ -224,18 +288,22 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
     int acc = 0;
     uint32_t acc_phase = 0;
     const int es = p.c_f32 ? 4 : 2;
-    for (int unit = blockIdx.x; unit < p.num_units; unit += gridDim.x) {
-      const int tile = unit / p.ksplit;
+    const uint32_t tempty_leader = CG == 2 ? mapa_shared(smem_u32(&tempty[0]), 0) : 0u;
+    for (int unit = cid; unit < p.num_units; unit += ncl) {
+      int tile, ks, hsel;
+      decode_unit(p, unit, tile, ks, hsel);
       int b1, b2, m0, nt;
       decode_tile(p, tile, b1, b2, m0, nt);
-      int n0 = nt * BN;
+      m0 += int(rank) * BM;
+      const int n0 = nt * BN + (hsel < 0 ? 0 : hsel * (BN / 2));
+      const int nchunks = (hsel < 0 ? BN : BN / 2) / 32;
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const int row = m0 + q * 32 + lane;
       const bool row_ok = row < p.M;
       const int64_t cbase = int64_t(b1) * p.cbs1 + int64_t(b2) * p.cbs2 + int64_t(row) * p.ldc;
 #pragma unroll 1
-      for (int c = half; c < BN / 32; c += kGrp) {
+      for (int c = half; c < nchunks; c += kGrp) {
         uint32_t r[32];
         tmem_ld32(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * BN + c * 32), r);
         const int col0 = n0 + c * 32;
@@ -350,7 +418,11 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
         __syncwarp();
       }
       tc_fence_before();
-      mbar_arrive(&tempty[acc]);
+      __syncwarp();
+      if (lane == 0) {
+        if constexpr (CG == 1) mbar_arrive(&tempty[acc]);
+        else mbar_arrive_cluster(tempty_leader + uint32_t(acc * 8));
+      }
       if (++acc == 2) {
         acc = 0;
         acc_phase ^= 1;
@@ -362,9 +434,13 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
   __syncwarp();
   tc_fence_before();
   __syncthreads();
+  if constexpr (CG == 2) cluster_sync();  // no CTA leaves while its peer may still signal it
   if (warp == 1) {
     tc_fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(TMEM_COLS));
+    if constexpr (CG == 1)
+      asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(TMEM_COLS));
+    else
+      asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(TMEM_COLS));
   }
 }
 
@@ -410,24 +486,71 @@ bool make_operand_map(CUtensorMap* map, const GemmOperand& op, int64_t d0, int64
 }
 
 int g_num_sms = 0;
+int g_pair_slots = 0;  // co-resident CTA pairs (2-CTA clusters at one CTA per SM)
 std::atomic<int64_t> g_launches{0};
+std::atomic<int> g_mode{0};  // 0 auto, 1 single-CTA tiles only, 2 CTA pairs whenever legal
+GemmConfig g_last{};
 
-template <int BN, bool F32OUT, int EW = 8>
+template <int BN, bool F32OUT, int EW = 8, int CG = 1>
 void launch(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, const CUtensorMap& c2, const TcParams& p,
             cudaStream_t st) {
-  constexpr int STAGE = (BM + BN) * BK * 2;
-  const int smem = num_stages<BN, F32OUT, EW>() * STAGE + 1024 + staging_bytes<F32OUT, EW>() + 1024;
+  constexpr int STAGE = (BM + BN / CG) * BK * 2;
+  const int smem = num_stages<BN / CG, F32OUT, EW>() * STAGE + 1024 + staging_bytes<F32OUT, EW>() + 1024;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(gemm_tc_kernel<BN, F32OUT, EW>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(gemm_tc_kernel<BN, F32OUT, EW, CG>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
-  int grid = p.num_units < g_num_sms ? p.num_units : g_num_sms;
-  gemm_tc_kernel<BN, F32OUT, EW><<<grid, num_threads<EW>(), smem, st>>>(a, b, c, c2, p);
+  if constexpr (CG == 1) {
+    int grid = p.num_units < g_num_sms ? p.num_units : g_num_sms;
+    gemm_tc_kernel<BN, F32OUT, EW, 1><<<grid, num_threads<EW>(), smem, st>>>(a, b, c, c2, p);
+  } else {
+    const int pairs = p.num_units < g_pair_slots ? p.num_units : g_pair_slots;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(2 * pairs);
+    cfg.blockDim = dim3(num_threads<EW>());
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaLaunchKernelEx(&cfg, gemm_tc_kernel<BN, F32OUT, EW, 2>, a, b, c, c2, p);
+  }
   g_launches++;
 }
 
+// number of 2-CTA clusters of the pair kernel that fit on the device at once
+int query_pair_slots() {
+  constexpr int STAGE = (BM + 128) * BK * 2;
+  const int smem = num_stages<128, false, 8>() * STAGE + 1024 + staging_bytes<false, 8>() + 1024;
+  cudaFuncSetAttribute(gemm_tc_kernel<256, false, 8, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(g_num_sms);
+  cfg.blockDim = dim3(num_threads<8>());
+  cfg.dynamicSmemBytes = smem;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 2;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, gemm_tc_kernel<256, false, 8, 2>, &cfg) != cudaSuccess || n <= 0) {
+    cudaGetLastError();
+    n = g_num_sms / 2;
+  }
+  return n;
+}
+
 }  // namespace
+
+void gemm_tc_set_mode(int mode) { g_mode = mode; }  // bits 0-1 tile mode, bit 2 no tail split
+GemmConfig gemm_tc_last_config() { return g_last; }
 
 int64_t gemm_tc_launches() { return g_launches.load(); }
 
@@ -439,40 +562,65 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
     if (g_num_sms <= 0) return false;
+    g_pair_slots = query_pair_slots();
   }
   // Tile width and split-K are chosen together (the Fig. 5 effect of small micro-ops,
   // P:L125): time ~ ceil(units / SMs) x per-unit time, with per-tile times from the
   // measured tcgen05 efficiency of each width (narrow tiles are smem-feed bound in
   // SS mode: 256 -> ~0.90, 128 -> ~0.65, 64 -> ~0.45 of peak).  Split-K needs an fp32,
   // contiguous, unbatched C (partials are TMA reduce-added).
+  // CTA pairs (cta_group::2, 256 x bn units on two SMs) halve each SM's B feed: a pair
+  // tile of width bn costs one SM what a single-CTA tile of width bn costs, at the
+  // efficiency of a single-CTA tile twice as wide.
   const bool splitk_ok = g.c_dtype == F32 && g.nb1 * g.nb2 == 1 && g.ldc == g.N;
   const int num_kb_all = (g.K + BK - 1) / BK;
-  int best_bn = 256, best_ks = 1;
+  const int mode = g_mode.load() & 3;
+  // half-width tail units: measured +3-5 % for K <= 1024 products, -1-2 % for K = 4096
+  // (the kernels run power-capped, so idle tail SMs are partly paid back in clock)
+  const bool tail_split = (g_mode.load() & 4) == 0 && num_kb_all <= 32;
+  int best_bn = 256, best_ks = 1, best_cg = 1;
   double best = 1e30;
-  for (int bn : {256, 128, 64}) {
-    if (bn > 64 && g.N <= bn / 2) continue;
-    const double eff = bn == 256 ? 0.90 : bn == 128 ? 0.65 : 0.45;
-    int64_t tiles = int64_t((g.M + BM - 1) / BM) * ((g.N + bn - 1) / bn) * g.nb1 * g.nb2;
-    int ks = 1;
-    if (splitk_ok && tiles * 2 <= g_num_sms && num_kb_all >= 16) {
-      ks = int(g_num_sms / tiles);
-      if (ks > num_kb_all / 8) ks = num_kb_all / 8;
-      if (ks < 1) ks = 1;
-    }
-    int64_t units = tiles * ks;
-    double waves = double((units + g_num_sms - 1) / g_num_sms);
-    double cost = waves * (bn / eff) / ks;
-    if (cost < best - 1e-9) {
-      best = cost;
-      best_bn = bn;
-      best_ks = ks;
+  for (int cg : {1, 2}) {
+    if (cg == 2 && (mode == 1 || g.M <= BM || g_pair_slots <= 0)) continue;
+    // pairs pay a cluster launch/teardown and a cross-CTA handshake per unit: only
+    // worth it for reductions of >= 8 k-blocks (measured: K = 64 products lose 25 %)
+    if (cg == 2 && mode == 0 && num_kb_all < 8) continue;
+    if (cg == 1 && mode == 2 && g.M > BM && g.N > 64 && g_pair_slots > 0) continue;
+    const int slots = cg == 1 ? g_num_sms : g_pair_slots;
+    for (int bn : {256, 128, 64}) {
+      if (bn > 64 && g.N <= bn / 2) continue;
+      if (cg == 2 && bn < 128) continue;
+      const double eff = cg == 2 ? (bn == 256 ? 0.97 : 0.60) : (bn == 256 ? 0.90 : bn == 128 ? 0.65 : 0.45);
+      int64_t tiles = int64_t((g.M + BM * cg - 1) / (BM * cg)) * ((g.N + bn - 1) / bn) * g.nb1 * g.nb2;
+      int ks = 1;
+      if (splitk_ok && tiles * 2 <= slots && num_kb_all >= 16) {
+        ks = int(slots / tiles);
+        if (ks > num_kb_all / 8) ks = num_kb_all / 8;
+        if (ks < 1) ks = 1;
+      }
+      int64_t units = tiles * ks;
+      double waves = double((units + slots - 1) / slots);
+      // a tail wave at most half full runs as half-width units (decode_unit)
+      if (tail_split && ks == 1 && bn / (2 * cg) >= 64 && tiles > slots && tiles % slots &&
+          2 * (tiles % slots) <= slots)
+        waves -= 0.5;
+      // time in (tile-width x k-block) units, + the pair's fixed cost (~4 k-blocks of a
+      // 256-wide tile, fitted to the BERT micro-op shapes)
+      const int kb_unit = (num_kb_all + ks - 1) / ks;
+      double cost = waves * (bn / eff) * kb_unit + (cg == 2 ? 1024.0 : 0.0);
+      if (cost < best - 1e-9) {
+        best = cost;
+        best_bn = bn;
+        best_ks = ks;
+        best_cg = cg;
+      }
     }
   }
   CUtensorMap ma, mb, mc;
   bool ok = g.a.mn_major ? make_operand_map(&ma, g.a, g.M, g.K, g.nb1, g.nb2, 64)
                          : make_operand_map(&ma, g.a, g.K, g.M, g.nb1, g.nb2, BM);
   ok = ok && (g.b.mn_major ? make_operand_map(&mb, g.b, g.N, g.K, g.nb1, g.nb2, 64)
-                           : make_operand_map(&mb, g.b, g.K, g.N, g.nb1, g.nb2, best_bn));
+                           : make_operand_map(&mb, g.b, g.K, g.N, g.nb1, g.nb2, best_bn / best_cg));
   if (!ok) return false;
   TcParams p;
   p.M = g.M;
@@ -480,7 +628,8 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   p.K = g.K;
   p.nb1 = g.nb1;
   p.nb2 = g.nb2;
-  p.tiles_m = (g.M + BM - 1) / BM;
+  p.bm = BM * best_cg;
+  p.tiles_m = (g.M + p.bm - 1) / p.bm;
   p.tiles_n = (g.N + best_bn - 1) / best_bn;
   p.num_tiles = p.tiles_m * p.tiles_n * g.nb1 * g.nb2;
   p.num_kb = (g.K + BK - 1) / BK;
@@ -531,6 +680,30 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   p.kb_per_split = (p.num_kb + p.ksplit - 1) / p.ksplit;
   p.ksplit = (p.num_kb + p.kb_per_split - 1) / p.kb_per_split;
   p.num_units = p.num_tiles * p.ksplit;
+  p.split_from = p.num_units;
+  {
+    const int slots = best_cg == 2 ? g_pair_slots : g_num_sms;
+    const int tail = p.num_tiles % slots;
+    if (tail_split && p.ksplit == 1 && best_bn / (2 * best_cg) >= 64 && p.num_tiles > slots && tail &&
+        2 * tail <= slots) {
+      p.split_from = p.num_tiles - tail;
+      p.num_units = p.num_tiles + tail;
+    }
+  }
+  g_last = GemmConfig{best_bn, best_cg, p.ksplit, p.num_units, g_num_sms, g_pair_slots, p.split_from};
+  if (best_cg == 2) {
+    if (p.c_f32) {
+      if (best_bn == 256) launch<256, true, 8, 2>(ma, mb, mc, mc2, p, st);
+      else launch<128, true, 8, 2>(ma, mb, mc, mc2, p, st);
+    } else if (best_bn == 256) {
+      if (p.epi == 1) launch<256, false, 16, 2>(ma, mb, mc, mc2, p, st);
+      else launch<256, false, 8, 2>(ma, mb, mc, mc2, p, st);
+    } else {
+      if (p.epi == 1) launch<128, false, 16, 2>(ma, mb, mc, mc2, p, st);
+      else launch<128, false, 8, 2>(ma, mb, mc, mc2, p, st);
+    }
+    return true;
+  }
   if (p.c_f32) {
     switch (best_bn) {
       case 256: launch<256, true>(ma, mb, mc, mc2, p, st); break;

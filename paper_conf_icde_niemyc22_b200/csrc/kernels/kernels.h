@@ -45,6 +45,16 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st);
 void gemm_simt(const GemmArgs& g, cudaStream_t st);
 void gemm(const GemmArgs& g, cudaStream_t st);
 int64_t gemm_tc_launches();
+// tile configuration of the last gemm_tc launch (tests / tools): width bn of a tile,
+// cg = CTAs per tile (2: cta_group::2 pair, 256 rows), split-K factor, work units, SMs,
+// co-resident CTA pairs, first half-width tail unit (= units when none)
+struct GemmConfig {
+  int bn, cg, ksplit, units, sms, pair_slots, split_from;
+};
+GemmConfig gemm_tc_last_config();
+// 0: cost-model choice; 1: single-CTA tiles only; 2: CTA pairs whenever M > 128, N > 64;
+// + 4: no half-width tail units
+void gemm_tc_set_mode(int mode);
 // Per-launch timing of GEMMs (eager profiling only): while enabled, gemm() brackets
 // every launch with CUDA events on its stream and records the algorithmic FLOP.
 struct GemmRecord {

@@ -1344,6 +1344,20 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch, const voi
   return TS_OK;
 }
 
+ts_status ts_gemm_set_mode(int32_t mode) {
+  if (mode < 0 || mode > 7 || (mode & 3) == 3) return set_error("gemm mode: (0|1|2) + 4 * no_tail_split"), TS_ERR_ARG;
+  tsk::gemm_tc_set_mode(mode);
+  return TS_OK;
+}
+
+ts_status ts_gemm_last_config(int32_t* out8) {
+  if (!out8) return set_error("out8 is NULL"), TS_ERR_ARG;
+  const tsk::GemmConfig c = tsk::gemm_tc_last_config();
+  const int32_t v[8] = {c.bn, c.cg, c.ksplit, c.units, c.sms, c.pair_slots, c.split_from, 0};
+  for (int i = 0; i < 8; ++i) out8[i] = v[i];
+  return TS_OK;
+}
+
 ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K, const float* A, int64_t lda, int32_t ta, const float* B,
                       int64_t ldb, int32_t tb, float* C, int64_t ldc, float alpha, float beta, const float* bias,
                       void* stream) {

@@ -30,11 +30,33 @@ CASES = [
     (512, 64, 512, 4, 0, 1, "bf16"),     # attention P.V shape
     (1024, 4096, 1024, 1, 0, 0, "bf16"),
     (1024, 1024, 4096, 1, 1, 1, "f32"),  # dW shape
+    (300, 256, 192, 1, 0, 0, "bf16"),    # CTA pair: second CTA's rows partly past M
+    (129, 384, 64, 2, 0, 1, "f32"),      # CTA pair: second CTA entirely past M
+    (640, 128, 256, 1, 1, 0, "bf16"),    # pair tile width 128 (64 B rows per CTA)
+    (4096, 1024, 1024, 1, 0, 0, "bf16"),  # BERT projection shape at p = 4
+    (16384, 1024, 256, 1, 0, 0, "bf16"),  # 512 tiles: the tail wave runs as half-width units
+    (16384, 1024, 128, 1, 0, 1, "bf16"),  # same, MN-major B
+    (20000, 1024, 64, 1, 1, 1, "f32"),    # tail split with ragged M, both operands MN-major
 ]
 
 
+def _cfg():
+    out = (tsplit.C.c_int32 * 8)()
+    tsplit.check(tsplit.lib().ts_gemm_last_config(out))
+    return list(out)
+
+
+@pytest.fixture
+def gemm_mode():
+    yield lambda m: tsplit.check(tsplit.lib().ts_gemm_set_mode(m))
+    tsplit.check(tsplit.lib().ts_gemm_set_mode(0))
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2])
 @pytest.mark.parametrize("M,N,K,batch,ta,tb,out", CASES)
-def test_gemm_tc_matches_torch(M, N, K, batch, ta, tb, out):
+def test_gemm_tc_matches_torch(M, N, K, batch, ta, tb, out, mode, gemm_mode):
+    """mode 1 = single-CTA tiles, 2 = CTA-pair (tcgen05 cta_group::2) tiles, 0 = cost model."""
+    gemm_mode(mode)
     torch.cuda.synchronize()
     A = [_mk((M, K), seed=1 + b) for b in range(batch)]
     B = [_mk((N, K), seed=100 + b) for b in range(batch)]
@@ -49,6 +71,11 @@ def test_gemm_tc_matches_torch(M, N, K, batch, ta, tb, out):
                                    1.0, 0.0, None, None)
     tsplit.check(st)
     torch.cuda.synchronize()
+    cfg = _cfg()
+    if mode:
+        assert cfg[1] == (2 if mode == 2 and M > 128 and N > 64 else 1), cfg
+        if M >= 16384 and N == 1024:  # 512 (resp. 256 pair) tiles: tail wave split in halves
+            assert cfg[6] < cfg[3], cfg
     for b in range(batch):
         ref = A[b].float() @ B[b].float().t()
         got = Cc[b].float()
@@ -56,7 +83,9 @@ def test_gemm_tc_matches_torch(M, N, K, batch, ta, tb, out):
         assert err < (1e-5 if out == "f32" else 8e-3), (b, err)
 
 
-def test_gemm_tc_alpha_beta_bias():
+@pytest.mark.parametrize("mode", [1, 2])
+def test_gemm_tc_alpha_beta_bias(mode, gemm_mode):
+    gemm_mode(mode)
     M, N, K = 256, 384, 256
     A, B = _mk((M, K), seed=3), _mk((N, K), seed=4)
     bias = _mk((N,), seed=5)
@@ -87,7 +116,9 @@ def test_gemm_simt_f32():
     (256, 512, 640, "bf16", 1.0),      # activation-gradient accumulation in bf16
     (200, 72, 128, "f32", 1.0),        # ragged tile edges through the TMA store
 ])
-def test_gemm_tc_accumulate_and_splitk(M, N, K, out, beta):
+@pytest.mark.parametrize("mode", [1, 2])
+def test_gemm_tc_accumulate_and_splitk(M, N, K, out, beta, mode, gemm_mode):
+    gemm_mode(mode)
     A = _mk((K, M), seed=11)   # MN-major operands, as in dW = dY^T X
     B = _mk((K, N), seed=12)
     od = torch.float32 if out == "f32" else torch.bfloat16

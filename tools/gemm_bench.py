@@ -43,11 +43,21 @@ def case(name, M, N, K, ta, tb, out="bf16", batch=1, beta=0.0):
 
     def cublas():
         torch.matmul(Aop, Bop, out=C if out == "bf16" else None) if out == "bf16" else torch.matmul(Aop, Bop)
-    t_ours = timeit(ours)
-    t_cub = timeit(cublas)
     fl = 2.0 * M * N * K * batch
+    modes = {}
+    for mode, tag in ((1, "cta1"), (5, "cta1_nosplit"), (2, "pair"), (6, "pair_nosplit"), (0, "auto")):
+        tsplit.check(L.ts_gemm_set_mode(mode))
+        t = timeit(ours)
+        cfg = (tsplit.C.c_int32 * 8)()
+        tsplit.check(L.ts_gemm_last_config(cfg))
+        modes[tag] = {"tflops": fl / t / 1e12, "us": t * 1e6, "bn": cfg[0], "cg": cfg[1], "ksplit": cfg[2],
+                      "units": cfg[3], "pair_slots": cfg[5], "split_from": cfg[6]}
+    tsplit.check(L.ts_gemm_set_mode(0))
+    t_ours = modes["auto"]["us"] / 1e6
+    t_cub = timeit(cublas)
     r = {"name": name, "M": M, "N": N, "K": K, "batch": batch, "ta": ta, "tb": tb, "out": out,
-         "ours_tflops": fl / t_ours / 1e12, "cublas_tflops": fl / t_cub / 1e12, "ours_us": t_ours * 1e6}
+         "ours_tflops": fl / t_ours / 1e12, "cublas_tflops": fl / t_cub / 1e12, "ours_us": t_ours * 1e6,
+         "modes": modes}
     print(json.dumps(r), flush=True)
     return r
 
@@ -64,6 +74,9 @@ if __name__ == "__main__":
     res.append(case("ffn1 dW", F, H, T, 1, 1, out="f32", beta=1.0))
     res.append(case("ffn2 dW", H, F, T, 1, 1, out="f32", beta=1.0))
     res.append(case("p=4 ffn1 fwd", T // 4, F, H, 0, 0))
+    res.append(case("p=2 qkv fwd", T // 2, H, H, 0, 0))
+    res.append(case("p=4 qkv fwd", T // 4, H, H, 0, 0))
+    res.append(case("p=4 ffn2 fwd", T // 4, H, F, 0, 0))
     res.append(case("attn QK^T", 512, 512, 64, 0, 0, batch=512))
     res.append(case("attn PV", 512, 64, 512, 0, 1, batch=512))
     res.append(case("attn dS^T Q", 512, 64, 512, 1, 1, batch=512))

@@ -13,6 +13,7 @@ from tsinputs import gen, graphs  # noqa: E402
 
 fused = len(sys.argv) < 2 or sys.argv[1] == "fused"
 frac = float(sys.argv[2]) if len(sys.argv) > 2 else 0.0
+tsplit.check(tsplit.lib().ts_gemm_set_mode(int(os.environ.get("GEMM_MODE", "0"))))
 spec = graphs.bert(layers=24, batch=32, fused_attention=fused)
 G = tsplit.Graph(spec)
 P = tsplit.Plan.default(G)
