@@ -302,6 +302,20 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch,
                        const void* B, int64_t ldb, int64_t strideB, int32_t tb,
                        void* C, int64_t ldc, int64_t strideC, int32_t c_dtype,
                        float alpha, float beta, const void* bias_bf16, void* stream);
+/* Grouped product on the tcgen05 path (the session's q/k/v horizontal fusion), bf16
+ * operands, device pointers, arrays of `groups` (<= 3) host-side pointers.  M, N, K
+ * are TOTAL extents; a group spans 1/groups of the gdim extent:
+ *   gdim 1 (N): C[g] = alpha A[0] op(B[g]) + bias[g] (+ beta C[g]), C[g] is M x N/groups
+ *   gdim 2 (K): C[0] = alpha sum_g A[g] op(B[g]) + bias[0] (+ beta C[0]), A[g]: M x K/groups
+ *   gdim 3 (M): C[g] = alpha A[g] op(B[0]) + bias[0] (+ beta C[g]), A[g]: M/groups x K
+ * lda/ldb/ldc/ta/tb/c_dtype as in ts_gemm_bf16 (shared by all groups); beta 0 or 1;
+ * bias may be NULL.  TS_ERR_ARG when no tcgen05 tiling fits (the tile must not straddle
+ * groups: N/groups a multiple of 64, M/groups of 128, K/groups of 64). */
+ts_status ts_gemm_bf16_grouped(int32_t groups, int32_t gdim, int32_t M, int32_t N, int32_t K,
+                               const void* const* A, int64_t lda, int32_t ta,
+                               const void* const* B, int64_t ldb, int32_t tb,
+                               void* const* C, int64_t ldc, int32_t c_dtype, float alpha, float beta,
+                               const void* const* bias, void* stream);
 /* Tile-selection override for the tcgen05 GEMM (tests and microbenchmarks; process-
  * wide, not thread-safe against concurrent launches): mode 0 = cost model (default),
  * 1 = single-CTA 128-row tiles only, 2 = CTA-pair (cta_group::2, 256-row) tiles

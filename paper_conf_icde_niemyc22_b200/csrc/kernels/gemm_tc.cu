@@ -13,6 +13,7 @@
 #include <cudaTypedefs.h>
 
 #include <atomic>
+#include <cstring>
 #include <cstdio>
 #include <mutex>
 
@@ -51,6 +52,15 @@ struct TcParams {
   int epi;         // GemmArgs::epi (bf16 TMA-store path only): 1 GELU fwd (2nd output via tmC2), 2 GELU bwd
   const bf16* aux; // epi 2: U, row-major with leading dimension ldaux
   int64_t ldaux;
+  // grouped product (GemmArgs::groups): gdim 1 = N groups (B, C, bias per group), 2 = K
+  // groups (A, B per group, summed), 3 = M groups (A, C per group); gsize = extent of
+  // one group along gdim (a multiple of the tile along it)
+  int gdim, gsize;
+  const void* bias_g[kMaxGroups];
+};
+// operand / output tensor maps (one per group; a plain product uses index 0)
+struct TmSet {
+  CUtensorMap a[kMaxGroups], b[kMaxGroups], c[kMaxGroups], c2;
 };
 // epilogue staging: per warp, 32x32 output blocks (two for bf16; one for fp32, whose
 // products have long K and keep the smem for a deeper operand pipeline)
@@ -111,9 +121,7 @@ __device__ __forceinline__ void decode_tile(const TcParams& p, int tile, int& b1
 // (128 lanes x BN columns) and arrives on the leader's tempty barrier.
 template <int BN, bool F32OUT, int EW, int CG>
 __global__ void __launch_bounds__(num_threads<EW>(), 1)
-    gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                   const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmC2,
-                   const TcParams p) {
+    gemm_tc_kernel(const __grid_constant__ TmSet tm, const TcParams p) {
   constexpr int BNL = BN / CG;  // B rows staged by this CTA
   constexpr int A_BYTES = BM * BK * 2;
   constexpr int B_BYTES = BNL * BK * 2;
@@ -149,8 +157,8 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
       mbar_init(&tempty[s], EW * CG);  // one arrive per epilogue warp of each CTA
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmA)) : "memory");
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tmB)) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tm.a[0])) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&tm.b[0])) : "memory");
   }
   if (warp == 1) {
     if constexpr (CG == 1) {
@@ -182,43 +190,58 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
         m0 += int(rank) * BM;
         // a half-width unit stages B rows [n0 + hsel BN/2 + rank BN/(2 CG), +BNL) (the box
         // is fixed; the MMA reads only the first BN/(2 CG) rows of each CTA's half)
-        const int n0 = nt * BN + (hsel < 0 ? int(rank) * BNL : hsel * (BN / 2) + int(rank) * (BNL / 2));
+        int n0 = nt * BN + (hsel < 0 ? int(rank) * BNL : hsel * (BN / 2) + int(rank) * (BNL / 2));
+        // groups: the tile's group and its coordinates inside that group's maps
+        int ga = 0, gb = 0;
+        if (p.gdim == 1) {
+          gb = (nt * BN) / p.gsize;
+          n0 -= gb * p.gsize;
+        } else if (p.gdim == 3) {
+          ga = (m0 - int(rank) * BM) / p.gsize;
+          m0 -= ga * p.gsize;
+        }
         const int kb0 = ks * p.kb_per_split;
         const int kb1 = min(p.num_kb, kb0 + p.kb_per_split);
         for (int kb = kb0; kb < kb1; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           uint8_t* sa = smem + stage * STAGE;
           uint8_t* sb = sa + A_BYTES;
-          const int k0 = kb * BK;
+          int k0 = kb * BK;
+          if (p.gdim == 2) {
+            ga = gb = k0 / p.gsize;
+            k0 -= ga * p.gsize;
+          }
+          const CUtensorMap* tmA = &tm.a[ga];
+          const CUtensorMap* tmB = &tm.b[gb];
           if constexpr (CG == 1) {
             mbar_arrive_tx(&full[stage], STAGE);
             if (!p.a_mn) {
-              tma_load(sa, &tmA, &full[stage], k0, m0, b1, b2);
+              tma_load(sa, tmA, &full[stage], k0, m0, b1, b2);
             } else {
 #pragma unroll
-              for (int i = 0; i < BM / 64; ++i) tma_load(sa + i * 8192, &tmA, &full[stage], m0 + 64 * i, k0, b1, b2);
+              for (int i = 0; i < BM / 64; ++i) tma_load(sa + i * 8192, tmA, &full[stage], m0 + 64 * i, k0, b1, b2);
             }
             if (!p.b_mn) {
-              tma_load(sb, &tmB, &full[stage], k0, n0, b1, b2);
+              tma_load(sb, tmB, &full[stage], k0, n0, b1, b2);
             } else {
 #pragma unroll
-              for (int i = 0; i < BNL / 64; ++i) tma_load(sb + i * 8192, &tmB, &full[stage], n0 + 64 * i, k0, b1, b2);
+              for (int i = 0; i < BNL / 64; ++i) tma_load(sb + i * 8192, tmB, &full[stage], n0 + 64 * i, k0, b1, b2);
             }
           } else {
             // both CTAs' bytes complete on the leader's barrier; only the leader arrives
             if (rank == 0) mbar_arrive_tx(&full[stage], 2 * STAGE);
             const uint32_t fb = mapa_shared(smem_u32(&full[stage]), 0);
             if (!p.a_mn) {
-              tma_load_2sm(sa, &tmA, fb, k0, m0, b1, b2);
+              tma_load_2sm(sa, tmA, fb, k0, m0, b1, b2);
             } else {
 #pragma unroll
-              for (int i = 0; i < BM / 64; ++i) tma_load_2sm(sa + i * 8192, &tmA, fb, m0 + 64 * i, k0, b1, b2);
+              for (int i = 0; i < BM / 64; ++i) tma_load_2sm(sa + i * 8192, tmA, fb, m0 + 64 * i, k0, b1, b2);
             }
             if (!p.b_mn) {
-              tma_load_2sm(sb, &tmB, fb, k0, n0, b1, b2);
+              tma_load_2sm(sb, tmB, fb, k0, n0, b1, b2);
             } else {
 #pragma unroll
-              for (int i = 0; i < BNL / 64; ++i) tma_load_2sm(sb + i * 8192, &tmB, fb, n0 + 64 * i, k0, b1, b2);
+              for (int i = 0; i < BNL / 64; ++i) tma_load_2sm(sb + i * 8192, tmB, fb, n0 + 64 * i, k0, b1, b2);
             }
           }
           if (++stage == STAGES) {
@@ -297,6 +320,17 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
       m0 += int(rank) * BM;
       const int n0 = nt * BN + (hsel < 0 ? 0 : hsel * (BN / 2));
       const int nchunks = (hsel < 0 ? BN : BN / 2) / 32;
+      // output group and the tile's coordinates in that group's C map / bias
+      int gc = 0, cn0 = n0, cm0 = m0;
+      if (p.gdim == 1) {
+        gc = (nt * BN) / p.gsize;
+        cn0 = n0 - gc * p.gsize;
+      } else if (p.gdim == 3) {
+        gc = (m0 - int(rank) * BM) / p.gsize;
+        cm0 = m0 - gc * p.gsize;
+      }
+      const void* bias = p.gdim == 1 ? p.bias_g[gc] : p.bias;
+      const CUtensorMap* tmC = &tm.c[gc];
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const int row = m0 + q * 32 + lane;
@@ -307,15 +341,16 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
         uint32_t r[32];
         tmem_ld32(tmem_base + (uint32_t(q * 32) << 16) + uint32_t(acc * BN + c * 32), r);
         const int col0 = n0 + c * 32;
+        const int ccol = cn0 + c * 32;  // column in the group's C map / bias
         if (col0 < p.N) {
           float v[32];
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]) * p.alpha;
           const bool full_chunk = col0 + 32 <= p.N;
-          if (p.bias) {
-            if (full_chunk && !p.bias_f32 && (reinterpret_cast<uintptr_t>(p.bias) & 15) == 0) {
+          if (bias) {
+            if (full_chunk && !p.bias_f32 && (reinterpret_cast<uintptr_t>(bias) & 15) == 0) {
               // 32 bias values as four 16-byte loads (the same address across the warp: one broadcast each)
-              const uint4* bp = reinterpret_cast<const uint4*>(reinterpret_cast<const bf16*>(p.bias) + col0);
+              const uint4* bp = reinterpret_cast<const uint4*>(reinterpret_cast<const bf16*>(bias) + ccol);
 #pragma unroll
               for (int j = 0; j < 4; ++j) {
                 const uint4 u = __ldg(bp + j);
@@ -331,8 +366,8 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
 #pragma unroll
               for (int i = 0; i < 32; ++i)
                 if (full_chunk || col0 + i < p.N)
-                  v[i] += p.bias_f32 ? reinterpret_cast<const float*>(p.bias)[col0 + i]
-                                     : to_f(reinterpret_cast<const bf16*>(p.bias)[col0 + i]);
+                  v[i] += p.bias_f32 ? reinterpret_cast<const float*>(bias)[ccol + i]
+                                     : to_f(reinterpret_cast<const bf16*>(bias)[ccol + i]);
             }
           }
           if (p.tma_store) {
@@ -387,18 +422,18 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
               fence_async_smem();
               __syncwarp();
               if (lane == 0) {
-                if (radd) tma_reduce_add(map, buf, col0, m0 + q * 32, b1, b2);
-                else tma_store(map, buf, col0, m0 + q * 32, b1, b2);
+                if (radd) tma_reduce_add(map, buf, ccol, cm0 + q * 32, b1, b2);
+                else tma_store(map, buf, ccol, cm0 + q * 32, b1, b2);
                 bulk_commit();
               }
               nbuf = (nbuf + 1) % NBUF;
             };
-            stage_store(v, &tmC, p.reduce_add);
+            stage_store(v, tmC, p.reduce_add);
             if constexpr (!F32OUT) {
               if (p.epi == 1) {  // second output: gelu of the stored (bf16) U
 #pragma unroll
                 for (int i = 0; i < 32; ++i) v[i] = gelu_f(bf16_round(v[i]));
-                stage_store(v, &tmC2, false);
+                stage_store(v, &tm.c2, false);
               }
             }
           } else if (row_ok) {
@@ -492,8 +527,7 @@ std::atomic<int> g_mode{0};  // 0 auto, 1 single-CTA tiles only, 2 CTA pairs whe
 GemmConfig g_last{};
 
 template <int BN, bool F32OUT, int EW = 8, int CG = 1>
-void launch(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, const CUtensorMap& c2, const TcParams& p,
-            cudaStream_t st) {
+void launch(const TmSet& tm, const TcParams& p, cudaStream_t st) {
   constexpr int STAGE = (BM + BN / CG) * BK * 2;
   const int smem = num_stages<BN / CG, F32OUT, EW>() * STAGE + 1024 + staging_bytes<F32OUT, EW>() + 1024;
   static bool attr = false;
@@ -503,7 +537,7 @@ void launch(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, co
   }
   if constexpr (CG == 1) {
     int grid = p.num_units < g_num_sms ? p.num_units : g_num_sms;
-    gemm_tc_kernel<BN, F32OUT, EW, 1><<<grid, num_threads<EW>(), smem, st>>>(a, b, c, c2, p);
+    gemm_tc_kernel<BN, F32OUT, EW, 1><<<grid, num_threads<EW>(), smem, st>>>(tm, p);
   } else {
     const int pairs = p.num_units < g_pair_slots ? p.num_units : g_pair_slots;
     cudaLaunchConfig_t cfg = {};
@@ -518,7 +552,7 @@ void launch(const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& c, co
     at[0].val.clusterDim.z = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    cudaLaunchKernelEx(&cfg, gemm_tc_kernel<BN, F32OUT, EW, 2>, a, b, c, c2, p);
+    cudaLaunchKernelEx(&cfg, gemm_tc_kernel<BN, F32OUT, EW, 2>, tm, p);
   }
   g_launches++;
 }
@@ -572,6 +606,17 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   // CTA pairs (cta_group::2, 256 x bn units on two SMs) halve each SM's B feed: a pair
   // tile of width bn costs one SM what a single-CTA tile of width bn costs, at the
   // efficiency of a single-CTA tile twice as wide.
+  // grouped products (horizontal fusion of micro-ops sharing an operand, see GemmArgs)
+  const int G = g.groups > 1 ? g.groups : 1;
+  int gsize = 0;
+  if (G > 1) {
+    if (G > kMaxGroups || g.gdim < 1 || g.gdim > 3 || g.nb1 * g.nb2 != 1 || g.epi) return false;
+    if (g.beta != 0.f && g.beta != 1.f) return false;
+    const int ext = g.gdim == 1 ? g.N : g.gdim == 2 ? g.K : g.M;
+    if (ext % G) return false;
+    gsize = ext / G;
+    if (g.gdim == 2 && gsize % BK) return false;
+  }
   const bool splitk_ok = g.c_dtype == F32 && g.nb1 * g.nb2 == 1 && g.ldc == g.N;
   const int num_kb_all = (g.K + BK - 1) / BK;
   const int mode = g_mode.load() & 3;
@@ -587,8 +632,10 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
     if (cg == 2 && mode == 0 && num_kb_all < 8) continue;
     if (cg == 1 && mode == 2 && g.M > BM && g.N > 64 && g_pair_slots > 0) continue;
     const int slots = cg == 1 ? g_num_sms : g_pair_slots;
+    if (G > 1 && g.gdim == 3 && gsize % (BM * cg)) continue;  // a tile never straddles M groups
     for (int bn : {256, 128, 64}) {
       if (bn > 64 && g.N <= bn / 2) continue;
+      if (G > 1 && g.gdim == 1 && gsize % bn) continue;  // ... nor N groups
       if (cg == 2 && bn < 128) continue;
       const double eff = cg == 2 ? (bn == 256 ? 0.97 : 0.60) : (bn == 256 ? 0.90 : bn == 128 ? 0.65 : 0.45);
       int64_t tiles = int64_t((g.M + BM * cg - 1) / (BM * cg)) * ((g.N + bn - 1) / bn) * g.nb1 * g.nb2;
@@ -616,13 +663,28 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
       }
     }
   }
-  CUtensorMap ma, mb, mc;
-  bool ok = g.a.mn_major ? make_operand_map(&ma, g.a, g.M, g.K, g.nb1, g.nb2, 64)
-                         : make_operand_map(&ma, g.a, g.K, g.M, g.nb1, g.nb2, BM);
-  ok = ok && (g.b.mn_major ? make_operand_map(&mb, g.b, g.N, g.K, g.nb1, g.nb2, 64)
-                           : make_operand_map(&mb, g.b, g.K, g.N, g.nb1, g.nb2, best_bn / best_cg));
+  if (best > 1e29) return false;  // no legal tiling (grouped products)
+  // one A / B / C map per group over that group's extents (a plain product: index 0)
+  TmSet tm;
+  std::memset(&tm, 0, sizeof(tm));
+  const int Ma = g.gdim == 3 && G > 1 ? gsize : g.M;
+  const int Nb = g.gdim == 1 && G > 1 ? gsize : g.N;
+  const int Kg = g.gdim == 2 && G > 1 ? gsize : g.K;
+  bool ok = true;
+  for (int i = 0; i < G && ok; ++i) {
+    const GemmOperand& A = (G > 1 && g.gdim != 1) ? g.ag[i] : g.a;
+    const GemmOperand& Bo = (G > 1 && g.gdim != 3) ? g.bg[i] : g.b;
+    if (A.mn_major != g.a.mn_major || Bo.mn_major != g.b.mn_major) return false;
+    ok = A.mn_major ? make_operand_map(&tm.a[i], A, Ma, Kg, g.nb1, g.nb2, 64)
+                    : make_operand_map(&tm.a[i], A, Kg, Ma, g.nb1, g.nb2, BM);
+    ok = ok && (Bo.mn_major ? make_operand_map(&tm.b[i], Bo, Nb, Kg, g.nb1, g.nb2, 64)
+                            : make_operand_map(&tm.b[i], Bo, Kg, Nb, g.nb1, g.nb2, best_bn / best_cg));
+  }
   if (!ok) return false;
   TcParams p;
+  p.gdim = G > 1 ? g.gdim : 0;
+  p.gsize = gsize;
+  for (int i = 0; i < kMaxGroups; ++i) p.bias_g[i] = (G > 1 && g.gdim == 1 && i < G) ? g.biasg[i] : g.bias;
   p.M = g.M;
   p.N = g.N;
   p.K = g.K;
@@ -647,20 +709,27 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   p.bias_f32 = g.bias_dtype == F32;
   // output: TMA store (bf16/f32) or TMA reduce-add (f32, beta == 1) when the view is aligned
   const int es = p.c_f32 ? 4 : 2;
-  p.tma_store = make_map(&mc, g.c, g.ldc, g.cbs1, g.cbs2, g.N, g.M, g.nb1, g.nb2, 32, 32, es,
-                         p.c_f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16,
-                         p.c_f32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B)
-                    ? 1 : 0;
+  const int Nc = g.gdim == 1 && G > 1 ? gsize : g.N;
+  const int Mc = g.gdim == 3 && G > 1 ? gsize : g.M;
+  const int GC = (G > 1 && g.gdim != 2) ? G : 1;
+  p.tma_store = 1;
+  for (int i = 0; i < GC; ++i) {
+    void* C = (G > 1 && g.gdim != 2) ? g.cg[i] : g.c;
+    if (!make_map(&tm.c[i], C, g.ldc, g.cbs1, g.cbs2, Nc, Mc, g.nb1, g.nb2, 32, 32, es,
+                  p.c_f32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16,
+                  p.c_f32 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B))
+      p.tma_store = 0;
+  }
   if (g.beta != 0.f && g.beta != 1.f) p.tma_store = 0;
-  if (!p.tma_store) mc = ma;  // unused
+  if (G > 1 && !p.tma_store) return false;  // grouped outputs only through TMA stores
   // fused GELU epilogues need the bf16 TMA-store path (and no accumulation into C)
   p.epi = g.epi;
   p.aux = static_cast<const bf16*>(g.aux);
   p.ldaux = g.ldaux;
-  CUtensorMap mc2 = mc;
+  tm.c2 = tm.c[0];
   if (g.epi) {
     if (!p.tma_store || p.c_f32 || g.beta != 0.f || !g.aux) return false;
-    if (g.epi == 1 && !make_map(&mc2, g.aux, g.ldaux, 0, 0, g.N, g.M, 1, 1, 32, 32, 2,
+    if (g.epi == 1 && !make_map(&tm.c2, g.aux, g.ldaux, 0, 0, g.N, g.M, 1, 1, 32, 32, 2,
                                 CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, CU_TENSOR_MAP_SWIZZLE_64B))
       return false;
     if (g.epi == 2 && ((reinterpret_cast<uintptr_t>(g.aux) | uintptr_t(g.ldaux * 2)) & 15)) return false;
@@ -674,7 +743,12 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   p.ksplit = 1;
   if (best_ks > 1 && p.tma_store && p.c_f32) {
     p.ksplit = best_ks;
-    if (g.beta == 0.f) cudaMemsetAsync(g.c, 0, size_t(g.M) * g.N * 4, st);
+    if (g.beta == 0.f) {
+      if (G > 1 && g.gdim != 2)
+        for (int i = 0; i < G; ++i) cudaMemsetAsync(g.cg[i], 0, size_t(Mc) * Nc * 4, st);
+      else
+        cudaMemsetAsync(g.c, 0, size_t(g.M) * g.N * 4, st);
+    }
     p.reduce_add = 1;
   }
   p.kb_per_split = (p.num_kb + p.ksplit - 1) / p.ksplit;
@@ -693,31 +767,31 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   g_last = GemmConfig{best_bn, best_cg, p.ksplit, p.num_units, g_num_sms, g_pair_slots, p.split_from};
   if (best_cg == 2) {
     if (p.c_f32) {
-      if (best_bn == 256) launch<256, true, 8, 2>(ma, mb, mc, mc2, p, st);
-      else launch<128, true, 8, 2>(ma, mb, mc, mc2, p, st);
+      if (best_bn == 256) launch<256, true, 8, 2>(tm, p, st);
+      else launch<128, true, 8, 2>(tm, p, st);
     } else if (best_bn == 256) {
-      if (p.epi == 1) launch<256, false, 16, 2>(ma, mb, mc, mc2, p, st);
-      else launch<256, false, 8, 2>(ma, mb, mc, mc2, p, st);
+      if (p.epi == 1) launch<256, false, 16, 2>(tm, p, st);
+      else launch<256, false, 8, 2>(tm, p, st);
     } else {
-      if (p.epi == 1) launch<128, false, 16, 2>(ma, mb, mc, mc2, p, st);
-      else launch<128, false, 8, 2>(ma, mb, mc, mc2, p, st);
+      if (p.epi == 1) launch<128, false, 16, 2>(tm, p, st);
+      else launch<128, false, 8, 2>(tm, p, st);
     }
     return true;
   }
   if (p.c_f32) {
     switch (best_bn) {
-      case 256: launch<256, true>(ma, mb, mc, mc2, p, st); break;
-      case 128: launch<128, true>(ma, mb, mc, mc2, p, st); break;
-      default: launch<64, true>(ma, mb, mc, mc2, p, st); break;
+      case 256: launch<256, true>(tm, p, st); break;
+      case 128: launch<128, true>(tm, p, st); break;
+      default: launch<64, true>(tm, p, st); break;
     }
   } else {
     switch (best_bn) {
       case 256:
-        if (p.epi == 1) launch<256, false, 16>(ma, mb, mc, mc2, p, st);
-        else launch<256, false>(ma, mb, mc, mc2, p, st);
+        if (p.epi == 1) launch<256, false, 16>(tm, p, st);
+        else launch<256, false>(tm, p, st);
         break;
-      case 128: launch<128, false>(ma, mb, mc, mc2, p, st); break;
-      default: launch<64, false>(ma, mb, mc, mc2, p, st); break;
+      case 128: launch<128, false>(tm, p, st); break;
+      default: launch<64, false>(tm, p, st); break;
     }
   }
   return true;
@@ -735,7 +809,28 @@ void gemm(const GemmArgs& g, cudaStream_t st) {
     cudaEventRecord(rec.start, st);
   }
   rec.tc = gemm_tc(g, st) ? 1 : 0;
-  if (!rec.tc) {
+  if (!rec.tc && g.groups > 1) {
+    // no tcgen05 tiling for the grouped product: run its groups as plain products
+    const int G = g.groups;
+    for (int i = 0; i < G; ++i) {
+      GemmArgs s1 = g;
+      s1.groups = 1;
+      s1.gdim = 0;
+      if (g.gdim == 1) {
+        s1.N = g.N / G; s1.b = g.bg[i]; s1.c = g.cg[i]; s1.bias = g.biasg[i];
+      } else if (g.gdim == 2) {
+        s1.K = g.K / G; s1.a = g.ag[i]; s1.b = g.bg[i];
+        if (i > 0) s1.beta = 1.f;
+        if (i > 0) s1.bias = nullptr;
+      } else {
+        s1.M = g.M / G; s1.a = g.ag[i]; s1.c = g.cg[i];
+      }
+      std::vector<GemmRecord>* sink = g_sink;  // one record for the grouped product
+      g_sink = nullptr;
+      gemm(s1, st);
+      g_sink = sink;
+    }
+  } else if (!rec.tc) {
     GemmArgs plain = g;
     plain.epi = 0;
     gemm_simt(plain, st);

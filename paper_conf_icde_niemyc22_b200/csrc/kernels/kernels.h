@@ -20,6 +20,7 @@ struct GemmOperand {
   bool mn_major = false;
   int64_t bs1 = 0, bs2 = 0;
 };
+constexpr int kMaxGroups = 3;
 struct GemmArgs {
   int M = 0, N = 0, K = 0, nb1 = 1, nb2 = 1;
   int in_dtype = BF16;
@@ -37,6 +38,15 @@ struct GemmArgs {
   int epi = 0;
   void* aux = nullptr;
   int64_t ldaux = 0;
+  // grouped product (tcgen05 path only, unbatched, epi 0, beta 0 or 1): `groups` equal
+  // slices along gdim, M/N/K being the totals.  gdim 1 (N): C_g = A B_g^T + bias_g, per
+  // group bg/cg/biasg, shared a; gdim 2 (K): C = sum_g A_g B_g^T, per group ag/bg, shared
+  // c; gdim 3 (M): C_g = A_g B^T, per group ag/cg, shared b.  Used to run the q/k/v
+  // linears of one micro-op (same input X) as one launch.
+  int groups = 1, gdim = 0;
+  GemmOperand ag[kMaxGroups], bg[kMaxGroups];
+  void* cg[kMaxGroups] = {nullptr, nullptr, nullptr};
+  const void* biasg[kMaxGroups] = {nullptr, nullptr, nullptr};
 };
 
 // Returns false (and leaves nothing launched) when the shape/alignment does not

@@ -126,6 +126,80 @@ struct Fuse {
   char* u = nullptr;
 };
 
+// Horizontal fusion (reading D-QKV): G consecutive linear micro-ops of one kind over the
+// same samples that read the same X (BERT's q/k/v) lowered as grouped GEMMs: forward
+// Y_g = X W_g^T + b_g (N groups, X read once); backward dX (+)= sum_g dY_g W_g (K groups:
+// one accumulation into dX instead of G), dW_g (+)= dY_g^T X (M groups), db_g = colsum.
+struct LinGroup {
+  int G = 0;
+  int64_t R = 0, K = 0, N = 0;  // rows of the micro-op, in / out features of one group
+  char* x = nullptr;            // X view
+  char* gx = nullptr;           // dX view (backward; nullptr when X takes no gradient)
+  int gx_acc = 0;
+  char* out[tsk::kMaxGroups] = {};  // forward outputs
+  char* dy[tsk::kMaxGroups] = {};   // backward output gradients
+  int w[tsk::kMaxGroups] = {}, b[tsk::kMaxGroups] = {};
+  int wacc[tsk::kMaxGroups] = {}, bacc[tsk::kMaxGroups] = {};
+};
+
+std::function<void(cudaStream_t)> lower_linear_group(ts_session_t* s, const LinGroup& L, bool bwd, int& nk) {
+  const Graph& g = *s->g;
+  const int dt = g.dtype == TS_BF16 ? tsk::BF16 : tsk::F32;
+  const int G = L.G;
+  if (!bwd) {
+    tsk::GemmArgs a;
+    a.M = int(L.R); a.N = int(G * L.N); a.K = int(L.K); a.in_dtype = dt;
+    a.groups = G; a.gdim = 1;
+    a.a = {L.x, L.K, false, 0, 0};
+    for (int i = 0; i < G; ++i) {
+      a.bg[i] = {param_w(s, L.w[i]), L.K, false, 0, 0};
+      a.cg[i] = L.out[i];
+      a.biasg[i] = param_w(s, L.b[i]);
+    }
+    a.b = a.bg[0]; a.c = a.cg[0]; a.bias = a.biasg[0];
+    a.ldc = L.N; a.c_dtype = dt; a.bias_dtype = dt;
+    nk = 1;
+    return [a](cudaStream_t st) { tsk::gemm(a, st); };
+  }
+  std::vector<tsk::GemmArgs> gs;
+  if (L.gx) {
+    tsk::GemmArgs a;
+    a.M = int(L.R); a.N = int(L.K); a.K = int(G * L.N); a.in_dtype = dt;
+    a.groups = G; a.gdim = 2;
+    for (int i = 0; i < G; ++i) {
+      a.ag[i] = {L.dy[i], L.N, false, 0, 0};
+      a.bg[i] = {param_w(s, L.w[i]), L.K, true, 0, 0};
+    }
+    a.a = a.ag[0]; a.b = a.bg[0];
+    a.c = L.gx; a.ldc = L.K; a.c_dtype = dt; a.beta = L.gx_acc ? 1.f : 0.f;
+    gs.push_back(a);
+  }
+  {
+    tsk::GemmArgs d;
+    d.M = int(G * L.N); d.N = int(L.K); d.K = int(L.R); d.in_dtype = dt;
+    d.groups = G; d.gdim = 3;
+    for (int i = 0; i < G; ++i) {
+      d.ag[i] = {L.dy[i], L.N, true, 0, 0};
+      d.cg[i] = param_g(s, L.w[i]);
+    }
+    d.a = d.ag[0]; d.c = d.cg[0];
+    d.b = {L.x, L.K, true, 0, 0};
+    d.ldc = L.K; d.c_dtype = tsk::F32; d.beta = L.wacc[0] ? 1.f : 0.f;
+    gs.push_back(d);
+  }
+  float* ws = reinterpret_cast<float*>(s->slab + g.ws_off);
+  const uint64_t wsb = g.ws_bytes;
+  std::vector<std::pair<char*, std::pair<float*, int>>> cs;
+  for (int i = 0; i < G; ++i) cs.push_back({L.dy[i], {param_g(s, L.b[i]), L.bacc[i]}});
+  const int64_t R = L.R;
+  const int N = int(L.N);
+  nk = int(gs.size()) + G;
+  return [gs, cs, R, N, ws, wsb, dt](cudaStream_t st) {
+    for (auto& a : gs) tsk::gemm(a, st);
+    for (auto& c : cs) tsk::column_sum(dt, c.first, R, N, ws, wsb, c.second.first, c.second.second, nullptr, 0, st);
+  };
+}
+
 // Lower one micro-op to kernel launches (DESIGN.md §3 op table).
 std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bwd, int& nk,
                                         const Fuse* fz = nullptr) {
@@ -615,6 +689,9 @@ ts_status build_program(ts_session_t* s) {
   // TSPLIT_NO_FUSION=1 lowers every micro-op on its own (tests compare the two programs)
   const char* nf = std::getenv("TSPLIT_NO_FUSION");
   const bool fusion_on = !(nf && nf[0] == '1');
+  // TSPLIT_NO_QKV_FUSION=1 keeps the linear + gelu fusion but lowers q/k/v one by one
+  const char* nq = std::getenv("TSPLIT_NO_QKV_FUSION");
+  const bool qkv_on = fusion_on && !(nq && nq[0] == '1');
   auto overlaps = [](uint64_t a0, uint64_t al, uint64_t b0, uint64_t bl) { return a0 < b0 + bl && b0 < a0 + al; };
   for (size_t i = 0; i < s->ex.items.size(); ++i) {
     const Item& it = s->ex.items[i];
@@ -721,12 +798,85 @@ ts_status build_program(ts_session_t* s) {
         if (!list(o.in[0], m.all_x)) return set_error("batchnorm: too many pieces"), TS_ERR_GRAPH;
         if (bwd && !list(n + o.out[0], m.all_dy)) return set_error("batchnorm: too many pieces"), TS_ERR_GRAPH;
       }
+      // q/k/v horizontal fusion (bf16, reading D-QKV): the next G-1 items are linear micro-ops
+      // of the same kind, samples and group reading the same X with equally shaped weights;
+      // forward/replay: each sibling's only allocation is its output piece and no range freed
+      // since this item overlaps it; backward: the siblings allocate nothing, their weight
+      // gradients accumulate alike; no sibling has copy fences.
+      LinGroup lg;
+      if (qkv_on && g.dtype == TS_BF16 && o.kind == TS_OP_LINEAR && !fused_away.count(int(i)) &&
+          g.t[o.in[0]].kind == TS_ACT) {
+        const int64_t N0 = g.t[o.in[1]].shape[0], K0 = g.t[o.in[1]].shape[1];
+        std::vector<size_t> sib;
+        std::vector<char*> outs;
+        for (size_t j = i + 1; j < s->ex.items.size() && sib.size() + 1 < size_t(tsk::kMaxGroups); ++j) {
+          const Item& nx = s->ex.items[j];
+          const Op& no = g.ops[nx.op];
+          if (nx.kind != it.kind || nx.k != it.k || nx.group != it.group || s->ex.P[nx.op] != m.P) break;
+          if (no.kind != TS_OP_LINEAR || no.in[0] != o.in[0] || nx.op == it.op) break;
+          if (g.t[no.in[1]].shape[0] != N0 || g.t[no.in[1]].shape[1] != K0) break;
+          if (!s->sim.wait_so[j].empty()) break;
+          bool okj = true;
+          if (!bwd) {
+            const int ot = no.out[0];
+            const Event* a = nullptr;
+            for (const Event* e : allocs_of[j]) {
+              if (e->key == ot && !a) a = e;
+              else okj = false;
+            }
+            if (!a) okj = false;
+            for (size_t f = i; okj && f < j; ++f)
+              for (const Event* e : frees_of[f])
+                if (overlaps(a->offset, align_up(a->bytes), e->offset, align_up(e->bytes))) okj = false;
+            if (okj) {
+              const Tensor& y = g.t[ot];
+              const int py = piece_count(g, s->cfg, ot);
+              const int jj = int(m.s0 * py / B);
+              const int64_t first = int64_t(jj) * B / py;
+              if (a->piece != jj) okj = false;
+              else outs.push_back(s->slab + a->offset + (m.s0 - first) * y.elems_per_sample * es);
+            }
+          } else {
+            if (!allocs_of[j].empty()) okj = false;
+            const int ot = no.out[0];
+            const int pg = piece_count(g, s->cfg, ot);
+            if (okj && !where.count(pk(n + ot, int(m.s0 * pg / B)))) okj = false;
+            if (okj && (param_started.count(no.in[1]) != param_started.count(o.in[1]) ||
+                        param_started.count(no.in[2]) != param_started.count(o.in[2])))
+              okj = false;
+          }
+          if (!okj) break;
+          sib.push_back(j);
+        }
+        const bool out_ok = !bwd ? m.val.count(o.out[0]) > 0 : m.grad.count(o.out[0]) > 0;
+        if (!sib.empty() && out_ok && m.val.count(o.in[0])) {
+          lg.G = int(sib.size()) + 1;
+          lg.R = (m.s1 - m.s0) * g.t[o.in[0]].rows_per_sample;
+          lg.K = K0;
+          lg.N = N0;
+          lg.x = m.val.at(o.in[0]);
+          for (int gi = 0; gi < lg.G; ++gi) {
+            const Op& go2 = g.ops[gi == 0 ? it.op : s->ex.items[sib[gi - 1]].op];
+            lg.w[gi] = go2.in[1];
+            lg.b[gi] = go2.in[2];
+            lg.wacc[gi] = param_started.count(go2.in[1]) ? 1 : 0;
+            lg.bacc[gi] = param_started.count(go2.in[2]) ? 1 : 0;
+            if (!bwd) lg.out[gi] = gi == 0 ? m.val.at(o.out[0]) : outs[gi - 1];
+            else lg.dy[gi] = gi == 0 ? m.grad.at(o.out[0]) : view(n + go2.out[0]);
+          }
+          if (bwd && m.grad.count(o.in[0]) && g.t[o.in[0]].needs_grad) {
+            lg.gx = m.grad.at(o.in[0]);
+            lg.gx_acc = m.acc.count(n + o.in[0]) ? m.acc.at(n + o.in[0]) : 0;
+          }
+          for (size_t j : sib) fused_away.insert(int(j));
+        }
+      }
       // linear + gelu peephole fusion (bf16): the next item is the gelu micro-op over the same
       // samples; its output (forward) / input gradient (backward) range must already be free
       // while this item runs — it is allocated at the next item and no range freed after this
       // item overlaps it — and the next item must have no copy fences of its own.
       Fuse fz;
-      if (fusion_on && g.dtype == TS_BF16 && o.kind == TS_OP_LINEAR && i + 1 < s->ex.items.size()) {
+      if (fusion_on && !lg.G && g.dtype == TS_BF16 && o.kind == TS_OP_LINEAR && i + 1 < s->ex.items.size()) {
         const Item& nx = s->ex.items[i + 1];
         const Op& go = g.ops[nx.op];
         const bool same = nx.kind == it.kind && nx.k == it.k && s->ex.P[nx.op] == m.P && nx.group == it.group &&
@@ -770,7 +920,9 @@ ts_status build_program(ts_session_t* s) {
         }
       }
       int nk = 0;
-      if (fused_away.count(int(i))) {
+      if (lg.G) {
+        cmd.fn = lower_linear_group(s, lg, bwd, nk);
+      } else if (fused_away.count(int(i))) {
         cmd.fn = [](cudaStream_t) {};
       } else {
         cmd.fn = lower(s, m, bwd, nk, fz.mode ? &fz : nullptr);
@@ -1340,6 +1492,31 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch, const voi
   g.alpha = alpha; g.beta = beta; g.bias = bias; g.bias_dtype = tsk::BF16;
   if (!tsk::gemm_tc(g, static_cast<cudaStream_t>(stream)))
     return set_error("shape/alignment not eligible for the tcgen05/TMA path"), TS_ERR_ARG;
+  CU(cudaGetLastError());
+  return TS_OK;
+}
+
+ts_status ts_gemm_bf16_grouped(int32_t groups, int32_t gdim, int32_t M, int32_t N, int32_t K,
+                               const void* const* A, int64_t lda, int32_t ta, const void* const* B, int64_t ldb,
+                               int32_t tb, void* const* C, int64_t ldc, int32_t c_dtype, float alpha, float beta,
+                               const void* const* bias, void* stream) {
+  if (groups < 1 || groups > tsk::kMaxGroups || gdim < 1 || gdim > 3 || !A || !B || !C)
+    return set_error("grouped gemm: 1 <= groups <= 3, gdim in {1, 2, 3}, A/B/C arrays required"), TS_ERR_ARG;
+  tsk::GemmArgs g;
+  g.M = M; g.N = N; g.K = K; g.in_dtype = tsk::BF16;
+  g.groups = groups; g.gdim = gdim;
+  g.a = {A[0], lda, ta != 0, 0, 0};
+  g.b = {B[0], ldb, tb != 0, 0, 0};
+  g.c = C[0]; g.ldc = ldc; g.c_dtype = c_dtype == TS_F32 ? tsk::F32 : tsk::BF16;
+  g.alpha = alpha; g.beta = beta; g.bias = bias ? bias[0] : nullptr; g.bias_dtype = tsk::BF16;
+  for (int i = 0; i < groups; ++i) {
+    g.ag[i] = {gdim == 1 ? A[0] : A[i], lda, ta != 0, 0, 0};
+    g.bg[i] = {gdim == 3 ? B[0] : B[i], ldb, tb != 0, 0, 0};
+    g.cg[i] = gdim == 2 ? C[0] : C[i];
+    g.biasg[i] = bias ? (gdim == 1 ? bias[i] : bias[0]) : nullptr;
+  }
+  if (!tsk::gemm_tc(g, static_cast<cudaStream_t>(stream)))
+    return set_error("grouped product not eligible for the tcgen05/TMA path"), TS_ERR_ARG;
   CU(cudaGetLastError());
   return TS_OK;
 }

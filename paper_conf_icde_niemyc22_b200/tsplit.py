@@ -131,6 +131,8 @@ def lib():
             "ts_nccl_comm_destroy": (i32, [vp]),
             "ts_gemm_bf16": (i32, [i32, i32, i32, i32, vp, i64, i64, i32, vp, i64, i64, i32,
                                    vp, i64, i64, i32, C.c_float, C.c_float, vp, vp]),
+            "ts_gemm_bf16_grouped": (i32, [i32, i32, i32, i32, i32, P(vp), i64, i32, P(vp), i64, i32, P(vp), i64,
+                                           i32, C.c_float, C.c_float, P(vp), vp]),
             "ts_gemm_set_mode": (i32, [i32]),
             "ts_gemm_last_config": (i32, [P(i32)]),
             "ts_gemm_f32": (i32, [i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, C.c_float,

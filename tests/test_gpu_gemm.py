@@ -131,3 +131,48 @@ def test_gemm_tc_accumulate_and_splitk(M, N, K, out, beta, mode, gemm_mode):
     err = ((C.double() - ref).norm() / ref.norm()).item()
     # fp32 accumulation over K terms: ~sqrt(K) * 2^-24 relative
     assert err < (3e-5 if out == "f32" else 8e-3), err
+
+
+def _ptrs(ts):
+    return (tsplit.C.c_void_p * len(ts))(*[t.data_ptr() for t in ts])
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2])
+@pytest.mark.parametrize("gdim,M,N,K,ta,tb,out,beta", [
+    (1, 1024, 3 * 256, 256, 0, 0, "bf16", 0.0),    # q/k/v forward: shared X, per-group W, C, bias
+    (1, 600, 3 * 512, 192, 0, 0, "bf16", 0.0),     # ragged M
+    (2, 1024, 256, 3 * 256, 0, 1, "bf16", 1.0),    # q/k/v dX: sum over groups into one C (accumulate)
+    (2, 640, 384, 3 * 128, 0, 1, "bf16", 0.0),
+    (3, 3 * 256, 256, 2048, 1, 1, "f32", 1.0),     # q/k/v dW: per-group dY^T, shared X, per-group dW
+    (3, 3 * 512, 512, 1024, 1, 1, "f32", 0.0),
+])
+def test_gemm_tc_grouped(gdim, M, N, K, ta, tb, out, beta, mode, gemm_mode):
+    """Grouped product = the per-group plain products (fp32 torch reference)."""
+    gemm_mode(mode)
+    G = 3
+    Mg, Ng, Kg = (M // G if gdim == 3 else M), (N // G if gdim == 1 else N), (K // G if gdim == 2 else K)
+    A = [_mk((Mg, Kg), seed=1 + i) for i in range(G if gdim != 1 else 1)]
+    B = [_mk((Ng, Kg), seed=10 + i) for i in range(G if gdim != 3 else 1)]
+    od = torch.float32 if out == "f32" else torch.bfloat16
+    nC = G if gdim != 2 else 1
+    Cs = [torch.randn(Mg, Ng, device="cuda").to(od) for _ in range(nC)]
+    C0 = [c.clone() for c in Cs]
+    bias = [_mk((Ng,), seed=40 + i) for i in range(G if gdim == 1 else 1)] if gdim == 1 else None
+    Aop = [_op(a, ta) for a in A]
+    Bop = [_op(b, tb) for b in B]
+    lda = Mg if ta else Kg
+    ldb = Ng if tb else Kg
+    st = tsplit.lib().ts_gemm_bf16_grouped(G, gdim, M, N, K, _ptrs(Aop), lda, ta, _ptrs(Bop), ldb, tb, _ptrs(Cs), Ng,
+                                           0 if out == "f32" else 1, 1.0, beta, _ptrs(bias) if bias else None, None)
+    tsplit.check(st)
+    torch.cuda.synchronize()
+    for i in range(nC):
+        if gdim == 1:
+            ref = A[0].float() @ B[i].float().t() + bias[i].float()
+        elif gdim == 2:
+            ref = sum(A[j].float() @ B[j].float().t() for j in range(G))
+        else:
+            ref = A[i].float() @ B[0].float().t()
+        ref = ref + beta * C0[i].float()
+        err = ((Cs[i].float() - ref).norm() / ref.norm()).item()
+        assert err < (2e-5 if out == "f32" else 8e-3), (i, err)

@@ -171,18 +171,45 @@ def test_nccl_bucketed_allreduce_single_rank():
     assert np.allclose(out[1][1], out[0][1], rtol=1e-6, atol=1e-9)
 
 
-def _fusion_pair(g, cfg):
-    """The same step with and without the linear + gelu peephole fusion (TSPLIT_NO_FUSION)."""
+def _fusion_pair(g, cfg, var="TSPLIT_NO_FUSION", qkv=False):
+    """The same step with and without a session fusion: `var` = 1 turns it off.  The
+    linear + gelu comparison keeps the q/k/v grouping off in both runs (qkv=False)."""
     import os
     out = []
     for off in ("1", "0"):
-        os.environ["TSPLIT_NO_FUSION"] = off
+        os.environ[var] = off
+        if not qkv:
+            os.environ["TSPLIT_NO_QKV_FUSION"] = "1"
         try:
             loss, grads, S, _ = _run(g, cfg)
             out.append((loss, grads, S.launches()))
         finally:
-            os.environ.pop("TSPLIT_NO_FUSION", None)
+            os.environ.pop(var, None)
+            os.environ.pop("TSPLIT_NO_QKV_FUSION", None)
     return out
+
+
+@pytest.mark.parametrize("plan", ["reside", "recompute_qkv", "split"])
+def test_qkv_grouped_fusion(plan):
+    """bf16 graphs (reading D-QKV): the q/k/v linear micro-ops of a layer run as grouped
+    GEMMs — forward and recompute replays one N-grouped product, backward one K-grouped dX
+    (summed in fp32, a single accumulation into dX) and one M-grouped dW.  The forward is
+    the same arithmetic (loss bit-identical); the backward differs only by the bf16
+    rounding of the dX accumulation; both stay within the bf16 bar of the oracle."""
+    g = graphs.config_graph("bert_tiny", fused_attention=True)
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    cfg = {}
+    if plan == "recompute_qkv":
+        cfg = {names[f"l0.{x}"]: (tsplit.RECOMPUTE, 1, 1) for x in ("q", "k", "v")}
+    elif plan == "split":
+        cfg = {names[f"l1.{x}"]: (tsplit.RESIDE, 2, 1) for x in ("q", "k", "v")}
+    (l0, g0, n0), (l1, g1, n1) = _fusion_pair(g, cfg, var="TSPLIT_NO_QKV_FUSION", qkv=True)
+    assert n1 < n0, (n0, n1)
+    assert l1 == l0
+    assert global_rel_err(g1, g0) <= 5e-3
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    _, ogb, _, _ = net.train_step(g, params, inputs, storage="bf16")
+    assert global_rel_err(g1, ogb) <= 2e-2
 
 
 @pytest.mark.parametrize("fused_attention", [False, True])
