@@ -101,7 +101,10 @@ typedef struct {
 /* Per-tensor configuration: Fig. 9 `struct config` {opt, p_num, dim} plus the
  * prefetch lead of a swapped tensor (swap-in starts `prefetch_lead` compute
  * items before its first backward use; 1 = "the previous computation
- * operation").  dim 0 = the sample dim (the only one in this build). */
+ * operation").  dim 0 = the sample dim ("sample dim"); dim 1 = the
+ * channel / parameter dim of a 2-D activation [rows, C] (Fig. 6): p_num
+ * contiguous column blocks [rows, C/p_num], legal per DESIGN.md reading D-CH (produced by
+ * a linear or relu/gelu/tanh, read by a linear as X or relu/gelu/tanh). */
 typedef struct {
   int32_t tensor_id;
   int32_t opt;           /* ts_opt */
@@ -202,8 +205,14 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
                      ts_plan_t** out);
 ts_status ts_plan_get(const ts_plan_t* p, int32_t tensor_id, ts_tensor_cfg* out);
 /* Forced configuration (Fig. 9 set_config); the plan is re-expanded and
- * re-simulated.  Only TS_ACT tensors accept opt != RESIDE or p_num > 1. */
+ * re-simulated.  Only TS_ACT tensors accept opt != RESIDE or p_num > 1.  p_num divides
+ * the samples (dim 0) or the columns (dim 1).  TS_ERR_ARG (plan unchanged) when a field
+ * is out of range or the resulting plan breaks the channel-split rules (D-CH). */
 ts_status ts_plan_set(ts_plan_t* p, const ts_tensor_cfg* cfg);
+/* Several configurations applied together, then validated as one (a channel-split chain,
+ * e.g. linear -> gelu, is only legal as a whole).  cfgs: host array of n entries, copied.
+ * TS_ERR_ARG leaves the plan unchanged. */
+ts_status ts_plan_set_many(ts_plan_t* p, const ts_tensor_cfg* cfgs, int32_t n);
 ts_status ts_plan_stats(const ts_plan_t* p, ts_plan_stats_t* out);
 /* LRU-based recomputation ("execute as the speed-centric manner and abandon the
  * least recently used intermediate tensor once the available memory is not enough";

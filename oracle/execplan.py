@@ -29,12 +29,20 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
     def p_of(t):
         return cfg[t][1] if (an.sample[t] and ts[t]["kind"] == "act") else 1
 
+    def chan(t):  # channel-split (D-CH): p blocks of columns, each over every sample
+        return an.sample[t] and ts[t]["kind"] == "act" and sim.dim_of(cfg, t) == 1 and p_of(t) > 1
+
+    def cmode(o):
+        return any(chan(t) for t in ops[o]["outputs"])
+
     def rows_per_sample(t):
         return ts[t]["shape"][0] // B
 
     def piece_shape(t):
         sh = list(ts[t]["shape"])
-        if an.sample[t]:
+        if chan(t):
+            sh[1] //= p_of(t)
+        elif an.sample[t]:
             sh[0] //= p_of(t)
         return tuple(sh)
 
@@ -44,9 +52,11 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
             store[(t["id"], 0)] = a.astype(np.int64) if t["dtype"] == "i32" else a.astype(F)
 
     def P_op(o):
+        if cmode(o):
+            return max(p_of(t) for t in ops[o]["outputs"] if chan(t))
         P = 1
         for t in ops[o]["inputs"] + ops[o]["outputs"]:
-            if an.sample[t]:
+            if an.sample[t] and not chan(t):
                 P = max(P, p_of(t))
         return P
 
@@ -54,6 +64,9 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
         """Rows of samples [s0, s1) of tensor t inside its resident piece."""
         if not an.sample[t]:
             return store[(n + t if grad else t, 0)]
+        if chan(t):  # every block's rows, side by side (a copy: read-only use)
+            r = rows_per_sample(t)
+            return np.concatenate([store[(n + t if grad else t, j)][s0 * r:s1 * r] for j in range(p_of(t))], axis=1)
         p = p_of(t)
         per = B // p
         j = s0 // per
@@ -63,6 +76,48 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
         return arr[(s0 - j * per) * r:(s1 - j * per) * r]
 
     bn_stats, bn_sums = {}, {}
+
+    def channel_micro_op(it):
+        """Micro-op k of an op in channel mode (D-CH): output channels block k over all
+        samples.  A linear's block k is the same linear with weight rows / bias block k;
+        an elementwise op maps block k of its input to block k of its output."""
+        o = ops[it.op]
+        k = it.k
+        out = o["outputs"][0]
+        w = ts[out]["shape"][1] // p_of(out)
+        val = dict(pval)
+        if o["kind"] == "linear":
+            x, wid, bid = o["inputs"]
+            val[wid] = pval[wid][k * w:(k + 1) * w]
+            val[bid] = pval[bid][k * w:(k + 1) * w]
+            val[x] = view(x, 0, B)
+        elif it.kind in ("F", "R"):
+            val[o["inputs"][0]] = store[(o["inputs"][0], k)]
+        else:  # the backward reads block k of what the op saved (gelu X, relu / tanh Y)
+            for t in an.saved[it.op]:
+                val[t] = store[(t, k)]
+        if it.kind in ("F", "R"):
+            store[(out, k)][...] = net.forward_op(graph, o, val, row0=0, elem0=0, step=step)
+            return
+        dy = store[(n + out, k)]
+        contrib = net.backward_op(graph, o, val, dy, row0=0, elem0=0, step=step)
+        for tid, g in contrib.items():
+            if o["kind"] == "linear" and tid == o["inputs"][1]:
+                pgrad[tid][k * w:(k + 1) * w] += g
+            elif o["kind"] == "linear" and tid == o["inputs"][2]:
+                pgrad[tid][k * w:(k + 1) * w] += g
+            elif ts[tid]["kind"] == "param":
+                pgrad[tid] += g
+            elif tid not in an.needs_grad:
+                continue
+            elif o["kind"] != "linear":  # elementwise: block k of its input's gradient
+                store[(n + tid, k)][...] += g
+            elif chan(tid):
+                r_w = g.shape[1] // p_of(tid)
+                for j in range(p_of(tid)):
+                    store[(n + tid, j)][...] += g[:, j * r_w:(j + 1) * r_w]
+            else:
+                view(tid, 0, B, grad=True)[...] += g
 
     def whole(t, grad=False):
         """All pieces of tensor t concatenated (the full batch)."""
@@ -76,7 +131,9 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
                 store[pc] = host.pop(pc)
             else:
                 store[pc] = np.zeros(piece_shape(t), F)
-        if it.kind in ("F", "R", "B"):
+        if it.kind in ("F", "R", "B") and cmode(it.op):
+            channel_micro_op(it)
+        elif it.kind in ("F", "R", "B"):
             o = ops[it.op]
             P = P_op(it.op)
             s0, s1 = it.k * B // P, (it.k + 1) * B // P
@@ -121,6 +178,10 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
                 for tid, g in contrib.items():
                     if ts[tid]["kind"] == "param":
                         pgrad[tid] += g
+                    elif tid in an.needs_grad and chan(tid):  # scatter the columns into the blocks
+                        r, w = rows_per_sample(tid), g.shape[1] // p_of(tid)
+                        for j in range(p_of(tid)):
+                            store[(n + tid, j)][s0 * r:s1 * r] += g[:, j * w:(j + 1) * w]
                     elif tid in an.needs_grad:
                         view(tid, s0, s1, grad=True)[...] += g
         elif it.kind == "SO":

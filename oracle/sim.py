@@ -64,6 +64,68 @@ AUX_OUTPUTS = {"attention": (1, 2)}  # never differentiated (same rule as net.AU
 # static per-op buffer, so replays and later micro-ops read only their own piece.
 BATCH_REDUCE = {"batchnorm"}
 
+# Channel (parameter-dim) split, Fig. 6 / P:L258-260, reading D-CH: a 2-D
+# activation [rows, C] split along C into p contiguous blocks [rows, C/p] (the "parameter
+# dim" of its producer).  Legal when its producer is a linear (micro-op k computes output
+# channels block k with weight rows block k) or one of CHANNEL_EW with a channel-split
+# input of the same p (micro-op k maps block k to block k), and every consumer is a linear
+# reading it as X (it reads every block: the contraction over C is the merge-by-sum of
+# P:L260) or one of CHANNEL_EW.  An op with a channel-split output runs in "channel mode":
+# P = that p micro-ops over channel blocks, each over all samples; its other activations
+# are channel-split (read whole / block k as above) or unsplit.
+CHANNEL_EW = {"relu", "gelu", "tanh"}
+
+
+def dim_of(cfg, t):
+    c = cfg.get(t)
+    return c[3] if c is not None and len(c) > 3 else 0
+
+
+def check_channel(graph, cfg):
+    """Raise ValueError when a channel-split configuration breaks reading D-CH."""
+    ts, ops = graph["tensors"], graph["ops"]
+    producer, consumers = {}, {}
+    for o in ops:
+        for t in o["outputs"]:
+            producer[t] = o
+        for t in o["inputs"]:
+            consumers.setdefault(t, []).append(o)
+
+    def chan(t):
+        return dim_of(cfg, t) == 1 and cfg[t][1] > 1
+
+    for t in ts:
+        tid = t["id"]
+        if dim_of(cfg, tid) not in (0, 1):
+            raise ValueError(f"tensor {tid}: split dim must be 0 (samples) or 1 (channels)")
+        if not chan(tid):
+            continue
+        p = cfg[tid][1]
+        if t["kind"] != "act" or len(t["shape"]) != 2 or t["shape"][1] % p:
+            raise ValueError(f"tensor {tid}: channel split needs a 2-D activation with C % p == 0")
+        po = producer[tid]
+        if po["kind"] == "linear":
+            x = po["inputs"][0]
+            if not chan(x) and cfg[x][1] != 1:
+                raise ValueError(f"tensor {tid}: its linear's input must be unsplit or channel-split")
+        elif po["kind"] in CHANNEL_EW:
+            x = po["inputs"][0]
+            if not chan(x) or cfg[x][1] != p:
+                raise ValueError(f"tensor {tid}: an elementwise producer needs a channel-split input of the same p")
+        else:
+            raise ValueError(f"tensor {tid}: producer {po['kind']} cannot write channel blocks")
+        for c in consumers.get(tid, []):
+            if c["kind"] == "linear" and c["inputs"][0] == tid:
+                y = c["outputs"][0]
+                if not chan(y) and cfg[y][1] != 1 and ts[y]["kind"] == "act":
+                    raise ValueError(f"tensor {tid}: its linear consumer's output must be unsplit or channel-split")
+            elif c["kind"] in CHANNEL_EW:
+                y = c["outputs"][0]
+                if not chan(y) or cfg[y][1] != p:
+                    raise ValueError(f"tensor {tid}: an elementwise consumer needs a channel-split output of the same p")
+            else:
+                raise ValueError(f"tensor {tid}: consumer {c['kind']} cannot read channel blocks")
+
 
 def align(n):
     return (n + ALIGN - 1) // ALIGN * ALIGN
@@ -257,6 +319,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
     order = order if order is not None else schedule(graph)
     ts, ops = graph["tensors"], graph["ops"]
     n = an.n
+    check_channel(graph, cfg)
 
     def p_of(t):
         if t >= n:
@@ -269,16 +332,31 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
         return cfg[t][0]
 
     def P_op(o):
+        if cmode(o):  # channel mode: one micro-op per channel block of the output (D-CH)
+            return max(p_of(t) for t in ops[o]["outputs"] if chan(t))
         P = 1
         for t in ops[o]["inputs"] + ops[o]["outputs"]:
-            if an.sample[t]:
+            if an.sample[t] and not chan(t):
                 P = max(P, p_of(t))
         return P
 
-    def piece(t, k, P):
+    def chan(t):
+        if t >= n:
+            t -= n
+        return an.sample[t] and ts[t]["kind"] == "act" and dim_of(cfg, t) == 1 and cfg[t][1] > 1
+
+    def cmode(o):
+        return any(chan(t) for t in ops[o]["outputs"])
+
+    def pieces(t, k, P, o):
+        """The pieces of t (or of its gradient) micro-op k of op o touches (D-CH)."""
         if t < n and not an.sample[t]:
-            return 0
-        return k * p_of(t) // P
+            return [0]
+        if chan(t):
+            if cmode(o) and (t in ops[o]["outputs"] or ops[o]["kind"] in CHANNEL_EW):
+                return [k]
+            return list(range(p_of(t)))
+        return [k * p_of(t) // P]
 
     def ins_sample(o):
         return [t for t in ops[o]["inputs"] if an.sample[t]]
@@ -288,13 +366,13 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
         P = P_op(o)
         for k in range(P):
             it = Item("F", o, k)
-            it.reads = [(t, piece(t, k, P)) for t in ins_sample(o)]
+            it.reads = [(t, j) for t in ins_sample(o) for j in pieces(t, k, P, o)]
             if ops[o]["kind"] in BATCH_REDUCE and k == 0:
                 for t in ins_sample(o):
                     for j in range(p_of(t)):
                         if (t, j) not in it.reads:
                             it.reads.append((t, j))
-            it.writes = [(t, piece(t, k, P)) for t in ops[o]["outputs"]]
+            it.writes = [(t, j) for t in ops[o]["outputs"] for j in pieces(t, k, P, o)]
             items.append(it)
     fwd_end = len(items)
 
@@ -323,15 +401,16 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
                 pt = p_of(t)
                 for kk in range(j * Q // pt, (j + 1) * Q // pt):
                     for u in ins_sample(po):
-                        need(u, piece(u, kk, Q))
+                        for jj in pieces(u, kk, Q, po):
+                            need(u, jj)
                     r = Item("R", po, kk, group=gid)
-                    r.reads = [(u, piece(u, kk, Q)) for u in ins_sample(po)]
+                    r.reads = [(u, jj) for u in ins_sample(po) for jj in pieces(u, kk, Q, po)]
                     r.writes = [(t, j)]
                     group.append(r)
                 live_temp.add((t, j))
                 cache[(t, j)] = piece_nbytes(t)
 
-            saved_pieces = [(t, piece(t, k, P)) for t in an.saved[o]]
+            saved_pieces = [(t, j) for t in an.saved[o] for j in pieces(t, k, P, o)]
             if ops[o]["kind"] in BATCH_REDUCE and k == 0:
                 for t in an.saved[o]:
                     for j in range(p_of(t)):
@@ -343,16 +422,18 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
             b.reads = list(saved_pieces)
             for t in ops[o]["outputs"]:
                 if not an.is_loss[t] and t in an.needs_grad:
-                    b.reads.append((n + t, piece(t, k, P)))
+                    for j in pieces(t, k, P, o):
+                        b.reads.append((n + t, j))
                     if ops[o]["kind"] in BATCH_REDUCE and k == 0:
                         for j in range(p_of(t)):
                             if (n + t, j) not in b.reads:
                                 b.reads.append((n + t, j))
             for t in ops[o]["inputs"]:
                 if ts[t]["kind"] == "act" and t in an.needs_grad:
-                    w = (n + t, piece(t, k, P))
-                    if w not in b.writes:
-                        b.writes.append(w)
+                    for j in pieces(t, k, P, o):
+                        w = (n + t, j)
+                        if w not in b.writes:
+                            b.writes.append(w)
             group.append(b)
             items.extend(group)
             gid += 1

@@ -133,27 +133,55 @@ ts_status ts_plan_get(const ts_plan_t* p, int32_t tid, ts_tensor_cfg* out) {
   return TS_OK;
 }
 
-ts_status ts_plan_set(ts_plan_t* p, const ts_tensor_cfg* cfg) {
-  if (!p || !cfg) return set_error("null argument"), TS_ERR_ARG;
-  const Graph& g = *p->graph;
+namespace {
+// Validate one tensor configuration in isolation (its own fields); D-CH consistency of the
+// whole plan is checked after all changes of a ts_plan_set / ts_plan_set_many call.
+bool cfg_fields_ok(const Graph& g, const ts_tensor_cfg* cfg) {
   int t = cfg->tensor_id;
-  if (t < 0 || t >= g.n()) return set_error("bad tensor id"), TS_ERR_ARG;
+  if (t < 0 || t >= g.n()) return set_error("bad tensor id"), false;
   bool pow2 = cfg->p_num >= 1 && cfg->p_num <= 16 && (cfg->p_num & (cfg->p_num - 1)) == 0;
-  if (!pow2 || g.samples % cfg->p_num) return set_error("p_num must be a power of 2 <= 16 dividing samples"), TS_ERR_ARG;
-  if (cfg->opt < 0 || cfg->opt > 2 || cfg->dim != 0 || cfg->prefetch_lead < 1)
-    return set_error("bad opt/dim/prefetch_lead (only the sample dim 0 is splittable)"), TS_ERR_ARG;
+  if (cfg->opt < 0 || cfg->opt > 2 || cfg->dim < 0 || cfg->dim > 1 || cfg->prefetch_lead < 1)
+    return set_error("bad opt/dim/prefetch_lead (dim 0 = samples, 1 = channels)"), false;
   const Tensor& x = g.t[t];
+  if (!pow2) return set_error("p_num must be a power of 2 <= 16"), false;
+  if (cfg->dim == 0 && g.samples % cfg->p_num) return set_error("p_num must divide the samples"), false;
+  if (cfg->dim == 1 && (x.ndim != 2 || x.shape[1] % cfg->p_num))
+    return set_error("a channel split needs a 2-D tensor whose columns p_num divides"), false;
   if ((x.kind != TS_ACT || x.is_loss) && (cfg->opt != TS_RESIDE || cfg->p_num != 1))
-    return set_error("only activations can be split, swapped or recomputed"), TS_ERR_ARG;
-  Cfg& c = p->st.cfg[t];
-  c.opt = cfg->opt;
-  c.p = cfg->p_num;
-  c.dim = cfg->dim;
-  c.lead = cfg->prefetch_lead;
+    return set_error("only activations can be split, swapped or recomputed"), false;
+  return true;
+}
+
+ts_status apply_cfgs(ts_plan_t* p, const ts_tensor_cfg* cfgs, int32_t n) {
+  const Graph& g = *p->graph;
+  for (int32_t i = 0; i < n; ++i)
+    if (!cfg_fields_ok(g, &cfgs[i])) return TS_ERR_ARG;
+  std::vector<Cfg> next = p->st.cfg;
+  for (int32_t i = 0; i < n; ++i) {
+    Cfg& c = next[cfgs[i].tensor_id];
+    c.opt = cfgs[i].opt;
+    c.p = cfgs[i].p_num;
+    c.dim = cfgs[i].p_num > 1 ? cfgs[i].dim : 0;
+    c.lead = cfgs[i].prefetch_lead;
+  }
+  std::string why;
+  if (!channel_ok(g, next, why)) return set_error("channel split (D-CH): " + why), TS_ERR_ARG;
+  p->st.cfg = std::move(next);
   Profile pr;
   profile_analytic(g, default_hw(), pr);
   plan_refresh(g, p->st, &pr);
   return TS_OK;
+}
+}  // namespace
+
+ts_status ts_plan_set(ts_plan_t* p, const ts_tensor_cfg* cfg) {
+  if (!p || !cfg) return set_error("null argument"), TS_ERR_ARG;
+  return apply_cfgs(p, cfg, 1);
+}
+
+ts_status ts_plan_set_many(ts_plan_t* p, const ts_tensor_cfg* cfgs, int32_t n) {
+  if (!p || !cfgs || n < 0) return set_error("null argument"), TS_ERR_ARG;
+  return apply_cfgs(p, cfgs, n);
 }
 
 ts_status ts_plan_stats(const ts_plan_t* p, ts_plan_stats_t* out) {

@@ -91,6 +91,11 @@ struct Expansion {
   std::vector<int> P;  // micro-op count per op
 };
 
+// D-CH channel (parameter-dim) splits (expand.cpp)
+bool is_chan(const Graph& g, const std::vector<Cfg>& cfg, int key);
+bool channel_mode(const Graph& g, const std::vector<Cfg>& cfg, int op);
+bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why);
+
 struct Event {
   int64_t seq;
   int item, kind, key, piece;

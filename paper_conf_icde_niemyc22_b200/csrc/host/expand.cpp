@@ -30,21 +30,86 @@ uint64_t piece_bytes(const Graph& g, const std::vector<Cfg>& cfg, int key) {
   return g.t[t].bytes / uint64_t(piece_count(g, cfg, key));
 }
 
+// Channel (parameter-dim) split, reading D-CH (Fig. 6; oracle/sim.py
+// check_channel): a 2-D activation split along its columns into p contiguous blocks.
+bool is_chan(const Graph& g, const std::vector<Cfg>& cfg, int key) {
+  int t = key >= g.n() ? key - g.n() : key;
+  const Tensor& x = g.t[t];
+  return x.sample && x.kind == TS_ACT && cfg[t].dim == 1 && cfg[t].p > 1;
+}
+bool channel_mode(const Graph& g, const std::vector<Cfg>& cfg, int op) {
+  for (int x : g.ops[op].out)
+    if (is_chan(g, cfg, x)) return true;
+  return false;
+}
+static bool chan_ew(int kind) { return kind == TS_OP_RELU || kind == TS_OP_GELU || kind == TS_OP_TANH; }
+
+bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
+  for (int t = 0; t < g.n(); ++t) {
+    if (cfg[t].dim != 0 && cfg[t].dim != 1) return (why = "split dim must be 0 (samples) or 1 (channels)"), false;
+    if (!is_chan(g, cfg, t)) continue;
+    const Tensor& x = g.t[t];
+    const int p = cfg[t].p;
+    if (x.ndim != 2 || x.shape[1] % p) return (why = "channel split needs a 2-D activation with C % p == 0"), false;
+    const Op& po = g.ops[x.producer];
+    const int xi = po.in.empty() ? -1 : po.in[0];
+    if (po.kind == TS_OP_LINEAR) {
+      if (!is_chan(g, cfg, xi) && g.t[xi].kind == TS_ACT && cfg[xi].p != 1)
+        return (why = "a channel-split linear output needs an unsplit or channel-split input"), false;
+    } else if (chan_ew(po.kind)) {
+      if (!is_chan(g, cfg, xi) || cfg[xi].p != p)
+        return (why = "an elementwise producer needs a channel-split input of the same p"), false;
+    } else {
+      return (why = "only linear / relu / gelu / tanh can write channel blocks"), false;
+    }
+    for (int c : x.consumers) {
+      const Op& co = g.ops[c];
+      const int y = co.out[0];
+      if (co.kind == TS_OP_LINEAR && co.in[0] == t) {
+        if (!is_chan(g, cfg, y) && g.t[y].kind == TS_ACT && cfg[y].p != 1)
+          return (why = "a linear reading channel blocks needs an unsplit or channel-split output"), false;
+      } else if (chan_ew(co.kind)) {
+        if (!is_chan(g, cfg, y) || cfg[y].p != p)
+          return (why = "an elementwise consumer needs a channel-split output of the same p"), false;
+      } else {
+        return (why = "only linear (as X) / relu / gelu / tanh can read channel blocks"), false;
+      }
+    }
+  }
+  return true;
+}
+
 void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t cache_bytes) {
   const int n = g.n();
   ex = Expansion();
   ex.P.assign(g.ops.size(), 1);
+  std::vector<char> cm(g.ops.size(), 0);
   for (auto& o : g.ops) {
     int P = 1;
-    for (int x : o.in)
-      if (g.t[x].sample) P = std::max(P, piece_count(g, cfg, x));
-    for (int x : o.out)
-      if (g.t[x].sample) P = std::max(P, piece_count(g, cfg, x));
+    cm[o.id] = channel_mode(g, cfg, o.id) ? 1 : 0;
+    if (cm[o.id]) {  // D-CH: one micro-op per channel block of the output
+      for (int x : o.out)
+        if (is_chan(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
+    } else {
+      for (int x : o.in)
+        if (g.t[x].sample && !is_chan(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
+      for (int x : o.out)
+        if (g.t[x].sample && !is_chan(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
+    }
     ex.P[o.id] = P;
   }
-  auto piece = [&](int t, int k, int P) -> int {
-    if (!g.t[t].sample) return 0;
-    return k * piece_count(g, cfg, t) / P;
+  // the pieces of t (or of its gradient) micro-op k of op `op` touches (D-CH: a channel-split
+  // tensor is block k in its channel-mode producer / elementwise consumer, else all blocks)
+  auto pieces = [&](int t, int k, int P, int op) -> std::vector<int> {
+    if (!g.t[t].sample) return {0};
+    if (is_chan(g, cfg, t)) {
+      const Op& o = g.ops[op];
+      if (cm[op] && (std::find(o.out.begin(), o.out.end(), t) != o.out.end() || chan_ew(o.kind))) return {k};
+      std::vector<int> all(piece_count(g, cfg, t));
+      for (size_t j = 0; j < all.size(); ++j) all[j] = int(j);
+      return all;
+    }
+    return {k * piece_count(g, cfg, t) / P};
   };
   std::vector<Item>& items = ex.items;
   // ---- forward phase: op-major micro-ops (R10) ------------------------------
@@ -57,13 +122,15 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       it.op = o;
       it.k = k;
       for (int x : op.in)
-        if (g.t[x].sample) it.reads.push_back(pk(x, piece(x, k, P)));
+        if (g.t[x].sample)
+          for (int j : pieces(x, k, P, o)) it.reads.push_back(pk(x, j));
       if (batch_reduce(op.kind) && k == 0)  // full-batch statistics (R13)
         for (int x : op.in)
           if (g.t[x].sample)
             for (int j = 0; j < piece_count(g, cfg, x); ++j)
               if (std::find(it.reads.begin(), it.reads.end(), pk(x, j)) == it.reads.end()) it.reads.push_back(pk(x, j));
-      for (int x : op.out) it.writes.push_back(pk(x, piece(x, k, P)));
+      for (int x : op.out)
+        for (int j : pieces(x, k, P, o)) it.writes.push_back(pk(x, j));
       items.push_back(std::move(it));
     }
   }
@@ -101,14 +168,16 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
         int pt = piece_count(g, cfg, t);
         for (int kk = j * Q / pt; kk < (j + 1) * Q / pt; ++kk) {
           for (int u : po.in)
-            if (g.t[u].sample) regen(u, piece(u, kk, Q));
+            if (g.t[u].sample)
+              for (int jj : pieces(u, kk, Q, po.id)) regen(u, jj);
           Item r;
           r.kind = IT_R;
           r.op = po.id;
           r.k = kk;
           r.group = gid;
           for (int u : po.in)
-            if (g.t[u].sample) r.reads.push_back(pk(u, piece(u, kk, Q)));
+            if (g.t[u].sample)
+              for (int jj : pieces(u, kk, Q, po.id)) r.reads.push_back(pk(u, jj));
           r.writes.push_back(pk(t, j));
           group.push_back(std::move(r));
         }
@@ -116,7 +185,8 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
         cache.push_back({pk(t, j), piece_bytes(g, cfg, t)});
       };
       std::vector<PieceKey> saved;
-      for (int t : op.saved) saved.push_back(pk(t, piece(t, k, P)));
+      for (int t : op.saved)
+        for (int j : pieces(t, k, P, op.id)) saved.push_back(pk(t, j));
       if (batch_reduce(op.kind) && k == 0)
         for (int t : op.saved)
           for (int j = 0; j < piece_count(g, cfg, t); ++j)
@@ -130,7 +200,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       b.reads = saved;
       for (int x : op.out)
         if (!g.t[x].is_loss && g.t[x].needs_grad) {
-          b.reads.push_back(pk(n + x, piece(x, k, P)));
+          for (int j : pieces(x, k, P, op.id)) b.reads.push_back(pk(n + x, j));
           if (batch_reduce(op.kind) && k == 0)
             for (int j = 0; j < piece_count(g, cfg, x); ++j)
               if (std::find(b.reads.begin(), b.reads.end(), pk(n + x, j)) == b.reads.end())
@@ -138,8 +208,10 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
         }
       for (int x : op.in)
         if (g.t[x].kind == TS_ACT && g.t[x].needs_grad) {
-          PieceKey w = pk(n + x, piece(x, k, P));
-          if (std::find(b.writes.begin(), b.writes.end(), w) == b.writes.end()) b.writes.push_back(w);
+          for (int j : pieces(x, k, P, op.id)) {
+            PieceKey w = pk(n + x, j);
+            if (std::find(b.writes.begin(), b.writes.end(), w) == b.writes.end()) b.writes.push_back(w);
+          }
         }
       group.push_back(std::move(b));
       for (auto& it : group) items.push_back(std::move(it));

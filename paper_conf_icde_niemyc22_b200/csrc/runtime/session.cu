@@ -114,6 +114,11 @@ struct Micro {
   std::set<int> writes;          // tensor ids (values) this item writes
   std::unordered_map<int, char*> val, grad;
   std::unordered_map<int, int> acc;  // grad key -> accumulate flag
+  // D-CH channel splits: cb = the output channel block of a channel-mode micro-op (-1 in
+  // sample mode); a channel-split tensor the micro-op reads whole appears as one pointer per
+  // block (its rows [s0, s1)) in vblk / gblk instead of val / grad
+  int cb = -1, cp = 1;
+  std::unordered_map<int, std::vector<char*>> vblk, gblk;
 };
 
 // Peephole fusion of a linear micro-op with the gelu micro-op next to it (build_program
@@ -216,7 +221,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
     return it == m.acc.end() ? 0 : it->second;
   };
   const Tensor& out = g.t[o.out[0]];
-  const int64_t n_out = out.sample ? ns * out.elems_per_sample : out.numel;
+  const int64_t n_out = (out.sample ? ns * out.elems_per_sample : out.numel) / (m.cb >= 0 ? m.cp : 1);
   const int64_t elem0 = out.sample ? m.s0 * out.elems_per_sample : 0;
   uint32_t* stepp = &s->step;
   switch (o.kind) {
@@ -224,6 +229,61 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       const Tensor& x = g.t[o.in[0]];
       const int64_t R = ns * x.rows_per_sample, K = x.shape[1], N = g.t[o.in[1]].shape[0];
       const int w = o.in[1], bb = o.in[2];
+      if (m.cb >= 0 || m.vblk.count(o.in[0])) {
+        // D-CH: output channel block cb (rows cb Nb.. of W, bias) and / or X read as column
+        // blocks: Y_cb = sum_j X_j W[cb rows, block j]^T + b_cb (merge = sum over K)
+        const int64_t Nb = m.cb >= 0 ? N / m.cp : N;
+        const int64_t r0 = m.cb >= 0 ? int64_t(m.cb) * Nb : 0;  // first weight row
+        const int es = dt == tsk::BF16 ? 2 : 4;
+        std::vector<char*> xb = m.vblk.count(o.in[0]) ? m.vblk.at(o.in[0]) : std::vector<char*>{V(o.in[0])};
+        const int64_t Kb = K / int64_t(xb.size());
+        char* W = param_w(s, w) + r0 * K * es;
+        std::vector<tsk::GemmArgs> gs;
+        if (!bwd) {
+          for (size_t j = 0; j < xb.size(); ++j) {
+            tsk::GemmArgs a;
+            a.M = int(R); a.N = int(Nb); a.K = int(Kb); a.in_dtype = dt;
+            a.a = {xb[j], Kb, false, 0, 0};
+            a.b = {W + int64_t(j) * Kb * es, K, false, 0, 0};
+            a.c = V(o.out[0]); a.ldc = Nb; a.c_dtype = dt; a.beta = j ? 1.f : 0.f;
+            if (j == 0) { a.bias = param_w(s, bb) + r0 * es; a.bias_dtype = dt; }
+            gs.push_back(a);
+          }
+          nk = int(gs.size());
+          return [gs](cudaStream_t st) { for (auto& a : gs) tsk::gemm(a, st); };
+        }
+        char* dY = G(o.out[0]);
+        if (x.kind == TS_ACT && x.needs_grad) {
+          std::vector<char*> gxb = m.gblk.count(o.in[0]) ? m.gblk.at(o.in[0]) : std::vector<char*>{G(o.in[0])};
+          const int acc0 = A(g.n() + o.in[0]);
+          for (size_t j = 0; j < gxb.size(); ++j) {
+            tsk::GemmArgs a;  // dX_j (+)= dY_cb W[cb rows, block j]
+            a.M = int(R); a.N = int(Kb); a.K = int(Nb); a.in_dtype = dt;
+            a.a = {dY, Nb, false, 0, 0};
+            a.b = {W + int64_t(j) * Kb * es, K, true, 0, 0};
+            a.c = gxb[j]; a.ldc = Kb; a.c_dtype = dt; a.beta = acc0 ? 1.f : 0.f;
+            gs.push_back(a);
+          }
+        }
+        float* dWb = param_g(s, w) + r0 * K;
+        const int wacc = A(w);
+        for (size_t j = 0; j < xb.size(); ++j) {
+          tsk::GemmArgs d;  // dW[cb rows, block j] (+)= dY_cb^T X_j
+          d.M = int(Nb); d.N = int(Kb); d.K = int(R); d.in_dtype = dt;
+          d.a = {dY, Nb, true, 0, 0};
+          d.b = {xb[j], Kb, true, 0, 0};
+          d.c = dWb + int64_t(j) * Kb; d.ldc = K; d.c_dtype = tsk::F32; d.beta = wacc ? 1.f : 0.f;
+          gs.push_back(d);
+        }
+        float* db = param_g(s, bb) + r0;
+        const int dacc = A(bb);
+        const uint64_t wsb = g.ws_bytes;
+        nk = int(gs.size()) + 1;
+        return [gs, dY, R, Nb, db, dacc, ws, wsb, dt](cudaStream_t st) {
+          for (auto& a : gs) tsk::gemm(a, st);
+          tsk::column_sum(dt, dY, R, int(Nb), ws, wsb, db, dacc, nullptr, 0, st);
+        };
+      }
       if (!bwd) {
         tsk::GemmArgs a;
         a.M = int(R); a.N = int(N); a.K = int(K); a.in_dtype = dt;
@@ -678,6 +738,7 @@ ts_status build_program(ts_session_t* s) {
   std::map<int, int> grad_first_op; // grad key -> first bwd op writing it
   std::set<int> param_started;
   std::map<int, int> param_first_item;
+  std::map<int, int> param_started_by;  // param -> op whose backward first wrote its gradient
   s->ev_d2h.assign(s->ex.items.size(), nullptr);
   s->ev_h2d.assign(s->ex.items.size(), nullptr);
   // per item: the trace's ALLOC / FREE events (for the linear + gelu fusion check)
@@ -740,10 +801,23 @@ ts_status build_program(ts_session_t* s) {
       m.P = s->ex.P[it.op];
       m.s0 = int64_t(it.k) * B / m.P;
       m.s1 = int64_t(it.k + 1) * B / m.P;
+      const bool cmode = channel_mode(g, s->cfg, it.op);
+      if (cmode) {  // D-CH: micro-op k = output channel block k over every sample
+        m.cb = it.k;
+        m.cp = m.P;
+        m.s0 = 0;
+        m.s1 = B;
+      }
+      const bool ew_op = o.kind == TS_OP_RELU || o.kind == TS_OP_GELU || o.kind == TS_OP_TANH;
+      // a channel-split tensor this micro-op touches as block k only (else: every block)
+      auto own_block = [&](int t) {
+        return cmode && (ew_op || std::find(o.out.begin(), o.out.end(), t) != o.out.end());
+      };
       auto view = [&](int key) -> char* {
         int t = key >= n ? key - n : key;
         const Tensor& x = g.t[t];
         if (!x.sample) return s->slab + where.at(pk(key, 0));
+        if (is_chan(g, s->cfg, t)) return s->slab + where.at(pk(key, m.k));  // own_block(t)
         int p = piece_count(g, s->cfg, t);
         int j = int(m.s0 * p / B);
         int64_t first = int64_t(j) * B / p;
@@ -755,6 +829,24 @@ ts_status build_program(ts_session_t* s) {
       for (int t : ts_all) {
         if (g.t[t].kind == TS_PARAM) continue;
         int key = t;
+        if (is_chan(g, s->cfg, t)) {
+          const bool gr = bwd && g.t[t].needs_grad && g.t[t].kind == TS_ACT && !g.t[t].is_loss;
+          if (own_block(t)) {
+            if (where.count(pk(t, m.k))) m.val[t] = view(t);
+            if (gr && where.count(pk(n + t, m.k))) m.grad[t] = view(n + t);
+          } else {  // every block, rows [s0, s1) of each
+            const int pc = piece_count(g, s->cfg, t);
+            const int64_t roff = m.s0 * g.t[t].elems_per_sample / pc * es;
+            std::vector<char*> vb, gb;
+            for (int j = 0; j < pc; ++j) {
+              if (where.count(pk(t, j))) vb.push_back(s->slab + where.at(pk(t, j)) + roff);
+              if (gr && where.count(pk(n + t, j))) gb.push_back(s->slab + where.at(pk(n + t, j)) + roff);
+            }
+            if (int(vb.size()) == pc) m.vblk[t] = vb;
+            if (int(gb.size()) == pc) m.gblk[t] = gb;
+          }
+          continue;
+        }
         if (where.count(pk(key, g.t[t].sample ? int(m.s0 * piece_count(g, s->cfg, t) / B) : 0))) m.val[t] = view(key);
         if (bwd && g.t[t].needs_grad && g.t[t].kind == TS_ACT && !g.t[t].is_loss) {
           int gk = n + t;
@@ -764,12 +856,18 @@ ts_status build_program(ts_session_t* s) {
       if (bwd) {
         for (int t : o.in) {
           if (g.t[t].kind == TS_PARAM) {
-            m.acc[t] = param_started.count(t) ? 1 : 0;
+            // channel mode: micro-op k writes weight rows block k, fresh unless an earlier op
+            // started this parameter's gradient
+            auto sb = param_started_by.find(t);
+            m.acc[t] = cmode ? (sb != param_started_by.end() && sb->second != it.op ? 1 : 0)
+                             : (param_started.count(t) ? 1 : 0);
           } else if (g.t[t].kind == TS_ACT && g.t[t].needs_grad) {
             int gk = n + t;
             auto f = grad_first_op.find(gk);
             if (f == grad_first_op.end()) grad_first_op[gk] = it.op;
             m.acc[gk] = grad_first_op[gk] != it.op ? 1 : 0;
+            // a channel-mode linear's micro-ops all write the whole dX: block 0 overwrites
+            if (cmode && o.kind == TS_OP_LINEAR && !m.acc[gk] && m.k > 0) m.acc[gk] = 1;
           }
         }
       }
@@ -803,8 +901,15 @@ ts_status build_program(ts_session_t* s) {
       // forward/replay: each sibling's only allocation is its output piece and no range freed
       // since this item overlaps it; backward: the siblings allocate nothing, their weight
       // gradients accumulate alike; no sibling has copy fences.
+      bool any_chan = false;
+      for (int t : ts_all) any_chan |= is_chan(g, s->cfg, t);
+      auto op_chan = [&](int op) {
+        for (int t : g.ops[op].in) if (is_chan(g, s->cfg, t)) return true;
+        for (int t : g.ops[op].out) if (is_chan(g, s->cfg, t)) return true;
+        return false;
+      };
       LinGroup lg;
-      if (qkv_on && g.dtype == TS_BF16 && o.kind == TS_OP_LINEAR && !fused_away.count(int(i)) &&
+      if (qkv_on && !any_chan && g.dtype == TS_BF16 && o.kind == TS_OP_LINEAR && !fused_away.count(int(i)) &&
           g.t[o.in[0]].kind == TS_ACT) {
         const int64_t N0 = g.t[o.in[1]].shape[0], K0 = g.t[o.in[1]].shape[1];
         std::vector<size_t> sib;
@@ -813,7 +918,7 @@ ts_status build_program(ts_session_t* s) {
           const Item& nx = s->ex.items[j];
           const Op& no = g.ops[nx.op];
           if (nx.kind != it.kind || nx.k != it.k || nx.group != it.group || s->ex.P[nx.op] != m.P) break;
-          if (no.kind != TS_OP_LINEAR || no.in[0] != o.in[0] || nx.op == it.op) break;
+          if (no.kind != TS_OP_LINEAR || no.in[0] != o.in[0] || nx.op == it.op || op_chan(nx.op)) break;
           if (g.t[no.in[1]].shape[0] != N0 || g.t[no.in[1]].shape[1] != K0) break;
           if (!s->sim.wait_so[j].empty()) break;
           bool okj = true;
@@ -876,7 +981,8 @@ ts_status build_program(ts_session_t* s) {
       // while this item runs — it is allocated at the next item and no range freed after this
       // item overlaps it — and the next item must have no copy fences of its own.
       Fuse fz;
-      if (fusion_on && !lg.G && g.dtype == TS_BF16 && o.kind == TS_OP_LINEAR && i + 1 < s->ex.items.size()) {
+      if (fusion_on && !lg.G && !any_chan && g.dtype == TS_BF16 && o.kind == TS_OP_LINEAR && i + 1 < s->ex.items.size() &&
+          !op_chan(s->ex.items[i + 1].op)) {
         const Item& nx = s->ex.items[i + 1];
         const Op& go = g.ops[nx.op];
         const bool same = nx.kind == it.kind && nx.k == it.k && s->ex.P[nx.op] == m.P && nx.group == it.group &&
@@ -931,7 +1037,10 @@ ts_status build_program(ts_session_t* s) {
       s->launches += nk;
       if (bwd)
         for (int t : o.in)
-          if (g.t[t].kind == TS_PARAM) param_started.insert(t);
+          if (g.t[t].kind == TS_PARAM) {
+            param_started.insert(t);
+            param_started_by.emplace(t, it.op);
+          }
     }
     // frees after this item
     while (ev < tr.size() && tr[ev].item == int(i) && tr[ev].kind == 1) {

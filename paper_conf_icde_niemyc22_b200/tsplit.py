@@ -97,6 +97,7 @@ def lib():
             "ts_plan_ex": (i32, [vp, C.c_uint64, vp, C.c_uint32, P(vp)]),
             "ts_plan_get": (i32, [vp, i32, P(TensorCfg)]),
             "ts_plan_set": (i32, [vp, P(TensorCfg)]),
+            "ts_plan_set_many": (i32, [vp, P(TensorCfg), i32]),
             "ts_plan_stats": (i32, [vp, P(PlanStats)]),
             "ts_plan_set_recompute_cache": (i32, [vp, C.c_uint64]),
             "ts_plan_trace": (i32, [vp, P(AllocEvent), u64, P(u64)]),
@@ -325,6 +326,19 @@ class Plan:
     def set(self, tid, opt=RESIDE, p_num=1, prefetch_lead=1, dim=0):
         c = TensorCfg(tid, opt, p_num, dim, prefetch_lead)
         check(lib().ts_plan_set(self.h, C.byref(c)))
+
+    def get_dim(self, tid) -> int:
+        c = TensorCfg()
+        check(lib().ts_plan_get(self.h, tid, C.byref(c)))
+        return c.dim
+
+    def set_many(self, cfgs: dict):
+        """{tensor id: (opt, p_num, prefetch_lead[, dim])} applied and validated together
+        (a channel-split chain is legal only as a whole, reading D-CH)."""
+        arr = (TensorCfg * len(cfgs))()
+        for i, (t, c) in enumerate(cfgs.items()):
+            arr[i] = TensorCfg(t, c[0], c[1], c[3] if len(c) > 3 else 0, c[2])
+        check(lib().ts_plan_set_many(self.h, arr, len(cfgs)))
 
     def set_recompute_cache(self, cache_bytes: int):
         """D-LRU recompute cache limit in bytes (0 = memory-centric; 2**64-1 = unbounded)."""

@@ -22,8 +22,11 @@ def _run(g, plan_cfg=None, budget=None, graph_mode=True, on_host=False):
         P = tsplit.Plan.plan(G, budget)
     else:
         P = tsplit.Plan.default(G)
-        for t, (o, p, lead) in (plan_cfg or {}).items():
-            P.set(t, o, p, lead)
+        if plan_cfg and any(len(c) > 3 for c in plan_cfg.values()):  # channel splits: one validated batch
+            P.set_many(plan_cfg)
+        else:
+            for t, (o, p, lead) in (plan_cfg or {}).items():
+                P.set(t, o, p, lead)
     S = tsplit.Session(G, P, use_cuda_graph=graph_mode)
     params, inputs = gen.init_params(g), gen.make_inputs(g)
     S.set_params(params)

@@ -212,3 +212,39 @@ def test_planner_lru_cache_feasible_and_not_slower():
     mc.set_recompute_cache(0)
     assert s["predicted_s"] <= mc.stats()["predicted_s"] + 1e-12
     assert s["n_replay"] <= mc.stats()["n_replay"]
+
+
+@pytest.mark.parametrize("gname,seed", [("mlp", s) for s in range(6)] + [("bert_tiny", s) for s in range(4)])
+def test_trace_bit_exact_channel_split_plans(gname, seed):
+    """D-CH channel (parameter-dim) splits: the C++ expansion, pool and trace equal the
+    oracle simulator's bit for bit (plans applied with ts_plan_set_many)."""
+    from test_oracle_channel import CHAINS, channel_cfg
+    g = graphs.config_graph(gname)
+    cfg = channel_cfg(g, random.Random(100 + seed), CHAINS[gname], prob=0.9)
+    G = tsplit.Graph(g)
+    plan = tsplit.Plan.default(G)
+    plan.set_many({t: cfg[t] for t in brute.act_tensors(g)})
+    ref = sim.simulate(g, cfg)
+    got = plan.trace()
+    assert len(got) == len(ref.trace)
+    for a, b in zip(got, ref.trace):
+        assert a == tuple(b), (a, b)
+    st = plan.stats()
+    assert (st["peak_live"], st["peak_extent"], st["n_replay"]) == (ref.peak_live, ref.peak_extent, ref.n_replay)
+    assert [it[0] for it in plan.items()] == [it.kind for it in ref.items]
+    for t in brute.act_tensors(g):
+        assert plan.get_dim(t) == (sim.dim_of(cfg, t) if cfg[t][1] > 1 else 0)
+
+
+def test_channel_split_rejected_unless_legal():
+    g = graphs.config_graph("bert_tiny")
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    plan = tsplit.Plan.default(tsplit.Graph(g))
+    before = plan.trace()
+    with pytest.raises(tsplit.TsError):   # gelu alone: its input is not channel-split
+        plan.set(names["l0.gelu"], 0, 2, 1, dim=1)
+    with pytest.raises(tsplit.TsError):   # layernorm output
+        plan.set_many({names["l0.ln1"]: (0, 2, 1, 1)})
+    assert plan.trace() == before          # unchanged after a rejected call
+    plan.set_many({names["l0.ffn1"]: (2, 2, 1, 1), names["l0.gelu"]: (1, 2, 1, 1)})
+    assert plan.get_dim(names["l0.ffn1"]) == 1

@@ -45,7 +45,11 @@ def case(name, M, N, K, ta, tb, out="bf16", batch=1, beta=0.0):
         torch.matmul(Aop, Bop, out=C if out == "bf16" else None) if out == "bf16" else torch.matmul(Aop, Bop)
     fl = 2.0 * M * N * K * batch
     modes = {}
-    for mode, tag in ((1, "cta1"), (5, "cta1_nosplit"), (2, "pair"), (6, "pair_nosplit"), (0, "auto")):
+    all_modes = ((1, "cta1"), (5, "cta1_nosplit"), (2, "pair"), (6, "pair_nosplit"), (0, "auto"))
+    only = os.environ.get("MODES")  # e.g. MODES=0 (ncu captures of the cost model's choice)
+    for mode, tag in all_modes:
+        if only is not None and str(mode) not in only.split(","):
+            continue
         tsplit.check(L.ts_gemm_set_mode(mode))
         t = timeit(ours)
         cfg = (tsplit.C.c_int32 * 8)()
@@ -53,7 +57,7 @@ def case(name, M, N, K, ta, tb, out="bf16", batch=1, beta=0.0):
         modes[tag] = {"tflops": fl / t / 1e12, "us": t * 1e6, "bn": cfg[0], "cg": cfg[1], "ksplit": cfg[2],
                       "units": cfg[3], "pair_slots": cfg[5], "split_from": cfg[6]}
     tsplit.check(L.ts_gemm_set_mode(0))
-    t_ours = modes["auto"]["us"] / 1e6
+    t_ours = modes[next(iter(modes))]["us"] / 1e6
     t_cub = timeit(cublas)
     r = {"name": name, "M": M, "N": N, "K": K, "batch": batch, "ta": ta, "tb": tb, "out": out,
          "ours_tflops": fl / t_ours / 1e12, "cublas_tflops": fl / t_cub / 1e12, "ours_us": t_ours * 1e6,
