@@ -289,6 +289,8 @@ void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& 
   plan_refresh(g, ps, &pr);
   const int n = g.n();
   auto try_cfg = [&](const std::vector<Cfg>& cfg, PlanState& out) {
+    std::string why;
+    if (!channel_ok(g, cfg, why)) return false;  // e.g. reverting one block of a D-CH chain
     out.cfg = cfg;
     out.cache = ps.cache;
     plan_refresh(g, out, &pr);
@@ -477,7 +479,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
     };
     // ---- candidates ---------------------------------------------------------------
     struct Change {
-      int t, opt, p, lead;
+      int t, opt, p, lead, dim = -1;  // dim -1: keep the tensor's split dim
     };
     struct Cand2 {
       std::vector<Change> ch;
@@ -589,6 +591,40 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
           step2.push_back(opt == TS_RECOMPUTE ? with_feeders(c, t) : c);
         }
       }
+    // D-CH: channel (parameter-dim) splits of the bottleneck op's 2-D activations, with the
+    // elementwise neighbours that must share the blocks (linear -> gelu -> linear: the
+    // FFN's [T, 4h] pair); illegal combinations are dropped by channel_ok in consider()
+    auto ew = [&](int kind) { return kind == TS_OP_RELU || kind == TS_OP_GELU || kind == TS_OP_TANH; };
+    for (int t : split_cands) {
+      const Tensor& x = g.t[t];
+      if (no_split || x.ndim != 2 || first_bw[t] < 0 || is_chan(g, ps.cfg, t)) continue;
+      // only once the sample dim is exhausted (Fig. 6: the sample split is bounded by the
+      // batch — small-batch / large-model training is where the parameter dim pays)
+      bool sample_room = false;
+      for (int p = 2 * ps.cfg[t].p; p <= 16; p *= 2) sample_room |= g.samples % p == 0;
+      if (sample_room) continue;
+      std::vector<int> chain{t};
+      for (int u = t; g.t[u].producer >= 0 && ew(g.ops[g.t[u].producer].kind);) {
+        u = g.ops[g.t[u].producer].in[0];
+        if (g.t[u].kind != TS_ACT) break;
+        chain.push_back(u);
+      }
+      for (size_t q = 0; q < chain.size(); ++q)
+        for (int c : g.t[chain[q]].consumers)
+          if (ew(g.ops[c].kind) && g.ops[c].in[0] == chain[q] &&
+              std::find(chain.begin(), chain.end(), g.ops[c].out[0]) == chain.end())
+            chain.push_back(g.ops[c].out[0]);
+      for (int p = 2; p <= 16; p *= 2) {
+        if (x.shape[1] % p || (x.shape[1] / p) % 8) break;
+        for (int opt : {TS_RESIDE, TS_SWAP, TS_RECOMPUTE}) {
+          Cand2 c;
+          c.birth = birth[t];
+          c.tensor = t;
+          for (int u : chain) c.ch.push_back({u, u == t ? opt : ps.cfg[u].opt, p, ps.cfg[u].lead, 1});
+          step2.push_back(opt == TS_RECOMPUTE ? with_feeders(c, t) : c);
+        }
+      }
+    }
     // D-R8e: a recomputed tensor regenerated for the bottleneck (a replay chain member,
     // P:L294) is allocated piece by piece at its own split; splitting it finer shrinks
     // the replay's working set, so live recompute-opt tensors get split-only proposals.
@@ -653,7 +689,11 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
         cs.cfg[chg.t].opt = chg.opt;
         cs.cfg[chg.t].p = chg.p;
         cs.cfg[chg.t].lead = chg.lead;
+        if (chg.dim >= 0) cs.cfg[chg.t].dim = chg.dim;
+        if (chg.p == 1) cs.cfg[chg.t].dim = 0;
       }
+      std::string why;
+      if (!channel_ok(g, cs.cfg, why)) return;
       plan_refresh(g, cs, &pr);
       uint64_t nt = top_of_op(cs);
       if (nt >= cur_top) return;
@@ -724,6 +764,8 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       ps.cfg[chg.t].opt = chg.opt;
       ps.cfg[chg.t].p = chg.p;
       ps.cfg[chg.t].lead = chg.lead;
+      if (chg.dim >= 0) ps.cfg[chg.t].dim = chg.dim;
+      if (chg.p == 1) ps.cfg[chg.t].dim = 0;
     }
   }
   set_error("planner did not converge");

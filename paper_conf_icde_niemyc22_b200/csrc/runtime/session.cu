@@ -904,6 +904,7 @@ ts_status build_program(ts_session_t* s) {
       bool any_chan = false;
       for (int t : ts_all) any_chan |= is_chan(g, s->cfg, t);
       auto op_chan = [&](int op) {
+        if (op < 0) return false;  // swap items
         for (int t : g.ops[op].in) if (is_chan(g, s->cfg, t)) return true;
         for (int t : g.ops[op].out) if (is_chan(g, s->cfg, t)) return true;
         return false;

@@ -74,3 +74,18 @@ def test_bert_tiny_ffn_channel_split(dtype):
         _, ogb, _, _ = net.train_step(g, params, inputs, storage="bf16")
         assert global_rel_err(grads, ogb) <= 2e-2
     assert S.trace() == [tuple(e) for e in sim.simulate(g, _full(g, cfg)).trace]
+
+
+def test_planned_channel_split_batch1_mlp():
+    """Alg. 2 at batch 1 chooses parameter-dim splits (D-CH); the GPU step under that plan
+    matches the fp64 oracle (fp32 <= 1e-5) and the runtime trace is the planned one."""
+    g = graphs.mlp(batch=1, in_dim=64, hidden=2048, depth=3, classes=10)
+    G = tsplit.Graph(g)
+    st = tsplit.Plan.default(G).stats()
+    budget = st["static_bytes"] + int(0.75 * (st["peak_extent"] - st["static_bytes"]))
+    loss, grads, S, P = _run(g, budget=budget)
+    assert any(P.get_dim(t) == 1 for t in brute.act_tensors(g))
+    ol, og = _oracle(g)
+    assert abs(loss - ol) <= 1e-5 * abs(ol)
+    assert max(rel_errs(grads, og).values()) <= 1e-5
+    assert S.trace() == P.trace()

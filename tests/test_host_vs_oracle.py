@@ -248,3 +248,31 @@ def test_channel_split_rejected_unless_legal():
     assert plan.trace() == before          # unchanged after a rejected call
     plan.set_many({names["l0.ffn1"]: (2, 2, 1, 1), names["l0.gelu"]: (1, 2, 1, 1)})
     assert plan.get_dim(names["l0.ffn1"]) == 1
+
+
+@pytest.mark.parametrize("frac", [0.9, 0.75])
+def test_planner_uses_channel_splits_when_the_batch_is_one(frac):
+    """Batch 1 leaves no sample dim to split (Fig. 6), so Alg. 2's split step proposes the
+    parameter dim (D-CH): the plan fits, splits along dim 1, its trace is the oracle
+    simulator's, and executing it gives the unsplit gradients (fp64 oracle)."""
+    from oracle import execplan, net
+    from tsinputs import gen
+    g = graphs.mlp(batch=1, in_dim=64, hidden=2048, depth=3, classes=10)
+    G = tsplit.Graph(g)
+    st = tsplit.Plan.default(G).stats()
+    budget = st["static_bytes"] + int(frac * (st["peak_extent"] - st["static_bytes"]))
+    P = tsplit.Plan.plan(G, budget)
+    assert P.stats()["peak_extent"] <= budget
+    cfg = sim.default_cfg(g)
+    for t in brute.act_tensors(g):
+        o, p, lead = P.get(t)
+        cfg[t] = (o, p, lead, P.get_dim(t))
+    assert any(c[1] > 1 and c[3] == 1 for c in cfg.values())
+    ref = sim.simulate(g, cfg)
+    assert P.trace() == [tuple(e) for e in ref.trace]
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    l0, g0, _, _ = net.train_step(g, params, inputs)
+    l1, g1 = execplan.execute(g, cfg, params, inputs)
+    assert abs(l1 - l0) <= 1e-12 * abs(l0)
+    from test_oracle_net_sim import rel_errs
+    assert max(rel_errs(g1, g0).values()) <= 1e-12
