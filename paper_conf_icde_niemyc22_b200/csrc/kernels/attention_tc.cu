@@ -288,12 +288,23 @@ __global__ void __launch_bounds__(kDqThreads, 1)
     const int i = qw * 32 + lane;
     const uint32_t trow = tmem + (uint32_t(qw * 32) << 16);
     int it = 0, kc = 0;
+    // the row's D (attn_row_dot) and raw lse, loaded one item ahead (the loads complete while
+    // the current item computes; nothing waits on them until the next item starts)
+    auto item_consts = [&](int itm, float& D_, float& lse_) {
+      const int qt_ = itm % nqt, ah_ = itm / nqt;
+      const int64_t hr = (int64_t(ah_ / p.heads) * p.heads + ah_ % p.heads) * S + qt_ * 128 + i;
+      D_ = p.D[hr];
+      lse_ = p.lse[hr];
+    };
+    float nD = 0.f, nlse = 0.f;
+    if (int(blockIdx.x) < items) item_consts(blockIdx.x, nD, nlse);
     for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
       const int qt = item % nqt, ah = item / nqt, a = ah % p.heads, b = ah / p.heads;
       const int q = qt * 128 + i;
       const int64_t hrow = (int64_t(b) * p.heads + a) * S + q;
-      const float D = p.D[hrow];  // attn_row_dot
-      const float l2 = p.lse[hrow] * kLog2e;
+      const float D = nD;
+      const float l2 = nlse * kLog2e;
+      if (item + int(gridDim.x) < items) item_consts(item + gridDim.x, nD, nlse);
       const uint32_t* mrow = p.mask + hrow * (S / 32);
       for (int kt = 0; kt < nkt; ++kt, ++kc) {
         const uint32_t bits = p.drop ? mrow[kt * 4 + cg] : ~0u;
@@ -466,23 +477,26 @@ __global__ void __launch_bounds__(kKvThreads, 1)
     const uint32_t trow = tmem + (uint32_t(qw * 32) << 16);
     const uint32_t pd = smem_u32(smem + kKvSmemPd), ds = smem_u32(smem + kKvSmemDS);
     int it = 0, qc = 0;
+    // row constants (raw lse, D, keep word) of query tile t of a work item
+    auto row_consts = [&](int itm, int t, float& lse_, float& D_, uint32_t& bits_) {
+      const int kt_ = itm % nkt, ah_ = itm / nkt;
+      const int64_t hr = (int64_t(ah_ / p.heads) * p.heads + ah_ % p.heads) * S + t * 128 + i;
+      lse_ = p.lse[hr];
+      D_ = p.D[hr];
+      bits_ = p.drop ? p.mask[hr * (S / 32) + kt_ * 4 + cg] : ~0u;
+    };
+    float nlse = 0.f, nD = 0.f;
+    uint32_t nbits = ~0u;
+    if (int(blockIdx.x) < items) row_consts(blockIdx.x, 0, nlse, nD, nbits);
     for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
       const int kt = item % nkt, ah = item / nkt, a = ah % p.heads, b = ah / p.heads;
-      const int64_t hbase = (int64_t(b) * p.heads + a) * S;
-      // row constants of query tile t (lse, D, keep word), prefetched one tile ahead
-      auto row_consts = [&](int t, float& l2, float& D, uint32_t& bits) {
-        const int64_t hrow = hbase + t * 128 + i;
-        l2 = p.lse[hrow] * kLog2e;
-        D = p.D[hrow];
-        bits = p.drop ? p.mask[hrow * (S / 32) + kt * 4 + cg] : ~0u;
-      };
-      float nl2, nD;
-      uint32_t nbits;
-      row_consts(0, nl2, nD, nbits);
       for (int t = 0; t < nqt; ++t, ++qc) {
-        const float l2 = nl2, D = nD;
+        // this tile's constants were loaded one tile (or, for t = 0, one item) ahead; the
+        // raw lse is scaled only now, so no instruction waits on a load issued just before
+        const float l2 = nlse * kLog2e, D = nD;
         const uint32_t bits = nbits;
-        if (t + 1 < nqt) row_consts(t + 1, nl2, nD, nbits);
+        if (t + 1 < nqt) row_consts(item, t + 1, nlse, nD, nbits);
+        else if (item + int(gridDim.x) < items) row_consts(item + gridDim.x, 0, nlse, nD, nbits);
         mbar_wait(s_full, qc & 1);
         tc_fence_after();
         uint32_t rs[32], rp[32];
