@@ -284,6 +284,8 @@ def main():
     ap.add_argument("--budget-frac", type=float, default=None)
     ap.add_argument("--layers", type=int, default=LAYERS)
     ap.add_argument("--no-unbudgeted", action="store_true")
+    ap.add_argument("--no-plan-trial", action="store_true",
+                    help="take the measured-profile plan without the short trial against the analytic-profile plan")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--analytic-profile", action="store_true", help="plan with the analytic model, not measured times")
     args = ap.parse_args()
@@ -337,21 +339,42 @@ def main():
     t0 = time.time()
     blob, pcie, pst0 = None, None, None
     plan_profile = "measured (rank 0)"
+    plan_trials = {}
     if rank == 0:
         # profile every op (and split widths) on the GPU before planning
         prof = tsplit.Profile.measure(G, dev_inputs, max_p=4, device=local) if not args.analytic_profile else None
         pcie = prof.pcie() if prof else None
         plan_profile = "measured" if prof else "analytic"
-        try:
-            plan0 = tsplit.Plan.plan(G, budget, prof)
-        except tsplit.TsError as e:
-            # Alg. 2 is a path-dependent greedy heuristic: when the measured profile leads it
-            # into a dead end, plan with the analytic cost model instead (reported in config)
-            if prof is None or e.status != "ERR_INFEASIBLE":
-                raise
-            plan_profile = f"analytic (the measured-profile plan was infeasible: {str(e)[:80]})"
-            plan0 = tsplit.Plan.plan(G, budget, None)
-        pst0 = plan0.stats()  # predicted time with the measured profile
+        # Alg. 2 is a path-dependent greedy heuristic: plan with the measured profile and with
+        # the analytic cost model, then keep the candidate that runs faster in a short untimed
+        # trial (a dead end of one of them is reported in config)
+        cands = []
+        for label, pr in (("measured", prof), ("analytic", None)):
+            if label == "measured" and prof is None:
+                continue
+            try:
+                cands.append((label, tsplit.Plan.plan(G, budget, pr)))
+            except tsplit.TsError as e:
+                if e.status != "ERR_INFEASIBLE":
+                    raise
+                plan_trials[label] = f"infeasible: {str(e)[:80]}"
+        if not cands:
+            raise RuntimeError(f"no feasible plan: {plan_trials}")
+        if len(cands) > 1 and not args.no_plan_trial:
+            tstream = torch.cuda.Stream()
+            prm = gen.init_params(spec, seed=1)
+            for label, pl in cands:
+                s_ = tsplit.Session(G, pl, device=local, lr=1e-4,
+                                    streams=(tstream, torch.cuda.Stream(), torch.cuda.Stream()))
+                s_.set_params(prm)
+                for _ in range(2):
+                    s_.step(dev_inputs)
+                plan_trials[label] = round(time_steps(torch, s_, dev_inputs, tstream, 3) / 3 * 1e3, 2)
+                del s_
+                torch.cuda.empty_cache()
+            cands.sort(key=lambda c: plan_trials[c[0]])
+        plan_profile, plan0 = cands[0]
+        pst0 = plan0.stats()  # predicted time with the profile it was planned with
         blob = plan0.serialize()
     plan_s = time.time() - t0
     plan = tsplit.Plan.deserialize(G, bcast_bytes(blob))
@@ -462,6 +485,7 @@ def main():
                  "d2h_bytes": pst["d2h_bytes"], "h2d_bytes": pst["h2d_bytes"],
                  "step_flop": pst["compute_flop"], "predicted_ms": pst["predicted_s"] * 1e3,
                  "profile_and_planning_s": round(plan_s, 2), "planned_with": plan_profile,
+                 "plan_trial_ms_per_step": plan_trials or None,
                  "recompute_cache_bytes": pst["recompute_cache_bytes"],
                  "measured_pcie_gbs": [round(x / 1e9, 1) for x in pcie] if pcie else None},
         "l2": "no flush needed: every step streams >10 GB of activations through a 126 MB L2"

@@ -1478,7 +1478,13 @@ ts_status ts_profile_measure(const ts_graph_t* gh, void* slab, uint64_t slab_byt
     if (st != TS_OK) return st;
     st = ts_session_profile_items(s, 1);
     if (st == TS_OK) st = run_step(s, inputs, inputs_on_host);  // warm-up
-    if (st == TS_OK) st = run_step(s, inputs, inputs_on_host);  // timed
+    // three timed steps, per-item median: one step's clock / power state does not steer the
+    // planner (a noisy profile makes the greedy Alg. 2 land on different plans run to run)
+    std::vector<std::vector<float>> reps;
+    for (int r = 0; r < 3 && st == TS_OK; ++r) {
+      st = run_step(s, inputs, inputs_on_host);
+      if (st == TS_OK) reps.push_back(s->item_ms);
+    }
     if (st != TS_OK) {
       ts_session_destroy(s);
       return st;
@@ -1486,8 +1492,10 @@ ts_status ts_profile_measure(const ts_graph_t* gh, void* slab, uint64_t slab_byt
     std::vector<double> tf(g.ops.size(), 0.0), tb(g.ops.size(), 0.0);
     for (size_t i = 0; i < s->ex.items.size(); ++i) {
       const Item& it = s->ex.items[i];
-      if (it.kind == IT_F) tf[it.op] += 1e-3 * s->item_ms[i];
-      else if (it.kind == IT_B) tb[it.op] += 1e-3 * s->item_ms[i];
+      float v[3] = {reps[0][i], reps[1][i], reps[2][i]};
+      std::sort(v, v + 3);
+      if (it.kind == IT_F) tf[it.op] += 1e-3 * v[1];
+      else if (it.kind == IT_B) tb[it.op] += 1e-3 * v[1];
     }
     int l = 0;
     while ((1 << l) < p) ++l;
