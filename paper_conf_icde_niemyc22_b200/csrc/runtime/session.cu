@@ -205,6 +205,9 @@ std::function<void(cudaStream_t)> lower_linear_group(ts_session_t* s, const LinG
   };
 }
 
+// set while ts_profile_measure builds its sessions: lower every micro-op on its own
+thread_local bool g_profiling_session = false;
+
 // Lower one micro-op to kernel launches (DESIGN.md §3 op table).
 std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bwd, int& nk,
                                         const Fuse* fz = nullptr) {
@@ -749,7 +752,7 @@ ts_status build_program(ts_session_t* s) {
   std::set<int> fused_away;  // gelu items whose work the previous linear item's GEMM does
   // TSPLIT_NO_FUSION=1 lowers every micro-op on its own (tests compare the two programs)
   const char* nf = std::getenv("TSPLIT_NO_FUSION");
-  const bool fusion_on = !(nf && nf[0] == '1');
+  const bool fusion_on = !(nf && nf[0] == '1') && !g_profiling_session;
   // TSPLIT_NO_QKV_FUSION=1 keeps the linear + gelu fusion but lowers q/k/v one by one
   const char* nq = std::getenv("TSPLIT_NO_QKV_FUSION");
   const bool qkv_on = fusion_on && !(nq && nq[0] == '1');
@@ -1474,7 +1477,11 @@ ts_status ts_profile_measure(const ts_graph_t* gh, void* slab, uint64_t slab_byt
     sc.world_size = 1;
     sc.use_cuda_graph = 0;
     ts_session_t* s = nullptr;
+    // the profile times every op on its own (no fusion): a fused-away micro-op would read as
+    // free and the planner would recompute it without cost
+    g_profiling_session = true;
     ts_status st = ts_session_create(gh, &plan, &sc, &s);
+    g_profiling_session = false;
     if (st != TS_OK) return st;
     st = ts_session_profile_items(s, 1);
     if (st == TS_OK) st = run_step(s, inputs, inputs_on_host);  // warm-up
