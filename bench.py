@@ -422,7 +422,7 @@ def main():
     recs = sess.gemm_times()
     kinds = sess.gemm_kinds()
     sess.profile_items(False)
-    conv = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and kd > 0 and tc]
+    conv = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and kd > 0 and tc == 1]
     lin = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and bt == 1 and kd == 0 and tc]
     att = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and bt > 1 and tc]
     c_flop, c_ms = sum(f for f, _ in conv), sum(ms for _, ms in conv)
@@ -540,6 +540,17 @@ def main():
             "kernel": "gemm_tc on the fc layers", "launches": len(lin),
             "achieved_tflops": g_flop / (g_ms / 1e3) / 1e12 if g_ms > 0 else None,
             "share_of_step": g_ms / step_ms_prof if step_ms_prof else None}
+    # BASELINE metric part 2 (config 5): max trainable batch x hidden under the whole HBM, measured
+    # by tools/max_scale.py (planning up to 1024 x 512 tokens takes minutes, so not in this run)
+    msf = os.path.join(ROOT, "profiles", "r1_max_scale.json")
+    if not cnn and os.path.exists(msf):
+        ms = json.load(open(msf))
+        line["max_trainable"] = {
+            "source": "profiles/r1_max_scale.json (tools/max_scale.py, 24L s512 BERT, heads = h/64, capacity = "
+                      "free HBM - 6 GB; not re-measured in this run)",
+            "capacity_bytes": ms.get("capacity_bytes"),
+            "per_hidden": [{k: e.get(k) for k in ("hidden", "max_batch_unsplit", "max_batch_tsplit", "scale",
+                                                   "scale_unsplit", "samples_per_s")} for e in ms.get("summary", [])]}
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cnn_cpu_baseline(args.workload) if cnn else cpu_baseline_measure()
     print(json.dumps(line), flush=True)
