@@ -351,9 +351,7 @@ ts_status ts_gemm_f32(int32_t M, int32_t N, int32_t K,
  *   mode 3 wgrad: out = dw (fp32 [K,R,S,C]) (+)= sum over pixels of dy (x) im2col(x)
  * dtype TS_BF16: tcgen05/TMEM implicit GEMM with cp.async gathers (fp32 accumulate)
  * when eligible (K % 8 == 0; dgrad also C % 8 == 0), else CUDA cores; TS_F32: CUDA
- * cores with fp64 accumulation.  *used_tc (may be NULL) reports the path taken: 1 tcgen05,
- * 2 the direct CUDA-core image-layer kernels (bf16, C <= 4, K % 64 == 0, fprop / wgrad:
- * the input patch in shared memory, 8 pixels x 1 channel per thread), 0 SIMT.
+ * cores with fp64 accumulation.  *used_tc (may be NULL) reports the path taken.
  * Layers with C % 64 == 0, K % 64 == 0 and stride <= 2 take the TMA-fed kernel
  * (spatial-box M tiles); mode | 0x10 forces the cp.async gather kernel (tests).
  * Errors: TS_ERR_ARG for bad geometry, TS_ERR_CUDA for launch failures. */

@@ -643,8 +643,7 @@ void record(int kind, const ConvArgs& a, cudaStream_t st, int tc, GemmRecord& re
 void conv_run(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st) {
   GemmRecord rec{};
   record(mode, a, st, 0, rec, true);
-  // 1 = tcgen05 implicit GEMM, 2 = direct image-layer kernel, 0 = fp32 / fallback SIMT
-  int tc = conv_direct(mode, a, out, bias, acc, st) ? 2 : (conv_tc(mode, a, out, bias, acc, st) ? 1 : 0);
+  int tc = conv_tc(mode, a, out, bias, acc, st) ? 1 : 0;
   if (!tc) conv_simt(mode, a, out, bias, acc, st);
   record(mode, a, st, tc, rec, false);
 }

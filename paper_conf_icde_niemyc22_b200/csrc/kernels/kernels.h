@@ -100,8 +100,6 @@ bool conv_tma(int mode, const ConvArgs& a, void* out, const void* bias, int acc,
 // the cp.async gather kernel alone (tests; conv_tc tries conv_tma first)
 bool conv_gather(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
 void conv_simt(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
-// direct CUDA-core kernels for the image layer (bf16, C <= 4, K % 64 == 0; fprop and wgrad)
-bool conv_direct(int mode, const ConvArgs& a, void* out, const void* bias, int acc, cudaStream_t st);
 
 // ---- batch normalisation over all pieces of a split tensor ----------
 // A piece list: `np` pointers, each holding `rows[i]` rows of C channels.

@@ -1694,9 +1694,7 @@ ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   int tc = 0;
   if (a.dtype == tsk::BF16)
-    tc = gather_only ? (tsk::conv_gather(mode, a, out, bias, acc, st) ? 1 : 0)
-                     : tsk::conv_direct(mode, a, out, bias, acc, st) ? 2
-                     : (tsk::conv_tc(mode, a, out, bias, acc, st) ? 1 : 0);
+    tc = (gather_only ? tsk::conv_gather(mode, a, out, bias, acc, st) : tsk::conv_tc(mode, a, out, bias, acc, st)) ? 1 : 0;
   if (!tc) tsk::conv_simt(mode, a, out, bias, acc, st);
   CU(cudaGetLastError());
   if (used_tc) *used_tc = tc;

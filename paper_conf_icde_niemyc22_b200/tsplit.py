@@ -544,8 +544,8 @@ def nccl_comm(rank: int, world: int, broadcast):
 def conv2d(mode: int, geom, x, w, dy, out, bias=None, acc: int = 0, stream=None) -> bool:
     """Run one conv micro-op kernel through the C ABI (`ts_conv2d`, include/ts.h) on
     torch device tensors (argument marshalling only).  mode 1 fprop -> out = y,
-    2 dgrad -> out = dx, 3 wgrad -> out = dw (fp32).  Returns the path taken: 1 (truthy)
-    tcgen05 implicit GEMM, 2 the direct image-layer kernels (C <= 4), 0 CUDA-core SIMT."""
+    2 dgrad -> out = dx, 3 wgrad -> out = dw (fp32).  Returns True when the tcgen05
+    implicit-GEMM path ran."""
     import torch
     dt = DTYPES["bf16"] if w.dtype == torch.bfloat16 else DTYPES["f32"]
     g = (C.c_int32 * 9)(*[int(v) for v in geom])
@@ -553,7 +553,7 @@ def conv2d(mode: int, geom, x, w, dy, out, bias=None, acc: int = 0, stream=None)
     used = C.c_int32(0)
     st = C.c_void_p(stream if stream is not None else torch.cuda.current_stream().cuda_stream)
     check(lib().ts_conv2d(mode, dt, g, ptr(x), ptr(w), ptr(dy), ptr(out), ptr(bias), acc, st, C.byref(used)))
-    return int(used.value)
+    return bool(used.value)
 
 
 def attention(mode: int, geom, alpha: float, p: float, q, k, v, c=None, lse=None, dc=None, dq=None, dk=None,
