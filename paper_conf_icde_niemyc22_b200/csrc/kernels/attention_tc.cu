@@ -297,17 +297,28 @@ __global__ void __launch_bounds__(kDqThreads, 1)
       lse_ = p.lse[hr];
     };
     float nD = 0.f, nlse = 0.f;
-    if (int(blockIdx.x) < items) item_consts(blockIdx.x, nD, nlse);
+    // keep word of (item, key tile kt) for this row and 32-key group, loaded a tile ahead
+    auto keep_word = [&](int itm, int kt_) -> uint32_t {
+      if (!p.drop) return ~0u;
+      const int qt_ = itm % nqt, ah_ = itm / nqt;
+      const int64_t hr = (int64_t(ah_ / p.heads) * p.heads + ah_ % p.heads) * S + qt_ * 128 + i;
+      return p.mask[hr * (S / 32) + kt_ * 4 + cg];
+    };
+    uint32_t nbits = ~0u;
+    if (int(blockIdx.x) < items) {
+      item_consts(blockIdx.x, nD, nlse);
+      nbits = keep_word(blockIdx.x, 0);
+    }
     for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
       const int qt = item % nqt, ah = item / nqt, a = ah % p.heads, b = ah / p.heads;
       const int q = qt * 128 + i;
-      const int64_t hrow = (int64_t(b) * p.heads + a) * S + q;
       const float D = nD;
       const float l2 = nlse * kLog2e;
       if (item + int(gridDim.x) < items) item_consts(item + gridDim.x, nD, nlse);
-      const uint32_t* mrow = p.mask + hrow * (S / 32);
       for (int kt = 0; kt < nkt; ++kt, ++kc) {
-        const uint32_t bits = p.drop ? mrow[kt * 4 + cg] : ~0u;
+        const uint32_t bits = nbits;
+        if (kt + 1 < nkt) nbits = keep_word(item, kt + 1);
+        else if (item + int(gridDim.x) < items) nbits = keep_word(item + gridDim.x, 0);
         mbar_wait(s_full, kc & 1);
         tc_fence_after();
         uint32_t rs[32], rp[32];
