@@ -551,6 +551,14 @@ def main():
             "capacity_bytes": ms.get("capacity_bytes"),
             "per_hidden": [{k: e.get(k) for k in ("hidden", "max_batch_unsplit", "max_batch_tsplit", "scale",
                                                    "scale_unsplit", "samples_per_s")} for e in ms.get("summary", [])]}
+    if not cnn:
+        # north_star: the paper's ratios, quoted with the GPU PAPER.md names — context only
+        line["paper_context"] = {
+            "gpu": "NVIDIA TITAN RTX (24 GB), FP32 (PAPER.md L8, L46, L450; BASELINE.md)",
+            "max_model_scale_vs_vdnn": 10.5, "max_model_scale_vs_superneurons": 3.1,
+            "throughput_vs_vdnn": 4.7, "throughput_vs_superneurons": 2.7,
+            "note": "comparison systems are out of scope here; this run's own scale ratio is "
+                    "max_trainable (TSPLIT vs unsplit on the same B200)"}
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cnn_cpu_baseline(args.workload) if cnn else cpu_baseline_measure()
     print(json.dumps(line), flush=True)
