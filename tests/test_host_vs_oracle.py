@@ -276,3 +276,17 @@ def test_planner_uses_channel_splits_when_the_batch_is_one(frac):
     assert abs(l1 - l0) <= 1e-12 * abs(l0)
     from test_oracle_net_sim import rel_errs
     assert max(rel_errs(g1, g0).values()) <= 1e-12
+
+
+def test_channel_plan_serialize_roundtrip():
+    """A channel-split plan (D-CH) survives ts_plan_serialize / _deserialize (the DP
+    broadcast): same per-tensor dims and the same trace."""
+    g = graphs.config_graph("bert_tiny")
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    G = tsplit.Graph(g)
+    P = tsplit.Plan.default(G)
+    P.set_many({names["l0.ffn1"]: (2, 4, 1, 1), names["l0.gelu"]: (1, 4, 3, 1), names["l1.q"]: (2, 2, 1, 0)})
+    Q = tsplit.Plan.deserialize(G, P.serialize())
+    assert Q.trace() == P.trace()
+    for t in brute.act_tensors(g):
+        assert (Q.get(t), Q.get_dim(t)) == (P.get(t), P.get_dim(t))
