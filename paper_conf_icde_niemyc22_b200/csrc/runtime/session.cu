@@ -921,7 +921,9 @@ ts_status build_program(ts_session_t* s) {
         for (size_t j = i + 1; j < s->ex.items.size() && sib.size() + 1 < size_t(tsk::kMaxGroups); ++j) {
           const Item& nx = s->ex.items[j];
           const Op& no = g.ops[nx.op];
-          if (nx.kind != it.kind || nx.k != it.k || nx.group != it.group || s->ex.P[nx.op] != m.P) break;
+          // (every backward micro-op is its own group; consecutive B items have no replay between)
+          if (nx.kind != it.kind || nx.k != it.k || s->ex.P[nx.op] != m.P) break;
+          if (it.kind != IT_B && nx.group != it.group) break;
           if (no.kind != TS_OP_LINEAR || no.in[0] != o.in[0] || nx.op == it.op || op_chan(nx.op)) break;
           if (g.t[no.in[1]].shape[0] != N0 || g.t[no.in[1]].shape[1] != K0) break;
           if (!s->sim.wait_so[j].empty()) break;
@@ -989,7 +991,8 @@ ts_status build_program(ts_session_t* s) {
           !op_chan(s->ex.items[i + 1].op)) {
         const Item& nx = s->ex.items[i + 1];
         const Op& go = g.ops[nx.op];
-        const bool same = nx.kind == it.kind && nx.k == it.k && s->ex.P[nx.op] == m.P && nx.group == it.group &&
+        const bool same = nx.kind == it.kind && nx.k == it.k && s->ex.P[nx.op] == m.P &&
+                          (it.kind == IT_B || nx.group == it.group) &&
                           go.kind == TS_OP_GELU && s->sim.wait_so[i + 1].empty();
         // `ok_key`: a tensor freed after this item that the fused product may overwrite because
         // its last reader runs first (backward: the gelu output H, read only by the dW product)

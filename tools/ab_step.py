@@ -15,9 +15,8 @@ from paper_conf_icde_niemyc22_b200 import tsplit  # noqa: E402
 from tsinputs import gen, graphs  # noqa: E402
 
 VARIANTS = {
-    "base(cta1,noqkv)": ({"TSPLIT_NO_QKV_FUSION": "1"}, 1),
-    "pair,noqkv": ({"TSPLIT_NO_QKV_FUSION": "1"}, 0),
-    "pair,qkv": ({}, 0),
+    "nofusion": ({"TSPLIT_NO_FUSION": "1"}, 0),
+    "fusion": ({}, 0),
 }
 
 
