@@ -639,12 +639,19 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
       if (cg == 2 && bn < 128) continue;
       const double eff = cg == 2 ? (bn == 256 ? 0.97 : 0.60) : (bn == 256 ? 0.90 : bn == 128 ? 0.65 : 0.45);
       int64_t tiles = int64_t((g.M + BM * cg - 1) / (BM * cg)) * ((g.N + bn - 1) / bn) * g.nb1 * g.nb2;
-      int ks = 1;
-      if (splitk_ok && tiles * 2 <= slots && num_kb_all >= 16) {
-        ks = int(slots / tiles);
-        if (ks > num_kb_all / 8) ks = num_kb_all / 8;
-        if (ks < 1) ks = 1;
+      // split-K: the widest split that still fills the machine when there are few tiles, plus
+      // small splits (2..8) that even out a partial last wave (e.g. q/k/v dW: 48 pair tiles on
+      // 74 slots -> 3 splits, two full waves); fp32, unbatched C only (partials reduce-added)
+      int ks_cands[10], nks = 0;
+      ks_cands[nks++] = 1;
+      // (only when one wave of whole tiles leaves over a quarter of the machine idle: measured,
+      // splitting 64 pair tiles on 74 slots (86 %) costs 13 % on the FFN dW products)
+      if (splitk_ok && num_kb_all >= 16 && tiles * 4 < int64_t(slots) * 3) {
+        if (tiles * 2 <= slots) ks_cands[nks++] = std::max(1, std::min(int(slots / tiles), num_kb_all / 8));
+        for (int k2 = 2; k2 <= 8 && k2 <= num_kb_all / 8; ++k2) ks_cands[nks++] = k2;
       }
+      for (int ci = 0; ci < nks; ++ci) {
+      const int ks = ks_cands[ci];
       int64_t units = tiles * ks;
       double waves = double((units + slots - 1) / slots);
       // a tail wave at most half full runs as half-width units (decode_unit)
@@ -652,14 +659,15 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
           2 * (tiles % slots) <= slots)
         waves -= 0.5;
       // time in (tile-width x k-block) units, + the pair's fixed cost (~4 k-blocks of a
-      // 256-wide tile, fitted to the BERT micro-op shapes)
+      // 256-wide tile, fitted to the BERT micro-op shapes), + the partial-tile reduce-adds
       const int kb_unit = (num_kb_all + ks - 1) / ks;
-      double cost = waves * (bn / eff) * kb_unit + (cg == 2 ? 1024.0 : 0.0);
+      double cost = waves * (bn / eff) * kb_unit + (cg == 2 ? 1024.0 : 0.0) + (ks > 1 ? 256.0 * ks : 0.0);
       if (cost < best - 1e-9) {
         best = cost;
         best_bn = bn;
         best_ks = ks;
         best_cg = cg;
+      }
       }
     }
   }

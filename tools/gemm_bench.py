@@ -78,6 +78,7 @@ if __name__ == "__main__":
     res.append(case("ffn1 dW", F, H, T, 1, 1, out="f32", beta=1.0))
     res.append(case("ffn2 dW", H, F, T, 1, 1, out="f32", beta=1.0))
     res.append(case("p=4 ffn1 fwd", T // 4, F, H, 0, 0))
+    res.append(case("qkv dW grouped-size", 3 * H, H, T, 1, 1, out="f32", beta=1.0))
     res.append(case("p=2 qkv fwd", T // 2, H, H, 0, 0))
     res.append(case("p=4 qkv fwd", T // 4, H, H, 0, 0))
     res.append(case("p=4 ffn2 fwd", T // 4, H, F, 0, 0))
