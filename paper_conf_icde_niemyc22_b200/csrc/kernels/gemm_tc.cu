@@ -778,10 +778,10 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
       if (best_bn == 256) launch<256, true, 8, 2>(tm, p, st);
       else launch<128, true, 8, 2>(tm, p, st);
     } else if (best_bn == 256) {
-      if (p.epi == 1) launch<256, false, 16, 2>(tm, p, st);
+      if (p.epi) launch<256, false, 16, 2>(tm, p, st);
       else launch<256, false, 8, 2>(tm, p, st);
     } else {
-      if (p.epi == 1) launch<128, false, 16, 2>(tm, p, st);
+      if (p.epi) launch<128, false, 16, 2>(tm, p, st);
       else launch<128, false, 8, 2>(tm, p, st);
     }
     return true;
@@ -795,7 +795,7 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
   } else {
     switch (best_bn) {
       case 256:
-        if (p.epi == 1) launch<256, false, 16>(tm, p, st);
+        if (p.epi) launch<256, false, 16>(tm, p, st);
         else launch<256, false>(tm, p, st);
         break;
       case 128: launch<128, false>(tm, p, st); break;
