@@ -1031,6 +1031,14 @@ ts_status build_program(ts_session_t* s) {
             fz.u = view(u);
           }
         }
+        static const bool flog = std::getenv("TSPLIT_FUSION_LOG") != nullptr;
+        if (flog && bwd && go.kind == TS_OP_GELU && go.out[0] == o.in[0]) {
+          uint64_t o2 = 0, b2 = 0;
+          std::fprintf(stderr, "fuse-bwd item %zu op %d: same %d acc %d first %d free %d where %d -> mode %d\n", i, it.op,
+                       int(same), m.acc.count(n + o.in[0]) ? m.acc.at(n + o.in[0]) : -1,
+                       int(grad_first_op.count(n + go.in[0])), int(free_while_here(n + go.in[0], o2, b2, o.in[0])),
+                       int(where.count(pk(go.in[0], int(m.s0 * piece_count(g, s->cfg, go.in[0]) / B)))), fz.mode);
+        }
       }
       int nk = 0;
       if (lg.G) {
