@@ -267,3 +267,19 @@ def test_lru_recompute_cache_session(cache):
     assert max(rel_errs(out[1][1], out[0][1]).values()) <= 1e-6
     ol, og = _oracle(g)
     assert max(rel_errs(out[1][1], og).values()) <= 1e-5
+
+
+@pytest.mark.parametrize("hidden", [512, 1024])
+def test_bert_wide_hidden_bf16_parity(hidden):
+    """Row kernels at BERT-Large widths (LayerNorm fwd/bwd with 2 / 4 sixteen-byte chunks per
+    lane, fused bias / LN-gradient partials) through a whole bf16 step, split + recompute,
+    against the oracle's bf16-storage reading (D-TOL)."""
+    g = graphs.bert(layers=1, hidden=hidden, heads=hidden // 64, seq=128, batch=4, vocab=512, fused_attention=True)
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    cfg = {names["l0.ln1"]: (tsplit.RECOMPUTE, 2, 1), names["l0.ffn1"]: (tsplit.RESIDE, 2, 1)}
+    loss, grads, S, P = _run(g, cfg)
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    _, ogb, _, _ = net.train_step(g, params, inputs, storage="bf16")
+    assert global_rel_err(grads, ogb) <= 2e-2
+    errs = rel_errs(grads, ogb)
+    assert errs["l0.ln1.g"] <= 2e-2 and errs["l0.ln2.g"] <= 2e-2, errs
