@@ -11,17 +11,22 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, gname="bert_tiny"):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         from paper_conf_icde_niemyc22_b200 import tsplit
         from tsinputs import graphs
-        g = graphs.config_graph("bert_tiny")
+        if gname == "mlp_b1":  # batch 1: the planner splits channels (reading D-CH)
+            g = graphs.mlp(batch=1, in_dim=64, hidden=2048, depth=3, classes=10)
+            base = tsplit.Plan.default(tsplit.Graph(g)).stats()
+            budget = base["static_bytes"] + (base["peak_extent"] - base["static_bytes"]) * 3 // 4
+        else:
+            g = graphs.config_graph("bert_tiny")
+            base = tsplit.Plan.default(tsplit.Graph(g)).stats()
+            budget = base["static_bytes"] + (base["peak_extent"] - base["static_bytes"]) // 3
         G = tsplit.Graph(g)
-        base = tsplit.Plan.default(G).stats()
-        budget = base["static_bytes"] + (base["peak_extent"] - base["static_bytes"]) // 3
         blob = tsplit.Plan.plan(G, budget).serialize() if rank == 0 else None
         obj = [blob]
         dist.broadcast_object_list(obj, src=0)
@@ -38,23 +43,27 @@ def _worker(rank, world, port, q):
         # max-over-ranks step time (bench.py reduction)
         t = torch.tensor([0.1 * (rank + 1)], dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        q.put((rank, [int(x.item()) for x in gathered], float(t.item()), plan.stats()["peak_extent"] <= budget))
+        dims = sorted({plan.get_dim(t["id"]) for t in g["tensors"] if t["kind"] == "act"})
+        q.put((rank, [int(x.item()) for x in gathered], float(t.item()), plan.stats()["peak_extent"] <= budget, dims))
     finally:
         dist.destroy_process_group()
 
 
-def test_plan_broadcast_world2():
+@pytest.mark.parametrize("gname", ["bert_tiny", "mlp_b1"])
+def test_plan_broadcast_world2(gname):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    port = 29500 + (os.getpid() % 1000)
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    port = 29500 + (os.getpid() % 1000) + (7 if gname == "mlp_b1" else 0)
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q, gname)) for r in range(2)]
     for p in procs:
         p.start()
     res = [q.get(timeout=120) for _ in procs]
     for p in procs:
         p.join(timeout=60)
         assert p.exitcode == 0
-    for rank, digests, tmax, fits in res:
+    for rank, digests, tmax, fits, dims in res:
         assert len(set(digests)) == 1, digests
         assert tmax == pytest.approx(0.2)
         assert fits
+        if gname == "mlp_b1":
+            assert 1 in dims  # the broadcast plan carries the channel dim
