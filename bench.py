@@ -348,16 +348,13 @@ def main():
         # Alg. 2 is a path-dependent greedy heuristic: plan with the measured profile and with
         # the analytic cost model, then keep the candidate that runs faster in a short untimed
         # trial (a dead end of one of them is reported in config)
-        # (the third candidate is Alg. 2 without split proposals, "TSPLIT w/o Split" of P:L463:
-        # at batch 32 the greedy can take split decisions early that its own timeline later
-        # rates slower — profiles/r1_ablation_bert_large.json — while at larger batches
-        # splitting wins)
+        # (ts_plan itself keeps the faster of Alg. 2 with and without split proposals)
         cands = []
-        for label, pr, ns in (("measured", prof, False), ("analytic", None, False), ("measured_no_split", prof, True)):
+        for label, pr in (("measured", prof), ("analytic", None)):
             if pr is None and label != "analytic":
                 continue
             try:
-                cands.append((label, tsplit.Plan.plan(G, budget, pr, no_split=ns)))
+                cands.append((label, tsplit.Plan.plan(G, budget, pr)))
             except tsplit.TsError as e:
                 if e.status != "ERR_INFEASIBLE":
                     raise

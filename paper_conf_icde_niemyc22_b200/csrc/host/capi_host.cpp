@@ -117,6 +117,16 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
   }
   if (st == TS_ERR_INFEASIBLE) set_error(first_error);
   if (st != TS_OK) return st;
+  // The greedy takes split proposals wherever their local dT/dM ratio is best, which can lock
+  // it into a plan its own timeline rates slower than the one it finds without them
+  // (profiles/r1_ablation_bert_large.json: BERT-Large b32 at 25 %).  The full planner's
+  // search space contains the "w/o Split" plan, so keep whichever predicts faster.
+  if (!(flags & TS_PLAN_NO_SPLIT)) {
+    PlanState alt;
+    if (plan_greedy(g->g, budget_bytes, *pr, alt, flags | TS_PLAN_NO_SPLIT) == TS_OK &&
+        alt.predicted_s < p->st.predicted_s)
+      p->st = std::move(alt);
+  }
   p->budget = budget_bytes;
   *out = p.release();
   return TS_OK;
