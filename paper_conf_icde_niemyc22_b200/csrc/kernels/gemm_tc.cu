@@ -434,6 +434,21 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
 #pragma unroll
                 for (int i = 0; i < 32; ++i) v[i] = gelu_f(bf16_round(v[i]));
                 stage_store(v, &tm.c2, false);
+              } else if (p.epi == 3) {  // second output: bf16(U) + residual, as the add kernel rounds
+                const bf16* rp = p.aux + int64_t(row) * p.ldaux + col0;
+                if (row_ok && full_chunk) {
+                  uint4 u[4];
+#pragma unroll
+                  for (int j = 0; j < 4; ++j) u[j] = __ldg(reinterpret_cast<const uint4*>(rp) + j);
+                  const bf16* rb = reinterpret_cast<const bf16*>(u);
+#pragma unroll
+                  for (int i = 0; i < 32; ++i) v[i] = bf16_round(v[i]) + to_f(rb[i]);
+                } else {
+#pragma unroll
+                  for (int i = 0; i < 32; ++i)
+                    v[i] = bf16_round(v[i]) + ((row_ok && col0 + i < p.N) ? to_f(rp[i]) : 0.f);
+                }
+                stage_store(v, &tm.c2, false);
               }
             }
           } else if (row_ok) {
@@ -741,6 +756,10 @@ bool gemm_tc(const GemmArgs& g, cudaStream_t st) {
                                 CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, CU_TENSOR_MAP_SWIZZLE_64B))
       return false;
     if (g.epi == 2 && ((reinterpret_cast<uintptr_t>(g.aux) | uintptr_t(g.ldaux * 2)) & 15)) return false;
+    if (g.epi == 3 && (((reinterpret_cast<uintptr_t>(g.aux) | uintptr_t(g.ldaux * 2)) & 15) || !g.aux2 ||
+                       !make_map(&tm.c2, g.aux2, g.ldaux2, 0, 0, g.N, g.M, 1, 1, 32, 32, 2,
+                                 CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, CU_TENSOR_MAP_SWIZZLE_64B)))
+      return false;
     if (g.nb1 * g.nb2 != 1) return false;
   }
   // beta = 1 accumulates with a TMA reduce-add of the new tile (fp32, or bf16 gradients that
@@ -845,6 +864,7 @@ void gemm(const GemmArgs& g, cudaStream_t st) {
     // the fused epilogue's effect, unfused: gelu of the stored U / dU = dH * gelu'(U) in place
     if (g.epi == 1) gelu_fwd(BF16, g.c, g.aux, int64_t(g.M) * g.N, st);
     if (g.epi == 2) gelu_bwd(BF16, g.c, g.aux, g.c, 0, int64_t(g.M) * g.N, st);
+    if (g.epi == 3) add_fwd(BF16, g.c, g.aux, g.aux2, int64_t(g.M) * g.N, st);
   }
   if (g_sink) {
     cudaEventRecord(rec.stop, st);

@@ -35,9 +35,13 @@ struct GemmArgs {
   // aux = gelu(U) (the linear -> gelu pair of one micro-op); 2 = GELU backward, C = dU =
   // bf16(alpha AB) * gelu'(aux) with aux = U (the dX product of the layer after a gelu).
   // Values pass through bf16 exactly where the separate kernels would store them.
+  // 3 = residual add, C = U = alpha AB + bias and aux2 = bf16(U) + aux (the linear -> add
+  // pair whose add reads the linear's output and a residual aux, e.g. res1 = proj + x).
   int epi = 0;
   void* aux = nullptr;
   int64_t ldaux = 0;
+  void* aux2 = nullptr;  // epi 3 output (row-major, leading dimension ldaux2)
+  int64_t ldaux2 = 0;
   // grouped product (tcgen05 path only, unbatched, epi 0, beta 0 or 1): `groups` equal
   // slices along gdim, M/N/K being the totals.  gdim 1 (N): C_g = A B_g^T + bias_g, per
   // group bg/cg/biasg, shared a; gdim 2 (K): C = sum_g A_g B_g^T, per group ag/bg, shared

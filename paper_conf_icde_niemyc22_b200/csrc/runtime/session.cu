@@ -125,10 +125,11 @@ struct Micro {
 // decides when it is safe): mode 1 = forward, the GEMM epilogue also writes gelu(U) to `y`;
 // mode 2 = backward, the dX product writes dU = dH * gelu'(U) to `du` (reading `u`) instead of dH.
 struct Fuse {
-  int mode = 0;
+  int mode = 0;  // 1 gelu forward, 2 gelu backward, 3 residual add (D-FUSE)
   char* y = nullptr;
   char* du = nullptr;
   char* u = nullptr;
+  char* r = nullptr;  // mode 3: the add's other input
 };
 
 // Horizontal fusion (reading D-QKV): G consecutive linear micro-ops of one kind over the
@@ -296,6 +297,9 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
         a.bias = param_w(s, bb); a.bias_dtype = dt;
         if (fz && fz->mode == 1) {
           a.epi = 1; a.aux = fz->y; a.ldaux = N;
+        }
+        if (fz && fz->mode == 3) {
+          a.epi = 3; a.aux = fz->r; a.ldaux = N; a.aux2 = fz->y; a.ldaux2 = N;
         }
         nk = 1;
         return [a](cudaStream_t st) { tsk::gemm(a, st); };
@@ -991,9 +995,9 @@ ts_status build_program(ts_session_t* s) {
           !op_chan(s->ex.items[i + 1].op)) {
         const Item& nx = s->ex.items[i + 1];
         const Op& go = g.ops[nx.op];
-        const bool same = nx.kind == it.kind && nx.k == it.k && s->ex.P[nx.op] == m.P &&
-                          (it.kind == IT_B || nx.group == it.group) &&
-                          go.kind == TS_OP_GELU && s->sim.wait_so[i + 1].empty();
+        const bool adjacent = nx.kind == it.kind && nx.k == it.k && s->ex.P[nx.op] == m.P &&
+                              (it.kind == IT_B || nx.group == it.group) && s->sim.wait_so[i + 1].empty();
+        const bool same = adjacent && go.kind == TS_OP_GELU;
         // `ok_key`: a tensor freed after this item that the fused product may overwrite because
         // its last reader runs first (backward: the gelu output H, read only by the dW product)
         auto free_while_here = [&](int key, uint64_t& off, uint64_t& bytes, int ok_key) -> bool {
@@ -1016,7 +1020,21 @@ ts_status build_program(ts_session_t* s) {
           return s->slab + piece_off + (m.s0 - first) * x.elems_per_sample * es;
         };
         uint64_t off = 0, bytes = 0;
-        if (same && !bwd && go.in[0] == o.out[0] && free_while_here(go.out[0], off, bytes, -1)) {
+        // linear -> add (res = Y + residual): the add's output comes from the GEMM epilogue (mode 3);
+        // the linear's own output is still written, so any later reader of it is unaffected
+        const int res_in = (go.kind == TS_OP_ADD && go.in.size() == 2)
+                               ? (go.in[0] == o.out[0] ? go.in[1] : (go.in[1] == o.out[0] ? go.in[0] : -1))
+                               : -1;
+        if (adjacent && !bwd && res_in >= 0 && res_in != o.out[0] && g.t[res_in].sample &&
+            g.t[go.out[0]].numel == g.t[o.out[0]].numel && free_while_here(go.out[0], off, bytes, -1)) {
+          const int pr = piece_count(g, s->cfg, res_in);
+          const PieceKey rpc = pk(res_in, int(m.s0 * pr / B));
+          if (where.count(rpc) && !si_live.count(rpc)) {
+            fz.mode = 3;
+            fz.y = sub_view(go.out[0], off);
+            fz.r = view(res_in);
+          }
+        } else if (same && !bwd && go.in[0] == o.out[0] && free_while_here(go.out[0], off, bytes, -1)) {
           fz.mode = 1;
           fz.y = sub_view(go.out[0], off);
         } else if (same && bwd && go.out[0] == o.in[0] && g.t[go.out[0]].consumers.size() == 1 &&
