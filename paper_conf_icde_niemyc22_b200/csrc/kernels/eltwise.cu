@@ -211,6 +211,50 @@ void add_fwd(int dt, const void* a, const void* b, void* y, int64_t n, cudaStrea
 void axpy(int dt, const void* dy, void* dx, int acc, int64_t n, cudaStream_t st) {
   ew<AXPY>(dt, dy, nullptr, dx, n, acc, kNoP, st);
 }
+
+namespace {
+// add backward: dy passes to both inputs' gradients (each overwritten or accumulated), dy read once
+template <class T>
+__global__ void __launch_bounds__(256) axpy2_kernel(const T* __restrict__ dy, T* d1, int acc1, T* d2, int acc2,
+                                                    int64_t n) {
+  constexpr int V = 16 / sizeof(T);
+  const int64_t nv = n / V, stride = int64_t(gridDim.x) * blockDim.x;
+  for (int64_t v = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; v < nv; v += stride) {
+    T g[V], o1[V], o2[V];
+    *reinterpret_cast<uint4*>(g) = reinterpret_cast<const uint4*>(dy)[v];
+    if (acc1) *reinterpret_cast<uint4*>(o1) = reinterpret_cast<const uint4*>(d1)[v];
+    if (acc2) *reinterpret_cast<uint4*>(o2) = reinterpret_cast<const uint4*>(d2)[v];
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+      o1[i] = acc1 ? from_f<T>(to_f(g[i]) + to_f(o1[i])) : g[i];
+      o2[i] = acc2 ? from_f<T>(to_f(g[i]) + to_f(o2[i])) : g[i];
+    }
+    reinterpret_cast<uint4*>(d1)[v] = *reinterpret_cast<uint4*>(o1);
+    reinterpret_cast<uint4*>(d2)[v] = *reinterpret_cast<uint4*>(o2);
+  }
+  for (int64_t i = nv * V + int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += stride) {
+    const float gv = to_f(dy[i]);
+    d1[i] = acc1 ? from_f<T>(gv + to_f(d1[i])) : dy[i];
+    d2[i] = acc2 ? from_f<T>(gv + to_f(d2[i])) : dy[i];
+  }
+}
+}  // namespace
+
+void axpy2(int dt, const void* dy, void* d1, int acc1, void* d2, int acc2, int64_t n, cudaStream_t st) {
+  const bool aligned = ((reinterpret_cast<uintptr_t>(dy) | reinterpret_cast<uintptr_t>(d1) |
+                         reinterpret_cast<uintptr_t>(d2)) & 15) == 0;
+  if (!aligned || n <= 0) {  // rare: two single-output passes
+    axpy(dt, dy, d1, acc1, n, st);
+    axpy(dt, dy, d2, acc2, n, st);
+    return;
+  }
+  const int64_t work = n / (dt == F32 ? 4 : 8) + 1;
+  const int grid = int(work / 256 + 1 < 148 * 8 ? work / 256 + 1 : 148 * 8);
+  if (dt == F32)
+    axpy2_kernel<float><<<grid, 256, 0, st>>>((const float*)dy, (float*)d1, acc1, (float*)d2, acc2, n);
+  else
+    axpy2_kernel<bf16><<<grid, 256, 0, st>>>((const bf16*)dy, (bf16*)d1, acc1, (bf16*)d2, acc2, n);
+}
 void dropout(int dt, const void* x, void* y, int acc, int64_t n, int64_t elem0, float p, uint32_t seed,
              uint32_t step, cudaStream_t st) {
   EwP q;

@@ -177,6 +177,8 @@ void tanh_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t 
 void add_fwd(int dt, const void* a, const void* b, void* y, int64_t n, cudaStream_t st);
 // dx (+)= scale * dy (acc: accumulate into dx)
 void axpy(int dt, const void* dy, void* dx, int acc, int64_t n, cudaStream_t st);
+// add backward: d1 (+)= dy and d2 (+)= dy in one pass (acc flags per output)
+void axpy2(int dt, const void* dy, void* d1, int acc1, void* d2, int acc2, int64_t n, cudaStream_t st);
 void dropout(int dt, const void* x, void* y, int acc, int64_t n, int64_t elem0, float p, uint32_t seed,
              uint32_t step, cudaStream_t st);
 // ---- row ops -----------------------------------------------------------------

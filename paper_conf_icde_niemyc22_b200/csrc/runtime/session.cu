@@ -389,9 +389,12 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
         const Tensor& x = g.t[o.in[i]];
         if (x.kind == TS_ACT && x.needs_grad) outs.push_back({G(o.in[i]), A(g.n() + o.in[i])});
       }
-      nk = int(outs.size());
+      nk = outs.size() == 2 ? 1 : int(outs.size());
       return [=](cudaStream_t st) {
-        for (auto& pr : outs) tsk::axpy(dt, dy, pr.first, pr.second, n_out, st);
+        if (outs.size() == 2 && outs[0].first != outs[1].first)
+          tsk::axpy2(dt, dy, outs[0].first, outs[0].second, outs[1].first, outs[1].second, n_out, st);
+        else
+          for (auto& pr : outs) tsk::axpy(dt, dy, pr.first, pr.second, n_out, st);
       };
     }
     case TS_OP_DROPOUT: {
