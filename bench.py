@@ -420,6 +420,13 @@ def main():
     sess.profile_items(True)
     sess.step(dev_inputs)
     item_ms = sess.item_times()
+    # fused attention micro-ops: summed event times of the forward (F), replay (R) and backward (B)
+    # items of the profiled step
+    att_ms = {"F": 0.0, "R": 0.0, "B": 0.0}
+    if not (args.workload != "bert_large") and args.attention == "fused":
+        for (kind, op, k, aux), t in zip(plan.items(), item_ms):
+            if op >= 0 and kind in att_ms and spec["ops"][op]["kind"] == "attention":
+                att_ms[kind] += t
     recs = sess.gemm_times()
     kinds = sess.gemm_kinds()
     sess.profile_items(False)
@@ -531,7 +538,20 @@ def main():
         "pcie_gbs": [round(x / 1e9, 1) for x in bw], "pcie_source": "measured" if pcie else "fallback 55 GB/s",
         "how": "t_roof = max(plan FLOP / bf16_tflops_sustained, max(D2H bytes / B_d2h, H2D bytes / B_h2d)); "
                "frac = t_roof / measured step time"}
-    if not cnn:
+    if not cnn and args.attention == "fused":
+        # FA accounting per layer: forward 2 products (QK^T, PV), backward 5 (S recompute, dP, dV, dK,
+        # dQ), each 2 b a s^2 d FLOP; the F and B items cover every layer's batch exactly once
+        prod = 2.0 * BATCH * HEADS * SEQ * SEQ * (HID // HEADS)
+        line["roofline_attention"] = {
+            "bound": "alu", "kernel": "fa5_fwd / fa5_bwd_dq / fa5_bwd_dkv (tcgen05; softmax, Philox dropout on CUDA cores)",
+            "forward_us_per_layer": 1e3 * att_ms["F"] / args.layers,
+            "backward_us_per_layer": 1e3 * att_ms["B"] / args.layers,
+            "replay_ms": att_ms["R"],
+            "forward_tflops": 2 * prod * args.layers / (att_ms["F"] / 1e3) / 1e12 if att_ms["F"] > 0 else None,
+            "backward_tflops": 5 * prod * args.layers / (att_ms["B"] / 1e3) / 1e12 if att_ms["B"] > 0 else None,
+            "share_of_step": sum(att_ms.values()) / step_ms_prof if step_ms_prof else None,
+            "how": "summed cudaEvent times of the attention micro-op items of one eager step"}
+    elif not cnn:  # the paper's unfused graph: per-(sample, head) attention products on gemm_tc
         line["roofline_attention_gemm"] = {
             "bound": "hbm", "kernel": "gemm_tc on per-(sample, head) attention products",
             "achieved_tflops": a_flop / (a_ms / 1e3) / 1e12 if a_ms > 0 else None, "launches": len(att),
