@@ -79,6 +79,12 @@ class Clocks:
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.thread = threading.Thread(target=self._read, daemon=True)
             self.thread.start()
+            # nvidia-smi takes a few hundred ms to start: wait for its first line so the sampler
+            # is live when the timed region begins; only later lines are summarised
+            t0 = time.time()
+            while not self.lines and time.time() - t0 < 3.0:
+                time.sleep(0.01)
+            self.start_idx = len(self.lines)
         except FileNotFoundError:
             self.proc = None
         return self
@@ -98,7 +104,9 @@ class Clocks:
     def summary(self):
         sm, mx, reasons = [], None, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        start = getattr(self, "start_idx", 0)
+        lines = self.lines[start:] if len(self.lines) > start else self.lines
+        for ln in lines:
             parts = [x.strip() for x in ln.split(",")]
             if len(parts) < 8:
                 continue
