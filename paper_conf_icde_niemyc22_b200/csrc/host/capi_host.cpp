@@ -106,6 +106,25 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
     pr = &local;
   }
   ts_status st = plan_greedy(g->g, budget_bytes, *pr, p->st, flags);
+  // With a measured profile, Alg. 2 also runs on the analytic cost model and that plan is
+  // re-scored on the measured timeline: the greedy's single path depends on the costs it sees
+  // (profiles/r1_plan_variants.txt: the measured-cost greedy runs out of candidates on VGG-16
+  // and lands 19 % slower on ResNet-50 than the analytic-cost one, both judged on measurement)
+  PlanState from_analytic;
+  bool have_analytic = false;
+  if (profile) {
+    Profile ana;
+    profile_analytic(g->g, default_hw(), ana);
+    if (plan_greedy(g->g, budget_bytes, ana, from_analytic, flags) == TS_OK) {
+      plan_refresh(g->g, from_analytic, pr);  // predicted time on the measured profile
+      have_analytic = true;
+    }
+  }
+  if (st != TS_OK && have_analytic) {
+    p->st = std::move(from_analytic);
+    have_analytic = false;
+    st = TS_OK;
+  }
   // Alg. 2 is greedy and path-dependent: when it runs out of candidates, plan again for a
   // slightly tighter budget (different early decisions); any plan found fits the real one
   const std::string first_error = st == TS_OK ? std::string() : std::string(ts_last_error());
@@ -117,6 +136,7 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
   }
   if (st == TS_ERR_INFEASIBLE) set_error(first_error);
   if (st != TS_OK) return st;
+  if (have_analytic && from_analytic.predicted_s < p->st.predicted_s) p->st = std::move(from_analytic);
   // The greedy takes split proposals wherever their local dT/dM ratio is best, which can lock
   // it into a plan its own timeline rates slower than the one it finds without them
   // (profiles/r1_ablation_bert_large.json: BERT-Large b32 at 25 %).  The full planner's
