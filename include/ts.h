@@ -318,8 +318,9 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch,
  *   gdim 2 (K): C[0] = alpha sum_g A[g] op(B[g]) + bias[0] (+ beta C[0]), A[g]: M x K/groups
  *   gdim 3 (M): C[g] = alpha A[g] op(B[0]) + bias[0] (+ beta C[g]), A[g]: M/groups x K
  * lda/ldb/ldc/ta/tb/c_dtype as in ts_gemm_bf16 (shared by all groups); beta 0 or 1;
- * bias may be NULL.  TS_ERR_ARG when no tcgen05 tiling fits (the tile must not straddle
- * groups: N/groups a multiple of 64, M/groups of 128, K/groups of 64). */
+ * bias may be NULL.  One grouped tcgen05 launch when a tiling fits (the tile must not
+ * straddle groups: N/groups a multiple of 64, M/groups of 128, K/groups of 64), else the
+ * groups run as plain products (same results).  TS_ERR_ARG for bad groups / gdim. */
 ts_status ts_gemm_bf16_grouped(int32_t groups, int32_t gdim, int32_t M, int32_t N, int32_t K,
                                const void* const* A, int64_t lda, int32_t ta,
                                const void* const* B, int64_t ldb, int32_t tb,

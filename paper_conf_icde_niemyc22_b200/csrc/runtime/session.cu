@@ -1672,8 +1672,8 @@ ts_status ts_gemm_bf16_grouped(int32_t groups, int32_t gdim, int32_t M, int32_t 
     g.cg[i] = gdim == 2 ? C[0] : C[i];
     g.biasg[i] = bias ? (gdim == 1 ? bias[i] : bias[0]) : nullptr;
   }
-  if (!tsk::gemm_tc(g, static_cast<cudaStream_t>(stream)))
-    return set_error("grouped product not eligible for the tcgen05/TMA path"), TS_ERR_ARG;
+  // gemm(): the grouped tcgen05 launch, or (no tiling fits) the groups as plain products
+  tsk::gemm(g, static_cast<cudaStream_t>(stream));
   CU(cudaGetLastError());
   return TS_OK;
 }

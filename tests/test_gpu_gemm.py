@@ -145,6 +145,8 @@ def _ptrs(ts):
     (2, 640, 384, 3 * 128, 0, 1, "bf16", 0.0),
     (3, 3 * 256, 256, 2048, 1, 1, "f32", 1.0),     # q/k/v dW: per-group dY^T, shared X, per-group dW
     (3, 3 * 512, 512, 1024, 1, 1, "f32", 0.0),
+    (1, 512, 3 * 96, 128, 0, 0, "bf16", 0.0),      # N/groups = 96: no grouped tiling, per-group fallback
+    (3, 3 * 64, 256, 512, 1, 1, "f32", 1.0),       # M/groups = 64: per-group fallback
 ])
 def test_gemm_tc_grouped(gdim, M, N, K, ta, tb, out, beta, mode, gemm_mode):
     """Grouped product = the per-group plain products (fp32 torch reference)."""
