@@ -108,10 +108,11 @@ __global__ void attn_fwd_simt(AttnArgs A) {
   const Acc lse = m + log(l);
   const uint64_t e0 = ((uint64_t(A.b0 + b) * A.heads + a) * S + i) * uint64_t(S);
   const Acc scale = A.p > 0.f ? Acc(1) / (Acc(1) - Acc(A.p)) : Acc(1);
+  const uint32_t step = A.step_ptr ? *A.step_ptr : A.step;
   __syncthreads();
   for (int j = threadIdx.x; j < S; j += blockDim.x) {
     Acc pj = exp(s[j] - lse);
-    if (A.p > 0.f) pj = philox_one(e0 + j, A.seed, A.step) >= A.thr ? pj * scale : Acc(0);
+    if (A.p > 0.f) pj = philox_one(e0 + j, A.seed, step) >= A.thr ? pj * scale : Acc(0);
     s[j] = pj;
   }
   __syncthreads();
@@ -130,7 +131,7 @@ __global__ void attn_fwd_simt(AttnArgs A) {
     for (int w = threadIdx.x; w < nw; w += blockDim.x) {
       uint32_t bits = 0;
       for (int j = 0; j < 32 && 32 * w + j < S; ++j)
-        if (A.p <= 0.f || philox_one(e0 + 32 * w + j, A.seed, A.step) >= A.thr) bits |= 1u << j;
+        if (A.p <= 0.f || philox_one(e0 + 32 * w + j, A.seed, step) >= A.thr) bits |= 1u << j;
       mrow[w] = bits;
     }
   }
@@ -313,6 +314,7 @@ __global__ void __launch_bounds__(128) fa_fwd(AttnArgs A) {
   const int qb = blockIdx.x, a = blockIdx.y, b = blockIdx.z;
   const int S = A.seq;
   const int64_t ld = A.ld;
+  const uint32_t step = A.step_ptr ? *A.step_ptr : A.step;
   const bf16* Q = static_cast<const bf16*>(A.q) + (int64_t(b) * S + qb * kBM) * ld + a * kD;
   const bf16* K = static_cast<const bf16*>(A.k) + int64_t(b) * S * ld + a * kD;
   const bf16* V = static_cast<const bf16*>(A.v) + int64_t(b) * S * ld + a * kD;
@@ -386,7 +388,7 @@ __global__ void __launch_bounds__(128) fa_fwd(AttnArgs A) {
       l[1] += p2 + p3;
       bool kp[4] = {true, true, true, true};
       if (A.p > 0.f) {
-        quad_keep(equad + uint64_t(kb * kBN + n * 8), uint64_t(S), A.seed, A.step, A.thr, kp);
+        quad_keep(equad + uint64_t(kb * kBN + n * 8), uint64_t(S), A.seed, step, A.thr, kp);
         p0 = kp[0] ? p0 : 0.f;
         p1 = kp[1] ? p1 : 0.f;
         p2 = kp[2] ? p2 : 0.f;
@@ -501,17 +503,13 @@ __global__ void __launch_bounds__(128) fa_bwd_dq(AttnArgs A) {
   }
   const float* Lrow = A.lse + (int64_t(b) * A.heads + a) * S + q0;
   const float lse2[2] = {Lrow[0] * kLog2e, Lrow[8] * kLog2e};
-  if ((lane & 3) == 0) {
-    float* Dw = A.ws + (int64_t(b) * A.heads + a) * S + q0;
-    Dw[0] = Dr[0];
-    Dw[8] = Dr[1];
-  }
   const float sl2 = A.alpha * kLog2e;
   const float keep_scale = A.p > 0.f ? 1.f / (1.f - A.p) : 1.f;
   const uint32_t* mrow0 = A.mask + ((int64_t(b) * A.heads + a) * S + q0) * (S / 32);
   const uint32_t* mrow1 = mrow0 + 8 * (S / 32);
   uint32_t qa[4][4], ga[4][4];
   float dq[8][4] = {};
+  float rsum[2] = {0.f, 0.f};  // row sums of dS (D consistency, below)
   const int nkb = S / kBN;
   for (int kb = 0; kb < nkb; ++kb) {
     if (kb + 1 < nkb) {
@@ -564,6 +562,8 @@ __global__ void __launch_bounds__(128) fa_bwd_dq(AttnArgs A) {
       }
       const float s0 = v4[0] * (d0 - Dr[0]), s1 = v4[1] * (d1 - Dr[0]);
       const float s2 = v4[2] * (d2 - Dr[1]), s3 = v4[3] * (d3 - Dr[1]);
+      rsum[0] += s0 + s1;
+      rsum[1] += s2 + s3;
       const int kk = n >> 1;
       if ((n & 1) == 0) {
         da[kk][0] = pack_bf16(s0, s1);
@@ -583,6 +583,20 @@ __global__ void __launch_bounds__(128) fa_bwd_dq(AttnArgs A) {
         mma(dq[2 * nn + 1], da[kk][0], da[kk][1], da[kk][2], da[kk][3], bb[2], bb[3]);
       }
     __syncthreads();
+  }
+  // D for the dK/dV kernel: D_i = sum_j P_ij dP_ij exactly over the P this kernel rebuilt.
+  // dO . O differs from it by the bf16 rounding of O, and sum_j dS_ij = sum_j P_ij dP_ij - D_i
+  // (sum_j P_ij = 1), so D + sum_j dS_ij is the consistent row term: with it dS has zero row
+  // sums and the key-bias gradient keeps its analytic zero (softmax shift invariance).
+#pragma unroll
+  for (int h = 0; h < 2; ++h) {
+    rsum[h] += __shfl_xor_sync(0xffffffffu, rsum[h], 1);
+    rsum[h] += __shfl_xor_sync(0xffffffffu, rsum[h], 2);
+  }
+  if ((lane & 3) == 0) {
+    float* Dw = A.ws + (int64_t(b) * A.heads + a) * S + q0;
+    Dw[0] = Dr[0] + rsum[0];
+    Dw[8] = Dr[1] + rsum[1];
   }
   if (A.dq) {
     bf16* dQ = static_cast<bf16*>(A.dq) + (int64_t(b) * S + q0) * ld + a * kD;

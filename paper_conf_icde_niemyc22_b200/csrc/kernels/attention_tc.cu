@@ -52,6 +52,7 @@ struct Fa5P {
   float sl2;          // alpha * log2(e)
   float p, keep_scale;
   uint32_t seed, step, thr;
+  const uint32_t* step_ptr;  // live step counter (null: step)
   int64_t b0;
   void* c;
   float* lse;
@@ -173,12 +174,12 @@ __global__ void __launch_bounds__(256) attn_row_dot(const bf16* __restrict__ o, 
 // are double-buffered per item, and dQ accumulates in one of two TMEM buffers so an item's
 // epilogue overlaps the next item's products.  One TMA thread, one MMA thread, 16 compute
 // warps.  D_q = dO_q . O_q comes from attn_row_dot (launched first).
-// smem: Q 2 x 16K | dO 2 x 16K | K,V ring 3 x 32K | dS 2 x 32K | D 2 x 512 B | barriers
+// smem: Q 2 x 16K | dO 2 x 16K | K,V ring 3 x 32K | dS 2 x 32K | dS row partials 3 x 512 B | barriers
 // TMEM: S 0..127, dP 128..255, dQ 256..319 / 320..383
 constexpr int kDqStages = 3;
 constexpr int kDqThreads = 32 * (kBwdCW + 2);
 constexpr int kDqSmemQ = 0, kDqSmemG = 32768, kDqSmemKV = 65536, kDqSmemDS = kDqSmemKV + kDqStages * 32768;
-constexpr int kDqSmemD = kDqSmemDS + 65536, kDqSmemBar = kDqSmemD + 1024;
+constexpr int kDqSmemD = kDqSmemDS + 65536, kDqSmemBar = kDqSmemD + 1536;  // D: 3 x 128 row partials
 constexpr int kDqSmem = kDqSmemBar + 256 + 1024;
 __global__ void __launch_bounds__(kDqThreads, 1)
     fa5_bwd_dq(const __grid_constant__ CUtensorMap mQ, const __grid_constant__ CUtensorMap mdO,
@@ -314,6 +315,7 @@ __global__ void __launch_bounds__(kDqThreads, 1)
       const int q = qt * 128 + i;
       const float D = nD;
       const float l2 = nlse * kLog2e;
+      float rsum = 0.f;  // this thread's share of sum_j dS_ij
       if (item + int(gridDim.x) < items) item_consts(item + gridDim.x, nD, nlse);
       for (int kt = 0; kt < nkt; ++kt, ++kc) {
         const uint32_t bits = nbits;
@@ -331,13 +333,29 @@ __global__ void __launch_bounds__(kDqThreads, 1)
         for (int j = 0; j < 32; ++j) {
           const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
           const float dp = ((bits >> j) & 1u) ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
-          rs[j] = __float_as_uint(pr * (dp - D));
+          const float ds = pr * (dp - D);
+          rsum += ds;
+          rs[j] = __float_as_uint(ds);
         }
         if (kc >= 2) mbar_wait(&ds_free[kc & 1], ((kc >> 1) - 1) & 1);  // the dQ product of tile kc-2 read it
         st_row32(smem_u32(smem + kDqSmemDS + (kc & 1) * 32768), i, cg * 32, reinterpret_cast<const float*>(rs));
         fence_async_smem();
         tc_fence_before();
         mbar_arrive(&ds_full[kc & 1]);
+      }
+      // the dK/dV kernel's row term: D_i = sum_j P_ij dP_ij over the P rebuilt here, i.e. the
+      // dO . O of attn_row_dot plus sum_j dS_ij (dO . O carries the bf16 rounding of O; with
+      // the consistent D, dS has zero row sums and the key-bias gradient its analytic zero).
+      // Four column groups per row: fixed-order sum through shared memory (deterministic).
+      {
+        float* red = reinterpret_cast<float*>(smem + kDqSmemD);
+        if (cg > 0) red[(cg - 1) * 128 + i] = rsum;
+        named_sync(1, 32 * kBwdCW);
+        if (cg == 0) {
+          const int64_t hr = (int64_t(b) * p.heads + a) * S + q;
+          p.D[hr] = D + (((rsum + red[i]) + red[128 + i]) + red[256 + i]);
+        }
+        named_sync(1, 32 * kBwdCW);  // the slots are rewritten by the next item
       }
       mbar_wait(&dq_full[it & 1], (it >> 1) & 1);
       tc_fence_after();
@@ -624,6 +642,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = p.seq, nqt = S / 128, npair = (nqt + 1) / 2, nkc = S / kFwdKC;
   const int items = p.nb * p.heads * npair;
+  const uint32_t step = p.step_ptr ? *p.step_ptr : p.step;
   if (threadIdx.x == 0) {
     mbar_init(&q_full[0], 1);
     mbar_init(&q_full[1], 1);
@@ -799,7 +818,7 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
           const uint64_t cnt0 = (erow + uint64_t(key)) >> 3;
 #pragma unroll
           for (int u = 0; u < 4; ++u) {
-            const uint4 w = philox4x32_10(uint32_t(cnt0) + uint32_t(u), uint32_t(cnt0 >> 32), p.step, 0u, p.seed,
+            const uint4 w = philox4x32_10(uint32_t(cnt0) + uint32_t(u), uint32_t(cnt0 >> 32), step, 0u, p.seed,
                                           kPhiloxKey1);
             bits |= keep_bits8(w, p.thr) << (8 * u);
           }
@@ -896,6 +915,7 @@ bool attention_fwd_tc5(const AttnArgs& A, cudaStream_t st) {
   p.keep_scale = A.p > 0.f ? 1.f / (1.f - A.p) : 1.f;
   p.seed = A.seed;
   p.step = A.step;
+  p.step_ptr = A.step_ptr;
   p.thr = A.thr;
   p.b0 = A.b0;
   p.c = A.c;

@@ -15,6 +15,7 @@ struct EwP {
   int64_t elem0;
   float p, scale;
   uint32_t seed, step, thr;
+  const uint32_t* step_ptr;
 };
 
 // GELU: gelu_f / gelu_d from common.cuh (shared with the GEMM epilogue).
@@ -69,6 +70,8 @@ template <class T, int OP, int V>
 __global__ void __launch_bounds__(256) ew_kernel(const T* __restrict__ a, const T* __restrict__ b, T* y, int64_t n,
                                                  int acc, EwP q) {
   constexpr int U = 2;  // two 16-byte vectors in flight per thread (HBM latency)
+  if constexpr (OP == DROP)
+    if (q.step_ptr) q.step = *q.step_ptr;
   const int64_t nv = n / V;
   const int64_t stride = int64_t(gridDim.x) * blockDim.x;
   for (int64_t v0 = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; v0 < nv; v0 += stride * U) {
@@ -149,6 +152,7 @@ __global__ void cast_kernel(const float* __restrict__ s, bf16* __restrict__ d, i
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
     d[i] = __float2bfloat16_rn(s[i]);
 }
+__global__ void step_advance_kernel(uint32_t* c) { *c += 1u; }
 __global__ void scale_kernel(float* x, int64_t n, float s) {
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
     x[i] *= s;
@@ -256,13 +260,14 @@ void axpy2(int dt, const void* dy, void* d1, int acc1, void* d2, int acc2, int64
     axpy2_kernel<bf16><<<grid, 256, 0, st>>>((const bf16*)dy, (bf16*)d1, acc1, (bf16*)d2, acc2, n);
 }
 void dropout(int dt, const void* x, void* y, int acc, int64_t n, int64_t elem0, float p, uint32_t seed,
-             uint32_t step, cudaStream_t st) {
+             uint32_t step, const uint32_t* step_ptr, cudaStream_t st) {
   EwP q;
   q.elem0 = elem0;
   q.p = p;
   q.scale = p > 0.f ? 1.f / (1.f - p) : 1.f;
   q.seed = seed;
   q.step = step;
+  q.step_ptr = step_ptr;
   q.thr = dropout_thr16(p);
   ew<DROP>(dt, x, nullptr, y, n, acc, q, st);
 }
@@ -275,6 +280,7 @@ void sgd_fused(const SgdChunk* chunks, int n_chunks, char* slab, float lr, float
 void cast_f32_bf16(const float* src, void* dst, int64_t n, cudaStream_t st) {
   cast_kernel<<<grid_for(n), 256, 0, st>>>(src, reinterpret_cast<bf16*>(dst), n);
 }
+void step_advance(uint32_t* counter, cudaStream_t st) { step_advance_kernel<<<1, 1, 0, st>>>(counter); }
 void scale_f32(float* x, int64_t n, float s, cudaStream_t st) { scale_kernel<<<grid_for(n), 256, 0, st>>>(x, n, s); }
 
 }  // namespace tsk

@@ -144,6 +144,9 @@ struct AttnArgs {
   int acc_q = 0, acc_k = 0, acc_v = 0;
   float alpha = 1.f, p = 0.f;
   uint32_t seed = 0, step = 0, thr = 0;
+  // device copy of the step counter: when set, kernels read the dropout step from it at run
+  // time (a captured CUDA graph replays with the live value); null = use `step`
+  const uint32_t* step_ptr = nullptr;
   int64_t b0 = 0;
   float* ws = nullptr;
   int no_tc5 = 0;  // tests: skip the tcgen05 kernels (mma.sync path instead)
@@ -179,8 +182,11 @@ void add_fwd(int dt, const void* a, const void* b, void* y, int64_t n, cudaStrea
 void axpy(int dt, const void* dy, void* dx, int acc, int64_t n, cudaStream_t st);
 // add backward: d1 (+)= dy and d2 (+)= dy in one pass (acc flags per output)
 void axpy2(int dt, const void* dy, void* d1, int acc1, void* d2, int acc2, int64_t n, cudaStream_t st);
+// step_ptr: device step counter read at run time (null: `step`)
 void dropout(int dt, const void* x, void* y, int acc, int64_t n, int64_t elem0, float p, uint32_t seed,
-             uint32_t step, cudaStream_t st);
+             uint32_t step, const uint32_t* step_ptr, cudaStream_t st);
+// *counter += 1 on the stream (the session's dropout step, advanced at the end of every step)
+void step_advance(uint32_t* counter, cudaStream_t st);
 // ---- row ops -----------------------------------------------------------------
 void layernorm_fwd(int dt, const void* x, const void* g, const void* b, void* y, int64_t rows, int H,
                    float eps, cudaStream_t st);

@@ -76,7 +76,9 @@ struct ts_session_s {
   int n_sgd_chunks = 0;
   int world = 1;
   float lr = 0.f;
-  uint32_t step = 0;
+  uint32_t step = 0;        // host mirror of the dropout step (reporting, eager kernel tests)
+  uint32_t* step_dev = nullptr;  // the step the kernels read: advanced on the device at the end of
+                                 // every step, so CUDA-graph replays see the live value (R15)
   bool use_graph = true;
   cudaGraphExec_t gexec = nullptr;
   int64_t graph_kernels = 0;
@@ -227,7 +229,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
   const Tensor& out = g.t[o.out[0]];
   const int64_t n_out = (out.sample ? ns * out.elems_per_sample : out.numel) / (m.cb >= 0 ? m.cp : 1);
   const int64_t elem0 = out.sample ? m.s0 * out.elems_per_sample : 0;
-  uint32_t* stepp = &s->step;
+  const uint32_t* stepp = s->step_dev;
   switch (o.kind) {
     case TS_OP_LINEAR: {
       const Tensor& x = g.t[o.in[0]];
@@ -403,11 +405,11 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       nk = 1;
       if (!bwd) {
         char *x = V(o.in[0]), *y = V(o.out[0]);
-        return [=](cudaStream_t st) { tsk::dropout(dt, x, y, 0, n_out, elem0, p, seed, *stepp, st); };
+        return [=](cudaStream_t st) { tsk::dropout(dt, x, y, 0, n_out, elem0, p, seed, 0u, stepp, st); };
       }
       char *dy = G(o.out[0]), *dx = G(o.in[0]);
       int acc = A(g.n() + o.in[0]);
-      return [=](cudaStream_t st) { tsk::dropout(dt, dy, dx, acc, n_out, elem0, p, seed, *stepp, st); };
+      return [=](cudaStream_t st) { tsk::dropout(dt, dy, dx, acc, n_out, elem0, p, seed, 0u, stepp, st); };
     }
     case TS_OP_SOFTMAX: {
       const int L = int(out.shape[out.ndim - 1]);
@@ -658,11 +660,8 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
         a.lse = m.writes.count(o.out[1]) ? reinterpret_cast<float*>(V(o.out[1])) : nullptr;
         a.mask = m.writes.count(o.out[2]) ? reinterpret_cast<uint32_t*>(V(o.out[2])) : nullptr;
         nk = 1;
-        return [a, stepp](cudaStream_t st) {
-          tsk::AttnArgs b = a;
-          b.step = *stepp;
-          tsk::attention_fwd(b, st);
-        };
+        a.step_ptr = stepp;
+        return [a](cudaStream_t st) { tsk::attention_fwd(a, st); };
       }
       a.c = V(o.out[0]);
       a.lse = reinterpret_cast<float*>(V(o.out[1]));
@@ -679,11 +678,8 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       gslot(1, a.dk, a.acc_k);
       gslot(2, a.dv, a.acc_v);
       nk = 2;
-      return [a, stepp](cudaStream_t st) {
-        tsk::AttnArgs b = a;
-        b.step = *stepp;
-        tsk::attention_bwd(b, st);
-      };
+      a.step_ptr = stepp;
+      return [a](cudaStream_t st) { tsk::attention_bwd(a, st); };
     }
     case TS_OP_XENT: {
       const int C = int(g.t[o.in[0]].shape[1]);
@@ -710,6 +706,10 @@ ts_status build_program(ts_session_t* s) {
   const int n = g.n();
   const int B = g.samples;
   const int es = dtype_bytes(g.dtype);
+  // the device step counter the dropout / attention kernels read (one word outside the slab,
+  // like the optimiser's chunk table)
+  CU(cudaMalloc(&s->step_dev, sizeof(uint32_t)));
+  CU(cudaMemcpyAsync(s->step_dev, &s->step, sizeof(uint32_t), cudaMemcpyHostToDevice, s->cs));
   // host slots for swapped pieces (pinned, allocated once)
   std::map<PieceKey, uint64_t> host_off;
   uint64_t hb = 0;
@@ -831,7 +831,9 @@ ts_status build_program(ts_session_t* s) {
         int p = piece_count(g, s->cfg, t);
         int j = int(m.s0 * p / B);
         int64_t first = int64_t(j) * B / p;
-        return s->slab + where.at(pk(key, j)) + (m.s0 - first) * x.elems_per_sample * es;
+        // (the tensor's own element size: an f32 / i32 auxiliary output of a bf16 graph,
+        // e.g. the attention's lse and keep bits, read through a sub-view of its piece)
+        return s->slab + where.at(pk(key, j)) + (m.s0 - first) * x.elems_per_sample * dtype_bytes(x.dtype);
       };
       std::vector<int> ts_all(o.in.begin(), o.in.end());
       ts_all.insert(ts_all.end(), o.out.begin(), o.out.end());
@@ -846,7 +848,7 @@ ts_status build_program(ts_session_t* s) {
             if (gr && where.count(pk(n + t, m.k))) m.grad[t] = view(n + t);
           } else {  // every block, rows [s0, s1) of each
             const int pc = piece_count(g, s->cfg, t);
-            const int64_t roff = m.s0 * g.t[t].elems_per_sample / pc * es;
+            const int64_t roff = m.s0 * g.t[t].elems_per_sample / pc * dtype_bytes(g.t[t].dtype);
             std::vector<char*> vb, gb;
             for (int j = 0; j < pc; ++j) {
               if (where.count(pk(t, j))) vb.push_back(s->slab + where.at(pk(t, j)) + roff);
@@ -1121,6 +1123,7 @@ ts_status build_program(ts_session_t* s) {
       CU(cudaMemcpy(s->sgd_chunks, ch.data(), ch.size() * sizeof(tsk::SgdChunk), cudaMemcpyHostToDevice));
     }
   }
+  s->launches += 1;  // step_advance
   CU(cudaEventCreateWithFlags(&s->ev_mark, cudaEventDisableTiming));
   CU(cudaEventCreateWithFlags(&s->ev_join_d2h, cudaEventDisableTiming));
   CU(cudaEventCreateWithFlags(&s->ev_join_h2d, cudaEventDisableTiming));
@@ -1190,6 +1193,7 @@ void issue_step(ts_session_t* s) {
     cudaEventRecord(s->ev_join_h2d, s->h2d);
     cudaStreamWaitEvent(cs, s->ev_join_h2d, 0);
   }
+  tsk::step_advance(s->step_dev, cs);  // the next step's dropout masks (graph replays included)
 }
 
 ts_status copy_inputs(ts_session_t* s, const void* const* inputs, int on_host) {
@@ -1243,7 +1247,7 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
   } else {
     issue_step(s);
   }
-  ++s->step;  // dropout counter (graph mode keeps the captured step value)
+  ++s->step;  // host mirror; the kernels read s->step_dev, advanced by the step itself
   CU(cudaGetLastError());
   if (s->profile) {
     tsk::gemm_records_enable(nullptr);
@@ -1344,6 +1348,7 @@ void ts_session_destroy(ts_session_t* s) {
     if (e) cudaEventDestroy(e);
   if (s->ev_comm_done) cudaEventDestroy(s->ev_comm_done);
   if (s->sgd_chunks) cudaFree(s->sgd_chunks);
+  if (s->step_dev) cudaFree(s->step_dev);
   if (s->comm) cudaStreamDestroy(s->comm);
   if (s->ev_mark) cudaEventDestroy(s->ev_mark);
   if (s->ev_join_d2h) cudaEventDestroy(s->ev_join_d2h);

@@ -37,3 +37,15 @@ def global_rel_err(got: dict, ref: dict):
               for k, r in ref.items())
     den = sum(float(np.sum(np.asarray(r, np.float64) ** 2)) for r in ref.values())
     return (num / den) ** 0.5
+
+
+BF16_TOL = 2e-2  # north_star: bf16 gradients within 2e-2 of the fp64 oracle (per tensor, R17)
+
+
+def assert_bf16_parity(got: dict, ref: dict, tol: float = BF16_TOL):
+    """Per-tensor relative L2 <= tol against the plain fp64 oracle (`net.train_step`,
+    storage=None), with rel_errs' floor for analytically-zero tensors."""
+    errs = rel_errs(got, ref)
+    worst = sorted(errs.items(), key=lambda kv: -kv[1])[:5]
+    assert worst[0][1] <= tol, worst
+    return errs

@@ -6,7 +6,8 @@
   multi-tap K blocks (C < 64), stride-2 dgrad, 1x1 convs, the C = 3 image layer
   (scalar gather) and split-K wgrad;
 * whole training steps of the tiny VGG / ResNet graphs under random split / swap /
-  recompute plans against the oracle (fp32: 1e-5 per tensor; bf16: reading D-TOL),
+  recompute plans against the oracle (fp32: 1e-5 per tensor; bf16: reading D-TOL-CNN —
+  the bar is the precision's own distance from fp64, measured by the oracle alone),
   split vs unsplit on the GPU (fp32: 1e-6), and trace equality with the simulator.
 """
 
@@ -173,22 +174,28 @@ def test_cnn_tiny_fp32_random_plans(name, seed):
     assert S.trace() == [tuple(e) for e in sim.simulate(g, {**sim.default_cfg(g), **cfg}).trace]
 
 
-@pytest.mark.parametrize("name", ["vgg_tiny", "resnet_tiny"])
-def test_cnn_tiny_bf16_parity_and_budget(name):
-    """bf16 graphs store activations and their gradients in bf16 (R20); the oracle's
-    bf16-storage reading rounds the same values (DESIGN.md D-TOL).  Against it: whole
-    gradient <= 2e-2 and every tensor <= 1e-1; a budgeted plan trains the same function."""
+@pytest.mark.parametrize("name", ["vgg_small", "resnet_small"])
+def test_cnn_bf16_precision_and_budget(name):
+    """bf16 CNN steps (reading D-TOL-CNN).  Any execution that stores ReLU-network
+    activations in bf16 is far from fp64 here: the oracle alone, rounding only its stored
+    values, is 3-17 % away on the early conv / BN gradients (tests/test_oracle_bf16_gap.py
+    pins this; the mechanism is ReLU and max-pool decisions flipped by forward rounding).
+    So the bar is that distance, not 2e-2: per tensor the GPU is within max(2e-2, 1.5 x)
+    the bf16-storage reading's own error against the plain fp64 oracle, and the whole
+    gradient within max(2e-2, 1.25 x).  fp32 graphs meet 1e-5 (test above).  A planned
+    budget trains the same function (<= 1e-3 of the all-reside plan)."""
     g = graphs.config_graph(name)
-    ol, og = _oracle(g, storage="bf16")
+    ol, og = _oracle(g)
+    _, ob = _oracle(g, storage="bf16")
     loss, grads, S, P = _run(g)
     assert abs(loss - ol) <= 2e-2 * abs(ol)
-    assert global_rel_err(grads, og) <= 2e-2
-    errs = rel_errs(grads, og)
-    assert max(errs.values()) <= 1e-1, sorted(errs.items(), key=lambda kv: -kv[1])[:5]
+    e_gpu, e_ref = rel_errs(grads, og), rel_errs(ob, og)
+    print(name, "gpu vs fp64: global", global_rel_err(grads, og), "bf16 reading vs fp64:", global_rel_err(ob, og))
+    bad = {k: (e_gpu[k], e_ref[k]) for k in e_gpu if e_gpu[k] > max(2e-2, 1.5 * e_ref[k])}
+    assert not bad, bad
+    assert global_rel_err(grads, og) <= max(2e-2, 1.25 * global_rel_err(ob, og))
     base = P.stats()
-    # the greedy planner (Alg. 2, a heuristic) is not monotone in the budget on graphs this
-    # small (batch 4, so p <= 4): take the first of 50/60/70% of the dynamic peak it solves
-    for frac in (5, 6, 7):
+    for frac in (3, 4, 5, 6, 7):
         budget = base["static_bytes"] + (base["peak_extent"] - base["static_bytes"]) * frac // 10
         try:
             tsplit.Plan.plan(tsplit.Graph(g), budget)
@@ -199,5 +206,5 @@ def test_cnn_tiny_bf16_parity_and_budget(name):
     st = P2.stats()
     assert st["peak_extent"] <= budget and st["n_split_tensors"] + st["n_swap_tensors"] > 0
     assert S2.trace() == P2.trace()
-    assert global_rel_err(g2, og) <= 2e-2
-    assert global_rel_err(g2, grads) <= 1e-2
+    print(name, "budget", frac, "/10: split-vs-unsplit", global_rel_err(g2, grads))
+    assert global_rel_err(g2, grads) <= 1e-3

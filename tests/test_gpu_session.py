@@ -10,7 +10,7 @@ import pytest
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
 
-from conftest import global_rel_err, rel_errs  # noqa: E402
+from conftest import assert_bf16_parity, global_rel_err, rel_errs  # noqa: E402
 from oracle import brute, net, sim  # noqa: E402
 from paper_conf_icde_niemyc22_b200 import tsplit  # noqa: E402
 from tsinputs import gen, graphs  # noqa: E402
@@ -33,6 +33,18 @@ def _run(g, plan_cfg=None, budget=None, graph_mode=True, on_host=False):
     dev = tsplit.inputs_to_device(G, inputs, pinned_host=on_host)
     loss = S.step(dev)
     return loss, S.grads(), S, P
+
+
+def _run_unfused(g, **kw):
+    """_run with the session's peephole fusions (D-FUSE, D-QKV) off: which fusions apply
+    depends on the plan's allocations, and the fused q/k/v backward rounds dX to bf16 once
+    instead of three times, so plan invariance is checked with both programs unfused."""
+    import os
+    os.environ["TSPLIT_NO_FUSION"] = "1"
+    try:
+        return _run(g, **kw)
+    finally:
+        os.environ.pop("TSPLIT_NO_FUSION", None)
 
 
 def _oracle(g):
@@ -76,23 +88,27 @@ def test_bert_tiny_fp32_random_plans(seed):
     assert max(e0.values()) <= 1e-6, sorted(e0.items(), key=lambda kv: -kv[1])[:5]
 
 
-def test_bert_tiny_bf16_parity_and_budget():
-    """bf16 reading D-TOL: whole-gradient relative L2 <= 2e-2 vs the fp64 oracle,
-    every tensor <= 1e-1 (row sums of bf16-rounded gradients, e.g. bias grads,
-    carry the rounding of every summand)."""
-    g = graphs.config_graph("bert_tiny")
+@pytest.mark.parametrize("fused_attention", [False, True])
+def test_bert_small_bf16_parity_and_budget(fused_attention):
+    """bf16 (R17, D-TOL): every parameter gradient within 2e-2 (per-tensor relative L2) of
+    the plain fp64 oracle, unbudgeted and under a planned 40 % budget; with the peephole
+    fusions off in both, the budgeted plan computes the all-reside plan's gradients
+    (<= 1e-6: splits change only fp32 accumulation order)."""
+    g = graphs.config_graph("bert_small", fused_attention=fused_attention)
     ol, og = _oracle(g)
     loss, grads, S, P = _run(g)
     assert abs(loss - ol) <= 2e-2 * abs(ol)
-    assert global_rel_err(grads, og) <= 2e-2
-    errs = rel_errs(grads, og)
-    assert max(errs.values()) <= 1e-1, sorted(errs.items(), key=lambda kv: -kv[1])[:5]
+    assert_bf16_parity(grads, og)
     base = P.stats()
     budget = base["static_bytes"] + (base["peak_extent"] - base["static_bytes"]) * 4 // 10
     l2, g2, S2, P2 = _run(g, budget=budget)
-    assert P2.stats()["peak_extent"] <= budget
-    assert global_rel_err(g2, og) <= 2e-2
-    assert global_rel_err(g2, grads) <= 1e-2
+    st = P2.stats()
+    assert st["peak_extent"] <= budget and st["n_split_tensors"] + st["n_swap_tensors"] + st["n_recompute_tensors"] > 0
+    assert S2.trace() == P2.trace()
+    assert_bf16_parity(g2, og)
+    _, u0, _, _ = _run_unfused(g)
+    _, u2, _, _ = _run_unfused(g, budget=budget)
+    assert global_rel_err(u2, u0) <= 1e-6
 
 
 def test_eager_equals_graph_and_host_inputs():
@@ -146,7 +162,7 @@ def test_bert_large_full_size_properties():
     torch.cuda.empty_cache()
     assert abs(l_b - math.log(2.0)) < 0.05 and abs(l_0 - l_b) <= 1e-3 * abs(l_0)
     assert all(np.isfinite(v).all() for v in g_b.values())
-    assert global_rel_err(g_b, g_0) <= 1e-2
+    assert global_rel_err(g_b, g_0) <= 1e-3
 
 
 def test_nccl_bucketed_allreduce_single_rank():
@@ -199,7 +215,7 @@ def test_qkv_grouped_fusion(plan):
     (summed in fp32, a single accumulation into dX) and one M-grouped dW.  The forward is
     the same arithmetic (loss bit-identical); the backward differs only by the bf16
     rounding of the dX accumulation; both stay within the bf16 bar of the oracle."""
-    g = graphs.config_graph("bert_tiny", fused_attention=True)
+    g = graphs.config_graph("bert_small", fused_attention=True)
     names = {t["name"]: t["id"] for t in g["tensors"]}
     cfg = {}
     if plan == "recompute_qkv":
@@ -210,9 +226,7 @@ def test_qkv_grouped_fusion(plan):
     assert n1 < n0, (n0, n1)
     assert l1 == l0
     assert global_rel_err(g1, g0) <= 5e-3
-    params, inputs = gen.init_params(g), gen.make_inputs(g)
-    _, ogb, _, _ = net.train_step(g, params, inputs, storage="bf16")
-    assert global_rel_err(g1, ogb) <= 2e-2
+    assert_bf16_parity(g1, _oracle(g)[1])
 
 
 @pytest.mark.parametrize("fused_attention", [False, True])
@@ -223,7 +237,7 @@ def test_linear_gelu_fusion_equals_unfused(fused_attention, plan):
     (session.cu build_program).  The fused program computes what the unfused one does —
     the epilogue rounds through bf16 exactly where the separate kernels store — and
     launches fewer kernels; it also stays within the bf16 bar of the fp64 oracle."""
-    g = graphs.config_graph("bert_tiny", fused_attention=fused_attention)
+    g = graphs.config_graph("bert_small", fused_attention=fused_attention)
     names = {t["name"]: t["id"] for t in g["tensors"]}
     cfg = {}
     if plan == "recompute_ffn":  # replays R(ffn1), R(gelu) are adjacent too
@@ -236,9 +250,7 @@ def test_linear_gelu_fusion_equals_unfused(fused_attention, plan):
     assert n1 < n0, (n0, n1)
     assert abs(l1 - l0) <= 1e-6 * abs(l0)
     assert global_rel_err(g1, g0) <= 1e-6
-    params, inputs = gen.init_params(g), gen.make_inputs(g)
-    _, ogb, _, _ = net.train_step(g, params, inputs, storage="bf16")
-    assert global_rel_err(g1, ogb) <= 2e-2
+    assert_bf16_parity(g1, _oracle(g)[1])
 
 
 @pytest.mark.parametrize("cache", [1 << 20, 2 ** 64 - 1])
@@ -269,17 +281,74 @@ def test_lru_recompute_cache_session(cache):
     assert max(rel_errs(out[1][1], og).values()) <= 1e-5
 
 
-@pytest.mark.parametrize("hidden", [512, 1024])
-def test_bert_wide_hidden_bf16_parity(hidden):
-    """Row kernels at BERT-Large widths (LayerNorm fwd/bwd with 2 / 4 sixteen-byte chunks per
-    lane, fused bias / LN-gradient partials) through a whole bf16 step, split + recompute,
-    against the oracle's bf16-storage reading (D-TOL)."""
-    g = graphs.bert(layers=1, hidden=hidden, heads=hidden // 64, seq=128, batch=4, vocab=512, fused_attention=True)
+def test_bert_large_shaped_layer_bf16_parity():
+    """A BERT-Large-shaped encoder layer (hidden 1024, 16 heads, seq 512, batch 4, the real
+    vocabulary; fused attention, dropout 0.1) under a plan with sample splits, a swap and
+    recomputes, against the plain fp64 oracle per tensor (north_star bf16 bar, R17)."""
+    g = graphs.config_graph("bert_large", layers=1, batch=4, fused_attention=True)
     names = {t["name"]: t["id"] for t in g["tensors"]}
-    cfg = {names["l0.ln1"]: (tsplit.RECOMPUTE, 2, 1), names["l0.ffn1"]: (tsplit.RESIDE, 2, 1)}
+    cfg = {names["l0.ln1"]: (tsplit.RECOMPUTE, 2, 1), names["l0.ffn1"]: (tsplit.RESIDE, 2, 1),
+           names["l0.gelu"]: (tsplit.SWAP, 2, 1), names["l0.q"]: (tsplit.RECOMPUTE, 1, 1),
+           names["l0.k"]: (tsplit.RECOMPUTE, 1, 1), names["l0.ctx"]: (tsplit.SWAP, 1, 2),
+           names["l0.res2"]: (tsplit.RESIDE, 4, 1)}
     loss, grads, S, P = _run(g, cfg)
+    st = P.stats()
+    assert st["n_split_tensors"] > 0 and st["n_swap_tensors"] > 0 and st["n_recompute_tensors"] > 0
+    assert S.trace() == [tuple(e) for e in sim.simulate(g, {**sim.default_cfg(g), **cfg}).trace]
+    ol, og = _oracle(g)
+    assert abs(loss - ol) <= 2e-2 * abs(ol)
+    errs = assert_bf16_parity(grads, og)
+    print("bert-large-shaped layer: worst", sorted(errs.items(), key=lambda kv: -kv[1])[:4])
+    _, g0, _, _ = _run(g)
+    assert global_rel_err(grads, g0) <= 1e-3
+
+
+@pytest.mark.parametrize("fused_attention", [False, True])
+@pytest.mark.parametrize("graph_mode", [True, False])
+def test_dropout_masks_follow_the_step_counter(fused_attention, graph_mode):
+    """R15 / D-RNG: the dropout masks of step k use Philox counter word `step` = k.  The
+    session keeps the step in device memory and advances it at the end of every step, so a
+    captured CUDA graph replays with the live value.  Three steps with lr = 0 (parameters
+    fixed) give gradients equal to the oracle's `train_step(step=k)` for k = 0, 1, 2 — and
+    different from one another (the masks change)."""
+    g = graphs.config_graph("bert_tiny", dtype="f32", fused_attention=fused_attention)
+    G = tsplit.Graph(g)
+    P = tsplit.Plan.default(G)
     params, inputs = gen.init_params(g), gen.make_inputs(g)
-    _, ogb, _, _ = net.train_step(g, params, inputs, storage="bf16")
-    assert global_rel_err(grads, ogb) <= 2e-2
-    errs = rel_errs(grads, ogb)
-    assert errs["l0.ln1.g"] <= 2e-2 and errs["l0.ln2.g"] <= 2e-2, errs
+    S = tsplit.Session(G, P, use_cuda_graph=graph_mode, lr=0.0)
+    S.set_params(params)
+    dev = tsplit.inputs_to_device(G, inputs)
+    prev = None
+    for k in range(3):
+        loss = S.step(dev)
+        grads = S.grads()
+        ol, og, _, _ = net.train_step(g, params, inputs, step=k)
+        assert abs(loss - ol) <= 1e-5 * abs(ol), (k, loss, ol)
+        errs = rel_errs(grads, og)
+        assert max(errs.values()) <= 1e-5, (k, sorted(errs.items(), key=lambda kv: -kv[1])[:3])
+        if prev is not None:
+            assert global_rel_err(grads, prev) > 1e-3  # a new mask, not a replayed one
+        prev = grads
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_bert_small_bf16_random_plans(seed):
+    """bf16 graphs under random split / swap / recompute plans (the fused-attention graph:
+    its f32 / i32 auxiliary outputs are then read through sub-views of other sizes): per
+    tensor within 2e-2 of the plain fp64 oracle, and — with the peephole fusions off in
+    both — equal to the all-reside plan up to fp32 accumulation order.  In a bf16 graph a
+    reordered fp32 sum (a different GEMM split-K, dW summed over micro-ops) moves a stored
+    value across a bf16 rounding boundary with probability ~2^-24 sqrt(K) / 2^-9, i.e. a
+    few elements in 10^4 by one bf16 ulp (2^-8): <= 1e-4 globally (the fp32 graphs'
+    1e-6 bar is that of fp32 storage)."""
+    g = graphs.config_graph("bert_small", fused_attention=True)
+    r = random.Random(300 + seed)
+    cfg = {t: (r.choice([0, 1, 2]), r.choice([1, 2, 4]), r.choice([1, 2])) for t in brute.act_tensors(g)}
+    loss, grads, S, P = _run(g, cfg)
+    assert S.trace() == [tuple(e) for e in sim.simulate(g, {**sim.default_cfg(g), **cfg}).trace]
+    ol, og = _oracle(g)
+    assert abs(loss - ol) <= 2e-2 * abs(ol)
+    assert_bf16_parity(grads, og)
+    _, u1, _, _ = _run_unfused(g, plan_cfg=cfg)
+    _, u0, _, _ = _run_unfused(g)
+    assert global_rel_err(u1, u0) <= 1e-4

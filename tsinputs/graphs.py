@@ -212,6 +212,10 @@ def config_graph(name: str, **over) -> dict:
         kw = dict(layers=2, hidden=128, heads=2, seq=64, batch=4, vocab=512)
         kw.update(over)
         return bert(**kw)
+    if name == "bert_small":  # the bf16 parity size (DESIGN.md D-TOL): hidden 256, 4 heads of 64
+        kw = dict(layers=2, hidden=256, heads=4, seq=128, batch=8, vocab=512)
+        kw.update(over)
+        return bert(**kw)
     if name == "vgg16":
         return vgg16(**over)
     if name == "vgg_tiny":
@@ -219,10 +223,19 @@ def config_graph(name: str, **over) -> dict:
                   cfg=[64, "M", 128, "M", 256, 256, "M"])
         kw.update(over)
         return vgg16(**kw)
+    if name == "vgg_small":  # bf16 precision study size (DESIGN.md D-TOL)
+        kw = dict(batch=16, img=32, width=0.25, fc=128, classes=10,
+                  cfg=[64, "M", 128, "M", 256, 256, "M"])
+        kw.update(over)
+        return vgg16(**kw)
     if name == "resnet50":
         return resnet50(**over)
     if name == "resnet_tiny":
         kw = dict(batch=4, img=32, width=0.125, blocks=(1, 1), classes=10)
+        kw.update(over)
+        return resnet50(**kw)
+    if name == "resnet_small":
+        kw = dict(batch=16, img=32, width=0.25, blocks=(1, 1), classes=10)
         kw.update(over)
         return resnet50(**kw)
     if name == "bert_scaled":
