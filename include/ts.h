@@ -234,6 +234,11 @@ ts_status ts_plan_items(const ts_plan_t* p, int32_t* buf, uint64_t cap, uint64_t
  * order; *n = number of triples (buf may be NULL).  Every rank derives the identical
  * list from the broadcast plan, so NCCL calls match across ranks. */
 ts_status ts_plan_grad_buckets(const ts_plan_t* p, uint64_t bucket_bytes, int64_t* buf, uint64_t cap, uint64_t* n);
+/* Plan blob for the data-parallel broadcast (rank 0 plans, every rank deserializes):
+ * serialize writes *n bytes (buf NULL: size query; TS_ERR_ARG when cap < *n).  The blob
+ * carries a fingerprint of the graph; deserialize returns TS_ERR_ARG for a blob of another
+ * graph, a malformed one, or any entry ts_plan_set would reject (opt / p_num / dim / lead,
+ * parameters not reside, an illegal D-CH channel chain) — nothing is adopted then. */
 ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n);
 ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, ts_plan_t** out);
 void ts_plan_destroy(ts_plan_t* p);
@@ -320,7 +325,10 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch,
  * lda/ldb/ldc/ta/tb/c_dtype as in ts_gemm_bf16 (shared by all groups); beta 0 or 1;
  * bias may be NULL.  One grouped tcgen05 launch when a tiling fits (the tile must not
  * straddle groups: N/groups a multiple of 64, M/groups of 128, K/groups of 64), else the
- * groups run as plain products (same results).  TS_ERR_ARG for bad groups / gdim. */
+ * groups run as plain products — the same values except for gdim 2 with a bf16 C, where
+ * the per-group fallback rounds the running sum to bf16 after every group (the grouped
+ * launch rounds once).  TS_ERR_ARG for bad groups / gdim, a grouped extent (N, K or M)
+ * that `groups` does not divide, or beta other than 0 / 1. */
 ts_status ts_gemm_bf16_grouped(int32_t groups, int32_t gdim, int32_t M, int32_t N, int32_t K,
                                const void* const* A, int64_t lda, int32_t ta,
                                const void* const* B, int64_t ldb, int32_t tb,

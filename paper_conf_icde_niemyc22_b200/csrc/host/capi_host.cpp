@@ -106,6 +106,8 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
     pr = &local;
   }
   ts_status st = plan_greedy(g->g, budget_bytes, *pr, p->st, flags);
+  // the first run's message (the analytic-cost run below may overwrite the thread's error)
+  const std::string first_error = st == TS_OK ? std::string() : std::string(ts_last_error());
   // With a measured profile, Alg. 2 also runs on the analytic cost model and that plan is
   // re-scored on the measured timeline: the greedy's single path depends on the costs it sees
   // (profiles/r1_plan_variants.txt: the measured-cost greedy runs out of candidates on VGG-16
@@ -127,7 +129,6 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
   }
   // Alg. 2 is greedy and path-dependent: when it runs out of candidates, plan again for a
   // slightly tighter budget (different early decisions); any plan found fits the real one
-  const std::string first_error = st == TS_OK ? std::string() : std::string(ts_last_error());
   for (int k = 1; st == TS_ERR_INFEASIBLE && k <= 6; ++k) {
     const uint64_t tight = g->g.static_bytes + uint64_t(double(budget_bytes - g->g.static_bytes) * (1.0 - 0.03 * k));
     if (tight <= g->g.static_bytes) break;
@@ -297,27 +298,59 @@ ts_status ts_plan_grad_buckets(const ts_plan_t* p, uint64_t bucket_bytes, int64_
   return TS_OK;
 }
 
-// Serialized form: magic, n_tensors, budget, then (opt, p, dim, lead) per tensor, then the
-// D-LRU recompute cache limit.
+namespace {
+// FNV-1a over everything that shapes a plan: samples, dtype, every tensor's (dtype, kind,
+// shape) and every op's (kind, inputs, outputs, attributes).
+uint64_t graph_fingerprint(const Graph& g) {
+  uint64_t h = 1469598103934665603ull;
+  auto mix = [&](int64_t v) {
+    for (int b = 0; b < 8; ++b) {
+      h ^= uint64_t(v >> (8 * b)) & 0xFF;
+      h *= 1099511628211ull;
+    }
+  };
+  mix(g.samples);
+  mix(g.dtype);
+  for (const Tensor& t : g.t) {
+    mix(t.dtype);
+    mix(t.kind);
+    mix(t.ndim);
+    for (int d = 0; d < t.ndim; ++d) mix(t.shape[d]);
+  }
+  for (const Op& o : g.ops) {
+    mix(o.kind);
+    for (int i : o.in) mix(i);
+    for (int i : o.out) mix(1000000 + i);
+    for (int64_t a : o.ia) mix(a);
+  }
+  return h;
+}
+constexpr int32_t kPlanMagic = 0x54535032;  // 'TSP2'
+}  // namespace
+
+// Serialized form (int32 words): magic, n_tensors, budget (u64), graph fingerprint (u64),
+// then (opt, p, dim, lead) per tensor, then the D-LRU recompute cache limit (u64).
 ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n) {
   if (!p || !n) return set_error("null argument"), TS_ERR_ARG;
   const int nt = p->graph->n();
-  uint64_t need = 16 + 16ull * nt + 8;
+  uint64_t need = 24 + 16ull * nt + 8;
   *n = need;
   if (!buf) return TS_OK;
   if (cap < need) return set_error("buffer too small"), TS_ERR_ARG;
   auto* w = static_cast<int32_t*>(buf);
-  w[0] = 0x54535031;  // 'TSP1'
+  w[0] = kPlanMagic;
   w[1] = nt;
   std::memcpy(w + 2, &p->budget, 8);
+  const uint64_t fp = graph_fingerprint(*p->graph);
+  std::memcpy(w + 4, &fp, 8);
   for (int t = 0; t < nt; ++t) {
     const Cfg& c = p->st.cfg[t];
-    w[4 + 4 * t + 0] = c.opt;
-    w[4 + 4 * t + 1] = c.p;
-    w[4 + 4 * t + 2] = c.dim;
-    w[4 + 4 * t + 3] = c.lead;
+    w[6 + 4 * t + 0] = c.opt;
+    w[6 + 4 * t + 1] = c.p;
+    w[6 + 4 * t + 2] = c.dim;
+    w[6 + 4 * t + 3] = c.lead;
   }
-  std::memcpy(w + 4 + 4 * nt, &p->st.cache, 8);
+  std::memcpy(w + 6 + 4 * nt, &p->st.cache, 8);
   return TS_OK;
 }
 
@@ -325,21 +358,27 @@ ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, 
   if (!g || !buf || !out) return set_error("null argument"), TS_ERR_ARG;
   auto* r = static_cast<const int32_t*>(buf);
   const int nt = g->g.n();
-  if (n < 16 || r[0] != 0x54535031 || r[1] != nt || n < 16 + 16ull * nt + 8)
-    return set_error("not a plan for this graph"), TS_ERR_ARG;
+  if (n < 24 || r[0] != kPlanMagic || r[1] != nt || n < 24 + 16ull * nt + 8)
+    return set_error("not a serialized plan for a graph of this size"), TS_ERR_ARG;
+  uint64_t fp = 0;
+  std::memcpy(&fp, r + 4, 8);
+  if (fp != graph_fingerprint(g->g)) return set_error("the plan was made for another graph (fingerprint)"), TS_ERR_ARG;
+  // every entry passes the checks ts_plan_set applies (opt / p / dim / lead legality), and
+  // the whole assignment the channel-chain rule (D-CH), before anything is adopted
+  std::vector<ts_tensor_cfg> cfgs(nt);
+  for (int t = 0; t < nt; ++t) {
+    cfgs[t].tensor_id = t;
+    cfgs[t].opt = static_cast<ts_opt>(r[6 + 4 * t]);
+    cfgs[t].p_num = r[6 + 4 * t + 1];
+    cfgs[t].dim = r[6 + 4 * t + 2];
+    cfgs[t].prefetch_lead = r[6 + 4 * t + 3];
+    if (!cfg_fields_ok(g->g, &cfgs[t])) return TS_ERR_ARG;
+  }
   std::unique_ptr<ts_plan_t> p(new_plan(g));
   std::memcpy(&p->budget, r + 2, 8);
-  for (int t = 0; t < nt; ++t) {
-    Cfg& c = p->st.cfg[t];
-    c.opt = r[4 + 4 * t];
-    c.p = r[4 + 4 * t + 1];
-    c.dim = r[4 + 4 * t + 2];
-    c.lead = r[4 + 4 * t + 3];
-  }
-  std::memcpy(&p->st.cache, r + 4 + 4 * nt, 8);
-  Profile pr;
-  profile_analytic(g->g, default_hw(), pr);
-  plan_refresh(g->g, p->st, &pr);
+  std::memcpy(&p->st.cache, r + 6 + 4 * nt, 8);
+  ts_status st = apply_cfgs(p.get(), cfgs.data(), nt);
+  if (st != TS_OK) return st;
   *out = p.release();
   return TS_OK;
 }

@@ -1664,6 +1664,9 @@ ts_status ts_gemm_bf16_grouped(int32_t groups, int32_t gdim, int32_t M, int32_t 
                                const void* const* bias, void* stream) {
   if (groups < 1 || groups > tsk::kMaxGroups || gdim < 1 || gdim > 3 || !A || !B || !C)
     return set_error("grouped gemm: 1 <= groups <= 3, gdim in {1, 2, 3}, A/B/C arrays required"), TS_ERR_ARG;
+  const int32_t ext = gdim == 1 ? N : (gdim == 2 ? K : M);
+  if (ext % groups != 0) return set_error("grouped gemm: the grouped extent must be a multiple of groups"), TS_ERR_ARG;
+  if (beta != 0.f && beta != 1.f) return set_error("grouped gemm: beta must be 0 or 1"), TS_ERR_ARG;
   tsk::GemmArgs g;
   g.M = M; g.N = N; g.K = K; g.in_dtype = tsk::BF16;
   g.groups = groups; g.gdim = gdim;

@@ -290,3 +290,28 @@ def test_channel_plan_serialize_roundtrip():
     assert Q.trace() == P.trace()
     for t in brute.act_tensors(g):
         assert (Q.get(t), Q.get_dim(t)) == (P.get(t), P.get_dim(t))
+
+
+def test_plan_deserialize_rejects_bad_blobs():
+    """ts_plan_deserialize validates like ts_plan_set: a blob of another graph (fingerprint),
+    a truncated one, p = 0 / 3, a swapped parameter — TS_ERR_ARG, nothing adopted."""
+    import struct
+    g = graphs.config_graph("bert_tiny")
+    G = tsplit.Graph(g)
+    blob = bytearray(tsplit.Plan.default(G).serialize())
+    tsplit.Plan.deserialize(G, bytes(blob))  # the round trip itself is fine
+    other = tsplit.Graph(graphs.config_graph("bert_tiny", hidden=256, heads=4))
+    with pytest.raises(tsplit.TsError):
+        tsplit.Plan.deserialize(other, bytes(blob))
+    g2 = tsplit.Graph(graphs.config_graph("bert_tiny", batch=8))  # same tensor count, other shapes
+    with pytest.raises(tsplit.TsError):
+        tsplit.Plan.deserialize(g2, bytes(blob))
+    with pytest.raises(tsplit.TsError):
+        tsplit.Plan.deserialize(G, bytes(blob[:-12]))
+    act = brute.act_tensors(g)[0]
+    param = next(t["id"] for t in g["tensors"] if t["kind"] == "param")
+    for tid, word, value in ((act, 1, 0), (act, 1, 3), (param, 0, tsplit.SWAP)):
+        bad = bytearray(blob)
+        struct.pack_into("<i", bad, 24 + 16 * tid + 4 * word, value)
+        with pytest.raises(tsplit.TsError):
+            tsplit.Plan.deserialize(G, bytes(bad))
