@@ -505,11 +505,20 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       if (x.kind != TS_ACT || x.is_loss || ps.cfg[t].opt != TS_RESIDE || own.count(t)) continue;
       if (first_bw[t] < 0) continue;                 // not held for backward: nothing to gain
       if (!bwd_phase && last_fw[t] >= bi) continue;  // still read later in the forward pass
-      if (bwd_phase && first_bw[t] - std::max(1, ps.cfg[t].lead) <= bi) continue;
+      if (bwd_phase && first_bw[t] <= bi) continue;  // read by the bottleneck or before it
       double dm = double(x.bytes);
       Cand2 c;
       c.birth = birth[t];
       c.tensor = t;
+      // a recompute replays in the group of the first backward reader, after the bottleneck,
+      // so it frees t there even when that reader is the very next item; a swap-in lands
+      // `lead` compute items earlier, so it frees t only when that is still after bi
+      if (bwd_phase && first_bw[t] - std::max(1, ps.cfg[t].lead) <= bi) {
+        c.ch = {{t, TS_RECOMPUTE, ps.cfg[t].p, 1}};
+        c.analytic = double(bw_ops[t].size()) * rc_time(rc_time, t, 0) / dm;
+        step1.push_back(with_feeders(c, t));
+        continue;
+      }
       c.ch = {{t, TS_SWAP, ps.cfg[t].p, 1}};
       c.analytic = swap_cost(t, dm) / dm;
       step1.push_back(c);
@@ -747,6 +756,9 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
                    best->ch[0].p, best->ch[0].lead, best_ratio, 1e3 * ps.predicted_s);
     if (!best && log) {
       std::fprintf(stderr, "stuck at item %d op %d (%s): live tensors\n", bi, bop, bwd_phase ? "bwd" : "fwd");
+      for (int t = 0; t < n; ++t)
+        if (ps.cfg[t].opt != TS_RESIDE || ps.cfg[t].p != 1)
+          std::fprintf(stderr, "  cfg t=%d opt=%d p=%d\n", t, ps.cfg[t].opt, ps.cfg[t].p);
       for (int t : live)
         std::fprintf(stderr, "  t=%d opt=%d p=%d bytes=%llu own=%d first_bw=%d last_fw=%d\n", t, ps.cfg[t].opt,
                      ps.cfg[t].p, (unsigned long long)g.t[t].bytes, (int)own.count(t), first_bw[t], last_fw[t]);

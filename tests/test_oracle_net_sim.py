@@ -212,6 +212,48 @@ def test_t7_eq3_special_cases():
     assert cost.eq3_swap_cost(S, B, B, T2, [1.0] * 10, 0, 9, 2, 9) == pytest.approx(2 * S / B)
 
 
+def test_eq2_delta_m_is_the_size_by_simulation():
+    """Eq. 2: swapping or recomputing a tensor that is live across op i but
+    not touched by it lowers the memory requirement at op i by exactly size(s_j) (256-B
+    aligned pieces) — checked against the simulator's live bytes, not restated."""
+    g = graphs.mlp()
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    base = sim.simulate(g)
+    t = names["relu0"]  # held for fc1's backward, not read by relu1 / fc2 / loss forward
+    for opt in (sim.SWAP, sim.RECOMPUTE):
+        cfg = sim.default_cfg(g)
+        cfg[t] = (opt, 1, 1)
+        if opt == sim.RECOMPUTE:  # the replay's input fc0 is recomputed too (else it is held instead)
+            cfg[names["fc0"]] = (sim.RECOMPUTE, 1, 1)
+        r = sim.simulate(g, cfg)
+        for op_name in ("relu1", "fc2", "loss"):
+            i0 = next(i for i, it in enumerate(base.items) if it.kind == "F" and g["ops"][it.op]["name"] == op_name)
+            i1 = next(i for i, it in enumerate(r.items) if it.kind == "F" and g["ops"][it.op]["name"] == op_name)
+            dm = base.live_after_alloc[i0] - r.live_after_alloc[i1]
+            assert dm == sim.align(cost.eq2_delta_m(sim.tbytes(g["tensors"][t]))), (opt, op_name, dm)
+
+
+def test_eq6_split_term_equals_the_planner_timeline():
+    """Eq. 6 (reading R7) with c = reside: the cost of splitting is the
+    dT_split term alone, sum_k T(op on split k) - T(op), over every op whose micro-op count
+    changes.  The C++ planner's predicted step time (D-TIME timeline over the analytic
+    profile) must move by exactly that when a tensor is split 2 or 4 ways."""
+    from paper_conf_icde_niemyc22_b200 import tsplit
+    g = graphs.mlp()
+    G = tsplit.Graph(g)
+    prof = tsplit.Profile(G)
+    base = tsplit.Plan.default(G).stats()["predicted_s"]
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    for name, p in (("relu0", 2), ("fc1", 4), ("relu1", 2)):
+        t = names[name]
+        P = tsplit.Plan.default(G)
+        P.set(t, tsplit.RESIDE, p, 1)
+        got = P.stats()["predicted_s"] - base
+        touched = [o for o, op in enumerate(g["ops"]) if t in op["inputs"] + op["outputs"]]
+        want = sum(cost.eq6_split_cost(p, 0.0, sum(prof.get(o, p)), sum(prof.get(o, 1))) for o in touched)
+        assert got == pytest.approx(want, rel=1e-9, abs=1e-15), (name, got, want)
+
+
 # ------------------------------------------------------------ T9 brute force
 def _tiny():
     return graphs.mlp(batch=4, hidden=8, depth=2, in_dim=8, classes=3)
