@@ -356,7 +356,7 @@ def main():
     plan_trials = {}
     if rank == 0:
         # profile every op (and split widths) on the GPU before planning
-        prof = tsplit.Profile.measure(G, dev_inputs, max_p=4, device=local) if not args.analytic_profile else None
+        prof = tsplit.Profile.measure(G, dev_inputs, max_p=16, device=local) if not args.analytic_profile else None
         pcie = prof.pcie() if prof else None
         plan_profile = "measured" if prof else "analytic"
         # Alg. 2 is a path-dependent greedy heuristic: plan with the measured profile and with
@@ -408,7 +408,8 @@ def main():
                     for t in spec["tensors"] if t["kind"] in ("input", "label"))
 
     def make_session(p):
-        s = tsplit.Session(G, p, device=local, lr=1e-4, streams=streams, nccl_comm=comm, world_size=world)
+        s = tsplit.Session(G, p, device=local, lr=1e-4, streams=streams, nccl_comm=comm, world_size=world,
+                           sample_offset=rank * spec["samples"])
         s.set_params(params)
         return s
 

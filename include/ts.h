@@ -181,7 +181,9 @@ void ts_profile_destroy(ts_profile_t* pr);
  * one cudaEvent-timed eager step of the all-reside plan with every activation split p
  * ways, on the caller's scratch `slab` (device, >= the unsplit peak; parameters are
  * zero — op times do not depend on the data), and records each op's forward
- * and backward time; wider splits reuse the widest measured one.  Also measures pinned
+ * and backward time (per-item median of three timed steps).  p values above max_p or
+ * the batch (p must divide it) extrapolate from the widest measured one (+5 % per
+ * doubling: the launch / tail overhead of one more level of micro-ops).  Also measures pinned
  * D2H/H2D bandwidth (256 MiB copies).  `inputs` as in ts_step. */
 ts_status ts_profile_measure(const ts_graph_t* g, void* slab, uint64_t slab_bytes, const void* const* inputs,
                              int32_t inputs_on_host, int32_t max_p, ts_profile_t** out);
@@ -256,6 +258,12 @@ typedef struct {
   int32_t use_cuda_graph;    /* capture the whole step once and replay it             */
   float lr;                  /* SGD learning rate (0 = no update)                     */
   uint32_t step0;            /* dropout counter base                                  */
+  int64_t sample_offset;     /* global index of this rank's first sample: dropout
+                                counters (R15) use global sample indices, so the N ranks
+                                of a data-parallel step draw disjoint masks and together
+                                compute the step of the concatenated batch (0 on 1 GPU)   */
+  int32_t host_numa_node;    /* NUMA node of the pinned swap pool: >= 0 that node, -1 the
+                                GPU's own node (sysfs), -2 no binding (cudaHostAlloc)     */
 } ts_session_cfg;
 
 /* Lays out the static region, allocates the pinned host swap pool, uploads
@@ -280,6 +288,9 @@ ts_status ts_step(ts_session_t* s, const void* const* inputs, int32_t inputs_on_
 ts_status ts_step_async(ts_session_t* s, const void* const* inputs, int32_t inputs_on_host);
 /* Allocation trace the runtime recorded on its last step (must equal ts_plan_trace). */
 ts_status ts_session_trace(const ts_session_t* s, ts_alloc_event* buf, uint64_t cap, uint64_t* n);
+/* The pinned host swap pool: bytes (= the plan's swapped bytes, 256-B slots) and the NUMA
+ * node its pages are bound to (-1: unbound / unknown). */
+ts_status ts_session_host_pool(const ts_session_t* s, uint64_t* bytes, int32_t* numa_node);
 /* Kernel launches per step issued by the session (for gpu_launches accounting). */
 ts_status ts_session_launches(const ts_session_t* s, int64_t* n);
 /* Device time of the last step's compute-stream items, by op kind and phase

@@ -8,9 +8,14 @@
 // copied out waits on that copy's event.  Recompute replays re-run
 // the producer's forward micro-op (memory-centric).
 #include <dlfcn.h>
+#include <sys/mman.h>
+#include <sys/syscall.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <array>
+#include <cctype>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 #include <functional>
@@ -84,6 +89,10 @@ struct ts_session_s {
   int64_t graph_kernels = 0;
   char* host = nullptr;
   uint64_t host_bytes = 0;
+  int host_numa_req = -1;     // requested node (-1 GPU's own, -2 none)
+  int host_numa = -1;         // node the pool is bound to (-1: unbound)
+  bool host_registered = false;  // mmap + cudaHostRegister (else cudaHostAlloc)
+  int64_t sample0 = 0;        // global index of this rank's first sample (dropout counters)
   std::vector<Cmd> prog;
   std::vector<cudaEvent_t> ev_d2h, ev_h2d;  // indexed by item
   cudaEvent_t ev_mark = nullptr, ev_join_d2h = nullptr, ev_join_h2d = nullptr;
@@ -228,7 +237,8 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
   };
   const Tensor& out = g.t[o.out[0]];
   const int64_t n_out = (out.sample ? ns * out.elems_per_sample : out.numel) / (m.cb >= 0 ? m.cp : 1);
-  const int64_t elem0 = out.sample ? m.s0 * out.elems_per_sample : 0;
+  // dropout counters index the GLOBAL batch: a data-parallel rank's samples start at sample0
+  const int64_t elem0 = out.sample ? (m.s0 + s->sample0) * out.elems_per_sample : 0;
   const uint32_t* stepp = s->step_dev;
   switch (o.kind) {
     case TS_OP_LINEAR: {
@@ -652,7 +662,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       a.alpha = float(o.fa[0]);
       a.p = float(o.fa[1]);
       a.seed = uint32_t(o.ia[2]);
-      a.b0 = m.s0;
+      a.b0 = m.s0 + s->sample0;  // Philox sample index (global batch)
       a.ws = ws;
       if (!bwd) {
         // a replay writes only the output it regenerates
@@ -701,6 +711,51 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
   return [](cudaStream_t) {};
 }
 
+// NUMA node of the session's GPU from sysfs (-1 if unknown)
+int gpu_numa_node(int device) {
+  char bus[64] = {0};
+  if (cudaDeviceGetPCIBusId(bus, sizeof(bus), device) != cudaSuccess) return -1;
+  for (char* c = bus; *c; ++c) *c = char(std::tolower(*c));
+  const std::string path = std::string("/sys/bus/pci/devices/") + bus + "/numa_node";
+  FILE* f = std::fopen(path.c_str(), "r");
+  if (!f) return -1;
+  int node = -1;
+  if (std::fscanf(f, "%d", &node) != 1) node = -1;
+  std::fclose(f);
+  return node;
+}
+
+// The pinned swap pool, on the GPU's NUMA node (north_star: each GPU swaps over its own
+// PCIe link to host memory next to it): anonymous pages bound with mbind(MPOL_PREFERRED)
+// before first touch, then page-locked with cudaHostRegister.  Where binding is not
+// possible (no node, mbind refused) the pages stay unbound; where registration fails,
+// cudaHostAlloc.  Host memory either way — the copies are the same DMA transfers.
+bool alloc_host_pool(ts_session_t* s, uint64_t bytes) {
+  int node = s->host_numa_req == -1 ? gpu_numa_node(s->device) : s->host_numa_req;
+  if (s->host_numa_req != -2) {
+    void* p = mmap(nullptr, bytes, PROT_READ | PROT_WRITE, MAP_PRIVATE | MAP_ANONYMOUS, -1, 0);
+    if (p != MAP_FAILED) {
+      bool bound = false;
+      if (node >= 0 && node < 1024) {
+        unsigned long mask[1024 / (8 * sizeof(unsigned long))] = {0};
+        mask[node / (8 * sizeof(unsigned long))] |= 1ul << (node % (8 * sizeof(unsigned long)));
+        constexpr int kMpolPreferred = 1;
+        bound = syscall(SYS_mbind, p, bytes, kMpolPreferred, mask, 1024ul, 0u) == 0;
+      }
+      if (cudaHostRegister(p, bytes, cudaHostRegisterDefault) == cudaSuccess) {
+        s->host = static_cast<char*>(p);
+        s->host_registered = true;
+        s->host_numa = bound ? node : -1;
+        return true;
+      }
+      cudaGetLastError();
+      munmap(p, bytes);
+    }
+  }
+  s->host_numa = -1;
+  return cudaHostAlloc(reinterpret_cast<void**>(&s->host), bytes, cudaHostAllocDefault) == cudaSuccess;
+}
+
 ts_status build_program(ts_session_t* s) {
   const Graph& g = *s->g;
   const int n = g.n();
@@ -722,11 +777,9 @@ ts_status build_program(ts_session_t* s) {
       }
     }
   s->host_bytes = hb;
-  if (hb) {
-    if (cudaHostAlloc(reinterpret_cast<void**>(&s->host), hb, cudaHostAllocDefault) != cudaSuccess) {
-      set_error("cudaHostAlloc of the swap pool failed");
-      return TS_ERR_HOST_MEM;
-    }
+  if (hb && !alloc_host_pool(s, hb)) {
+    set_error("pinned host allocation of the swap pool (" + std::to_string(hb) + " B) failed");
+    return TS_ERR_HOST_MEM;
   }
   // replay the trace: per item, the offset of every live piece
   std::unordered_map<PieceKey, uint64_t> where;
@@ -1305,6 +1358,8 @@ ts_status ts_session_create(const ts_graph_t* gh, const ts_plan_t* ph, const ts_
   s->world = cfg->world_size > 0 ? cfg->world_size : 1;
   s->lr = cfg->lr;
   s->step = cfg->step0;
+  s->sample0 = cfg->sample_offset;
+  s->host_numa_req = cfg->host_numa_node;
   s->use_graph = cfg->use_cuda_graph != 0;
   if (cfg->stream_compute) {
     s->cs = static_cast<cudaStream_t>(cfg->stream_compute);
@@ -1353,7 +1408,12 @@ void ts_session_destroy(ts_session_t* s) {
   if (s->ev_mark) cudaEventDestroy(s->ev_mark);
   if (s->ev_join_d2h) cudaEventDestroy(s->ev_join_d2h);
   if (s->ev_join_h2d) cudaEventDestroy(s->ev_join_h2d);
-  if (s->host) cudaFreeHost(s->host);
+  if (s->host && s->host_registered) {
+    cudaHostUnregister(s->host);
+    munmap(s->host, s->host_bytes);
+  } else if (s->host) {
+    cudaFreeHost(s->host);
+  }
   if (s->own_streams) {
     cudaStreamDestroy(s->cs);
     cudaStreamDestroy(s->d2h);
@@ -1384,6 +1444,13 @@ ts_status ts_get_grad(ts_session_t* s, int32_t t, float* host) {
   if (!s || !host || t < 0 || t >= s->g->n() || s->g->t[t].kind != TS_PARAM) return set_error("bad param"), TS_ERR_ARG;
   CU(cudaStreamSynchronize(s->cs));
   CU(cudaMemcpy(host, s->slab + s->g->grad_off[t], s->g->t[t].numel * 4, cudaMemcpyDeviceToHost));
+  return TS_OK;
+}
+
+ts_status ts_session_host_pool(const ts_session_t* s, uint64_t* bytes, int32_t* numa_node) {
+  if (!s || !bytes || !numa_node) return set_error("null argument"), TS_ERR_ARG;
+  *bytes = s->host_bytes;
+  *numa_node = s->host_numa;
   return TS_OK;
 }
 

@@ -60,7 +60,8 @@ class SessionCfg(C.Structure):
     _fields_ = [("device", C.c_int32), ("slab", C.c_void_p), ("slab_bytes", C.c_uint64),
                 ("stream_compute", C.c_void_p), ("stream_d2h", C.c_void_p), ("stream_h2d", C.c_void_p),
                 ("nccl_comm", C.c_void_p), ("world_size", C.c_int32), ("use_cuda_graph", C.c_int32),
-                ("lr", C.c_float), ("step0", C.c_uint32)]
+                ("lr", C.c_float), ("step0", C.c_uint32), ("sample_offset", C.c_int64),
+                ("host_numa_node", C.c_int32)]
 
 
 class TsError(RuntimeError):
@@ -119,6 +120,7 @@ def lib():
             "ts_step_async": (i32, [vp, P(vp), i32]),
             "ts_session_trace": (i32, [vp, P(AllocEvent), u64, P(u64)]),
             "ts_session_launches": (i32, [vp, P(i64)]),
+            "ts_session_host_pool": (i32, [vp, P(u64), P(i32)]),
             "ts_session_profile_items": (i32, [vp, i32]),
             "ts_session_item_times": (i32, [vp, P(C.c_float), u64, P(u64)]),
             "ts_session_gemm_times": (i32, [vp, P(C.c_double), P(C.c_float), P(i32), u64, P(u64)]),
@@ -230,7 +232,7 @@ class Profile:
         self.h = h
 
     @classmethod
-    def measure(cls, graph: Graph, inputs: dict, max_p: int = 4, device: int = 0):
+    def measure(cls, graph: Graph, inputs: dict, max_p: int = 16, device: int = 0):
         """Measured profile (ts_profile_measure) on a scratch slab of the unsplit peak."""
         import torch
         peak = Plan.default(graph).stats()["peak_extent"]
@@ -390,7 +392,8 @@ class Session:
 
     def __init__(self, graph: Graph, plan: Plan, device: int = 0, slab_bytes: int | None = None,
                  lr: float = 0.0, use_cuda_graph: bool = True, nccl_comm: int | None = None,
-                 world_size: int = 1, step0: int = 0, streams=None):
+                 world_size: int = 1, step0: int = 0, streams=None, sample_offset: int = 0,
+                 host_numa_node: int = -1):
         import torch
         if not torch.cuda.is_available():
             raise TsError(9, "no CUDA device: the TSPLIT runtime has no CPU fallback")
@@ -410,6 +413,8 @@ class Session:
         cfg.use_cuda_graph = 1 if use_cuda_graph else 0
         cfg.lr = lr
         cfg.step0 = step0
+        cfg.sample_offset = sample_offset
+        cfg.host_numa_node = host_numa_node
         h = C.c_void_p()
         check(lib().ts_session_create(graph.h, plan.h, C.byref(cfg), C.byref(h)))
         self.h = h
@@ -444,6 +449,12 @@ class Session:
         loss = C.c_float()
         check(lib().ts_step(self.h, self._ptrs(inputs), 1 if on_host else 0, C.byref(loss)))
         return loss.value
+
+    def host_pool(self):
+        """(bytes, NUMA node or -1) of the pinned swap pool."""
+        b, n = C.c_uint64(), C.c_int32()
+        check(lib().ts_session_host_pool(self.h, C.byref(b), C.byref(n)))
+        return b.value, n.value
 
     def step_async(self, inputs: dict, on_host: bool = False):
         check(lib().ts_step_async(self.h, self._ptrs(inputs), 1 if on_host else 0))

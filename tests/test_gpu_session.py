@@ -353,3 +353,31 @@ def test_bert_small_bf16_random_plans(seed):
     _, u1, _, _ = _run_unfused(g, plan_cfg=cfg)
     _, u0, _, _ = _run_unfused(g)
     assert global_rel_err(u1, u0) <= 1e-3
+
+
+def test_profile_measure_times_every_split_width():
+    """a2 ("profiles every single operation before training", P:L281 cudaEvent,
+    P:L125 Fig. 5): ts_profile_measure times every op's forward and backward at p = 1, 2,
+    4, 8 (batch 8 bounds the sample split), with the per-micro-op degradation the planner
+    must see — the GEMM-heavy ops cost more as 8 micro-ops than as one — and measures the
+    pinned PCIe bandwidth; the planner plans with it."""
+    g = graphs.config_graph("bert_small", fused_attention=True)
+    G = tsplit.Graph(g)
+    dev = tsplit.inputs_to_device(G, gen.make_inputs(g))
+    prof = tsplit.Profile.measure(G, dev, max_p=16)
+    ana = tsplit.Profile(G)
+    names = [o["name"] for o in g["ops"]]
+    for o, op in enumerate(g["ops"]):
+        for p in (1, 2, 4, 8):
+            f, b = prof.get(o, p)
+            assert f > 0, (op["name"], p)
+            assert prof.get(o, p) != ana.get(o, p)  # measured, not the analytic model
+    ffn = [names.index(f"l{i}.ffn{j}") for i in range(2) for j in (1, 2)]
+    slower = [sum(prof.get(o, 8)) > sum(prof.get(o, 1)) for o in ffn]
+    assert all(slower), [(names[o], prof.get(o, 1), prof.get(o, 8)) for o in ffn]
+    d2h, h2d = prof.pcie()
+    assert 5e9 < d2h < 2e11 and 5e9 < h2d < 2e11, (d2h, h2d)
+    base = tsplit.Plan.default(G).stats()
+    budget = base["static_bytes"] + (base["peak_extent"] - base["static_bytes"]) // 3
+    P = tsplit.Plan.plan(G, budget, profile=prof)
+    assert P.stats()["peak_extent"] <= budget

@@ -37,7 +37,7 @@ def main():
     dev = tsplit.inputs_to_device(G, gen.make_inputs(spec))
     if frac > 0:
         st = P.stats()
-        prof = tsplit.Profile.measure(G, dev, max_p=4)
+        prof = tsplit.Profile.measure(G, dev, max_p=16)
         P = tsplit.Plan.plan(G, st["static_bytes"] + int(frac * (st["peak_extent"] - st["static_bytes"])), prof)
     params = gen.init_params(spec)
     res = {k: [] for k in VARIANTS}

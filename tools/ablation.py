@@ -80,7 +80,7 @@ for b in batches:
     G = tsplit.Graph(spec)
     dev = tsplit.inputs_to_device(G, gen.make_inputs(spec))
     t0 = time.time()
-    prof = tsplit.Profile.measure(G, dev, max_p=4)
+    prof = tsplit.Profile.measure(G, dev, max_p=16)
     prof_s = time.time() - t0
     for name, kw in VARIANTS.items():
         row = {"batch": b, "variant": name}

@@ -15,6 +15,6 @@ out = sys.argv[2] if len(sys.argv) > 2 else f"gpurun_out/profile_{wl}.json"
 spec = bench.workload_graph(wl)
 G = tsplit.Graph(spec)
 dev = tsplit.inputs_to_device(G, gen.make_inputs(spec))
-prof = tsplit.Profile.measure(G, dev, max_p=4)
+prof = tsplit.Profile.measure(G, dev, max_p=16)
 json.dump(prof.to_dict(), open(out, "w"))
 print("wrote", out)

@@ -19,7 +19,7 @@ G = tsplit.Graph(spec)
 st = tsplit.Plan.default(G).stats()
 budget = st["static_bytes"] + int(frac * (st["peak_extent"] - st["static_bytes"]))
 dev = tsplit.inputs_to_device(G, gen.make_inputs(spec))
-prof = tsplit.Profile.measure(G, dev, max_p=4)
+prof = tsplit.Profile.measure(G, dev, max_p=16)
 P = tsplit.Plan.plan(G, budget, prof)
 S = tsplit.Session(G, P, lr=1e-4, use_cuda_graph=(mode == "graph"))
 S.set_params(gen.init_params(spec))

@@ -19,7 +19,7 @@ G = tsplit.Graph(spec)
 st = tsplit.Plan.default(G).stats()
 budget = st["static_bytes"] + int(W["frac"] * (st["peak_extent"] - st["static_bytes"]))
 dev = tsplit.inputs_to_device(G, gen.make_inputs(spec))
-prof = tsplit.Profile.measure(G, dev, max_p=4)
+prof = tsplit.Profile.measure(G, dev, max_p=16)
 params = gen.init_params(spec, seed=1)
 out = {}
 for pname, pr in (("measured", prof), ("analytic", None)):

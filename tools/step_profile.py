@@ -42,7 +42,7 @@ def main():
     st = base.stats()
     budget = st["static_bytes"] + int(frac * (st["peak_extent"] - st["static_bytes"]))
     dev0 = tsplit.inputs_to_device(G, gen.make_inputs(spec))
-    prof = tsplit.Profile.measure(G, dev0, max_p=4)
+    prof = tsplit.Profile.measure(G, dev0, max_p=16)
     plan = tsplit.Plan.plan(G, budget, prof)
     print("plan stats", {k: v for k, v in plan.stats().items()})
     # tensors by opt
