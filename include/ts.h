@@ -293,8 +293,10 @@ ts_status ts_session_trace(const ts_session_t* s, ts_alloc_event* buf, uint64_t 
 ts_status ts_session_host_pool(const ts_session_t* s, uint64_t* bytes, int32_t* numa_node);
 /* Kernel launches per step issued by the session (for gpu_launches accounting). */
 ts_status ts_session_launches(const ts_session_t* s, int64_t* n);
-/* Device time of the last step's compute-stream items, by op kind and phase
- * (seconds, cudaEvent; only when profiling was enabled). */
+/* Profiling (eager steps, cudaEvent pairs): enable / disable; then per item of the
+ * augmented schedule (plan item order) the duration of its last execution in ms —
+ * compute items on the compute stream, swap-out / swap-in copies on the D2H / H2D
+ * stream (achieved PCIe bandwidth = piece bytes / copy time). */
 ts_status ts_session_profile_items(ts_session_t* s, int32_t enable);
 ts_status ts_session_item_times(const ts_session_t* s, float* ms, uint64_t cap, uint64_t* n);
 /* Per-GEMM-launch records of the last profiled step: algorithmic FLOP (0 for the SIMT

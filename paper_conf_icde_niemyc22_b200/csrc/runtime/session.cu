@@ -101,7 +101,7 @@ struct ts_session_s {
   std::vector<int> zero_grads;                   // params whose grad is accumulated atomically
   int64_t launches = 0;
   bool profile = false;
-  std::vector<cudaEvent_t> prof_ev;  // 2 per program command (compute items)
+  std::vector<cudaEvent_t> prof_ev;  // 2 per program command (compute items; copies on their stream)
   std::vector<float> item_ms;
   std::vector<tsk::GemmRecord> gemm_recs;
   std::vector<double> gemm_flop, gemm_ms;
@@ -1200,7 +1200,9 @@ void issue_step(ts_session_t* s) {
     } else if (c.kind == 1) {
       cudaEventRecord(s->ev_mark, cs);
       cudaStreamWaitEvent(s->d2h, s->ev_mark, 0);
+      if (prof) cudaEventRecord(s->prof_ev[2 * c.item], s->d2h);
       cudaMemcpyAsync(s->host + c.host_off, c.dev, c.bytes, cudaMemcpyDeviceToHost, s->d2h);
+      if (prof) cudaEventRecord(s->prof_ev[2 * c.item + 1], s->d2h);
       cudaEventRecord(s->ev_d2h[c.item], s->d2h);
       d2h_used = true;
     } else {
@@ -1208,7 +1210,9 @@ void issue_step(ts_session_t* s) {
       cudaStreamWaitEvent(s->h2d, s->ev_mark, 0);
       cudaStreamWaitEvent(s->h2d, s->ev_d2h[c.so_of_piece], 0);
       for (int so : c.wait_so) cudaStreamWaitEvent(s->h2d, s->ev_d2h[so], 0);
+      if (prof) cudaEventRecord(s->prof_ev[2 * c.item], s->h2d);
       cudaMemcpyAsync(c.dev, s->host + c.host_off, c.bytes, cudaMemcpyHostToDevice, s->h2d);
+      if (prof) cudaEventRecord(s->prof_ev[2 * c.item + 1], s->h2d);
       cudaEventRecord(s->ev_h2d[c.item], s->h2d);
       h2d_used = true;
     }
@@ -1323,7 +1327,7 @@ ts_status run_step(ts_session_t* s, const void* const* inputs, int on_host) {
     }
     s->item_ms.assign(s->prog.size(), 0.f);
     for (auto& c : s->prog)
-      if (c.kind == 0) cudaEventElapsedTime(&s->item_ms[c.item], s->prof_ev[2 * c.item], s->prof_ev[2 * c.item + 1]);
+      cudaEventElapsedTime(&s->item_ms[c.item], s->prof_ev[2 * c.item], s->prof_ev[2 * c.item + 1]);
   }
   return TS_OK;
 }

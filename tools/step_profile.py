@@ -30,7 +30,7 @@ def profile(G, P, spec, params, dev):
         cnt[key] += 1
     del S
     torch.cuda.empty_cache()
-    return agg, cnt, sum(ms)
+    return agg, cnt, sum(t for (kind, _, _, _), t in zip(items, ms) if kind not in ("SO", "SI"))
 
 
 def main():
