@@ -111,6 +111,10 @@ typedef struct {
   int32_t p_num;         /* 1, 2, 4, 8, 16; must divide `samples` */
   int32_t dim;
   int32_t prefetch_lead; /* >= 1 */
+  int32_t release_lag;   /* swap only (reading D-LAG): the range a swap-out frees
+                            returns to the pool after this many compute items behind it
+                            (0: at the swap-out), so a later allocation does not wait on
+                            the copy (R12); capped before the swap-in */
 } ts_tensor_cfg;
 
 typedef struct {

@@ -81,6 +81,13 @@ def dim_of(cfg, t):
     return c[3] if c is not None and len(c) > 3 else 0
 
 
+def lag_of(cfg, t):
+    """Release lag of a swapped tensor (reading D-LAG): the number of compute
+    items after its swap-out before its range returns to the pool (0: at the swap-out)."""
+    c = cfg.get(t)
+    return c[4] if c is not None and len(c) > 4 else 0
+
+
 def check_channel(graph, cfg):
     """Raise ValueError when a channel-split configuration breaks reading D-CH."""
     ts, ops = graph["tensors"], graph["ops"]
@@ -460,6 +467,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
     alloc_at, free_after = {}, {}
     swap_out_after = {}       # forward item index -> [pieces]
     swap_in_before = {}       # pre-insertion item index -> [pieces]
+    lag_free = {}             # pre-insertion item index -> [swapped-out pieces freed after it]
     temp_spans = []
     for pc, idxs in touches.items():
         key, j = pc
@@ -486,6 +494,11 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
             pos = max(min(bw) - lead, fwd_end)
             swap_in_before.setdefault(pos, []).append(pc)
             free_after.setdefault(max(bw), []).append(pc)
+            # D-LAG: the range the swap-out frees returns to the pool only after the
+            # lag-th compute item behind it (the copy's time), and before the swap-in
+            q = min(max(fw) + lag_of(cfg, key), pos - 1)
+            if lag_of(cfg, key) > 0 and q > max(fw):
+                lag_free.setdefault(q, []).append(pc)
         else:  # RECOMPUTE: forward lifetime, then one residency per regeneration
             free_after.setdefault(max(fw), []).append(pc)
             # a residency starts at the replay writing the piece and ends at its last
@@ -522,12 +535,13 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
         assert len(ordered) == len(set(allocs)), (it, allocs)
         if ordered:
             f_alloc[idx] = ordered
-        if i in free_after:
-            f_free[idx] = sorted(free_after[i])
+        if i in free_after or i in lag_free:
+            f_free[idx] = sorted(free_after.get(i, []) + lag_free.get(i, []))
         for pc in sorted(swap_out_after.get(i, [])):
             so = Item("SO")
             so.reads = [pc]
-            f_free[len(final)] = [pc]
+            if not any(pc in v for v in lag_free.values()):
+                f_free[len(final)] = [pc]
             final.append(so)
     return final, f_alloc, f_free, fwd_end, an
 

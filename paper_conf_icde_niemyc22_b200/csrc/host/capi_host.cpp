@@ -105,7 +105,7 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
     profile_analytic(g->g, default_hw(), local);
     pr = &local;
   }
-  ts_status st = plan_greedy(g->g, budget_bytes, *pr, p->st, flags);
+  ts_status st = plan_greedy_lag(g->g, budget_bytes, *pr, p->st, flags);
   // the first run's message (the analytic-cost run below may overwrite the thread's error)
   const std::string first_error = st == TS_OK ? std::string() : std::string(ts_last_error());
   // With a measured profile, Alg. 2 also runs on the analytic cost model and that plan is
@@ -117,7 +117,7 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
   if (profile) {
     Profile ana;
     profile_analytic(g->g, default_hw(), ana);
-    if (plan_greedy(g->g, budget_bytes, ana, from_analytic, flags) == TS_OK) {
+    if (plan_greedy_lag(g->g, budget_bytes, ana, from_analytic, flags) == TS_OK) {
       plan_refresh(g->g, from_analytic, pr);  // predicted time on the measured profile
       have_analytic = true;
     }
@@ -133,7 +133,7 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
     const uint64_t tight = g->g.static_bytes + uint64_t(double(budget_bytes - g->g.static_bytes) * (1.0 - 0.03 * k));
     if (tight <= g->g.static_bytes) break;
     p->st = PlanState();
-    st = plan_greedy(g->g, tight, *pr, p->st, flags);
+    st = plan_greedy_lag(g->g, tight, *pr, p->st, flags);
   }
   if (st == TS_ERR_INFEASIBLE) set_error(first_error);
   if (st != TS_OK) return st;
@@ -144,7 +144,7 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
   // search space contains the "w/o Split" plan, so keep whichever predicts faster.
   if (!(flags & TS_PLAN_NO_SPLIT)) {
     PlanState alt;
-    if (plan_greedy(g->g, budget_bytes, *pr, alt, flags | TS_PLAN_NO_SPLIT) == TS_OK &&
+    if (plan_greedy_lag(g->g, budget_bytes, *pr, alt, flags | TS_PLAN_NO_SPLIT) == TS_OK &&
         alt.predicted_s < p->st.predicted_s)
       p->st = std::move(alt);
   }
@@ -161,6 +161,7 @@ ts_status ts_plan_get(const ts_plan_t* p, int32_t tid, ts_tensor_cfg* out) {
   out->p_num = c.p;
   out->dim = c.dim;
   out->prefetch_lead = c.lead;
+  out->release_lag = c.lag;
   return TS_OK;
 }
 
@@ -171,8 +172,10 @@ bool cfg_fields_ok(const Graph& g, const ts_tensor_cfg* cfg) {
   int t = cfg->tensor_id;
   if (t < 0 || t >= g.n()) return set_error("bad tensor id"), false;
   bool pow2 = cfg->p_num >= 1 && cfg->p_num <= 16 && (cfg->p_num & (cfg->p_num - 1)) == 0;
-  if (cfg->opt < 0 || cfg->opt > 2 || cfg->dim < 0 || cfg->dim > 1 || cfg->prefetch_lead < 1)
-    return set_error("bad opt/dim/prefetch_lead (dim 0 = samples, 1 = channels)"), false;
+  if (cfg->opt < 0 || cfg->opt > 2 || cfg->dim < 0 || cfg->dim > 1 || cfg->prefetch_lead < 1 ||
+      cfg->release_lag < 0 || (cfg->release_lag > 0 && cfg->opt != TS_SWAP))
+    return set_error("bad opt/dim/prefetch_lead/release_lag (dim 0 = samples, 1 = channels; a lag needs swap)"),
+           false;
   const Tensor& x = g.t[t];
   if (!pow2) return set_error("p_num must be a power of 2 <= 16"), false;
   if (cfg->dim == 0 && g.samples % cfg->p_num) return set_error("p_num must divide the samples"), false;
@@ -194,6 +197,7 @@ ts_status apply_cfgs(ts_plan_t* p, const ts_tensor_cfg* cfgs, int32_t n) {
     c.p = cfgs[i].p_num;
     c.dim = cfgs[i].p_num > 1 ? cfgs[i].dim : 0;
     c.lead = cfgs[i].prefetch_lead;
+    c.lag = cfgs[i].release_lag;
   }
   std::string why;
   if (!channel_ok(g, next, why)) return set_error("channel split (D-CH): " + why), TS_ERR_ARG;
@@ -325,15 +329,15 @@ uint64_t graph_fingerprint(const Graph& g) {
   }
   return h;
 }
-constexpr int32_t kPlanMagic = 0x54535032;  // 'TSP2'
+constexpr int32_t kPlanMagic = 0x54535033;  // 'TSP3'
 }  // namespace
 
 // Serialized form (int32 words): magic, n_tensors, budget (u64), graph fingerprint (u64),
-// then (opt, p, dim, lead) per tensor, then the D-LRU recompute cache limit (u64).
+// then (opt, p, dim, lead, lag) per tensor, then the D-LRU recompute cache limit (u64).
 ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n) {
   if (!p || !n) return set_error("null argument"), TS_ERR_ARG;
   const int nt = p->graph->n();
-  uint64_t need = 24 + 16ull * nt + 8;
+  uint64_t need = 24 + 20ull * nt + 8;
   *n = need;
   if (!buf) return TS_OK;
   if (cap < need) return set_error("buffer too small"), TS_ERR_ARG;
@@ -345,12 +349,13 @@ ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_
   std::memcpy(w + 4, &fp, 8);
   for (int t = 0; t < nt; ++t) {
     const Cfg& c = p->st.cfg[t];
-    w[6 + 4 * t + 0] = c.opt;
-    w[6 + 4 * t + 1] = c.p;
-    w[6 + 4 * t + 2] = c.dim;
-    w[6 + 4 * t + 3] = c.lead;
+    w[6 + 5 * t + 0] = c.opt;
+    w[6 + 5 * t + 1] = c.p;
+    w[6 + 5 * t + 2] = c.dim;
+    w[6 + 5 * t + 3] = c.lead;
+    w[6 + 5 * t + 4] = c.lag;
   }
-  std::memcpy(w + 6 + 4 * nt, &p->st.cache, 8);
+  std::memcpy(w + 6 + 5 * nt, &p->st.cache, 8);
   return TS_OK;
 }
 
@@ -358,7 +363,7 @@ ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, 
   if (!g || !buf || !out) return set_error("null argument"), TS_ERR_ARG;
   auto* r = static_cast<const int32_t*>(buf);
   const int nt = g->g.n();
-  if (n < 24 || r[0] != kPlanMagic || r[1] != nt || n < 24 + 16ull * nt + 8)
+  if (n < 24 || r[0] != kPlanMagic || r[1] != nt || n < 24 + 20ull * nt + 8)
     return set_error("not a serialized plan for a graph of this size"), TS_ERR_ARG;
   uint64_t fp = 0;
   std::memcpy(&fp, r + 4, 8);
@@ -368,15 +373,16 @@ ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, 
   std::vector<ts_tensor_cfg> cfgs(nt);
   for (int t = 0; t < nt; ++t) {
     cfgs[t].tensor_id = t;
-    cfgs[t].opt = static_cast<ts_opt>(r[6 + 4 * t]);
-    cfgs[t].p_num = r[6 + 4 * t + 1];
-    cfgs[t].dim = r[6 + 4 * t + 2];
-    cfgs[t].prefetch_lead = r[6 + 4 * t + 3];
+    cfgs[t].opt = static_cast<ts_opt>(r[6 + 5 * t]);
+    cfgs[t].p_num = r[6 + 5 * t + 1];
+    cfgs[t].dim = r[6 + 5 * t + 2];
+    cfgs[t].prefetch_lead = r[6 + 5 * t + 3];
+    cfgs[t].release_lag = r[6 + 5 * t + 4];
     if (!cfg_fields_ok(g->g, &cfgs[t])) return TS_ERR_ARG;
   }
   std::unique_ptr<ts_plan_t> p(new_plan(g));
   std::memcpy(&p->budget, r + 2, 8);
-  std::memcpy(&p->st.cache, r + 6 + 4 * nt, 8);
+  std::memcpy(&p->st.cache, r + 6 + 5 * nt, 8);
   ts_status st = apply_cfgs(p.get(), cfgs.data(), nt);
   if (st != TS_OK) return st;
   *out = p.release();

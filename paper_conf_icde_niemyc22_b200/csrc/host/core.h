@@ -68,6 +68,7 @@ ts_status build_graph(const ts_tensor_desc* td, int nt, const ts_op_desc* od, in
 
 struct Cfg {
   int opt = TS_RESIDE, p = 1, dim = 0, lead = 1;
+  int lag = 0;  // D-LAG: compute items after a swap-out before its range is reusable
 };
 
 // Piece = (key, j) with key = tensor id or n + id for the gradient of id.
@@ -170,6 +171,12 @@ struct PlanState {
 };
 void plan_refresh(const Graph& g, PlanState& ps, const Profile* pr);
 ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps, uint32_t flags = 0);
+// internal planner flag: Alg. 2 without D-LAG swap candidates (the post-pass may still add lags)
+constexpr uint32_t kPlanNoLag = 1u << 30;
+// Alg. 2 with D-LAG candidates, falling back to the run without them when that path dead-ends
+// (lagged swaps hold their range for the copy; a later bottleneck inside the window can leave
+// the greedy without candidates)
+ts_status plan_greedy_lag(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps, uint32_t flags = 0);
 void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps);
 
 }  // namespace ts

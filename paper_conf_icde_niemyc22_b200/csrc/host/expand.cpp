@@ -233,6 +233,8 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
     for (PieceKey p : items[i].reads) touches[p].push_back(i);
   }
   std::vector<std::vector<PieceKey>> alloc_at(nitems), free_after(nitems), so_after(nitems), si_before(nitems);
+  std::vector<std::vector<PieceKey>> lag_free(nitems);  // D-LAG: swapped-out pieces freed after item i
+  std::set<PieceKey> lagged;
   for (auto& [pc, idx] : touches) {
     std::sort(idx.begin(), idx.end());
     idx.erase(std::unique(idx.begin(), idx.end()), idx.end());
@@ -266,6 +268,13 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       int pos = std::max(first_bw - std::max(1, cfg[key].lead), ex.fwd_end);
       si_before[pos].push_back(pc);
       free_after[lastt].push_back(pc);
+      // D-LAG: the swapped-out range returns to the pool after the lag-th compute item
+      // behind the swap-out (the copy's time), always before the swap-in
+      const int q = std::min(last_fw + cfg[key].lag, pos - 1);
+      if (cfg[key].lag > 0 && q > last_fw) {
+        lag_free[q].push_back(pc);
+        lagged.insert(pc);
+      }
     } else {  // recompute: forward lifetime, then one residency per regeneration
       free_after[last_fw].push_back(pc);
       // a residency starts at the group's first replay writing the piece and ends at its
@@ -311,6 +320,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       if (std::find(al.begin(), al.end(), p) != al.end() && std::find(order.begin(), order.end(), p) == order.end())
         order.push_back(p);
     std::vector<PieceKey> fr = free_after[i];
+    fr.insert(fr.end(), lag_free[i].begin(), lag_free[i].end());
     std::sort(fr.begin(), fr.end());
     ex.alloc_at.push_back(order);
     ex.free_after.push_back(fr);
@@ -321,7 +331,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       so.kind = IT_SO;
       so.reads.push_back(pc);
       ex.alloc_at.push_back({});
-      ex.free_after.push_back({pc});
+      ex.free_after.push_back(lagged.count(pc) ? std::vector<PieceKey>{} : std::vector<PieceKey>{pc});
       fin.push_back(std::move(so));
     }
   }

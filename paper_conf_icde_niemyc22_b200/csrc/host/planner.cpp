@@ -230,6 +230,31 @@ void timeline(const Graph& g, const PlanState& ps, const Profile& pr, Timeline& 
   occ(busy_h2d, tl.oc_h2d);
 }
 
+// D-LAG release lag for swapping t in plan ps: the number of compute items after t's last
+// forward toucher whose timeline time covers the D2H copy of all its bytes (+25 %).
+int release_lag(const Graph& g, const PlanState& ps, const Timeline& tl, const Profile& pr, int t) {
+  const auto& items = ps.ex.items;
+  int last_fw = -1;
+  for (int i = 0; i < ps.ex.fwd_end && i < (int)items.size(); ++i) {
+    const Item& it = items[i];
+    if (it.kind == IT_SO || it.kind == IT_SI) continue;
+    for (PieceKey p : it.reads)
+      if (pk_key(p) == t) last_fw = i;
+    for (PieceKey p : it.writes)
+      if (pk_key(p) == t) last_fw = i;
+  }
+  if (last_fw < 0) return 0;
+  const double need = 1.25 * double(g.t[t].bytes) / pr.hw.d2h_bw;
+  double acc_t = 0;
+  int lag = 0;
+  for (size_t u = size_t(last_fw) + 1; u < items.size() && acc_t < need && lag < 4096; ++u) {
+    if (items[u].kind == IT_SO || items[u].kind == IT_SI) continue;
+    acc_t += tl.T[u];
+    ++lag;
+  }
+  return lag;
+}
+
 double flops_of(const Graph& g, const PlanState& ps) {
   double f = 0;
   for (auto& it : ps.ex.items) {
@@ -317,22 +342,45 @@ void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& 
     PlanState cand;
     if (try_cfg(cfg, cand) && cand.predicted_s < ps.predicted_s) ps = std::move(cand);
   }
-  // recompute -> swap with a prefetch lead that hides the copy behind compute
+  // swaps whose freed range is reused while the copy still runs: release it later (D-LAG)
+  for (int t = 0; t < n; ++t) {
+    if (ps.cfg[t].opt != TS_SWAP || ps.cfg[t].lag > 0) continue;
+    Timeline tl;
+    timeline(g, ps, pr, tl);
+    const int lag = release_lag(g, ps, tl, pr, t);
+    if (lag <= 0) continue;
+    std::vector<Cfg> cfg = ps.cfg;
+    cfg[t].lag = lag;
+    PlanState cand;
+    if (try_cfg(cfg, cand) && cand.predicted_s < ps.predicted_s - 1e-6) ps = std::move(cand);
+  }
+  // recompute -> swap with a prefetch lead that hides the copy behind compute, and the
+  // range released only after the copy (D-LAG)
   std::vector<std::pair<double, int>> rc;
   for (int t = 0; t < n; ++t)
     if (ps.cfg[t].opt == TS_RECOMPUTE) rc.push_back({double(g.t[t].bytes), t});
   std::sort(rc.begin(), rc.end(), [](auto& a, auto& b) { return a.first > b.first; });
   for (auto& [bytes, t] : rc) {
     (void)bytes;
+    Timeline tl;
+    timeline(g, ps, pr, tl);
+    const int lag = release_lag(g, ps, tl, pr, t);
+    bool done = false;
     for (int lead : {4, 16, 64}) {
-      std::vector<Cfg> cfg = ps.cfg;
-      cfg[t].opt = TS_SWAP;
-      cfg[t].lead = lead;
-      PlanState cand;
-      if (try_cfg(cfg, cand) && cand.predicted_s < ps.predicted_s - 1e-6) {
-        ps = std::move(cand);
-        break;
+      for (int lg : {lag, 0}) {
+        std::vector<Cfg> cfg = ps.cfg;
+        cfg[t].opt = TS_SWAP;
+        cfg[t].lead = lead;
+        cfg[t].lag = lg;
+        PlanState cand;
+        if (try_cfg(cfg, cand) && cand.predicted_s < ps.predicted_s - 1e-6) {
+          ps = std::move(cand);
+          done = true;
+          break;
+        }
+        if (lag == 0) break;
       }
+      if (done) break;
     }
   }
 }
@@ -477,9 +525,24 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       for (int u = p; u < q; ++u) bw += (1.0 - tl.oc_h2d[u]) * tl.T[u];
       return std::max(0.0, size / pr.hw.d2h_bw - fw) + std::max(0.0, size / pr.hw.h2d_bw - bw);
     };
+    // D-LAG: compute items after t's swap-out whose profiled time covers the copy of all its
+    // pieces at the D2H bandwidth (+25 %), so the freed range is reused after the copy ends
+    auto lag_for = [&](int t) -> int {
+      if (last_fw[t] < 0 || (flags & kPlanNoLag)) return 0;
+      const double need = 1.25 * double(g.t[t].bytes) / pr.hw.d2h_bw;
+      double acc_t = 0;
+      int lag = 0;
+      for (size_t u = size_t(last_fw[t]) + 1; u < items.size() && acc_t < need && lag < 4096; ++u) {
+        if (items[u].kind == IT_SO || items[u].kind == IT_SI) continue;
+        acc_t += tl.T[u];
+        ++lag;
+      }
+      return lag;
+    };
     // ---- candidates ---------------------------------------------------------------
     struct Change {
       int t, opt, p, lead, dim = -1;  // dim -1: keep the tensor's split dim
+      int lag = 0;                    // D-LAG release lag (swap only)
     };
     struct Cand2 {
       std::vector<Change> ch;
@@ -522,6 +585,12 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       c.ch = {{t, TS_SWAP, ps.cfg[t].p, 1}};
       c.analytic = swap_cost(t, dm) / dm;
       step1.push_back(c);
+      const int lag = lag_for(t);
+      if (lag > 0) {  // the same swap with its range released after the copy (D-LAG)
+        Cand2 cl = c;
+        cl.ch[0].lag = lag;
+        step1.push_back(cl);
+      }
       // the same swap with the prefetch issued early enough to hide the H2D copy
       // (B200 computes ~30x more per PCIe byte than the paper's GPUs)
       {
@@ -539,6 +608,12 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
           for (int u = last_fw[t] + 1; u < bi && u < (int)items.size(); ++u) fw += (1.0 - tl.oc_d2h[u]) * tl.T[u];
           c2.analytic = std::max(0.0, dm / pr.hw.d2h_bw - fw) / dm;
           step1.push_back(c2);
+          if (lag > 0) {
+            Cand2 c3 = c2;
+            c3.ch[0].lag = lag;
+            c3.analytic = 0.0;  // both copies hidden behind profiled compute
+            step1.push_back(c3);
+          }
         }
       }
       c.ch = {{t, TS_RECOMPUTE, ps.cfg[t].p, 1}};
@@ -575,7 +650,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       for (auto& c : step1) (c.ch[0].opt == TS_SWAP ? sw : rc).push_back(c);
       std::stable_sort(sw.begin(), sw.end(), by);
       std::stable_sort(rc.begin(), rc.end(), by);
-      if (sw.size() > 6) sw.resize(6);
+      if (sw.size() > 10) sw.resize(10);
       if (rc.size() > 8) rc.resize(8);
       step1 = sw;
       step1.insert(step1.end(), rc.begin(), rc.end());
@@ -598,6 +673,10 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
           c.tensor = t;
           c.ch = {{t, opt, p, ps.cfg[t].lead}};
           step2.push_back(opt == TS_RECOMPUTE ? with_feeders(c, t) : c);
+          if (opt == TS_SWAP && lag_for(t) > 0) {  // D-LAG variant
+            c.ch[0].lag = lag_for(t);
+            step2.push_back(c);
+          }
         }
       }
     // D-CH: channel (parameter-dim) splits of the bottleneck op's 2-D activations, with the
@@ -698,6 +777,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
         cs.cfg[chg.t].opt = chg.opt;
         cs.cfg[chg.t].p = chg.p;
         cs.cfg[chg.t].lead = chg.lead;
+        cs.cfg[chg.t].lag = chg.opt == TS_SWAP ? chg.lag : 0;
         if (chg.dim >= 0) cs.cfg[chg.t].dim = chg.dim;
         if (chg.p == 1) cs.cfg[chg.t].dim = 0;
       }
@@ -728,6 +808,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
           cs.cfg[chg.t].opt = chg.opt;
           cs.cfg[chg.t].p = chg.p;
           cs.cfg[chg.t].lead = chg.lead;
+          cs.cfg[chg.t].lag = chg.opt == TS_SWAP ? chg.lag : 0;
         }
         plan_refresh(g, cs, &pr);
         std::fprintf(stderr, "  cand t=%d opt=%d lead=%d analytic=%.3g dT=%.3gms top %llu->%llu\n", c.tensor,
@@ -744,6 +825,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
           cs.cfg[chg.t].opt = chg.opt;
           cs.cfg[chg.t].p = chg.p;
           cs.cfg[chg.t].lead = chg.lead;
+          cs.cfg[chg.t].lag = chg.opt == TS_SWAP ? chg.lag : 0;
         }
         plan_refresh(g, cs, &pr);
         std::fprintf(stderr, "  cand2 t=%d n=%zu opt=%d p=%d top %llu->%llu\n", c.tensor, c.ch.size(), c.ch[0].opt,
@@ -776,12 +858,26 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
       ps.cfg[chg.t].opt = chg.opt;
       ps.cfg[chg.t].p = chg.p;
       ps.cfg[chg.t].lead = chg.lead;
+      ps.cfg[chg.t].lag = chg.opt == TS_SWAP ? chg.lag : 0;
       if (chg.dim >= 0) ps.cfg[chg.t].dim = chg.dim;
       if (chg.p == 1) ps.cfg[chg.t].dim = 0;
     }
   }
   set_error("planner did not converge");
   return TS_ERR_INFEASIBLE;
+}
+
+ts_status plan_greedy_lag(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps, uint32_t flags) {
+  ts_status st = plan_greedy(g, budget, pr, ps, flags);
+  if (st != TS_ERR_INFEASIBLE) return st;
+  const std::string msg = ts_last_error();
+  PlanState alt;
+  if (plan_greedy(g, budget, pr, alt, flags | kPlanNoLag) == TS_OK) {
+    ps = std::move(alt);
+    return TS_OK;
+  }
+  set_error(msg);
+  return st;
 }
 
 }  // namespace ts

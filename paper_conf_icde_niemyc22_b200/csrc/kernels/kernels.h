@@ -155,8 +155,9 @@ bool attention_tc_eligible(const AttnArgs& a);  // bf16, d = 64, seq % 64 == 0 (
 void attention_fwd(const AttnArgs& a, cudaStream_t st);
 void attention_bwd(const AttnArgs& a, cudaStream_t st);  // needs a.c (= O), a.lse, a.dc
 void attention_simt(const AttnArgs& a, bool bwd, cudaStream_t st);  // CUDA-core kernels only (tests)
-// tcgen05 forward (attention_tc.cu): bf16, d = 64, seq % 128 == 0, seq <= 512, C and lse both
-// written; false = not eligible (nothing launched).  a.thr must be set.
+// tcgen05 forward (attention_tc.cu): bf16, d = 64, seq % 128 == 0; writes each of C, lse and
+// the keep bits whose pointer is set (a replay regenerates only its target); false = not
+// eligible (nothing launched).  a.thr must be set.
 bool attention_fwd_tc5(const AttnArgs& a, cudaStream_t st);
 // tcgen05 backward (same eligibility; needs c, lse, mask, dc, ws)
 bool attention_bwd_tc5(const AttnArgs& a, cudaStream_t st);

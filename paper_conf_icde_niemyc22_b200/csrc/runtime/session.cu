@@ -1839,7 +1839,8 @@ ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const f
   a.no_tc5 = mma_only ? 1 : 0;
   const bool tc = !simt_only && tsk::attention_tc_eligible(a);
   // tcgen05: forward for any seq % 128 == 0, backward up to seq 512 (K, V resident in smem)
-  const bool tc5 = tc && !mma_only && a.seq % 128 == 0 && (mode == 1 || a.seq <= 512) && a.c && a.lse;
+  const bool tc5 = tc && !mma_only && a.seq % 128 == 0 && (mode == 1 || a.seq <= 512) &&
+                   (mode == 1 ? (a.c || a.lse || a.mask) : (a.c && a.lse));
   if (tc) {
     if (mode == 1) tsk::attention_fwd(a, st);
     else tsk::attention_bwd(a, st);

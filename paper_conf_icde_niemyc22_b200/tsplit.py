@@ -35,7 +35,7 @@ class OpDesc(C.Structure):
 
 class TensorCfg(C.Structure):
     _fields_ = [("tensor_id", C.c_int32), ("opt", C.c_int32), ("p_num", C.c_int32), ("dim", C.c_int32),
-                ("prefetch_lead", C.c_int32)]
+                ("prefetch_lead", C.c_int32), ("release_lag", C.c_int32)]
 
 
 class PlanStats(C.Structure):
@@ -325,8 +325,8 @@ class Plan:
         check(lib().ts_plan_get(self.h, tid, C.byref(c)))
         return (c.opt, c.p_num, c.prefetch_lead)
 
-    def set(self, tid, opt=RESIDE, p_num=1, prefetch_lead=1, dim=0):
-        c = TensorCfg(tid, opt, p_num, dim, prefetch_lead)
+    def set(self, tid, opt=RESIDE, p_num=1, prefetch_lead=1, dim=0, release_lag=0):
+        c = TensorCfg(tid, opt, p_num, dim, prefetch_lead, release_lag)
         check(lib().ts_plan_set(self.h, C.byref(c)))
 
     def get_dim(self, tid) -> int:
@@ -334,12 +334,27 @@ class Plan:
         check(lib().ts_plan_get(self.h, tid, C.byref(c)))
         return c.dim
 
+    def get_lag(self, tid) -> int:
+        """Release lag of a swapped tensor (reading D-LAG)."""
+        c = TensorCfg()
+        check(lib().ts_plan_get(self.h, tid, C.byref(c)))
+        return c.release_lag
+
+    def oracle_cfg(self) -> dict:
+        """{tensor id: (opt, p_num, lead, dim, lag)} — the plan in the oracle simulator's form."""
+        out = {}
+        for t in range(self.graph.n):
+            c = TensorCfg()
+            check(lib().ts_plan_get(self.h, t, C.byref(c)))
+            out[t] = (c.opt, c.p_num, c.prefetch_lead, c.dim, c.release_lag)
+        return out
+
     def set_many(self, cfgs: dict):
-        """{tensor id: (opt, p_num, prefetch_lead[, dim])} applied and validated together
+        """{tensor id: (opt, p_num, prefetch_lead[, dim[, release_lag]])} applied and validated together
         (a channel-split chain is legal only as a whole, reading D-CH)."""
         arr = (TensorCfg * len(cfgs))()
         for i, (t, c) in enumerate(cfgs.items()):
-            arr[i] = TensorCfg(t, c[0], c[1], c[3] if len(c) > 3 else 0, c[2])
+            arr[i] = TensorCfg(t, c[0], c[1], c[3] if len(c) > 3 else 0, c[2], c[4] if len(c) > 4 else 0)
         check(lib().ts_plan_set_many(self.h, arr, len(cfgs)))
 
     def set_recompute_cache(self, cache_bytes: int):

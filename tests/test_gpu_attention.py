@@ -193,3 +193,24 @@ def test_fused_bert_small_bf16_tensor_cores(seq):
     finally:
         os.environ.pop("TSPLIT_NO_FUSION", None)
     assert global_rel_err(u2, u0) <= 1e-6
+
+
+def test_tc_forward_partial_outputs_for_replays():
+    """A recompute replay regenerates only the output it targets (C, or lse, or the keep
+    bits): the tcgen05 forward runs with the other pointers null (it used to fall back to
+    the mma.sync kernel) and writes exactly what the full call writes."""
+    nb, heads, seq, d = 2, 3, 256, 64
+    q, k, v, _ = _inputs(nb, heads, seq, d, seed=8)
+    dev = lambda a: torch.from_numpy(a).to("cuda").to(torch.bfloat16)  # noqa: E731
+    Q, K, V = dev(q), dev(k), dev(v)
+    geom = (nb, heads, seq, d, 21, 1, 2)
+    C = torch.empty_like(Q)
+    L = torch.empty((nb, heads, seq), dtype=torch.float32, device="cuda")
+    M = torch.empty((nb, heads, seq, seq // 32), dtype=torch.int32, device="cuda")
+    assert tsplit.attention(1, geom, 0.125, 0.1, Q, K, V, c=C, lse=L, mask=M) == 2
+    C2, L2, M2 = torch.zeros_like(C), torch.zeros_like(L), torch.zeros_like(M)
+    assert tsplit.attention(1, geom, 0.125, 0.1, Q, K, V, c=C2) == 2
+    assert tsplit.attention(1, geom, 0.125, 0.1, Q, K, V, lse=L2) == 2
+    assert tsplit.attention(1, geom, 0.125, 0.1, Q, K, V, mask=M2) == 2
+    torch.cuda.synchronize()
+    assert torch.equal(C, C2) and torch.equal(L, L2) and torch.equal(M, M2)

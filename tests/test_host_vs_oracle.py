@@ -13,8 +13,8 @@ from tsinputs import graphs
 
 def _apply(plan, cfg, acts):
     for t in acts:
-        o, p, lead = cfg[t]
-        plan.set(t, o, p, lead)
+        c = cfg[t]
+        plan.set(t, c[0], c[1], c[2], c[3] if len(c) > 3 else 0, c[4] if len(c) > 4 else 0)
 
 
 def _compare(g, cfg, cache=0):
@@ -69,6 +69,21 @@ def test_trace_bit_exact_random_plans_bert_tiny(seed):
     _compare(g, cfg)
 
 
+@pytest.mark.parametrize("gname", ["bert_tiny", "resnet_tiny"])
+@pytest.mark.parametrize("seed", range(4))
+def test_trace_bit_exact_random_plans_with_release_lags(gname, seed):
+    """D-LAG: swapped tensors with release lags 0..12 (the range a swap-out frees returns
+    to the pool after that many compute items, before the swap-in) — the C++ expansion
+    and pool trace equal the oracle's bit for bit."""
+    g = graphs.config_graph(gname)
+    r = random.Random(500 + seed)
+    cfg = sim.default_cfg(g)
+    for t in brute.act_tensors(g):
+        o = r.choice([0, 1, 1, 2])
+        cfg[t] = (o, r.choice([1, 2, 4]), r.choice([1, 2, 5]), 0, r.choice([0, 1, 3, 12]) if o == 1 else 0)
+    _compare(g, cfg)
+
+
 def test_default_trace_bert_large():
     g = graphs.config_graph("bert_large")
     _compare(g, sim.default_cfg(g))
@@ -109,7 +124,7 @@ def test_planner_feasible_plans_fit_and_simulate_exactly():
         P = tsplit.Plan.plan(G, budget)
         st = P.stats()
         assert st["peak_extent"] <= budget
-        cfg = {t: P.get(t) for t in range(G.n)}
+        cfg = P.oracle_cfg()
         ref = sim.simulate(g, cfg)
         assert ref.peak_extent == st["peak_extent"]
         assert [tuple(e) for e in ref.trace] == P.trace()
@@ -278,10 +293,7 @@ def test_planner_uses_channel_splits_when_the_batch_is_one(frac):
     budget = st["static_bytes"] + int(frac * (st["peak_extent"] - st["static_bytes"]))
     P = tsplit.Plan.plan(G, budget)
     assert P.stats()["peak_extent"] <= budget
-    cfg = sim.default_cfg(g)
-    for t in brute.act_tensors(g):
-        o, p, lead = P.get(t)
-        cfg[t] = (o, p, lead, P.get_dim(t))
+    cfg = P.oracle_cfg()
     assert any(c[1] > 1 and c[3] == 1 for c in cfg.values())
     ref = sim.simulate(g, cfg)
     assert P.trace() == [tuple(e) for e in ref.trace]
@@ -325,8 +337,8 @@ def test_plan_deserialize_rejects_bad_blobs():
         tsplit.Plan.deserialize(G, bytes(blob[:-12]))
     act = brute.act_tensors(g)[0]
     param = next(t["id"] for t in g["tensors"] if t["kind"] == "param")
-    for tid, word, value in ((act, 1, 0), (act, 1, 3), (param, 0, tsplit.SWAP)):
+    for tid, word, value in ((act, 1, 0), (act, 1, 3), (param, 0, tsplit.SWAP), (act, 4, 3)):  # (a lag needs swap)
         bad = bytearray(blob)
-        struct.pack_into("<i", bad, 24 + 16 * tid + 4 * word, value)
+        struct.pack_into("<i", bad, 24 + 20 * tid + 4 * word, value)
         with pytest.raises(tsplit.TsError):
             tsplit.Plan.deserialize(G, bytes(bad))
