@@ -75,9 +75,52 @@ __global__ void __launch_bounds__(256) gemm_simt_kernel(GemmArgs g) {
     }
   }
 }
+// Tiny products (the classifier / pooler of a small batch: M x N of a few thousand outputs,
+// K up to thousands): one warp per output, lanes striding K (coalesced for K-major
+// operands), a fixed xor-shuffle tree — deterministic, and no 64-step K loop on one CTA.
+template <class TI, class TO, class AccT>
+__global__ void __launch_bounds__(256) gemm_small_kernel(GemmArgs g) {
+  const int64_t w = (int64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const int lane = threadIdx.x & 31;
+  const int64_t per = int64_t(g.M) * g.N;
+  if (w >= per * g.nb1 * g.nb2) return;
+  const int bz = int(w / per);
+  const int m = int((w % per) / g.N), n = int(w % g.N);
+  const int b1 = bz % g.nb1, b2 = bz / g.nb1;
+  const TI* A = reinterpret_cast<const TI*>(g.a.ptr) + b1 * g.a.bs1 + b2 * g.a.bs2;
+  const TI* B = reinterpret_cast<const TI*>(g.b.ptr) + b1 * g.b.bs1 + b2 * g.b.bs2;
+  AccT acc = 0;
+  for (int k = lane; k < g.K; k += 32) {
+    const float a = to_f(A[g.a.mn_major ? int64_t(k) * g.a.ld + m : int64_t(m) * g.a.ld + k]);
+    const float b = to_f(B[g.b.mn_major ? int64_t(k) * g.b.ld + n : int64_t(n) * g.b.ld + k]);
+    acc = fma(AccT(a), AccT(b), acc);
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if (lane) return;
+  TO* cp = reinterpret_cast<TO*>(g.c) + b1 * g.cbs1 + b2 * g.cbs2 + int64_t(m) * g.ldc + n;
+  AccT v = acc * AccT(g.alpha);
+  if (g.bias)
+    v += g.bias_dtype == F32 ? AccT(reinterpret_cast<const float*>(g.bias)[n])
+                             : AccT(to_f(reinterpret_cast<const bf16*>(g.bias)[n]));
+  if (g.beta != 0.f) v += AccT(g.beta) * AccT(to_f(*cp));
+  *cp = from_f<TO>(float(v));
+}
 }  // namespace
 
 void gemm_simt(const GemmArgs& g, cudaStream_t st) {
+  const int64_t outs = int64_t(g.M) * g.N * g.nb1 * g.nb2;
+  if (outs <= 16384 && g.K >= 64) {  // tiny output, long reduction: a warp per output
+    const int blocks = int((outs * 32 + 255) / 256);
+    if (g.in_dtype == F32) {
+      if (g.c_dtype == F32) gemm_small_kernel<float, float, double><<<blocks, 256, 0, st>>>(g);
+      else gemm_small_kernel<float, bf16, double><<<blocks, 256, 0, st>>>(g);
+    } else {
+      if (g.c_dtype == F32) gemm_small_kernel<bf16, float, float><<<blocks, 256, 0, st>>>(g);
+      else gemm_small_kernel<bf16, bf16, float><<<blocks, 256, 0, st>>>(g);
+    }
+    return;
+  }
   dim3 grid((g.N + TN - 1) / TN, (g.M + TM - 1) / TM, g.nb1 * g.nb2);
   if (g.in_dtype == F32) {
     if (g.c_dtype == F32) gemm_simt_kernel<float, float, double><<<grid, 256, 0, st>>>(g);

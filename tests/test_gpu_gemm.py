@@ -98,8 +98,10 @@ def test_gemm_tc_alpha_beta_bias(mode, gemm_mode):
     assert ((C - ref).norm() / ref.norm()).item() < 1e-5
 
 
-def test_gemm_simt_f32():
-    M, N, K = 70, 33, 45
+@pytest.mark.parametrize("M,N,K", [(70, 33, 45), (32, 2, 1024), (2, 1024, 32), (4, 3, 4096)])
+def test_gemm_simt_f32(M, N, K):
+    """CUDA-core paths: the tiled kernel, and the warp-per-output kernel for tiny outputs with
+    a long reduction (the 2-class classifier of BERT: 32 x 2 x 1024)."""
     A = torch.randn(K, M, device="cuda")  # MN-major
     B = torch.randn(N, K, device="cuda")
     C = torch.zeros(M, N, device="cuda")
