@@ -57,7 +57,8 @@ typedef enum {
   TS_OP_LAYERNORM = 4, /* in X[R,H], gamma, beta; fattr[0] = eps                       */
   TS_OP_ADD = 5,
   TS_OP_DROPOUT = 6,   /* fattr[0] = p; iattr[0] = seed (Philox4x32-10 key)             */
-  TS_OP_SOFTMAX = 7,   /* over the last dim                                            */
+  TS_OP_SOFTMAX = 7,   /* over the last dim; iattr[0] = 1: causal over [.., s, s] scores
+                          (keys j > query i dropped: decoder self-attention, f4)          */
   TS_OP_ATTN_QK = 8,   /* in Q[T,h], K[T,h] out S[b,a,s,s]; iattr {heads, seq}; fattr[0] = alpha */
   TS_OP_ATTN_PV = 9,   /* in P[b,a,s,s], V[T,h] out C[T,h]; iattr {heads, seq}         */
   TS_OP_EMBED = 10,    /* in ids, type_ids (i32 [T]), Wword, Wpos, Wtype; iattr[0] = seq */

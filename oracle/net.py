@@ -41,7 +41,7 @@ def forward_op(graph, op, val, row0=0, elem0=0, step=0):
     if k == "dropout":
         return ops.dropout_fwd(x[0], fa[0], ia[0], elem0, step)
     if k == "softmax":
-        return ops.softmax_fwd(x[0])
+        return ops.softmax_fwd(x[0], causal=bool(ia and ia[0]))
     if k == "attn_qk":
         return ops.attn_qk_fwd(x[0], x[1], ia[0], ia[1], fa[0])
     if k == "attn_pv":

@@ -153,7 +153,13 @@ def dropout_bwd(dy, p, seed, elem0, step=0):
     return dropout_fwd(dy, p, seed, elem0, step)
 
 
-def softmax_fwd(x):
+def softmax_fwd(x, causal=False):
+    """Row softmax over the last dim.  causal: x is [..., s, s] attention scores (query i,
+    key j) and keys j > i are excluded (probability 0) — the decoder self-attention of the
+    encoder-decoder Transformer."""
+    if causal:
+        s = x.shape[-1]
+        x = np.where(np.triu(np.ones((s, s), bool), 1), -np.inf, x)
     m = x.max(axis=-1, keepdims=True)
     e = np.exp(x - m)
     return e / e.sum(axis=-1, keepdims=True)

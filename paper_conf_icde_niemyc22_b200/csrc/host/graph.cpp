@@ -52,6 +52,10 @@ bool validate_op(const Graph& g, const Op& o, std::string& why) {
       if (!need(1, 1)) return false;
       if (!same_shape(T(o.in[0]), T(o.out[0]))) return (why = "elementwise shapes"), false;
       if (o.kind == TS_OP_DROPOUT && (o.fa.size() < 1 || o.ia.size() < 1)) return (why = "dropout attrs"), false;
+      if (o.kind == TS_OP_SOFTMAX && !o.ia.empty() && o.ia[0] != 0) {  // causal: square [.., s, s] scores
+        const Tensor& x = T(o.in[0]);
+        if (x.ndim < 2 || x.shape[x.ndim - 1] != x.shape[x.ndim - 2]) return (why = "causal softmax needs [.., s, s]"), false;
+      }
       if (o.kind == TS_OP_DROPOUT && (o.fa[0] < 0 || o.fa[0] >= 1)) return (why = "dropout p"), false;
       return true;
     case TS_OP_ADD:

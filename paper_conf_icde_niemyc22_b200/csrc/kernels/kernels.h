@@ -195,7 +195,8 @@ void layernorm_fwd(int dt, const void* x, const void* g, const void* b, void* y,
 void layernorm_bwd(int dt, const void* dy, const void* x, const void* g, void* dx, int acc, float* ws,
                    uint64_t ws_bytes, float* dgamma, float* dbeta, int pacc, int64_t rows, int H, float eps,
                    cudaStream_t st);
-void softmax_fwd(int dt, const void* x, void* y, int64_t rows, int L, cudaStream_t st);
+// causal: rows are queries i = row % L of [.., L, L] scores; keys j > i get probability 0
+void softmax_fwd(int dt, const void* x, void* y, int64_t rows, int L, int causal, cudaStream_t st);
 void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t rows, int L,
                  cudaStream_t st);
 // out[n] (+)= sum_r x[r, n] (rows filtered by `filter[r] == fval` when filter != null)
@@ -210,8 +211,10 @@ void embed_bwd_pos(int dt, const void* dy, float* dpos, int64_t nsamp, int seq, 
 void cls_fwd(int dt, const void* x, void* y, int64_t nsamp, int seq, int H, cudaStream_t st);
 void cls_bwd(int dt, const void* dy, void* dx, int acc, int64_t nsamp, int seq, int H, cudaStream_t st);
 // loss[0] (+)= sum_rows CE / b_global ; dz = (softmax - onehot)/b_global
+// (ws: >= rows floats; with many rows (token-level losses) per-row values go there and one
+// block sums them in a fixed order)
 void xent_fwd(int dt, const void* z, const int* labels, float* loss, int acc, int64_t rows, int C,
-              float inv_b, cudaStream_t st);
+              float inv_b, float* ws, cudaStream_t st);
 void xent_bwd(int dt, const void* z, const int* labels, void* dz, int acc, int64_t rows, int C, float inv_b,
               cudaStream_t st);
 // ---- optimiser / static region ------------------------------------------------

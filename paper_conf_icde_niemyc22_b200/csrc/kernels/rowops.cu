@@ -659,17 +659,22 @@ __global__ void __launch_bounds__(256) colsum_bf16_kernel(const bf16* __restrict
 // ------------------------------------------------------------------ softmax
 template <class T, int NCH>
 __global__ void __launch_bounds__(kWarps * 32) softmax_fwd_kernel(const T* __restrict__ x, T* __restrict__ y,
-                                                                   int64_t rows, int L) {
+                                                                   int64_t rows, int L, int causal) {
   constexpr int V = Vec<T>::N;
   const int lane = threadIdx.x & 31;
   for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
     float v[NCH][V];
     float m = -INFINITY;
+    // causal: the row is query i = r % L of an [.., L, L] score tensor; keys j > i drop out
+    const int lim = causal ? int(r % L) : L - 1;
 #pragma unroll
     for (int c = 0; c < NCH; ++c) {
       int col = (c * 32 + lane) * V;
       if (col < L) {
         load_vec(x + r * L + col, v[c]);
+#pragma unroll
+        for (int i = 0; i < V; ++i)
+          if (col + i > lim) v[c][i] = -INFINITY;
 #pragma unroll
         for (int i = 0; i < V; ++i) m = fmaxf(m, v[c][i]);
       }
@@ -733,16 +738,17 @@ __global__ void __launch_bounds__(kWarps * 32) softmax_bwd_kernel(const T* __res
 }
 
 template <class T>
-__global__ void softmax_generic(const T* x, T* y, int64_t rows, int L) {
+__global__ void softmax_generic(const T* x, T* y, int64_t rows, int L, int causal) {
   const int lane = threadIdx.x & 31;
   for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    const int lim = causal ? int(r % L) : L - 1;
     float m = -INFINITY;
-    for (int i = lane; i < L; i += 32) m = fmaxf(m, to_f(x[r * L + i]));
+    for (int i = lane; i <= lim; i += 32) m = fmaxf(m, to_f(x[r * L + i]));
     m = warp_max(m);
     float s = 0.f;
-    for (int i = lane; i < L; i += 32) s += __expf(to_f(x[r * L + i]) - m);
+    for (int i = lane; i <= lim; i += 32) s += __expf(to_f(x[r * L + i]) - m);
     const float inv = 1.f / warp_sum(s);
-    for (int i = lane; i < L; i += 32) y[r * L + i] = from_f<T>(__expf(to_f(x[r * L + i]) - m) * inv);
+    for (int i = lane; i < L; i += 32) y[r * L + i] = from_f<T>(i <= lim ? __expf(to_f(x[r * L + i]) - m) * inv : 0.f);
   }
 }
 template <class T>
@@ -781,6 +787,33 @@ __global__ void xent_fwd_kernel(const T* z, const int* labels, float* loss, int 
     float t = 0.f;
     for (int i = 0; i < int(blockDim.x / 32); ++i) t += part[i];
     loss[0] = (acc ? loss[0] : 0.f) + t * inv_b;
+  }
+}
+// per-row cross entropy (lse - z[label]) into out[row]
+template <class T>
+__global__ void xent_rows_kernel(const T* z, const int* labels, float* out, int64_t rows, int C) {
+  const int lane = threadIdx.x & 31;
+  for (int64_t r = int64_t(blockIdx.x) * kWarps + (threadIdx.x >> 5); r < rows; r += int64_t(gridDim.x) * kWarps) {
+    float m = -INFINITY;
+    for (int i = lane; i < C; i += 32) m = fmaxf(m, to_f(z[r * C + i]));
+    m = warp_max(m);
+    float s = 0.f;
+    for (int i = lane; i < C; i += 32) s += __expf(to_f(z[r * C + i]) - m);
+    s = warp_sum(s);
+    if (lane == 0) out[r] = (m + logf(s)) - to_f(z[r * C + labels[r]]);
+  }
+}
+// loss (+)= inv_b * sum of the per-row values, one block, fixed order (fp64 partials)
+__global__ void xent_sum_kernel(const float* v, int64_t rows, float* loss, int acc, float inv_b) {
+  __shared__ double part[256];
+  double t = 0.0;
+  for (int64_t r = threadIdx.x; r < rows; r += 256) t += v[r];
+  part[threadIdx.x] = t;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double tot = 0.0;
+    for (int i = 0; i < 256; ++i) tot += part[i];
+    loss[0] = (acc ? loss[0] : 0.f) + float(tot * inv_b);
   }
 }
 template <class T>
@@ -901,20 +934,20 @@ void ln_fwd_t(const void* x, const void* g, const void* b, void* y, int64_t rows
 }
 
 template <class T>
-void softmax_fwd_t(const void* x, void* y, int64_t rows, int L, cudaStream_t st) {
+void softmax_fwd_t(const void* x, void* y, int64_t rows, int L, int causal, cudaStream_t st) {
   constexpr int V = Vec<T>::N;
   int nch = (L + 32 * V - 1) / (32 * V);
   bool vec = L % V == 0 && al16(x) && al16(y);
   int grid = grid_rows(rows);
   if (vec && nch <= 8) {
     switch (nch) {
-      case 1: softmax_fwd_kernel<T, 1><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L); return;
-      case 2: softmax_fwd_kernel<T, 2><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L); return;
-      case 3: case 4: softmax_fwd_kernel<T, 4><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L); return;
-      default: softmax_fwd_kernel<T, 8><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L); return;
+      case 1: softmax_fwd_kernel<T, 1><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L, causal); return;
+      case 2: softmax_fwd_kernel<T, 2><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L, causal); return;
+      case 3: case 4: softmax_fwd_kernel<T, 4><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L, causal); return;
+      default: softmax_fwd_kernel<T, 8><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L, causal); return;
     }
   }
-  softmax_generic<T><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L);
+  softmax_generic<T><<<grid, kWarps * 32, 0, st>>>((const T*)x, (T*)y, rows, L, causal);
 }
 
 template <class T>
@@ -1212,9 +1245,9 @@ void layernorm_bwd(int dt, const void* dy, const void* x, const void* g, void* d
   reduce_partials<<<(H + 31) / 32, 256, 0, st>>>(ws, int(G), 2 * H, H, H, dbeta, pacc);
 }
 
-void softmax_fwd(int dt, const void* x, void* y, int64_t rows, int L, cudaStream_t st) {
-  if (dt == F32) softmax_fwd_t<float>(x, y, rows, L, st);
-  else softmax_fwd_t<bf16>(x, y, rows, L, st);
+void softmax_fwd(int dt, const void* x, void* y, int64_t rows, int L, int causal, cudaStream_t st) {
+  if (dt == F32) softmax_fwd_t<float>(x, y, rows, L, causal, st);
+  else softmax_fwd_t<bf16>(x, y, rows, L, causal, st);
 }
 void softmax_bwd(int dt, const void* dy, const void* y, void* dx, int acc, int64_t rows, int L, cudaStream_t st) {
   if (dt == F32) softmax_bwd_t<float>(dy, y, dx, acc, rows, L, st);
@@ -1292,7 +1325,14 @@ void cls_bwd(int dt, const void* dy, void* dx, int acc, int64_t nsamp, int seq, 
   else cls_bwd_kernel<bf16><<<grid, 256, 0, st>>>((const bf16*)dy, (bf16*)dx, acc, nsamp, seq, H);
 }
 void xent_fwd(int dt, const void* z, const int* labels, float* loss, int acc, int64_t rows, int C, float inv_b,
-              cudaStream_t st) {
+              float* ws, cudaStream_t st) {
+  if (ws && rows > 64) {  // token-level losses (many rows): a warp per row, then a fixed-order sum
+    const int grid = grid_rows(rows);
+    if (dt == F32) xent_rows_kernel<float><<<grid, kWarps * 32, 0, st>>>((const float*)z, labels, ws, rows, C);
+    else xent_rows_kernel<bf16><<<grid, kWarps * 32, 0, st>>>((const bf16*)z, labels, ws, rows, C);
+    xent_sum_kernel<<<1, 256, 0, st>>>(ws, rows, loss, acc, inv_b);
+    return;
+  }
   if (dt == F32) xent_fwd_kernel<float><<<1, 256, 0, st>>>((const float*)z, labels, loss, acc, rows, C, inv_b);
   else xent_fwd_kernel<bf16><<<1, 256, 0, st>>>((const bf16*)z, labels, loss, acc, rows, C, inv_b);
 }

@@ -427,7 +427,8 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       nk = 1;
       if (!bwd) {
         char *x = V(o.in[0]), *y = V(o.out[0]);
-        return [=](cudaStream_t st) { tsk::softmax_fwd(dt, x, y, rows, L, st); };
+        const int causal = (!o.ia.empty() && o.ia[0] != 0) ? 1 : 0;  // decoder self-attention
+        return [=](cudaStream_t st) { tsk::softmax_fwd(dt, x, y, rows, L, causal, st); };
       }
       char *dy = G(o.out[0]), *y = V(o.out[0]), *dx = G(o.in[0]);
       int acc = A(g.n() + o.in[0]);
@@ -694,17 +695,22 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
     case TS_OP_XENT: {
       const int C = int(g.t[o.in[0]].shape[1]);
       const float inv_b = 1.f / float(B);
+      // rows of this micro-op: one per sample (classification) or per token (the
+      // encoder-decoder's next-token loss: the per-sentence sum, averaged over the batch)
+      const int64_t rows = ns * g.t[o.in[0]].rows_per_sample;
       char* z = V(o.in[0]);
       const int* lab = reinterpret_cast<const int*>(V(o.in[1]));
       nk = 1;
       if (!bwd) {
         float* loss = reinterpret_cast<float*>(V(o.out[0]));
         int acc = m.k > 0;
-        return [=](cudaStream_t st) { tsk::xent_fwd(dt, z, lab, loss, acc, ns, C, inv_b, st); };
+        float* xws = uint64_t(rows) * 4 + 4096 <= g.ws_bytes ? ws : nullptr;
+        nk = xws && rows > 64 ? 2 : 1;
+        return [=](cudaStream_t st) { tsk::xent_fwd(dt, z, lab, loss, acc, rows, C, inv_b, xws, st); };
       }
       char* dz = G(o.in[0]);
       int acc = A(g.n() + o.in[0]);
-      return [=](cudaStream_t st) { tsk::xent_bwd(dt, z, lab, dz, acc, ns, C, inv_b, st); };
+      return [=](cudaStream_t st) { tsk::xent_bwd(dt, z, lab, dz, acc, rows, C, inv_b, st); };
     }
   }
   nk = 0;

@@ -351,6 +351,10 @@ class Runtime:
             keep = dropout_keep(tuple(x[0].shape), elem0, fa[0], ia[0], step, x[0].device)
             return torch.where(keep, x[0] / (1.0 - fa[0]), torch.zeros_like(x[0]))
         if kd == "softmax":
+            if ia and ia[0]:  # causal: keys j > query i dropped
+                s = x[0].shape[-1]
+                mask = torch.triu(torch.ones(s, s, dtype=torch.bool, device=x[0].device), 1)
+                return torch.softmax(x[0].masked_fill(mask, float("-inf")), -1)
             return torch.softmax(x[0], -1)
         if kd == "attn_qk":
             return fa[0] * (_heads(x[0], ia[0], ia[1]) @ _heads(x[1], ia[0], ia[1]).transpose(-1, -2))

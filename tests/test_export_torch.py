@@ -37,7 +37,8 @@ def _random_plan(g, G, seed, cache=0):
 
 
 CASES = [("mlp", {}), ("bert_tiny", dict(dtype="f32")), ("bert_tiny", dict(dtype="f32", fused_attention=True)),
-         ("vgg_tiny", dict(dtype="f32")), ("resnet_tiny", dict(dtype="f32"))]
+         ("vgg_tiny", dict(dtype="f32")), ("resnet_tiny", dict(dtype="f32")),
+         ("transformer_tiny", dict(dtype="f32", seq=32))]
 
 
 @pytest.mark.parametrize("case", range(len(CASES)))

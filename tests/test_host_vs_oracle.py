@@ -84,6 +84,21 @@ def test_trace_bit_exact_random_plans_with_release_lags(gname, seed):
     _compare(g, cfg)
 
 
+@pytest.mark.parametrize("seed", range(3))
+def test_trace_bit_exact_random_plans_transformer(seed):
+    """The encoder-decoder workload (f4): Alg. 1 order, static region and the trace of random
+    split / swap / recompute plans (with release lags) equal the oracle simulator's."""
+    g = graphs.config_graph("transformer_tiny")
+    G = tsplit.Graph(g)
+    assert G.schedule() == sim.schedule(g) and G.static_bytes() == sim.static_bytes(g)
+    r = random.Random(700 + seed)
+    cfg = sim.default_cfg(g)
+    for t in brute.act_tensors(g):
+        o = r.choice([0, 1, 2])
+        cfg[t] = (o, r.choice([1, 2, 4]), r.choice([1, 2]), 0, r.choice([0, 4]) if o == 1 else 0)
+    _compare(g, cfg)
+
+
 def test_default_trace_bert_large():
     g = graphs.config_graph("bert_large")
     _compare(g, sim.default_cfg(g))

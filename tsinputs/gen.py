@@ -3,6 +3,8 @@
 Recipes (DESIGN.md §5 "Input recipe"):
   * MLP (config 1): x ~ N(0,1) [seed 0]; W, b ~ U(+-1/sqrt(fan_in)) [seed 1 + param index];
     labels uniform in [0, classes) [seed 2].
+  * Transformer (f4, IWSLT-shaped): source / target ids and next-token labels uniform in
+    [0, vocab) [seeds 3000 / 4000 / 5000 + rank]; parameters as BERT's.
   * BERT: token ids uniform in [0, vocab) [seed 1000 + rank]; token-type ids 0 (one
     segment, P:L16 MRPC-like pairs are not modelled); labels uniform in {0,1};
     weights and embeddings ~ N(0, 0.02); biases ~ N(0, 0.02) (non-zero so that bias
@@ -34,7 +36,7 @@ def _rng(seed: int, name: str) -> np.random.Generator:
 def init_params(graph: dict, seed: int = 1) -> dict[str, np.ndarray]:
     """fp32 parameter values keyed by tensor name."""
     out = {}
-    is_bert = graph["name"].startswith("bert")
+    is_bert = graph["name"].startswith(("bert", "transformer"))  # same recipe for the Transformer
     is_cnn = graph["name"].startswith(("vgg", "resnet"))
     for t in graph["tensors"]:
         if t["kind"] != "param":
@@ -83,7 +85,13 @@ def make_inputs(graph: dict, seed: int = 0) -> dict[str, np.ndarray]:
         if t["kind"] not in ("input", "label"):
             continue
         name, shape = t["name"], t["shape"]
-        if is_bert:
+        if graph["name"].startswith("transformer"):  # token ids / next-token labels uniform in the vocab
+            tag = {"src_ids": 3000, "tgt_ids": 4000, "tgt_labels": 5000}.get(name)
+            if tag is None:
+                out[name] = np.zeros(shape, np.int32)
+            else:
+                out[name] = np.random.default_rng(tag + seed).integers(0, classes, size=shape).astype(np.int32)
+        elif is_bert:
             r = np.random.default_rng(1000 + seed)
             if name == "input_ids":
                 out[name] = r.integers(0, vocab, size=shape, dtype=np.int64).astype(np.int32)

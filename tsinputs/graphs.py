@@ -193,6 +193,92 @@ def bert(layers=24, hidden=1024, heads=16, seq=512, batch=32, vocab=30522, ffn=N
     return g.done()
 
 
+def transformer(enc_layers=6, dec_layers=6, hidden=512, heads=8, ffn=2048, seq=128, batch=64, vocab=32000,
+                dtype="bf16", dropout=0.1, seed=4321) -> dict:
+    """Encoder-decoder Transformer shaped like the paper's IWSLT2016 workload (P:L306:
+    "the IWSLT2016 dataset for Transformer"), source and target of `seq`
+    tokens, post-LN layers as in bert().  Encoder layer: self-attention (fused op, no mask)
+    + add&LN + FFN + add&LN.  Decoder layer: causal self-attention (unfused: attn_qk ->
+    softmax(causal) -> dropout -> attn_pv), add&LN, cross-attention (q from the decoder,
+    k / v from the encoder output; equal lengths, so the same attention op) + add&LN,
+    FFN + add&LN.  Head: linear to the target vocabulary and the token-level cross
+    entropy (labels [T]): the loss is the per-sentence sum of token losses, averaged over
+    the batch (R14: mean over the global batch of samples)."""
+    assert hidden % heads == 0
+    dh = hidden // heads
+    T = batch * seq
+    g = GraphBuilder(f"transformer_E{enc_layers}D{dec_layers}_h{hidden}_a{heads}_s{seq}_b{batch}", dtype, batch)
+    src = g.tensor("src_ids", (T,), "input", dtype="i32")
+    tgt = g.tensor("tgt_ids", (T,), "input", dtype="i32")
+    seg = g.tensor("token_type_ids", (T,), "input", dtype="i32")
+    labels = g.tensor("tgt_labels", (T,), "label", dtype="i32")
+    alpha = 1.0 / math.sqrt(dh)
+    sd = [seed]
+
+    def nseed():
+        sd[0] += 1
+        return sd[0]
+
+    def embed(name, ids):
+        w = g.param(name + ".word", (vocab, hidden))
+        p = g.param(name + ".pos", (seq, hidden))
+        ty = g.param(name + ".type", (2, hidden))
+        e = g.op("embed", name, [ids, seg, w, p, ty], (T, hidden), iattrs=[seq])
+        e = ln(name + ".ln", e)
+        return g.op("dropout", name + ".drop", [e], (T, hidden), fattrs=[dropout], iattrs=[nseed()])
+
+    def lin(name, inp, n_out, n_in):
+        w = g.param(name + ".w", (n_out, n_in))
+        b = g.param(name + ".b", (n_out,))
+        return g.op("linear", name, [inp, w, b], (T, n_out))
+
+    def ln(name, x):
+        gm = g.param(name + ".g", (hidden,))
+        bt = g.param(name + ".b", (hidden,))
+        return g.op("layernorm", name, [x, gm, bt], (T, hidden), fattrs=[1e-12])
+
+    def fused_attn(p, xq, xkv):
+        q = lin(p + "q", xq, hidden, hidden)
+        k = lin(p + "k", xkv, hidden, hidden)
+        v = lin(p + "v", xkv, hidden, hidden)
+        c, _, _ = g.op_multi("attention", p + "attn", [q, k, v],
+                             [(p + "ctx", (T, hidden), None), (p + "lse", (batch, heads, seq), "f32"),
+                              (p + "dmask", (batch, heads, seq, seq // 32), "i32")],
+                             iattrs=[heads, seq, nseed()], fattrs=[alpha, dropout])
+        return lin(p + "proj", c, hidden, hidden)
+
+    def causal_attn(p, x):
+        q = lin(p + "q", x, hidden, hidden)
+        k = lin(p + "k", x, hidden, hidden)
+        v = lin(p + "v", x, hidden, hidden)
+        s = g.op("attn_qk", p + "scores", [q, k], (batch, heads, seq, seq), iattrs=[heads, seq], fattrs=[alpha])
+        pr = g.op("softmax", p + "probs", [s], (batch, heads, seq, seq), iattrs=[1])
+        pd = g.op("dropout", p + "attn_drop", [pr], (batch, heads, seq, seq), fattrs=[dropout], iattrs=[nseed()])
+        c = g.op("attn_pv", p + "ctx", [pd, v], (T, hidden), iattrs=[heads, seq])
+        return lin(p + "proj", c, hidden, hidden)
+
+    def mlp_block(p, x):
+        f1 = lin(p + "ffn1", x, ffn, hidden)
+        ge = g.op("gelu", p + "gelu", [f1], (T, ffn))
+        return lin(p + "ffn2", ge, hidden, ffn)
+
+    x = embed("src", src)
+    for l in range(enc_layers):
+        p = f"e{l}."
+        x = ln(p + "ln1", g.op("add", p + "res1", [fused_attn(p, x, x), x], (T, hidden)))
+        x = ln(p + "ln2", g.op("add", p + "res2", [mlp_block(p, x), x], (T, hidden)))
+    enc = x
+    y = embed("tgt", tgt)
+    for l in range(dec_layers):
+        p = f"d{l}."
+        y = ln(p + "ln1", g.op("add", p + "res1", [causal_attn(p + "self.", y), y], (T, hidden)))
+        y = ln(p + "ln2", g.op("add", p + "res2", [fused_attn(p + "cross.", y, enc), y], (T, hidden)))
+        y = ln(p + "ln3", g.op("add", p + "res3", [mlp_block(p, y), y], (T, hidden)))
+    logits = lin("out", y, vocab, hidden)
+    g.op("xent", "loss", [logits, labels], (1,), out_dtype="f32")
+    return g.done()
+
+
 def tensor_bytes(t: dict) -> int:
     n = 1
     for s in t["shape"]:
@@ -238,6 +324,16 @@ def config_graph(name: str, **over) -> dict:
         kw = dict(batch=16, img=32, width=0.25, blocks=(1, 1), classes=10)
         kw.update(over)
         return resnet50(**kw)
+    if name == "transformer_iwslt":  # f4 workload, IWSLT-shaped
+        return transformer(**over)
+    if name == "transformer_tiny":
+        kw = dict(enc_layers=1, dec_layers=1, hidden=128, heads=2, ffn=256, seq=64, batch=4, vocab=512)
+        kw.update(over)
+        return transformer(**kw)
+    if name == "transformer_small":  # the bf16 parity size
+        kw = dict(enc_layers=1, dec_layers=2, hidden=256, heads=4, ffn=1024, seq=128, batch=8, vocab=1024)
+        kw.update(over)
+        return transformer(**kw)
     if name == "bert_scaled":
         kw = dict(layers=24, hidden=2560, heads=40, seq=512, batch=64)
         kw.update(over)
