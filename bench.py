@@ -40,6 +40,10 @@ WORKLOADS = {
     "vgg16": dict(batch=64, frac=0.30, name="vgg16_b64_i224_budget30",
                   metric="samples/sec under HBM budget (VGG-16)", model="vgg-16 (13 conv3x3 + 3 fc, 224x224)",
                   seq_len=None, data="synthetic (N(0,1) images, uniform labels, Kaiming-normal weights)"),
+    "transformer": dict(batch=64, frac=0.25, name="transformer_iwslt_b64_s128_budget25",
+                        metric="samples/sec under HBM budget (IWSLT-shaped Transformer)",
+                        model="transformer enc-dec 6+6L h512 a8 ffn2048 s128 vocab32000 (P:L306, f4)", seq_len=128,
+                        data="synthetic (uniform source / target ids and next-token labels, random-init weights)"),
     "resnet50": dict(batch=256, frac=0.25, name="resnet50_b256_i224_budget25",
                      metric="samples/sec under HBM budget (ResNet-50)", model="resnet-50 v1.5 (224x224)",
                      seq_len=None, data="synthetic (N(0,1) images, uniform labels, Kaiming-normal weights)"),
@@ -50,7 +54,10 @@ def workload_graph(wl, layers=LAYERS, fused=True):
     from tsinputs import graphs
     if wl == "bert_large":
         return graphs.bert(layers=layers, batch=BATCH, fused_attention=fused)
-    return graphs.config_graph(wl)
+    return graphs.config_graph(ORACLE_GRAPH.get(wl, wl))
+
+
+ORACLE_GRAPH = {"transformer": "transformer_iwslt"}  # bench workload -> graphs.config_graph name
 
 
 def peaks():
@@ -162,7 +169,7 @@ def cnn_oracle_time(wl, reps=1):
     batch; BN statistics then span that sample's pixels)."""
     from oracle import net
     from tsinputs import gen, graphs
-    g = graphs.config_graph(wl, batch=1)
+    g = graphs.config_graph(ORACLE_GRAPH.get(wl, wl), batch=1)
     P, I = gen.init_params(g), gen.make_inputs(g)
     ts = []
     for _ in range(reps):
@@ -174,8 +181,9 @@ def cnn_oracle_time(wl, reps=1):
 
 def cnn_cpu_baseline(wl):
     t = min(cnn_oracle_time(wl))
+    what = "1 sentence pair (128 + 128 tokens)" if wl == "transformer" else "1 image (224x224)"
     return {"value": 1.0 / t, "unit": "samples/s", "cores": cpu_threads(), "kind": "oracle",
-            "sample": f"1 image (224x224) through the full {wl} fp64 fwd+bwd: {t:.2f}s/sample"}
+            "sample": f"{what} through the full {wl} fp64 fwd+bwd: {t:.2f}s/sample"}
 
 
 def run_reference(args, rank, world):
@@ -449,10 +457,11 @@ def main():
     lin = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and bt == 1 and kd == 0 and tc]
     att = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and bt > 1 and tc]
     c_flop, c_ms = sum(f for f, _ in conv), sum(ms for _, ms in conv)
-    cnn = args.workload != "bert_large"
+    cnn = args.workload in ("vgg16", "resnet50")
+    bert = args.workload == "bert_large"
     g_flop, g_ms = sum(f for f, _ in lin), sum(ms for _, ms in lin)
     a_flop, a_ms = sum(f for f, _ in att), sum(ms for _, ms in att)
-    step_ms_prof = sum(item_ms)
+    step_ms_prof = sum(t for (kind, _, _, _), t in zip(plan.items(), item_ms) if kind in ("F", "B", "R"))
     del sess
     torch.cuda.empty_cache()
 
@@ -497,8 +506,8 @@ def main():
                        "algorithmic FLOP (2MNK) / summed launch durations; traffic = dram read+write of "
                        "one FFN1-forward launch from the committed ncu --set full capture"}
     config = {
-        "workload": W["name"], "model": W["model"] if cnn else f"bert-large ({args.layers}L h{HID} a{HEADS} s{SEQ})",
-        "attention": None if cnn else args.attention,
+        "workload": W["name"], "model": W["model"] if not bert else f"bert-large ({args.layers}L h{HID} a{HEADS} s{SEQ})",
+        "attention": args.attention if bert else None,
         "global_batch": batch * world, "seq_len": W["seq_len"], "parallelism": f"dp{world}",
         "budget_frac_of_unsplit_dynamic_peak": args.budget_frac,
         "budget_bytes": budget, "unsplit_peak_bytes": unsplit_peak, "static_bytes": static,
@@ -512,7 +521,7 @@ def main():
                  "recompute_cache_bytes": pst["recompute_cache_bytes"],
                  "measured_pcie_gbs": [round(x / 1e9, 1) for x in pcie] if pcie else None},
         "l2": "no flush needed: every step streams >10 GB of activations through a 126 MB L2"
-              if not cnn else "no flush needed: every step streams several GB of activations through a 126 MB L2",
+              if bert else "no flush needed: every step streams several GB of activations through a 126 MB L2",
     }
     if cnn:
         config.pop("seq_len")
@@ -553,7 +562,7 @@ def main():
         "pcie_gbs": [round(x / 1e9, 1) for x in bw], "pcie_source": "measured" if pcie else "fallback 55 GB/s",
         "how": "t_roof = max(plan FLOP / bf16_tflops_sustained, max(D2H bytes / B_d2h, H2D bytes / B_h2d)); "
                "frac = t_roof / measured step time"}
-    if not cnn and args.attention == "fused":
+    if bert and args.attention == "fused":
         # FA accounting per layer: forward 2 products (QK^T, PV), backward 5 (S recompute, dP, dV, dK,
         # dQ), each 2 b a s^2 d FLOP; the F and B items cover every layer's batch exactly once
         prod = 2.0 * BATCH * HEADS * SEQ * SEQ * (HID // HEADS)
@@ -566,7 +575,7 @@ def main():
             "backward_tflops": 5 * prod * args.layers / (att_ms["B"] / 1e3) / 1e12 if att_ms["B"] > 0 else None,
             "share_of_step": sum(att_ms.values()) / step_ms_prof if step_ms_prof else None,
             "how": "summed cudaEvent times of the attention micro-op items of one eager step"}
-    elif not cnn:  # the paper's unfused graph: per-(sample, head) attention products on gemm_tc
+    elif bert:  # the paper's unfused graph: per-(sample, head) attention products on gemm_tc
         line["roofline_attention_gemm"] = {
             "bound": "hbm", "kernel": "gemm_tc on per-(sample, head) attention products",
             "achieved_tflops": a_flop / (a_ms / 1e3) / 1e12 if a_ms > 0 else None, "launches": len(att),
@@ -579,7 +588,7 @@ def main():
     # BASELINE metric part 2 (config 5): max trainable batch x hidden under the whole HBM, measured
     # by tools/max_scale.py (planning up to 1024 x 512 tokens takes minutes, so not in this run)
     msf = os.path.join(ROOT, "profiles", "r1_max_scale.json")
-    if not cnn and os.path.exists(msf):
+    if bert and os.path.exists(msf):
         ms = json.load(open(msf))
         line["max_trainable"] = {
             "source": "profiles/r1_max_scale.json (tools/max_scale.py, 24L s512 BERT, heads = h/64, capacity = "
@@ -587,7 +596,7 @@ def main():
             "capacity_bytes": ms.get("capacity_bytes"),
             "per_hidden": [{k: e.get(k) for k in ("hidden", "max_batch_unsplit", "max_batch_tsplit", "scale",
                                                    "scale_unsplit", "samples_per_s")} for e in ms.get("summary", [])]}
-    if not cnn:
+    if bert:
         # north_star: the paper's ratios, quoted with the GPU PAPER.md names — context only
         line["paper_context"] = {
             "gpu": "NVIDIA TITAN RTX (24 GB), FP32 (PAPER.md L8, L46, L450; BASELINE.md)",
@@ -596,7 +605,7 @@ def main():
             "note": "comparison systems are out of scope here; this run's own scale ratio is "
                     "max_trainable (TSPLIT vs unsplit on the same B200)"}
     if world == 1 and not args.no_cpu_baseline:
-        line["cpu_baseline"] = cnn_cpu_baseline(args.workload) if cnn else cpu_baseline_measure()
+        line["cpu_baseline"] = cpu_baseline_measure() if bert else cnn_cpu_baseline(args.workload)
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
