@@ -562,6 +562,13 @@ def main():
         "pcie_gbs": [round(x / 1e9, 1) for x in bw], "pcie_source": "measured" if pcie else "fallback 55 GB/s",
         "how": "t_roof = max(plan FLOP / bf16_tflops_sustained, max(D2H bytes / B_d2h, H2D bytes / B_h2d)); "
                "frac = t_roof / measured step time"}
+    # per-kernel roofline of the plan: sum over micro-ops of max(F / P_tensor,
+    # bytes / BW_hbm) with the sustained tensor peak and the measured HBM bandwidth
+    t_k, f_k, b_k = plan.roofline(peak * 1e12, pk.get("hbm_gbs", 6554.9) * 1e9)
+    line["roofline_kernels"] = {
+        "t_roof_ms": t_k * 1e3, "ms_per_step": step_s * 1e3, "frac": t_k / step_s, "flop": f_k, "hbm_bytes": b_k,
+        "how": "sum over the plan's compute micro-ops of max(algorithmic FLOP / bf16_tflops_sustained, "
+               "algorithmic HBM bytes / hbm_gbs) (ts_plan_roofline); frac = t_roof / measured step time"}
     if bert and args.attention == "fused":
         # FA accounting per layer: forward 2 products (QK^T, PV), backward 5 (S recompute, dP, dV, dK,
         # dQ), each 2 b a s^2 d FLOP; the F and B items cover every layer's batch exactly once

@@ -246,6 +246,12 @@ ts_status ts_plan_grad_buckets(const ts_plan_t* p, uint64_t bucket_bytes, int64_
  * carries a fingerprint of the graph; deserialize returns TS_ERR_ARG for a blob of another
  * graph, a malformed one, or any entry ts_plan_set would reject (opt / p_num / dim / lead,
  * parameters not reside, an illegal D-CH channel chain) — nothing is adopted then. */
+/* Per-kernel roofline of the plan's compute items: the sum over every F / B / R
+ * micro-op of max(algorithmic FLOP / tensor_flops, algorithmic HBM bytes / hbm_bw), with the
+ * same per-op FLOP and byte counts as the analytic profile (no launch or wave terms); also the
+ * totals.  A lower bound on the step's compute-stream time on this plan. */
+ts_status ts_plan_roofline(const ts_plan_t* p, double tensor_flops, double hbm_bw, double* seconds, double* flop,
+                           double* bytes);
 ts_status ts_plan_serialize(const ts_plan_t* p, void* buf, uint64_t cap, uint64_t* n);
 ts_status ts_plan_deserialize(const ts_graph_t* g, const void* buf, uint64_t n, ts_plan_t** out);
 void ts_plan_destroy(ts_plan_t* p);

@@ -219,6 +219,28 @@ ts_status ts_plan_set_many(ts_plan_t* p, const ts_tensor_cfg* cfgs, int32_t n) {
   return apply_cfgs(p, cfgs, n);
 }
 
+ts_status ts_plan_roofline(const ts_plan_t* p, double tensor_flops, double hbm_bw, double* seconds, double* flop,
+                           double* bytes) {
+  if (!p || !seconds || tensor_flops <= 0 || hbm_bw <= 0) return set_error("bad argument"), TS_ERR_ARG;
+  const Graph& g = *p->graph;
+  std::vector<OpCost> oc(g.ops.size());
+  for (size_t o = 0; o < g.ops.size(); ++o) oc[o] = op_cost(g, int(o));
+  double s = 0, f = 0, b = 0;
+  for (const Item& it : p->st.ex.items) {
+    if (it.kind == IT_SO || it.kind == IT_SI) continue;
+    const double P = double(p->st.ex.P[it.op]);
+    const double fi = (it.kind == IT_B ? oc[it.op].flop_b : oc[it.op].flop_f) / P;
+    const double bi = (it.kind == IT_B ? oc[it.op].bytes_b : oc[it.op].bytes_f) / P;
+    s += std::max(fi / tensor_flops, bi / hbm_bw);
+    f += fi;
+    b += bi;
+  }
+  *seconds = s;
+  if (flop) *flop = f;
+  if (bytes) *bytes = b;
+  return TS_OK;
+}
+
 ts_status ts_plan_stats(const ts_plan_t* p, ts_plan_stats_t* out) {
   if (!p || !out) return set_error("null argument"), TS_ERR_ARG;
   const auto& s = p->st;

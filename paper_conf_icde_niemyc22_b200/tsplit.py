@@ -105,6 +105,7 @@ def lib():
             "ts_plan_items": (i32, [vp, P(i32), u64, P(u64)]),
             "ts_plan_grad_buckets": (i32, [vp, u64, P(i64), u64, P(u64)]),
             "ts_plan_serialize": (i32, [vp, vp, u64, P(u64)]),
+            "ts_plan_roofline": (i32, [vp, C.c_double, C.c_double, P(C.c_double), P(C.c_double), P(C.c_double)]),
             "ts_plan_deserialize": (i32, [vp, vp, u64, P(vp)]),
             "ts_plan_destroy": (None, [vp]),
         }
@@ -388,6 +389,12 @@ class Plan:
         buf = (C.c_int64 * (3 * n.value))()
         check(lib().ts_plan_grad_buckets(self.h, bucket_bytes, buf, len(buf), C.byref(n)))
         return [(buf[3 * i], buf[3 * i + 1], buf[3 * i + 2]) for i in range(n.value)]
+
+    def roofline(self, tensor_flops: float, hbm_bw: float):
+        """(seconds, flop, bytes): sum over the plan's micro-ops of max(F / peak, bytes / bw)."""
+        s, f, b = C.c_double(), C.c_double(), C.c_double()
+        check(lib().ts_plan_roofline(self.h, tensor_flops, hbm_bw, C.byref(s), C.byref(f), C.byref(b)))
+        return s.value, f.value, b.value
 
     def serialize(self) -> bytes:
         n = C.c_uint64()

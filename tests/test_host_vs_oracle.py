@@ -357,3 +357,22 @@ def test_plan_deserialize_rejects_bad_blobs():
         struct.pack_into("<i", bad, 24 + 20 * tid + 4 * word, value)
         with pytest.raises(tsplit.TsError):
             tsplit.Plan.deserialize(G, bytes(bad))
+
+
+def test_plan_roofline_bounds():
+    """ts_plan_roofline: sum over micro-ops of max(F / P, bytes / BW) — at least each of the
+    two totals' own bound, at most their sum; its FLOP equal the plan's compute FLOP (recompute
+    replays included); splitting changes no algorithmic FLOP."""
+    g = graphs.config_graph("bert_tiny")
+    G = tsplit.Graph(g)
+    P0 = tsplit.Plan.default(G)
+    pk, bw = 1.4e15, 6.5e12
+    s, f, b = P0.roofline(pk, bw)
+    assert max(f / pk, b / bw) <= s <= f / pk + b / bw
+    assert f == pytest.approx(P0.stats()["compute_flop"], rel=1e-12)
+    P1 = tsplit.Plan.default(G)
+    names = G.names
+    P1.set(names["l0.ffn1"], tsplit.RESIDE, 4, 1)
+    P1.set(names["l1.q"], tsplit.RECOMPUTE, 1, 1)
+    s1, f1, b1 = P1.roofline(pk, bw)
+    assert f1 == pytest.approx(P1.stats()["compute_flop"], rel=1e-12) and f1 > f
