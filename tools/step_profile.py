@@ -28,6 +28,10 @@ def profile(G, P, spec, params, dev):
         key = f"{kind}:{spec['ops'][op]['kind']}"
         agg[key] += t
         cnt[key] += 1
+        if spec["ops"][op]["kind"] == "linear":  # per linear role (q, k, v, proj, ffn1, ffn2, ...)
+            role = f"{kind}:linear.{spec['ops'][op]['name'].split('.', 1)[-1]}"
+            agg[role] += t
+            cnt[role] += 1
     del S
     torch.cuda.empty_cache()
     return agg, cnt, sum(t for (kind, _, _, _), t in zip(items, ms) if kind not in ("SO", "SI"))

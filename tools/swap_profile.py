@@ -88,6 +88,14 @@ def main():
     out = {"workload": wl, "budget_bytes": budget, "budget_frac": frac,
            "measured_pcie_gbs": {"d2h": d2h_bw / 1e9, "h2d": h2d_bw / 1e9}, "plans": {}}
     variants = [("planned", plan)]
+    if wl == "vgg16" and len(sys.argv) > 3:  # C2's "conv offload": swap conv #i's output
+        convs = [o for o in spec["ops"] if o["kind"] == "conv2d"]
+        t = convs[int(sys.argv[3])]["outputs"][0]
+        for lead, lag in ((1, 0), (4, 4), (16, 24)):
+            forced = tsplit.Plan.deserialize(G, plan.serialize())
+            forced.set(t, tsplit.SWAP, forced.get(t)[1], lead, 0, lag)
+            if forced.stats()["peak_extent"] <= budget:
+                variants.append((f"conv{sys.argv[3]}_offload_lead{lead}_lag{lag}", forced))
     if wl == "bert_large" and len(sys.argv) > 3:
         names = {t["name"]: t["id"] for t in spec["tensors"]}
         forced = tsplit.Plan.deserialize(G, plan.serialize())
