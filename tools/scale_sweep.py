@@ -68,17 +68,28 @@ def plan_phase(args):
 
 
 def run_phase(args):
+    """Time the largest plan per hidden size whose pinned host pool (the plan's swapped
+    bytes) fits the box's host memory cap; plan-feasible batches beyond it are reported as
+    HBM-feasible only."""
     import torch
     res = json.load(open(OUT))
     free, total = torch.cuda.mem_get_info()
     res["device_free_bytes"] = free
+    res["host_cap_bytes"] = args.host_cap_bytes
     for s in res["summary"]:
-        if not s.get("plan_blob"):
+        h = s["hidden"]
+        rows = [r for r in res["rows"] if r["hidden"] == h and r.get("feasible")]
+        ok = [r for r in rows if r.get("swap_bytes", 0) <= args.host_cap_bytes]
+        if not ok:
             continue
-        h, b = s["hidden"], s["max_batch_tsplit"]
+        b = max(r["batch"] for r in ok)
+        s["max_batch_tsplit_host_limited"] = b
         spec = spec_of(h, b)
         G = tsplit.Graph(spec)
-        P = tsplit.Plan.deserialize(G, base64.b64decode(s["plan_blob"]))
+        if b == s["max_batch_tsplit"] and s.get("plan_blob"):
+            P = tsplit.Plan.deserialize(G, base64.b64decode(s["plan_blob"]))
+        else:
+            P = tsplit.Plan.plan(G, res["capacity_bytes"])
         S = tsplit.Session(G, P, lr=0.0, slab_bytes=res["capacity_bytes"])
         dev = tsplit.inputs_to_device(G, gen.make_inputs(spec))
         loss = S.step(dev)
@@ -87,7 +98,8 @@ def run_phase(args):
         for _ in range(args.steps):
             loss = S.step(dev)
         dt = (time.perf_counter() - t0) / args.steps
-        s.update(samples_per_s=b / dt, ms_per_step=dt * 1e3, loss=loss, host_pool_bytes=S.host_pool()[0])
+        s.update(timed_batch=b, samples_per_s=b / dt, ms_per_step=dt * 1e3, loss=loss,
+                 host_pool_bytes=S.host_pool()[0], timed_scale=b * h)
         print(json.dumps({k: v for k, v in s.items() if k != "plan_blob"}), flush=True)
         del S
         torch.cuda.empty_cache()
@@ -101,6 +113,8 @@ if __name__ == "__main__":
     ap.add_argument("--capacity-bytes", type=int, default=184404344832)
     ap.add_argument("--max-batch", type=int, default=8192)
     ap.add_argument("--steps", type=int, default=2)
+    ap.add_argument("--host-cap-bytes", type=int, default=100 * 2 ** 30,
+                    help="largest pinned swap pool to run (the GPU box has ~196 GB of host RAM)")
     a = ap.parse_args()
     os.makedirs("gpurun_out", exist_ok=True)
     plan_phase(a) if a.phase == "plan" else run_phase(a)
