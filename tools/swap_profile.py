@@ -98,13 +98,15 @@ def main():
                 variants.append((f"conv{sys.argv[3]}_offload_lead{lead}_lag{lag}", forced))
     if wl == "bert_large" and len(sys.argv) > 3:
         names = {t["name"]: t["id"] for t in spec["tensors"]}
-        forced = tsplit.Plan.deserialize(G, plan.serialize())
-        for l in range(int(sys.argv[3])):
-            forced.set(names[f"l{l}.ffn1"], tsplit.SWAP, 1, 4)
-        if forced.stats()["peak_extent"] <= budget:
-            variants.append((f"ffn1_swapped_first_{sys.argv[3]}", forced))
-        else:
-            out["forced_variant"] = "exceeds the budget"
+        for lead, lag in ((4, 0), (8, 8), (16, 16), (32, 24)):
+            forced = tsplit.Plan.deserialize(G, plan.serialize())
+            for l in range(int(sys.argv[3])):
+                forced.set(names[f"l{l}.ffn1"], tsplit.SWAP, 1, lead, 0, lag)
+            fs = forced.stats()
+            print("forced", lead, lag, fs["peak_extent"] <= budget, fs["predicted_s"] * 1e3, plan.stats()["predicted_s"] * 1e3,
+                  flush=True)
+            if fs["peak_extent"] <= budget:
+                variants.append((f"ffn1_swapped_first_{sys.argv[3]}_lead{lead}_lag{lag}", forced))
     for name, P in variants:
         st = P.stats()
         r = measure(spec, G, P, params, dev)
