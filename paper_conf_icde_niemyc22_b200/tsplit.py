@@ -10,7 +10,8 @@ import os
 import numpy as np
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libtsplit.so")
+# (TSPLIT_LIB: another in-tree build of the same library, for same-box A/B timing runs)
+LIB_PATH = os.environ.get("TSPLIT_LIB") or os.path.join(_PKG, "libtsplit.so")
 
 OPS = {"linear": 0, "relu": 1, "gelu": 2, "tanh": 3, "layernorm": 4, "add": 5, "dropout": 6,
        "softmax": 7, "attn_qk": 8, "attn_pv": 9, "embed": 10, "cls": 11, "xent": 12,
