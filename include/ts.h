@@ -353,6 +353,12 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch,
  * the per-group fallback rounds the running sum to bf16 after every group (the grouped
  * launch rounds once).  TS_ERR_ARG for bad groups / gdim, a grouped extent (N, K or M)
  * that `groups` does not divide, or beta other than 0 / 1. */
+/* Row kernels for unit tests / microbenchmarks: op 0 = bias-gradient column sum,
+ * out[j] (+)= sum_r x[r, j] over a [rows, n] row-major tensor (fp32 out; ws: device
+ * workspace of ws_bytes >= 8 KB, its last 4 KB hold completion tickets that must start
+ * zeroed).  `aux` unused.  Asynchronous on `stream`. */
+ts_status ts_row_op(int32_t op, int32_t dtype, const void* x, const void* aux, void* out, int64_t rows, int32_t n,
+                    float* ws, uint64_t ws_bytes, int32_t acc, void* stream);
 ts_status ts_gemm_bf16_grouped(int32_t groups, int32_t gdim, int32_t M, int32_t N, int32_t K,
                                const void* const* A, int64_t lda, int32_t ta,
                                const void* const* B, int64_t ldb, int32_t tb,

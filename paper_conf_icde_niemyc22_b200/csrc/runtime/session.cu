@@ -1818,6 +1818,23 @@ ts_status ts_conv2d(int32_t mode, int32_t dtype, const int32_t* geom, const void
   return TS_OK;
 }
 
+ts_status ts_row_op(int32_t op, int32_t dtype, const void* x, const void* aux, void* out, int64_t rows, int32_t n,
+                    float* ws, uint64_t ws_bytes, int32_t acc, void* stream) {
+  if (!x || !out || rows < 1 || n < 1 || (dtype != TS_BF16 && dtype != TS_F32))
+    return set_error("ts_row_op: bad argument"), TS_ERR_ARG;
+  const int dt = dtype == TS_BF16 ? tsk::BF16 : tsk::F32;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (op == 0) {  // out[n] (+)= sum_rows x[rows, n] (fp32 out; ws >= ... + 4 KB tickets)
+    if (!ws || ws_bytes < 8192) return set_error("ts_row_op: column sum needs a workspace"), TS_ERR_ARG;
+    tsk::column_sum(dt, x, rows, n, ws, ws_bytes, static_cast<float*>(out), acc, nullptr, 0, st);
+  } else {
+    return set_error("ts_row_op: unknown op"), TS_ERR_ARG;
+  }
+  (void)aux;
+  CU(cudaGetLastError());
+  return TS_OK;
+}
+
 ts_status ts_attention(int32_t mode, int32_t dtype, const int32_t* geom, const float* fattr, const void* q,
                        const void* k, const void* v, void* c, float* lse, uint32_t* mask, const void* dc, void* dq,
                        void* dk, void* dv, int32_t acc, float* ws, void* stream, int32_t* used_tc) {

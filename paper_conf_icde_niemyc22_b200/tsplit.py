@@ -143,6 +143,7 @@ def lib():
             "ts_gemm_f32": (i32, [i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, C.c_float,
                                   vp, vp]),
             "ts_conv2d": (i32, [i32, i32, P(i32), vp, vp, vp, vp, vp, i32, vp, P(i32)]),
+            "ts_row_op": (i32, [i32, i32, vp, vp, vp, i64, i32, vp, u64, i32, vp]),
             "ts_attention": (i32, [i32, i32, P(i32), P(C.c_float), vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, i32, vp,
                                    vp, P(i32)]),
         }
@@ -607,3 +608,13 @@ def attention(mode: int, geom, alpha: float, p: float, q, k, v, c=None, lse=None
     check(lib().ts_attention(mode, dt, g, fa, ptr(q), ptr(k), ptr(v), ptr(c), lse_p, ptr(mask), ptr(dc), ptr(dq),
                              ptr(dk), ptr(dv), acc, ws_p, st, C.byref(used)))
     return used.value
+
+
+def column_sum(x, out, ws, acc: int = 0, stream=None):
+    """out (+)= x.sum(0) through ts_row_op (x: [rows, n] bf16 / fp32 torch device tensor,
+    out: fp32 [n], ws: fp32 workspace whose last 4 KB start zeroed)."""
+    import torch
+    dt = DTYPES["bf16"] if x.dtype == torch.bfloat16 else DTYPES["f32"]
+    st = C.c_void_p(stream if stream is not None else torch.cuda.current_stream().cuda_stream)
+    check(lib().ts_row_op(0, dt, C.c_void_p(x.data_ptr()), None, C.c_void_p(out.data_ptr()), x.shape[0], x.shape[1],
+                          C.c_void_p(ws.data_ptr()), ws.numel() * 4, acc, st))

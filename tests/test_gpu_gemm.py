@@ -180,3 +180,24 @@ def test_gemm_tc_grouped(gdim, M, N, K, ta, tb, out, beta, mode, gemm_mode):
         ref = ref + beta * C0[i].float()
         err = ((Cs[i].float() - ref).norm() / ref.norm()).item()
         assert err < (2e-5 if out == "f32" else 8e-3), (i, err)
+
+
+@pytest.mark.parametrize("rows,n", [(16384, 1024), (16384, 4096), (100, 24), (4096, 8), (77, 1000)])
+@pytest.mark.parametrize("dtype", ["bf16", "f32"])
+def test_bias_column_sum(rows, n, dtype):
+    """Bias-gradient column sums (ts_row_op 0): fp32 result within fp32 summation error of
+    the fp64 sum, deterministic across calls, accumulate flag."""
+    dt = torch.bfloat16 if dtype == "bf16" else torch.float32
+    x = torch.randn(rows, n, device="cuda").to(dt)
+    out = torch.zeros(n, device="cuda")
+    ws = torch.zeros(256 * 2 * 4096 + 1024, device="cuda")
+    tsplit.column_sum(x, out, ws)
+    torch.cuda.synchronize()
+    ref = x.double().sum(0)
+    scale = x.double().abs().sum(0).max()
+    assert float((out.double() - ref).abs().max() / scale) < 1e-6
+    again = torch.zeros(n, device="cuda")
+    tsplit.column_sum(x, again, ws)
+    tsplit.column_sum(x, again, ws, acc=1)
+    torch.cuda.synchronize()
+    assert torch.equal(2 * out, again) or float((again.double() - 2 * ref).abs().max() / scale) < 2e-6
