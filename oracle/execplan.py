@@ -38,9 +38,18 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
     def rows_per_sample(t):
         return ts[t]["shape"][0] // B
 
+    def band(t):  # attribute (height) split (D-ATTR): p bands of rows, each over every sample
+        return an.sample[t] and sim.is_attr(graph, cfg, t)
+
+    def amode(o):
+        return any(band(t) for t in ops[o]["outputs"])
+
+    def staged(o):
+        return ops[o]["kind"] in sim.ATTR_WINDOW and (band(ops[o]["inputs"][0]) or amode(o))
+
     def piece_shape(t):
         sh = list(ts[t]["shape"])
-        if chan(t):
+        if chan(t) or band(t):
             sh[1] //= p_of(t)
         elif an.sample[t]:
             sh[0] //= p_of(t)
@@ -54,9 +63,11 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
     def P_op(o):
         if cmode(o):
             return max(p_of(t) for t in ops[o]["outputs"] if chan(t))
+        if amode(o):
+            return max(p_of(t) for t in ops[o]["outputs"] if band(t))
         P = 1
         for t in ops[o]["inputs"] + ops[o]["outputs"]:
-            if an.sample[t] and not chan(t):
+            if an.sample[t] and not chan(t) and not band(t):
                 P = max(P, p_of(t))
         return P
 
@@ -119,6 +130,90 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
             else:
                 view(tid, 0, B, grad=True)[...] += g
 
+    def input_rows(x, b0, b1, r, grad=False):
+        """Row r of samples [b0, b1) of the window input x (band-split or unsplit)."""
+        if band(x):
+            hb = ts[x]["shape"][1] // p_of(x)
+            return store[(n + x if grad else x, r // hb)][b0:b1, r % hb]
+        return store[(n + x if grad else x, 0)][b0:b1, r]
+
+    def attr_micro_op(it):
+        """Micro-op k of an op in attribute mode or of a window op reading bands (D-ATTR).
+        A window op stages the input rows its output block needs (the physical merge of
+        Fig. 10, padding written out: 0 for conv, -inf for max pooling), runs unpadded on
+        the staged copy and, in its backward, adds the staged input gradient back into the
+        pieces its rows came from.  A band-local op maps band k to band k."""
+        o = ops[it.op]
+        k, P = it.k, P_op(it.op)
+        y = o["outputs"][0]
+        val = dict(pval)
+        if o["kind"] in sim.ATTR_WINDOW:
+            x = o["inputs"][0]
+            H, W = ts[x]["shape"][1], ts[x]["shape"][2]
+            lo, hi, hs, nb = sim.staged_rows(graph, cfg, it.op, k, P)
+            R, s, pad = sim.window_geom(o, ts)
+            b0 = 0 if amode(it.op) else k * B // P
+            fill = -np.inf if o["kind"] == "maxpool" else 0.0
+            xs = np.full((nb, hs, W + 2 * pad, ts[x]["shape"][3]), fill)
+            for r in range(max(lo, 0), min(hi, H - 1) + 1):
+                xs[:, r - lo, pad:pad + W] = input_rows(x, b0, b0 + nb, r)
+            assert (2 * n + it.op, k) in store  # the staging temporary is allocated
+            store[(2 * n + it.op, k)] = xs
+            o2 = dict(o, iattrs=list(o["iattrs"]))
+            o2["iattrs"][1 if o["kind"] == "conv2d" else 2] = 0
+            val[x] = xs
+            if it.kind in ("F", "R"):
+                yv = net.forward_op(graph, o2, val)
+                if amode(it.op):
+                    store[(y, k)][...] = yv
+                else:
+                    view(y, b0, b0 + nb)[...] = yv
+                return
+            dy = store[(n + y, k)] if amode(it.op) else view(y, b0, b0 + nb, grad=True)
+            for tid, g in net.backward_op(graph, o2, val, dy).items():
+                if ts[tid]["kind"] == "param":
+                    pgrad[tid] += g
+                elif tid in an.needs_grad:
+                    store[(3 * n + it.op, k)] = g
+                    for r in range(max(lo, 0), min(hi, H - 1) + 1):
+                        input_rows(x, b0, b0 + nb, r, grad=True)[...] += g[:, r - lo, pad:pad + W]
+            return
+        if it.kind in ("F", "R"):
+            for t in o["inputs"]:
+                if an.sample[t]:
+                    val[t] = store[(t, k)]
+        else:
+            for t in an.saved[it.op]:
+                val[t] = store[(t, k)]
+        if o["kind"] == "batchnorm":  # statistics over every band (BATCH_REDUCE)
+            xin, gid, bid = o["inputs"]
+            eps = o["fattrs"][0]
+            if it.kind == "F" and k == 0:
+                bn_stats[it.op] = O.batchnorm_stats(whole(xin))
+            mu, var = bn_stats[it.op]
+            if it.kind in ("F", "R"):
+                store[(y, k)][...] = O.batchnorm_fwd_with(val[xin], pval[gid], pval[bid], mu, var, eps)
+                return
+            if k == 0:
+                sums = O.batchnorm_bwd_sums(whole(y, grad=True), whole(xin), pval[gid], mu, var, eps)
+                bn_sums[it.op] = sums
+                pgrad[gid] += sums[2]
+                pgrad[bid] += sums[3]
+            s1_, s2_ = bn_sums[it.op][:2]
+            m = int(np.prod(ts[xin]["shape"][:-1]))
+            if xin in an.needs_grad:
+                store[(n + xin, k)][...] += O.batchnorm_bwd_with(
+                    store[(n + y, k)], val[xin], pval[gid], mu, var, s1_, s2_, m, eps)
+            return
+        if it.kind in ("F", "R"):
+            store[(y, k)][...] = net.forward_op(graph, o, val)
+            return
+        for tid, g in net.backward_op(graph, o, val, store[(n + y, k)]).items():
+            if ts[tid]["kind"] == "param":
+                pgrad[tid] += g
+            elif tid in an.needs_grad:
+                store[(n + tid, k)][...] += g
+
     def whole(t, grad=False):
         """All pieces of tensor t concatenated (the full batch)."""
         return np.concatenate([store[(n + t if grad else t, j)] for j in range(p_of(t))], axis=0)
@@ -127,12 +222,16 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
         for pc in f_alloc.get(i, []):
             key, j = pc
             t = key - n if key >= n else key
-            if it.kind == "SI":
+            if key >= 2 * n:  # staging temporary: filled by the micro-op (D-ATTR)
+                store[pc] = None
+            elif it.kind == "SI":
                 store[pc] = host.pop(pc)
             else:
                 store[pc] = np.zeros(piece_shape(t), F)
         if it.kind in ("F", "R", "B") and cmode(it.op):
             channel_micro_op(it)
+        elif it.kind in ("F", "R", "B") and (amode(it.op) or staged(it.op)):
+            attr_micro_op(it)
         elif it.kind in ("F", "R", "B"):
             o = ops[it.op]
             P = P_op(it.op)

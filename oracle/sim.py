@@ -81,6 +81,87 @@ def dim_of(cfg, t):
     return c[3] if c is not None and len(c) > 3 else 0
 
 
+# Attribute (height) split, P:L258-260 ("split along the dim of sample, model parameter, or
+# attribute (e.g., batch, channel, height, and width dimensions for images)"), DESIGN.md
+# reading D-ATTR: a 4-D NHWC activation [B, H, W, C] split along H into p bands of H/p rows,
+# piece j = rows [j H/p, (j+1) H/p) of every sample, stored [B, H/p, W, C].  An op with a
+# band-split output runs in "attribute mode": micro-op k computes output band k over all
+# samples.  Band-local ops (ATTR_LOCAL) read band k of band-split inputs of the same p.
+# Window ops (conv2d, maxpool) read the input rows their output band needs — its own band
+# plus halo rows from the neighbouring bands (or an unsplit input) — through a staged copy:
+# the physical merge & split of Fig. 10, a temporary [B, Hs, W + 2 pad, C] with the
+# padding written out, so the window op runs unpadded on it; its backward scatters the staged
+# input gradient back into the band pieces (overlapping halos add: merge = sum).  A
+# window op whose output is not band-split reads every band of its samples the same way (a
+# full merge).  Batch normalisation in band mode keeps BATCH_REDUCE's rule (its first
+# micro-op reads every band: statistics over all of (N, H, W)).  The staged input of a window
+# micro-op is a pool temporary allocated at the item and freed after it (key 2n + op; the
+# backward's staged input gradient is key 3n + op), so the pool trace accounts for it.
+ATTR_LOCAL = {"relu", "add", "batchnorm"}
+ATTR_WINDOW = {"conv2d", "maxpool"}
+
+
+def is_attr(graph, cfg, t):
+    return dim_of(cfg, t) == 2 and cfg[t][1] > 1 and graph["tensors"][t]["kind"] == "act"
+
+
+def window_geom(op, ts):
+    """(R, stride, pad) of a conv2d / maxpool."""
+    if op["kind"] == "conv2d":
+        return ts[op["inputs"][1]]["shape"][1], op["iattrs"][0], op["iattrs"][1]
+    return op["iattrs"][0], op["iattrs"][1], op["iattrs"][2]
+
+
+def band_rows(op, ts, k, P):
+    """Input rows [lo, hi] (inclusive, may lie outside [0, H)) the output band k of P of a
+    window op reads, and the staged row count Hs = hi - lo + 1."""
+    R, s, pad = window_geom(op, ts)
+    Ho = ts[op["outputs"][0]]["shape"][1]
+    hb = Ho // P
+    lo = k * hb * s - pad
+    hi = ((k + 1) * hb - 1) * s - pad + R - 1
+    return lo, hi, hi - lo + 1
+
+
+def check_attr(graph, cfg):
+    """Raise ValueError when a band (attribute) split breaks reading D-ATTR."""
+    ts, ops = graph["tensors"], graph["ops"]
+    producer, consumers = {}, {}
+    for o in ops:
+        for t in o["outputs"]:
+            producer[t] = o
+        for t in o["inputs"]:
+            consumers.setdefault(t, []).append(o)
+    for t in ts:
+        tid = t["id"]
+        if not is_attr(graph, cfg, tid):
+            continue
+        p = cfg[tid][1]
+        if len(t["shape"]) != 4 or t["shape"][1] % p:
+            raise ValueError(f"tensor {tid}: a band split needs an NHWC activation with H % p == 0")
+        po = producer[tid]
+        if po["kind"] in ATTR_LOCAL:
+            for x in po["inputs"]:
+                if ts[x]["kind"] == "act" and (not is_attr(graph, cfg, x) or cfg[x][1] != p):
+                    raise ValueError(f"tensor {tid}: a band-local producer needs band-split inputs of the same p")
+        elif po["kind"] in ATTR_WINDOW:
+            x = po["inputs"][0]
+            if not is_attr(graph, cfg, x) and cfg[x][1] != 1:
+                raise ValueError(f"tensor {tid}: its window producer's input must be unsplit or band-split")
+        else:
+            raise ValueError(f"tensor {tid}: producer {po['kind']} cannot write bands")
+        for c in consumers.get(tid, []):
+            y = c["outputs"][0]
+            if c["kind"] in ATTR_LOCAL:
+                if not is_attr(graph, cfg, y) or cfg[y][1] != p:
+                    raise ValueError(f"tensor {tid}: a band-local consumer needs a band-split output of the same p")
+            elif c["kind"] in ATTR_WINDOW:
+                if dim_of(cfg, y) == 1 and cfg[y][1] > 1:
+                    raise ValueError(f"tensor {tid}: a window consumer's output cannot be channel-split")
+            else:
+                raise ValueError(f"tensor {tid}: consumer {c['kind']} cannot read bands")
+
+
 def lag_of(cfg, t):
     """Release lag of a swapped tensor (reading D-LAG): the number of compute
     items after its swap-out before its range returns to the pool (0: at the swap-out)."""
@@ -103,8 +184,8 @@ def check_channel(graph, cfg):
 
     for t in ts:
         tid = t["id"]
-        if dim_of(cfg, tid) not in (0, 1):
-            raise ValueError(f"tensor {tid}: split dim must be 0 (samples) or 1 (channels)")
+        if dim_of(cfg, tid) not in (0, 1, 2):
+            raise ValueError(f"tensor {tid}: split dim must be 0 (samples), 1 (channels) or 2 (height)")
         if not chan(tid):
             continue
         p = cfg[tid][1]
@@ -217,6 +298,7 @@ class Analysis:
     has_bwd: list
     saved: list             # op id -> tensor ids bwd reads (non-param)
     bytes_: list
+    temp: dict = field(default_factory=dict)   # staging temporary (key >= 2n, piece) -> bytes (D-ATTR)
 
 
 def analyze(graph):
@@ -252,6 +334,25 @@ def analyze(graph):
     return Analysis(n, producer, sample, is_loss, ng, has_bwd, saved, [tbytes(t) for t in ts])
 
 
+def staged_rows(graph, cfg, o, k, P):
+    """(lo, hi, Hs, samples) of the staged input of micro-op k of window op o (D-ATTR): band
+    mode stages rows band_rows(k) of every sample, sample mode every row of B / P samples."""
+    ts, op = graph["tensors"], graph["ops"][o]
+    if is_attr(graph, cfg, op["outputs"][0]):
+        lo, hi, hs = band_rows(op, ts, k, P)
+        return lo, hi, hs, graph["samples"]
+    lo, hi, hs = band_rows(op, ts, 0, 1)
+    return lo, hi, hs, graph["samples"] // P
+
+
+def staged_bytes(graph, cfg, o, k, P):
+    ts, op = graph["tensors"], graph["ops"][o]
+    x = ts[op["inputs"][0]]
+    R, s, pad = window_geom(op, ts)
+    _, _, hs, nb = staged_rows(graph, cfg, o, k, P)
+    return nb * hs * (x["shape"][2] + 2 * pad) * x["shape"][3] * DTYPE_BYTES[x["dtype"]]
+
+
 @dataclass
 class Item:
     kind: str          # 'F' forward, 'B' backward, 'R' recompute replay, 'SO' swap-out, 'SI' swap-in
@@ -260,6 +361,7 @@ class Item:
     reads: list = field(default_factory=list)    # (key, piece)
     writes: list = field(default_factory=list)
     group: int = -1    # backward group id (replays + the B item they serve)
+    temps: list = field(default_factory=list)    # staging temporaries live during the item (D-ATTR)
 
 
 class Pool:
@@ -326,7 +428,9 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
     order = order if order is not None else schedule(graph)
     ts, ops = graph["tensors"], graph["ops"]
     n = an.n
+    an.temp = {}
     check_channel(graph, cfg)
+    check_attr(graph, cfg)
 
     def p_of(t):
         if t >= n:
@@ -341,11 +445,24 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
     def P_op(o):
         if cmode(o):  # channel mode: one micro-op per channel block of the output (D-CH)
             return max(p_of(t) for t in ops[o]["outputs"] if chan(t))
+        if amode(o):  # attribute mode: one micro-op per band of the output (D-ATTR)
+            return max(p_of(t) for t in ops[o]["outputs"] if band(t))
         P = 1
         for t in ops[o]["inputs"] + ops[o]["outputs"]:
-            if an.sample[t] and not chan(t):
+            if an.sample[t] and not chan(t) and not band(t):
                 P = max(P, p_of(t))
         return P
+
+    def band(t):
+        if t >= n:
+            t -= n
+        return an.sample[t] and is_attr(graph, cfg, t)
+
+    def amode(o):
+        return any(band(t) for t in ops[o]["outputs"])
+
+    def staged(o):
+        return ops[o]["kind"] in ATTR_WINDOW and (band(ops[o]["inputs"][0]) or amode(o))
 
     def chan(t):
         if t >= n:
@@ -363,7 +480,27 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
             if cmode(o) and (t in ops[o]["outputs"] or ops[o]["kind"] in CHANNEL_EW):
                 return [k]
             return list(range(p_of(t)))
+        if band(t):
+            if ops[o]["kind"] in ATTR_WINDOW and t == ops[o]["inputs"][0]:
+                # the bands holding the rows the staged input of micro-op k covers
+                lo, hi, _, _ = staged_rows(graph, cfg, o, k, P)
+                H = ts[t]["shape"][1]
+                hb = H // p_of(t)
+                lo, hi = max(lo, 0), min(hi, H - 1)
+                if lo > hi:
+                    raise ValueError(f"op {o}: micro-op {k} reads no input row")
+                return list(range(lo // hb, hi // hb + 1))
+            return [k]
         return [k * p_of(t) // P]
+
+    def add_temps(o, k, P, bwd):
+        if not staged(o):
+            return []
+        nb = staged_bytes(graph, cfg, o, k, P)
+        keys = [(2 * n + o, k)] + ([(3 * n + o, k)] if bwd else [])
+        for pc in keys:
+            an.temp[pc] = nb
+        return keys
 
     def ins_sample(o):
         return [t for t in ops[o]["inputs"] if an.sample[t]]
@@ -380,6 +517,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
                         if (t, j) not in it.reads:
                             it.reads.append((t, j))
             it.writes = [(t, j) for t in ops[o]["outputs"] for j in pieces(t, k, P, o)]
+            it.temps = add_temps(o, k, P, False)
             items.append(it)
     fwd_end = len(items)
 
@@ -413,6 +551,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
                     r = Item("R", po, kk, group=gid)
                     r.reads = [(u, jj) for u in ins_sample(po) for jj in pieces(u, kk, Q, po)]
                     r.writes = [(t, j)]
+                    r.temps = add_temps(po, kk, Q, False)
                     group.append(r)
                 live_temp.add((t, j))
                 cache[(t, j)] = piece_nbytes(t)
@@ -426,6 +565,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
             for (t, j) in saved_pieces:
                 need(t, j)
             b = Item("B", o, k, group=gid)
+            b.temps = add_temps(o, k, P, True)
             b.reads = list(saved_pieces)
             for t in ops[o]["outputs"]:
                 if not an.is_loss[t] and t in an.needs_grad:
@@ -533,10 +673,11 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
         allocs = alloc_at.get(i, [])
         ordered = [pc for pc in it.writes if pc in allocs] + [pc for pc in it.reads if pc in allocs and pc not in it.writes]
         assert len(ordered) == len(set(allocs)), (it, allocs)
+        ordered += it.temps  # staging temporaries last (D-ATTR)
         if ordered:
             f_alloc[idx] = ordered
-        if i in free_after or i in lag_free:
-            f_free[idx] = sorted(free_after.get(i, []) + lag_free.get(i, []))
+        if i in free_after or i in lag_free or it.temps:
+            f_free[idx] = sorted(free_after.get(i, []) + lag_free.get(i, []) + it.temps)
         for pc in sorted(swap_out_after.get(i, [])):
             so = Item("SO")
             so.reads = [pc]
@@ -569,6 +710,8 @@ def simulate(graph, cfg=None, order=None, capacity=INF, cache_bytes=0):
 
     def pbytes(pc):
         key, j = pc
+        if key >= 2 * n:
+            return an.temp[pc]
         t = key - n if key >= n else key
         if not an.sample[t] or ts[t]["kind"] != "act":
             return an.bytes_[t]

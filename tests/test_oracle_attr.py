@@ -1,0 +1,156 @@
+"""Attribute (height) splits, reading D-ATTR (Fig. 10, Fig. 6):
+the staged-row geometry against a brute-force scan of the direct convolution loop, any band /
+sample / swap / recompute plan computing the unsplit gradients (T1) in fp64, and the pool
+trace accounting for the staging temporaries."""
+
+import random
+
+import numpy as np
+import pytest
+
+from conftest import rel_errs
+from oracle import execplan, net, sim
+from tsinputs import gen, graphs
+
+
+def _rows_touched(H, R, s, pad, out_lo, out_hi):
+    """Input rows the direct window loop (ops.conv2d_fwd docstring: X[n, p*st + r - pad])
+    reads for output rows [out_lo, out_hi), padding rows included."""
+    rows = {p * s + r - pad for p in range(out_lo, out_hi) for r in range(R)}
+    return min(rows), max(rows)
+
+
+@pytest.mark.parametrize("H,R,s,pad,P", [(8, 3, 1, 1, 2), (8, 3, 1, 1, 4), (32, 7, 2, 3, 4), (16, 1, 2, 0, 2),
+                                        (16, 3, 2, 1, 4), (8, 2, 2, 0, 2), (16, 3, 2, 1, 2), (12, 1, 1, 0, 3)])
+def test_band_rows_equal_the_direct_loop(H, R, s, pad, P):
+    Ho = (H + 2 * pad - R) // s + 1
+    ts = [{"shape": (1, H, H, 4)}, {"shape": (4, R, R, 4)}, {"shape": (1, Ho, Ho, 4)}]
+    conv = {"kind": "conv2d", "inputs": [0, 1], "outputs": [2], "iattrs": [s, pad]}
+    pool = {"kind": "maxpool", "inputs": [0], "outputs": [2], "iattrs": [R, s, pad]}
+    hb = Ho // P
+    for op in (conv, pool):
+        assert sim.window_geom(op, ts) == (R, s, pad)
+        for k in range(P):
+            lo, hi, hs = sim.band_rows(op, ts, k, P)
+            assert (lo, hi) == _rows_touched(H, R, s, pad, k * hb, (k + 1) * hb)
+            assert hs == hi - lo + 1 and (hs - R) // s + 1 == hb   # the unpadded window op yields the band
+
+
+def _components(g):
+    """Groups of 4-D activations joined by band-local ops (they must share one band split)."""
+    ts, ops = g["tensors"], g["ops"]
+    parent = {t["id"]: t["id"] for t in ts if t["kind"] == "act" and len(t["shape"]) == 4}
+
+    def find(a):
+        while parent[a] != a:
+            a = parent[a]
+        return a
+    for o in ops:
+        if o["kind"] in sim.ATTR_LOCAL:
+            for x in o["inputs"]:
+                if x in parent:
+                    parent[find(x)] = find(o["outputs"][0])
+    comp = {}
+    for t in parent:
+        comp.setdefault(find(t), []).append(t)
+    return list(comp.values())
+
+
+def _rand_attr_cfg(g, r, ps=(2, 4)):
+    ts = g["tensors"]
+    acts = [t["id"] for t in ts if t["kind"] == "act" and t["name"] != "loss"]
+    for _ in range(200):
+        cfg = {t["id"]: (0, 1, 1) for t in ts}
+        for t in acts:
+            cfg[t] = (r.choice([0, 1, 2]), r.choice([1, 2]), 1)
+        for comp in _components(g):
+            mode = r.choice(["band", "band", "sample", "none"])
+            p = r.choice(ps)
+            for t in comp:
+                opt = cfg[t][0]
+                if mode == "band":
+                    cfg[t] = (opt, p, 1, 2)
+                elif mode == "sample":
+                    cfg[t] = (opt, p, 1, 0)
+                else:
+                    cfg[t] = (opt, 1, 1)
+        try:
+            sim.expand(g, cfg)
+        except ValueError:
+            continue
+        if any(sim.is_attr(g, cfg, t) for t in acts):
+            return cfg
+    raise AssertionError("no legal band plan drawn")
+
+
+@pytest.mark.parametrize("gname,seed", [("vgg_tiny", 0), ("vgg_tiny", 1), ("resnet_tiny", 0), ("resnet_tiny", 1),
+                                        ("resnet_tiny", 2)])
+def test_t1_band_plans_compute_the_unsplit_gradients(gname, seed):
+    g = graphs.config_graph(gname, dtype="f32")
+    P, I = gen.init_params(g), gen.make_inputs(g)
+    loss, pg, _, _ = net.train_step(g, P, I)
+    r = random.Random(seed)
+    for trial in range(2):
+        cfg = _rand_attr_cfg(g, r)
+        l2, pg2 = execplan.execute(g, cfg, P, I, cache_bytes=r.choice([0, 1 << 20]))
+        assert abs(l2 - loss) <= 1e-12 * abs(loss)
+        assert max(rel_errs(pg2, pg).values()) <= 1e-12
+
+
+def test_batch1_band_split_lowers_the_peak():
+    """Fig. 6: at batch 1 the sample dim cannot be split; splitting the height
+    lowers the swapped plan's peak, staging temporaries included."""
+    g = graphs.config_graph("vgg_tiny", dtype="f32", batch=1)
+    comps = _components(g)
+    base = {t["id"]: (0, 1, 1) for t in g["tensors"]}
+    acts = [t["id"] for t in g["tensors"] if t["kind"] == "act" and t["name"] != "loss"]
+    for t in acts:
+        base[t] = (sim.SWAP, 1, 1)
+    band = dict(base)
+    for comp in comps:
+        trial = dict(band)
+        for t in comp:
+            trial[t] = (sim.SWAP, 4, 1, 2)
+        try:
+            sim.expand(g, trial)
+            band = trial
+        except ValueError:   # the group feeding the flatten stays whole
+            pass
+    r0 = sim.simulate(g, base)
+    r1 = sim.simulate(g, band)
+    assert r1.peak_live < r0.peak_live
+    temps = [e for e in r1.trace if e[3] >= 2 * len(g["tensors"])]
+    assert temps and all(e[6] > 0 for e in temps)
+    # every temporary is freed by the item that allocated it
+    seen = {}
+    for seq, item, kind, key, j, off, nb in temps:
+        if kind == "A":
+            seen[(key, j)] = item
+        else:
+            assert seen.pop((key, j)) == item
+    assert not seen
+
+
+def test_band_split_legality():
+    g = graphs.config_graph("vgg_tiny", dtype="f32")
+    ts = g["tensors"]
+    byname = {t["name"]: t["id"] for t in ts}
+    cfg = {t["id"]: (0, 1, 1) for t in ts}
+    cfg[byname["conv0"]] = (0, 2, 1, 2)   # relu0 reads it: a band-local consumer needs the same split
+    with pytest.raises(ValueError):
+        sim.expand(g, cfg)
+    cfg[byname["relu0"]] = (0, 2, 1, 2)
+    sim.expand(g, cfg)
+    cfg[byname["relu0"]] = (0, 4, 1, 2)
+    with pytest.raises(ValueError):
+        sim.expand(g, cfg)
+    last = [t for t in ts if t["kind"] == "act" and len(t["shape"]) == 4][-1]   # read by flatten
+    cfg2 = {t["id"]: (0, 1, 1) for t in ts}
+    cfg2[last["id"]] = (0, 2, 1, 2)
+    with pytest.raises(ValueError):
+        sim.expand(g, cfg2)
+    cfg3 = {t["id"]: (0, 1, 1) for t in ts}
+    cfg3[byname["conv0"]] = (0, 3, 1, 2)  # H % p != 0
+    cfg3[byname["relu0"]] = (0, 3, 1, 2)
+    with pytest.raises(ValueError):
+        sim.expand(g, cfg3)
