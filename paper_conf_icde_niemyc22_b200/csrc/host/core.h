@@ -82,6 +82,7 @@ enum ItemKind : int { IT_F = 0, IT_B = 1, IT_R = 2, IT_SO = 3, IT_SI = 4 };
 struct Item {
   int kind = IT_F, op = -1, k = 0, group = -1;
   std::vector<PieceKey> reads, writes;
+  std::vector<PieceKey> temps;  // D-ATTR staging temporaries (key 2n + op / 3n + op), live during the item
 };
 
 struct Expansion {
@@ -90,12 +91,32 @@ struct Expansion {
   std::vector<std::vector<PieceKey>> free_after;
   int fwd_end = 0;
   std::vector<int> P;  // micro-op count per op
+  std::unordered_map<PieceKey, uint64_t> temp_bytes;  // D-ATTR staging temporaries
+  uint64_t bytes(const Graph& g, const std::vector<Cfg>& cfg, PieceKey pc) const;
 };
 
 // D-CH channel (parameter-dim) splits (expand.cpp)
 bool is_chan(const Graph& g, const std::vector<Cfg>& cfg, int key);
 bool channel_mode(const Graph& g, const std::vector<Cfg>& cfg, int op);
 bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why);
+
+// D-ATTR attribute (height) splits (expand.cpp; oracle/sim.py check_attr / staged_rows)
+bool is_attr(const Graph& g, const std::vector<Cfg>& cfg, int key);
+bool attr_mode(const Graph& g, const std::vector<Cfg>& cfg, int op);   // an output is band-split
+bool attr_window(int kind);                                              // conv2d / maxpool
+bool attr_staged(const Graph& g, const std::vector<Cfg>& cfg, int op);  // window op reading / writing bands
+bool attr_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why);
+struct Window {
+  int R, stride, pad;
+};
+Window window_geom(const Graph& g, int op);
+struct Staged {
+  int64_t lo, hi, hs, nb;  // input rows [lo, hi] (padding rows included), hs rows, nb samples
+};
+// staged input of micro-op k (of P) of window op `op`: band mode stages rows band k needs of
+// every sample, sample mode (a full merge) every row of samples block k
+Staged staged_rows(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P);
+uint64_t staged_bytes(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P);
 
 struct Event {
   int64_t seq;

@@ -46,7 +46,7 @@ static bool chan_ew(int kind) { return kind == TS_OP_RELU || kind == TS_OP_GELU 
 
 bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
   for (int t = 0; t < g.n(); ++t) {
-    if (cfg[t].dim != 0 && cfg[t].dim != 1) return (why = "split dim must be 0 (samples) or 1 (channels)"), false;
+    if (cfg[t].dim < 0 || cfg[t].dim > 2) return (why = "split dim must be 0 (samples), 1 (channels) or 2 (height)"), false;
     if (!is_chan(g, cfg, t)) continue;
     const Tensor& x = g.t[t];
     const int p = cfg[t].p;
@@ -79,27 +79,130 @@ bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
   return true;
 }
 
+// Attribute (height) split, reading D-ATTR (Fig. 10; oracle/sim.py
+// check_attr): a 4-D NHWC activation split along H into p bands [B, H/p, W, C].
+bool is_attr(const Graph& g, const std::vector<Cfg>& cfg, int key) {
+  int t = key >= g.n() ? key - g.n() : key;
+  const Tensor& x = g.t[t];
+  return x.sample && x.kind == TS_ACT && cfg[t].dim == 2 && cfg[t].p > 1;
+}
+bool attr_mode(const Graph& g, const std::vector<Cfg>& cfg, int op) {
+  for (int x : g.ops[op].out)
+    if (is_attr(g, cfg, x)) return true;
+  return false;
+}
+static bool attr_local(int kind) { return kind == TS_OP_RELU || kind == TS_OP_ADD || kind == TS_OP_BATCHNORM; }
+bool attr_window(int kind) { return kind == TS_OP_CONV2D || kind == TS_OP_MAXPOOL; }
+bool attr_staged(const Graph& g, const std::vector<Cfg>& cfg, int op) {
+  const Op& o = g.ops[op];
+  return attr_window(o.kind) && (is_attr(g, cfg, o.in[0]) || attr_mode(g, cfg, op));
+}
+
+Window window_geom(const Graph& g, int op) {
+  const Op& o = g.ops[op];
+  if (o.kind == TS_OP_CONV2D) return {int(g.t[o.in[1]].shape[1]), int(o.ia[0]), int(o.ia[1])};
+  return {int(o.ia[0]), int(o.ia[1]), int(o.ia[2])};
+}
+
+Staged staged_rows(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P) {
+  const Op& o = g.ops[op];
+  const Window w = window_geom(g, op);
+  const bool band = is_attr(g, cfg, o.out[0]);
+  const int64_t ho = g.t[o.out[0]].shape[1];
+  const int64_t hb = band ? ho / P : ho;
+  const int kk = band ? k : 0;
+  Staged s;
+  s.lo = kk * hb * w.stride - w.pad;
+  s.hi = ((kk + 1) * hb - 1) * w.stride - w.pad + w.R - 1;
+  s.hs = s.hi - s.lo + 1;
+  s.nb = band ? g.samples : g.samples / P;
+  return s;
+}
+
+uint64_t staged_bytes(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P) {
+  const Tensor& x = g.t[g.ops[op].in[0]];
+  const Window w = window_geom(g, op);
+  const Staged s = staged_rows(g, cfg, op, k, P);
+  return uint64_t(s.nb * s.hs * (x.shape[2] + 2 * w.pad) * x.shape[3]) * uint64_t(dtype_bytes(x.dtype));
+}
+
+bool attr_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
+  for (int t = 0; t < g.n(); ++t) {
+    if (!is_attr(g, cfg, t)) continue;
+    const Tensor& x = g.t[t];
+    const int p = cfg[t].p;
+    if (x.ndim != 4 || x.shape[1] % p) return (why = "a band split needs an NHWC activation with H % p == 0"), false;
+    const Op& po = g.ops[x.producer];
+    if (attr_local(po.kind)) {
+      for (int u : po.in)
+        if (g.t[u].kind == TS_ACT && (!is_attr(g, cfg, u) || cfg[u].p != p))
+          return (why = "a band-local producer needs band-split inputs of the same p"), false;
+    } else if (attr_window(po.kind)) {
+      const int u = po.in[0];
+      if (!is_attr(g, cfg, u) && cfg[u].p != 1)
+        return (why = "a band-split window output needs an unsplit or band-split input"), false;
+    } else {
+      return (why = "only conv2d / maxpool / relu / add / batchnorm can write bands"), false;
+    }
+    for (int c : x.consumers) {
+      const Op& co = g.ops[c];
+      const int y = co.out[0];
+      if (attr_local(co.kind)) {
+        if (!is_attr(g, cfg, y) || cfg[y].p != p)
+          return (why = "a band-local consumer needs a band-split output of the same p"), false;
+      } else if (attr_window(co.kind)) {
+        if (is_chan(g, cfg, y)) return (why = "a window op reading bands cannot write channel blocks"), false;
+      } else {
+        return (why = "only conv2d / maxpool / relu / add / batchnorm can read bands"), false;
+      }
+    }
+  }
+  // every band of a band-mode window op reads at least one input row
+  for (auto& o : g.ops) {
+    if (!attr_window(o.kind) || !attr_mode(g, cfg, o.id)) continue;
+    const int P = cfg[o.out[0]].p;
+    const int64_t H = g.t[o.in[0]].shape[1];
+    for (int k = 0; k < P; ++k) {
+      const Staged s = staged_rows(g, cfg, o.id, k, P);
+      if (std::max<int64_t>(s.lo, 0) > std::min<int64_t>(s.hi, H - 1))
+        return (why = "a band of a window op reads no input row"), false;
+    }
+  }
+  return true;
+}
+
+uint64_t Expansion::bytes(const Graph& g, const std::vector<Cfg>& cfg, PieceKey pc) const {
+  if (pk_key(pc) >= 2 * g.n()) return temp_bytes.at(pc);
+  return piece_bytes(g, cfg, pk_key(pc));
+}
+
 void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t cache_bytes) {
   const int n = g.n();
   ex = Expansion();
   ex.P.assign(g.ops.size(), 1);
-  std::vector<char> cm(g.ops.size(), 0);
+  std::vector<char> cm(g.ops.size(), 0), am(g.ops.size(), 0), st(g.ops.size(), 0);
   for (auto& o : g.ops) {
     int P = 1;
     cm[o.id] = channel_mode(g, cfg, o.id) ? 1 : 0;
+    am[o.id] = attr_mode(g, cfg, o.id) ? 1 : 0;
+    st[o.id] = attr_staged(g, cfg, o.id) ? 1 : 0;
     if (cm[o.id]) {  // D-CH: one micro-op per channel block of the output
       for (int x : o.out)
         if (is_chan(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
+    } else if (am[o.id]) {  // D-ATTR: one micro-op per band of the output
+      for (int x : o.out)
+        if (is_attr(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
     } else {
       for (int x : o.in)
-        if (g.t[x].sample && !is_chan(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
+        if (g.t[x].sample && !is_chan(g, cfg, x) && !is_attr(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
       for (int x : o.out)
-        if (g.t[x].sample && !is_chan(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
+        if (g.t[x].sample && !is_chan(g, cfg, x) && !is_attr(g, cfg, x)) P = std::max(P, piece_count(g, cfg, x));
     }
     ex.P[o.id] = P;
   }
   // the pieces of t (or of its gradient) micro-op k of op `op` touches (D-CH: a channel-split
-  // tensor is block k in its channel-mode producer / elementwise consumer, else all blocks)
+  // tensor is block k in its channel-mode producer / elementwise consumer, else all blocks;
+  // D-ATTR: a band-split window input is the bands holding the staged rows, else band k)
   auto pieces = [&](int t, int k, int P, int op) -> std::vector<int> {
     if (!g.t[t].sample) return {0};
     if (is_chan(g, cfg, t)) {
@@ -109,7 +212,26 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       for (size_t j = 0; j < all.size(); ++j) all[j] = int(j);
       return all;
     }
+    if (is_attr(g, cfg, t)) {
+      const Op& o = g.ops[op];
+      if (attr_window(o.kind) && o.in[0] == t) {
+        const Staged s = staged_rows(g, cfg, op, k, P);
+        const int64_t H = g.t[t].shape[1], hb = H / piece_count(g, cfg, t);
+        const int64_t lo = std::max<int64_t>(s.lo, 0), hi = std::min<int64_t>(s.hi, H - 1);
+        std::vector<int> js;
+        for (int64_t j = lo / hb; j <= hi / hb; ++j) js.push_back(int(j));
+        return js;
+      }
+      return {k};
+    }
     return {k * piece_count(g, cfg, t) / P};
+  };
+  auto add_temps = [&](Item& it, int op, int k, int P, bool bwd) {
+    if (!st[op]) return;
+    const uint64_t b = staged_bytes(g, cfg, op, k, P);
+    it.temps.push_back(pk(2 * n + op, k));
+    if (bwd) it.temps.push_back(pk(3 * n + op, k));
+    for (PieceKey pc : it.temps) ex.temp_bytes[pc] = b;
   };
   std::vector<Item>& items = ex.items;
   // ---- forward phase: op-major micro-ops (R10) ------------------------------
@@ -131,6 +253,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
               if (std::find(it.reads.begin(), it.reads.end(), pk(x, j)) == it.reads.end()) it.reads.push_back(pk(x, j));
       for (int x : op.out)
         for (int j : pieces(x, k, P, o)) it.writes.push_back(pk(x, j));
+      add_temps(it, o, k, P, false);
       items.push_back(std::move(it));
     }
   }
@@ -179,6 +302,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
             if (g.t[u].sample)
               for (int jj : pieces(u, kk, Q, po.id)) r.reads.push_back(pk(u, jj));
           r.writes.push_back(pk(t, j));
+          add_temps(r, po.id, kk, Q, false);
           group.push_back(std::move(r));
         }
         regenerated.insert(pk(t, j));
@@ -197,6 +321,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       b.op = op.id;
       b.k = k;
       b.group = gid;
+      add_temps(b, op.id, k, P, true);
       b.reads = saved;
       for (int x : op.out)
         if (!g.t[x].is_loss && g.t[x].needs_grad) {
@@ -319,8 +444,10 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
     for (PieceKey p : it.reads)
       if (std::find(al.begin(), al.end(), p) != al.end() && std::find(order.begin(), order.end(), p) == order.end())
         order.push_back(p);
+    order.insert(order.end(), it.temps.begin(), it.temps.end());  // staging temporaries last (D-ATTR)
     std::vector<PieceKey> fr = free_after[i];
     fr.insert(fr.end(), lag_free[i].begin(), lag_free[i].end());
+    fr.insert(fr.end(), it.temps.begin(), it.temps.end());
     std::sort(fr.begin(), fr.end());
     ex.alloc_at.push_back(order);
     ex.free_after.push_back(fr);
@@ -411,7 +538,7 @@ bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, 
   int64_t seq = 0;
   bool ok = true;
   auto do_alloc = [&](int item, PieceKey pc) {
-    uint64_t b = piece_bytes(g, cfg, pk_key(pc)), off = 0;
+    uint64_t b = ex.bytes(g, cfg, pc), off = 0;
     if (!pool.alloc(b, &off)) {
       ok = false;
       return;
@@ -435,7 +562,7 @@ bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, 
     if (placements && item >= 0) (*placements)[item].push_back({pc, off});
   };
   auto do_free = [&](int item, PieceKey pc) {
-    uint64_t b = piece_bytes(g, cfg, pk_key(pc));
+    uint64_t b = ex.bytes(g, cfg, pc);
     auto it = where.find(pc);
     uint64_t off = it->second;
     where.erase(it);
@@ -460,13 +587,13 @@ bool simulate(const Graph& g, const std::vector<Cfg>& cfg, const Expansion& ex, 
     r.top[i] = top;
     r.live[i] = live;
     peak = std::max(peak, live);
-    if (it.kind == IT_SO) r.d2h += piece_bytes(g, cfg, pk_key(it.reads[0]));
-    else if (it.kind == IT_SI) r.h2d += piece_bytes(g, cfg, pk_key(it.writes[0]));
+    if (it.kind == IT_SO) r.d2h += ex.bytes(g, cfg, it.reads[0]);
+    else if (it.kind == IT_SI) r.h2d += ex.bytes(g, cfg, it.writes[0]);
     else if (it.kind == IT_R) ++r.n_replay;
     else ++r.n_compute;
     if (it.kind == IT_SO) {
       const PieceKey pc = it.reads[0];
-      Fence f{where.at(pc), align_up(piece_bytes(g, cfg, pk_key(pc))), (int)i};
+      Fence f{where.at(pc), align_up(ex.bytes(g, cfg, pc)), (int)i};
       pend_cs.push_back(f);
       pend_h2d.push_back(f);
     }

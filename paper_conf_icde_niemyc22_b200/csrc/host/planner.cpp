@@ -315,7 +315,7 @@ void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& 
   const int n = g.n();
   auto try_cfg = [&](const std::vector<Cfg>& cfg, PlanState& out) {
     std::string why;
-    if (!channel_ok(g, cfg, why)) return false;  // e.g. reverting one block of a D-CH chain
+    if (!channel_ok(g, cfg, why) || !attr_ok(g, cfg, why)) return false;  // e.g. reverting one block of a D-CH chain
     out.cfg = cfg;
     out.cache = ps.cache;
     plan_refresh(g, out, &pr);
@@ -782,7 +782,7 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
         if (chg.p == 1) cs.cfg[chg.t].dim = 0;
       }
       std::string why;
-      if (!channel_ok(g, cs.cfg, why)) return;
+      if (!channel_ok(g, cs.cfg, why) || !attr_ok(g, cs.cfg, why)) return;
       plan_refresh(g, cs, &pr);
       uint64_t nt = top_of_op(cs);
       if (nt >= cur_top) return;

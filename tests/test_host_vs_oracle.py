@@ -376,3 +376,45 @@ def test_plan_roofline_bounds():
     P1.set(names["l1.q"], tsplit.RECOMPUTE, 1, 1)
     s1, f1, b1 = P1.roofline(pk, bw)
     assert f1 == pytest.approx(P1.stats()["compute_flop"], rel=1e-12) and f1 > f
+
+
+@pytest.mark.parametrize("gname,seed", [("vgg_tiny", 0), ("vgg_tiny", 1), ("resnet_tiny", 0), ("resnet_tiny", 1),
+                                        ("vgg16", 2), ("resnet50", 3)])
+def test_trace_bit_exact_band_split_plans(gname, seed):
+    """D-ATTR attribute (height) splits: the C++ expansion, staging temporaries, pool and
+    trace equal the oracle simulator's bit for bit."""
+    from test_oracle_attr import _rand_attr_cfg
+    over = {"batch": 4} if gname in ("vgg16", "resnet50") else {}
+    g = graphs.config_graph(gname, **over)
+    cfg = _rand_attr_cfg(g, random.Random(200 + seed))
+    for t in brute.act_tensors(g):   # random D-LAG lags on swapped tensors
+        if cfg[t][0] == sim.SWAP and seed % 2:
+            cfg[t] = cfg[t][:3] + ((cfg[t][3] if len(cfg[t]) > 3 else 0), 2)
+    G = tsplit.Graph(g)
+    plan = tsplit.Plan.default(G)
+    plan.set_many({t: cfg[t] for t in brute.act_tensors(g)})
+    ref = sim.simulate(g, cfg)
+    got = plan.trace()
+    assert any(k >= 2 * len(g["tensors"]) for _, _, _, k, _, _, _ in got)   # staging temporaries present
+    assert len(got) == len(ref.trace)
+    for a, b in zip(got, ref.trace):
+        assert a == tuple(b), (a, b)
+    st = plan.stats()
+    assert (st["peak_live"], st["peak_extent"], st["n_replay"]) == (ref.peak_live, ref.peak_extent, ref.n_replay)
+    assert [it[0] for it in plan.items()] == [it.kind for it in ref.items]
+    for t in brute.act_tensors(g):
+        assert plan.get_dim(t) == (sim.dim_of(cfg, t) if cfg[t][1] > 1 else 0)
+
+
+def test_band_split_rejected_unless_legal():
+    g = graphs.config_graph("vgg_tiny")
+    names = {t["name"]: t["id"] for t in g["tensors"]}
+    plan = tsplit.Plan.default(tsplit.Graph(g))
+    with pytest.raises(tsplit.TsError):   # relu0 must follow conv0's band split
+        plan.set(names["conv0"], tsplit.RESIDE, 2, 1, dim=2)
+    plan.set_many({names["conv0"]: (0, 2, 1, 2), names["relu0"]: (0, 2, 1, 2)})
+    with pytest.raises(tsplit.TsError):   # a 2-D tensor has no height
+        plan.set(names["fc0"], tsplit.RESIDE, 2, 1, dim=2)
+    last = [t for t in g["tensors"] if t["kind"] == "act" and len(t["shape"]) == 4][-1]
+    with pytest.raises(tsplit.TsError):   # read by flatten
+        plan.set(last["id"], tsplit.RESIDE, 2, 1, dim=2)

@@ -57,30 +57,38 @@ def _components(g):
 
 
 def _rand_attr_cfg(g, r, ps=(2, 4)):
+    """A random legal plan with band splits: memory options at random, then each group of
+    band-joined tensors in turn takes a band split, a sample split or none when legal."""
     ts = g["tensors"]
     acts = [t["id"] for t in ts if t["kind"] == "act" and t["name"] != "loss"]
-    for _ in range(200):
-        cfg = {t["id"]: (0, 1, 1) for t in ts}
-        for t in acts:
-            cfg[t] = (r.choice([0, 1, 2]), r.choice([1, 2]), 1)
-        for comp in _components(g):
-            mode = r.choice(["band", "band", "sample", "none"])
-            p = r.choice(ps)
-            for t in comp:
-                opt = cfg[t][0]
-                if mode == "band":
-                    cfg[t] = (opt, p, 1, 2)
-                elif mode == "sample":
-                    cfg[t] = (opt, p, 1, 0)
-                else:
-                    cfg[t] = (opt, 1, 1)
+    cfg = {t["id"]: (0, 1, 1) for t in ts}
+    for t in acts:
+        cfg[t] = (r.choice([0, 1, 2]), 1, 1)
+    comps = _components(g)
+    r.shuffle(comps)
+    for comp in comps:
+        mode = r.choice(["band", "band", "sample", "none"])
+        p = r.choice(ps)
+        trial = dict(cfg)
+        for t in comp:
+            opt = cfg[t][0]
+            trial[t] = (opt, p, 1, 2) if mode == "band" else (opt, p, 1, 0) if mode == "sample" else (opt, 1, 1)
         try:
-            sim.expand(g, cfg)
+            sim.expand(g, trial)
+            cfg = trial
         except ValueError:
-            continue
-        if any(sim.is_attr(g, cfg, t) for t in acts):
-            return cfg
-    raise AssertionError("no legal band plan drawn")
+            pass
+    for t in acts:   # the rest of the 2-D tensors: sample splits
+        if len(ts[t]["shape"]) != 4 and cfg[t][1] == 1 and r.random() < 0.5:
+            trial = dict(cfg)
+            trial[t] = (cfg[t][0], 2, 1)
+            try:
+                sim.expand(g, trial)
+                cfg = trial
+            except ValueError:
+                pass
+    assert any(sim.is_attr(g, cfg, t) for t in acts), "no band split drawn"
+    return cfg
 
 
 @pytest.mark.parametrize("gname,seed", [("vgg_tiny", 0), ("vgg_tiny", 1), ("resnet_tiny", 0), ("resnet_tiny", 1),
