@@ -762,6 +762,123 @@ bool alloc_host_pool(ts_session_t* s, uint64_t bytes) {
   return cudaHostAlloc(reinterpret_cast<void**>(&s->host), bytes, cudaHostAllocDefault) == cudaSuccess;
 }
 
+// D-ATTR: micro-op k of a window op (conv2d / maxpool) whose input or output is band-split.
+// The rows its output block needs are staged into the item's pool temporary (key 2n + op,
+// padding written out: 0 for conv, -inf for max pooling) and the op runs unpadded on it; the
+// backward regathers, writes the staged input gradient to the second temporary (3n + op)
+// and adds it into the input gradient's pieces (overlapping halos sum), zeroing a
+// piece first when no earlier item wrote it.
+std::function<void(cudaStream_t)> lower_staged(ts_session_t* s, const Item& it, const Micro& m,
+                                               const std::unordered_map<PieceKey, uint64_t>& where,
+                                               const std::set<PieceKey>& gwritten, int& nk, std::string& why) {
+  const Graph& g = *s->g;
+  const int n = g.n();
+  const Op& o = g.ops[it.op];
+  const int dt = g.dtype == TS_BF16 ? tsk::BF16 : tsk::F32;
+  const int xi = o.in[0], yi = o.out[0];
+  const Tensor& x = g.t[xi];
+  const Tensor& y = g.t[yi];
+  const Window wg = window_geom(g, it.op);
+  const Staged sr = staged_rows(g, s->cfg, it.op, it.k, m.P);
+  const bool band_out = attr_mode(g, s->cfg, it.op);
+  const int H = int(x.shape[1]), W = int(x.shape[2]), C = int(x.shape[3]);
+  const int Wp = W + 2 * wg.pad;
+  const int b0 = band_out ? 0 : int(int64_t(it.k) * g.samples / m.P);
+  const int nb = int(sr.nb), lo = int(sr.lo), hs = int(sr.hs);
+  const int Pr = int(band_out ? y.shape[1] / m.P : y.shape[1]), Q = int(y.shape[2]);
+  const bool bwd = it.kind == IT_B;
+  auto at = [&](PieceKey pc) -> char* {
+    auto f = where.find(pc);
+    return f == where.end() ? nullptr : s->slab + f->second;
+  };
+  auto pieces_of = [&](int key, tsk::BandPieces& bp) {
+    const int px = is_attr(g, s->cfg, xi) ? piece_count(g, s->cfg, xi) : 1;
+    bp.hb = H / px;
+    for (int j = 0; j < px; ++j) bp.ptr[j] = at(pk(key, j));
+  };
+  tsk::BandPieces src;
+  pieces_of(xi, src);
+  char* tmp = at(pk(2 * n + it.op, it.k));
+  if (!tmp) return (why = "staging temporary not allocated"), nullptr;
+  const int fill = o.kind == TS_OP_MAXPOOL ? 1 : 0;
+  char* yv = m.val.count(yi) ? m.val.at(yi) : nullptr;
+  if (!bwd) {
+    if (!yv) return (why = "output block not resident"), nullptr;
+    if (o.kind == TS_OP_CONV2D) {
+      const Tensor& w = g.t[o.in[1]];
+      tsk::ConvArgs a;
+      a.dtype = dt; a.n = nb; a.H = hs; a.W = Wp; a.C = C;
+      a.K = int(w.shape[0]); a.R = int(w.shape[1]); a.S = int(w.shape[2]);
+      a.P = Pr; a.Q = Q; a.stride = wg.stride; a.pad = 0;
+      a.w = param_w(s, o.in[1]);
+      a.x = tmp;
+      const void* bias = o.in.size() > 2 ? param_w(s, o.in[2]) : nullptr;
+      nk = 2;
+      return [=](cudaStream_t st) {
+        tsk::band_gather(dt, src, H, W, C, b0, nb, lo, hs, wg.pad, fill, tmp, st);
+        tsk::conv_fprop(a, yv, bias, st);
+      };
+    }
+    nk = 2;
+    return [=](cudaStream_t st) {
+      tsk::band_gather(dt, src, H, W, C, b0, nb, lo, hs, wg.pad, fill, tmp, st);
+      tsk::maxpool_fwd(dt, tmp, yv, nb, hs, Wp, C, Pr, Q, wg.R, wg.stride, 0, st);
+    };
+  }
+  char* dy = m.grad.count(yi) ? m.grad.at(yi) : nullptr;
+  if (!dy) return (why = "output gradient block not resident"), nullptr;
+  char* tmp2 = at(pk(3 * n + it.op, it.k));
+  if (!tmp2) return (why = "staging temporary not allocated"), nullptr;
+  const bool gx = x.kind == TS_ACT && x.needs_grad;
+  tsk::BandPieces dst;
+  std::vector<std::pair<char*, uint64_t>> zero;
+  if (gx) {
+    pieces_of(n + xi, dst);
+    for (PieceKey pc : it.writes)
+      if (pk_key(pc) == n + xi && !gwritten.count(pc)) zero.push_back({at(pc), piece_bytes(g, s->cfg, n + xi)});
+  }
+  if (o.kind == TS_OP_CONV2D) {
+    const Tensor& w = g.t[o.in[1]];
+    tsk::ConvArgs a;
+    a.dtype = dt; a.n = nb; a.H = hs; a.W = Wp; a.C = C;
+    a.K = int(w.shape[0]); a.R = int(w.shape[1]); a.S = int(w.shape[2]);
+    a.P = Pr; a.Q = Q; a.stride = wg.stride; a.pad = 0;
+    a.w = param_w(s, o.in[1]);
+    a.x = tmp;
+    a.dy = dy;
+    float* dw = param_g(s, o.in[1]);
+    auto A = [&](int key) {
+      auto f = m.acc.find(key);
+      return f == m.acc.end() ? 0 : f->second;
+    };
+    const int dwacc = A(o.in[1]);
+    float* db = o.in.size() > 2 ? param_g(s, o.in[2]) : nullptr;
+    const int dbacc = db ? A(o.in[2]) : 0;
+    const int64_t pix = int64_t(nb) * Pr * Q;
+    float* ws = reinterpret_cast<float*>(s->slab + g.ws_off);
+    const uint64_t wsb = g.ws_bytes;
+    nk = 2 + (db ? 2 : 0) + (gx ? 2 : 0);
+    return [=](cudaStream_t st) {
+      tsk::band_gather(dt, src, H, W, C, b0, nb, lo, hs, wg.pad, 0, tmp, st);
+      tsk::conv_wgrad(a, dw, dwacc, st);
+      if (db) tsk::column_sum(dt, dy, pix, a.K, ws, wsb, db, dbacc, nullptr, 0, st);
+      if (gx) {
+        tsk::conv_dgrad(a, tmp2, 0, st);
+        for (auto& z : zero) cudaMemsetAsync(z.first, 0, z.second, st);
+        tsk::band_scatter_add(dt, tmp2, dst, H, W, C, b0, nb, lo, hs, wg.pad, st);
+      }
+    };
+  }
+  if (!gx) return (why = "max pooling of an input without gradient"), nullptr;
+  nk = 3;
+  return [=](cudaStream_t st) {
+    tsk::band_gather(dt, src, H, W, C, b0, nb, lo, hs, wg.pad, 1, tmp, st);
+    tsk::maxpool_bwd(dt, dy, tmp, tmp2, 0, nb, hs, Wp, C, Pr, Q, wg.R, wg.stride, 0, st);
+    for (auto& z : zero) cudaMemsetAsync(z.first, 0, z.second, st);
+    tsk::band_scatter_add(dt, tmp2, dst, H, W, C, b0, nb, lo, hs, wg.pad, st);
+  };
+}
+
 ts_status build_program(ts_session_t* s) {
   const Graph& g = *s->g;
   const int n = g.n();
@@ -806,6 +923,7 @@ ts_status build_program(ts_session_t* s) {
   std::set<int> act_grad_started;   // grad keys already written by an earlier bwd op
   std::map<int, int> grad_first_op; // grad key -> first bwd op writing it
   std::set<int> param_started;
+  std::set<PieceKey> gpiece_written;  // gradient pieces some earlier item wrote (D-ATTR accumulation)
   std::map<int, int> param_first_item;
   std::map<int, int> param_started_by;  // param -> op whose backward first wrote its gradient
   s->ev_d2h.assign(s->ex.items.size(), nullptr);
@@ -871,7 +989,9 @@ ts_status build_program(ts_session_t* s) {
       m.s0 = int64_t(it.k) * B / m.P;
       m.s1 = int64_t(it.k + 1) * B / m.P;
       const bool cmode = channel_mode(g, s->cfg, it.op);
-      if (cmode) {  // D-CH: micro-op k = output channel block k over every sample
+      const bool amode = attr_mode(g, s->cfg, it.op);      // D-ATTR: micro-op k = band k of every sample
+      const bool staged = attr_staged(g, s->cfg, it.op);   // D-ATTR window op on a staged input copy
+      if (cmode || amode) {  // D-CH: micro-op k = output channel block k over every sample
         m.cb = it.k;
         m.cp = m.P;
         m.s0 = 0;
@@ -886,7 +1006,7 @@ ts_status build_program(ts_session_t* s) {
         int t = key >= n ? key - n : key;
         const Tensor& x = g.t[t];
         if (!x.sample) return s->slab + where.at(pk(key, 0));
-        if (is_chan(g, s->cfg, t)) return s->slab + where.at(pk(key, m.k));  // own_block(t)
+        if (is_chan(g, s->cfg, t) || is_attr(g, s->cfg, t)) return s->slab + where.at(pk(key, m.k));  // own block / band
         int p = piece_count(g, s->cfg, t);
         int j = int(m.s0 * p / B);
         int64_t first = int64_t(j) * B / p;
@@ -900,6 +1020,13 @@ ts_status build_program(ts_session_t* s) {
       for (int t : ts_all) {
         if (g.t[t].kind == TS_PARAM) continue;
         int key = t;
+        if (is_attr(g, s->cfg, t)) {  // band k in attribute mode; a staged window input is gathered
+          if (amode && !(staged && t == o.in[0])) {
+            if (where.count(pk(t, m.k))) m.val[t] = view(t);
+            if (bwd && g.t[t].needs_grad && where.count(pk(n + t, m.k))) m.grad[t] = view(n + t);
+          }
+          continue;
+        }
         if (is_chan(g, s->cfg, t)) {
           const bool gr = bwd && g.t[t].needs_grad && g.t[t].kind == TS_ACT && !g.t[t].is_loss;
           if (own_block(t)) {
@@ -939,6 +1066,8 @@ ts_status build_program(ts_session_t* s) {
             m.acc[gk] = grad_first_op[gk] != it.op ? 1 : 0;
             // a channel-mode linear's micro-ops all write the whole dX: block 0 overwrites
             if (cmode && o.kind == TS_OP_LINEAR && !m.acc[gk] && m.k > 0) m.acc[gk] = 1;
+            // D-ATTR: a band's gradient is started by whichever item wrote it first
+            if (is_attr(g, s->cfg, t)) m.acc[gk] = gpiece_written.count(pk(gk, m.k)) ? 1 : 0;
           }
         }
       }
@@ -960,7 +1089,7 @@ ts_status build_program(ts_session_t* s) {
           L.np = p;
           for (int j = 0; j < p; ++j) {
             L.ptr[j] = s->slab + where.at(pk(key, j));
-            L.rows[j] = int64_t(B / p) * (g.t[t].elems_per_sample / C);
+            L.rows[j] = g.t[t].numel / C / p;  // (a sample block or a band: equal pieces)
           }
           return true;
         };
@@ -1123,13 +1252,30 @@ ts_status build_program(ts_session_t* s) {
         }
       }
       int nk = 0;
-      if (lg.G) {
+      // gradient pieces this item allocates without writing them (a band no staged window
+      // micro-op reaches, D-ATTR) hold zeros: the oracle's "no contribution"
+      std::vector<std::pair<char*, uint64_t>> zero_first;
+      for (PieceKey pc : s->ex.alloc_at[i])
+        if (pk_key(pc) >= n && pk_key(pc) < 2 * n && std::find(it.writes.begin(), it.writes.end(), pc) == it.writes.end())
+          zero_first.push_back({s->slab + where.at(pc), piece_bytes(g, s->cfg, pk_key(pc))});
+      if (staged) {
+        std::string why;
+        cmd.fn = lower_staged(s, it, m, where, gpiece_written, nk, why);
+        if (!cmd.fn) return set_error("band split (D-ATTR): " + why), TS_ERR_GRAPH;
+      } else if (lg.G) {
         cmd.fn = lower_linear_group(s, lg, bwd, nk);
       } else if (fused_away.count(int(i))) {
         cmd.fn = [](cudaStream_t) {};
       } else {
         cmd.fn = lower(s, m, bwd, nk, fz.mode ? &fz : nullptr);
         if (fz.mode) fused_away.insert(int(i) + 1);
+      }
+      if (!zero_first.empty()) {
+        auto body = std::move(cmd.fn);
+        cmd.fn = [zero_first, body](cudaStream_t st) {
+          for (auto& z : zero_first) cudaMemsetAsync(z.first, 0, z.second, st);
+          body(st);
+        };
       }
       s->launches += nk;
       if (bwd)
@@ -1138,6 +1284,8 @@ ts_status build_program(ts_session_t* s) {
             param_started.insert(t);
             param_started_by.emplace(t, it.op);
           }
+      for (PieceKey pc : it.writes)
+        if (pk_key(pc) >= n) gpiece_written.insert(pc);
     }
     // frees after this item
     while (ev < tr.size() && tr[ev].item == int(i) && tr[ev].kind == 1) {
