@@ -209,6 +209,11 @@ void timeline(const Graph& g, const PlanState& ps, const Profile& pr, Timeline& 
     for (int f : ps.sim.wait_so[i]) clock = std::max(clock, so_end_item[size_t(f)]);
     int l = lg2(ps.ex.P[it.op]);
     double t = (it.kind == IT_B ? pr.tb[it.op][l] : pr.tf[it.op][l]) / double(ps.ex.P[it.op]);
+    if (!it.temps.empty()) {  // D-ATTR staging: gather (read + write the staged rows), and in the
+                              // backward the scatter-add (read the staged gradient, read + write dX)
+      const double b = double(ps.ex.temp_bytes.at(it.temps[0]));
+      t += it.kind == IT_B ? 2 * pr.hw.launch_s + 5 * b / pr.hw.hbm_bw : pr.hw.launch_s + 2 * b / pr.hw.hbm_bw;
+    }
     start[i] = clock;
     tl.T[i] = t;
     clock += t;
@@ -712,6 +717,60 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
           step2.push_back(opt == TS_RECOMPUTE ? with_feeders(c, t) : c);
         }
       }
+    }
+    // D-ATTR: band (height) splits of the bottleneck op's 4-D activations, with every tensor
+    // a band-local op (ReLU, add, batch norm) ties to them — also only once the sample dim is
+    // exhausted (Fig. 6: the attribute dim is what is left at batch 1); illegal groups (one
+    // that feeds a flatten, a band without input rows) are dropped by attr_ok in consider()
+    auto band_group = [&](int t) {
+      std::vector<int> grp{t};
+      auto local = [](int kind) { return kind == TS_OP_RELU || kind == TS_OP_ADD || kind == TS_OP_BATCHNORM; };
+      for (size_t q = 0; q < grp.size(); ++q) {
+        const Tensor& u = g.t[grp[q]];
+        std::vector<int> nb;
+        if (u.producer >= 0 && local(g.ops[u.producer].kind))
+          for (int v : g.ops[u.producer].in) if (g.t[v].kind == TS_ACT) nb.push_back(v);
+        for (int c : u.consumers)
+          if (local(g.ops[c].kind)) nb.push_back(g.ops[c].out[0]);
+        for (int v : nb)
+          if (std::find(grp.begin(), grp.end(), v) == grp.end()) grp.push_back(v);
+      }
+      return grp;
+    };
+    std::vector<int> band_all;
+    for (int t : split_cands) {
+      const Tensor& x = g.t[t];
+      if (no_split || x.ndim != 4) continue;
+      const bool banded = is_attr(g, ps.cfg, t);  // a band split may grow finer
+      bool sample_room = false;
+      for (int p = 2 * ps.cfg[t].p; p <= 16 && !banded; p *= 2) sample_room |= g.samples % p == 0;
+      if (sample_room) continue;
+      const std::vector<int> grp = band_group(t);
+      for (int u : grp)
+        if (std::find(band_all.begin(), band_all.end(), u) == band_all.end()) band_all.push_back(u);
+      for (int p = 2; p <= 16; p *= 2) {
+        if (x.shape[1] % p) break;
+        if (banded && p <= ps.cfg[t].p) continue;
+        for (int opt : {TS_RESIDE, TS_SWAP, TS_RECOMPUTE}) {
+          if (opt != TS_RESIDE && first_bw[t] < 0) continue;
+          Cand2 c;
+          c.birth = birth[t];
+          c.tensor = t;
+          for (int u : grp) c.ch.push_back({u, u == t ? opt : ps.cfg[u].opt, p, ps.cfg[u].lead, 2});
+          step2.push_back(opt == TS_RECOMPUTE ? with_feeders(c, t) : c);
+        }
+      }
+    }
+    // the whole window micro-op in bands: its input's and its output's groups at once
+    for (int p = 2; p <= 16 && band_all.size() > 1; p *= 2) {
+      Cand2 c;
+      for (int u : band_all)
+        if (g.t[u].shape[1] % p == 0 && !(is_attr(g, ps.cfg, u) && ps.cfg[u].p >= p))
+          c.ch.push_back({u, ps.cfg[u].opt, p, ps.cfg[u].lead, 2});
+      if (c.ch.size() < 2) continue;
+      c.birth = birth[c.ch[0].t];
+      c.tensor = c.ch[0].t;
+      step2.push_back(c);
     }
     // D-R8e: a recomputed tensor regenerated for the bottleneck (a replay chain member,
     // P:L294) is allocated piece by piece at its own split; splitting it finer shrinks

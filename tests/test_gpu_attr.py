@@ -96,3 +96,31 @@ def test_batch1_vgg_band_chain_under_swap():
     l0, g0, S0, P0 = _run(g, {t: (sim.SWAP, 1, 1) for t in brute.act_tensors(g)})
     assert max(rel_errs(grads, g0).values()) <= 1e-6
     assert P.stats()["peak_live"] < P0.stats()["peak_live"]
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+def test_vgg16_batch1_planned_band_step(dtype):
+    """Full-size VGG-16 at batch 1 (224 x 224) planned at 45 % of its dynamic peak — below
+    what swap / recompute alone reach (65 %, tests/test_host_vs_oracle.py) — runs in budget
+    and trains the unsplit step's function (f32 3e-6 per tensor; bf16 1e-2 global)."""
+    g = graphs.config_graph("vgg16", batch=1, dtype=dtype)
+    G = tsplit.Graph(g)
+    st = tsplit.Plan.default(G).stats()
+    budget = st["static_bytes"] + int(0.45 * (st["peak_extent"] - st["static_bytes"]))
+    P = tsplit.Plan.plan(G, budget)
+    cfg = P.oracle_cfg()
+    assert any(c[1] > 1 and len(c) > 3 and c[3] == 2 for c in cfg.values())
+    S = tsplit.Session(G, P)   # (the planner's plan itself: its D-LRU cache is not in oracle_cfg)
+    S.set_params(gen.init_params(g))
+    loss = S.step(tsplit.inputs_to_device(G, gen.make_inputs(g)))
+    grads = S.grads()
+    assert S.trace() == P.trace() and P.stats()["peak_extent"] <= budget
+    assert S.trace() == [tuple(e) for e in sim.simulate(g, cfg, cache_bytes=P.stats()["recompute_cache_bytes"]).trace]
+    l0, g0, _, _ = _run(g)
+    if dtype == "f32":
+        assert abs(loss - l0) <= 1e-6 * abs(l0)
+        e0 = rel_errs(grads, g0)
+        assert max(e0.values()) <= 3e-6, sorted(e0.items(), key=lambda kv: -kv[1])[:5]
+    else:
+        assert abs(loss - l0) <= 1e-3 * abs(l0)
+        assert global_rel_err(grads, g0) <= 1e-2

@@ -418,3 +418,38 @@ def test_band_split_rejected_unless_legal():
     last = [t for t in g["tensors"] if t["kind"] == "act" and len(t["shape"]) == 4][-1]
     with pytest.raises(tsplit.TsError):   # read by flatten
         plan.set(last["id"], tsplit.RESIDE, 2, 1, dim=2)
+
+
+def test_planner_uses_band_splits_when_the_batch_is_one():
+    """Batch 1 (Fig. 6): with no sample dim Alg. 2's split step proposes the height
+    (D-ATTR).  VGG at half its dynamic peak is infeasible without splits and feasible with
+    bands; the plan's trace is the simulator's and executing it (fp64 oracle) gives the
+    unsplit gradients."""
+    from oracle import execplan, net
+    from tsinputs import gen
+    from test_oracle_net_sim import rel_errs
+    g = graphs.config_graph("vgg_small", batch=1, dtype="f32")
+    G = tsplit.Graph(g)
+    st = tsplit.Plan.default(G).stats()
+    budget = st["static_bytes"] + int(0.5 * (st["peak_extent"] - st["static_bytes"]))
+    with pytest.raises(tsplit.TsError):
+        tsplit.Plan.plan(G, budget, no_split=True)
+    P = tsplit.Plan.plan(G, budget)
+    assert P.stats()["peak_extent"] <= budget
+    cfg = P.oracle_cfg()
+    assert any(c[1] > 1 and len(c) > 3 and c[3] == 2 for c in cfg.values())
+    assert P.trace() == [tuple(e) for e in sim.simulate(g, cfg).trace]
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    l0, g0, _, _ = net.train_step(g, params, inputs)
+    l1, g1 = execplan.execute(g, cfg, params, inputs)
+    assert abs(l1 - l0) <= 1e-12 * abs(l0)
+    assert max(rel_errs(g1, g0).values()) <= 1e-12
+
+
+def test_band_plan_serialize_roundtrip():
+    g = graphs.config_graph("vgg_small", batch=1)
+    G = tsplit.Graph(g)
+    st = tsplit.Plan.default(G).stats()
+    P = tsplit.Plan.plan(G, st["static_bytes"] + int(0.5 * (st["peak_extent"] - st["static_bytes"])))
+    Q = tsplit.Plan.deserialize(G, P.serialize())
+    assert Q.trace() == P.trace() and Q.oracle_cfg() == P.oracle_cfg()
