@@ -497,7 +497,9 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
         if not staged(o):
             return []
         nb = staged_bytes(graph, cfg, o, k, P)
-        keys = [(2 * n + o, k)] + ([(3 * n + o, k)] if bwd else [])
+        x = ops[o]["inputs"][0]
+        dx = bwd and ts[x]["kind"] == "act" and x in an.needs_grad   # (the image takes no gradient)
+        keys = [(2 * n + o, k)] + ([(3 * n + o, k)] if dx else [])
         for pc in keys:
             an.temp[pc] = nb
         return keys

@@ -230,7 +230,8 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
     if (!st[op]) return;
     const uint64_t b = staged_bytes(g, cfg, op, k, P);
     it.temps.push_back(pk(2 * n + op, k));
-    if (bwd) it.temps.push_back(pk(3 * n + op, k));
+    const Tensor& x = g.t[g.ops[op].in[0]];
+    if (bwd && x.kind == TS_ACT && x.needs_grad) it.temps.push_back(pk(3 * n + op, k));  // (the image: no dX)
     for (PieceKey pc : it.temps) ex.temp_bytes[pc] = b;
   };
   std::vector<Item>& items = ex.items;

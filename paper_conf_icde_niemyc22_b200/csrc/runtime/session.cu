@@ -827,9 +827,9 @@ std::function<void(cudaStream_t)> lower_staged(ts_session_t* s, const Item& it, 
   }
   char* dy = m.grad.count(yi) ? m.grad.at(yi) : nullptr;
   if (!dy) return (why = "output gradient block not resident"), nullptr;
-  char* tmp2 = at(pk(3 * n + it.op, it.k));
-  if (!tmp2) return (why = "staging temporary not allocated"), nullptr;
   const bool gx = x.kind == TS_ACT && x.needs_grad;
+  char* tmp2 = gx ? at(pk(3 * n + it.op, it.k)) : nullptr;
+  if (gx && !tmp2) return (why = "staging temporary not allocated"), nullptr;
   tsk::BandPieces dst;
   std::vector<std::pair<char*, uint64_t>> zero;
   if (gx) {

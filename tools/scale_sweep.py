@@ -72,7 +72,7 @@ def run_phase(args):
     bytes) fits the box's host memory cap; plan-feasible batches beyond it are reported as
     HBM-feasible only."""
     import torch
-    res = json.load(open(OUT))
+    res = json.load(open(args.plans or OUT))
     free, total = torch.cuda.mem_get_info()
     res["device_free_bytes"] = free
     res["host_cap_bytes"] = args.host_cap_bytes
@@ -113,6 +113,7 @@ if __name__ == "__main__":
     ap.add_argument("--capacity-bytes", type=int, default=184404344832)
     ap.add_argument("--max-batch", type=int, default=8192)
     ap.add_argument("--steps", type=int, default=2)
+    ap.add_argument("--plans", default=None, help="plan-phase output to run (default: " + OUT + ")")
     ap.add_argument("--host-cap-bytes", type=int, default=100 * 2 ** 30,
                     help="largest pinned swap pool to run (the GPU box has ~196 GB of host RAM)")
     a = ap.parse_args()
