@@ -38,7 +38,7 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
     def rows_per_sample(t):
         return ts[t]["shape"][0] // B
 
-    def band(t):  # attribute (height) split (D-ATTR): p bands of rows, each over every sample
+    def band(t):  # attribute split (D-ATTR): p bands of rows (columns), each over every sample
         return an.sample[t] and sim.is_attr(graph, cfg, t)
 
     def amode(o):
@@ -49,8 +49,10 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
 
     def piece_shape(t):
         sh = list(ts[t]["shape"])
-        if chan(t) or band(t):
+        if chan(t):
             sh[1] //= p_of(t)
+        elif band(t):
+            sh[sim.axis_of(cfg, t)] //= p_of(t)
         elif an.sample[t]:
             sh[0] //= p_of(t)
         return tuple(sh)
@@ -130,12 +132,20 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
             else:
                 view(tid, 0, B, grad=True)[...] += g
 
-    def input_rows(x, b0, b1, r, grad=False):
-        """Row r of samples [b0, b1) of the window input x (band-split or unsplit)."""
-        if band(x):
-            hb = ts[x]["shape"][1] // p_of(x)
-            return store[(n + x if grad else x, r // hb)][b0:b1, r % hb]
-        return store[(n + x if grad else x, 0)][b0:b1, r]
+    def input_pieces(x, b0, b1, grad=False):
+        """(piece index, its [b0:b1] block, the slice of the whole tensor it covers) of the
+        resident pieces of the window input x (band-split or unsplit)."""
+        key = n + x if grad else x
+        if not band(x):
+            return [(0, store[(key, 0)][b0:b1], (slice(None), slice(None)))]
+        ax, p = sim.axis_of(cfg, x), p_of(x)
+        hb = ts[x]["shape"][ax] // p
+        out = []
+        for j in range(p):
+            if (key, j) in store:
+                sl = slice(j * hb, (j + 1) * hb)
+                out.append((j, store[(key, j)][b0:b1], (sl, slice(None)) if ax == 1 else (slice(None), sl)))
+        return out
 
     def attr_micro_op(it):
         """Micro-op k of an op in attribute mode or of a window op reading bands (D-ATTR).
@@ -150,13 +160,16 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
         if o["kind"] in sim.ATTR_WINDOW:
             x = o["inputs"][0]
             H, W = ts[x]["shape"][1], ts[x]["shape"][2]
-            lo, hi, hs, nb = sim.staged_rows(graph, cfg, it.op, k, P)
-            R, s, pad = sim.window_geom(o, ts)
+            rlo, hs, clo, ws, nb = sim.staged_rect(graph, cfg, it.op, k, P)
             b0 = 0 if amode(it.op) else k * B // P
             fill = -np.inf if o["kind"] == "maxpool" else 0.0
-            xs = np.full((nb, hs, W + 2 * pad, ts[x]["shape"][3]), fill)
-            for r in range(max(lo, 0), min(hi, H - 1) + 1):
-                xs[:, r - lo, pad:pad + W] = input_rows(x, b0, b0 + nb, r)
+            # the rows [rlo, rlo + hs) x columns [clo, clo + ws) of samples [b0, b0 + nb):
+            # the resident pieces placed in a padded canvas, then the rectangle cut out
+            pr, pc = max(0, -rlo), max(0, -clo)
+            canvas = np.full((nb, H + pr + max(0, rlo + hs - H), W + pc + max(0, clo + ws - W), ts[x]["shape"][3]), fill)
+            for j, blk, (sr, sc) in input_pieces(x, b0, b0 + nb):
+                canvas[:, pr:pr + H, pc:pc + W][:, sr, sc] = blk
+            xs = canvas[:, rlo + pr:rlo + pr + hs, clo + pc:clo + pc + ws].copy()
             assert (2 * n + it.op, k) in store  # the staging temporary is allocated
             store[(2 * n + it.op, k)] = xs
             o2 = dict(o, iattrs=list(o["iattrs"]))
@@ -175,8 +188,11 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
                     pgrad[tid] += g
                 elif tid in an.needs_grad:
                     store[(3 * n + it.op, k)] = g
-                    for r in range(max(lo, 0), min(hi, H - 1) + 1):
-                        input_rows(x, b0, b0 + nb, r, grad=True)[...] += g[:, r - lo, pad:pad + W]
+                    canvas = np.zeros((nb, H + pr + max(0, rlo + hs - H), W + pc + max(0, clo + ws - W), g.shape[3]))
+                    canvas[:, rlo + pr:rlo + pr + hs, clo + pc:clo + pc + ws] = g
+                    inside = canvas[:, pr:pr + H, pc:pc + W]   # the padding's gradient is dropped
+                    for j, blk, (sr, sc) in input_pieces(x, b0, b0 + nb, grad=True):
+                        blk[...] += inside[:, sr, sc]
             return
         if it.kind in ("F", "R"):
             for t in o["inputs"]:

@@ -81,16 +81,18 @@ def dim_of(cfg, t):
     return c[3] if c is not None and len(c) > 3 else 0
 
 
-# Attribute (height) split, P:L258-260 ("split along the dim of sample, model parameter, or
-# attribute (e.g., batch, channel, height, and width dimensions for images)"), DESIGN.md
-# reading D-ATTR: a 4-D NHWC activation [B, H, W, C] split along H into p bands of H/p rows,
-# piece j = rows [j H/p, (j+1) H/p) of every sample, stored [B, H/p, W, C].  An op with a
+# Attribute (height / width) split, P:L258-260 ("split along the dim of sample, model
+# parameter, or attribute (e.g., batch, channel, height, and width dimensions for images)"),
+# DESIGN.md reading D-ATTR: a 4-D NHWC activation [B, H, W, C] split along H (dim 2) into p
+# bands of H/p rows, piece j = rows [j H/p, (j+1) H/p) of every sample, stored [B, H/p, W, C]
+# — or along W (dim 3) into p bands of W/p columns, stored [B, H, W/p, C].  An op with a
 # band-split output runs in "attribute mode": micro-op k computes output band k over all
 # samples.  Band-local ops (ATTR_LOCAL) read band k of band-split inputs of the same p.
 # Window ops (conv2d, maxpool) read the input rows their output band needs — its own band
 # plus halo rows from the neighbouring bands (or an unsplit input) — through a staged copy:
-# the physical merge & split of Fig. 10, a temporary [B, Hs, W + 2 pad, C] with the
-# padding written out, so the window op runs unpadded on it; its backward scatters the staged
+# the physical merge & split of Fig. 10, a temporary [B, Hs, Ws, C] (the rows and
+# columns the output block reads, padding written out: Ws = W + 2 pad for a height band), so
+# the window op runs unpadded on it; its backward scatters the staged
 # input gradient back into the band pieces (overlapping halos add: merge = sum).  A
 # window op whose output is not band-split reads every band of its samples the same way (a
 # full merge).  Batch normalisation in band mode keeps BATCH_REDUCE's rule (its first
@@ -102,21 +104,27 @@ ATTR_WINDOW = {"conv2d", "maxpool"}
 
 
 def is_attr(graph, cfg, t):
-    return dim_of(cfg, t) == 2 and cfg[t][1] > 1 and graph["tensors"][t]["kind"] == "act"
+    return dim_of(cfg, t) in (2, 3) and cfg[t][1] > 1 and graph["tensors"][t]["kind"] == "act"
 
 
-def window_geom(op, ts):
-    """(R, stride, pad) of a conv2d / maxpool."""
+def axis_of(cfg, t):
+    """NHWC array axis of a band split: 1 (height, dim 2) or 2 (width, dim 3)."""
+    return 1 if dim_of(cfg, t) == 2 else 2
+
+
+def window_geom(op, ts, axis=1):
+    """(window extent along `axis`, stride, pad) of a conv2d (R for rows, S for columns) /
+    maxpool (square)."""
     if op["kind"] == "conv2d":
-        return ts[op["inputs"][1]]["shape"][1], op["iattrs"][0], op["iattrs"][1]
+        return ts[op["inputs"][1]]["shape"][axis], op["iattrs"][0], op["iattrs"][1]
     return op["iattrs"][0], op["iattrs"][1], op["iattrs"][2]
 
 
-def band_rows(op, ts, k, P):
-    """Input rows [lo, hi] (inclusive, may lie outside [0, H)) the output band k of P of a
-    window op reads, and the staged row count Hs = hi - lo + 1."""
-    R, s, pad = window_geom(op, ts)
-    Ho = ts[op["outputs"][0]]["shape"][1]
+def band_rows(op, ts, k, P, axis=1):
+    """Input rows (axis 1; columns for axis 2) [lo, hi] (inclusive, may lie outside the
+    tensor) the output band k of P of a window op reads, and the staged count hi - lo + 1."""
+    R, s, pad = window_geom(op, ts, axis)
+    Ho = ts[op["outputs"][0]]["shape"][axis]
     hb = Ho // P
     lo = k * hb * s - pad
     hi = ((k + 1) * hb - 1) * s - pad + R - 1
@@ -136,14 +144,15 @@ def check_attr(graph, cfg):
         tid = t["id"]
         if not is_attr(graph, cfg, tid):
             continue
-        p = cfg[tid][1]
-        if len(t["shape"]) != 4 or t["shape"][1] % p:
-            raise ValueError(f"tensor {tid}: a band split needs an NHWC activation with H % p == 0")
+        p, d = cfg[tid][1], dim_of(cfg, tid)
+        if len(t["shape"]) != 4 or t["shape"][axis_of(cfg, tid)] % p:
+            raise ValueError(f"tensor {tid}: a band split needs an NHWC activation whose H (W) p divides")
+        same = lambda u: is_attr(graph, cfg, u) and cfg[u][1] == p and dim_of(cfg, u) == d  # noqa: E731
         po = producer[tid]
         if po["kind"] in ATTR_LOCAL:
             for x in po["inputs"]:
-                if ts[x]["kind"] == "act" and (not is_attr(graph, cfg, x) or cfg[x][1] != p):
-                    raise ValueError(f"tensor {tid}: a band-local producer needs band-split inputs of the same p")
+                if ts[x]["kind"] == "act" and not same(x):
+                    raise ValueError(f"tensor {tid}: a band-local producer needs band-split inputs of the same p and dim")
         elif po["kind"] in ATTR_WINDOW:
             x = po["inputs"][0]
             if not is_attr(graph, cfg, x) and cfg[x][1] != 1:
@@ -153,8 +162,8 @@ def check_attr(graph, cfg):
         for c in consumers.get(tid, []):
             y = c["outputs"][0]
             if c["kind"] in ATTR_LOCAL:
-                if not is_attr(graph, cfg, y) or cfg[y][1] != p:
-                    raise ValueError(f"tensor {tid}: a band-local consumer needs a band-split output of the same p")
+                if not same(y):
+                    raise ValueError(f"tensor {tid}: a band-local consumer needs a band-split output of the same p and dim")
             elif c["kind"] in ATTR_WINDOW:
                 if dim_of(cfg, y) == 1 and cfg[y][1] > 1:
                     raise ValueError(f"tensor {tid}: a window consumer's output cannot be channel-split")
@@ -184,8 +193,8 @@ def check_channel(graph, cfg):
 
     for t in ts:
         tid = t["id"]
-        if dim_of(cfg, tid) not in (0, 1, 2):
-            raise ValueError(f"tensor {tid}: split dim must be 0 (samples), 1 (channels) or 2 (height)")
+        if dim_of(cfg, tid) not in (0, 1, 2, 3):
+            raise ValueError(f"tensor {tid}: split dim must be 0 (samples), 1 (channels), 2 (height) or 3 (width)")
         if not chan(tid):
             continue
         p = cfg[tid][1]
@@ -334,23 +343,29 @@ def analyze(graph):
     return Analysis(n, producer, sample, is_loss, ng, has_bwd, saved, [tbytes(t) for t in ts])
 
 
-def staged_rows(graph, cfg, o, k, P):
-    """(lo, hi, Hs, samples) of the staged input of micro-op k of window op o (D-ATTR): band
-    mode stages rows band_rows(k) of every sample, sample mode every row of B / P samples."""
+def staged_rect(graph, cfg, o, k, P):
+    """(rlo, hs, clo, ws, samples) of the staged input of micro-op k of window op o (D-ATTR):
+    input rows [rlo, rlo + hs) x columns [clo, clo + ws) (padding included).  Band mode stages
+    what output band k reads along the band's axis and everything along the other, for every
+    sample; sample mode (a full merge) everything for B / P samples."""
     ts, op = graph["tensors"], graph["ops"][o]
-    if is_attr(graph, cfg, op["outputs"][0]):
-        lo, hi, hs = band_rows(op, ts, k, P)
-        return lo, hi, hs, graph["samples"]
-    lo, hi, hs = band_rows(op, ts, 0, 1)
-    return lo, hi, hs, graph["samples"] // P
+    y = op["outputs"][0]
+    band = is_attr(graph, cfg, y)
+    span = []
+    for axis in (1, 2):
+        if band and axis == axis_of(cfg, y):
+            lo, _, n_ = band_rows(op, ts, k, P, axis)
+        else:
+            lo, _, n_ = band_rows(op, ts, 0, 1, axis)
+        span += [lo, n_]
+    return span[0], span[1], span[2], span[3], graph["samples"] if band else graph["samples"] // P
 
 
 def staged_bytes(graph, cfg, o, k, P):
     ts, op = graph["tensors"], graph["ops"][o]
     x = ts[op["inputs"][0]]
-    R, s, pad = window_geom(op, ts)
-    _, _, hs, nb = staged_rows(graph, cfg, o, k, P)
-    return nb * hs * (x["shape"][2] + 2 * pad) * x["shape"][3] * DTYPE_BYTES[x["dtype"]]
+    _, hs, _, ws, nb = staged_rect(graph, cfg, o, k, P)
+    return nb * hs * ws * x["shape"][3] * DTYPE_BYTES[x["dtype"]]
 
 
 @dataclass
@@ -482,11 +497,13 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
             return list(range(p_of(t)))
         if band(t):
             if ops[o]["kind"] in ATTR_WINDOW and t == ops[o]["inputs"][0]:
-                # the bands holding the rows the staged input of micro-op k covers
-                lo, hi, _, _ = staged_rows(graph, cfg, o, k, P)
-                H = ts[t]["shape"][1]
+                # the bands holding the rows (columns) the staged input of micro-op k covers
+                rlo, hs, clo, ws, _ = staged_rect(graph, cfg, o, k, P)
+                ax = axis_of(cfg, t)
+                lo, n_ = (rlo, hs) if ax == 1 else (clo, ws)
+                H = ts[t]["shape"][ax]
                 hb = H // p_of(t)
-                lo, hi = max(lo, 0), min(hi, H - 1)
+                lo, hi = max(lo, 0), min(lo + n_ - 1, H - 1)
                 if lo > hi:
                     raise ValueError(f"op {o}: micro-op {k} reads no input row")
                 return list(range(lo // hb, hi // hb + 1))

@@ -172,17 +172,17 @@ bool cfg_fields_ok(const Graph& g, const ts_tensor_cfg* cfg) {
   int t = cfg->tensor_id;
   if (t < 0 || t >= g.n()) return set_error("bad tensor id"), false;
   bool pow2 = cfg->p_num >= 1 && cfg->p_num <= 16 && (cfg->p_num & (cfg->p_num - 1)) == 0;
-  if (cfg->opt < 0 || cfg->opt > 2 || cfg->dim < 0 || cfg->dim > 2 || cfg->prefetch_lead < 1 ||
+  if (cfg->opt < 0 || cfg->opt > 2 || cfg->dim < 0 || cfg->dim > 3 || cfg->prefetch_lead < 1 ||
       cfg->release_lag < 0 || (cfg->release_lag > 0 && cfg->opt != TS_SWAP))
-    return set_error("bad opt/dim/prefetch_lead/release_lag (dim 0 = samples, 1 = channels, 2 = height; a lag needs swap)"),
+    return set_error("bad opt/dim/prefetch_lead/release_lag (dim 0 = samples, 1 = channels, 2 = height, 3 = width; a lag needs swap)"),
            false;
   const Tensor& x = g.t[t];
   if (!pow2) return set_error("p_num must be a power of 2 <= 16"), false;
   if (cfg->dim == 0 && g.samples % cfg->p_num) return set_error("p_num must divide the samples"), false;
   if (cfg->dim == 1 && (x.ndim != 2 || x.shape[1] % cfg->p_num))
     return set_error("a channel split needs a 2-D tensor whose columns p_num divides"), false;
-  if (cfg->dim == 2 && (x.ndim != 4 || x.shape[1] % cfg->p_num))
-    return set_error("a band split needs a 4-D NHWC tensor whose height p_num divides"), false;
+  if (cfg->dim >= 2 && (x.ndim != 4 || x.shape[cfg->dim - 1] % cfg->p_num))
+    return set_error("a band split needs a 4-D NHWC tensor whose height (dim 2) / width (dim 3) p_num divides"), false;
   if ((x.kind != TS_ACT || x.is_loss) && (cfg->opt != TS_RESIDE || cfg->p_num != 1))
     return set_error("only activations can be split, swapped or recomputed"), false;
   return true;

@@ -100,22 +100,25 @@ bool is_chan(const Graph& g, const std::vector<Cfg>& cfg, int key);
 bool channel_mode(const Graph& g, const std::vector<Cfg>& cfg, int op);
 bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why);
 
-// D-ATTR attribute (height) splits (expand.cpp; oracle/sim.py check_attr / staged_rows)
+// D-ATTR attribute (height / width) splits (expand.cpp; oracle/sim.py check_attr / staged_rect)
 bool is_attr(const Graph& g, const std::vector<Cfg>& cfg, int key);
+inline int attr_axis(const std::vector<Cfg>& cfg, int t) { return cfg[t].dim == 2 ? 1 : 2; }  // NHWC axis
 bool attr_mode(const Graph& g, const std::vector<Cfg>& cfg, int op);   // an output is band-split
 bool attr_window(int kind);                                              // conv2d / maxpool
 bool attr_staged(const Graph& g, const std::vector<Cfg>& cfg, int op);  // window op reading / writing bands
 bool attr_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why);
 struct Window {
-  int R, stride, pad;
+  int R, stride, pad;  // window extent along the axis (conv: R rows / S columns), stride, pad
 };
-Window window_geom(const Graph& g, int op);
+Window window_geom(const Graph& g, int op, int axis = 1);
 struct Staged {
-  int64_t lo, hi, hs, nb;  // input rows [lo, hi] (padding rows included), hs rows, nb samples
+  int64_t rlo, hs, clo, ws, nb;  // input rows [rlo, rlo + hs) x columns [clo, clo + ws) (padding
+                                 // included) of nb samples
 };
-// staged input of micro-op k (of P) of window op `op`: band mode stages rows band k needs of
-// every sample, sample mode (a full merge) every row of samples block k
-Staged staged_rows(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P);
+// staged input of micro-op k (of P) of window op `op`: band mode stages what output band k
+// reads along the band's axis (everything along the other) of every sample, sample mode (a
+// full merge) everything of samples block k
+Staged staged_rect(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P);
 uint64_t staged_bytes(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P);
 
 struct Event {

@@ -46,7 +46,8 @@ static bool chan_ew(int kind) { return kind == TS_OP_RELU || kind == TS_OP_GELU 
 
 bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
   for (int t = 0; t < g.n(); ++t) {
-    if (cfg[t].dim < 0 || cfg[t].dim > 2) return (why = "split dim must be 0 (samples), 1 (channels) or 2 (height)"), false;
+    if (cfg[t].dim < 0 || cfg[t].dim > 3)
+      return (why = "split dim must be 0 (samples), 1 (channels), 2 (height) or 3 (width)"), false;
     if (!is_chan(g, cfg, t)) continue;
     const Tensor& x = g.t[t];
     const int p = cfg[t].p;
@@ -79,12 +80,13 @@ bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
   return true;
 }
 
-// Attribute (height) split, reading D-ATTR (Fig. 10; oracle/sim.py
-// check_attr): a 4-D NHWC activation split along H into p bands [B, H/p, W, C].
+// Attribute split, reading D-ATTR (Fig. 10; oracle/sim.py check_attr): a
+// 4-D NHWC activation split along H (dim 2) into p bands [B, H/p, W, C] or along W (dim 3)
+// into [B, H, W/p, C].
 bool is_attr(const Graph& g, const std::vector<Cfg>& cfg, int key) {
   int t = key >= g.n() ? key - g.n() : key;
   const Tensor& x = g.t[t];
-  return x.sample && x.kind == TS_ACT && cfg[t].dim == 2 && cfg[t].p > 1;
+  return x.sample && x.kind == TS_ACT && (cfg[t].dim == 2 || cfg[t].dim == 3) && cfg[t].p > 1;
 }
 bool attr_mode(const Graph& g, const std::vector<Cfg>& cfg, int op) {
   for (int x : g.ops[op].out)
@@ -98,45 +100,48 @@ bool attr_staged(const Graph& g, const std::vector<Cfg>& cfg, int op) {
   return attr_window(o.kind) && (is_attr(g, cfg, o.in[0]) || attr_mode(g, cfg, op));
 }
 
-Window window_geom(const Graph& g, int op) {
+Window window_geom(const Graph& g, int op, int axis) {
   const Op& o = g.ops[op];
-  if (o.kind == TS_OP_CONV2D) return {int(g.t[o.in[1]].shape[1]), int(o.ia[0]), int(o.ia[1])};
+  if (o.kind == TS_OP_CONV2D) return {int(g.t[o.in[1]].shape[axis]), int(o.ia[0]), int(o.ia[1])};
   return {int(o.ia[0]), int(o.ia[1]), int(o.ia[2])};
 }
 
-Staged staged_rows(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P) {
+Staged staged_rect(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P) {
   const Op& o = g.ops[op];
-  const Window w = window_geom(g, op);
-  const bool band = is_attr(g, cfg, o.out[0]);
-  const int64_t ho = g.t[o.out[0]].shape[1];
-  const int64_t hb = band ? ho / P : ho;
-  const int kk = band ? k : 0;
-  Staged s;
-  s.lo = kk * hb * w.stride - w.pad;
-  s.hi = ((kk + 1) * hb - 1) * w.stride - w.pad + w.R - 1;
-  s.hs = s.hi - s.lo + 1;
-  s.nb = band ? g.samples : g.samples / P;
-  return s;
+  const int y = o.out[0];
+  const bool band = is_attr(g, cfg, y);
+  int64_t lo[3] = {0, 0, 0}, cnt[3] = {0, 0, 0};
+  for (int axis = 1; axis <= 2; ++axis) {
+    const Window w = window_geom(g, op, axis);
+    const bool here = band && attr_axis(cfg, y) == axis;  // the output's band axis
+    const int64_t ho = g.t[y].shape[axis];
+    const int64_t hb = here ? ho / P : ho;
+    const int64_t kk = here ? k : 0;
+    lo[axis] = kk * hb * w.stride - w.pad;
+    cnt[axis] = ((kk + 1) * hb - 1) * w.stride - w.pad + w.R - 1 - lo[axis] + 1;
+  }
+  return {lo[1], cnt[1], lo[2], cnt[2], band ? g.samples : g.samples / P};
 }
 
 uint64_t staged_bytes(const Graph& g, const std::vector<Cfg>& cfg, int op, int k, int P) {
   const Tensor& x = g.t[g.ops[op].in[0]];
-  const Window w = window_geom(g, op);
-  const Staged s = staged_rows(g, cfg, op, k, P);
-  return uint64_t(s.nb * s.hs * (x.shape[2] + 2 * w.pad) * x.shape[3]) * uint64_t(dtype_bytes(x.dtype));
+  const Staged s = staged_rect(g, cfg, op, k, P);
+  return uint64_t(s.nb * s.hs * s.ws * x.shape[3]) * uint64_t(dtype_bytes(x.dtype));
 }
 
 bool attr_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
   for (int t = 0; t < g.n(); ++t) {
     if (!is_attr(g, cfg, t)) continue;
     const Tensor& x = g.t[t];
-    const int p = cfg[t].p;
-    if (x.ndim != 4 || x.shape[1] % p) return (why = "a band split needs an NHWC activation with H % p == 0"), false;
+    const int p = cfg[t].p, d = cfg[t].dim;
+    if (x.ndim != 4 || x.shape[attr_axis(cfg, t)] % p)
+      return (why = "a band split needs an NHWC activation whose H (W) p divides"), false;
+    auto same = [&](int u) { return is_attr(g, cfg, u) && cfg[u].p == p && cfg[u].dim == d; };
     const Op& po = g.ops[x.producer];
     if (attr_local(po.kind)) {
       for (int u : po.in)
-        if (g.t[u].kind == TS_ACT && (!is_attr(g, cfg, u) || cfg[u].p != p))
-          return (why = "a band-local producer needs band-split inputs of the same p"), false;
+        if (g.t[u].kind == TS_ACT && !same(u))
+          return (why = "a band-local producer needs band-split inputs of the same p and dim"), false;
     } else if (attr_window(po.kind)) {
       const int u = po.in[0];
       if (!is_attr(g, cfg, u) && cfg[u].p != 1)
@@ -148,8 +153,7 @@ bool attr_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
       const Op& co = g.ops[c];
       const int y = co.out[0];
       if (attr_local(co.kind)) {
-        if (!is_attr(g, cfg, y) || cfg[y].p != p)
-          return (why = "a band-local consumer needs a band-split output of the same p"), false;
+        if (!same(y)) return (why = "a band-local consumer needs a band-split output of the same p and dim"), false;
       } else if (attr_window(co.kind)) {
         if (is_chan(g, cfg, y)) return (why = "a window op reading bands cannot write channel blocks"), false;
       } else {
@@ -161,10 +165,12 @@ bool attr_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
   for (auto& o : g.ops) {
     if (!attr_window(o.kind) || !attr_mode(g, cfg, o.id)) continue;
     const int P = cfg[o.out[0]].p;
-    const int64_t H = g.t[o.in[0]].shape[1];
+    const int ax = attr_axis(cfg, o.out[0]);
+    const int64_t H = g.t[o.in[0]].shape[ax];
     for (int k = 0; k < P; ++k) {
-      const Staged s = staged_rows(g, cfg, o.id, k, P);
-      if (std::max<int64_t>(s.lo, 0) > std::min<int64_t>(s.hi, H - 1))
+      const Staged s = staged_rect(g, cfg, o.id, k, P);
+      const int64_t lo = ax == 1 ? s.rlo : s.clo, cnt = ax == 1 ? s.hs : s.ws;
+      if (std::max<int64_t>(lo, 0) > std::min<int64_t>(lo + cnt - 1, H - 1))
         return (why = "a band of a window op reads no input row"), false;
     }
   }
@@ -215,9 +221,11 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
     if (is_attr(g, cfg, t)) {
       const Op& o = g.ops[op];
       if (attr_window(o.kind) && o.in[0] == t) {
-        const Staged s = staged_rows(g, cfg, op, k, P);
-        const int64_t H = g.t[t].shape[1], hb = H / piece_count(g, cfg, t);
-        const int64_t lo = std::max<int64_t>(s.lo, 0), hi = std::min<int64_t>(s.hi, H - 1);
+        const Staged s = staged_rect(g, cfg, op, k, P);
+        const int ax = attr_axis(cfg, t);
+        const int64_t H = g.t[t].shape[ax], hb = H / piece_count(g, cfg, t);
+        const int64_t lo0 = ax == 1 ? s.rlo : s.clo, cnt = ax == 1 ? s.hs : s.ws;
+        const int64_t lo = std::max<int64_t>(lo0, 0), hi = std::min<int64_t>(lo0 + cnt - 1, H - 1);
         std::vector<int> js;
         for (int64_t j = lo / hb; j <= hi / hb; ++j) js.push_back(int(j));
         return js;

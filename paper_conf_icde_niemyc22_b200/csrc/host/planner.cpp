@@ -778,12 +778,24 @@ ts_status plan_greedy(const Graph& g, uint64_t budget, const Profile& pr, PlanSt
     for (int t : live) {
       const Tensor& x = g.t[t];
       if (x.kind != TS_ACT || x.is_loss || own.count(t) || ps.cfg[t].opt != TS_RECOMPUTE) continue;
-      for (int p = ps.cfg[t].p * 2; p <= 16 && !no_split; p *= 2) {
+      const bool banded = is_attr(g, ps.cfg, t);
+      for (int p = ps.cfg[t].p * 2; p <= 16 && !no_split && !banded; p *= 2) {
         if (g.samples % p) break;
         Cand2 c;
         c.birth = birth[t];
         c.tensor = t;
         c.ch = {{t, TS_RECOMPUTE, p, ps.cfg[t].lead}};
+        step2.push_back(c);
+      }
+      // D-ATTR: with the sample dim exhausted, finer height bands for the tensor's group
+      if (no_split || x.ndim != 4 || (!banded && g.samples % (2 * ps.cfg[t].p) == 0)) continue;
+      const std::vector<int> grp = band_group(t);
+      for (int p = banded ? ps.cfg[t].p * 2 : 2; p <= 16; p *= 2) {
+        if (x.shape[1] % p) break;
+        Cand2 c;
+        c.birth = birth[t];
+        c.tensor = t;
+        for (int u : grp) c.ch.push_back({u, u == t ? TS_RECOMPUTE : ps.cfg[u].opt, p, ps.cfg[u].lead, 2});
         step2.push_back(c);
       }
     }

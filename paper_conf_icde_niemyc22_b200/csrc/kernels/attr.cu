@@ -1,13 +1,13 @@
-// Staging copies of attribute (height) band splits — DESIGN.md reading D-ATTR, the physical
-// merge & split of P:L264 (Fig. 10) for window ops (conv2d, maxpool) whose input or output is
-// split along H.
+// Staging copies of attribute (height / width) band splits — DESIGN.md reading D-ATTR, the
+// physical merge & split of P:L264 (Fig. 10) for window ops (conv2d, maxpool) whose input or
+// output is split along H or W.
 //
-//   gather:      S[b, r, w, c] = X[b0 + b, lo + r, w - pad, c]   (rows / columns outside X: fill)
-//   scatter-add: dX[b0 + b, h, w, c] += dS[b, h - lo, w + pad, c] for the rows h in [lo, lo+hs) ∩ [0, H)
+//   gather:      S[b, r, c', ch] = X[b0 + b, rlo + r, clo + c', ch]   (outside X: fill)
+//   scatter-add: dX[b0 + b, h, w, ch] += dS[b, h - rlo, w - clo, ch] for (h, w) in the rectangle ∩ X
 //
-// X is p pieces of hb rows each, piece j = rows [j hb, (j+1) hb) of every sample, stored
-// [B, hb, W, C] (an unsplit tensor is one piece of H rows).  Both are HBM-bound copies: one
-// 16-byte vector per thread when a pixel row is whole vectors (every activation but the
+// X is p pieces of hb rows (piece j = rows [j hb, (j+1) hb) of every sample, stored
+// [B, hb, W, C]) or of hb columns ([B, H, hb, C]); an unsplit tensor is one piece of H rows.
+// Both are HBM-bound copies: one 16-byte vector per thread when a pixel row is whole vectors (every activation but the
 // 3-channel image), one element otherwise; grid-stride loops over 8 CTAs per SM.
 #include "common.cuh"
 #include "kernels.h"
@@ -23,21 +23,30 @@ int grid_for(int64_t n) {
   return int(b < 148 * 8 ? b : 148 * 8);
 }
 
+// element offset of (b, h, w) inside its piece, and the piece
+__device__ __forceinline__ int64_t band_off(const BandPieces& x, int H, int W, int b, int h, int w, int& j) {
+  if (x.axis == 1) {
+    j = h / x.hb;
+    return (int64_t(b) * x.hb + (h - j * x.hb)) * W + w;
+  }
+  j = w / x.hb;
+  return (int64_t(b) * H + h) * x.hb + (w - j * x.hb);
+}
+
 template <class T, int V>
-__global__ void band_gather_k(BandPieces x, int H, int W, int C, int b0, int nb, int lo, int hs, int pad, T fill,
-                              T* __restrict__ out) {
-  const int CV = C / V, Wp = W + 2 * pad;
-  const int64_t total = int64_t(nb) * hs * Wp * CV;
+__global__ void band_gather_k(BandPieces x, int H, int W, int C, Rect r, T fill, T* __restrict__ out) {
+  const int CV = C / V;
+  const int64_t total = int64_t(r.nb) * r.hs * r.ws * CV;
   for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < total; i += int64_t(gridDim.x) * blockDim.x) {
     const int cv = int(i % CV);
     const int64_t pix = i / CV;
-    const int w = int(pix % Wp), r = int((pix / Wp) % hs), b = int(pix / (int64_t(Wp) * hs));
-    const int h = lo + r, ww = w - pad;
+    const int w = int(pix % r.ws), rr = int((pix / r.ws) % r.hs), b = int(pix / (int64_t(r.ws) * r.hs));
+    const int h = r.rlo + rr, ww = r.clo + w;
     T* o = out + pix * C + int64_t(cv) * V;
     if (h >= 0 && h < H && ww >= 0 && ww < W) {
-      const int j = h / x.hb;
-      const T* src = static_cast<const T*>(x.ptr[j]) + ((int64_t(b0 + b) * x.hb + (h - j * x.hb)) * W + ww) * C +
-                     int64_t(cv) * V;
+      int j;
+      const int64_t off = band_off(x, H, W, r.b0 + b, h, ww, j);
+      const T* src = static_cast<const T*>(x.ptr[j]) + off * C + int64_t(cv) * V;
       if constexpr (V * sizeof(T) == 16) {
         *reinterpret_cast<uint4*>(o) = *reinterpret_cast<const uint4*>(src);
       } else {
@@ -51,20 +60,20 @@ __global__ void band_gather_k(BandPieces x, int H, int W, int C, int b0, int nb,
   }
 }
 
+// over the rectangle's pixels inside X: rows [h0, h0 + nh) x columns [w0, w0 + nw)
 template <class T, int V>
-__global__ void band_scatter_add_k(const T* __restrict__ src, BandPieces dx, int H, int W, int C, int b0, int nb,
-                                   int lo, int hs, int pad, int rlo, int nr) {
-  const int CV = C / V, Wp = W + 2 * pad;
-  const int64_t total = int64_t(nb) * nr * W * CV;
+__global__ void band_scatter_add_k(const T* __restrict__ src, BandPieces dx, int H, int W, int C, Rect r, int h0,
+                                   int nh, int w0, int nw) {
+  const int CV = C / V;
+  const int64_t total = int64_t(r.nb) * nh * nw * CV;
   for (int64_t i = blockIdx.x * int64_t(blockDim.x) + threadIdx.x; i < total; i += int64_t(gridDim.x) * blockDim.x) {
     const int cv = int(i % CV);
     const int64_t pix = i / CV;
-    const int w = int(pix % W), rr = int((pix / W) % nr), b = int(pix / (int64_t(W) * nr));
-    const int h = rlo + rr;
-    const int j = h / dx.hb;
-    T* d = static_cast<T*>(const_cast<void*>(dx.ptr[j])) + ((int64_t(b0 + b) * dx.hb + (h - j * dx.hb)) * W + w) * C +
-           int64_t(cv) * V;
-    const T* s = src + ((int64_t(b) * hs + (h - lo)) * Wp + w + pad) * C + int64_t(cv) * V;
+    const int w = w0 + int(pix % nw), h = h0 + int((pix / nw) % nh), b = int(pix / (int64_t(nw) * nh));
+    int j;
+    const int64_t off = band_off(dx, H, W, r.b0 + b, h, w, j);
+    T* d = static_cast<T*>(const_cast<void*>(dx.ptr[j])) + off * C + int64_t(cv) * V;
+    const T* s = src + ((int64_t(b) * r.hs + (h - r.rlo)) * r.ws + (w - r.clo)) * C + int64_t(cv) * V;
     if constexpr (V * sizeof(T) == 16) {
       uint4 dv = *reinterpret_cast<const uint4*>(d);
       const uint4 sv = *reinterpret_cast<const uint4*>(s);
@@ -81,48 +90,44 @@ __global__ void band_scatter_add_k(const T* __restrict__ src, BandPieces dx, int
 }
 
 template <class T>
-void gather_launch(const BandPieces& x, int H, int W, int C, int b0, int nb, int lo, int hs, int pad, T fill, void* out,
-                   cudaStream_t st) {
+void gather_launch(const BandPieces& x, int H, int W, int C, const Rect& r, T fill, void* out, cudaStream_t st) {
   constexpr int V = 16 / sizeof(T);
-  const int64_t pix = int64_t(nb) * hs * (W + 2 * pad);
+  const int64_t pix = int64_t(r.nb) * r.hs * r.ws;
   if (C % V == 0)
-    band_gather_k<T, V><<<grid_for(pix * (C / V)), kT, 0, st>>>(x, H, W, C, b0, nb, lo, hs, pad, fill,
-                                                                  static_cast<T*>(out));
+    band_gather_k<T, V><<<grid_for(pix * (C / V)), kT, 0, st>>>(x, H, W, C, r, fill, static_cast<T*>(out));
   else
-    band_gather_k<T, 1><<<grid_for(pix * C), kT, 0, st>>>(x, H, W, C, b0, nb, lo, hs, pad, fill, static_cast<T*>(out));
+    band_gather_k<T, 1><<<grid_for(pix * C), kT, 0, st>>>(x, H, W, C, r, fill, static_cast<T*>(out));
 }
 
 template <class T>
-void scatter_launch(const void* src, const BandPieces& dx, int H, int W, int C, int b0, int nb, int lo, int hs, int pad,
-                    cudaStream_t st) {
+void scatter_launch(const void* src, const BandPieces& dx, int H, int W, int C, const Rect& r, cudaStream_t st) {
   constexpr int V = 16 / sizeof(T);
-  const int rlo = lo > 0 ? lo : 0, rhi = lo + hs - 1 < H - 1 ? lo + hs - 1 : H - 1;
-  const int nr = rhi - rlo + 1;
-  if (nr <= 0) return;
-  const int64_t pix = int64_t(nb) * nr * W;
+  const int h0 = r.rlo > 0 ? r.rlo : 0, h1 = r.rlo + r.hs < H ? r.rlo + r.hs : H;
+  const int w0 = r.clo > 0 ? r.clo : 0, w1 = r.clo + r.ws < W ? r.clo + r.ws : W;
+  if (h1 <= h0 || w1 <= w0) return;
+  const int64_t pix = int64_t(r.nb) * (h1 - h0) * (w1 - w0);
   if (C % V == 0)
-    band_scatter_add_k<T, V><<<grid_for(pix * (C / V)), kT, 0, st>>>(static_cast<const T*>(src), dx, H, W, C, b0, nb,
-                                                                       lo, hs, pad, rlo, nr);
+    band_scatter_add_k<T, V><<<grid_for(pix * (C / V)), kT, 0, st>>>(static_cast<const T*>(src), dx, H, W, C, r, h0,
+                                                                       h1 - h0, w0, w1 - w0);
   else
-    band_scatter_add_k<T, 1><<<grid_for(pix * C), kT, 0, st>>>(static_cast<const T*>(src), dx, H, W, C, b0, nb, lo, hs,
-                                                                 pad, rlo, nr);
+    band_scatter_add_k<T, 1><<<grid_for(pix * C), kT, 0, st>>>(static_cast<const T*>(src), dx, H, W, C, r, h0, h1 - h0,
+                                                                 w0, w1 - w0);
 }
 
 }  // namespace
 
-void band_gather(int dt, const BandPieces& x, int H, int W, int C, int b0, int nb, int lo, int hs, int pad,
-                 int neg_inf_fill, void* out, cudaStream_t st) {
+void band_gather(int dt, const BandPieces& x, int H, int W, int C, const Rect& r, int neg_inf_fill, void* out,
+                 cudaStream_t st) {
   if (dt == BF16)
-    gather_launch<bf16>(x, H, W, C, b0, nb, lo, hs, pad, neg_inf_fill ? __float2bfloat16_rn(-INFINITY) : bf16(0.f), out,
-                        st);
+    gather_launch<bf16>(x, H, W, C, r, neg_inf_fill ? __float2bfloat16_rn(-INFINITY) : bf16(0.f), out, st);
   else
-    gather_launch<float>(x, H, W, C, b0, nb, lo, hs, pad, neg_inf_fill ? -INFINITY : 0.f, out, st);
+    gather_launch<float>(x, H, W, C, r, neg_inf_fill ? -INFINITY : 0.f, out, st);
 }
 
-void band_scatter_add(int dt, const void* src, const BandPieces& dx, int H, int W, int C, int b0, int nb, int lo, int hs,
-                      int pad, cudaStream_t st) {
-  if (dt == BF16) scatter_launch<bf16>(src, dx, H, W, C, b0, nb, lo, hs, pad, st);
-  else scatter_launch<float>(src, dx, H, W, C, b0, nb, lo, hs, pad, st);
+void band_scatter_add(int dt, const void* src, const BandPieces& dx, int H, int W, int C, const Rect& r,
+                      cudaStream_t st) {
+  if (dt == BF16) scatter_launch<bf16>(src, dx, H, W, C, r, st);
+  else scatter_launch<float>(src, dx, H, W, C, r, st);
 }
 
 }  // namespace tsk

@@ -168,18 +168,23 @@ void maxpool_fwd(int dt, const void* x, void* y, int n, int H, int W, int C, int
 // gradient to the first maximum of each window in row-major order
 void maxpool_bwd(int dt, const void* dy, const void* x, void* dx, int acc, int n, int H, int W, int C, int P, int Q,
                  int k, int stride, int pad, cudaStream_t st);
-// D-ATTR staging (attr.cu): a band-split NHWC tensor is np pieces of hb rows (piece j = rows
-// [j hb, (j+1) hb) of every sample, [B, hb, W, C]); an unsplit one is one piece of H rows.
+// D-ATTR staging (attr.cu): a band-split NHWC tensor [B, H, W, C] is pieces of hb rows
+// (axis 1: piece j = rows [j hb, (j+1) hb) of every sample, [B, hb, W, C]) or of hb columns
+// (axis 2: [B, H, hb, C]); an unsplit one is one piece with axis 1, hb = H.
 struct BandPieces {
   const void* ptr[16] = {};
-  int hb = 0;
+  int hb = 0, axis = 1;
 };
-// out[b, r, w, c] = X[b0 + b, lo + r, w - pad, c], fill (0 or -inf) outside X; out [nb, hs, W + 2 pad, C]
-void band_gather(int dt, const BandPieces& x, int H, int W, int C, int b0, int nb, int lo, int hs, int pad,
-                 int neg_inf_fill, void* out, cudaStream_t st);
-// dX[b0 + b, h, w, c] += src[b, h - lo, w + pad, c] for the rows of [lo, lo + hs) inside [0, H)
-void band_scatter_add(int dt, const void* src, const BandPieces& dx, int H, int W, int C, int b0, int nb, int lo,
-                      int hs, int pad, cudaStream_t st);
+// The staged rectangle: rows [rlo, rlo + hs) x columns [clo, clo + ws) of samples [b0, b0 + nb).
+struct Rect {
+  int b0, nb, rlo, hs, clo, ws;
+};
+// out[b, r, c', ch] = X[b0 + b, rlo + r, clo + c', ch], fill (0 or -inf) outside X; out [nb, hs, ws, C]
+void band_gather(int dt, const BandPieces& x, int H, int W, int C, const Rect& r, int neg_inf_fill, void* out,
+                 cudaStream_t st);
+// dX[b0 + b, h, w, ch] += src[b, h - rlo, w - clo, ch] for the (h, w) of the rectangle inside X
+void band_scatter_add(int dt, const void* src, const BandPieces& dx, int H, int W, int C, const Rect& r,
+                      cudaStream_t st);
 void avgpool_fwd(int dt, const void* x, void* y, int n, int HW, int C, cudaStream_t st);
 void avgpool_bwd(int dt, const void* dy, void* dx, int acc, int n, int HW, int C, cudaStream_t st);
 

@@ -688,9 +688,28 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       gslot(0, a.dq, a.acc_q);
       gslot(1, a.dk, a.acc_k);
       gslot(2, a.dv, a.acc_v);
-      nk = 2;
       a.step_ptr = stepp;
-      return [a](cudaStream_t st) { tsk::attention_bwd(a, st); };
+      // the row terms D = rowsum(dO * O) of a micro-op live in the workspace: a micro-op with
+      // more samples than it holds runs its backward in sample chunks (large unsplit batches)
+      const int64_t per = int64_t(a.heads) * a.seq * 4;
+      const int chunk = int(std::max<int64_t>(1, std::min<int64_t>(a.nb, (int64_t(g.ws_bytes) - 4096) / per)));
+      std::vector<tsk::AttnArgs> parts;
+      const int es = dt == tsk::BF16 ? 2 : 4;
+      for (int c0 = 0; c0 < a.nb; c0 += chunk) {
+        tsk::AttnArgs b = a;
+        b.nb = std::min(chunk, a.nb - c0);
+        b.b0 = a.b0 + c0;
+        const int64_t tok = int64_t(c0) * a.seq * a.ld * es;  // byte offset of the chunk's first row
+        auto sh = [&](const void* ptr) { return ptr ? static_cast<const char*>(ptr) + tok : nullptr; };
+        auto shm = [&](void* ptr) { return ptr ? static_cast<char*>(ptr) + tok : nullptr; };
+        b.q = sh(a.q); b.k = sh(a.k); b.v = sh(a.v); b.dc = sh(a.dc);
+        b.c = shm(a.c); b.dq = shm(a.dq); b.dk = shm(a.dk); b.dv = shm(a.dv);
+        b.lse = a.lse + int64_t(c0) * a.heads * a.seq;
+        b.mask = a.mask + int64_t(c0) * a.heads * a.seq * (a.seq / 32);
+        parts.push_back(b);
+      }
+      nk = 2 * int(parts.size());
+      return [parts](cudaStream_t st) { for (auto& b : parts) tsk::attention_bwd(b, st); };
     }
     case TS_OP_XENT: {
       const int C = int(g.t[o.in[0]].shape[1]);
@@ -778,22 +797,26 @@ std::function<void(cudaStream_t)> lower_staged(ts_session_t* s, const Item& it, 
   const int xi = o.in[0], yi = o.out[0];
   const Tensor& x = g.t[xi];
   const Tensor& y = g.t[yi];
-  const Window wg = window_geom(g, it.op);
-  const Staged sr = staged_rows(g, s->cfg, it.op, it.k, m.P);
+  const Window wg = window_geom(g, it.op, 1);
+  const Staged sr = staged_rect(g, s->cfg, it.op, it.k, m.P);
   const bool band_out = attr_mode(g, s->cfg, it.op);
+  const int ax_out = band_out ? attr_axis(s->cfg, yi) : 0;
   const int H = int(x.shape[1]), W = int(x.shape[2]), C = int(x.shape[3]);
-  const int Wp = W + 2 * wg.pad;
   const int b0 = band_out ? 0 : int(int64_t(it.k) * g.samples / m.P);
-  const int nb = int(sr.nb), lo = int(sr.lo), hs = int(sr.hs);
-  const int Pr = int(band_out ? y.shape[1] / m.P : y.shape[1]), Q = int(y.shape[2]);
+  const int nb = int(sr.nb), hs = int(sr.hs), Wp = int(sr.ws);
+  const tsk::Rect rect{b0, nb, int(sr.rlo), hs, int(sr.clo), Wp};
+  // the output block: a band of rows or columns (attribute mode) or every pixel (full merge)
+  const int Pr = int(ax_out == 1 ? y.shape[1] / m.P : y.shape[1]), Q = int(ax_out == 2 ? y.shape[2] / m.P : y.shape[2]);
   const bool bwd = it.kind == IT_B;
   auto at = [&](PieceKey pc) -> char* {
     auto f = where.find(pc);
     return f == where.end() ? nullptr : s->slab + f->second;
   };
   auto pieces_of = [&](int key, tsk::BandPieces& bp) {
-    const int px = is_attr(g, s->cfg, xi) ? piece_count(g, s->cfg, xi) : 1;
-    bp.hb = H / px;
+    const bool bx = is_attr(g, s->cfg, xi);
+    const int px = bx ? piece_count(g, s->cfg, xi) : 1;
+    bp.axis = bx ? attr_axis(s->cfg, xi) : 1;
+    bp.hb = int(x.shape[bp.axis] / px);
     for (int j = 0; j < px; ++j) bp.ptr[j] = at(pk(key, j));
   };
   tsk::BandPieces src;
@@ -815,13 +838,13 @@ std::function<void(cudaStream_t)> lower_staged(ts_session_t* s, const Item& it, 
       const void* bias = o.in.size() > 2 ? param_w(s, o.in[2]) : nullptr;
       nk = 2;
       return [=](cudaStream_t st) {
-        tsk::band_gather(dt, src, H, W, C, b0, nb, lo, hs, wg.pad, fill, tmp, st);
+        tsk::band_gather(dt, src, H, W, C, rect, fill, tmp, st);
         tsk::conv_fprop(a, yv, bias, st);
       };
     }
     nk = 2;
     return [=](cudaStream_t st) {
-      tsk::band_gather(dt, src, H, W, C, b0, nb, lo, hs, wg.pad, fill, tmp, st);
+      tsk::band_gather(dt, src, H, W, C, rect, fill, tmp, st);
       tsk::maxpool_fwd(dt, tmp, yv, nb, hs, Wp, C, Pr, Q, wg.R, wg.stride, 0, st);
     };
   }
@@ -859,23 +882,23 @@ std::function<void(cudaStream_t)> lower_staged(ts_session_t* s, const Item& it, 
     const uint64_t wsb = g.ws_bytes;
     nk = 2 + (db ? 2 : 0) + (gx ? 2 : 0);
     return [=](cudaStream_t st) {
-      tsk::band_gather(dt, src, H, W, C, b0, nb, lo, hs, wg.pad, 0, tmp, st);
+      tsk::band_gather(dt, src, H, W, C, rect, 0, tmp, st);
       tsk::conv_wgrad(a, dw, dwacc, st);
       if (db) tsk::column_sum(dt, dy, pix, a.K, ws, wsb, db, dbacc, nullptr, 0, st);
       if (gx) {
         tsk::conv_dgrad(a, tmp2, 0, st);
         for (auto& z : zero) cudaMemsetAsync(z.first, 0, z.second, st);
-        tsk::band_scatter_add(dt, tmp2, dst, H, W, C, b0, nb, lo, hs, wg.pad, st);
+        tsk::band_scatter_add(dt, tmp2, dst, H, W, C, rect, st);
       }
     };
   }
   if (!gx) return (why = "max pooling of an input without gradient"), nullptr;
   nk = 3;
   return [=](cudaStream_t st) {
-    tsk::band_gather(dt, src, H, W, C, b0, nb, lo, hs, wg.pad, 1, tmp, st);
+    tsk::band_gather(dt, src, H, W, C, rect, 1, tmp, st);
     tsk::maxpool_bwd(dt, dy, tmp, tmp2, 0, nb, hs, Wp, C, Pr, Q, wg.R, wg.stride, 0, st);
     for (auto& z : zero) cudaMemsetAsync(z.first, 0, z.second, st);
-    tsk::band_scatter_add(dt, tmp2, dst, H, W, C, b0, nb, lo, hs, wg.pad, st);
+    tsk::band_scatter_add(dt, tmp2, dst, H, W, C, rect, st);
   };
 }
 
@@ -1075,7 +1098,7 @@ ts_status build_program(ts_session_t* s) {
       for (PieceKey pc : it.writes)
         if (pk_key(pc) < n) m.writes.insert(pk_key(pc));
       if (o.kind == TS_OP_ATTENTION) {
-        const uint64_t need = uint64_t(m.s1 - m.s0) * uint64_t(o.ia[0]) * uint64_t(o.ia[1]) * 4;
+        const uint64_t need = uint64_t(o.ia[0]) * uint64_t(o.ia[1]) * 4;  // one sample's row terms (chunked)
         if (need + 4096 > g.ws_bytes) return set_error("attention: workspace too small for the row terms"), TS_ERR_GRAPH;
       }
       if (batch_reduce(o.kind) && it.k == 0 && it.kind != IT_R) {  // replays reuse the step's statistics

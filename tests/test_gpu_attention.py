@@ -214,3 +214,15 @@ def test_tc_forward_partial_outputs_for_replays():
     assert tsplit.attention(1, geom, 0.125, 0.1, Q, K, V, mask=M2) == 2
     torch.cuda.synchronize()
     assert torch.equal(C, C2) and torch.equal(L, L2) and torch.equal(M, M2)
+
+
+def test_attention_backward_in_workspace_chunks():
+    """A fused-attention micro-op whose row terms D = rowsum(dO * O) exceed the workspace
+    (h1024 a16 s512: 255 samples fit; an unsplit batch of 288) runs its backward in sample
+    chunks; the step equals the plan whose micro-ops hold 144 samples (no chunking)."""
+    g = graphs.bert(layers=1, hidden=1024, heads=16, seq=512, batch=288, vocab=512, fused_attention=True)
+    l0, g0, S0, _ = _run(g)
+    cfg = {t: (0, 2, 1) for t in brute.act_tensors(g)}
+    l1, g1, S1, _ = _run(g, cfg)
+    assert abs(l0 - l1) <= 1e-3 * abs(l1)
+    assert global_rel_err(g0, g1) <= 1e-3

@@ -36,6 +36,26 @@ def test_band_rows_equal_the_direct_loop(H, R, s, pad, P):
             assert hs == hi - lo + 1 and (hs - R) // s + 1 == hb   # the unpadded window op yields the band
 
 
+@pytest.mark.parametrize("H,W,R,S,s,pad,P", [(8, 12, 3, 3, 1, 1, 4), (16, 8, 7, 7, 2, 3, 2), (12, 16, 1, 1, 2, 0, 4)])
+def test_width_and_rect_geometry(H, W, R, S, s, pad, P):
+    """The staged rectangle of a width band (columns by the direct loop, every row) and of a
+    full merge (every row and column the output reads)."""
+    Ho, Wo = (H + 2 * pad - R) // s + 1, (W + 2 * pad - S) // s + 1
+    g = {"samples": 2, "tensors": [{"shape": (2, H, W, 4), "kind": "act"}, {"shape": (4, R, S, 4), "kind": "param"},
+                                   {"shape": (2, Ho, Wo, 4), "kind": "act"}],
+         "ops": [{"kind": "conv2d", "inputs": [0, 1], "outputs": [2], "iattrs": [s, pad]}]}
+    wb = Wo // P
+    cfg = {0: (0, 1, 1), 1: (0, 1, 1), 2: (0, P, 1, 3)}
+    for k in range(P):
+        rlo, hs, clo, ws, nb = sim.staged_rect(g, cfg, 0, k, P)
+        assert (rlo, rlo + hs - 1) == _rows_touched(H, R, s, pad, 0, Ho)
+        assert (clo, clo + ws - 1) == _rows_touched(W, S, s, pad, k * wb, (k + 1) * wb)
+        assert nb == 2 and (ws - S) // s + 1 == wb and (hs - R) // s + 1 == Ho
+    cfg[2] = (0, 2, 1, 0)   # sample split of the output: a full merge of 1 sample per micro-op
+    rlo, hs, clo, ws, nb = sim.staged_rect(g, cfg, 0, 1, 2)
+    assert (rlo, hs, clo, ws, nb) == (-pad, (Ho - 1) * s + R, -pad, (Wo - 1) * s + S, 1)
+
+
 def _components(g):
     """Groups of 4-D activations joined by band-local ops (they must share one band split)."""
     ts, ops = g["tensors"], g["ops"]
@@ -56,9 +76,10 @@ def _components(g):
     return list(comp.values())
 
 
-def _rand_attr_cfg(g, r, ps=(2, 4)):
+def _draw_attr_cfg(g, r, ps, dims):
     """A random legal plan with band splits: memory options at random, then each group of
-    band-joined tensors in turn takes a band split, a sample split or none when legal."""
+    band-joined tensors in turn takes a height or width band split, a sample split or none
+    when legal."""
     ts = g["tensors"]
     acts = [t["id"] for t in ts if t["kind"] == "act" and t["name"] != "loss"]
     cfg = {t["id"]: (0, 1, 1) for t in ts}
@@ -68,11 +89,11 @@ def _rand_attr_cfg(g, r, ps=(2, 4)):
     r.shuffle(comps)
     for comp in comps:
         mode = r.choice(["band", "band", "sample", "none"])
-        p = r.choice(ps)
+        p, d = r.choice(ps), r.choice(dims)
         trial = dict(cfg)
         for t in comp:
             opt = cfg[t][0]
-            trial[t] = (opt, p, 1, 2) if mode == "band" else (opt, p, 1, 0) if mode == "sample" else (opt, 1, 1)
+            trial[t] = (opt, p, 1, d) if mode == "band" else (opt, p, 1, 0) if mode == "sample" else (opt, 1, 1)
         try:
             sim.expand(g, trial)
             cfg = trial
@@ -87,8 +108,15 @@ def _rand_attr_cfg(g, r, ps=(2, 4)):
                 cfg = trial
             except ValueError:
                 pass
-    assert any(sim.is_attr(g, cfg, t) for t in acts), "no band split drawn"
     return cfg
+
+
+def _rand_attr_cfg(g, r, ps=(2, 4), dims=(2, 3)):
+    for _ in range(20):
+        cfg = _draw_attr_cfg(g, r, ps, dims)
+        if any(sim.is_attr(g, cfg, t) for t in cfg):
+            return cfg
+    raise AssertionError("no band split drawn")
 
 
 @pytest.mark.parametrize("gname,seed", [("vgg_tiny", 0), ("vgg_tiny", 1), ("resnet_tiny", 0), ("resnet_tiny", 1),
