@@ -179,8 +179,8 @@ class Runtime:
                 aux = AUX_OUTPUTS.get(o["kind"], ())
                 self.needs_grad.update(t for j, t in enumerate(o["outputs"]) if j not in aux)
         for t, c in cfg.items():
-            if len(c) > 3 and c[3] == 1 and c[1] > 1:
-                raise NotImplementedError("channel-split (D-CH) plans are not exported")
+            if len(c) > 3 and c[3] != 0 and c[1] > 1:
+                raise NotImplementedError("channel-split (D-CH) and band-split (D-ATTR) plans are not exported")
         self.cuda = self.device.type == "cuda"
         if self.cuda:
             self.s_d2h, self.s_h2d = torch.cuda.Stream(self.device), torch.cuda.Stream(self.device)
