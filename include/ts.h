@@ -105,15 +105,16 @@ typedef struct {
  * operation").  dim 0 = the sample dim ("sample dim"); dim 1 = the
  * channel / parameter dim of a 2-D activation [rows, C] (Fig. 6): p_num
  * contiguous column blocks [rows, C/p_num], legal per DESIGN.md reading D-CH (produced by
- * a linear or relu/gelu/tanh, read by a linear as X or relu/gelu/tanh); dim 2 = the height
- * (attribute dim) of a 4-D NHWC activation [B, H, W, C]: p_num bands
- * [B, H/p_num, W, C] (rows [j H/p, (j+1) H/p) of every sample), legal per reading D-ATTR
+ * a linear or relu/gelu/tanh, read by a linear as X or relu/gelu/tanh); dim 2 / 3 = the
+ * height / width (attribute dims) of a 4-D NHWC activation [B, H, W, C]: p_num
+ * bands [B, H/p_num, W, C] (rows [j H/p, (j+1) H/p) of every sample) / [B, H, W/p_num, C],
+ * legal per reading D-ATTR
  * (produced by conv2d / maxpool / relu / add / batchnorm, read by those; a window op reads
  * its halo rows through a staged copy — a pool temporary in the trace). */
 typedef struct {
   int32_t tensor_id;
   int32_t opt;           /* ts_opt */
-  int32_t p_num;         /* 1, 2, 4, 8, 16; must divide `samples` (dim 0), C (dim 1) or H (dim 2) */
+  int32_t p_num;         /* 1, 2, 4, 8, 16; must divide `samples` (dim 0), C (dim 1), H (dim 2) or W (dim 3) */
   int32_t dim;
   int32_t prefetch_lead; /* >= 1 */
   int32_t release_lag;   /* swap only (reading D-LAG): the range a swap-out frees
@@ -217,7 +218,7 @@ ts_status ts_plan_ex(const ts_graph_t* g, uint64_t budget_bytes, const ts_profil
 ts_status ts_plan_get(const ts_plan_t* p, int32_t tensor_id, ts_tensor_cfg* out);
 /* Forced configuration (Fig. 9 set_config); the plan is re-expanded and
  * re-simulated.  Only TS_ACT tensors accept opt != RESIDE or p_num > 1.  p_num divides
- * the samples (dim 0), the columns (dim 1) or the height (dim 2).  TS_ERR_ARG (plan
+ * the samples (dim 0), the columns (dim 1), the height (dim 2) or the width (dim 3).  TS_ERR_ARG (plan
  * unchanged) when a field is out of range or the resulting plan breaks the channel-split
  * (D-CH) or band-split (D-ATTR) rules. */
 ts_status ts_plan_set(ts_plan_t* p, const ts_tensor_cfg* cfg);
