@@ -45,12 +45,13 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
         return any(band(t) for t in ops[o]["outputs"])
 
     def staged(o):
-        return ops[o]["kind"] in sim.ATTR_WINDOW and (band(ops[o]["inputs"][0]) or amode(o))
+        x = ops[o]["inputs"][0]
+        return ops[o]["kind"] in sim.ATTR_WINDOW and (band(x) or amode(o) or (ops[o]["kind"] == "conv2d" and chan(x)))
 
     def piece_shape(t):
         sh = list(ts[t]["shape"])
         if chan(t):
-            sh[1] //= p_of(t)
+            sh[-1] //= p_of(t)
         elif band(t):
             sh[sim.axis_of(cfg, t)] //= p_of(t)
         elif an.sample[t]:
@@ -79,7 +80,7 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
             return store[(n + t if grad else t, 0)]
         if chan(t):  # every block's rows, side by side (a copy: read-only use)
             r = rows_per_sample(t)
-            return np.concatenate([store[(n + t if grad else t, j)][s0 * r:s1 * r] for j in range(p_of(t))], axis=1)
+            return np.concatenate([store[(n + t if grad else t, j)][s0 * r:s1 * r] for j in range(p_of(t))], axis=-1)
         p = p_of(t)
         per = B // p
         j = s0 // per
@@ -92,43 +93,52 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
 
     def channel_micro_op(it):
         """Micro-op k of an op in channel mode (D-CH): output channels block k over all
-        samples.  A linear's block k is the same linear with weight rows / bias block k;
-        an elementwise op maps block k of its input to block k of its output."""
+        samples.  A linear's (conv's) block k is the same op with weight rows / bias block k;
+        a channel-local op (elementwise, batch norm with block k's parameters and statistics,
+        max pooling, add) maps block k of its inputs to block k of its output."""
         o = ops[it.op]
         k = it.k
         out = o["outputs"][0]
-        w = ts[out]["shape"][1] // p_of(out)
+        w = ts[out]["shape"][-1] // p_of(out)
+        blk = slice(k * w, (k + 1) * w)
         val = dict(pval)
-        if o["kind"] == "linear":
-            x, wid, bid = o["inputs"]
-            val[wid] = pval[wid][k * w:(k + 1) * w]
-            val[bid] = pval[bid][k * w:(k + 1) * w]
+        sliced = set()   # parameters read as block k (their gradient is block k)
+        if o["kind"] in ("linear", "conv2d"):
+            x = o["inputs"][0]
+            for pid in o["inputs"][1:]:
+                val[pid] = pval[pid][blk]
+                sliced.add(pid)
             val[x] = view(x, 0, B)
-        elif it.kind in ("F", "R"):
-            val[o["inputs"][0]] = store[(o["inputs"][0], k)]
-        else:  # the backward reads block k of what the op saved (gelu X, relu / tanh Y)
-            for t in an.saved[it.op]:
-                val[t] = store[(t, k)]
+        else:
+            for pid in o["inputs"]:
+                if ts[pid]["kind"] == "param":
+                    val[pid] = pval[pid][blk]
+                    sliced.add(pid)
+            if it.kind in ("F", "R"):
+                for t in o["inputs"]:
+                    if ts[t]["kind"] == "act":
+                        val[t] = store[(t, k)]
+            else:  # the backward reads block k of what the op saved
+                for t in an.saved[it.op]:
+                    val[t] = store[(t, k)]
         if it.kind in ("F", "R"):
             store[(out, k)][...] = net.forward_op(graph, o, val, row0=0, elem0=0, step=step)
             return
         dy = store[(n + out, k)]
         contrib = net.backward_op(graph, o, val, dy, row0=0, elem0=0, step=step)
         for tid, g in contrib.items():
-            if o["kind"] == "linear" and tid == o["inputs"][1]:
-                pgrad[tid][k * w:(k + 1) * w] += g
-            elif o["kind"] == "linear" and tid == o["inputs"][2]:
-                pgrad[tid][k * w:(k + 1) * w] += g
+            if tid in sliced:
+                pgrad[tid][blk] += g
             elif ts[tid]["kind"] == "param":
                 pgrad[tid] += g
             elif tid not in an.needs_grad:
                 continue
-            elif o["kind"] != "linear":  # elementwise: block k of its input's gradient
+            elif o["kind"] not in ("linear", "conv2d"):  # channel-local: block k of its input's gradient
                 store[(n + tid, k)][...] += g
             elif chan(tid):
-                r_w = g.shape[1] // p_of(tid)
+                r_w = g.shape[-1] // p_of(tid)
                 for j in range(p_of(tid)):
-                    store[(n + tid, j)][...] += g[:, j * r_w:(j + 1) * r_w]
+                    store[(n + tid, j)][...] += g[..., j * r_w:(j + 1) * r_w]
             else:
                 view(tid, 0, B, grad=True)[...] += g
 
@@ -136,15 +146,17 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
         """(piece index, its [b0:b1] block, the slice of the whole tensor it covers) of the
         resident pieces of the window input x (band-split or unsplit)."""
         key = n + x if grad else x
-        if not band(x):
-            return [(0, store[(key, 0)][b0:b1], (slice(None), slice(None)))]
-        ax, p = sim.axis_of(cfg, x), p_of(x)
+        al = slice(None)
+        if not band(x) and not chan(x):
+            return [(0, store[(key, 0)][b0:b1], (al, al, al))]
+        ax, p = (3 if chan(x) else sim.axis_of(cfg, x)), p_of(x)
         hb = ts[x]["shape"][ax] // p
         out = []
         for j in range(p):
             if (key, j) in store:
-                sl = slice(j * hb, (j + 1) * hb)
-                out.append((j, store[(key, j)][b0:b1], (sl, slice(None)) if ax == 1 else (slice(None), sl)))
+                sl = [al, al, al]
+                sl[ax - 1] = slice(j * hb, (j + 1) * hb)
+                out.append((j, store[(key, j)][b0:b1], tuple(sl)))
         return out
 
     def attr_micro_op(it):
@@ -167,8 +179,8 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
             # the resident pieces placed in a padded canvas, then the rectangle cut out
             pr, pc = max(0, -rlo), max(0, -clo)
             canvas = np.full((nb, H + pr + max(0, rlo + hs - H), W + pc + max(0, clo + ws - W), ts[x]["shape"][3]), fill)
-            for j, blk, (sr, sc) in input_pieces(x, b0, b0 + nb):
-                canvas[:, pr:pr + H, pc:pc + W][:, sr, sc] = blk
+            for j, blk, sl in input_pieces(x, b0, b0 + nb):
+                canvas[:, pr:pr + H, pc:pc + W][(slice(None),) + sl] = blk
             xs = canvas[:, rlo + pr:rlo + pr + hs, clo + pc:clo + pc + ws].copy()
             assert (2 * n + it.op, k) in store  # the staging temporary is allocated
             store[(2 * n + it.op, k)] = xs
@@ -191,8 +203,8 @@ def execute(graph, cfg, params, inputs, step=0, cache_bytes=0):
                     canvas = np.zeros((nb, H + pr + max(0, rlo + hs - H), W + pc + max(0, clo + ws - W), g.shape[3]))
                     canvas[:, rlo + pr:rlo + pr + hs, clo + pc:clo + pc + ws] = g
                     inside = canvas[:, pr:pr + H, pc:pc + W]   # the padding's gradient is dropped
-                    for j, blk, (sr, sc) in input_pieces(x, b0, b0 + nb, grad=True):
-                        blk[...] += inside[:, sr, sc]
+                    for j, blk, sl in input_pieces(x, b0, b0 + nb, grad=True):
+                        blk[...] += inside[(slice(None),) + sl]
             return
         if it.kind in ("F", "R"):
             for t in o["inputs"]:

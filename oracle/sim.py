@@ -74,6 +74,21 @@ BATCH_REDUCE = {"batchnorm"}
 # P = that p micro-ops over channel blocks, each over all samples; its other activations
 # are channel-split (read whole / block k as above) or unsplit.
 CHANNEL_EW = {"relu", "gelu", "tanh"}
+# Images (DESIGN.md D-CH, 4-D part): an NHWC activation split along C into p blocks
+# [B, H, W, C/p].  Producers: a conv2d in channel mode (micro-op k = output channels block k
+# from weight rows / bias block k, over every sample; its input unsplit), or a
+# CHANNEL_LOCAL4 op whose activation inputs are channel-split with the same p (ReLU, add and
+# max pooling act per channel; batch norm's statistics are per channel, so block k's are
+# complete within micro-op k).  Consumers: CHANNEL_LOCAL4 ops writing block k, or a conv2d
+# with an unsplit or sample-split output that reads every block through a staged merge
+# (D-ATTR's staging temporary, the blocks concatenated: the contraction over C needs them all).
+CHANNEL_LOCAL4 = {"relu", "add", "batchnorm", "maxpool"}
+
+
+def chan_local(graph, op):
+    """Ops that map channel block k of their inputs to block k of their output."""
+    k = op["kind"]
+    return k in CHANNEL_EW or (k in CHANNEL_LOCAL4 and len(graph["tensors"][op["outputs"][0]]["shape"]) == 4)
 
 
 def dim_of(cfg, t):
@@ -198,26 +213,31 @@ def check_channel(graph, cfg):
         if not chan(tid):
             continue
         p = cfg[tid][1]
-        if t["kind"] != "act" or len(t["shape"]) != 2 or t["shape"][1] % p:
-            raise ValueError(f"tensor {tid}: channel split needs a 2-D activation with C % p == 0")
+        nd = len(t["shape"])
+        if t["kind"] != "act" or nd not in (2, 4) or t["shape"][-1] % p:
+            raise ValueError(f"tensor {tid}: channel split needs a 2-D or NHWC activation with C % p == 0")
         po = producer[tid]
-        if po["kind"] == "linear":
+        if po["kind"] == "linear" or (po["kind"] == "conv2d" and nd == 4):
             x = po["inputs"][0]
-            if not chan(x) and cfg[x][1] != 1:
+            if not chan(x) and cfg[x][1] != 1 and ts[x]["kind"] == "act":
                 raise ValueError(f"tensor {tid}: its linear's input must be unsplit or channel-split")
-        elif po["kind"] in CHANNEL_EW:
-            x = po["inputs"][0]
-            if not chan(x) or cfg[x][1] != p:
-                raise ValueError(f"tensor {tid}: an elementwise producer needs a channel-split input of the same p")
+            if po["kind"] == "conv2d" and chan(x):
+                raise ValueError(f"tensor {tid}: a channel-split conv output needs an unsplit input")
+        elif chan_local(graph, po):
+            for x in po["inputs"]:
+                if ts[x]["kind"] == "act" and (not chan(x) or cfg[x][1] != p):
+                    raise ValueError(f"tensor {tid}: an elementwise producer needs a channel-split input of the same p")
         else:
             raise ValueError(f"tensor {tid}: producer {po['kind']} cannot write channel blocks")
         for c in consumers.get(tid, []):
-            if c["kind"] == "linear" and c["inputs"][0] == tid:
-                y = c["outputs"][0]
+            y = c["outputs"][0]
+            if c["kind"] == "linear" and c["inputs"][0] == tid and nd == 2:
                 if not chan(y) and cfg[y][1] != 1 and ts[y]["kind"] == "act":
                     raise ValueError(f"tensor {tid}: its linear consumer's output must be unsplit or channel-split")
-            elif c["kind"] in CHANNEL_EW:
-                y = c["outputs"][0]
+            elif c["kind"] == "conv2d" and nd == 4:
+                if dim_of(cfg, y) != 0 and cfg[y][1] > 1:
+                    raise ValueError(f"tensor {tid}: a conv reading channel blocks needs an unsplit or sample-split output")
+            elif chan_local(graph, c):
                 if not chan(y) or cfg[y][1] != p:
                     raise ValueError(f"tensor {tid}: an elementwise consumer needs a channel-split output of the same p")
             else:
@@ -477,7 +497,8 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
         return any(band(t) for t in ops[o]["outputs"])
 
     def staged(o):
-        return ops[o]["kind"] in ATTR_WINDOW and (band(ops[o]["inputs"][0]) or amode(o))
+        x = ops[o]["inputs"][0]
+        return ops[o]["kind"] in ATTR_WINDOW and (band(x) or amode(o) or (ops[o]["kind"] == "conv2d" and chan(x)))
 
     def chan(t):
         if t >= n:
@@ -492,7 +513,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
         if t < n and not an.sample[t]:
             return [0]
         if chan(t):
-            if cmode(o) and (t in ops[o]["outputs"] or ops[o]["kind"] in CHANNEL_EW):
+            if cmode(o) and (t in ops[o]["outputs"] or chan_local(graph, ops[o])):
                 return [k]
             return list(range(p_of(t)))
         if band(t):
@@ -530,7 +551,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
         for k in range(P):
             it = Item("F", o, k)
             it.reads = [(t, j) for t in ins_sample(o) for j in pieces(t, k, P, o)]
-            if ops[o]["kind"] in BATCH_REDUCE and k == 0:
+            if ops[o]["kind"] in BATCH_REDUCE and k == 0 and not cmode(o):  # (channel mode: per-block statistics)
                 for t in ins_sample(o):
                     for j in range(p_of(t)):
                         if (t, j) not in it.reads:
@@ -576,7 +597,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
                 cache[(t, j)] = piece_nbytes(t)
 
             saved_pieces = [(t, j) for t in an.saved[o] for j in pieces(t, k, P, o)]
-            if ops[o]["kind"] in BATCH_REDUCE and k == 0:
+            if ops[o]["kind"] in BATCH_REDUCE and k == 0 and not cmode(o):
                 for t in an.saved[o]:
                     for j in range(p_of(t)):
                         if (t, j) not in saved_pieces:
@@ -590,7 +611,7 @@ def expand(graph, cfg, order=None, an=None, cache_bytes=0):
                 if not an.is_loss[t] and t in an.needs_grad:
                     for j in pieces(t, k, P, o):
                         b.reads.append((n + t, j))
-                    if ops[o]["kind"] in BATCH_REDUCE and k == 0:
+                    if ops[o]["kind"] in BATCH_REDUCE and k == 0 and not cmode(o):
                         for j in range(p_of(t)):
                             if (n + t, j) not in b.reads:
                                 b.reads.append((n + t, j))

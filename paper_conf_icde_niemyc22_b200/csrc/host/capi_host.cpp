@@ -179,8 +179,8 @@ bool cfg_fields_ok(const Graph& g, const ts_tensor_cfg* cfg) {
   const Tensor& x = g.t[t];
   if (!pow2) return set_error("p_num must be a power of 2 <= 16"), false;
   if (cfg->dim == 0 && g.samples % cfg->p_num) return set_error("p_num must divide the samples"), false;
-  if (cfg->dim == 1 && (x.ndim != 2 || x.shape[1] % cfg->p_num))
-    return set_error("a channel split needs a 2-D tensor whose columns p_num divides"), false;
+  if (cfg->dim == 1 && ((x.ndim != 2 && x.ndim != 4) || x.shape[x.ndim - 1] % cfg->p_num))
+    return set_error("a channel split needs a 2-D or NHWC tensor whose channels p_num divides"), false;
   if (cfg->dim >= 2 && (x.ndim != 4 || x.shape[cfg->dim - 1] % cfg->p_num))
     return set_error("a band split needs a 4-D NHWC tensor whose height (dim 2) / width (dim 3) p_num divides"), false;
   if ((x.kind != TS_ACT || x.is_loss) && (cfg->opt != TS_RESIDE || cfg->p_num != 1))

@@ -99,6 +99,7 @@ struct Expansion {
 bool is_chan(const Graph& g, const std::vector<Cfg>& cfg, int key);
 bool channel_mode(const Graph& g, const std::vector<Cfg>& cfg, int op);
 bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why);
+bool chan_local(const Graph& g, int op);  // maps channel block k to block k
 
 // D-ATTR attribute (height / width) splits (expand.cpp; oracle/sim.py check_attr / staged_rect)
 bool is_attr(const Graph& g, const std::vector<Cfg>& cfg, int key);

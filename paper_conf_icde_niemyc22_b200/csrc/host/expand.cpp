@@ -43,6 +43,14 @@ bool channel_mode(const Graph& g, const std::vector<Cfg>& cfg, int op) {
   return false;
 }
 static bool chan_ew(int kind) { return kind == TS_OP_RELU || kind == TS_OP_GELU || kind == TS_OP_TANH; }
+// ops that map channel block k of their inputs to block k of their output: the elementwise
+// ones, and for NHWC images (D-CH 4-D part) ReLU, add, batch norm and max pooling
+bool chan_local(const Graph& g, int op) {
+  const Op& o = g.ops[op];
+  if (chan_ew(o.kind)) return true;
+  return g.t[o.out[0]].ndim == 4 &&
+         (o.kind == TS_OP_ADD || o.kind == TS_OP_BATCHNORM || o.kind == TS_OP_MAXPOOL);
+}
 
 bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
   for (int t = 0; t < g.n(); ++t) {
@@ -51,29 +59,36 @@ bool channel_ok(const Graph& g, const std::vector<Cfg>& cfg, std::string& why) {
     if (!is_chan(g, cfg, t)) continue;
     const Tensor& x = g.t[t];
     const int p = cfg[t].p;
-    if (x.ndim != 2 || x.shape[1] % p) return (why = "channel split needs a 2-D activation with C % p == 0"), false;
+    if ((x.ndim != 2 && x.ndim != 4) || x.shape[x.ndim - 1] % p)
+      return (why = "channel split needs a 2-D or NHWC activation with C % p == 0"), false;
     const Op& po = g.ops[x.producer];
     const int xi = po.in.empty() ? -1 : po.in[0];
-    if (po.kind == TS_OP_LINEAR) {
+    if (po.kind == TS_OP_LINEAR || (po.kind == TS_OP_CONV2D && x.ndim == 4)) {
       if (!is_chan(g, cfg, xi) && g.t[xi].kind == TS_ACT && cfg[xi].p != 1)
         return (why = "a channel-split linear output needs an unsplit or channel-split input"), false;
-    } else if (chan_ew(po.kind)) {
-      if (!is_chan(g, cfg, xi) || cfg[xi].p != p)
-        return (why = "an elementwise producer needs a channel-split input of the same p"), false;
+      if (po.kind == TS_OP_CONV2D && is_chan(g, cfg, xi))
+        return (why = "a channel-split conv output needs an unsplit input"), false;
+    } else if (chan_local(g, po.id)) {
+      for (int u : po.in)
+        if (g.t[u].kind == TS_ACT && (!is_chan(g, cfg, u) || cfg[u].p != p))
+          return (why = "an elementwise producer needs a channel-split input of the same p"), false;
     } else {
-      return (why = "only linear / relu / gelu / tanh can write channel blocks"), false;
+      return (why = "only linear / conv / relu / gelu / tanh / add / batchnorm / maxpool can write channel blocks"), false;
     }
     for (int c : x.consumers) {
       const Op& co = g.ops[c];
       const int y = co.out[0];
-      if (co.kind == TS_OP_LINEAR && co.in[0] == t) {
+      if (co.kind == TS_OP_LINEAR && co.in[0] == t && x.ndim == 2) {
         if (!is_chan(g, cfg, y) && g.t[y].kind == TS_ACT && cfg[y].p != 1)
           return (why = "a linear reading channel blocks needs an unsplit or channel-split output"), false;
-      } else if (chan_ew(co.kind)) {
+      } else if (co.kind == TS_OP_CONV2D && x.ndim == 4) {
+        if (cfg[y].dim != 0 && cfg[y].p > 1)
+          return (why = "a conv reading channel blocks needs an unsplit or sample-split output"), false;
+      } else if (chan_local(g, c)) {
         if (!is_chan(g, cfg, y) || cfg[y].p != p)
           return (why = "an elementwise consumer needs a channel-split output of the same p"), false;
       } else {
-        return (why = "only linear (as X) / relu / gelu / tanh can read channel blocks"), false;
+        return (why = "only linear (as X) / conv / elementwise ops can read channel blocks"), false;
       }
     }
   }
@@ -97,7 +112,8 @@ static bool attr_local(int kind) { return kind == TS_OP_RELU || kind == TS_OP_AD
 bool attr_window(int kind) { return kind == TS_OP_CONV2D || kind == TS_OP_MAXPOOL; }
 bool attr_staged(const Graph& g, const std::vector<Cfg>& cfg, int op) {
   const Op& o = g.ops[op];
-  return attr_window(o.kind) && (is_attr(g, cfg, o.in[0]) || attr_mode(g, cfg, op));
+  return attr_window(o.kind) && (is_attr(g, cfg, o.in[0]) || attr_mode(g, cfg, op) ||
+                                 (o.kind == TS_OP_CONV2D && is_chan(g, cfg, o.in[0])));  // D-CH staged merge
 }
 
 Window window_geom(const Graph& g, int op, int axis) {
@@ -213,7 +229,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
     if (!g.t[t].sample) return {0};
     if (is_chan(g, cfg, t)) {
       const Op& o = g.ops[op];
-      if (cm[op] && (std::find(o.out.begin(), o.out.end(), t) != o.out.end() || chan_ew(o.kind))) return {k};
+      if (cm[op] && (std::find(o.out.begin(), o.out.end(), t) != o.out.end() || chan_local(g, op))) return {k};
       std::vector<int> all(piece_count(g, cfg, t));
       for (size_t j = 0; j < all.size(); ++j) all[j] = int(j);
       return all;
@@ -255,7 +271,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       for (int x : op.in)
         if (g.t[x].sample)
           for (int j : pieces(x, k, P, o)) it.reads.push_back(pk(x, j));
-      if (batch_reduce(op.kind) && k == 0)  // full-batch statistics (R13)
+      if (batch_reduce(op.kind) && k == 0 && !cm[o])  // full-batch statistics (R13; channel mode: per block)
         for (int x : op.in)
           if (g.t[x].sample)
             for (int j = 0; j < piece_count(g, cfg, x); ++j)
@@ -320,7 +336,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       std::vector<PieceKey> saved;
       for (int t : op.saved)
         for (int j : pieces(t, k, P, op.id)) saved.push_back(pk(t, j));
-      if (batch_reduce(op.kind) && k == 0)
+      if (batch_reduce(op.kind) && k == 0 && !cm[op.id])
         for (int t : op.saved)
           for (int j = 0; j < piece_count(g, cfg, t); ++j)
             if (std::find(saved.begin(), saved.end(), pk(t, j)) == saved.end()) saved.push_back(pk(t, j));
@@ -335,7 +351,7 @@ void expand(const Graph& g, const std::vector<Cfg>& cfg, Expansion& ex, uint64_t
       for (int x : op.out)
         if (!g.t[x].is_loss && g.t[x].needs_grad) {
           for (int j : pieces(x, k, P, op.id)) b.reads.push_back(pk(n + x, j));
-          if (batch_reduce(op.kind) && k == 0)
+          if (batch_reduce(op.kind) && k == 0 && !cm[op.id])
             for (int j = 0; j < piece_count(g, cfg, x); ++j)
               if (std::find(b.reads.begin(), b.reads.end(), pk(n + x, j)) == b.reads.end())
                 b.reads.push_back(pk(n + x, j));

@@ -23,14 +23,20 @@ int grid_for(int64_t n) {
   return int(b < 148 * 8 ? b : 148 * 8);
 }
 
-// element offset of (b, h, w) inside its piece, and the piece
-__device__ __forceinline__ int64_t band_off(const BandPieces& x, int H, int W, int b, int h, int w, int& j) {
+// element offset of (b, h, w, c) inside its piece, and the piece (axis 3: channel blocks of
+// hb channels, D-CH's staged merge)
+__device__ __forceinline__ int64_t band_off(const BandPieces& x, int H, int W, int C, int b, int h, int w, int c,
+                                            int& j) {
   if (x.axis == 1) {
     j = h / x.hb;
-    return (int64_t(b) * x.hb + (h - j * x.hb)) * W + w;
+    return ((int64_t(b) * x.hb + (h - j * x.hb)) * W + w) * C + c;
   }
-  j = w / x.hb;
-  return (int64_t(b) * H + h) * x.hb + (w - j * x.hb);
+  if (x.axis == 2) {
+    j = w / x.hb;
+    return ((int64_t(b) * H + h) * x.hb + (w - j * x.hb)) * C + c;
+  }
+  j = c / x.hb;
+  return ((int64_t(b) * H + h) * W + w) * x.hb + (c - j * x.hb);
 }
 
 template <class T, int V>
@@ -45,8 +51,8 @@ __global__ void band_gather_k(BandPieces x, int H, int W, int C, Rect r, T fill,
     T* o = out + pix * C + int64_t(cv) * V;
     if (h >= 0 && h < H && ww >= 0 && ww < W) {
       int j;
-      const int64_t off = band_off(x, H, W, r.b0 + b, h, ww, j);
-      const T* src = static_cast<const T*>(x.ptr[j]) + off * C + int64_t(cv) * V;
+      const int64_t off = band_off(x, H, W, C, r.b0 + b, h, ww, cv * V, j);
+      const T* src = static_cast<const T*>(x.ptr[j]) + off;
       if constexpr (V * sizeof(T) == 16) {
         *reinterpret_cast<uint4*>(o) = *reinterpret_cast<const uint4*>(src);
       } else {
@@ -71,8 +77,8 @@ __global__ void band_scatter_add_k(const T* __restrict__ src, BandPieces dx, int
     const int64_t pix = i / CV;
     const int w = w0 + int(pix % nw), h = h0 + int((pix / nw) % nh), b = int(pix / (int64_t(nw) * nh));
     int j;
-    const int64_t off = band_off(dx, H, W, r.b0 + b, h, w, j);
-    T* d = static_cast<T*>(const_cast<void*>(dx.ptr[j])) + off * C + int64_t(cv) * V;
+    const int64_t off = band_off(dx, H, W, C, r.b0 + b, h, w, cv * V, j);
+    T* d = static_cast<T*>(const_cast<void*>(dx.ptr[j])) + off;
     const T* s = src + ((int64_t(b) * r.hs + (h - r.rlo)) * r.ws + (w - r.clo)) * C + int64_t(cv) * V;
     if constexpr (V * sizeof(T) == 16) {
       uint4 dv = *reinterpret_cast<const uint4*>(d);
@@ -93,7 +99,7 @@ template <class T>
 void gather_launch(const BandPieces& x, int H, int W, int C, const Rect& r, T fill, void* out, cudaStream_t st) {
   constexpr int V = 16 / sizeof(T);
   const int64_t pix = int64_t(r.nb) * r.hs * r.ws;
-  if (C % V == 0)
+  if (C % V == 0 && (x.axis != 3 || x.hb % V == 0))  // (a vector never straddles two channel blocks)
     band_gather_k<T, V><<<grid_for(pix * (C / V)), kT, 0, st>>>(x, H, W, C, r, fill, static_cast<T*>(out));
   else
     band_gather_k<T, 1><<<grid_for(pix * C), kT, 0, st>>>(x, H, W, C, r, fill, static_cast<T*>(out));
@@ -106,7 +112,7 @@ void scatter_launch(const void* src, const BandPieces& dx, int H, int W, int C, 
   const int w0 = r.clo > 0 ? r.clo : 0, w1 = r.clo + r.ws < W ? r.clo + r.ws : W;
   if (h1 <= h0 || w1 <= w0) return;
   const int64_t pix = int64_t(r.nb) * (h1 - h0) * (w1 - w0);
-  if (C % V == 0)
+  if (C % V == 0 && (dx.axis != 3 || dx.hb % V == 0))
     band_scatter_add_k<T, V><<<grid_for(pix * (C / V)), kT, 0, st>>>(static_cast<const T*>(src), dx, H, W, C, r, h0,
                                                                        h1 - h0, w0, w1 - w0);
   else

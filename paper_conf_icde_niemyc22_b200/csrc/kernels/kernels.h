@@ -173,7 +173,7 @@ void maxpool_bwd(int dt, const void* dy, const void* x, void* dx, int acc, int n
 // (axis 2: [B, H, hb, C]); an unsplit one is one piece with axis 1, hb = H.
 struct BandPieces {
   const void* ptr[16] = {};
-  int hb = 0, axis = 1;
+  int hb = 0, axis = 1;  // axis 3: channel blocks of hb channels [B, H, W, hb] (D-CH staged merge)
 };
 // The staged rectangle: rows [rlo, rlo + hs) x columns [clo, clo + ws) of samples [b0, b0 + nb).
 struct Rect {

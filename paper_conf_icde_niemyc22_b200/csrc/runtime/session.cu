@@ -552,12 +552,18 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       a.K = int(w.shape[0]); a.R = int(w.shape[1]); a.S = int(w.shape[2]);
       a.P = int(out.shape[1]); a.Q = int(out.shape[2]);
       a.stride = int(o.ia[0]); a.pad = int(o.ia[1]);
-      a.w = param_w(s, o.in[1]);
+      // D-CH channel mode: output channels block cb = the same conv with weight rows (and
+      // bias) block cb, over every sample
+      const int64_t k0 = m.cb >= 0 ? int64_t(m.cb) * (a.K / m.cp) : 0;
+      if (m.cb >= 0) a.K /= m.cp;
+      const int es = dt == tsk::BF16 ? 2 : 4;
+      const int64_t wrow = int64_t(a.R) * a.S * a.C;  // elements per weight row
+      a.w = param_w(s, o.in[1]) + k0 * wrow * es;
       const bool has_bias = o.in.size() > 2;
       if (!bwd) {
         a.x = V(o.in[0]);
         char* y = V(o.out[0]);
-        const void* bias = has_bias ? param_w(s, o.in[2]) : nullptr;
+        const void* bias = has_bias ? param_w(s, o.in[2]) + k0 * es : nullptr;
         nk = 1;
         return [a, y, bias](cudaStream_t st) { tsk::conv_fprop(a, y, bias, st); };
       }
@@ -565,9 +571,9 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       a.dy = G(o.out[0]);
       char* dx = (x.kind == TS_ACT && x.needs_grad) ? G(o.in[0]) : nullptr;
       const int dxacc = dx ? A(g.n() + o.in[0]) : 0;
-      float* dw = param_g(s, o.in[1]);
+      float* dw = param_g(s, o.in[1]) + k0 * wrow;
       const int dwacc = A(o.in[1]);
-      float* db = has_bias ? param_g(s, o.in[2]) : nullptr;
+      float* db = has_bias ? param_g(s, o.in[2]) + k0 : nullptr;
       const int dbacc = has_bias ? A(o.in[2]) : 0;
       const int64_t pix = ns * int64_t(a.P) * a.Q;
       const uint64_t wsb = g.ws_bytes;
@@ -580,15 +586,19 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
     }
     case TS_OP_BATCHNORM: {
       const Tensor& x = g.t[o.in[0]];
-      const int C = int(x.shape[x.ndim - 1]);
+      // D-CH channel mode: micro-op cb normalises channels block cb over every sample, with its
+      // own statistics (the stats buffer holds p consecutive [mean | rstd | sums] blocks)
+      const int C = int(x.shape[x.ndim - 1]) / (m.cb >= 0 ? m.cp : 1);
+      const int64_t c0 = m.cb >= 0 ? int64_t(m.cb) * C : 0;
+      const int es = dt == tsk::BF16 ? 2 : 4;
       const int64_t rows = n_out / C;
-      const int64_t m_total = out.numel / C;
-      float* bs = reinterpret_cast<float*>(s->slab + g.bn_off[o.id]);
-      char *gw = param_w(s, o.in[1]), *bw = param_w(s, o.in[2]);
+      const int64_t m_total = out.numel / x.shape[x.ndim - 1];
+      float* bs = reinterpret_cast<float*>(s->slab + g.bn_off[o.id]) + 4 * c0;
+      char *gw = param_w(s, o.in[1]) + c0 * es, *bw = param_w(s, o.in[2]) + c0 * es;
       const uint64_t wsb = g.ws_bytes;
       if (!bwd) {
         const float eps = float(o.fa[0]);
-        const bool stats = m.k == 0 && !m.replay;
+        const bool stats = (m.k == 0 || m.cb >= 0) && !m.replay;
         const tsk::PieceList px = m.all_x;
         char *xp = V(o.in[0]), *y = V(o.out[0]);
         nk = stats ? 3 : 1;
@@ -597,9 +607,9 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
           tsk::bn_apply(dt, xp, bs, gw, bw, y, rows, C, st);
         };
       }
-      const bool sums = m.k == 0;
+      const bool sums = m.k == 0 || m.cb >= 0;
       const tsk::PieceList px = m.all_x, pdy = m.all_dy;
-      float *dg = param_g(s, o.in[1]), *dbt = param_g(s, o.in[2]);
+      float *dg = param_g(s, o.in[1]) + c0, *dbt = param_g(s, o.in[2]) + c0;
       const int pacc = A(o.in[1]);
       char* dx = (x.kind == TS_ACT && x.needs_grad) ? G(o.in[0]) : nullptr;
       const int acc = dx ? A(g.n() + o.in[0]) : 0;
@@ -612,7 +622,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
     }
     case TS_OP_MAXPOOL: {
       const Tensor& x = g.t[o.in[0]];
-      const int H = int(x.shape[1]), W = int(x.shape[2]), C = int(x.shape[3]);
+      const int H = int(x.shape[1]), W = int(x.shape[2]), C = int(x.shape[3]) / (m.cb >= 0 ? m.cp : 1);
       const int P = int(out.shape[1]), Q = int(out.shape[2]);
       const int kk = int(o.ia[0]), st_ = int(o.ia[1]), pad = int(o.ia[2]);
       const int nn = int(ns);
@@ -813,9 +823,9 @@ std::function<void(cudaStream_t)> lower_staged(ts_session_t* s, const Item& it, 
     return f == where.end() ? nullptr : s->slab + f->second;
   };
   auto pieces_of = [&](int key, tsk::BandPieces& bp) {
-    const bool bx = is_attr(g, s->cfg, xi);
-    const int px = bx ? piece_count(g, s->cfg, xi) : 1;
-    bp.axis = bx ? attr_axis(s->cfg, xi) : 1;
+    const bool bx = is_attr(g, s->cfg, xi), cx = is_chan(g, s->cfg, xi);
+    const int px = bx || cx ? piece_count(g, s->cfg, xi) : 1;
+    bp.axis = bx ? attr_axis(s->cfg, xi) : cx ? 3 : 1;
     bp.hb = int(x.shape[bp.axis] / px);
     for (int j = 0; j < px; ++j) bp.ptr[j] = at(pk(key, j));
   };
@@ -1020,7 +1030,7 @@ ts_status build_program(ts_session_t* s) {
         m.s0 = 0;
         m.s1 = B;
       }
-      const bool ew_op = o.kind == TS_OP_RELU || o.kind == TS_OP_GELU || o.kind == TS_OP_TANH;
+      const bool ew_op = chan_local(g, it.op);  // maps channel block k to block k
       // a channel-split tensor this micro-op touches as block k only (else: every block)
       auto own_block = [&](int t) {
         return cmode && (ew_op || std::find(o.out.begin(), o.out.end(), t) != o.out.end());
@@ -1088,7 +1098,7 @@ ts_status build_program(ts_session_t* s) {
             if (f == grad_first_op.end()) grad_first_op[gk] = it.op;
             m.acc[gk] = grad_first_op[gk] != it.op ? 1 : 0;
             // a channel-mode linear's micro-ops all write the whole dX: block 0 overwrites
-            if (cmode && o.kind == TS_OP_LINEAR && !m.acc[gk] && m.k > 0) m.acc[gk] = 1;
+            if (cmode && (o.kind == TS_OP_LINEAR || o.kind == TS_OP_CONV2D) && !m.acc[gk] && m.k > 0) m.acc[gk] = 1;
             // D-ATTR: a band's gradient is started by whichever item wrote it first
             if (is_attr(g, s->cfg, t)) m.acc[gk] = gpiece_written.count(pk(gk, m.k)) ? 1 : 0;
           }
@@ -1101,14 +1111,20 @@ ts_status build_program(ts_session_t* s) {
         const uint64_t need = uint64_t(o.ia[0]) * uint64_t(o.ia[1]) * 4;  // one sample's row terms (chunked)
         if (need + 4096 > g.ws_bytes) return set_error("attention: workspace too small for the row terms"), TS_ERR_GRAPH;
       }
-      if (batch_reduce(o.kind) && it.k == 0 && it.kind != IT_R) {  // replays reuse the step's statistics
-        const int C = int(g.t[o.in[0]].shape[g.t[o.in[0]].ndim - 1]);
+      if (batch_reduce(o.kind) && (it.k == 0 || cmode) && it.kind != IT_R) {  // replays reuse the step's statistics
+        const int C = int(g.t[o.in[0]].shape[g.t[o.in[0]].ndim - 1]) / (cmode ? m.P : 1);
         if (!tsk::bn_supported(g.dtype == TS_BF16 ? tsk::BF16 : tsk::F32, C))
           return set_error("batchnorm: channel count " + std::to_string(C) + " not supported"), TS_ERR_GRAPH;
         auto list = [&](int key, tsk::PieceList& L) -> bool {
           int t = key >= n ? key - n : key;
           int p = piece_count(g, s->cfg, t);
           if (p > tsk::PieceList::kMax) return false;
+          if (cmode) {  // D-CH: block k holds every sample of its channels
+            L.np = 1;
+            L.ptr[0] = s->slab + where.at(pk(key, m.k));
+            L.rows[0] = g.t[t].numel / C;
+            return true;
+          }
           L.np = p;
           for (int j = 0; j < p; ++j) {
             L.ptr[j] = s->slab + where.at(pk(key, j));

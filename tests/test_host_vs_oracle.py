@@ -453,3 +453,24 @@ def test_band_plan_serialize_roundtrip():
     P = tsplit.Plan.plan(G, st["static_bytes"] + int(0.5 * (st["peak_extent"] - st["static_bytes"])))
     Q = tsplit.Plan.deserialize(G, P.serialize())
     assert Q.trace() == P.trace() and Q.oracle_cfg() == P.oracle_cfg()
+
+
+@pytest.mark.parametrize("gname,seed", [("vgg_tiny", 0), ("vgg_tiny", 1), ("resnet_tiny", 0), ("resnet_tiny", 1),
+                                        ("vgg16", 2), ("resnet50", 3)])
+def test_trace_bit_exact_channel4_plans(gname, seed):
+    """D-CH on NHWC images (conv / BN / pool / add channel blocks, staged merges): the C++
+    expansion and trace equal the oracle simulator's bit for bit."""
+    from test_oracle_channel4 import rand_chan4_cfg
+    over = {"batch": 4} if gname in ("vgg16", "resnet50") else {}
+    g = graphs.config_graph(gname, **over)
+    cfg = rand_chan4_cfg(g, random.Random(500 + seed))
+    plan = tsplit.Plan.default(tsplit.Graph(g))
+    plan.set_many({t: cfg[t] for t in brute.act_tensors(g)})
+    ref = sim.simulate(g, cfg)
+    got = plan.trace()
+    assert len(got) == len(ref.trace)
+    for a, b in zip(got, ref.trace):
+        assert a == tuple(b), (a, b)
+    assert [it[0] for it in plan.items()] == [it.kind for it in ref.items]
+    for t in brute.act_tensors(g):
+        assert plan.get_dim(t) == (sim.dim_of(cfg, t) if cfg[t][1] > 1 else 0)
