@@ -593,16 +593,19 @@ def main():
             "achieved_tflops": g_flop / (g_ms / 1e3) / 1e12 if g_ms > 0 else None,
             "share_of_step": g_ms / step_ms_prof if step_ms_prof else None}
     # BASELINE metric part 2 (config 5): max trainable batch x hidden under the whole HBM, measured
-    # by tools/max_scale.py (planning up to 1024 x 512 tokens takes minutes, so not in this run)
-    msf = os.path.join(ROOT, "profiles", "r1_max_scale.json")
+    # by tools/scale_sweep.py (planning up to 8192 x 512 tokens takes minutes, so not in this run)
+    msf = os.path.join(ROOT, "profiles", "r2_scale_sweep.json")
     if bert and os.path.exists(msf):
         ms = json.load(open(msf))
         line["max_trainable"] = {
-            "source": "profiles/r1_max_scale.json (tools/max_scale.py, 24L s512 BERT, heads = h/64, capacity = "
-                      "free HBM - 6 GB; not re-measured in this run)",
+            "source": "profiles/r2_scale_sweep.json (tools/scale_sweep.py, SURVEY C5 grid: 24L s512 BERT, heads = "
+                      "h/64, FFN 4h, batch doubled from 8 until Alg. 2 fails or 8192; capacity = free HBM - 6 GB; "
+                      "timed = the largest plan whose pinned swap pool fits 100 GiB of host memory; not re-measured "
+                      "in this run)",
             "capacity_bytes": ms.get("capacity_bytes"),
-            "per_hidden": [{k: e.get(k) for k in ("hidden", "max_batch_unsplit", "max_batch_tsplit", "scale",
-                                                   "scale_unsplit", "samples_per_s")} for e in ms.get("summary", [])]}
+            "per_hidden": [{k: e.get(k) for k in ("hidden", "max_batch_unsplit", "max_batch_tsplit", "scale_unsplit",
+                                                   "scale_tsplit", "timed_batch", "samples_per_s", "host_pool_bytes")}
+                           for e in ms.get("summary", [])]}
     if bert:
         # north_star: the paper's ratios, quoted with the GPU PAPER.md names — context only
         line["paper_context"] = {
