@@ -129,6 +129,7 @@ struct Micro {
   // sample mode); a channel-split tensor the micro-op reads whole appears as one pointer per
   // block (its rows [s0, s1)) in vblk / gblk instead of val / grad
   int cb = -1, cp = 1;
+  bool chan = false;  // channel mode (cb / cp are also set in attribute mode, D-ATTR: band k of P)
   std::unordered_map<int, std::vector<char*>> vblk, gblk;
 };
 
@@ -554,8 +555,8 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       a.stride = int(o.ia[0]); a.pad = int(o.ia[1]);
       // D-CH channel mode: output channels block cb = the same conv with weight rows (and
       // bias) block cb, over every sample
-      const int64_t k0 = m.cb >= 0 ? int64_t(m.cb) * (a.K / m.cp) : 0;
-      if (m.cb >= 0) a.K /= m.cp;
+      const int64_t k0 = m.chan ? int64_t(m.cb) * (a.K / m.cp) : 0;
+      if (m.chan) a.K /= m.cp;
       const int es = dt == tsk::BF16 ? 2 : 4;
       const int64_t wrow = int64_t(a.R) * a.S * a.C;  // elements per weight row
       a.w = param_w(s, o.in[1]) + k0 * wrow * es;
@@ -588,8 +589,8 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       const Tensor& x = g.t[o.in[0]];
       // D-CH channel mode: micro-op cb normalises channels block cb over every sample, with its
       // own statistics (the stats buffer holds p consecutive [mean | rstd | sums] blocks)
-      const int C = int(x.shape[x.ndim - 1]) / (m.cb >= 0 ? m.cp : 1);
-      const int64_t c0 = m.cb >= 0 ? int64_t(m.cb) * C : 0;
+      const int C = int(x.shape[x.ndim - 1]) / (m.chan ? m.cp : 1);
+      const int64_t c0 = m.chan ? int64_t(m.cb) * C : 0;
       const int es = dt == tsk::BF16 ? 2 : 4;
       const int64_t rows = n_out / C;
       const int64_t m_total = out.numel / x.shape[x.ndim - 1];
@@ -598,7 +599,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
       const uint64_t wsb = g.ws_bytes;
       if (!bwd) {
         const float eps = float(o.fa[0]);
-        const bool stats = (m.k == 0 || m.cb >= 0) && !m.replay;
+        const bool stats = (m.k == 0 || m.chan) && !m.replay;
         const tsk::PieceList px = m.all_x;
         char *xp = V(o.in[0]), *y = V(o.out[0]);
         nk = stats ? 3 : 1;
@@ -607,7 +608,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
           tsk::bn_apply(dt, xp, bs, gw, bw, y, rows, C, st);
         };
       }
-      const bool sums = m.k == 0 || m.cb >= 0;
+      const bool sums = m.k == 0 || m.chan;
       const tsk::PieceList px = m.all_x, pdy = m.all_dy;
       float *dg = param_g(s, o.in[1]) + c0, *dbt = param_g(s, o.in[2]) + c0;
       const int pacc = A(o.in[1]);
@@ -622,7 +623,7 @@ std::function<void(cudaStream_t)> lower(ts_session_t* s, const Micro& m, bool bw
     }
     case TS_OP_MAXPOOL: {
       const Tensor& x = g.t[o.in[0]];
-      const int H = int(x.shape[1]), W = int(x.shape[2]), C = int(x.shape[3]) / (m.cb >= 0 ? m.cp : 1);
+      const int H = int(x.shape[1]), W = int(x.shape[2]), C = int(x.shape[3]) / (m.chan ? m.cp : 1);
       const int P = int(out.shape[1]), Q = int(out.shape[2]);
       const int kk = int(o.ia[0]), st_ = int(o.ia[1]), pad = int(o.ia[2]);
       const int nn = int(ns);
@@ -1024,6 +1025,7 @@ ts_status build_program(ts_session_t* s) {
       const bool cmode = channel_mode(g, s->cfg, it.op);
       const bool amode = attr_mode(g, s->cfg, it.op);      // D-ATTR: micro-op k = band k of every sample
       const bool staged = attr_staged(g, s->cfg, it.op);   // D-ATTR window op on a staged input copy
+      m.chan = cmode;
       if (cmode || amode) {  // D-CH: micro-op k = output channel block k over every sample
         m.cb = it.k;
         m.cp = m.P;
@@ -1122,7 +1124,7 @@ ts_status build_program(ts_session_t* s) {
           if (cmode) {  // D-CH: block k holds every sample of its channels
             L.np = 1;
             L.ptr[0] = s->slab + where.at(pk(key, m.k));
-            L.rows[0] = g.t[t].numel / C;
+            L.rows[0] = g.t[t].numel / p / C;  // (C = the block's channels)
             return true;
           }
           L.np = p;
