@@ -306,8 +306,10 @@ def main():
     ap.add_argument("--budget-frac", type=float, default=None)
     ap.add_argument("--layers", type=int, default=LAYERS)
     ap.add_argument("--no-unbudgeted", action="store_true")
-    ap.add_argument("--no-plan-trial", action="store_true",
-                    help="take the measured-profile plan without the short trial against the analytic-profile plan")
+    ap.add_argument("--plan-trial", action="store_true",
+                    help="also plan with the analytic profile and keep whichever plan runs faster in a short "
+                         "untimed trial (default: ts_plan's own choice, which already scores both cost models "
+                         "on the measured timeline)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--analytic-profile", action="store_true", help="plan with the analytic model, not measured times")
     args = ap.parse_args()
@@ -367,14 +369,16 @@ def main():
         prof = tsplit.Profile.measure(G, dev_inputs, max_p=16, device=local) if not args.analytic_profile else None
         pcie = prof.pcie() if prof else None
         plan_profile = "measured" if prof else "analytic"
-        # Alg. 2 is a path-dependent greedy heuristic: plan with the measured profile and with
-        # the analytic cost model, then keep the candidate that runs faster in a short untimed
-        # trial (a dead end of one of them is reported in config)
-        # (ts_plan itself keeps the faster of Alg. 2 with and without split proposals)
+        # the plan is ts_plan's: given the measured profile it runs Alg. 2 on measured and on
+        # analytic costs, with and without split proposals, and keeps the plan the measured
+        # timeline predicts fastest.  --plan-trial adds the analytic-profile plan and keeps
+        # whichever runs faster in a short untimed trial (reported in config)
         cands = []
         for label, pr in (("measured", prof), ("analytic", None)):
             if pr is None and label != "analytic":
                 continue
+            if label == "analytic" and cands and not args.plan_trial:
+                continue   # (the analytic-profile plan only when the measured one dead-ends)
             try:
                 cands.append((label, tsplit.Plan.plan(G, budget, pr)))
             except tsplit.TsError as e:
@@ -383,7 +387,7 @@ def main():
                 plan_trials[label] = f"infeasible: {str(e)[:80]}"
         if not cands:
             raise RuntimeError(f"no feasible plan: {plan_trials}")
-        if len(cands) > 1 and not args.no_plan_trial:
+        if len(cands) > 1 and args.plan_trial:
             tstream = torch.cuda.Stream()
             prm = gen.init_params(spec, seed=1)
             for label, pl in cands:
