@@ -312,6 +312,8 @@ def main():
                          "on the measured timeline)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--analytic-profile", action="store_true", help="plan with the analytic model, not measured times")
+    ap.add_argument("--bf16-grads", action="store_true",
+                    help="data parallelism: bf16 gradient buckets on the link (fp32 masters and SGD)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     W = WORKLOADS[args.workload]
@@ -421,7 +423,7 @@ def main():
 
     def make_session(p):
         s = tsplit.Session(G, p, device=local, lr=1e-4, streams=streams, nccl_comm=comm, world_size=world,
-                           sample_offset=rank * spec["samples"])
+                           sample_offset=rank * spec["samples"], grad_allreduce_bf16=args.bf16_grads)
         s.set_params(params)
         return s
 

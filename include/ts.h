@@ -281,6 +281,12 @@ typedef struct {
                                 compute the step of the concatenated batch (0 on 1 GPU)   */
   int32_t host_numa_node;    /* NUMA node of the pinned swap pool: >= 0 that node, -1 the
                                 GPU's own node (sysfs), -2 no binding (cudaHostAlloc)     */
+  int32_t grad_allreduce_bf16; /* 1: each gradient bucket is rounded to bf16, summed by
+                                ncclAllReduce in bf16 and widened back into the fp32
+                                gradients (half the bytes on the link; the sum rounds to
+                                bf16 — the fp32 masters and SGD stay fp32).  Needs a bf16
+                                staging buffer of the largest bucket / 2 outside the slab.  0:
+                                fp32 buckets                                                */
 } ts_session_cfg;
 
 /* Lays out the static region, allocates the pinned host swap pool, uploads

@@ -152,6 +152,10 @@ __global__ void cast_kernel(const float* __restrict__ s, bf16* __restrict__ d, i
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
     d[i] = __float2bfloat16_rn(s[i]);
 }
+__global__ void uncast_kernel(const bf16* __restrict__ s, float* __restrict__ d, int64_t n) {
+  for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
+    d[i] = __bfloat162float(s[i]);
+}
 __global__ void step_advance_kernel(uint32_t* c) { *c += 1u; }
 __global__ void scale_kernel(float* x, int64_t n, float s) {
   for (int64_t i = int64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < n; i += int64_t(gridDim.x) * blockDim.x)
@@ -279,6 +283,9 @@ void sgd_fused(const SgdChunk* chunks, int n_chunks, char* slab, float lr, float
 }
 void cast_f32_bf16(const float* src, void* dst, int64_t n, cudaStream_t st) {
   cast_kernel<<<grid_for(n), 256, 0, st>>>(src, reinterpret_cast<bf16*>(dst), n);
+}
+void cast_bf16_f32(const void* src, float* dst, int64_t n, cudaStream_t st) {
+  uncast_kernel<<<grid_for(n), 256, 0, st>>>(reinterpret_cast<const bf16*>(src), dst, n);
 }
 void step_advance(uint32_t* counter, cudaStream_t st) { step_advance_kernel<<<1, 1, 0, st>>>(counter); }
 void scale_f32(float* x, int64_t n, float s, cudaStream_t st) { scale_kernel<<<grid_for(n), 256, 0, st>>>(x, n, s); }

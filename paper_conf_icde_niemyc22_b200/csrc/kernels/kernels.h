@@ -244,6 +244,7 @@ struct SgdChunk {
 };
 void sgd_fused(const SgdChunk* chunks, int n_chunks, char* slab, float lr, float gscale, cudaStream_t st);
 void cast_f32_bf16(const float* src, void* dst, int64_t n, cudaStream_t st);
+void cast_bf16_f32(const void* src, float* dst, int64_t n, cudaStream_t st);
 void scale_f32(float* x, int64_t n, float s, cudaStream_t st);
 
 }  // namespace tsk

@@ -44,7 +44,7 @@ namespace {
 // Minimal NCCL ABI (resolved with dlsym from the libnccl the process already has).
 typedef int (*nccl_allreduce_fn)(const void*, void*, size_t, int, int, void*, cudaStream_t);
 typedef int (*nccl_group_fn)();
-constexpr int kNcclFloat32 = 7, kNcclSum = 0;
+constexpr int kNcclFloat32 = 7, kNcclBfloat16 = 9, kNcclSum = 0;
 
 }  // namespace
 
@@ -93,6 +93,8 @@ struct ts_session_s {
   int host_numa = -1;         // node the pool is bound to (-1: unbound)
   bool host_registered = false;  // mmap + cudaHostRegister (else cudaHostAlloc)
   int64_t sample0 = 0;        // global index of this rank's first sample (dropout counters)
+  bool grad_bf16 = false;     // bf16 gradient buckets (ts_session_cfg.grad_allreduce_bf16)
+  char* bucket_stage = nullptr;  // bf16 staging of one bucket (outside the slab)
   std::vector<Cmd> prog;
   std::vector<cudaEvent_t> ev_d2h, ev_h2d;  // indexed by item
   cudaEvent_t ev_mark = nullptr, ev_join_d2h = nullptr, ev_join_h2d = nullptr;
@@ -1346,6 +1348,16 @@ ts_status build_program(ts_session_t* s) {
   if (s->nccl) {  // (a 1-rank communicator exercises the same path on one GPU)
     s->buckets = grad_buckets(g, s->ex, uint64_t(32) << 20);
     s->ev_bucket.assign(s->buckets.size(), nullptr);
+    if (s->grad_bf16) {  // one bf16 staging buffer, sized for the largest bucket
+      uint64_t mx = 0;
+      for (auto& bk : s->buckets) {
+        uint64_t tot = 0;
+        for (auto& sp : bk.spans) tot += sp.second / 2;
+        mx = std::max(mx, tot);
+      }
+      if (mx) CU(cudaMalloc(&s->bucket_stage, mx));
+      for (auto& bk : s->buckets) s->launches += 2 * int64_t(bk.spans.size());
+    }
     for (size_t b = 0; b < s->buckets.size(); ++b) {
       s->buckets_after[std::max(0, s->buckets[b].after_item)].push_back(int(b));
       CU(cudaEventCreateWithFlags(&s->ev_bucket[b], cudaEventDisableTiming));
@@ -1416,6 +1428,22 @@ void issue_step(ts_session_t* s) {
     for (int b : s->buckets_after[c.item]) {
       cudaEventRecord(s->ev_bucket[b], cs);
       cudaStreamWaitEvent(s->comm, s->ev_bucket[b], 0);
+      if (s->grad_bf16 && s->bucket_stage) {  // bf16 on the link: round, one sum, widen back
+        uint64_t o = 0;
+        for (auto& sp : s->buckets[b].spans) {
+          tsk::cast_f32_bf16(reinterpret_cast<const float*>(s->slab + sp.first), s->bucket_stage + o,
+                             int64_t(sp.second / 4), s->comm);
+          o += sp.second / 2;
+        }
+        s->allreduce(s->bucket_stage, s->bucket_stage, o / 2, kNcclBfloat16, kNcclSum, s->nccl, s->comm);
+        o = 0;
+        for (auto& sp : s->buckets[b].spans) {
+          tsk::cast_bf16_f32(s->bucket_stage + o, reinterpret_cast<float*>(s->slab + sp.first), int64_t(sp.second / 4),
+                             s->comm);
+          o += sp.second / 2;
+        }
+        continue;
+      }
       if (s->group_start) s->group_start();
       for (auto& sp : s->buckets[b].spans)
         s->allreduce(s->slab + sp.first, s->slab + sp.first, sp.second / 4, kNcclFloat32, kNcclSum, s->nccl,
@@ -1558,6 +1586,7 @@ ts_status ts_session_create(const ts_graph_t* gh, const ts_plan_t* ph, const ts_
   s->lr = cfg->lr;
   s->step = cfg->step0;
   s->sample0 = cfg->sample_offset;
+  s->grad_bf16 = cfg->grad_allreduce_bf16 != 0;
   s->host_numa_req = cfg->host_numa_node;
   s->use_graph = cfg->use_cuda_graph != 0;
   if (cfg->stream_compute) {
@@ -1603,6 +1632,7 @@ void ts_session_destroy(ts_session_t* s) {
   if (s->ev_comm_done) cudaEventDestroy(s->ev_comm_done);
   if (s->sgd_chunks) cudaFree(s->sgd_chunks);
   if (s->step_dev) cudaFree(s->step_dev);
+  if (s->bucket_stage) cudaFree(s->bucket_stage);
   if (s->comm) cudaStreamDestroy(s->comm);
   if (s->ev_mark) cudaEventDestroy(s->ev_mark);
   if (s->ev_join_d2h) cudaEventDestroy(s->ev_join_d2h);

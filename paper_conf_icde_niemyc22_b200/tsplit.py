@@ -62,7 +62,7 @@ class SessionCfg(C.Structure):
                 ("stream_compute", C.c_void_p), ("stream_d2h", C.c_void_p), ("stream_h2d", C.c_void_p),
                 ("nccl_comm", C.c_void_p), ("world_size", C.c_int32), ("use_cuda_graph", C.c_int32),
                 ("lr", C.c_float), ("step0", C.c_uint32), ("sample_offset", C.c_int64),
-                ("host_numa_node", C.c_int32)]
+                ("host_numa_node", C.c_int32), ("grad_allreduce_bf16", C.c_int32)]
 
 
 class TsError(RuntimeError):
@@ -417,7 +417,7 @@ class Session:
     def __init__(self, graph: Graph, plan: Plan, device: int = 0, slab_bytes: int | None = None,
                  lr: float = 0.0, use_cuda_graph: bool = True, nccl_comm: int | None = None,
                  world_size: int = 1, step0: int = 0, streams=None, sample_offset: int = 0,
-                 host_numa_node: int = -1):
+                 host_numa_node: int = -1, grad_allreduce_bf16: bool = False):
         import torch
         if not torch.cuda.is_available():
             raise TsError(9, "no CUDA device: the TSPLIT runtime has no CPU fallback")
@@ -439,6 +439,7 @@ class Session:
         cfg.step0 = step0
         cfg.sample_offset = sample_offset
         cfg.host_numa_node = host_numa_node
+        cfg.grad_allreduce_bf16 = 1 if grad_allreduce_bf16 else 0
         h = C.c_void_p()
         check(lib().ts_session_create(graph.h, plan.h, C.byref(cfg), C.byref(h)))
         self.h = h

@@ -190,6 +190,29 @@ def test_nccl_bucketed_allreduce_single_rank():
     assert np.allclose(out[1][1], out[0][1], rtol=1e-6, atol=1e-9)
 
 
+def test_nccl_bf16_gradient_buckets_single_rank():
+    """bf16 gradient buckets (ts_session_cfg.grad_allreduce_bf16): each bucket is
+    rounded to bf16, summed by ncclAllReduce in bf16 and widened back.  With a 1-rank
+    communicator the sum is the identity, so every gradient equals the fp32-bucket session's
+    rounded to bf16, bit for bit (lr = 0: both sessions read the same parameters)."""
+    import torch
+    g = graphs.config_graph("bert_tiny", dtype="f32")
+    G = tsplit.Graph(g)
+    P = tsplit.Plan.default(G)
+    comm = tsplit.nccl_comm(0, 1, lambda b: b)
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    dev = tsplit.inputs_to_device(G, inputs)
+    out = []
+    for bf in (False, True):
+        S = tsplit.Session(G, P, lr=0.0, nccl_comm=comm, world_size=1, grad_allreduce_bf16=bf)
+        S.set_params(params)
+        S.step(dev)
+        out.append(S.grads())
+    for k, v in out[0].items():
+        want = torch.from_numpy(np.asarray(v, np.float32)).to(torch.bfloat16).float().numpy()
+        assert np.array_equal(out[1][k], want), k
+
+
 def _fusion_pair(g, cfg, var="TSPLIT_NO_FUSION", qkv=False):
     """The same step with and without a session fusion: `var` = 1 turns it off.  The
     linear + gelu comparison keeps the q/k/v grouping off in both runs (qkv=False)."""
