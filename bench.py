@@ -16,6 +16,7 @@ bounded samples of the same workload; under torchrun only rank 0 runs it.
 from __future__ import annotations
 
 import argparse
+import collections
 import json
 import os
 import statistics
@@ -44,6 +45,11 @@ WORKLOADS = {
                         metric="samples/sec under HBM budget (IWSLT-shaped Transformer)",
                         model="transformer enc-dec 6+6L h512 a8 ffn2048 s128 vocab32000 (P:L306, f4)", seq_len=128,
                         data="synthetic (uniform source / target ids and next-token labels, random-init weights)"),
+    # f3 / Fig. 6: batch 1 leaves no sample dim; below 65 % only height bands fit (D-ATTR)
+    "vgg16_b1": dict(batch=1, frac=0.45, name="vgg16_b1_i224_budget45",
+                     metric="samples/sec under HBM budget (VGG-16, batch 1: attribute splits)",
+                     model="vgg-16 (13 conv3x3 + 3 fc, 224x224), batch 1",
+                     seq_len=None, data="synthetic (N(0,1) images, uniform labels, Kaiming-normal weights)"),
     "resnet50": dict(batch=256, frac=0.25, name="resnet50_b256_i224_budget25",
                      metric="samples/sec under HBM budget (ResNet-50)", model="resnet-50 v1.5 (224x224)",
                      seq_len=None, data="synthetic (N(0,1) images, uniform labels, Kaiming-normal weights)"),
@@ -54,10 +60,10 @@ def workload_graph(wl, layers=LAYERS, fused=True):
     from tsinputs import graphs
     if wl == "bert_large":
         return graphs.bert(layers=layers, batch=BATCH, fused_attention=fused)
-    return graphs.config_graph(ORACLE_GRAPH.get(wl, wl))
+    return graphs.config_graph(ORACLE_GRAPH.get(wl, wl), **({"batch": 1} if wl == "vgg16_b1" else {}))
 
 
-ORACLE_GRAPH = {"transformer": "transformer_iwslt"}  # bench workload -> graphs.config_graph name
+ORACLE_GRAPH = {"transformer": "transformer_iwslt", "vgg16_b1": "vgg16"}  # bench workload -> graph name
 
 
 def peaks():
@@ -463,7 +469,7 @@ def main():
     lin = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and bt == 1 and kd == 0 and tc]
     att = [(f, ms) for (f, ms, bt), (kd, tc) in zip(recs, kinds) if f > 0 and bt > 1 and tc]
     c_flop, c_ms = sum(f for f, _ in conv), sum(ms for _, ms in conv)
-    cnn = args.workload in ("vgg16", "resnet50")
+    cnn = args.workload in ("vgg16", "vgg16_b1", "resnet50")
     bert = args.workload == "bert_large"
     g_flop, g_ms = sum(f for f, _ in lin), sum(ms for _, ms in lin)
     a_flop, a_ms = sum(f for f, _ in att), sum(ms for _, ms in att)
@@ -518,7 +524,11 @@ def main():
         "budget_frac_of_unsplit_dynamic_peak": args.budget_frac,
         "budget_bytes": budget, "unsplit_peak_bytes": unsplit_peak, "static_bytes": static,
         "plan_peak_extent_bytes": pst["peak_extent"],
-        "plan": {"split_tensors": pst["n_split_tensors"], "swap_tensors": pst["n_swap_tensors"],
+        "plan": {"split_tensors": pst["n_split_tensors"],
+                 "split_dims": dict(collections.Counter(
+                     ("sample", "channel", "height", "width")[c[3]] for c in plan.oracle_cfg().values()
+                     if c[1] > 1 and len(c) > 3)),
+                 "swap_tensors": pst["n_swap_tensors"],
                  "recompute_tensors": pst["n_recompute_tensors"], "replays": pst["n_replay"],
                  "d2h_bytes": pst["d2h_bytes"], "h2d_bytes": pst["h2d_bytes"],
                  "step_flop": pst["compute_flop"], "predicted_ms": pst["predicted_s"] * 1e3,
@@ -527,7 +537,9 @@ def main():
                  "recompute_cache_bytes": pst["recompute_cache_bytes"],
                  "measured_pcie_gbs": [round(x / 1e9, 1) for x in pcie] if pcie else None},
         "l2": "no flush needed: every step streams >10 GB of activations through a 126 MB L2"
-              if bert else "no flush needed: every step streams several GB of activations through a 126 MB L2",
+              if bert else ("no flush needed: every step streams ~2.5 GB of weights (bf16 copies read twice), "
+                            "fp32 gradients and masters through a 126 MB L2" if args.workload == "vgg16_b1" else
+                            "no flush needed: every step streams several GB of activations through a 126 MB L2"),
     }
     if cnn:
         config.pop("seq_len")
