@@ -178,9 +178,6 @@ class Runtime:
             if any(i in self.needs_grad for i in o["inputs"]):
                 aux = AUX_OUTPUTS.get(o["kind"], ())
                 self.needs_grad.update(t for j, t in enumerate(o["outputs"]) if j not in aux)
-        for t, c in cfg.items():
-            if len(c) > 3 and c[3] != 0 and c[1] > 1:
-                raise NotImplementedError("channel-split (D-CH) and band-split (D-ATTR) plans are not exported")
         self.cuda = self.device.type == "cuda"
         if self.cuda:
             self.s_d2h, self.s_h2d = torch.cuda.Stream(self.device), torch.cuda.Stream(self.device)
@@ -189,10 +186,41 @@ class Runtime:
     def p_of(self, t):
         return self.cfg[t][1] if (self.sample[t] and self.ts[t]["kind"] == "act") else 1
 
+    # split dims (DESIGN.md D-CH, D-ATTR): 0 samples, 1 channels (last axis), 2 / 3 height / width bands
+    def dim(self, t):
+        c = self.cfg[t]
+        return c[3] if len(c) > 3 and c[1] > 1 and self.sample[t] and self.ts[t]["kind"] == "act" else 0
+
+    def chan(self, t):
+        return self.dim(t) == 1
+
+    def band(self, t):
+        return self.dim(t) in (2, 3)
+
+    def axis(self, t):  # NHWC array axis of a band split
+        return 1 if self.dim(t) == 2 else 2
+
+    def cmode(self, o):  # channel mode: micro-op k = channel block k of the output, every sample
+        return any(self.chan(t) for t in self.ops[o]["outputs"])
+
+    def amode(self, o):  # attribute mode: micro-op k = band k of the output, every sample
+        return any(self.band(t) for t in self.ops[o]["outputs"])
+
+    def staged(self, o):  # a window op reading its input through a staged rectangle
+        op = self.ops[o]
+        x = op["inputs"][0]
+        return op["kind"] in ("conv2d", "maxpool") and (
+            self.band(x) or self.amode(o) or (op["kind"] == "conv2d" and self.chan(x)))
+
     def P_op(self, o):
+        outs = self.ops[o]["outputs"]
+        if self.cmode(o):
+            return max(self.p_of(t) for t in outs if self.chan(t))
+        if self.amode(o):
+            return max(self.p_of(t) for t in outs if self.band(t))
         P = 1
-        for t in self.ops[o]["inputs"] + self.ops[o]["outputs"]:
-            if self.sample[t]:
+        for t in self.ops[o]["inputs"] + outs:
+            if self.sample[t] and not self.chan(t) and not self.band(t):
                 P = max(P, self.p_of(t))
         return P
 
@@ -201,7 +229,11 @@ class Runtime:
 
     def piece_shape(self, t):
         sh = list(self.ts[t]["shape"])
-        if self.sample[t]:
+        if self.chan(t):
+            sh[-1] //= self.p_of(t)
+        elif self.band(t):
+            sh[self.axis(t)] //= self.p_of(t)
+        elif self.sample[t]:
             sh[0] //= self.p_of(t)
         return sh
 
@@ -240,11 +272,17 @@ class Runtime:
             for i, (kind, op, k, aux) in enumerate(self.items):
                 for key, j in self.allocs[i]:
                     t = key - self.n if key >= self.n else key
-                    if kind == "SI":
+                    if key >= 2 * self.n:  # a staging temporary (D-ATTR): torch allocates its own
+                        self.store[(key, j)] = None
+                    elif kind == "SI":
                         self._swap_in(key, j)
                     else:
                         self.store[(key, j)] = torch.zeros(self.piece_shape(t), dtype=self.tdtype(t), device=dev)
-                if kind in ("F", "R"):
+                special = kind in ("F", "R", "B") and (self.cmode(op) or self.amode(op) or self.staged(op) or any(
+                    self.chan(t) for t in self.ops[op]["inputs"]))
+                if special:
+                    self._split_micro_op(op, k, kind, step)
+                elif kind in ("F", "R"):
                     self._forward(op, k, kind == "R", step)
                 elif kind == "B":
                     self._backward(op, k, step)
@@ -374,6 +412,187 @@ class Runtime:
         if kd == "flatten":
             return x[0].reshape(x[0].shape[0], -1)
         raise NotImplementedError(kd)
+
+    # -- channel (D-CH) and band (D-ATTR) micro-ops -------------------------------
+    def _rect(self, o, k, P):
+        """(rlo, hs, clo, ws, samples) of the input rectangle micro-op k of window op o reads
+        (padding included): what output band k needs along the band's axis, all else."""
+        op, ts = self.ops[o], self.ts
+        y = op["outputs"][0]
+        band = self.band(y)
+        span = []
+        for ax in (1, 2):
+            if op["kind"] == "conv2d":
+                R, s, pad = ts[op["inputs"][1]]["shape"][ax], op["iattrs"][0], op["iattrs"][1]
+            else:
+                R, s, pad = op["iattrs"][0], op["iattrs"][1], op["iattrs"][2]
+            here = band and self.axis(y) == ax
+            hb = ts[y]["shape"][ax] // P if here else ts[y]["shape"][ax]
+            kk = k if here else 0
+            lo = kk * hb * s - pad
+            span += [lo, ((kk + 1) * hb - 1) * s - pad + R - lo]
+        return span[0], span[1], span[2], span[3], (self.B if band else self.B // P)
+
+    def _pieces(self, t, b0, b1, grad=False):
+        """(rows of samples [b0, b1) of each resident piece of t, its index tuple into the
+        whole tensor's rows of those samples) — channel blocks, bands, or the unsplit tensor."""
+        key, al, r = (self.n + t if grad else t), slice(None), self.rows(t)
+        nd = len(self.ts[t]["shape"])
+        if not (self.chan(t) or self.band(t)):
+            return [(self.store[(key, 0)][b0 * r:b1 * r], (al,) * nd)]
+        ax = nd - 1 if self.chan(t) else self.axis(t)
+        w = self.ts[t]["shape"][ax] // self.p_of(t)
+        out = []
+        for j in range(self.p_of(t)):
+            if (key, j) in self.store:
+                sl = [al] * nd
+                sl[ax] = slice(j * w, (j + 1) * w)
+                out.append((self.store[(key, j)][b0 * r:b1 * r], tuple(sl)))
+        return out
+
+    def _gather(self, t, b0, nb, rlo, hs, clo, ws, fill):
+        """The staged rectangle of t: rows [rlo, rlo + hs) x columns [clo, clo + ws) of samples
+        [b0, b0 + nb), fill outside t (the physical merge of Fig. 10)."""
+        H, W, C = self.ts[t]["shape"][1:]
+        pr, pc = max(0, -rlo), max(0, -clo)
+        cv = torch.full((nb, H + pr + max(0, rlo + hs - H), W + pc + max(0, clo + ws - W), C), fill,
+                        dtype=torch.float64 if self.dtype == torch.float64 else torch.float32, device=self.device)
+        inner = cv[:, pr:pr + H, pc:pc + W]
+        for blk, sl in self._pieces(t, b0, b0 + nb):
+            inner[sl] = self.c(blk)
+        return cv[:, rlo + pr:rlo + pr + hs, clo + pc:clo + pc + ws]
+
+    def _scatter(self, t, b0, nb, rlo, hs, clo, ws, g):
+        """Add the staged rectangle's gradient g into t's gradient pieces (padding dropped)."""
+        H, W, C = self.ts[t]["shape"][1:]
+        pr, pc = max(0, -rlo), max(0, -clo)
+        cv = torch.zeros((nb, H + pr + max(0, rlo + hs - H), W + pc + max(0, clo + ws - W), C), dtype=g.dtype,
+                         device=g.device)
+        cv[:, rlo + pr:rlo + pr + hs, clo + pc:clo + pc + ws] = g
+        inner = cv[:, pr:pr + H, pc:pc + W]
+        for blk, sl in self._pieces(t, b0, b0 + nb, grad=True):
+            blk.copy_((self.c(blk) + inner[sl]).to(blk.dtype))
+
+    def _split_micro_op(self, op, k, kind, step):
+        """Micro-op k of an op in channel mode (output channels block k: a linear's / conv's
+        weight rows and bias block k, a channel-local op's block k), in attribute mode (output
+        band k) or of a window op reading bands or channel blocks through a staged rectangle."""
+        o = self.ops[op]
+        kd, ia, fa = o["kind"], list(o["iattrs"]), o["fattrs"]
+        P = self.P_op(op)
+        ins, out = o["inputs"], o["outputs"][0]
+        cm, am, st = self.cmode(op), self.amode(op), self.staged(op)
+        w = self.ts[out]["shape"][-1] // self.p_of(out) if cm else None
+        blk = slice(k * w, (k + 1) * w) if cm else None
+        b0 = 0 if (cm or am) else k * self.B // P
+        nb = self.B if (cm or am) else self.B // P
+        rect = self._rect(op, k, P) if st else None
+        x, sliced = [], set()
+        for i, t in enumerate(ins):
+            if t in self.pval:
+                sliced_here = cm and (kd in ("linear", "conv2d") or kd == "batchnorm")
+                x.append(self.pval[t][blk] if sliced_here else self.pval[t])
+                if sliced_here:
+                    sliced.add(t)
+            elif st and i == 0:
+                x.append(self._gather(t, b0, nb, rect[0], rect[1], rect[2], rect[3],
+                                      float("-inf") if kd == "maxpool" else 0.0))
+            elif (cm or am) and (self.chan(t) or self.band(t)) and kd not in ("linear", "conv2d"):
+                v = self.store.get((t, k))   # (a backward reads only what its op saved)
+                x.append(None if v is None else self.c(v))
+            elif self.chan(t):  # a linear / conv reading every block: merged along the channels
+                x.append(torch.cat([self.c(b) for b, _ in self._pieces(t, b0, b0 + nb)], -1))
+            else:
+                v = self.store[(t, 0)]
+                x.append(self.c(v) if v.dtype.is_floating_point else v)
+        if st:  # the window op runs unpadded on the staged rectangle
+            ia[1 if kd == "conv2d" else 2] = 0
+
+        def bn_stats():
+            xa = self.c(self.whole(ins[0]))
+            ax = tuple(range(xa.dim() - 1))
+            mu = xa.mean(ax)
+            self.bn[op] = (mu, ((xa - mu) ** 2).mean(ax))
+
+        def evaluate(xs):
+            if kd == "batchnorm":
+                if cm:  # block k holds every sample of its channels: its own statistics
+                    mu = xs[0].mean((0, 1, 2))
+                    var = ((xs[0] - mu) ** 2).mean((0, 1, 2))
+                else:
+                    mu, var = self.bn[op]
+                return (xs[0] - mu) / torch.sqrt(var + fa[0]) * xs[1] + xs[2]
+            return self._fwd_op(kd, xs, ia, fa, 0, 0, step)
+
+        if kind in ("F", "R"):
+            if kd == "batchnorm" and am and k == 0 and kind == "F":
+                bn_stats()
+            y = evaluate(x)
+            if cm or am:
+                if (out, k) in self.store:  # (a replay regenerates only its own piece)
+                    self.store[(out, k)].copy_(y)
+            else:
+                self.view(out, b0, b0 + nb).copy_(y)
+            return
+        dy = self.c(self.store[(self.n + out, k)] if (cm or am) else self.view(out, b0, b0 + nb, grad=True))
+        if kd == "batchnorm" and am:  # statistics over every band: the sums of all of dY and X (R13)
+            xin, gid, bid = ins
+            mu, var = self.bn[op]
+            rstd = 1.0 / torch.sqrt(var + fa[0])
+            g = self.pval[gid]
+            if k == 0:
+                dya, xa = self.c(self.whole(out, grad=True)), self.c(self.whole(xin))
+                ax = tuple(range(xa.dim() - 1))
+                xh = (xa - mu) * rstd
+                self.bn[(op, "sums")] = ((dya * g).sum(ax), (dya * g * xh).sum(ax))
+                self.pgrad[gid] += (dya * xh).sum(ax)
+                self.pgrad[bid] += dya.sum(ax)
+            sa, sb = self.bn[(op, "sums")]
+            m = math.prod(self.ts[xin]["shape"][:-1])
+            xh = (x[0] - mu) * rstd
+            grads = {xin: rstd * (dy * g - sa / m - xh * sb / m)}
+        elif kd == "maxpool":
+            grads = {ins[0]: maxpool_bwd(dy, x[0], ia[0], ia[1], ia[2])}
+        elif kd in ("relu", "tanh", "add"):  # these save their output (or nothing)
+            if kd == "add":
+                grads = {}
+                for t in ins:
+                    grads[t] = grads[t] + dy if t in grads else dy
+            else:
+                y = self.c(self.store[(out, k)])
+                grads = {ins[0]: dy * (y > 0) if kd == "relu" else dy * (1.0 - y * y)}
+        else:
+            leaves = {}
+            xs = []
+            for t, v in zip(ins, x):
+                if v.dtype.is_floating_point and t in self.needs_grad:
+                    v = v.detach().requires_grad_(True)
+                    leaves[t] = v
+                xs.append(v)
+            with torch.enable_grad():
+                y = evaluate(xs)
+                order = list(leaves)
+                gs = torch.autograd.grad(y, [leaves[t] for t in order], grad_outputs=dy, allow_unused=True)
+            grads = {t: g for t, g in zip(order, gs) if g is not None}
+        for i, t in enumerate(ins):
+            g = grads.get(t)
+            if g is None:
+                continue
+            if t in self.pgrad:
+                if t in sliced:
+                    self.pgrad[t][blk] += g.to(self.pgrad[t].dtype)
+                else:
+                    self.pgrad[t] += g.to(self.pgrad[t].dtype)
+            elif t not in self.needs_grad or self.ts[t]["kind"] != "act":
+                continue
+            elif st and i == 0:
+                self._scatter(t, b0, nb, rect[0], rect[1], rect[2], rect[3], g)
+            elif (cm or am) and (self.chan(t) or self.band(t)) and kd not in ("linear", "conv2d"):
+                v = self.store[(self.n + t, k)]
+                v.copy_((self.c(v) + g).to(v.dtype))
+            else:  # a linear / conv reading every block (or the unsplit tensor): dX of its samples
+                for blk_, sl in self._pieces(t, b0, b0 + nb, grad=True):
+                    blk_.copy_((self.c(blk_) + g[sl]).to(blk_.dtype))
 
     def _acc(self, t, s0, s1, g):
         if t in self.pgrad:

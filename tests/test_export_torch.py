@@ -62,14 +62,32 @@ def test_exported_step_equals_the_oracle(case, seed, tmp_path):
     assert max(errs.values()) <= 1e-12, sorted(errs.items(), key=lambda kv: -kv[1])[:3]
 
 
-def test_export_rejects_channel_plans(tmp_path):
-    g = graphs.mlp()
-    names = {t["name"]: t["id"] for t in g["tensors"]}
+SPLIT_CASES = [("mlp", "chan2"), ("bert_tiny", "chan2"), ("vgg_tiny", "band"), ("resnet_tiny", "band"),
+               ("vgg_tiny", "chan4"), ("resnet_tiny", "chan4")]
+
+
+@pytest.mark.parametrize("case", range(len(SPLIT_CASES)))
+def test_exported_channel_and_band_plans_equal_the_oracle(case, tmp_path):
+    """Channel (D-CH: 2-D and image blocks) and height / width band (D-ATTR: staged halo
+    rectangles) plans exported to torch: the fp64 module equals the fp64 oracle."""
+    from test_oracle_attr import _rand_attr_cfg
+    from test_oracle_channel import CHAINS, channel_cfg
+    from test_oracle_channel4 import rand_chan4_cfg
+    name, kind = SPLIT_CASES[case]
+    g = graphs.config_graph(name, **({} if name == "mlp" else {"dtype": "f32"}))
+    r = random.Random(40 + case)
+    cfg = (channel_cfg(g, r, CHAINS[name], prob=0.9) if kind == "chan2" else
+           _rand_attr_cfg(g, r) if kind == "band" else rand_chan4_cfg(g, r))
     G = tsplit.Graph(g)
     P = tsplit.Plan.default(G)
-    P.set_many({names["fc0"]: (0, 2, 1, 1), names["relu0"]: (0, 2, 1, 1)})
-    with pytest.raises(NotImplementedError):
-        export.export_torch(G, P, str(tmp_path / "x.py"))
+    P.set_many({t: cfg[t] for t in brute.act_tensors(g)})
+    mod = _load(export.export_torch(G, P, str(tmp_path / f"split_{case}.py")))
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    loss, grads = mod.AugmentedStep("cpu", torch.float64)(params, inputs)
+    ol, og, _, _ = net.train_step(g, params, inputs)
+    assert abs(loss - ol) <= 1e-12 * abs(ol)
+    errs = rel_errs({k: v.numpy() for k, v in grads.items()}, og)
+    assert max(errs.values()) <= 1e-12, sorted(errs.items(), key=lambda kv: -kv[1])[:3]
 
 
 @pytest.mark.gpu
