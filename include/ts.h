@@ -191,9 +191,12 @@ void ts_profile_destroy(ts_profile_t* pr);
  * one cudaEvent-timed eager step of the all-reside plan with every activation split p
  * ways, on the caller's scratch `slab` (device, >= the unsplit peak; parameters are
  * zero — op times do not depend on the data), and records each op's forward
- * and backward time (per-item median of three timed steps).  p values above max_p or
- * the batch (p must divide it) extrapolate from the widest measured one (+5 % per
- * doubling: the launch / tail overhead of one more level of micro-ops).  Also measures pinned
+ * and backward time (per-item median of three timed steps).  A p the batch does not divide
+ * (the sample dim exhausted, Fig. 6) is timed with height bands instead (reading D-ATTR:
+ * every group of 4-D activations that can take p bands legally; the ops it splits get that
+ * width's times, staging copies included).  p values above max_p, or that no split reaches,
+ * extrapolate from the widest measured one (+5 % per doubling: the launch / tail overhead
+ * of one more level of micro-ops).  Also measures pinned
  * D2H/H2D bandwidth (256 MiB copies).  `inputs` as in ts_step. */
 ts_status ts_profile_measure(const ts_graph_t* g, void* slab, uint64_t slab_bytes, const void* const* inputs,
                              int32_t inputs_on_host, int32_t max_p, ts_profile_t** out);

@@ -1794,12 +1794,55 @@ ts_status ts_profile_measure(const ts_graph_t* gh, void* slab, uint64_t slab_byt
   int dev = 0;
   cudaGetDevice(&dev);
   for (int p = 1; p <= 16 && p <= max_p; p *= 2) {
-    if (g.samples % p) break;
     ts_plan_t plan;
     plan.graph = &g;
     plan.st.cfg.assign(g.n(), Cfg());
-    for (auto& t : g.t)
-      if (t.kind == TS_ACT && !t.is_loss) plan.st.cfg[t.id].p = p;
+    const bool bands = g.samples % p != 0;
+    if (!bands) {
+      for (auto& t : g.t)
+        if (t.kind == TS_ACT && !t.is_loss) plan.st.cfg[t.id].p = p;
+    } else {
+      // the sample dim is exhausted (Fig. 6): time the ops at p height bands instead (D-ATTR),
+      // each group of 4-D activations tied by band-local ops split together when legal
+      std::vector<int> grp_of(g.n(), -1);
+      std::vector<std::vector<int>> grps;
+      auto local = [](int kind) { return kind == TS_OP_RELU || kind == TS_OP_ADD || kind == TS_OP_BATCHNORM; };
+      for (auto& t : g.t) {
+        if (t.kind != TS_ACT || t.ndim != 4 || grp_of[t.id] >= 0) continue;
+        std::vector<int> grp{t.id};
+        grp_of[t.id] = int(grps.size());
+        for (size_t q = 0; q < grp.size(); ++q) {
+          const Tensor& u = g.t[grp[q]];
+          std::vector<int> nb;
+          if (u.producer >= 0 && local(g.ops[u.producer].kind))
+            for (int v : g.ops[u.producer].in) if (g.t[v].kind == TS_ACT) nb.push_back(v);
+          for (int c : u.consumers)
+            if (local(g.ops[c].kind)) nb.push_back(g.ops[c].out[0]);
+          for (int v : nb)
+            if (grp_of[v] < 0) {
+              grp_of[v] = grp_of[t.id];
+              grp.push_back(v);
+            }
+        }
+        grps.push_back(grp);
+      }
+      std::string why;
+      int nband = 0;
+      for (auto& grp : grps) {
+        std::vector<Cfg> trial = plan.st.cfg;
+        bool ok = true;
+        for (int u : grp) {
+          if (g.t[u].shape[1] % p) ok = false;
+          trial[u].p = p;
+          trial[u].dim = 2;
+        }
+        if (ok && attr_ok(g, trial, why) && channel_ok(g, trial, why)) {
+          plan.st.cfg = trial;
+          ++nband;
+        }
+      }
+      if (!nband) break;
+    }
     plan_refresh(g, plan.st, nullptr);
     if (plan.st.sim.peak_extent > slab_bytes) continue;  // does not fit the scratch slab
     ts_session_cfg sc;
@@ -1840,6 +1883,7 @@ ts_status ts_profile_measure(const ts_graph_t* gh, void* slab, uint64_t slab_byt
     int l = 0;
     while ((1 << l) < p) ++l;
     for (size_t o = 0; o < g.ops.size(); ++o) {
+      if (bands && plan.st.ex.P[o] != p) continue;  // (an op the band plan leaves whole)
       prof->pr.tf[o][l] = tf[o];
       prof->pr.tb[o][l] = tb[o];
       // untested wider splits extrapolate from the widest measured one (per-micro-op overhead kept)
