@@ -124,3 +124,20 @@ def test_vgg16_batch1_planned_band_step(dtype):
     else:
         assert abs(loss - l0) <= 1e-3 * abs(l0)
         assert global_rel_err(grads, g0) <= 1e-2
+
+
+def test_profile_measures_band_widths_at_batch_one():
+    """ts_profile_measure at batch 1 (no sample split possible): the widths p = 2, 4 are timed
+    with height bands — the conv ops get measured, not extrapolated, times (the +5 %-per-
+    doubling extrapolation would give exactly 1.05 / 1.10 x the p = 1 time), and a band
+    micro-op over a quarter of one image costs more than a quarter of the whole op."""
+    g = graphs.config_graph("vgg16", batch=1)
+    G = tsplit.Graph(g)
+    pr = tsplit.Profile.measure(G, tsplit.inputs_to_device(G, gen.make_inputs(g)), max_p=4)
+    convs = [o["id"] for o in g["ops"] if o["kind"] == "conv2d"][1:4]
+    for o in convs:
+        f1, _ = pr.get(o, 1)
+        f2, _ = pr.get(o, 2)
+        f4, _ = pr.get(o, 4)
+        assert f1 > 0 and abs(f2 / f1 - 1.05) > 1e-6 and abs(f4 / f1 - 1.10) > 1e-6, (o, f1, f2, f4)
+        assert f4 > f1 * 0.25
