@@ -141,3 +141,30 @@ def test_profile_measures_band_widths_at_batch_one():
         f4, _ = pr.get(o, 4)
         assert f1 > 0 and abs(f2 / f1 - 1.05) > 1e-6 and abs(f4 / f1 - 1.10) > 1e-6, (o, f1, f2, f4)
         assert f4 > f1 * 0.25
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+def test_bands_no_window_reaches_are_zero_on_the_gpu(dtype):
+    """The stride-2 case of tests/test_oracle_attr.py: band 7 of relu's gradient has no writer
+    (allocated by relu's backward, which reads it) and must read as zeros."""
+    from test_oracle_attr import stride2_graph
+    g, cfg = stride2_graph(dtype)
+    G = tsplit.Graph(g)
+    P = tsplit.Plan.default(G)
+    P.set_many({t: cfg[t] for t in brute.act_tensors(g)})
+    S = tsplit.Session(G, P)
+    # poison the dynamic pool (the static region was zeroed by the session): a gradient piece
+    # nobody zeroes would read ~3e38
+    S.slab[P.stats()["static_bytes"]:].fill_(0x7F)
+    params, inputs = gen.init_params(g), gen.make_inputs(g)
+    S.set_params(params)
+    S.step(tsplit.inputs_to_device(G, inputs))
+    grads = S.grads()
+    l0, g0, _, _ = _run(g)
+    ol, og, _, _ = net.train_step(g, params, inputs)
+    if dtype == "f32":
+        assert max(rel_errs(grads, og).values()) <= 1e-5
+        assert max(rel_errs(grads, g0).values()) <= 3e-6
+    else:
+        assert global_rel_err(grads, g0) <= 1e-2
+    assert S.trace() == [tuple(e) for e in sim.simulate(g, cfg).trace]

@@ -190,3 +190,47 @@ def test_band_split_legality():
     cfg3[byname["relu0"]] = (0, 3, 1, 2)
     with pytest.raises(ValueError):
         sim.expand(g, cfg3)
+
+
+def stride2_graph(dtype="f32"):
+    """X [2, 8, 8, 8] -> conv a 3x3 / 1 -> relu -> conv b 1x1 / 2 -> flatten -> fc -> loss: with
+    relu's output in 8 one-row bands, conv b (unsplit output: a full merge) stages rows 0 .. 6
+    (and reads only the even ones), so band 7 is staged by no micro-op: its gradient is zero
+    without any writer."""
+    b = graphs.GraphBuilder("vgg_stride2", dtype, 2)  # (CNN parameter recipe)
+    X = b.tensor("X", (2, 8, 8, 8), "input")
+    Y = b.tensor("labels", (2,), "label", dtype="i32")
+    Wa, ba = b.param("Wa", (8, 3, 3, 8)), b.param("ba", (8,))
+    Wb, bb = b.param("Wb", (8, 1, 1, 8)), b.param("bb", (8,))
+    Wf, bf = b.param("Wf", (3, 128)), b.param("bf", (3,))
+    a = b.op("conv2d", "conv_a", [X, Wa, ba], (2, 8, 8, 8), iattrs=[1, 1])
+    r = b.op("relu", "relu", [a], (2, 8, 8, 8))
+    c = b.op("conv2d", "conv_b", [r, Wb, bb], (2, 4, 4, 8), iattrs=[2, 0])
+    f = b.op("flatten", "flat", [c], (2, 128))
+    y = b.op("linear", "fc", [f, Wf, bf], (2, 3))
+    b.op("xent", "loss", [y, Y], (1,), out_dtype="f32")
+    g = b.done()
+    cfg = sim.default_cfg(g)
+    cfg[a] = (sim.RESIDE, 8, 1, 2)
+    cfg[r] = (sim.RESIDE, 8, 1, 2)
+    return g, cfg
+
+
+def test_bands_no_window_reaches_have_zero_gradient():
+    g, cfg = stride2_graph()
+    items, fa, ff, _, an = sim.expand(g, cfg)
+    n = len(g["tensors"])
+    conv_b = next(o["id"] for o in g["ops"] if o["name"] == "conv_b")
+    relu = next(t["id"] for t in g["tensors"] if t["name"] == "relu")
+    written = {j for it in items if it.kind == "B" and it.op == conv_b for (key, j) in it.writes if key == n + relu}
+    assert written == set(range(7))   # the staged rectangle spans rows 0..6: band 7 is unread
+    reads = {j for it in items if it.kind == "F" and it.op == conv_b for (key, j) in it.reads if key == relu}
+    assert reads == set(range(7))
+    # drelu.7 is first touched by relu's backward reading it: allocated as zeros
+    b_relu = [it for it in items if it.kind == "B" and g["ops"][it.op]["name"] == "relu"]
+    assert {j for it in b_relu for (key, j) in it.reads if key == n + relu} == set(range(8))
+    P, I = gen.init_params(g), gen.make_inputs(g)
+    loss, pg, _, _ = net.train_step(g, P, I)
+    l2, pg2 = execplan.execute(g, cfg, P, I)
+    assert abs(l2 - loss) <= 1e-12 * abs(loss)
+    assert max(rel_errs(pg2, pg).values()) <= 1e-12
