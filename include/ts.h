@@ -368,6 +368,15 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch,
  * the per-group fallback rounds the running sum to bf16 after every group (the grouped
  * launch rounds once).  TS_ERR_ARG for bad groups / gdim, a grouped extent (N, K or M)
  * that `groups` does not divide, or beta other than 0 / 1. */
+/* Fused-epilogue product (the session's linear -> gelu / gelu' peepholes, reading
+ * D-FUSE), bf16 row-major operands as ts_gemm_bf16 with batch 1, bf16 C, beta 0:
+ *   epi 1: C = U = alpha A op(B) + bias, aux = gelu(bf16(U))            (aux written)
+ *   epi 2: C = dU = bf16(alpha A op(B)) * gelu'(aux), aux = U            (aux read)
+ * aux is [M, N] row-major with leading dimension ldaux (elements).  TS_ERR_ARG for an
+ * epi other than 1 / 2 or a shape / alignment the tcgen05 TMA-store path cannot take. */
+ts_status ts_gemm_bf16_epi(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t lda, int32_t ta,
+                           const void* B, int64_t ldb, int32_t tb, void* C, int64_t ldc, float alpha,
+                           const void* bias_bf16, void* aux, int64_t ldaux, void* stream);
 /* Row kernels for unit tests / microbenchmarks: op 0 = bias-gradient column sum,
  * out[j] (+)= sum_r x[r, j] over a [rows, n] row-major tensor (fp32 out; ws: device
  * workspace of ws_bytes >= 8 KB, its last 4 KB hold completion tickets that must start

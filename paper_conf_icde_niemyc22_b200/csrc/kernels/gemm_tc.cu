@@ -64,15 +64,18 @@ struct TmSet {
 };
 // epilogue staging: per warp, 32x32 output blocks (two for bf16; one for fp32, whose
 // products have long K and keep the smem for a deeper operand pipeline)
-template <bool F32OUT, int EW>
-constexpr int staging_nbuf() { return (!F32OUT && EW == 8) ? 2 : 1; }
+// (the 16-warp fused epilogues double-buffer too when the CTA stages at most 128 B rows — a CTA
+// pair's half tile — so the smem still holds five operand stages: U's store then never waits
+// for the previous store's smem read before gelu(U) is staged)
+template <bool F32OUT, int EW, int BNL>
+constexpr int staging_nbuf() { return (!F32OUT && (EW == 8 || BNL <= 128)) ? 2 : 1; }
 constexpr int kSmemLimit = 232448;  // 227 KB opt-in dynamic shared memory per CTA
-template <bool F32OUT, int EW>
-constexpr int staging_bytes() { return EW * staging_nbuf<F32OUT, EW>() * 32 * 32 * (F32OUT ? 4 : 2); }
+template <bool F32OUT, int EW, int BNL>
+constexpr int staging_bytes() { return EW * staging_nbuf<F32OUT, EW, BNL>() * 32 * 32 * (F32OUT ? 4 : 2); }
 template <int BN, bool F32OUT, int EW>
 constexpr int num_stages() {
   constexpr int stage = (BM + BN) * BK * 2;
-  constexpr int n = (kSmemLimit - staging_bytes<F32OUT, EW>() - 2048) / stage;
+  constexpr int n = (kSmemLimit - staging_bytes<F32OUT, EW, BN>() - 2048) / stage;
   return n > 8 ? 8 : n;
 }
 
@@ -305,7 +308,7 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
     const int ew = warp - 2;       // epilogue warp index
     const int half = ew >> 2;      // column group: chunks half, half + kGrp, ... of each tile
     constexpr int kGrp = EW / 4;
-    constexpr int NBUF = staging_nbuf<F32OUT, EW>();
+    constexpr int NBUF = staging_nbuf<F32OUT, EW, BNL>();
     uint8_t* wbuf = cstage + ew * NBUF * BUF;
     int nbuf = 0;
     int acc = 0;
@@ -405,8 +408,9 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
               if constexpr (F32OUT) {
 #pragma unroll
                 for (int j = 0; j < 8; ++j) {  // 128 B row, SWIZZLE_128B
-                  float4 o = make_float4(vals[4 * j], vals[4 * j + 1], vals[4 * j + 2], vals[4 * j + 3]);
-                  *reinterpret_cast<float4*>(buf + lane * 128 + ((j ^ (lane & 7)) << 4)) = o;
+                  st_shared_v4(smem_u32(buf + lane * 128 + ((j ^ (lane & 7)) << 4)), __float_as_uint(vals[4 * j]),
+                               __float_as_uint(vals[4 * j + 1]), __float_as_uint(vals[4 * j + 2]),
+                               __float_as_uint(vals[4 * j + 3]));
                 }
               } else {
 #pragma unroll
@@ -416,7 +420,7 @@ __global__ void __launch_bounds__(num_threads<EW>(), 1)
 #pragma unroll
                   for (int h = 0; h < 4; ++h)
                     o2[h] = __floats2bfloat162_rn(vals[8 * j + 2 * h], vals[8 * j + 2 * h + 1]);
-                  *reinterpret_cast<uint4*>(buf + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4)) = o;
+                  st_shared_v4(smem_u32(buf + lane * 64 + ((j ^ ((lane >> 1) & 3)) << 4)), o.x, o.y, o.z, o.w);
                 }
               }
               fence_async_smem();
@@ -544,7 +548,7 @@ GemmConfig g_last{};
 template <int BN, bool F32OUT, int EW = 8, int CG = 1>
 void launch(const TmSet& tm, const TcParams& p, cudaStream_t st) {
   constexpr int STAGE = (BM + BN / CG) * BK * 2;
-  const int smem = num_stages<BN / CG, F32OUT, EW>() * STAGE + 1024 + staging_bytes<F32OUT, EW>() + 1024;
+  const int smem = num_stages<BN / CG, F32OUT, EW>() * STAGE + 1024 + staging_bytes<F32OUT, EW, BN / CG>() + 1024;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(gemm_tc_kernel<BN, F32OUT, EW, CG>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
@@ -575,7 +579,7 @@ void launch(const TmSet& tm, const TcParams& p, cudaStream_t st) {
 // number of 2-CTA clusters of the pair kernel that fit on the device at once
 int query_pair_slots() {
   constexpr int STAGE = (BM + 128) * BK * 2;
-  const int smem = num_stages<128, false, 8>() * STAGE + 1024 + staging_bytes<false, 8>() + 1024;
+  const int smem = num_stages<128, false, 8>() * STAGE + 1024 + staging_bytes<false, 8, 128>() + 1024;
   cudaFuncSetAttribute(gemm_tc_kernel<256, false, 8, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(g_num_sms);

@@ -1998,6 +1998,24 @@ ts_status ts_gemm_bf16(int32_t M, int32_t N, int32_t K, int32_t batch, const voi
   return TS_OK;
 }
 
+ts_status ts_gemm_bf16_epi(int32_t epi, int32_t M, int32_t N, int32_t K, const void* A, int64_t lda, int32_t ta,
+                           const void* B, int64_t ldb, int32_t tb, void* C, int64_t ldc, float alpha,
+                           const void* bias, void* aux, int64_t ldaux, void* stream) {
+  if (epi != 1 && epi != 2) return set_error("gemm epi: epi must be 1 (gelu) or 2 (gelu')"), TS_ERR_ARG;
+  if (!aux) return set_error("gemm epi: aux required"), TS_ERR_ARG;
+  tsk::GemmArgs g;
+  g.M = M; g.N = N; g.K = K; g.in_dtype = tsk::BF16;
+  g.a = {A, lda, ta != 0, 0, 0};
+  g.b = {B, ldb, tb != 0, 0, 0};
+  g.c = C; g.ldc = ldc; g.c_dtype = tsk::BF16;
+  g.alpha = alpha; g.beta = 0.f; g.bias = bias; g.bias_dtype = tsk::BF16;
+  g.epi = epi; g.aux = aux; g.ldaux = ldaux;
+  if (!tsk::gemm_tc(g, static_cast<cudaStream_t>(stream)))
+    return set_error("gemm epi: shape/alignment not eligible for the tcgen05 TMA-store path"), TS_ERR_ARG;
+  CU(cudaGetLastError());
+  return TS_OK;
+}
+
 ts_status ts_gemm_bf16_grouped(int32_t groups, int32_t gdim, int32_t M, int32_t N, int32_t K,
                                const void* const* A, int64_t lda, int32_t ta, const void* const* B, int64_t ldb,
                                int32_t tb, void* const* C, int64_t ldc, int32_t c_dtype, float alpha, float beta,

@@ -138,6 +138,8 @@ def lib():
                                    vp, i64, i64, i32, C.c_float, C.c_float, vp, vp]),
             "ts_gemm_bf16_grouped": (i32, [i32, i32, i32, i32, i32, P(vp), i64, i32, P(vp), i64, i32, P(vp), i64,
                                            i32, C.c_float, C.c_float, P(vp), vp]),
+            "ts_gemm_bf16_epi": (i32, [i32, i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, vp, vp,
+                                       i64, vp]),
             "ts_gemm_set_mode": (i32, [i32]),
             "ts_gemm_last_config": (i32, [P(i32)]),
             "ts_gemm_f32": (i32, [i32, i32, i32, vp, i64, i32, vp, i64, i32, vp, i64, C.c_float, C.c_float,

@@ -97,7 +97,9 @@ def test_ranks_draw_disjoint_dropout_masks():
         S.step(dev)
         out.append(S.grads())
         del S
-    assert max(rel_errs(out[1], out[0]).values()) <= 1e-9  # (fp32 atomics of the word table)
+    # equal offsets: identical except the word-table gradient, whose fp32 atomicAdd order varies
+    # from run to run (measured up to 8e-9 relative)
+    assert max(rel_errs(out[1], out[0]).values()) <= 1e-7
     assert max(rel_errs(out[2], out[0]).values()) > 1e-3
 
 

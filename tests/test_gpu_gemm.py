@@ -201,3 +201,31 @@ def test_bias_column_sum(rows, n, dtype):
     tsplit.column_sum(x, again, ws, acc=1)
     torch.cuda.synchronize()
     assert torch.equal(2 * out, again) or float((again.double() - 2 * ref).abs().max() / scale) < 2e-6
+
+
+@pytest.mark.parametrize("mode", [0, 1, 2])
+@pytest.mark.parametrize("M,N,K", [(1024, 4096, 1024), (384, 1024, 4096), (256, 192, 320)])
+def test_gemm_tc_fused_gelu_epilogues(M, N, K, mode, gemm_mode):
+    """ts_gemm_bf16_epi (reading D-FUSE): epi 1 writes U = A B^T + bias and gelu(bf16(U));
+    epi 2 writes dU = bf16(A B^T) * gelu'(U) — against torch's exact erf GELU in fp32."""
+    gemm_mode(mode)
+    A, B, bias = _mk((M, K), seed=3), _mk((N, K), seed=4), _mk((N,), seed=5)
+    U = torch.empty(M, N, device="cuda", dtype=torch.bfloat16)
+    H = torch.empty_like(U)
+    tsplit.check(tsplit.lib().ts_gemm_bf16_epi(1, M, N, K, A.data_ptr(), K, 0, B.data_ptr(), K, 0, U.data_ptr(), N,
+                                               1.0, bias.data_ptr(), H.data_ptr(), N, None))
+    torch.cuda.synchronize()
+    u_ref = A.float() @ B.float().t() + bias.float()
+    assert ((U.float() - u_ref).norm() / u_ref.norm()).item() < 8e-3
+    h_ref = torch.nn.functional.gelu(U.float())  # from the stored bf16 U, as the kernel does
+    assert ((H.float() - h_ref).norm() / h_ref.norm()).item() < 8e-3
+    dU = torch.empty_like(U)
+    tsplit.check(tsplit.lib().ts_gemm_bf16_epi(2, M, N, K, A.data_ptr(), K, 0, B.data_ptr(), K, 0, dU.data_ptr(), N,
+                                               1.0, None, U.data_ptr(), N, None))
+    torch.cuda.synchronize()
+    x = U.float().requires_grad_()
+    torch.nn.functional.gelu(x).backward(torch.ones_like(x))
+    du_ref = (A.float() @ B.float().t()).bfloat16().float() * x.grad
+    assert ((dU.float() - du_ref).norm() / du_ref.norm()).item() < 8e-3
+    assert tsplit.lib().ts_gemm_bf16_epi(3, M, N, K, A.data_ptr(), K, 0, B.data_ptr(), K, 0, dU.data_ptr(), N, 1.0,
+                                         None, U.data_ptr(), N, None) == tsplit.STATUS.index("ERR_ARG")
