@@ -203,6 +203,8 @@ constexpr uint32_t kPlanNoLag = 1u << 30;
 // the greedy without candidates)
 ts_status plan_greedy_lag(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps, uint32_t flags = 0);
 void plan_refine(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps);
+// D-LRU post-pass: the recompute cache limit the timeline predicts fastest within `budget`
+void plan_lru(const Graph& g, uint64_t budget, const Profile& pr, PlanState& ps);
 
 }  // namespace ts
 

@@ -1,19 +1,13 @@
-// Fused attention forward on the 5th-generation tensor cores (sm_100a), head dim 64,
-// seq a multiple of 128 up to 512 (BERT-Large / scaled BERT) — the same arithmetic as
-// attention.cu's kernels (dropout reading D-RNG).
-//
-// One CTA = 128 queries of one (sample, head).  The whole score row fits TMEM
-// (128 lanes x seq fp32 columns <= 512), so the softmax is exact, not online:
-//   1. one thread issues TMA loads of Q (128 x 64), K and V (seq x 64) into 128B-swizzled
-//      shared memory and the tcgen05.mma products S = Q K^T into TMEM;
-//   2. eight softmax warps (two per TMEM lane quarter, each owning half of the keys)
-//      read S with tcgen05.ld, take the row max (exchanged through shared memory),
-//      form P = exp2(S*alpha*log2e - max) with the Philox keep mask — a thread owns a
-//      row, so one Philox call covers four consecutive keys — and store bf16 P in the
-//      K-major UMMA layout over the dead K / Q buffers;
-//   3. as each key half lands, O += P_half V_half runs on the tensor cores (V is the
-//      MN-major B operand straight from its TMA tile) into TMEM columns 0..63;
-//   4. the first four warps scale O by 1 / (rowsum (1-p)), write C and the log-sum-exp.
+// Fused attention on the 5th-generation tensor cores (sm_100a), head dim 64, seq a multiple
+// of 128 — the same arithmetic as attention.cu's kernels (dropout reading
+// D-RNG), so the [b, a, s, s] score / probability / dropout tensors are never materialised
+// (P:L119).  Three persistent warp-specialised kernels, each with TMA-fed operands in
+// 128B-swizzled shared memory, tcgen05.mma issued by one thread and TMEM accumulators:
+//   * fa5_fwd: online softmax over 64-key chunks (thresholded running max), O = P V, the row
+//     log-sum-exp and the dropout keep bits (Philox on the softmax warps);
+//   * fa5_bwd_dq: dQ per 128-query tile (P rebuilt from S and the log-sum-exp, keep bits read);
+//   * fa5_bwd_dkv: dK, dV per 128-key tile.
+// Each kernel's layout and pipeline is described above it.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 
@@ -291,19 +285,23 @@ __global__ void __launch_bounds__(kDqThreads, 1)
     int it = 0, kc = 0;
     // the row's D (attn_row_dot) and raw lse, loaded one item ahead (the loads complete while
     // the current item computes; nothing waits on them until the next item starts)
-    auto item_consts = [&](int itm, float& D_, float& lse_) {
+    // (row index of (sample, head) ah = b * heads + a: hr = ah * S + query)
+    auto row_of = [&](int itm) {
       const int qt_ = itm % nqt, ah_ = itm / nqt;
-      const int64_t hr = (int64_t(ah_ / p.heads) * p.heads + ah_ % p.heads) * S + qt_ * 128 + i;
+      return int64_t(ah_) * S + qt_ * 128 + i;
+    };
+    auto item_consts = [&](int itm, float& D_, float& lse_) {
+      const int64_t hr = row_of(itm);
       D_ = p.D[hr];
       lse_ = p.lse[hr];
     };
     float nD = 0.f, nlse = 0.f;
     // keep word of (item, key tile kt) for this row and 32-key group, loaded a tile ahead
+    int64_t khr = 0;  // row of the item whose keep words load next
     auto keep_word = [&](int itm, int kt_) -> uint32_t {
       if (!p.drop) return ~0u;
-      const int qt_ = itm % nqt, ah_ = itm / nqt;
-      const int64_t hr = (int64_t(ah_ / p.heads) * p.heads + ah_ % p.heads) * S + qt_ * 128 + i;
-      return p.mask[hr * (S / 32) + kt_ * 4 + cg];
+      if (kt_ == 0) khr = row_of(itm);
+      return p.mask[khr * (S / 32) + kt_ * 4 + cg];
     };
     uint32_t nbits = ~0u;
     if (int(blockIdx.x) < items) {
@@ -507,9 +505,16 @@ __global__ void __launch_bounds__(kKvThreads, 1)
     const uint32_t pd = smem_u32(smem + kKvSmemPd), ds = smem_u32(smem + kKvSmemDS);
     int it = 0, qc = 0;
     // row constants (raw lse, D, keep word) of query tile t of a work item
+    // (row index of (sample, head) ah = b * heads + a: hr = ah * S + query; one division per
+    // work item — the per-tile integer divisions were a twentieth of this kernel's stall samples)
+    int nah = 0, nkt_ = 0;  // (sample, head) and key tile of the item whose constants load next
     auto row_consts = [&](int itm, int t, float& lse_, float& D_, uint32_t& bits_) {
-      const int kt_ = itm % nkt, ah_ = itm / nkt;
-      const int64_t hr = (int64_t(ah_ / p.heads) * p.heads + ah_ % p.heads) * S + t * 128 + i;
+      if (t == 0) {
+        nkt_ = itm % nkt;
+        nah = itm / nkt;
+      }
+      const int kt_ = nkt_;
+      const int64_t hr = int64_t(nah) * S + t * 128 + i;
       lse_ = p.lse[hr];
       D_ = p.D[hr];
       bits_ = p.drop ? p.mask[hr * (S / 32) + kt_ * 4 + cg] : ~0u;

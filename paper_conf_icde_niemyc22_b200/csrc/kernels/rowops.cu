@@ -84,22 +84,17 @@ __global__ void __launch_bounds__(kWarps * 32) ln_fwd_kernel(const T* __restrict
   }
 }
 
-// bf16 LayerNorm forward at HBM rate: a persistent grid (~2 blocks per SM), gamma/beta held
-// packed in registers, and every warp loads its next row before normalising the current one
-// (two rows of loads in flight), one row per warp at a time held in registers.
+// bf16 LayerNorm forward at HBM rate: a persistent grid (3 blocks per SM), every warp loads
+// its next row before normalising the current one (two rows of loads in flight per warp, 24
+// warps per SM), gamma / beta read from L1 at use (they are 4 KB, and holding them packed in
+// registers would cost a third of the warps an SM keeps loading).
 template <int NCH>
-__global__ void __launch_bounds__(256) ln_fwd_bf16(const bf16* __restrict__ x, const bf16* __restrict__ g,
+__global__ void __launch_bounds__(256, 3) ln_fwd_bf16(const bf16* __restrict__ x, const bf16* __restrict__ g,
                                                    const bf16* __restrict__ b, bf16* __restrict__ y, int64_t rows,
                                                    int H, float eps) {
   const int lane = threadIdx.x & 31;
   const float invH = 1.f / float(H);
-  uint4 gv[NCH], bv[NCH], cur[NCH];
-#pragma unroll
-  for (int c = 0; c < NCH; ++c) {
-    const int col = (c * 32 + lane) * 8;
-    gv[c] = col < H ? *reinterpret_cast<const uint4*>(g + col) : make_uint4(0, 0, 0, 0);
-    bv[c] = col < H ? *reinterpret_cast<const uint4*>(b + col) : make_uint4(0, 0, 0, 0);
-  }
+  uint4 cur[NCH];
   const int64_t stride = int64_t(gridDim.x) * 8;
   int64_t r = int64_t(blockIdx.x) * 8 + (threadIdx.x >> 5);
   auto load = [&](int64_t row, uint4 (&v)[NCH]) {
@@ -141,8 +136,9 @@ __global__ void __launch_bounds__(256) ln_fwd_bf16(const bf16* __restrict__ x, c
       const int col = (c * 32 + lane) * 8;
       if (col < H) {
         const __nv_bfloat162* hx = reinterpret_cast<const __nv_bfloat162*>(&cur[c]);
-        const __nv_bfloat162* hg = reinterpret_cast<const __nv_bfloat162*>(&gv[c]);
-        const __nv_bfloat162* hb = reinterpret_cast<const __nv_bfloat162*>(&bv[c]);
+        const uint4 gu = __ldg(reinterpret_cast<const uint4*>(g + col)), bu = __ldg(reinterpret_cast<const uint4*>(b + col));
+        const __nv_bfloat162* hg = reinterpret_cast<const __nv_bfloat162*>(&gu);
+        const __nv_bfloat162* hb = reinterpret_cast<const __nv_bfloat162*>(&bu);
         uint4 o;
         __nv_bfloat162* ho = reinterpret_cast<__nv_bfloat162*>(&o);
 #pragma unroll
@@ -910,7 +906,7 @@ void ln_fwd_t(const void* x, const void* g, const void* b, void* y, int64_t rows
   auto Y = (T*)y;
   int grid = grid_rows(rows);
   if (vec && sizeof(T) == 2 && nch <= 4) {
-    int gb = 2 * 148;
+    int gb = 3 * 148;
     if (gb > (rows + 7) / 8) gb = int((rows + 7) / 8);
     auto Xb = reinterpret_cast<const bf16*>(x);
     auto Gb = reinterpret_cast<const bf16*>(g);
