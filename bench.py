@@ -496,7 +496,7 @@ def main():
     value = batch * world * args.steps / dt
     peak = pk.get("bf16_tflops_sustained", pk.get("bf16_tflops"))
     traffic = None
-    tp = os.path.join(ROOT, "profiles", "r1_conv_ncu.json" if cnn else "r1_gemm_ncu.json")
+    tp = os.path.join(ROOT, "profiles", "r1_conv_ncu.json" if cnn else "r2_gemm_ffn1_ncu.json")
     if os.path.exists(tp):
         traffic = json.load(open(tp)).get("traffic_per_launch_bytes")
     if cnn:
