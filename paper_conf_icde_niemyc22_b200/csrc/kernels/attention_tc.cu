@@ -4,7 +4,7 @@
 // (P:L119).  Three persistent warp-specialised kernels, each with TMA-fed operands in
 // 128B-swizzled shared memory, tcgen05.mma issued by one thread and TMEM accumulators:
 //   * fa5_fwd: online softmax over 64-key chunks (thresholded running max), O = P V, the row
-//     log-sum-exp and the dropout keep bits (Philox on the softmax warps);
+//     log-sum-exp and the dropout keep bits (Philox on separate RNG warps);
 //   * fa5_bwd_dq: dQ per 128-query tile (P rebuilt from S and the log-sum-exp, keep bits read);
 //   * fa5_bwd_dkv: dK, dV per 128-key tile.
 // Each kernel's layout and pipeline is described above it.
@@ -591,20 +591,31 @@ __global__ void __launch_bounds__(kKvThreads, 1)
 // between the halves through shared memory; the running max only moves when it grows by
 // more than 8 (log2 units) — then the warp rescales its half of the O_t rows in TMEM after
 // the previous P V product has landed — otherwise the stale max is kept (exponentials
-// stay <= 2^8; exact after the final 1/l).  P (dropout applied: Philox keep bits, one call
-// per four keys of a row, reading D-RNG) goes to shared memory in the K-major SW128 layout and
-// O_t += P V_j runs on the tensor cores.  One thread issues TMA, one issues tcgen05.mma;
-// the next item's Q and the next chunks' K / V load while the current item computes.
+// stay <= 2^8; exact after the final 1/l).  P (dropout applied) goes to shared memory in the
+// K-major SW128 layout and O_t += P V_j runs on the tensor cores.  The keep bits (one Philox
+// call per eight keys of a row, reading D-RNG) come from eight RNG warps — thread = (tile, row),
+// both key halves of a chunk, up to two chunks ahead through a double-buffered shared-memory
+// slot — which also write the mask output: the Philox integer work (about 40 % of the forward's
+// instructions) runs on warps of its own, interleaved with the softmax warps' MUFU / FMA work by
+// the schedulers, and setmaxnreg moves the RNG and control warps' unused registers to the
+// softmax warps (157 -> 146 us per BERT-Large layer at p = 0.1, the same bits and values).  One
+// thread issues TMA, one issues tcgen05.mma; the next item's Q and the next chunks' K / V load
+// while the current item computes.
 //   TMEM: S_0 [0,64) [64,128)  S_1 [128,192) [192,256)  O_0 [256,320)  O_1 [320,384)
 //   smem: Q 2 x 16K | K,V ring 4 x 16K | P 2 x 16K | barriers, row exchange
 constexpr int kFwdSoftWarps = 16;  // (tile t, key half h, lane quarter): warp = 8t + 4h + quarter
-constexpr int kFwdTma = kFwdSoftWarps, kFwdMma = kFwdSoftWarps + 1;
-constexpr int kFwdThreads = 32 * (kFwdSoftWarps + 2);
+constexpr int kFwdRngWarps = 8;    // (tile t, lane quarter): warp = kFwdSoftWarps + 4t + quarter
+constexpr int kFwdTma = kFwdSoftWarps + kFwdRngWarps, kFwdMma = kFwdTma + 1;
+constexpr int kFwdThreads = 32 * (kFwdSoftWarps + kFwdRngWarps + 4);  // + TMA, MMA and two idle warps
+// setmaxnreg split of the 896 x 72 registers allocated at launch (softmax warps hold a 32-key
+// S slice, the exchange and the P tile addressing; RNG threads eight Philox states)
+constexpr uint32_t kFwdRegSoft = 88, kFwdRegRng = 40, kFwdRegCtl = 72;
 constexpr int kFwdKC = 64;  // keys per chunk
 constexpr int kFwdStages = 4;
 constexpr int kFwdSmemQ = 0, kFwdSmemKV = 32768, kFwdSmemP = kFwdSmemKV + kFwdStages * 16384;
 constexpr int kFwdSmemBar = kFwdSmemP + 32768;
-constexpr int kFwdSmem = kFwdSmemBar + 512 + 6144 + 1024;  // barriers | exchange: maxima [t][h][2][128], sums [t][h][128] | align
+constexpr int kFwdSmemBits = kFwdSmemBar + 512 + 6144;  // keep words [t][chunk parity][128 rows][2]
+constexpr int kFwdSmem = kFwdSmemBits + 4096 + 1024;  // barriers | exchange: maxima [t][h][2][128], sums [t][h][128] | bits | align
 constexpr float kRescaleThr = 8.f;
 
 __device__ __forceinline__ void tmem_st32(uint32_t taddr, const uint32_t (&r)[32]) {
@@ -642,7 +653,12 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
   auto o_full = [&](int t) { return tb + 8 * t + 6; };
   auto o_free = [&](int t) { return tb + 8 * t + 7; };
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tb + 16);
+  // keep words produced by the RNG warps: b_full[t][k] (RNG threads of tile t), b_free[t][k]
+  // (its softmax threads), k = chunk parity
+  auto b_full = [&](int t, int k) { return bar + 40 + 2 * t + k; };
+  auto b_free = [&](int t, int k) { return bar + 44 + 2 * t + k; };
   const uint32_t xch = smem_u32(smem + kFwdSmemBar + 512);  // floats: maxima [t][h][2][128] | sums [t][h][128]
+  const uint32_t bits_smem = smem_u32(smem + kFwdSmemBits);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int S = p.seq, nqt = S / 128, npair = (nqt + 1) / 2, nkc = S / kFwdKC;
@@ -665,6 +681,10 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
       mbar_init(p_free(t), 1);
       mbar_init(o_full(t), 1);
       mbar_init(o_free(t), 256);
+      for (int kk = 0; kk < 2; ++kk) {
+        mbar_init(b_full(t, kk), 128);
+        mbar_init(b_free(t, kk), 256);
+      }
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -678,7 +698,9 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
-  if (warp == kFwdTma) {
+  if (warp >= kFwdTma) {
+   asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kFwdRegCtl));
+   if (warp == kFwdTma) {
     if (lane == 0) {
       int it = 0, kc = 0;  // items done by this CTA, K/V chunks loaded
       for (int item = blockIdx.x; item < items; item += gridDim.x, ++it) {
@@ -757,8 +779,55 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
         tc_commit(q_empty);
       }
     }
+   }
+  } else if (warp >= kFwdSoftWarps) {
+    // ===== RNG warps: tile t, row i — the keep bits of each 64-key chunk (both halves), up to two
+    // chunks ahead of the softmax warps, and the mask output
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(kFwdRegRng));
+    const int t = (warp - kFwdSoftWarps) >> 2, i = ((warp - kFwdSoftWarps) & 3) * 32 + lane;
+    uint32_t cb = 0;  // chunks produced (this tile)
+    for (int item = blockIdx.x; item < items; item += gridDim.x) {
+      const int pair = item % npair, ah = item / npair, a = ah % p.heads, b = ah / p.heads;
+      const int nt = min(2, nqt - 2 * pair);
+      if (t >= nt) continue;
+      const int q = (2 * pair + t) * 128 + i;
+      const uint64_t erow = ((uint64_t(p.b0 + b) * p.heads + a) * uint64_t(S) + uint64_t(q)) * uint64_t(S);
+      uint32_t* mrow = p.mask ? p.mask + ((int64_t(b) * p.heads + a) * S + q) * (S / 32) : nullptr;
+      for (int j = 0; j < nkc; ++j, ++cb) {
+        const int key = j * kFwdKC;
+        uint32_t w0 = 0xFFFFFFFFu, w1 = 0xFFFFFFFFu;
+        if (p.p > 0.f) {
+          // one Philox call per eight keys of the row (D-RNG); erow + key is a multiple of 64,
+          // so the eight counters share the high word
+          const uint64_t cnt0 = (erow + uint64_t(key)) >> 3;
+          w0 = 0u;
+          w1 = 0u;
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const uint4 x0 = philox4x32_10(uint32_t(cnt0) + uint32_t(u), uint32_t(cnt0 >> 32), step, 0u, p.seed,
+                                           kPhiloxKey1);
+            w0 |= keep_bits8(x0, p.thr) << (8 * u);
+          }
+#pragma unroll
+          for (int u = 0; u < 4; ++u) {
+            const uint4 x1 = philox4x32_10(uint32_t(cnt0) + uint32_t(4 + u), uint32_t(cnt0 >> 32), step, 0u, p.seed,
+                                           kPhiloxKey1);
+            w1 |= keep_bits8(x1, p.thr) << (8 * u);
+          }
+        }
+        if (mrow) *reinterpret_cast<uint2*>(mrow + (key >> 5)) = make_uint2(w0, w1);
+        if (!(p.p > 0.f)) continue;  // no dropout: the softmax warps need no bits
+        const int kb = cb & 1;
+        if (cb >= 2) mbar_wait(b_free(t, kb), ((cb >> 1) - 1) & 1);
+        asm volatile("st.shared.v2.b32 [%0], {%1, %2};" ::"r"(bits_smem + uint32_t(((t * 2 + kb) * 128 + i) * 8)),
+                     "r"(w0), "r"(w1)
+                     : "memory");
+        mbar_arrive(b_full(t, kb));
+      }
+    }
   } else {
     // ===== softmax warps: tile t, key half h (32 keys of each chunk), row i
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(kFwdRegSoft));
     const int t = warp >> 3, h = (warp >> 2) & 1, qq = warp & 3;
     const int i = qq * 32 + lane;
     const uint32_t srow = tmem + (uint32_t(qq * 32) << 16) + uint32_t(t * 128 + 32 * h);
@@ -773,8 +842,6 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
       const int nt = min(2, nqt - 2 * pair);
       if (t >= nt) continue;
       const int q = (2 * pair + t) * 128 + i;
-      const uint64_t erow = ((uint64_t(p.b0 + b) * p.heads + a) * uint64_t(S) + uint64_t(q)) * uint64_t(S);
-      uint32_t* mrow = p.mask ? p.mask + ((int64_t(b) * p.heads + a) * S + q) * (S / 32) : nullptr;
       float mrun = -INFINITY, l = 0.f;
       for (int j = 0; j < nkc; ++j, ++cs) {
         const uint32_t bsel = cs & 1;
@@ -808,30 +875,26 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
         }
         if (grow) mrun = m;
         // P = 2^(S alpha log2e - mrun) with the keep bits, bf16 into the K-major P tile
-        const int key = j * kFwdKC + 32 * h;
         float* v = reinterpret_cast<float*>(r);
 #pragma unroll
         for (int jj = 0; jj < 32; ++jj) {
           v[jj] = ex2(fmaf(v[jj], p.sl2, -mrun));
           l += v[jj];
         }
-        uint32_t bits = 0xFFFFFFFFu;
+        // this half's 32 keep bits from the RNG warp of the row (D-RNG; bit jj = key j kFwdKC + 32 h + jj)
         if (p.p > 0.f) {
-          bits = 0u;
-          // one Philox call per eight keys of the row (D-RNG); erow + key is a multiple of 32,
-          // so the four counters share the high word
-          const uint64_t cnt0 = (erow + uint64_t(key)) >> 3;
-#pragma unroll
-          for (int u = 0; u < 4; ++u) {
-            const uint4 w = philox4x32_10(uint32_t(cnt0) + uint32_t(u), uint32_t(cnt0 >> 32), step, 0u, p.seed,
-                                          kPhiloxKey1);
-            bits |= keep_bits8(w, p.thr) << (8 * u);
-          }
+          const int kb = cs & 1;
+          mbar_wait(b_full(t, kb), (cs >> 1) & 1);
+          uint32_t bits;
+          asm volatile("ld.shared.b32 %0, [%1];"
+                       : "=r"(bits)
+                       : "r"(bits_smem + uint32_t(((t * 2 + kb) * 128 + i) * 8 + h * 4))
+                       : "memory");
+          mbar_arrive(b_free(t, kb));
 #pragma unroll
           for (int jj = 0; jj < 32; ++jj)
             if (!((bits >> jj) & 1u)) v[jj] = 0.f;
         }
-        if (mrow) mrow[key >> 5] = bits;
         if (npw > 0) mbar_wait(p_free(t), (npw - 1) & 1);  // the previous P V has read the P tile
         st_row32(pbuf, i, 32 * h, v);
         ++npw;
