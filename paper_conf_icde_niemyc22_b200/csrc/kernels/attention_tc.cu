@@ -599,17 +599,19 @@ __global__ void __launch_bounds__(kKvThreads, 1)
 // instructions) runs on warps of its own, interleaved with the softmax warps' MUFU / FMA work by
 // the schedulers, and setmaxnreg moves the RNG and control warps' unused registers to the
 // softmax warps (157 -> 146 us per BERT-Large layer at p = 0.1, the same bits and values).  One
-// thread issues TMA, one issues tcgen05.mma; the next item's Q and the next chunks' K / V load
-// while the current item computes.
+// thread issues TMA and one thread per query tile issues that tile's tcgen05.mma products (S of
+// chunk j+1 before P V of chunk j), so neither tile's next S waits for the other tile's P
+// (146 -> 142.5 us); the next item's Q and the next chunks' K / V load while the current item
+// computes.
 //   TMEM: S_0 [0,64) [64,128)  S_1 [128,192) [192,256)  O_0 [256,320)  O_1 [320,384)
 //   smem: Q 2 x 16K | K,V ring 4 x 16K | P 2 x 16K | barriers, row exchange
 constexpr int kFwdSoftWarps = 16;  // (tile t, key half h, lane quarter): warp = 8t + 4h + quarter
 constexpr int kFwdRngWarps = 8;    // (tile t, lane quarter): warp = kFwdSoftWarps + 4t + quarter
 constexpr int kFwdTma = kFwdSoftWarps + kFwdRngWarps, kFwdMma = kFwdTma + 1;
-constexpr int kFwdThreads = 32 * (kFwdSoftWarps + kFwdRngWarps + 4);  // + TMA, MMA and two idle warps
+constexpr int kFwdThreads = 32 * (kFwdSoftWarps + kFwdRngWarps + 4);  // + TMA, 2 x MMA, one idle warp
 // setmaxnreg split of the 896 x 72 registers allocated at launch (softmax warps hold a 32-key
 // S slice, the exchange and the P tile addressing; RNG threads eight Philox states)
-constexpr uint32_t kFwdRegSoft = 88, kFwdRegRng = 40, kFwdRegCtl = 72;
+constexpr uint32_t kFwdRegSoft = 80, kFwdRegRng = 64, kFwdRegCtl = 56;
 constexpr int kFwdKC = 64;  // keys per chunk
 constexpr int kFwdStages = 4;
 constexpr int kFwdSmemQ = 0, kFwdSmemKV = 32768, kFwdSmemP = kFwdSmemKV + kFwdStages * 16384;
@@ -667,10 +669,10 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
   if (threadIdx.x == 0) {
     mbar_init(&q_full[0], 1);
     mbar_init(&q_full[1], 1);
-    mbar_init(q_empty, 1);
+    mbar_init(q_empty, 2);  // one arrival per tile's MMA thread
     for (int s = 0; s < kFwdStages; ++s) {
       mbar_init(&kv_full[s], 1);
-      mbar_init(&kv_empty[s], 1);
+      mbar_init(&kv_empty[s], 2);
     }
     for (int t = 0; t < 2; ++t) {
       for (int b = 0; b < 2; ++b) {
@@ -722,21 +724,23 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
         }
       }
     }
-  } else if (warp == kFwdMma) {
-    if (lane == 0) {
+  } else if ((warp == kFwdMma || warp == kFwdMma + 1) && lane == 0) {
+      // one tcgen05.mma-issuing thread per query tile, so neither tile's products wait behind
+      // the other tile's P (the K/V stage and Q buffers are released by both: counts of 2)
+      const int t = warp - kFwdMma;
       constexpr uint32_t idS = (1u << 4) | (1u << 7) | (1u << 10) | (uint32_t(kFwdKC >> 3) << 17) |
                                (uint32_t(128 >> 4) << 24);
       constexpr uint32_t idO = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | (uint32_t(64 >> 3) << 17) |
                                (uint32_t(128 >> 4) << 24);
       int kc = 0;
-      uint32_t cs[2] = {0, 0};   // S chunks issued per tile (running: buffer cs & 1)
-      uint32_t np[2] = {0, 0};   // p_full completions consumed per tile
-      uint32_t nit[2] = {0, 0};  // items per tile (q_full / o_free phases)
-      auto issue_s = [&](int t, int s) {
-        const uint32_t c = cs[t]++, bsel = c & 1;
+      uint32_t cs = 0;   // S chunks issued (running: buffer cs & 1)
+      uint32_t np = 0;   // p_full completions consumed
+      uint32_t nit = 0;  // items (q_full / o_free phases)
+      auto issue_s = [&](int st) {
+        const uint32_t c = cs++, bsel = c & 1;
         if (c >= 2) mbar_wait(s_free(t, bsel), ((c >> 1) - 1) & 1);  // the buffer's previous chunk is read
         tc_fence_after();
-        const uint32_t q = smem_u32(smem + kFwdSmemQ + t * 16384), k = smem_u32(smem + kFwdSmemKV + s * 16384);
+        const uint32_t q = smem_u32(smem + kFwdSmemQ + t * 16384), k = smem_u32(smem + kFwdSmemKV + st * 16384);
 #pragma unroll
         for (int kk = 0; kk < 4; ++kk)
           tc_mma(tmem + uint32_t(t * 128 + bsel * 64), smem_desc(q + kk * 32, 16, 1024),
@@ -746,39 +750,45 @@ __global__ void __launch_bounds__(kFwdThreads, 1)
       for (int item = blockIdx.x; item < items; item += gridDim.x) {
         const int pair = item % npair;
         const int nt = min(2, nqt - 2 * pair);
-        {
-          const int s = kc % kFwdStages;
-          mbar_wait(&kv_full[s], (kc / kFwdStages) & 1);
-          for (int t = 0; t < nt; ++t) {
-            mbar_wait(&q_full[t], nit[t] & 1);
-            issue_s(t, s);
+        if (t >= nt) {  // single-tile item: keep the shared stage / Q barriers' arrival counts
+          for (int j = 0; j < nkc; ++j, ++kc) {
+            const int st = kc % kFwdStages;
+            mbar_wait(&kv_full[st], (kc / kFwdStages) & 1);
+            if (j == 0) mbar_arrive(q_empty);
+            mbar_arrive(&kv_empty[st]);
           }
+          continue;
+        }
+        {
+          const int st = kc % kFwdStages;
+          mbar_wait(&kv_full[st], (kc / kFwdStages) & 1);
+          mbar_wait(&q_full[t], nit & 1);
+          issue_s(st);
         }
         for (int j = 0; j < nkc; ++j, ++kc) {
-          const int s = kc % kFwdStages;
-          const uint32_t v = smem_u32(smem + kFwdSmemKV + s * 16384 + 8192);
+          const int st = kc % kFwdStages;
+          const uint32_t v = smem_u32(smem + kFwdSmemKV + st * 16384 + 8192);
           const bool more = j + 1 < nkc;
-          if (more) mbar_wait(&kv_full[(kc + 1) % kFwdStages], ((kc + 1) / kFwdStages) & 1);
-          for (int t = 0; t < nt; ++t) {
-            if (more) issue_s(t, (kc + 1) % kFwdStages);  // chunk j+1 into the other S buffer
-            mbar_wait(p_full(t), np[t] & 1);
-            ++np[t];
-            if (j == 0 && nit[t] > 0) mbar_wait(o_free(t), (nit[t] - 1) & 1);
-            tc_fence_after();
-            const uint32_t pb = smem_u32(smem + kFwdSmemP + t * 16384);
-#pragma unroll
-            for (int kk = 0; kk < kFwdKC; kk += 16)
-              tc_mma(tmem + 256 + uint32_t(t * 64), smem_desc(pb + (kk >> 4) * 32, 16, 1024),
-                     smem_desc(v + uint32_t(kk) * 128, 8192, 1024), idO, (j > 0 || kk > 0) ? 1u : 0u);
-            tc_commit(p_free(t));
-            if (!more) tc_commit(o_full(t));
+          if (more) {  // chunk j+1 into the other S buffer
+            mbar_wait(&kv_full[(kc + 1) % kFwdStages], ((kc + 1) / kFwdStages) & 1);
+            issue_s((kc + 1) % kFwdStages);
           }
-          tc_commit(&kv_empty[s]);
+          mbar_wait(p_full(t), np & 1);
+          ++np;
+          if (j == 0 && nit > 0) mbar_wait(o_free(t), (nit - 1) & 1);
+          tc_fence_after();
+          const uint32_t pb = smem_u32(smem + kFwdSmemP + t * 16384);
+#pragma unroll
+          for (int kk = 0; kk < kFwdKC; kk += 16)
+            tc_mma(tmem + 256 + uint32_t(t * 64), smem_desc(pb + (kk >> 4) * 32, 16, 1024),
+                   smem_desc(v + uint32_t(kk) * 128, 8192, 1024), idO, (j > 0 || kk > 0) ? 1u : 0u);
+          tc_commit(p_free(t));
+          if (!more) tc_commit(o_full(t));
+          tc_commit(&kv_empty[st]);
         }
-        for (int t = 0; t < nt; ++t) ++nit[t];
+        ++nit;
         tc_commit(q_empty);
       }
-    }
    }
   } else if (warp >= kFwdSoftWarps) {
     // ===== RNG warps: tile t, row i — the keep bits of each 64-key chunk (both halves), up to two
