@@ -542,10 +542,12 @@ __global__ void __launch_bounds__(kKvThreads, 1)
         // in place: rp <- P_d, rs <- dS (fp32 bits)
 #pragma unroll
         for (int j = 0; j < 32; ++j) {
-          const bool keep = (bits >> j) & 1u;
+          // one select: km = keep_scale or 0, then dP_d = dP km and P_d = P km (a dropped dP of
+          // either sign gives +-0, and +-0 - D = -D: the same values as selecting each)
+          const float km = ((bits >> j) & 1u) ? p.keep_scale : 0.f;
           const float pr = ex2(__uint_as_float(rs[j]) * p.sl2 - l2);
-          const float dp = keep ? __uint_as_float(rp[j]) * p.keep_scale : 0.f;
-          rp[j] = __float_as_uint(keep ? pr * p.keep_scale : 0.f);
+          const float dp = __uint_as_float(rp[j]) * km;
+          rp[j] = __float_as_uint(pr * km);
           rs[j] = __float_as_uint(pr * (dp - D));
         }
         if (qc > 0) mbar_wait(ps_free, (qc - 1) & 1);  // the previous tile's dV, dK products read P_d / dS
